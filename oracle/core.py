@@ -1,0 +1,430 @@
+"""Buffalo CPU ORACLE (test infrastructure only; see oracle/__init__.py).
+
+A plain, slow, obviously-correct restatement of what Buffalo's hot path computes, written
+from /root/reference/PAPER.md (cited as PAPER.md:<line>) and the readings listed in
+DESIGN.md §"Readings of the paper" (cited as R<n>).  Integer work (sampling, blocks) is in
+oracle/buffalo_oracle.c (plain C, single thread); the scheduler is plain Python; the layer
+math is numpy/scipy in float64.  Nothing here is shared with the CUDA path.
+
+Functions and the passages they follow:
+  degree_bucketing     Alg. 3 l.1, PAPER.md:127 ("nodes with a larger degree than F are
+                       grouped together into a single bucket"), :164, :269; R1, R5
+  item_stats           Eq. 1 inputs I, O, D "obtained during the micro-batch generation"
+                       PAPER.md:386; R13
+  mem_model            BucketMemEstimator PAPER.md:314/:347 — delegated by the paper to
+                       Betty [93]; our reading R15 = exact arena bytes of one micro-batch
+  grouping_weight      Eq. 1 + Eq. 2, PAPER.md:359-363 (integer form, R14)
+  split_explosion      SplitExplosionBucket PAPER.md:273, :335 ("evenly splits"); R7, R8
+  mem_balanced_group   Alg. 4 PAPER.md:313-326 with text :343 (largest first, R10)
+  schedule             Alg. 3 PAPER.md:269-280 + :333 (K loop, K=1 special case)
+  build_blocks         Alg. 2 l.5 PAPER.md:237 + §IV-E :388-390 (C); transposes by definition
+  sage_forward         Alg. 2 l.8-9 PAPER.md:240-241 (Aggregate = mean, Update = W_l) with
+                       GraphSAGE-mean [16]; R20, R21
+  softmax_ce           Alg. 2 l.10 PAPER.md:242; normalisation by the global batch (R19)
+  sage_backward        Alg. 2 l.11-12 PAPER.md:243-244 (gradients accumulated over groups)
+  train_epoch          Alg. 2 PAPER.md:233-245 end to end (one optimizer step, R18)
+"""
+import ctypes
+import math
+import os
+import subprocess
+
+import numpy as np
+import scipy.sparse as sp
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "buffalo_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+INT64_MAX = (1 << 63) - 1
+
+
+# ============================================================================ C library
+def build_lib(force=False):
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-o", _LIB, _SRC])
+    return _LIB
+
+
+class _OBlock(ctypes.Structure):
+    _fields_ = [("n_dst", ctypes.c_int64), ("n_src", ctypes.c_int64), ("n_edges", ctypes.c_int64),
+                ("row_ptr", ctypes.POINTER(ctypes.c_int32)),
+                ("col_local", ctypes.POINTER(ctypes.c_int32)),
+                ("col_global", ctypes.POINTER(ctypes.c_int32)),
+                ("src_global", ctypes.POINTER(ctypes.c_int32))]
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        _lib = ctypes.CDLL(build_lib())
+        P = ctypes.c_void_p
+        _lib.oracle_philox.argtypes = [P, P, P]
+        _lib.oracle_sample_row.argtypes = [P, P, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64,
+                                           ctypes.c_int32, P]
+        _lib.oracle_sample_row.restype = ctypes.c_int64
+        _lib.oracle_build_blocks.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int64,
+                                             ctypes.c_int32, P, ctypes.c_uint64, P]
+        _lib.oracle_build_blocks.restype = ctypes.c_int
+        _lib.oracle_block_sizes.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int64,
+                                            ctypes.c_int32, P, ctypes.c_uint64, P, P]
+        _lib.oracle_block_sizes.restype = ctypes.c_int
+        _lib.oracle_free_blocks.argtypes = [P, ctypes.c_int32]
+    return _lib
+
+
+def _p(a):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+class Graph:
+    """CSR graph: row_ptr int64[N+1], col int32[nnz] (rows sorted, no duplicates)."""
+
+    def __init__(self, row_ptr, col):
+        self.row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+        self.col = np.ascontiguousarray(col, dtype=np.int32)
+        self.N = self.row_ptr.size - 1
+
+    def degree(self, v):
+        return self.row_ptr[np.asarray(v, dtype=np.int64) + 1] - self.row_ptr[np.asarray(v, dtype=np.int64)]
+
+
+def philox(ctr, key):
+    c = np.ascontiguousarray(ctr, dtype=np.uint32)
+    k = np.ascontiguousarray(key, dtype=np.uint32)
+    out = np.zeros(4, dtype=np.uint32)
+    lib().oracle_philox(_p(c), _p(k), _p(out))
+    return out
+
+
+def sample_row(g, v, f, seed, hop):
+    out = np.zeros(max(1, int(g.degree(v))), dtype=np.int32)
+    n = lib().oracle_sample_row(_p(g.row_ptr), _p(g.col), int(v), int(f), int(seed), int(hop), _p(out))
+    return out[:n].copy()
+
+
+# ============================================================================ blocks
+def build_blocks(g, seeds, L, fanout, seed):
+    """Blocks l = 1..L (returned as a list indexed l-1) of the micro-batch with output nodes
+    `seeds` (Alg. 2 l.5).  Each block is a dict with
+    n_dst, n_src, n_edges, row_ptr, col_local, col_global, src_global, D (= row lengths) and
+    the transposed block t_row_ptr / t_col (for each src j, the dst i with an edge to j,
+    ascending i)."""
+    seeds = np.ascontiguousarray(seeds, dtype=np.int32)
+    fan = np.ascontiguousarray(fanout, dtype=np.int32)
+    arr = (_OBlock * L)()
+    rc = lib().oracle_build_blocks(g.N, _p(g.row_ptr), _p(g.col), _p(seeds), seeds.size, L, _p(fan),
+                                   int(seed), ctypes.cast(arr, ctypes.c_void_p))
+    if rc != 0:
+        raise MemoryError("oracle_build_blocks failed")
+    blocks = []
+    for l in range(1, L + 1):
+        b = arr[l - 1]
+        nd, ns, ne = b.n_dst, b.n_src, b.n_edges
+        rp = np.ctypeslib.as_array(b.row_ptr, shape=(nd + 1,)).copy()
+        cl = np.ctypeslib.as_array(b.col_local, shape=(max(ne, 1),))[:ne].copy()
+        cg = np.ctypeslib.as_array(b.col_global, shape=(max(ne, 1),))[:ne].copy()
+        sg = np.ctypeslib.as_array(b.src_global, shape=(max(ns, 1),))[:ns].copy()
+        D = np.diff(rp).astype(np.int64)
+        dst_of_edge = np.repeat(np.arange(nd, dtype=np.int32), D)
+        order = np.argsort(cl, kind="stable")
+        t_col = dst_of_edge[order].astype(np.int32)
+        t_rp = np.zeros(ns + 1, dtype=np.int32)
+        np.cumsum(np.bincount(cl, minlength=ns), out=t_rp[1:])
+        blocks.append(dict(n_dst=nd, n_src=ns, n_edges=ne, row_ptr=rp, col_local=cl,
+                           col_global=cg, src_global=sg, D=D, t_row_ptr=t_rp, t_col=t_col))
+    lib().oracle_free_blocks(ctypes.cast(arr, ctypes.c_void_p), L)
+    return blocks
+
+
+def block_sizes(g, seeds, L, fanout, seed):
+    """(n[0..L], e[1..L] as a list indexed l-1) of the blocks of `seeds`."""
+    seeds = np.ascontiguousarray(seeds, dtype=np.int32)
+    fan = np.ascontiguousarray(fanout, dtype=np.int32)
+    n = np.zeros(L + 1, dtype=np.int64)
+    e = np.zeros(L, dtype=np.int64)
+    rc = lib().oracle_block_sizes(g.N, _p(g.row_ptr), _p(g.col), _p(seeds), seeds.size, L,
+                                  _p(fan), int(seed), _p(n), _p(e))
+    if rc != 0:
+        raise MemoryError("oracle_block_sizes failed")
+    return [int(x) for x in n], [int(x) for x in e]
+
+
+# ============================================================================ bucketing
+def degree_bucketing(g, seeds, f_L, F):
+    """Alg. 3 l.1 DegreeBucketing.  D(v) = min(deg(v), f_L) (deg(v) for
+    a full-neighbour output layer, f_L <= 0); bucket(v) = min(D(v), F); the degree-F bucket
+    holds every node with D >= F.  Returns (D, bucket, order, hist): `order` lists seed
+    positions grouped by bucket ascending, input order inside a bucket (R5)."""
+    seeds = np.asarray(seeds, dtype=np.int64)
+    deg = g.degree(seeds)
+    D = deg if f_L <= 0 else np.minimum(deg, f_L)
+    bucket = np.minimum(D, F)
+    order = np.argsort(bucket, kind="stable")
+    hist = np.bincount(bucket, minlength=F + 1)
+    return D.astype(np.int64), bucket.astype(np.int64), order.astype(np.int64), hist.astype(np.int64)
+
+
+# ============================================================================ memory model
+ALIGN = 256
+SCAN_WS = 8192
+HEAVY_T = 128          # rows with D > HEAVY_T go through the cooperative long-tail path
+FP32, BF16 = 0, 1
+
+
+def _R(x):
+    return ((int(x) + ALIGN - 1) // ALIGN) * ALIGN
+
+
+def pitch(d):
+    return ((int(d) + 7) // 8) * 8
+
+
+def dw_splits(n_l, d_out, d_in):
+    """Split count of the deterministic split-K dW reduction."""
+    tiles = math.ceil(d_out / 64) * math.ceil(2 * d_in / 64)
+    return max(1, min(math.ceil(296 / tiles), math.ceil(int(n_l) / 512)))
+
+
+def mem_model(n, e, dims, act_dtype=FP32):
+    """BucketMemEstimator reading R15: the exact arena bytes of one
+    micro-batch with layer sizes n[0..L], e[1..L] (e indexed l-1) and widths dims[0..L].
+    Returns (lo, hi): hi = capacity that always suffices (used as M_est), lo = bytes the
+    backward pass is certain to touch; the measured arena peak lies in [lo, hi].
+    Every buffer is rounded up to 256 B.  Layout restated from DESIGN.md §"Arena"."""
+    L = len(e)
+    s = 4 if act_dtype == FP32 else 2
+    blocks = 0
+    build = 0
+    for l in range(1, L + 1):
+        nl, nm, el = n[l], n[l - 1], e[l - 1]
+        blocks += _R(4 * (nl + 1)) + _R(4 * el) + _R(4 * nm) + _R(4 * nl)
+        if l == 1:
+            blocks += _R(4 * el)                               # col_global kept for layer 1
+        else:
+            blocks += _R(4 * (nm + 1)) + _R(4 * el)            # transposed block
+        frame = _R(4 * (nl + el + 1)) + SCAN_WS
+        if l >= 2:
+            frame += _R(4 * el) + _R(4 * nm)
+        build = max(build, frame)
+    acts = 0
+    for l in range(1, L + 1):
+        acts += _R(n[l] * pitch(dims[l - 1]) * s)              # saved h_agg
+        if l < L:
+            acts += _R(n[l] * pitch(dims[l]) * s)              # H_l
+    acts += _R(n[L] * pitch(dims[L]) * 4)                      # logits
+    bwd = 0
+    for l in range(L, 0, -1):
+        frame = _R(n[l] * pitch(dims[l]) * 4)                  # dH_l (dlogits at l = L)
+        if l >= 2:
+            frame += _R(n[l - 1] * pitch(dims[l - 1]) * 4)     # dH_{l-1}
+            frame += _R(n[l - 1] * pitch(dims[l]) * 4)         # transposed aggregate of dZ/D
+        frame += _R(dw_splits(n[l], dims[l], dims[l - 1]) * dims[l] * 2 * dims[l - 1] * 4)
+        bwd = max(bwd, frame)
+    lo = blocks + acts + bwd
+    hi = blocks + acts + max(bwd, build)
+    return lo, hi
+
+
+# ============================================================================ Eq. 1-2
+def grouping_weight(M, I, E, C_ppm):
+    """Eq. 1-2: item contribution M_est[i] * R_group[i] with
+    R = min(1, I / (O*D*C)), O*D = E (R13), evaluated exactly in integers:
+    floor(M * min(1, I*10^6 / (E*C_ppm))).  E = 0 or C_ppm <= 0 => R = 1 (R14)."""
+    M, I, E, C_ppm = int(M), int(I), int(E), int(C_ppm)
+    if E == 0 or C_ppm <= 0:
+        return M
+    return min(M, (M * I * 1_000_000) // (E * C_ppm))
+
+
+def item_stats(g, seeds, L, fanout, seed, dims, act_dtype):
+    """O, E = sum D, I = unique src of the item's own output block, sizes, M_est (R13, R15)."""
+    seeds = np.asarray(seeds, dtype=np.int32)
+    n, e = block_sizes(g, seeds, L, fanout, seed)
+    lo, hi = mem_model(n, e, dims, act_dtype)
+    return dict(O=int(seeds.size), E=int(e[L - 1]), I=int(n[L - 1]), n=n, e=e, M=hi)
+
+
+def split_explosion(seeds, K):
+    """SplitExplosionBucket: K contiguous pieces, numpy.array_split
+    sizes (the first O mod K pieces get one extra seed) (R8)."""
+    return np.array_split(np.asarray(seeds), K)
+
+
+def mem_balanced_grouping(items, K, M_ctr):
+    """Alg. 4 MemBalancedGrouping (text :343): items sorted by M_est
+    descending (ties: bucket degree asc, micro-bucket index asc — R12), each placed into the
+    group with the lowest Eq. 2 estimate so far (ties: lowest index); success iff every
+    group estimate <= M_ctr.  items: list of dicts with keys d, k, M, w."""
+    order = sorted(items, key=lambda it: (-it["M"], it["d"], it["k"]))
+    loads = [0] * K
+    groups = [[] for _ in range(K)]
+    for it in order:
+        gi = min(range(K), key=lambda j: (loads[j], j))
+        groups[gi].append(it)
+        loads[gi] += it["w"]
+    return max(loads) <= M_ctr, groups, loads
+
+
+def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT64_MAX,
+             C_ppm=0, k_min=1, k_max=4096, num_gpus=1):
+    """Alg. 3 Buffalo_Scheduler with the readings of DESIGN.md
+    (R7 explosion test, R11 sort/placement keys, R16 K_max, R17 empty groups dropped,
+    R27 k_min = #GPUs and LPT rank assignment).  Returns a dict plan or None (budget)."""
+    seeds = np.asarray(seeds, dtype=np.int32)
+    f_L = fanout[L - 1]
+    D, bucket, order, hist = degree_bucketing(g, seeds, f_L, F)
+    pos_of = {d: np.nonzero(bucket == d)[0] for d in range(F + 1)}
+    stats = {}
+    for d in range(F + 1):
+        if pos_of[d].size:
+            st = item_stats(g, seeds[pos_of[d]], L, fanout, seed, dims, act_dtype)
+            st["w"] = grouping_weight(st["M"], st["I"], st["E"], C_ppm)
+            stats[d] = st
+    non_split = [d for d in stats if d != F]
+    sum_M_all = sum(stats[d]["M"] for d in stats)
+    max_w = max([stats[d]["w"] for d in non_split], default=0)
+    sum_w = sum(stats[d]["w"] for d in non_split)
+    k_lo = max(k_min, num_gpus, 1)
+    for K in range(k_lo, k_max + 1):
+        if max_w > mem_budget:
+            return None                      # a never-split bucket exceeds M_ctr for every K
+        if sum_w > K * mem_budget:
+            continue                         # some group must exceed M_ctr (weights >= 0)
+        items = [dict(d=d, k=0, pos=pos_of[d], **stats[d]) for d in non_split]
+        if F in stats:
+            explosion = K >= 2 and stats[F]["M"] * K > sum_M_all
+            if explosion:
+                for k, piece in enumerate(split_explosion(pos_of[F], K)):
+                    if piece.size == 0:
+                        continue
+                    st = item_stats(g, seeds[piece], L, fanout, seed, dims, act_dtype)
+                    st["w"] = grouping_weight(st["M"], st["I"], st["E"], C_ppm)
+                    items.append(dict(d=F, k=k, pos=piece, **st))
+            else:
+                items.append(dict(d=F, k=0, pos=pos_of[F], **stats[F]))
+        ok, groups, loads = mem_balanced_grouping(items, K, mem_budget)
+        if not ok:
+            continue
+        kept = [(grp, ld) for grp, ld in zip(groups, loads) if grp]
+        offsets = [0]
+        group_seeds = []
+        group_of_seed = np.full(seeds.size, -1, dtype=np.int32)
+        for gi, (grp, _) in enumerate(kept):
+            for it in sorted(grp, key=lambda it: (it["d"], it["k"])):
+                group_seeds.append(seeds[it["pos"]])
+                group_of_seed[it["pos"]] = gi
+            offsets.append(offsets[-1] + sum(it["O"] for it in grp))
+        est = [ld for _, ld in kept]
+        rank_load = [0] * max(1, num_gpus)
+        rank_of_group = [0] * len(kept)
+        for gi in sorted(range(len(kept)), key=lambda j: (-est[j], j)):
+            r = min(range(len(rank_load)), key=lambda j: (rank_load[j], j))
+            rank_of_group[gi] = r
+            rank_load[r] += est[gi]
+        return dict(K=len(kept), K_tried=K, group_offsets=np.array(offsets, dtype=np.int64),
+                    group_seeds=(np.concatenate(group_seeds).astype(np.int32) if group_seeds
+                                 else np.zeros(0, np.int32)),
+                    group_of_seed=group_of_seed, est_bytes=np.array(est, dtype=np.int64),
+                    rank_of_group=np.array(rank_of_group, dtype=np.int32),
+                    D=D, bucket=bucket, hist=hist)
+    return None
+
+
+# ============================================================================ layer math
+def mean_adjacency(b):
+    """D^-1 A of a block: row i has 1/D(i) at the columns of its sampled neighbours."""
+    D = b["D"]
+    data = np.repeat(np.where(D > 0, 1.0 / np.maximum(D, 1), 0.0), D)
+    return sp.csr_matrix((data, b["col_local"], b["row_ptr"].astype(np.int64)),
+                         shape=(b["n_dst"], b["n_src"]))
+
+
+def sage_forward(blocks, X, Ws, bs):
+    """GraphSAGE-mean forward over the micro-batch's blocks in float64 (Alg. 2 l.8-9):
+    h_agg = D^-1 A H_{l-1};  Z_l = [H_{l-1}[:n_l] || h_agg] W_l^T + b_l;  H_l = ReLU(Z_l)
+    for l < L, logits = Z_L.  X is the global feature table (indexed via src_global of
+    block 1).  Returns (logits, cache) with cache for sage_backward."""
+    L = len(blocks)
+    H = np.asarray(X, dtype=np.float64)[blocks[0]["src_global"]]
+    cache = []
+    for l in range(1, L + 1):
+        b = blocks[l - 1]
+        W = np.asarray(Ws[l - 1], dtype=np.float64)
+        d_in = H.shape[1]
+        A = mean_adjacency(b)
+        agg = A @ H
+        self_ = H[: b["n_dst"]]
+        Z = self_ @ W[:, :d_in].T + agg @ W[:, d_in:].T + np.asarray(bs[l - 1], dtype=np.float64)
+        cache.append(dict(A=A, H_in=H, agg=agg, Z=Z))
+        H = np.maximum(Z, 0.0) if l < L else Z
+    return H, cache
+
+
+def softmax_ce(logits, y, S):
+    """Partial loss of one group, normalised by the global batch size S (R19):
+    loss = sum_i CE(softmax(Z_i), y_i) / S; dZ = (softmax - onehot) / S."""
+    Z = np.asarray(logits, dtype=np.float64)
+    m = Z.max(axis=1, keepdims=True)
+    ez = np.exp(Z - m)
+    ssum = ez.sum(axis=1, keepdims=True)
+    lse = (m + np.log(ssum))[:, 0]
+    y = np.asarray(y, dtype=np.int64)
+    loss = float(np.sum(lse - Z[np.arange(Z.shape[0]), y]) / S)
+    P = ez / ssum
+    P[np.arange(Z.shape[0]), y] -= 1.0
+    return loss, P / S
+
+
+def sage_backward(blocks, cache, Ws, dlogits):
+    """Backward of sage_forward (Alg. 2 l.11): returns per-layer (dW_l, db_l).
+    dZ_L = dlogits; dZ_l = dH_l * 1[Z_l > 0];  dW_l = dZ_l^T [H_{l-1}[:n_l] || h_agg];
+    db_l = sum_i dZ_l[i];  dH_{l-1} = pad(dZ_l W_self) + A^T (dZ_l W_neigh)."""
+    L = len(blocks)
+    grads = [None] * L
+    dH = np.asarray(dlogits, dtype=np.float64)
+    for l in range(L, 0, -1):
+        c = cache[l - 1]
+        W = np.asarray(Ws[l - 1], dtype=np.float64)
+        d_in = c["H_in"].shape[1]
+        dZ = dH if l == L else dH * (c["Z"] > 0)
+        n_dst = dZ.shape[0]
+        Afwd = np.concatenate([c["H_in"][:n_dst], c["agg"]], axis=1)
+        grads[l - 1] = (dZ.T @ Afwd, dZ.sum(axis=0))
+        if l > 1:
+            dHin = c["A"].T @ (dZ @ W[:, d_in:])
+            dHin[:n_dst] += dZ @ W[:, :d_in]
+            dH = dHin
+    return grads
+
+
+def microbatch_step(g, seeds_k, X, y, Ws, bs, L, fanout, seed, S):
+    """One micro-batch of Alg. 2 (l.4-12): blocks, forward, partial loss, gradients."""
+    blocks = build_blocks(g, seeds_k, L, fanout, seed)
+    logits, cache = sage_forward(blocks, X, Ws, bs)
+    loss, dlog = softmax_ce(logits, y[np.asarray(seeds_k)], S)
+    grads = sage_backward(blocks, cache, Ws, dlog)
+    return loss, grads, blocks
+
+
+def train_epoch(g, seeds, X, y, Ws, bs, L, fanout, F, seed, dims, lr=0.0, **sched_kw):
+    """Alg. 2: schedule, then every group's forward/backward with the
+    partial gradients accumulated, then ONE optimizer step (SGD with rate lr, R18)."""
+    plan = schedule(g, seeds, L, fanout, F, seed, dims, **sched_kw)
+    if plan is None:
+        raise RuntimeError("Buffalo scheduler: no K satisfies the memory budget")
+    S = len(seeds)
+    total = 0.0
+    acc = [(np.zeros_like(np.asarray(W, np.float64)), np.zeros(len(b))) for W, b in zip(Ws, bs)]
+    off = plan["group_offsets"]
+    for k in range(plan["K"]):
+        sk = plan["group_seeds"][off[k]:off[k + 1]]
+        loss, grads, _ = microbatch_step(g, sk, X, y, Ws, bs, L, fanout, seed, S)
+        total += loss
+        acc = [(a + gw, b + gb) for (a, b), (gw, gb) in zip(acc, grads)]
+    newW = [np.asarray(W, np.float64) - lr * gW for W, (gW, _) in zip(Ws, acc)]
+    newb = [np.asarray(b, np.float64) - lr * gb for b, (_, gb) in zip(bs, acc)]
+    return total, acc, newW, newb, plan
