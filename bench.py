@@ -1,0 +1,341 @@
+#!/usr/bin/env python
+"""Benchmark of Buffalo's data-parallel hot path on B200 (BASELINE.json metric:
+"epoch time & aggregated edges/s under fixed mem budget at 1/2/4/8 B200").
+
+A step = one Buffalo iteration (Alg. 2) over the whole seed batch:
+bucketize (Alg. 3/4 + Eq. 1-2) + for every own bucket group: block generation, L fused
+SAGE-mean forward layers, loss, L backward layers + NCCL gradient allreduce (N > 1) + SGD.
+value = aggregated block edges of all ranks / max-over-ranks device time (edges/s).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config arxiv|cora|products]
+                  [--gemm bf16|ffma] [--impl ours|reference]
+
+Under torchrun (N > 1) every rank runs its own groups (k_min = N, LPT by estimate).
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from synth.graphs import CONFIGS, features, labels, random_graph, seed_nodes, xavier_weights  # noqa: E402
+
+WORKLOADS = {
+    "arxiv": ("ogbn-arxiv-shaped power-law graph (169,343 nodes, 1,166,243 undirected edges, 128-d), "
+              "3-layer SAGE-mean 128-256-256-40, full-neighbour blocks, F=10, 90,941 seeds, K=4 bucket groups"),
+    "cora": ("Cora-sized synthetic graph (2,708 nodes, 5,278 edges, 1,433-d), 2-layer SAGE-mean "
+             "1433-256-7, fanout (10,25), 4 partitions"),
+    "products": ("ogbn-products-shaped power-law graph (2,449,029 nodes, 61,859,140 edges, 100-d), 3-layer "
+                 "SAGE-mean 100-256-256-47, fanout (10,25,30), budget forcing >= 8 bucket groups"),
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="arxiv", choices=list(WORKLOADS))
+    ap.add_argument("--gemm", default="bf16", choices=["bf16", "ffma"])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--cpu-baseline-seconds", type=float, default=20.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def make_inputs(cfg):
+    rp, col = random_graph(cfg.N, cfg.pairs, cfg.kind)
+    X = features(cfg.N, cfg.d0, ((cfg.d0 + 7) // 8) * 8)
+    y = labels(cfg.N, cfg.classes)
+    seeds = seed_nodes(cfg.N, cfg.S)
+    Ws, bs = xavier_weights(cfg.dims)
+    return rp, col, X, y, seeds, Ws, bs
+
+
+# ----------------------------------------------------------------------------- oracle arm
+def oracle_sample(cfg, rp, col, X, y, seeds, Ws, bs, seconds):
+    """The CPU oracle (oracle/, as it stands) on a bounded sample of the workload: one
+    micro-batch of a contiguous slice of the seed batch, grown until ~`seconds` of work."""
+    import oracle as O
+    g = O.Graph(rp, col)
+    frac = 64
+    n_edges, elapsed, used = 0, 0.0, 0
+    while True:
+        part = seeds[: max(1, len(seeds) // frac)]
+        t = time.perf_counter()
+        loss, grads, blocks = O.microbatch_step(g, part, X, y, Ws, bs, cfg.L, cfg.fanout, 3, len(seeds))
+        dt = time.perf_counter() - t
+        n_edges, elapsed, used = sum(b["n_edges"] for b in blocks), dt, len(part)
+        if dt * 3 > seconds or frac == 1:
+            break
+        frac = max(1, frac // 4)
+    return dict(value=n_edges / elapsed, unit="edges/s", cores=len(os.sched_getaffinity(0)), kind="oracle",
+                sample=f"one micro-batch of {used} of {len(seeds)} seeds ({n_edges} block edges, "
+                       f"{elapsed:.2f} s): C block generation + float64 numpy/scipy SAGE fwd/bwd")
+
+
+def run_reference(args, cfg):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    rp, col, X, y, seeds, Ws, bs = make_inputs(cfg)
+    import oracle as O
+    g = O.Graph(rp, col)
+    part = seeds[: max(1, len(seeds) // 16)]
+    times, edges = [], 0
+    for i in range(args.warmup + args.steps):
+        t = time.perf_counter()
+        _, _, blocks = O.microbatch_step(g, part, X, y, Ws, bs, cfg.L, cfg.fanout, 3 + i, len(seeds))
+        dt = time.perf_counter() - t
+        if i >= args.warmup:
+            times.append(dt)
+            edges += sum(b["n_edges"] for b in blocks)
+    v = edges / sum(times)
+    line = dict(metric="aggregated edges/s (epoch of Buffalo hot path)", value=v, unit="edges/s",
+                n_gpus=0, steps=args.steps, warmup=args.warmup, ms_per_step=1e3 * statistics.mean(times),
+                higher_is_better=True, scaling="strong", vs_baseline=None, dtype="f64", data="synthetic",
+                impl="reference",
+                config={"workload": WORKLOADS[args.config], "sample": f"{len(part)} seeds per step"},
+                cpu_baseline=dict(value=v, unit="edges/s", kind="oracle", cores=len(os.sched_getaffinity(0)),
+                                  sample=f"per step one micro-batch of {len(part)} of {len(seeds)} seeds"),
+                e2e=dict(value=v, unit="edges/s", h2d_bytes_per_step=0, d2h_bytes_per_step=0))
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- clocks
+class Clocks:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-i", str(self.index), "-lms", "200"], stdout=subprocess.PIPE,
+                                      stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        out, _ = self.p.communicate()
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in out.strip().splitlines():
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = max(mx, float(f[2]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- our arm
+def fwd_bytes(tr, groups_sizes, cfg, act_bytes, feat_bytes):
+    """Algorithmic bytes of the fused forward: per block edge one source row
+    + its 4-B index; per dst row_ptr, self row, saved h_agg and output row."""
+    from paper_conf_hpca_yangzl25_b200.buffalo import pitch
+    total = 0
+    for n, e in groups_sizes:
+        for l in range(1, cfg.L + 1):
+            s_in = feat_bytes if l == 1 else act_bytes
+            s_out = 4 if l == cfg.L else act_bytes
+            pin, pout = pitch(cfg.dims[l - 1]), pitch(cfg.dims[l])
+            total += e[l - 1] * (pin * s_in + 4)
+            total += n[l] * (4 + pin * s_in + pin * act_bytes + pout * s_out)
+    return total
+
+
+def run_ours(args, cfg):
+    import torch
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    pg = None
+    if world > 1:
+        torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local))
+        pg = torch.distributed.group.WORLD
+    from paper_conf_hpca_yangzl25_b200 import buffalo as B
+    from paper_conf_hpca_yangzl25_b200.train import Trainer
+
+    B.lib()
+    rp, col, X, y, seeds, Ws, bs = make_inputs(cfg)
+    gemm = B.GEMM_BF16 if args.gemm == "bf16" else B.GEMM_FFMA
+    feat_dtype = B.BF16 if args.gemm == "bf16" else B.FP32
+    feats = torch.as_tensor(X).cuda()
+    if feat_dtype == B.BF16:
+        feats = feats.to(torch.bfloat16).contiguous()      # k/128 features are exact in bf16
+    kmin = max(cfg.k_min, world)
+    budget = cfg.mem_budget
+    tr = Trainer((rp, col), feats, torch.as_tensor(y).cuda(), torch.as_tensor(seeds).cuda(), cfg.dims,
+                 cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, mem_budget=budget,
+                 k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg)
+    if args.config == "products":
+        # calibrate M_ctr once so that one GPU needs >= 8 groups, then freeze it for every N
+        B_full = Trainer((rp, col), feats, torch.as_tensor(y).cuda(), torch.as_tensor(seeds).cuda(), cfg.dims,
+                         cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, k_min=1, k_max=1)
+        _, _, est1, _ = B_full.schedule(0)
+        del B_full
+        tr.sched.mem_budget = int(est1[0]) // 8
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    fwd_events = []
+    orig_forward = tr.forward
+
+    def timed_forward():
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        orig_forward()
+        e1.record(stream)
+        fwd_events.append((e0, e1))
+
+    lr = 0.01
+    for i in range(args.warmup):
+        tr.run_epoch(epoch=i, lr=lr)
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    clocks = Clocks(local)
+    clocks.start()
+    tr.forward = timed_forward
+    l0 = B.launch_count()
+    step_ms, edges, sizes, ks = [], 0, [], []
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    for i in range(args.steps):
+        flush.zero_()                                  # L2 flushed between timed steps (outside events)
+        s0 = torch.cuda.Event(enable_timing=True)
+        s1 = torch.cuda.Event(enable_timing=True)
+        s0.record(stream)
+        st = tr.run_epoch(epoch=args.warmup + i, lr=lr)
+        s1.record(stream)
+        s1.synchronize()
+        step_ms.append(s0.elapsed_time(s1))
+        edges += st["edges"]
+        ks.append(st["K"])
+        sizes += [(g["n"], g["e"]) for g in st["groups"]]
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    launches = B.launch_count() - l0
+    clk = clocks.stop()
+    tr.forward = orig_forward
+    total_ms = sum(step_ms)
+    fwd_ms = sum(a.elapsed_time(b) for a, b in fwd_events)
+    act_bytes = 2 if gemm == B.GEMM_BF16 else 4
+    fbytes = fwd_bytes(tr, sizes, cfg, act_bytes, 2 if feat_dtype == B.BF16 else 4)
+    n_fwd = len(fwd_events)
+    if world > 1:
+        t = torch.tensor([total_ms, edges, fwd_ms, fbytes], dtype=torch.float64, device="cuda")
+        mx = t.clone()
+        torch.distributed.all_reduce(mx, op=torch.distributed.ReduceOp.MAX)
+        sm = t.clone()
+        torch.distributed.all_reduce(sm, op=torch.distributed.ReduceOp.SUM)
+        total_ms, edges = float(mx[0]), float(sm[1])
+    value = edges / (total_ms / 1e3)
+
+    # end to end through the public API with host buffers: H2D of the step's seed batch from
+    # pinned memory, D2H of the loss, copies inside the timed region
+    seeds_h = torch.as_tensor(seeds).pin_memory()
+    loss_h = torch.empty(1, dtype=torch.float32).pin_memory()
+    e2e_ms, e2e_edges = [], 0
+    for i in range(max(1, args.steps)):
+        flush.zero_()
+        s0 = torch.cuda.Event(enable_timing=True)
+        s1 = torch.cuda.Event(enable_timing=True)
+        s0.record(stream)
+        tr.seeds.copy_(seeds_h, non_blocking=True)
+        st = tr.run_epoch(epoch=1000 + i, lr=lr)
+        loss_h.copy_(tr.loss, non_blocking=True)
+        s1.record(stream)
+        s1.synchronize()
+        e2e_ms.append(s0.elapsed_time(s1))
+        e2e_edges += st["edges"]
+    e2e_val = e2e_edges / (sum(e2e_ms) / 1e3)
+    if world > 1:
+        t = torch.tensor([sum(e2e_ms), e2e_edges], dtype=torch.float64, device="cuda")
+        mx = t.clone()
+        torch.distributed.all_reduce(mx, op=torch.distributed.ReduceOp.MAX)
+        sm = t.clone()
+        torch.distributed.all_reduce(sm, op=torch.distributed.ReduceOp.SUM)
+        e2e_val = float(sm[1]) / (float(mx[0]) / 1e3)
+
+    peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(peaks_path):
+        peak, peak_src = json.load(open(peaks_path))["hbm_gbs"], "measured (MEASURED_PEAKS.json hbm_gbs)"
+    else:
+        peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
+    achieved = fbytes / (fwd_ms / 1e3) / 1e9 if fwd_ms > 0 else 0.0
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        traffic = json.load(open(tpath)).get(f"{args.config}/{args.gemm}")
+    if rank == 0:
+        cpu = None
+        if world == 1 and not args.no_cpu_baseline:
+            cpu = oracle_sample(cfg, rp, col, X, y, seeds, Ws, bs, args.cpu_baseline_seconds)
+        line = dict(
+            metric="aggregated edges/s (epoch of Buffalo hot path)", value=value, unit="edges/s",
+            n_gpus=world, steps=args.steps, warmup=args.warmup, ms_per_step=total_ms / args.steps,
+            higher_is_better=True, scaling="strong", vs_baseline=None,
+            dtype="bf16" if gemm == B.GEMM_BF16 else "f32", data="synthetic",
+            config={"workload": WORKLOADS[args.config], "config": args.config, "K": ks[-1],
+                    "gemm": args.gemm, "l2": "flushed (512 MiB write) between timed steps",
+                    "epoch_ms": total_ms / args.steps, "edges_per_epoch": edges / args.steps,
+                    "parallelism": f"dp{world} over bucket groups"},
+            roofline={"bound": "hbm", "kernel": "buffalo_sage_fwd (fused gather-mean + Update GEMM)",
+                      "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                      "traffic": traffic, "peak_source": peak_src,
+                      "algorithmic_bytes_per_launch": fbytes / max(1, n_fwd),
+                      "launch_ms": fwd_ms / max(1, n_fwd), "share_of_step": fwd_ms / total_ms},
+            cpu_baseline=cpu,
+            e2e={"value": e2e_val, "unit": "edges/s", "h2d_bytes_per_step": 4 * len(seeds),
+                 "d2h_bytes_per_step": 4},
+            gpu_launches=launches, clocks=clk)
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+def main():
+    args = parse()
+    cfg = CONFIGS[args.config]
+    if args.impl == "reference":
+        run_reference(args, cfg)
+    else:
+        run_ours(args, cfg)
+
+
+if __name__ == "__main__":
+    main()

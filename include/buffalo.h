@@ -1,0 +1,229 @@
+/*
+ * buffalo.h — C ABI of the B200-native hot path of Buffalo (Yang, Zhang, Li, HPCA'25).
+ *
+ * Paper text: /root/reference/PAPER.md (cited PAPER.md:<line>); readings R<n> are listed in
+ * DESIGN.md §2.  Implemented by libbuffalo.so (sm_100a CUDA; no CPU fallback).
+ *
+ * Conventions (all entry points):
+ *  - Pointers are DEVICE pointers unless the name ends in _h (host).  All device memory is
+ *    allocated and owned by the caller; the library never calls cudaMalloc/cudaFree.
+ *  - `stream` is a cudaStream_t passed as void*.  Work is stream-ordered; the only host
+ *    synchronisations are the documented ones (data-dependent sizes).
+ *  - Errors are returned as buffalo_status (never exceptions/abort); on error, outputs are
+ *    unspecified except *required_bytes_h.  buffalo_last_error() gives a thread-local message.
+ *  - Deterministic: identical inputs and seed give bit-identical outputs.
+ *  - Built for sm_100a only; on any other device BUFFALO_ERR_UNSUPPORTED.
+ *  - A graph's node_map workspace must not be used by two streams at once.
+ */
+#ifndef BUFFALO_H
+#define BUFFALO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define BUFFALO_API __attribute__((visibility("default")))
+#else
+#define BUFFALO_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  BUFFALO_OK = 0,
+  BUFFALO_ERR_INVALID_ARG = 1, /* null/misaligned pointer, bad dims, unsupported fanout > 32  */
+  BUFFALO_ERR_BUDGET = 2,      /* Alg. 3: no K in [k_min, k_max] satisfies M_ctr            */
+  BUFFALO_ERR_CAPACITY = 3,    /* caller buffer/arena too small; *required_bytes_h is set   */
+  BUFFALO_ERR_CUDA = 4,        /* CUDA launch/runtime error; see buffalo_last_error()       */
+  BUFFALO_ERR_UNSUPPORTED = 5  /* dtype/dim/arch combination not built (e.g. not sm_100a)   */
+} buffalo_status;
+
+enum { BUFFALO_FP32 = 0, BUFFALO_BF16 = 1 };            /* storage dtypes                  */
+enum { BUFFALO_GEMM_FFMA = 0, BUFFALO_GEMM_BF16 = 1 };  /* Update GEMM: fp32 SIMT | tcgen05 */
+enum { BUFFALO_MAX_LAYERS = 8, BUFFALO_MAX_FANOUT = 32, BUFFALO_MAX_DIM = 4096 };
+
+/* Input graph (the batch's host graph): CSR, rows sorted ascending, symmetric,
+ * no self loops or duplicates.  row_ptr int64[num_nodes+1], col int32[nnz].  node_map is a
+ * workspace int32[num_nodes] prepared once by buffalo_graph_prepare (all INT32_MAX) and
+ * restored by every call that uses it. */
+typedef struct {
+  int64_t num_nodes, nnz;
+  const int64_t* row_ptr;
+  const int32_t* col;
+  int32_t* node_map;
+} buffalo_graph;
+
+/* Sampling (R1, R2): fanout[l-1] is block l's fanout (<= 0: all neighbours, else <= 32);
+ * block l uses hop h = L-l+1; cutoff_F is the degree-bucketing cut-off F;
+ * seed keys Philox4x32-10 (per epoch: base + epoch). */
+typedef struct {
+  int32_t num_layers;
+  int32_t fanout[BUFFALO_MAX_LAYERS];
+  int32_t cutoff_F;
+  uint64_t seed;
+} buffalo_sampler;
+
+/* GraphSAGE-mean model (R20): dim[0] = input feature width, dim[L] = #classes.
+ * feat_dtype: dtype of the global feature table (row pitch feat_pitch elements, 16-B aligned
+ * rows).  gemm_mode FFMA keeps activations in fp32; BF16 stores activations (H_l, saved
+ * h_agg) in bf16 and runs the Update GEMM on tcgen05 tensor cores (fp32 accumulate). */
+typedef struct {
+  int32_t num_layers;
+  int32_t dim[BUFFALO_MAX_LAYERS + 1];
+  int32_t feat_dtype;
+  int32_t gemm_mode;
+  int64_t feat_pitch;
+} buffalo_model;
+
+/* Scheduler parameters (Alg. 3): mem_budget = M_ctr in bytes (arena bytes
+ * of one micro-batch, R15); C_ppm = average clustering coefficient x 10^6 (Eq. 1, <= 0: R = 1);
+ * K searched in [max(k_min, num_gpus), k_max]. */
+typedef struct {
+  int64_t mem_budget;
+  int64_t C_ppm;
+  int32_t k_min, k_max, num_gpus;
+} buffalo_sched;
+
+/* Output of buffalo_bucketize.  Device arrays sized by the caller: group_of_seed[n_seeds],
+ * group_seeds[n_seeds], group_offsets[k_max+1]; host arrays est_bytes_h[k_max],
+ * rank_of_group_h[k_max], group_offsets_h[k_max+1], hist_h[cutoff_F+1]. */
+typedef struct {
+  int32_t* group_of_seed;   /* group of seeds[i]                                            */
+  int32_t* group_seeds;     /* seeds grouped; inside a group by (bucket, micro-bucket), input order */
+  int64_t* group_offsets;   /* group k = group_seeds[off[k] .. off[k+1])                     */
+  int64_t* group_offsets_h;
+  int64_t* est_bytes_h;     /* Eq. 2 estimate per group                       */
+  int32_t* rank_of_group_h; /* LPT assignment of groups to num_gpus ranks (R24)              */
+  int64_t* hist_h;          /* degree-bucket histogram of the seeds, [cutoff_F + 1]           */
+  int32_t k_out;            /* number of non-empty groups                                     */
+  int32_t k_tried;          /* the K at which Alg. 4 succeeded                               */
+  int32_t exploded;         /* 1 if the degree-F bucket was split (R7)                       */
+  int32_t num_items;
+} buffalo_plan;
+
+/* One block (bipartite layer) of a micro-batch, all views into the caller's arena.
+ * src_global[0..n_dst) are the dst nodes (R3/R4).  row_ptr int32[n_dst+1] (CSR by dst,
+ * neighbours in ascending CSR position), col_local int32[n_edges] (index into src),
+ * col_global (block 1 only, else NULL) int32[n_edges], t_row_ptr/t_col: transposed block
+ * (block >= 2 only, else NULL): for each src j the dst i with an edge to j, ascending.
+ * heavy int32[n_heavy]: dst with D > 128 (long-tail cooperative path), ascending.
+ * Activations of the standard arena layout: agg (saved h_agg [n_dst][ld_agg]), out (H_l
+ * [n_dst][ld_out], act dtype, or logits fp32 at l = L), dh (dH_l / dlogits fp32 [n_dst][ld_dh],
+ * valid during the backward of layers l and l+1), bwd_scratch (bwd_scratch_bytes). */
+typedef struct {
+  int64_t n_dst, n_src, n_edges, n_heavy;
+  int32_t *row_ptr, *col_local, *col_global, *src_global, *t_row_ptr, *t_col, *heavy;
+  void* agg;
+  void* out;
+  float* dh;
+  void* bwd_scratch;
+  int64_t ld_agg, ld_out, ld_dh, bwd_scratch_bytes;
+} buffalo_block;
+
+typedef struct {
+  int32_t num_layers;
+  buffalo_block layer[BUFFALO_MAX_LAYERS]; /* layer[l-1] = block l                          */
+  int64_t arena_used;  /* bytes reserved at the bottom (blocks + activations)               */
+  int64_t arena_peak;  /* high-water mark incl. build and backward scratch frames           */
+  int64_t est_lo, est_hi; /* buffalo_estimate_mem of the built sizes                       */
+} buffalo_blocks;
+
+/* ------------------------------------------------------------------ graph workspace */
+/* Bytes of the node_map workspace (int32 per node, 256-B rounded). */
+BUFFALO_API size_t buffalo_graph_workspace_bytes(int64_t num_nodes);
+/* Sets g->node_map = workspace and fills it with INT32_MAX (stream-ordered). */
+BUFFALO_API buffalo_status buffalo_graph_prepare(buffalo_graph* g, void* workspace, size_t bytes, void* stream);
+
+/* ------------------------------------------------------------------ a1-a3: scheduler */
+/* Upper bound of the workspace buffalo_bucketize needs for n_seeds seeds. */
+BUFFALO_API size_t buffalo_bucketize_workspace_bytes(const buffalo_graph* g, int64_t n_seeds,
+                                         const buffalo_sampler* s, const buffalo_model* m);
+/* Buffalo_Scheduler (Alg. 3) with DegreeBucketing (l.1), per-item I/O/D and
+ * BucketMemEstimator (R13, R15, obtained by building each item's blocks on the GPU),
+ * Eq. 1-2, SplitExplosionBucket (R7, R8) and MemBalancedGrouping (Alg. 4,
+ * PAPER.md:313-326, R10-R12).  seeds: device int32[n_seeds] (distinct global ids).
+ * Synchronises the stream (data-dependent sizes).  BUFFALO_ERR_BUDGET if no K fits M_ctr;
+ * BUFFALO_ERR_CAPACITY if workspace_bytes is too small. */
+BUFFALO_API buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, int64_t n_seeds,
+                                 const buffalo_sampler* s, const buffalo_model* m,
+                                 const buffalo_sched* sc, buffalo_plan* plan, void* workspace,
+                                 size_t workspace_bytes, void* stream);
+
+/* ------------------------------------------------------------------ a4-a6: blocks */
+/* MicroBatchGenerator / BlockGenerate (Alg. 2 l.5 PAPER.md:237, §IV-E): the L
+ * blocks of the micro-batch whose output nodes are group_seeds[0..n), built top-down, plus the
+ * activation and backward buffers of the standard arena layout.  arena: device,
+ * 256-B aligned.  Synchronises twice per layer.  BUFFALO_ERR_CAPACITY: *required_bytes_h gets a
+ * lower bound of the bytes needed (the exact need once all sizes are known). */
+BUFFALO_API buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group_seeds, int64_t n,
+                                    const buffalo_sampler* s, const buffalo_model* m,
+                                    buffalo_blocks* out, void* arena, size_t arena_bytes,
+                                    int64_t* required_bytes_h, void* stream);
+
+/* ------------------------------------------------------------------ a7: forward */
+/* Packed copy of W_l [dim[l], 2*dim[l-1]] fp32 for the kernels (transposes / padded bf16). */
+BUFFALO_API size_t buffalo_packed_weight_bytes(const buffalo_model* m, int32_t layer);
+BUFFALO_API buffalo_status buffalo_pack_weights(const buffalo_model* m, int32_t layer, const float* W,
+                                    void* packed, void* stream);
+
+/* GraphSAGE-mean layer l (Aggregate + Update, Alg. 2 l.8-9, R20/R21):
+ *   h_agg[i] = (sum_{e in row i} H[col[e]]) / D(i)   (0 if D(i) = 0),
+ *   Z = [H[i] || h_agg[i]] W^T + b;  out = ReLU(Z) (act dtype) for l < L, Z (fp32) for l = L.
+ * h_src: for layer 1 the global feature table (feat dtype, row pitch m->feat_pitch, rows
+ * addressed by global id through col_global/src_global); for l > 1 H_{l-1} (act dtype, ld_src).
+ * saved_agg receives h_agg (act dtype, ld_agg) for the backward.  W fp32 [d_out][2 d_in],
+ * W_packed from buffalo_pack_weights, b fp32 [d_out]. */
+BUFFALO_API buffalo_status buffalo_sage_fwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                const void* h_src, int64_t ld_src, const float* W,
+                                const void* W_packed, const float* b, void* out, int64_t ld_out,
+                                void* saved_agg, int64_t ld_agg, void* stream);
+
+/* ------------------------------------------------------------------ a8: loss */
+/* Partial loss of a group (Alg. 2 l.10, R19): loss_accum[0] += sum_i CE(softmax(Z_i), y_i) / S
+ * and dlogits = (softmax(Z) - onehot(y)) / S, with y_i = labels[row_ids[i]]. */
+BUFFALO_API buffalo_status buffalo_softmax_ce(const float* logits, int64_t ld, int64_t n, int32_t classes,
+                                  const int32_t* labels, const int32_t* row_ids,
+                                  int64_t batch_size, float* loss_accum, float* dlogits,
+                                  int64_t ld_d, void* stream);
+
+/* ------------------------------------------------------------------ a9: backward */
+/* Scratch bytes buffalo_sage_bwd needs for block blk at layer l. */
+BUFFALO_API size_t buffalo_sage_bwd_scratch_bytes(const buffalo_block* blk, int32_t layer,
+                                      const buffalo_model* m);
+/* Backward of layer l (Alg. 2 l.11-12).  dh_dst: dH_l fp32 (l < L; turned
+ * into dZ_l = dH_l * 1[H_l > 0] IN PLACE using h_dst) or dlogits (l = L).
+ *   dW_accum += dZ^T [H[:n_dst] || h_agg];  db_accum += sum_i dZ[i]   (accumulated, R19)
+ *   l > 1: dh_src = pad(dZ W_self) + (sum_{i: j in N(i)} dZ[i] / D(i)) W_neigh   (dH_{l-1})
+ * Pass dh_src = NULL for layer 1 (features are not trained). */
+BUFFALO_API buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
+                                const void* saved_agg, int64_t ld_agg, const void* h_dst,
+                                int64_t ld_hdst, const float* W, const void* W_packed,
+                                float* dW_accum, float* db_accum, float* dh_src,
+                                int64_t ld_dh_src, void* scratch, size_t scratch_bytes,
+                                void* stream);
+
+/* ------------------------------------------------------------------ a10: optimizer */
+/* SGD (Alg. 2 l.13, R18): param -= lr * grad; grad = 0 (ready for the next epoch). */
+BUFFALO_API buffalo_status buffalo_sgd_step(float* param, float* grad, int64_t n, float lr, void* stream);
+
+/* ------------------------------------------------------------------ memory model */
+/* BucketMemEstimator reading R15: exact arena bytes of a micro-batch with
+ * layer sizes n[0..L] and e[0..L-1] (e[l-1] = edges of block l).  hi = capacity that always
+ * suffices (the scheduler's M_est), lo = bytes the backward is certain to touch; the measured
+ * arena peak lies in [lo, hi].  Pure host function. */
+BUFFALO_API buffalo_status buffalo_estimate_mem(int32_t num_layers, const int64_t* n, const int64_t* e,
+                                    const buffalo_model* m, int64_t* lo_bytes_h,
+                                    int64_t* hi_bytes_h);
+
+/* Number of kernels this thread has launched through the library (for bench accounting). */
+BUFFALO_API int64_t buffalo_launch_count(void);
+BUFFALO_API const char* buffalo_status_str(buffalo_status s);
+BUFFALO_API const char* buffalo_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BUFFALO_H */

@@ -170,13 +170,18 @@ def degree_bucketing(g, seeds, f_L, F):
 
 # ============================================================================ memory model
 ALIGN = 256
-SCAN_WS = 8192
 HEAVY_T = 128          # rows with D > HEAVY_T go through the cooperative long-tail path
 FP32, BF16 = 0, 1
+SCAN_TILE = 16384      # elements per scan tile of the implementation's device-wide scans
+PART_TILE = 4096       # elements per tile of its stable radix/bin partition passes
 
 
 def _R(x):
     return ((int(x) + ALIGN - 1) // ALIGN) * ALIGN
+
+
+def _ceil(a, b):
+    return (int(a) + int(b) - 1) // int(b)
 
 
 def pitch(d):
@@ -184,9 +189,17 @@ def pitch(d):
 
 
 def dw_splits(n_l, d_out, d_in):
-    """Split count of the deterministic split-K dW reduction (DESIGN.md "Arena")."""
-    tiles = math.ceil(d_out / 64) * math.ceil(2 * d_in / 64)
-    return max(1, min(math.ceil(296 / tiles), math.ceil(int(n_l) / 512)))
+    """Split count of the deterministic split-K dW reduction (DESIGN.md §5)."""
+    tiles = _ceil(d_out, 64) * _ceil(2 * d_in, 64)
+    return max(1, min(_ceil(296, tiles), _ceil(n_l, 512)))
+
+
+def _part_count_elems(e):
+    return 256 * _ceil(max(int(e), 1), PART_TILE)
+
+
+def _scan_ws_bytes(length):
+    return _R(4 * (_ceil(max(int(length), 1), SCAN_TILE) + 2))
 
 
 def mem_model(n, e, dims, act_dtype=FP32):
@@ -194,35 +207,37 @@ def mem_model(n, e, dims, act_dtype=FP32):
     micro-batch with layer sizes n[0..L], e[1..L] (e indexed l-1) and widths dims[0..L].
     Returns (lo, hi): hi = capacity that always suffices (used as M_est), lo = bytes the
     backward pass is certain to touch; the measured arena peak lies in [lo, hi].
-    Every buffer is rounded up to 256 B.  Layout restated from DESIGN.md §"Arena"."""
+    Every buffer is rounded up to 256 B.  Restated from DESIGN.md §5 "Arena"."""
     L = len(e)
     s = 4 if act_dtype == FP32 else 2
     blocks = 0
     build = 0
     for l in range(1, L + 1):
         nl, nm, el = n[l], n[l - 1], e[l - 1]
-        blocks += _R(4 * (nl + 1)) + _R(4 * el) + _R(4 * nm) + _R(4 * nl)
+        blocks += _R(4 * (nl + 1)) + _R(4 * nl) + _R(4 * el) + _R(4 * nm)   # row_ptr heavy col src
         if l == 1:
-            blocks += _R(4 * el)                               # col_global kept for layer 1
+            blocks += _R(4 * el)                                # col_global kept for layer 1
         else:
-            blocks += _R(4 * (nm + 1)) + _R(4 * el)            # transposed block
-        frame = _R(4 * (nl + el + 1)) + SCAN_WS
+            blocks += _R(4 * (nm + 1)) + _R(4 * el)             # transposed block
+        pc = _part_count_elems(el)
+        frame = _R(64) + _scan_ws_bytes(max(nl + el + 1, pc + 1))
         if l >= 2:
-            frame += _R(4 * el) + _R(4 * nm)
+            frame += 6 * _R(4 * el) + _R(4 * (pc + 1))          # col_global + radix buffers
         build = max(build, frame)
     acts = 0
     for l in range(1, L + 1):
-        acts += _R(n[l] * pitch(dims[l - 1]) * s)              # saved h_agg
+        acts += _R(n[l] * pitch(dims[l - 1]) * s)               # saved h_agg
         if l < L:
-            acts += _R(n[l] * pitch(dims[l]) * s)              # H_l
-    acts += _R(n[L] * pitch(dims[L]) * 4)                      # logits
+            acts += _R(n[l] * pitch(dims[l]) * s)               # H_l
+    acts += _R(n[L] * pitch(dims[L]) * 4)                       # logits
     bwd = 0
     for l in range(L, 0, -1):
-        frame = _R(n[l] * pitch(dims[l]) * 4)                  # dH_l (dlogits at l = L)
+        frame = _R(n[l] * pitch(dims[l]) * 4)                   # dH_l (dlogits at l = L)
         if l >= 2:
-            frame += _R(n[l - 1] * pitch(dims[l - 1]) * 4)     # dH_{l-1}
-            frame += _R(n[l - 1] * pitch(dims[l]) * 4)         # transposed aggregate of dZ/D
-        frame += _R(dw_splits(n[l], dims[l], dims[l - 1]) * dims[l] * 2 * dims[l - 1] * 4)
+            frame += _R(n[l - 1] * pitch(dims[l - 1]) * 4)      # dH_{l-1}
+            frame += _R(n[l - 1] * pitch(dims[l]) * 4)          # transposed aggregate of dZ/D
+        S = dw_splits(n[l], dims[l], dims[l - 1])
+        frame += _R(S * dims[l] * 2 * dims[l - 1] * 4) + _R(S * pitch(dims[l]) * 4)  # dW, db partials
         bwd = max(bwd, frame)
     lo = blocks + acts + bwd
     hi = blocks + acts + max(bwd, build)

@@ -1,0 +1,252 @@
+"""Thin ctypes binding of include/buffalo.h (argument marshalling only).
+
+Every function here forwards to libbuffalo.so with the same name minus the `buffalo_` prefix.
+Device buffers are torch CUDA tensors (PyTorch is used for device memory and streams only);
+there is no CPU fallback: loading fails loudly without the built library or a GPU.
+"""
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libbuffalo.so")
+
+c_i32, c_i64, c_u64, c_p, c_sz, c_f = (ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64,
+                                       ctypes.c_void_p, ctypes.c_size_t, ctypes.c_float)
+
+OK, ERR_INVALID_ARG, ERR_BUDGET, ERR_CAPACITY, ERR_CUDA, ERR_UNSUPPORTED = range(6)
+FP32, BF16 = 0, 1
+GEMM_FFMA, GEMM_BF16 = 0, 1
+MAX_LAYERS = 8
+
+EXPORTS = [
+    "buffalo_graph_workspace_bytes", "buffalo_graph_prepare", "buffalo_bucketize_workspace_bytes",
+    "buffalo_bucketize", "buffalo_build_blocks", "buffalo_packed_weight_bytes",
+    "buffalo_pack_weights", "buffalo_sage_fwd", "buffalo_softmax_ce",
+    "buffalo_sage_bwd_scratch_bytes", "buffalo_sage_bwd", "buffalo_sgd_step",
+    "buffalo_estimate_mem", "buffalo_launch_count", "buffalo_status_str", "buffalo_last_error",
+]
+
+
+class BuffaloError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+_STATUS = {0: "BUFFALO_OK", 1: "BUFFALO_ERR_INVALID_ARG", 2: "BUFFALO_ERR_BUDGET",
+           3: "BUFFALO_ERR_CAPACITY", 4: "BUFFALO_ERR_CUDA", 5: "BUFFALO_ERR_UNSUPPORTED"}
+
+
+class Graph(ctypes.Structure):
+    _fields_ = [("num_nodes", c_i64), ("nnz", c_i64), ("row_ptr", c_p), ("col", c_p), ("node_map", c_p)]
+
+
+class Sampler(ctypes.Structure):
+    _fields_ = [("num_layers", c_i32), ("fanout", c_i32 * MAX_LAYERS), ("cutoff_F", c_i32), ("seed", c_u64)]
+
+
+class Model(ctypes.Structure):
+    _fields_ = [("num_layers", c_i32), ("dim", c_i32 * (MAX_LAYERS + 1)), ("feat_dtype", c_i32),
+                ("gemm_mode", c_i32), ("feat_pitch", c_i64)]
+
+
+class Sched(ctypes.Structure):
+    _fields_ = [("mem_budget", c_i64), ("C_ppm", c_i64), ("k_min", c_i32), ("k_max", c_i32),
+                ("num_gpus", c_i32)]
+
+
+class Plan(ctypes.Structure):
+    _fields_ = [("group_of_seed", c_p), ("group_seeds", c_p), ("group_offsets", c_p),
+                ("group_offsets_h", c_p), ("est_bytes_h", c_p), ("rank_of_group_h", c_p),
+                ("hist_h", c_p), ("k_out", c_i32), ("k_tried", c_i32), ("exploded", c_i32),
+                ("num_items", c_i32)]
+
+
+class Block(ctypes.Structure):
+    _fields_ = [("n_dst", c_i64), ("n_src", c_i64), ("n_edges", c_i64), ("n_heavy", c_i64),
+                ("row_ptr", c_p), ("col_local", c_p), ("col_global", c_p), ("src_global", c_p),
+                ("t_row_ptr", c_p), ("t_col", c_p), ("heavy", c_p),
+                ("agg", c_p), ("out", c_p), ("dh", c_p), ("bwd_scratch", c_p),
+                ("ld_agg", c_i64), ("ld_out", c_i64), ("ld_dh", c_i64), ("bwd_scratch_bytes", c_i64)]
+
+
+class Blocks(ctypes.Structure):
+    _fields_ = [("num_layers", c_i32), ("layer", Block * MAX_LAYERS), ("arena_used", c_i64),
+                ("arena_peak", c_i64), ("est_lo", c_i64), ("est_hi", c_i64)]
+
+
+_lib = None
+
+
+def lib(require_gpu=True):
+    """Load libbuffalo.so (raises if it is missing or, with require_gpu, if there is no GPU)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"libbuffalo.so not built ({LIB_PATH}); run __graft_entry__.build()")
+        L = ctypes.CDLL(LIB_PATH)
+        P = c_p
+        sig = {
+            "buffalo_graph_workspace_bytes": (c_sz, [c_i64]),
+            "buffalo_graph_prepare": (c_i32, [P, P, c_sz, P]),
+            "buffalo_bucketize_workspace_bytes": (c_sz, [P, c_i64, P, P]),
+            "buffalo_bucketize": (c_i32, [P, P, c_i64, P, P, P, P, P, c_sz, P]),
+            "buffalo_build_blocks": (c_i32, [P, P, c_i64, P, P, P, P, c_sz, P, P]),
+            "buffalo_packed_weight_bytes": (c_sz, [P, c_i32]),
+            "buffalo_pack_weights": (c_i32, [P, c_i32, P, P, P]),
+            "buffalo_sage_fwd": (c_i32, [P, c_i32, P, P, c_i64, P, P, P, P, c_i64, P, c_i64, P]),
+            "buffalo_softmax_ce": (c_i32, [P, c_i64, c_i64, c_i32, P, P, c_i64, P, P, c_i64, P]),
+            "buffalo_sage_bwd_scratch_bytes": (c_sz, [P, c_i32, P]),
+            "buffalo_sage_bwd": (c_i32, [P, c_i32, P, P, c_i64, P, c_i64, P, c_i64, P, c_i64, P, P,
+                                         P, P, P, c_i64, P, c_sz, P]),
+            "buffalo_sgd_step": (c_i32, [P, P, c_i64, c_f, P]),
+            "buffalo_estimate_mem": (c_i32, [c_i32, P, P, P, P, P]),
+            "buffalo_launch_count": (c_i64, []),
+            "buffalo_status_str": (ctypes.c_char_p, [c_i32]),
+            "buffalo_last_error": (ctypes.c_char_p, []),
+        }
+        for name, (res, args) in sig.items():
+            fn = getattr(L, name)
+            fn.restype = res
+            fn.argtypes = args
+        _lib = L
+    if require_gpu and not torch.cuda.is_available():
+        raise RuntimeError("libbuffalo needs a CUDA device (sm_100a); there is no CPU fallback")
+    return _lib
+
+
+def _check(status):
+    if status != OK:
+        raise BuffaloError(status, lib(False).buffalo_last_error().decode())
+
+
+def ptr(t):
+    if t is None:
+        return None
+    if isinstance(t, int):
+        return t
+    return t.data_ptr()
+
+
+def stream_ptr(stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return s.cuda_stream
+
+
+def ref(x):
+    return ctypes.byref(x) if x is not None else None
+
+
+# ------------------------------------------------------------------------- wrappers
+def graph_workspace_bytes(num_nodes):
+    return lib(False).buffalo_graph_workspace_bytes(num_nodes)
+
+
+def graph_prepare(graph, workspace, stream=None):
+    _check(lib().buffalo_graph_prepare(ref(graph), ptr(workspace), workspace.numel() * workspace.element_size(),
+                                       stream_ptr(stream)))
+
+
+def bucketize_workspace_bytes(graph, n_seeds, sampler, model):
+    return lib(False).buffalo_bucketize_workspace_bytes(ref(graph), n_seeds, ref(sampler), ref(model))
+
+
+def bucketize(graph, seeds, sampler, model, sched, plan, workspace, stream=None):
+    _check(lib().buffalo_bucketize(ref(graph), ptr(seeds), seeds.numel(), ref(sampler), ref(model),
+                                   ref(sched), ref(plan), ptr(workspace), workspace.numel(),
+                                   stream_ptr(stream)))
+
+
+def build_blocks(graph, group_seeds, n, sampler, model, blocks, arena, stream=None):
+    """Returns BUFFALO_OK or raises; on BUFFALO_ERR_CAPACITY the error carries .required."""
+    req = c_i64(0)
+    st = lib().buffalo_build_blocks(ref(graph), ptr(group_seeds), n, ref(sampler), ref(model),
+                                    ref(blocks), ptr(arena), arena.numel(), ctypes.byref(req),
+                                    stream_ptr(stream))
+    if st == ERR_CAPACITY:
+        err = BuffaloError(st, lib(False).buffalo_last_error().decode())
+        err.required = req.value
+        raise err
+    _check(st)
+    return req.value
+
+
+def packed_weight_bytes(model, layer):
+    return lib(False).buffalo_packed_weight_bytes(ref(model), layer)
+
+
+def pack_weights(model, layer, W, packed, stream=None):
+    _check(lib().buffalo_pack_weights(ref(model), layer, ptr(W), ptr(packed), stream_ptr(stream)))
+
+
+def sage_fwd(blk, layer, model, h_src, ld_src, W, W_packed, b, out, ld_out, saved_agg, ld_agg, stream=None):
+    _check(lib().buffalo_sage_fwd(ref(blk), layer, ref(model), ptr(h_src), ld_src, ptr(W), ptr(W_packed),
+                                  ptr(b), ptr(out), ld_out, ptr(saved_agg), ld_agg, stream_ptr(stream)))
+
+
+def softmax_ce(logits, ld, n, classes, labels, row_ids, batch_size, loss_accum, dlogits, ld_d, stream=None):
+    _check(lib().buffalo_softmax_ce(ptr(logits), ld, n, classes, ptr(labels), ptr(row_ids), batch_size,
+                                    ptr(loss_accum), ptr(dlogits), ld_d, stream_ptr(stream)))
+
+
+def sage_bwd_scratch_bytes(blk, layer, model):
+    return lib(False).buffalo_sage_bwd_scratch_bytes(ref(blk), layer, ref(model))
+
+
+def sage_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg, h_dst, ld_hdst, W,
+             W_packed, dW, db, dh_src, ld_dh_src, scratch, scratch_bytes, stream=None):
+    _check(lib().buffalo_sage_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh, ptr(h_src), ld_src,
+                                  ptr(saved_agg), ld_agg, ptr(h_dst), ld_hdst, ptr(W), ptr(W_packed),
+                                  ptr(dW), ptr(db), ptr(dh_src), ld_dh_src, ptr(scratch), scratch_bytes,
+                                  stream_ptr(stream)))
+
+
+def sgd_step(param, grad, lr, stream=None):
+    _check(lib().buffalo_sgd_step(ptr(param), ptr(grad), param.numel(), lr, stream_ptr(stream)))
+
+
+def estimate_mem(n, e, model):
+    L = len(e)
+    na = (c_i64 * (L + 1))(*n)
+    ea = (c_i64 * L)(*e)
+    lo, hi = c_i64(0), c_i64(0)
+    _check(lib(False).buffalo_estimate_mem(L, na, ea, ref(model), ctypes.byref(lo), ctypes.byref(hi)))
+    return lo.value, hi.value
+
+
+def launch_count():
+    return lib(False).buffalo_launch_count()
+
+
+# ------------------------------------------------------------------------- struct helpers
+def make_sampler(fanout, F, seed):
+    s = Sampler()
+    s.num_layers = len(fanout)
+    for i, f in enumerate(fanout):
+        s.fanout[i] = int(f)
+    s.cutoff_F = int(F)
+    s.seed = int(seed)
+    return s
+
+
+def make_model(dims, feat_dtype=FP32, gemm_mode=GEMM_FFMA, feat_pitch=None):
+    m = Model()
+    m.num_layers = len(dims) - 1
+    for i, d in enumerate(dims):
+        m.dim[i] = int(d)
+    m.feat_dtype = feat_dtype
+    m.gemm_mode = gemm_mode
+    m.feat_pitch = int(feat_pitch if feat_pitch else ((dims[0] + 7) // 8) * 8)
+    return m
+
+
+def make_sched(mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096, num_gpus=1):
+    s = Sched()
+    s.mem_budget, s.C_ppm, s.k_min, s.k_max, s.num_gpus = int(mem_budget), int(C_ppm), k_min, k_max, num_gpus
+    return s
+
+
+def pitch(d):
+    return ((int(d) + 7) // 8) * 8

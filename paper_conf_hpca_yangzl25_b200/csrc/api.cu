@@ -1,0 +1,633 @@
+// api.cu — the C ABI (include/buffalo.h): validation, arena layout, the scheduler's K loop
+// (Alg. 3/4) and the memory model (R15).  Host code; all compute is in build.cu / sage.cu /
+// tc_sage.cu kernels.
+#include <algorithm>
+#include <atomic>
+#include <cstdarg>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "build.cuh"
+#include "common.cuh"
+#include "primitives.cuh"
+#include "sage.cuh"
+#include "tc_sage.cuh"
+
+namespace buffalo {
+
+static thread_local std::string g_err;
+static std::atomic<int64_t> g_launches{0};
+
+void set_error(const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+}
+void count_launch(int n) { g_launches += n; }
+
+buffalo_status check_cuda(const char* what) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    set_error("%s: %s", what, cudaGetErrorString(e));
+    return BUFFALO_ERR_CUDA;
+  }
+  return BUFFALO_OK;
+}
+
+buffalo_status require_sm100() {
+  int dev = 0;
+  BF_CUDA(cudaGetDevice(&dev));
+  int major = 0, minor = 0;
+  BF_CUDA(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev));
+  BF_CUDA(cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev));
+  if (major != 10 || minor != 0) {
+    set_error("libbuffalo is built for sm_100a only (device %d is sm_%d%d)", dev, major, minor);
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
+  return BUFFALO_OK;
+}
+
+__global__ void k_fill_i32(int32_t* a, int64_t n, int32_t v) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
+    a[k] = v;
+}
+
+// ------------------------------------------------------------------ memory model (R15)
+// Restated from DESIGN.md §5; must agree with the arena that buffalo_build_blocks lays out.
+static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_model* m,
+                      int64_t* lo, int64_t* hi) {
+  const int64_t s = m->gemm_mode == BUFFALO_GEMM_BF16 ? 2 : 4;
+  int64_t blocks = 0, build = 0, acts = 0, bwd = 0;
+  for (int l = 1; l <= L; ++l) {
+    const int64_t nl = n[l], nm = n[l - 1], el = e[l - 1];
+    blocks += R(4 * (nl + 1)) + R(4 * nl) + R(4 * el) + R(4 * nm);
+    blocks += (l == 1) ? R(4 * el) : R(4 * (nm + 1)) + R(4 * el);
+    build = std::max(build, build_frame_bytes(nl, el, l, false));
+  }
+  for (int l = 1; l <= L; ++l) {
+    acts += R(n[l] * pitch_of(m->dim[l - 1]) * s);
+    if (l < L) acts += R(n[l] * pitch_of(m->dim[l]) * s);
+  }
+  acts += R(n[L] * pitch_of(m->dim[L]) * 4);
+  for (int l = L; l >= 1; --l) {
+    int64_t f = R(n[l] * pitch_of(m->dim[l]) * 4);
+    if (l >= 2) f += R(n[l - 1] * pitch_of(m->dim[l - 1]) * 4);
+    f += bwd_scratch_bytes(n[l], n[l - 1], l, m->dim[l - 1], m->dim[l]);
+    bwd = std::max(bwd, f);
+  }
+  *lo = blocks + acts + bwd;
+  *hi = blocks + acts + std::max(bwd, build);
+}
+
+static buffalo_status validate_model(const buffalo_model* m) {
+  if (!m || m->num_layers < 1 || m->num_layers > BUFFALO_MAX_LAYERS) {
+    set_error("model: num_layers must be in [1, %d]", BUFFALO_MAX_LAYERS);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  for (int l = 0; l <= m->num_layers; ++l)
+    if (m->dim[l] < 1 || m->dim[l] > BUFFALO_MAX_DIM) {
+      set_error("model: dim[%d] = %d out of range", l, m->dim[l]);
+      return BUFFALO_ERR_INVALID_ARG;
+    }
+  if (m->feat_dtype != BUFFALO_FP32 && m->feat_dtype != BUFFALO_BF16) return BUFFALO_ERR_INVALID_ARG;
+  if (m->gemm_mode != BUFFALO_GEMM_FFMA && m->gemm_mode != BUFFALO_GEMM_BF16) return BUFFALO_ERR_INVALID_ARG;
+  if (m->feat_pitch < round_up(m->dim[0], 8) || m->feat_pitch % 8) {
+    set_error("model: feat_pitch must be a multiple of 8 and >= round_up(dim[0], 8)");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  return BUFFALO_OK;
+}
+
+static buffalo_status validate_sampler(const buffalo_sampler* s, int L) {
+  if (!s || s->num_layers != L) {
+    set_error("sampler.num_layers must equal model.num_layers");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  for (int l = 0; l < L; ++l)
+    if (s->fanout[l] > BUFFALO_MAX_FANOUT) {
+      set_error("fanout %d > %d not supported", s->fanout[l], BUFFALO_MAX_FANOUT);
+      return BUFFALO_ERR_UNSUPPORTED;
+    }
+  if (s->cutoff_F < 0 || s->cutoff_F > 254) {
+    set_error("cutoff_F must be in [0, 254]");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  return BUFFALO_OK;
+}
+
+// ------------------------------------------------------------------ scheduler (Alg. 3/4)
+struct Item {
+  int d, k;                  // bucket degree, micro-bucket index
+  int64_t start, count;      // slice of the bucket-sorted seeds
+  int64_t O, E, I, M, w;
+};
+
+// Item statistics (R13): build the item's blocks alone (sizes only) on the GPU.
+static buffalo_status item_stats(const buffalo_graph* g, const int32_t* ids, int64_t count,
+                                 const buffalo_sampler* sp, const buffalo_model* m, char* ws,
+                                 int64_t ws_bytes, Item* it, cudaStream_t s) {
+  const int L = m->num_layers;
+  Arena A;
+  A.base = ws;
+  A.cap = ws_bytes;
+  int64_t n[BUFFALO_MAX_LAYERS + 1], e[BUFFALO_MAX_LAYERS];
+  const int32_t* dst = ids;
+  int64_t nd = count;
+  for (int l = L; l >= 1; --l) {
+    buffalo_block b;
+    buffalo_status st = build_layer(g, dst, nd, sp->fanout[l - 1], (uint32_t)(L - l + 1), sp->seed, l,
+                                    true, A, &b, s);
+    if (st == BUFFALO_ERR_CAPACITY || A.overflow) {
+      set_error("bucketize workspace too small (need > %lld bytes)", (long long)A.need);
+      return BUFFALO_ERR_CAPACITY;
+    }
+    BF_CHECK(st);
+    n[l] = nd;
+    e[l - 1] = b.n_edges;
+    dst = b.src_global;
+    nd = b.n_src;
+  }
+  n[0] = nd;
+  int64_t lo, hi;
+  mem_model(L, n, e, m, &lo, &hi);
+  it->O = count;
+  it->E = e[L - 1];
+  it->I = n[L - 1];
+  it->M = hi;
+  return BUFFALO_OK;
+}
+
+// Eq. 1-2, integer form (R14): floor(M * min(1, I*10^6 / (E*C_ppm))).
+static int64_t grouping_weight(int64_t M, int64_t I, int64_t E, int64_t C_ppm) {
+  if (E == 0 || C_ppm <= 0) return M;
+  unsigned __int128 num = (unsigned __int128)M * (unsigned __int128)I * 1000000u;
+  unsigned __int128 den = (unsigned __int128)E * (unsigned __int128)C_ppm;
+  unsigned __int128 q = num / den;
+  return q < (unsigned __int128)M ? (int64_t)q : M;
+}
+
+__global__ void k_scatter_segments(const int64_t* __restrict__ seg, const int32_t* __restrict__ order,
+                                   const int32_t* __restrict__ sorted_ids, int32_t* __restrict__ group_seeds,
+                                   int32_t* __restrict__ group_of_seed) {
+  const int64_t start = seg[4 * blockIdx.x], len = seg[4 * blockIdx.x + 1];
+  const int64_t grp = seg[4 * blockIdx.x + 2], off = seg[4 * blockIdx.x + 3];
+  for (int64_t t = threadIdx.x; t < len; t += blockDim.x) {
+    group_seeds[off + t] = sorted_ids[start + t];
+    group_of_seed[order[start + t]] = (int32_t)grp;
+  }
+}
+
+static int64_t stats_arena_bound(const buffalo_graph* g, int64_t n_seeds, const buffalo_sampler* sp, int L) {
+  int64_t nl = n_seeds, total = 0, frame = 0;
+  for (int l = L; l >= 1; --l) {
+    const int f = sp->fanout[l - 1];
+    int64_t el = f > 0 ? std::min<int64_t>(g->nnz, nl * f) : g->nnz;
+    int64_t nm = std::min<int64_t>(g->num_nodes, nl + el);
+    total += R(4 * (nl + 1)) + R(4 * nm);
+    frame = std::max(frame, build_frame_bytes(nl, el, l, true));
+    nl = nm;
+  }
+  return total + frame;
+}
+
+static int64_t bucketize_fixed_bytes(int64_t S, int F, int k_max) {
+  const int64_t pc = part_count_elems(S);
+  (void)F;
+  return R(S) + 2 * R(4 * S) + R(4 * (pc + 1)) + R(4 * scan_ws_elems(pc + 1)) + R(4 * 258) +
+         R(32 * (int64_t)(256 + k_max + 1));
+}
+
+}  // namespace buffalo
+
+using namespace buffalo;
+
+// ===================================================================== C ABI
+extern "C" {
+
+const char* buffalo_status_str(buffalo_status s) {
+  switch (s) {
+    case BUFFALO_OK: return "BUFFALO_OK";
+    case BUFFALO_ERR_INVALID_ARG: return "BUFFALO_ERR_INVALID_ARG";
+    case BUFFALO_ERR_BUDGET: return "BUFFALO_ERR_BUDGET";
+    case BUFFALO_ERR_CAPACITY: return "BUFFALO_ERR_CAPACITY";
+    case BUFFALO_ERR_CUDA: return "BUFFALO_ERR_CUDA";
+    case BUFFALO_ERR_UNSUPPORTED: return "BUFFALO_ERR_UNSUPPORTED";
+  }
+  return "BUFFALO_ERR_UNKNOWN";
+}
+
+const char* buffalo_last_error(void) { return g_err.c_str(); }
+int64_t buffalo_launch_count(void) { return g_launches.load(); }
+
+size_t buffalo_graph_workspace_bytes(int64_t num_nodes) { return (size_t)R(4 * (num_nodes > 0 ? num_nodes : 1)); }
+
+buffalo_status buffalo_graph_prepare(buffalo_graph* g, void* workspace, size_t bytes, void* stream) {
+  BF_CHECK(require_sm100());
+  if (!g || !workspace || !g->row_ptr || !g->col || g->num_nodes <= 0) return BUFFALO_ERR_INVALID_ARG;
+  if ((int64_t)bytes < (int64_t)buffalo_graph_workspace_bytes(g->num_nodes)) return BUFFALO_ERR_CAPACITY;
+  g->node_map = (int32_t*)workspace;
+  cudaStream_t s = (cudaStream_t)stream;
+  k_fill_i32<<<grid_for(g->num_nodes, 256), 256, 0, s>>>(g->node_map, g->num_nodes, INT32_MAX);
+  BF_LAUNCHED("k_fill_i32");
+  return BUFFALO_OK;
+}
+
+buffalo_status buffalo_estimate_mem(int32_t num_layers, const int64_t* n, const int64_t* e,
+                                    const buffalo_model* m, int64_t* lo_bytes_h, int64_t* hi_bytes_h) {
+  if (!n || !e || !m || !lo_bytes_h || !hi_bytes_h || num_layers != m->num_layers) return BUFFALO_ERR_INVALID_ARG;
+  BF_CHECK(validate_model(m));
+  mem_model(num_layers, n, e, m, lo_bytes_h, hi_bytes_h);
+  return BUFFALO_OK;
+}
+
+size_t buffalo_bucketize_workspace_bytes(const buffalo_graph* g, int64_t n_seeds,
+                                         const buffalo_sampler* s, const buffalo_model* m) {
+  if (!g || !s || !m) return 0;
+  return (size_t)(bucketize_fixed_bytes(n_seeds, s->cutoff_F, 4096) +
+                  stats_arena_bound(g, n_seeds, s, m->num_layers));
+}
+
+buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, int64_t S,
+                                 const buffalo_sampler* sp, const buffalo_model* m,
+                                 const buffalo_sched* sc, buffalo_plan* plan, void* workspace,
+                                 size_t workspace_bytes, void* stream) {
+  BF_CHECK(require_sm100());
+  BF_CHECK(validate_model(m));
+  const int L = m->num_layers;
+  BF_CHECK(validate_sampler(sp, L));
+  if (!g || !g->node_map || !seeds || S <= 0 || !sc || !plan || !workspace) {
+    set_error("bucketize: null argument or empty seed set");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (sc->mem_budget <= 0 || sc->k_max < 1 || sc->k_max > 4096 || sc->num_gpus < 1) {
+    set_error("bucketize: bad scheduler parameters");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  const int F = sp->cutoff_F;
+  const int fL = sp->fanout[L - 1];
+  // carve the workspace
+  char* q = (char*)workspace;
+  const int64_t pc = part_count_elems(S);
+  uint8_t* bucket = (uint8_t*)q; q += R(S);
+  int32_t* order = (int32_t*)q; q += R(4 * S);
+  int32_t* sorted_ids = (int32_t*)q; q += R(4 * S);
+  int32_t* counts = (int32_t*)q; q += R(4 * (pc + 1));
+  int32_t* ws = (int32_t*)q; q += R(4 * scan_ws_elems(pc + 1));
+  int32_t* starts = (int32_t*)q; q += R(4 * 258);
+  int64_t* segs = (int64_t*)q; q += R(32 * (int64_t)(256 + 4096 + 1));
+  const int64_t used = q - (char*)workspace;
+  if (used > (int64_t)workspace_bytes) {
+    set_error("bucketize workspace too small");
+    return BUFFALO_ERR_CAPACITY;
+  }
+  char* stats_ws = q;
+  const int64_t stats_bytes = (int64_t)workspace_bytes - used;
+
+  // a1: DegreeBucketing (Alg. 3 l.1)
+  BF_CHECK(seed_bucketing(g, seeds, S, fL, F, bucket, order, sorted_ids, counts, ws, starts, plan->hist_h, s));
+  std::vector<int64_t> bstart(F + 2, 0);
+  for (int b = 0; b <= F; ++b) bstart[b + 1] = bstart[b] + plan->hist_h[b];
+
+  // a2: per-bucket statistics and estimates (K-independent)
+  std::vector<Item> bucket_item(F + 1);
+  std::vector<int> non_split;
+  int64_t sum_M_all = 0, sum_w = 0, max_w = 0;
+  for (int d = 0; d <= F; ++d) {
+    if (plan->hist_h[d] == 0) continue;
+    Item it{d, 0, bstart[d], plan->hist_h[d], 0, 0, 0, 0, 0};
+    BF_CHECK(item_stats(g, sorted_ids + it.start, it.count, sp, m, stats_ws, stats_bytes, &it, s));
+    it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
+    bucket_item[d] = it;
+    sum_M_all += it.M;
+    if (d != F) {
+      non_split.push_back(d);
+      sum_w += it.w;
+      max_w = std::max(max_w, it.w);
+    }
+  }
+  const bool hasF = plan->hist_h[F] > 0;
+
+  // a3: the K loop (Alg. 3) with MemBalancedGrouping (Alg. 4)
+  const int k_lo = std::max(std::max(sc->k_min, sc->num_gpus), 1);
+  for (int K = k_lo; K <= sc->k_max; ++K) {
+    if (max_w > sc->mem_budget) break;                         // R25: fails for every K
+    if ((__int128)sum_w > (__int128)K * sc->mem_budget) continue;  // R25: some group exceeds M_ctr
+    std::vector<Item> items;
+    for (int d : non_split) items.push_back(bucket_item[d]);
+    bool exploded = false;
+    if (hasF) {
+      const Item& itF = bucket_item[F];
+      exploded = K >= 2 && (__int128)itF.M * K > (__int128)sum_M_all;   // R7
+      if (exploded) {
+        // SplitExplosionBucket: K contiguous pieces, the first (O mod K) one seed larger (R8)
+        const int64_t O = itF.count, base = O / K, extra = O % K;
+        int64_t st0 = itF.start;
+        for (int k = 0; k < K; ++k) {
+          const int64_t len = base + (k < extra ? 1 : 0);
+          if (len > 0) {
+            Item it{F, k, st0, len, 0, 0, 0, 0, 0};
+            BF_CHECK(item_stats(g, sorted_ids + st0, len, sp, m, stats_ws, stats_bytes, &it, s));
+            it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
+            items.push_back(it);
+          }
+          st0 += len;
+        }
+      } else {
+        items.push_back(itF);
+      }
+    }
+    // Alg. 4: sort by M_est descending (ties: degree asc, micro index asc), place each item
+    // into the group with the lowest Eq. 2 estimate (ties: lowest index).
+    std::vector<int> idx(items.size());
+    for (size_t i = 0; i < idx.size(); ++i) idx[i] = (int)i;
+    std::sort(idx.begin(), idx.end(), [&](int a, int b) {
+      if (items[a].M != items[b].M) return items[a].M > items[b].M;
+      if (items[a].d != items[b].d) return items[a].d < items[b].d;
+      return items[a].k < items[b].k;
+    });
+    std::vector<int64_t> load(K, 0);
+    std::vector<std::vector<int>> members(K);
+    for (int i : idx) {
+      int best = 0;
+      for (int k = 1; k < K; ++k)
+        if (load[k] < load[best]) best = k;
+      members[best].push_back(i);
+      load[best] += items[i].w;
+    }
+    int64_t mx = 0;
+    for (int k = 0; k < K; ++k) mx = std::max(mx, load[k]);
+    if (mx > sc->mem_budget) continue;
+
+    // success: emit the plan (empty groups dropped, R17)
+    std::vector<int64_t> seg;
+    std::vector<int64_t> offs(1, 0), est;
+    int gk = 0;
+    for (int k = 0; k < K; ++k) {
+      if (members[k].empty()) continue;
+      std::vector<int> mem = members[k];
+      std::sort(mem.begin(), mem.end(), [&](int a, int b) {
+        if (items[a].d != items[b].d) return items[a].d < items[b].d;
+        return items[a].k < items[b].k;
+      });
+      int64_t off = offs.back();
+      for (int i : mem) {
+        seg.push_back(items[i].start);
+        seg.push_back(items[i].count);
+        seg.push_back(gk);
+        seg.push_back(off);
+        off += items[i].count;
+      }
+      offs.push_back(off);
+      est.push_back(load[k]);
+      ++gk;
+    }
+    const int nseg = (int)(seg.size() / 4);
+    BF_CUDA(cudaMemcpyAsync(segs, seg.data(), seg.size() * sizeof(int64_t), cudaMemcpyHostToDevice, s));
+    k_scatter_segments<<<nseg, 256, 0, s>>>(segs, order, sorted_ids, plan->group_seeds, plan->group_of_seed);
+    BF_LAUNCHED("k_scatter_segments");
+    BF_CUDA(cudaMemcpyAsync(plan->group_offsets, offs.data(), offs.size() * sizeof(int64_t),
+                            cudaMemcpyHostToDevice, s));
+    for (int k = 0; k <= gk; ++k) plan->group_offsets_h[k] = offs[k];
+    // LPT assignment of groups to ranks (R24)
+    std::vector<int> gi(gk);
+    for (int k = 0; k < gk; ++k) gi[k] = k;
+    std::sort(gi.begin(), gi.end(), [&](int a, int b) { return est[a] != est[b] ? est[a] > est[b] : a < b; });
+    std::vector<int64_t> rload(sc->num_gpus, 0);
+    for (int k : gi) {
+      int best = 0;
+      for (int r = 1; r < sc->num_gpus; ++r)
+        if (rload[r] < rload[best]) best = r;
+      plan->rank_of_group_h[k] = best;
+      rload[best] += est[k];
+    }
+    for (int k = 0; k < gk; ++k) plan->est_bytes_h[k] = est[k];
+    plan->k_out = gk;
+    plan->k_tried = K;
+    plan->exploded = exploded ? 1 : 0;
+    plan->num_items = (int)items.size();
+    BF_CUDA(cudaStreamSynchronize(s));
+    return BUFFALO_OK;
+  }
+  set_error("Buffalo scheduler: no K in [%d, %d] satisfies M_ctr = %lld", k_lo, sc->k_max,
+            (long long)sc->mem_budget);
+  return BUFFALO_ERR_BUDGET;
+}
+
+buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group_seeds, int64_t n,
+                                    const buffalo_sampler* sp, const buffalo_model* m,
+                                    buffalo_blocks* out, void* arena, size_t arena_bytes,
+                                    int64_t* required_bytes_h, void* stream) {
+  BF_CHECK(require_sm100());
+  BF_CHECK(validate_model(m));
+  const int L = m->num_layers;
+  BF_CHECK(validate_sampler(sp, L));
+  if (!g || !g->node_map || !group_seeds || n <= 0 || !out || !arena) {
+    set_error("build_blocks: null argument or empty group");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (((uintptr_t)arena) % 256) {
+    set_error("build_blocks: arena must be 256-B aligned");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  memset(out, 0, sizeof(*out));
+  out->num_layers = L;
+  Arena A;
+  A.base = (char*)arena;
+  A.cap = (int64_t)arena_bytes;
+  const int32_t* dst = group_seeds;
+  int64_t nd = n;
+  int64_t nn[BUFFALO_MAX_LAYERS + 1], ee[BUFFALO_MAX_LAYERS];
+  for (int l = L; l >= 1; --l) {
+    buffalo_block* b = &out->layer[l - 1];
+    buffalo_status st = build_layer(g, dst, nd, sp->fanout[l - 1], (uint32_t)(L - l + 1), sp->seed, l,
+                                    false, A, b, s);
+    if (st == BUFFALO_ERR_CAPACITY || A.overflow) {
+      if (required_bytes_h) *required_bytes_h = A.need;
+      set_error("build_blocks: arena of %lld bytes too small (need >= %lld)", (long long)A.cap,
+                (long long)A.need);
+      cudaStreamSynchronize(s);
+      return BUFFALO_ERR_CAPACITY;
+    }
+    BF_CHECK(st);
+    nn[l] = nd;
+    ee[l - 1] = b->n_edges;
+    dst = b->src_global;
+    nd = b->n_src;
+  }
+  nn[0] = nd;
+  // activations (R20): saved h_agg per layer, H_l (l < L), logits
+  const int64_t sa = m->gemm_mode == BUFFALO_GEMM_BF16 ? 2 : 4;
+  for (int l = 1; l <= L; ++l) {
+    buffalo_block* b = &out->layer[l - 1];
+    b->ld_agg = pitch_of(m->dim[l - 1]);
+    b->agg = A.take(b->n_dst * b->ld_agg * sa);
+    b->ld_out = pitch_of(m->dim[l]);
+    b->out = A.take(b->n_dst * b->ld_out * (l < L ? sa : 4));
+  }
+  // backward region: ping-pong dH buffers at the two ends, scratch in between
+  int64_t B = 0;
+  std::vector<int64_t> ah(L + 1, 0), tmp(L + 1, 0);
+  for (int l = 1; l <= L; ++l) ah[l] = R(nn[l] * pitch_of(m->dim[l]) * 4);
+  for (int l = L; l >= 1; --l) {
+    tmp[l] = bwd_scratch_bytes(nn[l], nn[l - 1], l, m->dim[l - 1], m->dim[l]);
+    B = std::max(B, ah[l] + (l >= 2 ? ah[l - 1] : 0) + tmp[l]);
+  }
+  char* region = (char*)A.take(B);
+  if (A.overflow) {
+    if (required_bytes_h) *required_bytes_h = A.need;
+    set_error("build_blocks: arena of %lld bytes too small (need %lld)", (long long)A.cap, (long long)A.need);
+    return BUFFALO_ERR_CAPACITY;
+  }
+  for (int l = L; l >= 1; --l) {
+    buffalo_block* b = &out->layer[l - 1];
+    const bool low = ((L - l) % 2) == 0;        // dH_L at the low end, dH_{L-1} at the high end, ...
+    b->dh = (float*)(low ? region : region + B - ah[l]);
+    b->ld_dh = pitch_of(m->dim[l]);
+    b->bwd_scratch = low ? region + ah[l] : region + (l >= 2 ? ah[l - 1] : 0);
+    b->bwd_scratch_bytes = tmp[l];
+  }
+  out->arena_used = A.bottom;
+  out->arena_peak = A.peak;
+  mem_model(L, nn, ee, m, &out->est_lo, &out->est_hi);
+  if (required_bytes_h) *required_bytes_h = A.peak;
+  return BUFFALO_OK;
+}
+
+size_t buffalo_packed_weight_bytes(const buffalo_model* m, int32_t layer) {
+  if (!m || layer < 1 || layer > m->num_layers) return 0;
+  const int64_t din = m->dim[layer - 1], dout = m->dim[layer];
+  int64_t b = R(2 * din * dout * 4);
+  if (m->gemm_mode == BUFFALO_GEMM_BF16) b += tc_packed_bytes(din, dout);
+  return (size_t)b;
+}
+
+buffalo_status buffalo_pack_weights(const buffalo_model* m, int32_t layer, const float* W, void* packed,
+                                    void* stream) {
+  BF_CHECK(require_sm100());
+  BF_CHECK(validate_model(m));
+  if (layer < 1 || layer > m->num_layers || !W || !packed) return BUFFALO_ERR_INVALID_ARG;
+  cudaStream_t s = (cudaStream_t)stream;
+  const int din = m->dim[layer - 1], dout = m->dim[layer];
+  BF_CHECK(launch_transpose_w(W, dout, 2 * din, (float*)packed, s));
+  if (m->gemm_mode == BUFFALO_GEMM_BF16)
+    BF_CHECK(tc_pack_weights(W, din, dout, (char*)packed + R((int64_t)2 * din * dout * 4), s));
+  return BUFFALO_OK;
+}
+
+buffalo_status buffalo_sage_fwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                const void* h_src, int64_t ld_src, const float* W, const void* W_packed,
+                                const float* b, void* out, int64_t ld_out, void* saved_agg,
+                                int64_t ld_agg, void* stream) {
+  BF_CHECK(require_sm100());
+  BF_CHECK(validate_model(m));
+  if (!blk || layer < 1 || layer > m->num_layers || !h_src || !W || !W_packed || !out || !saved_agg) {
+    set_error("sage_fwd: null argument or bad layer");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  FwdArgs a{};
+  a.blk = blk;
+  a.layer1 = layer == 1;
+  const bool act_bf16 = m->gemm_mode == BUFFALO_GEMM_BF16;
+  a.in_bf16 = a.layer1 ? m->feat_dtype == BUFFALO_BF16 : act_bf16;
+  a.act_bf16 = act_bf16;
+  a.out_f32 = layer == m->num_layers;
+  a.relu = layer < m->num_layers;
+  a.d_in = m->dim[layer - 1];
+  a.d_out = m->dim[layer];
+  a.h_src = h_src;
+  a.ld_src = a.layer1 ? m->feat_pitch : ld_src;
+  a.W = W;
+  a.W_packed = W_packed;
+  a.b = b;
+  a.out = out;
+  a.ld_out = ld_out;
+  a.agg = saved_agg;
+  a.ld_agg = ld_agg;
+  if (a.layer1 && !blk->col_global) return BUFFALO_ERR_INVALID_ARG;
+  if (ld_out < pitch_of(a.d_out) || ld_agg < pitch_of(a.d_in) || a.ld_src < pitch_of(a.d_in) ||
+      ld_out % 8 || ld_agg % 8 || a.ld_src % 8) {
+    set_error("sage_fwd: leading dimensions must be multiples of 8 and >= the padded widths");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  if (m->gemm_mode == BUFFALO_GEMM_BF16 && tc_fwd_supported(a)) return tc_sage_fwd(a, s);
+  return sage_fwd_ffma(a, s);
+}
+
+size_t buffalo_sage_bwd_scratch_bytes(const buffalo_block* blk, int32_t layer, const buffalo_model* m) {
+  if (!blk || !m || layer < 1 || layer > m->num_layers) return 0;
+  return (size_t)bwd_scratch_bytes(blk->n_dst, blk->n_src, layer, m->dim[layer - 1], m->dim[layer]);
+}
+
+buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
+                                const void* saved_agg, int64_t ld_agg, const void* h_dst,
+                                int64_t ld_hdst, const float* W, const void* W_packed, float* dW_accum,
+                                float* db_accum, float* dh_src, int64_t ld_dh_src, void* scratch,
+                                size_t scratch_bytes, void* stream) {
+  BF_CHECK(require_sm100());
+  BF_CHECK(validate_model(m));
+  if (!blk || layer < 1 || layer > m->num_layers || !dh_dst || !h_src || !saved_agg || !W ||
+      !dW_accum || !db_accum || !scratch) {
+    set_error("sage_bwd: null argument or bad layer");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (layer < m->num_layers && !h_dst) return BUFFALO_ERR_INVALID_ARG;
+  if (dh_src && (layer == 1 || !blk->t_row_ptr)) {
+    set_error("sage_bwd: dh_src needs a transposed block (layer >= 2)");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if ((int64_t)scratch_bytes < (int64_t)buffalo_sage_bwd_scratch_bytes(blk, layer, m)) return BUFFALO_ERR_CAPACITY;
+  BwdArgs a{};
+  a.blk = blk;
+  a.layer1 = layer == 1;
+  const bool act_bf16 = m->gemm_mode == BUFFALO_GEMM_BF16;
+  a.in_bf16 = a.layer1 ? m->feat_dtype == BUFFALO_BF16 : act_bf16;
+  a.act_bf16 = act_bf16;
+  a.last = layer == m->num_layers;
+  a.d_in = m->dim[layer - 1];
+  a.d_out = m->dim[layer];
+  a.dh = dh_dst;
+  a.ld_dh = ld_dh;
+  a.h_src = h_src;
+  a.ld_src = a.layer1 ? m->feat_pitch : ld_src;
+  a.agg = saved_agg;
+  a.ld_agg = ld_agg;
+  a.h_dst = h_dst;
+  a.ld_hdst = ld_hdst;
+  a.W = W;
+  a.W_packed = W_packed;
+  a.dW = dW_accum;
+  a.db = db_accum;
+  a.dh_src = dh_src;
+  a.ld_dh_src = ld_dh_src;
+  a.scratch = scratch;
+  a.scratch_bytes = (int64_t)scratch_bytes;
+  cudaStream_t s = (cudaStream_t)stream;
+  return sage_bwd_ffma(a, s);
+}
+
+buffalo_status buffalo_softmax_ce(const float* logits, int64_t ld, int64_t n, int32_t classes,
+                                  const int32_t* labels, const int32_t* row_ids, int64_t batch_size,
+                                  float* loss_accum, float* dlogits, int64_t ld_d, void* stream) {
+  BF_CHECK(require_sm100());
+  if (!logits || !labels || !row_ids || !loss_accum || !dlogits || batch_size <= 0 || classes < 1 ||
+      ld < classes || ld_d < classes)
+    return BUFFALO_ERR_INVALID_ARG;
+  return launch_softmax_ce(logits, ld, n, classes, labels, row_ids, batch_size, loss_accum, dlogits, ld_d,
+                           (cudaStream_t)stream);
+}
+
+buffalo_status buffalo_sgd_step(float* param, float* grad, int64_t n, float lr, void* stream) {
+  BF_CHECK(require_sm100());
+  if (!param || !grad || n < 0) return BUFFALO_ERR_INVALID_ARG;
+  return launch_sgd(param, grad, n, lr, (cudaStream_t)stream);
+}
+
+}  // extern "C"

@@ -1,0 +1,382 @@
+// build.cu — block generation and seed degree bucketing (a1).
+//
+// BlockGenerate / MicroBatchGenerator (Alg. 2 l.5; §IV-E):
+// for every dst row of the layer, in parallel at the node level ("tracking neighbors happens
+// in parallel at the node level"): count -> scan -> sample/slice -> relabel into
+// a bipartite block (dst prefix + first occurrence, R3/R4) -> transpose for the backward.
+#include "build.cuh"
+#include "philox.cuh"
+#include "primitives.cuh"
+
+namespace buffalo {
+
+// ------------------------------------------------------------------ scan tile pass
+__global__ void __launch_bounds__(1024) k_scan_tiles(int32_t* ts, int64_t ntiles, int32_t* total_out) {
+  __shared__ int32_t sw[33];
+  int32_t carry = 0;
+  for (int64_t b = 0; b < ntiles; b += 1024) {
+    int64_t i = b + threadIdx.x;
+    int32_t v = i < ntiles ? ts[i] : 0;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    int32_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      int32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) sw[warp] = x;
+    __syncthreads();
+    if (warp == 0) {
+      int32_t w = sw[lane];
+      int32_t s = w;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        int32_t y = __shfl_up_sync(0xffffffffu, s, o);
+        if (lane >= o) s += y;
+      }
+      sw[lane] = s - w;
+      if (lane == 31) sw[32] = s;
+    }
+    __syncthreads();
+    if (i < ntiles) ts[i] = carry + sw[warp] + x - v;
+    carry += sw[32];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *total_out = carry;
+}
+
+// ------------------------------------------------------------------ a4: count D per dst
+__global__ void k_count(const int32_t* __restrict__ dst, int64_t n, const int64_t* __restrict__ grow,
+                        int32_t f, int32_t* __restrict__ counts) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t v = dst[i];
+    int64_t deg = grow[v + 1] - grow[v];
+    counts[i] = (int32_t)((f > 0 && deg > f) ? f : deg);
+  }
+}
+
+// ------------------------------------------------------------------ a4: sample / slice
+// Warp per dst.  deg <= f or f <= 0: the warp copies the CSR row (coalesced).  Otherwise
+// Floyd's algorithm (R2): lane t computes r_t = floor(x_t (j_t + 1) / 2^32), j_t = deg - f + t;
+// the sequential membership test runs as f ballot steps; the chosen positions are then
+// ranked (sorted ascending) inside the warp and the neighbours gathered.
+__global__ void __launch_bounds__(256) k_sample_fill(const int32_t* __restrict__ dst, int64_t n,
+                                                     const int64_t* __restrict__ grow,
+                                                     const int32_t* __restrict__ gcol, int32_t f,
+                                                     uint32_t hop, uint64_t seed,
+                                                     const int32_t* __restrict__ row_ptr,
+                                                     int32_t* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n; i += warps) {
+    const uint32_t v = (uint32_t)dst[i];
+    const int64_t beg = grow[v];
+    const int64_t deg = grow[v + 1] - beg;
+    int32_t* o = out + row_ptr[i];
+    if (f <= 0 || deg <= f) {
+      for (int64_t k = lane; k < deg; k += 32) o[k] = gcol[beg + k];
+      continue;
+    }
+    const uint32_t j = (uint32_t)(deg - f) + (uint32_t)lane;
+    uint32_t r = 0;
+    if (lane < f) r = __umulhi(sample_draw(seed, v, hop, (uint32_t)lane), j + 1u);
+    int32_t S = -1;
+    for (int t = 0; t < f; ++t) {
+      const int32_t cand = (int32_t)__shfl_sync(0xffffffffu, r, t);
+      const unsigned present = __ballot_sync(0xffffffffu, lane < t && S == cand);
+      if (lane == t) S = present ? (int32_t)((uint32_t)(deg - f) + (uint32_t)t) : cand;
+    }
+    int rank = 0;
+    for (int u = 0; u < f; ++u) {
+      const int32_t su = __shfl_sync(0xffffffffu, S, u);
+      rank += (su < S) ? 1 : 0;
+    }
+    if (lane < f) o[rank] = gcol[beg + S];
+  }
+}
+
+// ------------------------------------------------------------------ a5: relabel
+// Candidate position p: p < n_dst -> dst[p], else col_global[p - n_dst].
+struct Cand {
+  const int32_t* dst;
+  const int32_t* colg;
+  int64_t n_dst;
+  __device__ __forceinline__ int32_t operator()(int64_t p) const {
+    return p < n_dst ? dst[p] : colg[p - n_dst];
+  }
+};
+
+__global__ void k_relabel_min(Cand c, int64_t total, int32_t* __restrict__ node_map) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < total;
+       p += (int64_t)gridDim.x * blockDim.x)
+    atomicMin(&node_map[c(p)], (int32_t)p);
+}
+
+struct FirstFlag {
+  Cand c;
+  const int32_t* node_map;
+  __device__ __forceinline__ int32_t operator()(int64_t p) const {
+    return node_map[c(p)] == (int32_t)p ? 1 : 0;
+  }
+};
+struct EmitSrc {
+  Cand c;
+  int32_t* src;
+  __device__ __forceinline__ void operator()(int64_t p, int32_t excl, int32_t v) const {
+    if (v) src[excl] = c(p);
+  }
+};
+
+__global__ void k_set_map(const int32_t* __restrict__ src, int64_t n, int32_t* __restrict__ node_map) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
+    node_map[src[j]] = (int32_t)j;
+}
+__global__ void k_reset_map(const int32_t* __restrict__ src, int64_t n, int32_t* __restrict__ node_map) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
+    node_map[src[j]] = INT32_MAX;
+}
+__global__ void k_col_local(const int32_t* __restrict__ colg, int64_t e, const int32_t* __restrict__ node_map,
+                            int32_t* __restrict__ col_local) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x)
+    col_local[k] = node_map[colg[k]];
+}
+
+// ------------------------------------------------------------------ a6: heavy rows, transpose
+struct HeavyFlag {
+  const int32_t* rp;
+  __device__ __forceinline__ int32_t operator()(int64_t i) const {
+    return (rp[i + 1] - rp[i]) > kHeavyT ? 1 : 0;
+  }
+};
+struct EmitIndex {
+  int32_t* out;
+  __device__ __forceinline__ void operator()(int64_t i, int32_t excl, int32_t v) const {
+    if (v) out[excl] = (int32_t)i;
+  }
+};
+
+__global__ void k_fill_zero(int32_t* a, int64_t n) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
+    a[k] = 0;
+}
+__global__ void k_tcount(const int32_t* __restrict__ col_local, int64_t e, int32_t* __restrict__ cnt) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(&cnt[col_local[k]], 1);
+}
+// ed[e] = dst index of edge e (warp per dst row).
+__global__ void k_edge_dst(const int32_t* __restrict__ rp, int64_t n, int32_t* __restrict__ ed) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n; i += warps)
+    for (int32_t k = rp[i] + lane; k < rp[i + 1]; k += 32) ed[k] = (int32_t)i;
+}
+
+struct RadixKey {
+  const int32_t* keys;
+  int shift;
+  __device__ __forceinline__ int operator()(int64_t i) const { return (keys[i] >> shift) & 255; }
+};
+struct RadixEmit {
+  const int32_t* kin;
+  const int32_t* pin;
+  int32_t* kout;
+  int32_t* pout;
+  __device__ __forceinline__ void operator()(int64_t i, int32_t pos) const {
+    kout[pos] = kin[i];
+    pout[pos] = pin[i];
+  }
+};
+
+// ------------------------------------------------------------------ host side
+static buffalo_status d2h_i32(const int32_t* d, int32_t* h, cudaStream_t s) {
+  BF_CUDA(cudaMemcpyAsync(h, d, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  return BUFFALO_OK;
+}
+
+int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only) {
+  int64_t pc = part_count_elems(e);
+  int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pc + 1);
+  int64_t fr = R(64) + R(4 * scan_ws_elems(scan_len));
+  if (sizes_only) return fr + R(4 * e);
+  if (layer >= 2) fr += 6 * R(4 * e) + R(4 * (pc + 1));
+  return fr;
+}
+
+buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
+                           uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
+                           buffalo_block* blk, cudaStream_t s) {
+  memset(blk, 0, sizeof(*blk));
+  blk->n_dst = n_dst;
+  int32_t* rp = (int32_t*)A.take(4 * (n_dst + 1));
+  int32_t* heavy = sizes_only ? nullptr : (int32_t*)A.take(4 * n_dst);
+  // frame 1: totals + scan workspace for the count scan and the heavy compaction
+  char* fr = A.push_frame(R(64) + R(4 * scan_ws_elems(n_dst + 1)));
+  if (A.overflow) return BUFFALO_ERR_CAPACITY;
+  int32_t* totals = (int32_t*)fr;
+  int32_t* ws = (int32_t*)(fr + R(64));
+  if (n_dst > 0) {
+    k_count<<<grid_for(n_dst, 256), 256, 0, s>>>(dst, n_dst, g->row_ptr, f, rp);
+    BF_LAUNCHED("k_count");
+  }
+  BF_CHECK(scan_inplace(rp, n_dst, ws, s));
+  int32_t e32 = 0, nh = 0;
+  if (!sizes_only) {
+    BF_CHECK(device_scan(HeavyFlag{rp}, EmitIndex{heavy}, n_dst, ws, totals, s));
+    BF_CHECK(d2h_i32(totals, &nh, s));
+  }
+  BF_CHECK(d2h_i32(rp + n_dst, &e32, s));
+  BF_CUDA(cudaStreamSynchronize(s));                               // sync 1: e_l, n_heavy
+  const int64_t e = e32;
+  blk->n_edges = e;
+  blk->n_heavy = nh;
+  blk->row_ptr = rp;
+  blk->heavy = heavy;
+
+  // frame 2
+  const int64_t pc = part_count_elems(e);
+  const int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pc + 1);
+  int32_t* col_local = (!sizes_only) ? (int32_t*)A.take(4 * e) : nullptr;
+  int32_t* colg_persist = (!sizes_only && layer == 1) ? (int32_t*)A.take(4 * e) : nullptr;
+  fr = A.push_frame(build_frame_bytes(n_dst, e, layer, sizes_only));
+  if (A.overflow) return BUFFALO_ERR_CAPACITY;
+  totals = (int32_t*)fr;
+  char* q = fr + R(64);
+  ws = (int32_t*)q; q += R(4 * scan_ws_elems(scan_len));
+  int32_t* colg = colg_persist;
+  if (!colg) { colg = (int32_t*)q; q += R(4 * e); }
+  if (n_dst > 0) {
+    k_sample_fill<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(dst, n_dst, g->row_ptr, g->col, f, hop,
+                                                               seed, rp, colg);
+    BF_LAUNCHED("k_sample_fill");
+  }
+  // relabel: first occurrence over the candidate sequence dst ++ col_global
+  Cand cand{dst, colg, n_dst};
+  const int64_t total = n_dst + e;
+  if (total > 0) {
+    k_relabel_min<<<grid_for(total, 256), 256, 0, s>>>(cand, total, g->node_map);
+    BF_LAUNCHED("k_relabel_min");
+  }
+  FirstFlag ff{cand, g->node_map};
+  const int64_t ntiles = ceil_div(total > 0 ? total : 1, kScanTile);
+  k_scan_reduce<<<(unsigned)ntiles, kScanThreads, 0, s>>>(ff, total, ws);
+  BF_LAUNCHED("k_scan_reduce");
+  k_scan_tiles<<<1, 1024, 0, s>>>(ws, ntiles, totals);
+  BF_LAUNCHED("k_scan_tiles");
+  int32_t ns32 = 0;
+  BF_CHECK(d2h_i32(totals, &ns32, s));
+  BF_CUDA(cudaStreamSynchronize(s));                               // sync 2: n_{l-1}
+  const int64_t n_src = ns32;
+  int32_t* src = (int32_t*)A.take(4 * n_src);
+  if (A.overflow) return BUFFALO_ERR_CAPACITY;
+  k_scan_apply<<<(unsigned)ntiles, kScanThreads, 0, s>>>(ff, EmitSrc{cand, src}, total, ws);
+  BF_LAUNCHED("k_scan_apply");
+  blk->n_src = n_src;
+  blk->src_global = src;
+  blk->col_global = colg_persist;
+  if (!sizes_only) {
+    if (n_src > 0) {
+      k_set_map<<<grid_for(n_src, 256), 256, 0, s>>>(src, n_src, g->node_map);
+      BF_LAUNCHED("k_set_map");
+    }
+    if (e > 0) {
+      k_col_local<<<grid_for(e, 256), 256, 0, s>>>(colg, e, g->node_map, col_local);
+      BF_LAUNCHED("k_col_local");
+    }
+    blk->col_local = col_local;
+  }
+  if (n_src > 0) {
+    k_reset_map<<<grid_for(n_src, 256), 256, 0, s>>>(src, n_src, g->node_map);
+    BF_LAUNCHED("k_reset_map");
+  }
+  if (!sizes_only && layer >= 2) {
+    // transposed block: t_row_ptr by counting, t_col by a stable LSD radix sort of the edges
+    // (dst-ordered) keyed by col_local => each transposed row lists its dst ascending.
+    int32_t* trp = (int32_t*)A.take(4 * (n_src + 1));
+    int32_t* tcol = (int32_t*)A.take(4 * e);
+    if (A.overflow) return BUFFALO_ERR_CAPACITY;
+    int32_t* ed = (int32_t*)q; q += R(4 * e);
+    int32_t* bufk[2] = {(int32_t*)q, (int32_t*)(q + R(4 * e))}; q += 2 * R(4 * e);
+    int32_t* bufp[2] = {(int32_t*)q, (int32_t*)(q + R(4 * e))}; q += 2 * R(4 * e);
+    int32_t* counts = (int32_t*)q;
+    k_fill_zero<<<grid_for(n_src + 1, 256), 256, 0, s>>>(trp, n_src + 1);
+    BF_LAUNCHED("k_fill_zero");
+    if (e > 0) {
+      k_tcount<<<grid_for(e, 256), 256, 0, s>>>(col_local, e, trp);
+      BF_LAUNCHED("k_tcount");
+    }
+    BF_CHECK(scan_inplace(trp, n_src, ws, s));
+    if (e > 0) {
+      k_edge_dst<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(rp, n_dst, ed);
+      BF_LAUNCHED("k_edge_dst");
+      int bits = 1;
+      while ((1LL << bits) < n_src) ++bits;
+      const int passes = (bits + 7) / 8;
+      const int32_t* kin = col_local;
+      const int32_t* pin = ed;
+      for (int p = 0; p < passes; ++p) {
+        int32_t* kout = bufk[p & 1];
+        int32_t* pout = (p == passes - 1) ? tcol : bufp[p & 1];
+        BF_CHECK(stable_partition(RadixKey{kin, 8 * p}, RadixEmit{kin, pin, kout, pout}, e, counts, ws, s));
+        kin = kout;
+        pin = pout;
+      }
+    }
+    blk->t_row_ptr = trp;
+    blk->t_col = tcol;
+  }
+  A.pop_frame();
+  return BUFFALO_OK;
+}
+
+// ------------------------------------------------------------------ a1: seed bucketing
+__global__ void k_seed_bucket(const int32_t* __restrict__ seeds, int64_t n, const int64_t* __restrict__ grow,
+                              int32_t fL, int32_t F, uint8_t* __restrict__ bucket) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t v = seeds[i];
+    int64_t deg = grow[v + 1] - grow[v];
+    int64_t D = (fL > 0 && deg > fL) ? fL : deg;
+    bucket[i] = (uint8_t)(D < F ? D : F);
+  }
+}
+struct BucketKey {
+  const uint8_t* b;
+  __device__ __forceinline__ int operator()(int64_t i) const { return b[i]; }
+};
+struct BucketEmit {
+  const int32_t* seeds;
+  int32_t* order;
+  int32_t* sorted_ids;
+  __device__ __forceinline__ void operator()(int64_t i, int32_t pos) const {
+    order[pos] = (int32_t)i;
+    sorted_ids[pos] = seeds[i];
+  }
+};
+// starts[b] = exclusive offset of bin b (b = 0..nbins), read from the scanned partition counts.
+__global__ void k_bin_starts(const int32_t* counts, int64_t ntiles, int nbins, int32_t total, int32_t* starts) {
+  int b = threadIdx.x;
+  if (b < nbins) starts[b] = counts[(int64_t)b * ntiles];
+  if (b == nbins) starts[b] = total;
+}
+
+buffalo_status seed_bucketing(const buffalo_graph* g, const int32_t* seeds, int64_t n, int32_t fL,
+                              int32_t F, uint8_t* bucket, int32_t* order, int32_t* sorted_ids,
+                              int32_t* counts, int32_t* ws, int32_t* starts_dev, int64_t* hist_h,
+                              cudaStream_t s) {
+  if (n <= 0) {
+    for (int b = 0; b <= F; ++b) hist_h[b] = 0;
+    return BUFFALO_OK;
+  }
+  k_seed_bucket<<<grid_for(n, 256), 256, 0, s>>>(seeds, n, g->row_ptr, fL, F, bucket);
+  BF_LAUNCHED("k_seed_bucket");
+  BF_CHECK(stable_partition(BucketKey{bucket}, BucketEmit{seeds, order, sorted_ids}, n, counts, ws, s));
+  k_bin_starts<<<1, 256, 0, s>>>(counts, part_tiles(n), F + 1, (int32_t)n, starts_dev);
+  BF_LAUNCHED("k_bin_starts");
+  int32_t st[258];
+  BF_CUDA(cudaMemcpyAsync(st, starts_dev, sizeof(int32_t) * (F + 2), cudaMemcpyDeviceToHost, s));
+  BF_CUDA(cudaStreamSynchronize(s));
+  for (int b = 0; b <= F; ++b) hist_h[b] = st[b + 1] - st[b];
+  return BUFFALO_OK;
+}
+
+}  // namespace buffalo

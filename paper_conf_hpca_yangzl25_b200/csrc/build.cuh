@@ -1,0 +1,26 @@
+// build.cuh — internal interface of block generation and seed bucketing.
+#pragma once
+#include <algorithm>
+#include <cstring>
+
+#include "common.cuh"
+
+namespace buffalo {
+
+int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only);
+
+// Builds block `layer` (1-based) whose dst are dst[0..n_dst).  sizes_only: only row_ptr and
+// src_global are produced (scheduler statistics).  Allocates from A (bottom: persistent block
+// arrays; top frame: scratch).  Synchronises the stream twice.
+buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
+                           uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
+                           buffalo_block* blk, cudaStream_t s);
+
+// Degree bucketing of the seeds (Alg. 3 l.1): bucket[i] = min(D(seed_i), F); order = seed
+// positions grouped by bucket (stable); sorted_ids = seeds[order]; hist_h[0..F].
+buffalo_status seed_bucketing(const buffalo_graph* g, const int32_t* seeds, int64_t n, int32_t fL,
+                              int32_t F, uint8_t* bucket, int32_t* order, int32_t* sorted_ids,
+                              int32_t* counts, int32_t* ws, int32_t* starts_dev, int64_t* hist_h,
+                              cudaStream_t s);
+
+}  // namespace buffalo

@@ -1,0 +1,92 @@
+// common.cuh — shared helpers of libbuffalo (CUDA side only; nothing here is shared with oracle/).
+#pragma once
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <string>
+
+#include "../../include/buffalo.h"
+
+namespace buffalo {
+
+constexpr int64_t kAlign = 256;
+constexpr int kHeavyT = 128;          // rows with D > kHeavyT take the cooperative long-tail path
+constexpr int kScanTile = 16384;      // elements per scan tile (512 threads x 32)
+
+__host__ __device__ inline int64_t round_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+__host__ __device__ inline int64_t R(int64_t bytes) { return round_up(bytes, kAlign); }
+__host__ __device__ inline int64_t pitch_of(int64_t d) { return round_up(d, 8); }
+
+void set_error(const char* fmt, ...);
+void count_launch(int n = 1);
+
+// Returns BUFFALO_ERR_CUDA with the message if the last launch failed.
+buffalo_status check_cuda(const char* what);
+
+#define BF_CHECK(...)                                                \
+  do {                                                               \
+    buffalo_status _s = (__VA_ARGS__);                                      \
+    if (_s != BUFFALO_OK) return _s;                                 \
+  } while (0)
+
+#define BF_CUDA(...)                                                 \
+  do {                                                               \
+    cudaError_t _e = (__VA_ARGS__);                                  \
+    if (_e != cudaSuccess) {                                         \
+      buffalo::set_error("%s: %s", #__VA_ARGS__, cudaGetErrorString(_e)); \
+      return BUFFALO_ERR_CUDA;                                       \
+    }                                                                \
+  } while (0)
+
+#define BF_LAUNCHED(name)                                            \
+  do {                                                               \
+    buffalo::count_launch();                                         \
+    buffalo_status _s = buffalo::check_cuda(name);                   \
+    if (_s != BUFFALO_OK) return _s;                                 \
+  } while (0)
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Grid size for grid-stride kernels: a multiple of the 148 SMs, capped by the work.
+inline int grid_for(int64_t work_items, int per_block, int blocks_per_sm = 8) {
+  int64_t g = ceil_div(work_items > 0 ? work_items : 1, per_block);
+  int64_t cap = 148LL * blocks_per_sm;
+  return (int)(g < cap ? g : cap);
+}
+
+// sm_100a check (once per process).
+buffalo_status require_sm100();
+
+// Simple bump allocator over the caller's arena: bottom grows up (persistent), frames are
+// placed at the top (temporary).  Tracks the high-water mark bottom + frame.
+struct Arena {
+  char* base = nullptr;
+  int64_t cap = 0, bottom = 0, frame = 0, peak = 0;
+  bool overflow = false;
+  int64_t need = 0;
+  void* take(int64_t bytes) {
+    int64_t b = R(bytes);
+    void* p = base + bottom;
+    bottom += b;
+    touch();
+    return p;
+  }
+  // Reserve a temporary frame of `bytes` at the top; returns its base.
+  char* push_frame(int64_t bytes) {
+    frame = R(bytes);
+    touch();
+    return base + (cap - frame);
+  }
+  void pop_frame() { frame = 0; }
+  void touch() {
+    if (bottom + frame > peak) peak = bottom + frame;
+    if (bottom + frame > cap) { overflow = true; if (bottom + frame > need) need = bottom + frame; }
+  }
+};
+
+// ---------------------------------------------------------------- device helpers
+__device__ __forceinline__ float bf2f(__nv_bfloat16 v) { return __bfloat162float(v); }
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+}  // namespace buffalo

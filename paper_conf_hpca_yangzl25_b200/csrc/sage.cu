@@ -1,0 +1,569 @@
+// sage.cu — GraphSAGE-mean layer kernels, CUDA-core path.
+//
+// Aggregate (Alg. 2 l.8): warp per destination row, 16-byte vector loads of the
+// neighbour rows, fp32 accumulation in CSR order, one IEEE division by D (R21).  Rows with
+// D > kHeavyT (the long tail of full-neighbour blocks) go to a CTA-cooperative kernel whose
+// per-warp partial sums are combined in warp order (deterministic, depends only on D).
+// Update (Alg. 2 l.9): fp32 SIMT GEMM over [h_self || h_agg] (gemm_mode FFMA, the parity
+// path); the tensor-core path is in tc_sage.cu.
+#include "common.cuh"
+#include "sage.cuh"
+
+namespace buffalo {
+
+// ------------------------------------------------------------------ vector loads
+template <class T, int C> struct VecIO;
+template <> struct VecIO<float, 4> {
+  static __device__ __forceinline__ void load(const float* p, float* v) {
+    float4 a = __ldg(reinterpret_cast<const float4*>(p));
+    v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+  }
+  static __device__ __forceinline__ void store(float* p, const float* v) {
+    *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+  }
+};
+template <> struct VecIO<float, 8> {
+  static __device__ __forceinline__ void load(const float* p, float* v) {
+    VecIO<float, 4>::load(p, v);
+    VecIO<float, 4>::load(p + 4, v + 4);
+  }
+  static __device__ __forceinline__ void store(float* p, const float* v) {
+    VecIO<float, 4>::store(p, v);
+    VecIO<float, 4>::store(p + 4, v + 4);
+  }
+};
+__device__ __forceinline__ void unpack_bf2(uint32_t w, float& a, float& b) {
+  a = __uint_as_float(w << 16);
+  b = __uint_as_float(w & 0xffff0000u);
+}
+__device__ __forceinline__ uint32_t pack_bf2(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+template <> struct VecIO<__nv_bfloat16, 4> {
+  static __device__ __forceinline__ void load(const __nv_bfloat16* p, float* v) {
+    uint2 a = __ldg(reinterpret_cast<const uint2*>(p));
+    unpack_bf2(a.x, v[0], v[1]); unpack_bf2(a.y, v[2], v[3]);
+  }
+  static __device__ __forceinline__ void store(__nv_bfloat16* p, const float* v) {
+    *reinterpret_cast<uint2*>(p) = make_uint2(pack_bf2(v[0], v[1]), pack_bf2(v[2], v[3]));
+  }
+};
+template <> struct VecIO<__nv_bfloat16, 8> {
+  static __device__ __forceinline__ void load(const __nv_bfloat16* p, float* v) {
+    uint4 a = __ldg(reinterpret_cast<const uint4*>(p));
+    unpack_bf2(a.x, v[0], v[1]); unpack_bf2(a.y, v[2], v[3]);
+    unpack_bf2(a.z, v[4], v[5]); unpack_bf2(a.w, v[6], v[7]);
+  }
+  static __device__ __forceinline__ void store(__nv_bfloat16* p, const float* v) {
+    *reinterpret_cast<uint4*>(p) = make_uint4(pack_bf2(v[0], v[1]), pack_bf2(v[2], v[3]),
+                                              pack_bf2(v[4], v[5]), pack_bf2(v[6], v[7]));
+  }
+};
+
+template <class T> __device__ __forceinline__ float ld1(const T* p);
+template <> __device__ __forceinline__ float ld1<float>(const float* p) { return __ldg(p); }
+template <> __device__ __forceinline__ float ld1<__nv_bfloat16>(const __nv_bfloat16* p) {
+  return __bfloat162float(*p);
+}
+template <class T> __device__ __forceinline__ void st1(T* p, float v);
+template <> __device__ __forceinline__ void st1<float>(float* p, float v) { *p = v; }
+template <> __device__ __forceinline__ void st1<__nv_bfloat16>(__nv_bfloat16* p, float v) {
+  *p = __float2bfloat16_rn(v);
+}
+
+// ------------------------------------------------------------------ aggregate (regular rows)
+template <class TI, class TO, int C>
+__global__ void __launch_bounds__(256) k_agg_rows(const int32_t* __restrict__ rp,
+                                                  const int32_t* __restrict__ col, int64_t n,
+                                                  const TI* __restrict__ h, int64_t ldh, int d,
+                                                  TO* __restrict__ agg, int64_t lda) {
+  const int lane = threadIdx.x & 31;
+  const int nch = (d + C - 1) / C;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n; i += warps) {
+    const int32_t b = rp[i], e_end = rp[i + 1];
+    const int32_t D = e_end - b;
+    if (D > kHeavyT) continue;
+    for (int c = lane; c < nch; c += 32) {
+      float acc[C];
+#pragma unroll
+      for (int k = 0; k < C; ++k) acc[k] = 0.f;
+      int32_t e = b;
+      for (; e + 4 <= e_end; e += 4) {
+        const int64_t j0 = col[e], j1 = col[e + 1], j2 = col[e + 2], j3 = col[e + 3];
+        float v0[C], v1[C], v2[C], v3[C];
+        VecIO<TI, C>::load(h + j0 * ldh + c * C, v0);
+        VecIO<TI, C>::load(h + j1 * ldh + c * C, v1);
+        VecIO<TI, C>::load(h + j2 * ldh + c * C, v2);
+        VecIO<TI, C>::load(h + j3 * ldh + c * C, v3);
+#pragma unroll
+        for (int k = 0; k < C; ++k) { acc[k] += v0[k]; acc[k] += v1[k]; acc[k] += v2[k]; acc[k] += v3[k]; }
+      }
+      for (; e < e_end; ++e) {
+        float v0[C];
+        VecIO<TI, C>::load(h + (int64_t)col[e] * ldh + c * C, v0);
+#pragma unroll
+        for (int k = 0; k < C; ++k) acc[k] += v0[k];
+      }
+      const float fd = (float)D;
+#pragma unroll
+      for (int k = 0; k < C; ++k) acc[k] = D > 0 ? acc[k] / fd : 0.f;
+      VecIO<TO, C>::store(agg + i * lda + c * C, acc);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ aggregate (long tail)
+template <class TI, class TO, int C>
+__global__ void __launch_bounds__(256) k_agg_heavy(const int32_t* __restrict__ heavy,
+                                                   const int32_t* __restrict__ rp,
+                                                   const int32_t* __restrict__ col,
+                                                   const TI* __restrict__ h, int64_t ldh, int d,
+                                                   TO* __restrict__ agg, int64_t lda) {
+  __shared__ float part[8][32][C];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t i = heavy[blockIdx.x];
+  const int32_t b = rp[i], e_end = rp[i + 1];
+  const float fd = (float)(e_end - b);
+  const int nch = (d + C - 1) / C;
+  for (int c0 = 0; c0 < nch; c0 += 32) {
+    const int c = c0 + lane;
+    float acc[C];
+#pragma unroll
+    for (int k = 0; k < C; ++k) acc[k] = 0.f;
+    if (c < nch) {
+      for (int32_t e = b + w; e < e_end; e += 8) {
+        float v[C];
+        VecIO<TI, C>::load(h + (int64_t)col[e] * ldh + c * C, v);
+#pragma unroll
+        for (int k = 0; k < C; ++k) acc[k] += v[k];
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < C; ++k) part[w][lane][k] = acc[k];
+    __syncthreads();
+    if (w == 0 && c < nch) {
+      float s[C];
+#pragma unroll
+      for (int k = 0; k < C; ++k) s[k] = part[0][lane][k];
+      for (int ww = 1; ww < 8; ++ww)
+#pragma unroll
+        for (int k = 0; k < C; ++k) s[k] += part[ww][lane][k];
+#pragma unroll
+      for (int k = 0; k < C; ++k) s[k] = s[k] / fd;
+      VecIO<TO, C>::store(agg + i * lda + c * C, s);
+    }
+    __syncthreads();
+  }
+}
+
+template <class TI, class TO>
+static buffalo_status launch_agg(const buffalo_block* blk, const int32_t* col, const TI* h,
+                                 int64_t ldh, int d, TO* agg, int64_t lda, cudaStream_t s) {
+  const int64_t n = blk->n_dst;
+  if (n <= 0) return BUFFALO_OK;
+  const bool wide = d > 128;
+  if (wide) {
+    k_agg_rows<TI, TO, 8><<<grid_for(n * 32, 256, 16), 256, 0, s>>>(blk->row_ptr, col, n, h, ldh, d, agg, lda);
+  } else {
+    k_agg_rows<TI, TO, 4><<<grid_for(n * 32, 256, 16), 256, 0, s>>>(blk->row_ptr, col, n, h, ldh, d, agg, lda);
+  }
+  BF_LAUNCHED("k_agg_rows");
+  if (blk->n_heavy > 0) {
+    if (wide)
+      k_agg_heavy<TI, TO, 8><<<(unsigned)blk->n_heavy, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, ldh, d, agg, lda);
+    else
+      k_agg_heavy<TI, TO, 4><<<(unsigned)blk->n_heavy, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, ldh, d, agg, lda);
+    BF_LAUNCHED("k_agg_heavy");
+  }
+  return BUFFALO_OK;
+}
+
+// ------------------------------------------------------------------ SIMT GEMM
+// C[M][Np] = A1[M][K1] B1[K1][N] + A2[M][K2] B2[K2][N] (+ bias) (ReLU); columns N..Np-1 = 0.
+// A1 row r is A1[gidx ? gidx[r] : r] and is zero for r >= m1.
+constexpr int GB_M = 64, GB_N = 64, GB_K = 16;
+
+template <class TA1, class TA2, class TO>
+__global__ void __launch_bounds__(256) k_gemm2(int64_t M, int N, int Np, int K1, int K2,
+                                               const TA1* __restrict__ A1, int64_t lda1,
+                                               const int32_t* __restrict__ gidx, int64_t m1,
+                                               const TA2* __restrict__ A2, int64_t lda2,
+                                               const float* __restrict__ B1, int64_t ldb1,
+                                               const float* __restrict__ B2, int64_t ldb2,
+                                               const float* __restrict__ bias, int relu,
+                                               TO* __restrict__ Cm, int64_t ldc) {
+  __shared__ float As[GB_K][GB_M + 4];
+  __shared__ float Bs[GB_K][GB_N];
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int64_t m0 = (int64_t)blockIdx.x * GB_M;
+  const int n0 = blockIdx.y * GB_N;
+  float acc[4][4] = {};
+  const int nk1 = (K1 + GB_K - 1) / GB_K, nk2 = (K2 + GB_K - 1) / GB_K;
+  const int ar = tid >> 2, ak = (tid & 3) * 4;     // A: row ar, k ak..ak+3
+  const int bk = tid >> 4, bn = (tid & 15) * 4;    // B: k bk, n bn..bn+3
+  for (int kt = 0; kt < nk1 + nk2; ++kt) {
+    const bool first = kt < nk1;
+    const int k0 = first ? kt * GB_K : (kt - nk1) * GB_K;
+    const int K = first ? K1 : K2;
+    {
+      const int64_t r = m0 + ar;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int k = k0 + ak + q;
+        float v = 0.f;
+        if (r < M && k < K) {
+          if (first) {
+            if (r < m1) {
+              const int64_t rr = gidx ? (int64_t)gidx[r] : r;
+              v = ld1<TA1>(A1 + rr * lda1 + k);
+            }
+          } else {
+            v = ld1<TA2>(A2 + r * lda2 + k);
+          }
+        }
+        As[ak + q][ar] = v;
+      }
+      const int k = k0 + bk;
+      const float* B = first ? B1 : B2;
+      const int64_t ldb = first ? ldb1 : ldb2;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int nn = n0 + bn + q;
+        Bs[bk][bn + q] = (k < K && nn < N) ? __ldg(B + (int64_t)k * ldb + nn) : 0.f;
+      }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int kk = 0; kk < GB_K; ++kk) {
+      float a[4], b[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) a[i] = As[kk][ty * 4 + i];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) b[j] = Bs[kk][tx * 4 + j];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int64_t r = m0 + ty * 4 + i;
+    if (r >= M) continue;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int nn = n0 + tx * 4 + j;
+      if (nn >= Np) continue;
+      float v = 0.f;
+      if (nn < N) {
+        v = acc[i][j] + (bias ? bias[nn] : 0.f);
+        if (relu) v = fmaxf(v, 0.f);
+      }
+      st1<TO>(Cm + r * ldc + nn, v);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ backward pieces
+template <class TH>
+__global__ void k_dz_mask(float* __restrict__ dz, int64_t ldz, const TH* __restrict__ h, int64_t ldh,
+                          int64_t n, int d) {
+  const int64_t total = n * d;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = t / d;
+    const int c = (int)(t - i * d);
+    if (!(ld1<TH>(h + i * ldh + c) > 0.f)) dz[i * ldz + c] = 0.f;
+  }
+}
+
+// Transposed aggregate: out[j] = sum_{t in T(j)} dZ[i_t] / D(i_t), ascending i_t.
+__global__ void __launch_bounds__(256) k_aggT(const int32_t* __restrict__ trp, const int32_t* __restrict__ tcol,
+                                              const int32_t* __restrict__ rp, int64_t n_src,
+                                              const float* __restrict__ dz, int64_t ldz, int d,
+                                              float* __restrict__ out, int64_t ldo, int dp) {
+  const int lane = threadIdx.x & 31;
+  const int nch = (dp + 3) / 4;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t j = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; j < n_src; j += warps) {
+    const int32_t b = trp[j], e_end = trp[j + 1];
+    for (int c = lane; c < nch; c += 32) {
+      float acc[4] = {0.f, 0.f, 0.f, 0.f};
+      for (int32_t t = b; t < e_end; ++t) {
+        const int64_t i = tcol[t];
+        const float fd = (float)(rp[i + 1] - rp[i]);
+        float v[4];
+        VecIO<float, 4>::load(dz + i * ldz + c * 4, v);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) acc[k] += v[k] / fd;
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+        if (c * 4 + k >= d) acc[k] = 0.f;
+      VecIO<float, 4>::store(out + j * ldo + c * 4, acc);
+    }
+  }
+}
+
+// dW partial of split s: part[s][n][k] = sum_{r in split s} dZ[r][n] * Afwd[r][k],
+// Afwd[r] = [self(r) || agg(r)].
+template <class TS, class TG>
+__global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, int d_in,
+                                                    const float* __restrict__ dz, int64_t ldz,
+                                                    const TS* __restrict__ self, int64_t lds,
+                                                    const int32_t* __restrict__ gidx,
+                                                    const TG* __restrict__ agg, int64_t ldg,
+                                                    int64_t rows_per_split, float* __restrict__ part) {
+  __shared__ float Zs[16][64];
+  __shared__ float As[16][64];
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int k0 = blockIdx.x * 64, n0 = blockIdx.y * 64;
+  const int64_t r_beg = (int64_t)blockIdx.z * rows_per_split;
+  const int64_t r_end = min(nrows, r_beg + rows_per_split);
+  const int K = 2 * d_in;
+  float acc[4][4] = {};
+  const int lr = tid >> 4, lc = (tid & 15) * 4;
+  for (int64_t r0 = r_beg; r0 < r_end; r0 += 16) {
+    const int64_t r = r0 + lr;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int nn = n0 + lc + q, k = k0 + lc + q;
+      float z = 0.f, a = 0.f;
+      if (r < r_end) {
+        if (nn < d_out) z = dz[r * ldz + nn];
+        if (k < d_in) {
+          const int64_t rr = gidx ? (int64_t)gidx[r] : r;
+          a = ld1<TS>(self + rr * lds + k);
+        } else if (k < K) {
+          a = ld1<TG>(agg + r * ldg + (k - d_in));
+        }
+      }
+      Zs[lr][lc + q] = z;
+      As[lr][lc + q] = a;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int rr = 0; rr < 16; ++rr) {
+      float zz[4], aa[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) zz[i] = Zs[rr][ty * 4 + i];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) aa[j] = As[rr][tx * 4 + j];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(zz[i], aa[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+  float* P = part + (int64_t)blockIdx.z * d_out * K;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int nn = n0 + ty * 4 + i;
+    if (nn >= d_out) continue;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int k = k0 + tx * 4 + j;
+      if (k < K) P[(int64_t)nn * K + k] = acc[i][j];
+    }
+  }
+}
+
+__global__ void k_colsum_partial(int64_t nrows, int d, const float* __restrict__ dz, int64_t ldz,
+                                 int64_t rows_per_split, float* __restrict__ part) {
+  const int64_t r_beg = (int64_t)blockIdx.x * rows_per_split;
+  const int64_t r_end = min(nrows, r_beg + rows_per_split);
+  for (int c = threadIdx.x; c < d; c += blockDim.x) {
+    float s = 0.f;
+    for (int64_t r = r_beg; r < r_end; ++r) s += dz[r * ldz + c];
+    part[(int64_t)blockIdx.x * d + c] = s;
+  }
+}
+
+__global__ void k_reduce_partials(const float* __restrict__ part, int S, int64_t count, float* __restrict__ out) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < count; j += (int64_t)gridDim.x * blockDim.x) {
+    float s = 0.f;
+    for (int q = 0; q < S; ++q) s += part[(int64_t)q * count + j];
+    out[j] += s;
+  }
+}
+
+// ------------------------------------------------------------------ loss, optimizer, packing
+__global__ void __launch_bounds__(256) k_softmax_ce(const float* __restrict__ z, int64_t ld, int64_t n, int classes,
+                                                    const int32_t* __restrict__ labels,
+                                                    const int32_t* __restrict__ ids, float invS,
+                                                    float* __restrict__ loss, float* __restrict__ dl,
+                                                    int64_t ldd) {
+  __shared__ float sw[8];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t warps = (int64_t)gridDim.x * 8;
+  float blk_loss = 0.f;
+  for (int64_t i = blockIdx.x * 8LL + w; i < n; i += warps) {
+    const float* zi = z + i * ld;
+    const int y = labels[ids[i]];
+    float m = -INFINITY;
+    for (int c = lane; c < classes; c += 32) m = fmaxf(m, zi[c]);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    float s = 0.f;
+    for (int c = lane; c < classes; c += 32) s += expf(zi[c] - m);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const float lse = m + logf(s);
+    for (int c = lane; c < (int)ldd; c += 32) {
+      float g = 0.f;
+      if (c < classes) g = (expf(zi[c] - m) / s - (c == y ? 1.f : 0.f)) * invS;
+      dl[i * ldd + c] = g;
+    }
+    if (lane == 0) blk_loss += (lse - zi[y]) * invS;
+  }
+  if (lane == 0) sw[w] = blk_loss;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float t = 0.f;
+    for (int k = 0; k < 8; ++k) t += sw[k];
+    atomicAdd(loss, t);
+  }
+}
+
+__global__ void k_sgd(float* __restrict__ p, float* __restrict__ g, int64_t n, float lr) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+    p[j] -= lr * g[j];
+    g[j] = 0.f;
+  }
+}
+
+__global__ void k_transpose_w(const float* __restrict__ W, int rows, int cols, float* __restrict__ Wt) {
+  const int64_t total = (int64_t)rows * cols;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int r = (int)(t / cols), c = (int)(t % cols);
+    Wt[(int64_t)c * rows + r] = W[t];
+  }
+}
+
+// ================================================================== host launchers
+buffalo_status launch_softmax_ce(const float* logits, int64_t ld, int64_t n, int classes,
+                                 const int32_t* labels, const int32_t* ids, int64_t S,
+                                 float* loss, float* dl, int64_t ldd, cudaStream_t s) {
+  if (n <= 0) return BUFFALO_OK;
+  k_softmax_ce<<<grid_for(n, 8, 16), 256, 0, s>>>(logits, ld, n, classes, labels, ids, 1.0f / (float)S,
+                                                  loss, dl, ldd);
+  BF_LAUNCHED("k_softmax_ce");
+  return BUFFALO_OK;
+}
+
+buffalo_status launch_sgd(float* p, float* g, int64_t n, float lr, cudaStream_t s) {
+  if (n <= 0) return BUFFALO_OK;
+  k_sgd<<<grid_for(n, 256), 256, 0, s>>>(p, g, n, lr);
+  BF_LAUNCHED("k_sgd");
+  return BUFFALO_OK;
+}
+
+buffalo_status launch_transpose_w(const float* W, int rows, int cols, float* Wt, cudaStream_t s) {
+  k_transpose_w<<<grid_for((int64_t)rows * cols, 256), 256, 0, s>>>(W, rows, cols, Wt);
+  BF_LAUNCHED("k_transpose_w");
+  return BUFFALO_OK;
+}
+
+template <class TI, class TA>
+static buffalo_status fwd_ffma_t(const FwdArgs& a, cudaStream_t s) {
+  const buffalo_block* blk = a.blk;
+  const int32_t* col = a.layer1 ? blk->col_global : blk->col_local;
+  BF_CHECK(launch_agg<TI, TA>(blk, col, (const TI*)a.h_src, a.ld_src, a.d_in, (TA*)a.agg, a.ld_agg, s));
+  const int64_t M = blk->n_dst;
+  if (M <= 0) return BUFFALO_OK;
+  const int Np = (int)pitch_of(a.d_out);
+  dim3 grid((unsigned)ceil_div(M, GB_M), (unsigned)ceil_div(Np, GB_N));
+  const float* Wt = (const float*)a.W_packed;   // [2 d_in][d_out]
+  if (a.out_f32) {
+    k_gemm2<TI, TA, float><<<grid, 256, 0, s>>>(M, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
+                                               a.layer1 ? blk->src_global : nullptr, M, (const TA*)a.agg,
+                                               a.ld_agg, Wt, a.d_out, Wt + (int64_t)a.d_in * a.d_out,
+                                               a.d_out, a.b, a.relu, (float*)a.out, a.ld_out);
+  } else {
+    k_gemm2<TI, TA, TA><<<grid, 256, 0, s>>>(M, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
+                                            a.layer1 ? blk->src_global : nullptr, M, (const TA*)a.agg,
+                                            a.ld_agg, Wt, a.d_out, Wt + (int64_t)a.d_in * a.d_out,
+                                            a.d_out, a.b, a.relu, (TA*)a.out, a.ld_out);
+  }
+  BF_LAUNCHED("k_gemm2");
+  return BUFFALO_OK;
+}
+
+buffalo_status sage_fwd_ffma(const FwdArgs& a, cudaStream_t s) {
+  if (a.in_bf16 && a.act_bf16) return fwd_ffma_t<__nv_bfloat16, __nv_bfloat16>(a, s);
+  if (a.in_bf16 && !a.act_bf16) return fwd_ffma_t<__nv_bfloat16, float>(a, s);
+  if (!a.in_bf16 && a.act_bf16) return fwd_ffma_t<float, __nv_bfloat16>(a, s);
+  return fwd_ffma_t<float, float>(a, s);
+}
+
+int dw_splits(int64_t n_l, int d_out, int d_in) {
+  int64_t tiles = ceil_div(d_out, 64) * ceil_div(2 * d_in, 64);
+  int64_t a = ceil_div(296, tiles), b = ceil_div(n_l, 512);
+  int64_t sp = a < b ? a : b;
+  return (int)(sp < 1 ? 1 : sp);
+}
+
+int64_t bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int layer, int d_in, int d_out) {
+  int S = dw_splits(n_dst, d_out, d_in);
+  int64_t b = R((int64_t)S * d_out * 2 * d_in * 4) + R((int64_t)S * pitch_of(d_out) * 4);
+  if (layer >= 2) b += R(n_src * pitch_of(d_out) * 4);
+  return b;
+}
+
+template <class TS, class TG, class TH>
+static buffalo_status bwd_ffma_t(const BwdArgs& a, cudaStream_t s) {
+  const buffalo_block* blk = a.blk;
+  const int64_t n = blk->n_dst;
+  const int d_in = a.d_in, d_out = a.d_out;
+  if (!a.last && n > 0) {
+    k_dz_mask<TH><<<grid_for(n * d_out, 256), 256, 0, s>>>(a.dh, a.ld_dh, (const TH*)a.h_dst, a.ld_hdst, n, d_out);
+    BF_LAUNCHED("k_dz_mask");
+  }
+  const int S = dw_splits(n, d_out, d_in);
+  char* q = (char*)a.scratch;
+  float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * d_in * 4);
+  float* db_part = (float*)q; q += R((int64_t)S * pitch_of(d_out) * 4);
+  float* aggT = (float*)q;
+  const int64_t rps = ceil_div(n > 0 ? n : 1, S);
+  if (n > 0) {
+    dim3 g((unsigned)ceil_div(2 * d_in, 64), (unsigned)ceil_div(d_out, 64), (unsigned)S);
+    k_dw_partial<TS, TG><<<g, 256, 0, s>>>(n, d_out, d_in, a.dh, a.ld_dh, (const TS*)a.h_src, a.ld_src,
+                                           a.layer1 ? blk->src_global : nullptr, (const TG*)a.agg,
+                                           a.ld_agg, rps, dw_part);
+    BF_LAUNCHED("k_dw_partial");
+    k_colsum_partial<<<S, 256, 0, s>>>(n, d_out, a.dh, a.ld_dh, rps, db_part);
+    BF_LAUNCHED("k_colsum_partial");
+    k_reduce_partials<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, (int64_t)d_out * 2 * d_in, a.dW);
+    BF_LAUNCHED("k_reduce_partials");
+    k_reduce_partials<<<1, 256, 0, s>>>(db_part, S, d_out, a.db);
+    BF_LAUNCHED("k_reduce_partials");
+  }
+  if (a.dh_src) {
+    const int64_t ns = blk->n_src;
+    if (ns <= 0) return BUFFALO_OK;
+    const int dp = (int)pitch_of(d_out);
+    k_aggT<<<grid_for(ns * 32, 256, 16), 256, 0, s>>>(blk->t_row_ptr, blk->t_col, blk->row_ptr, ns, a.dh,
+                                                     a.ld_dh, d_out, aggT, dp, dp);
+    BF_LAUNCHED("k_aggT");
+    const int Np = (int)pitch_of(d_in);
+    dim3 grid((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(Np, GB_N));
+    k_gemm2<float, float, float><<<grid, 256, 0, s>>>(ns, d_in, Np, d_out, d_out, a.dh, a.ld_dh, nullptr, n,
+                                                      aggT, dp, a.W, 2 * d_in, a.W + d_in, 2 * d_in,
+                                                      nullptr, 0, a.dh_src, a.ld_dh_src);
+    BF_LAUNCHED("k_gemm2");
+  }
+  return BUFFALO_OK;
+}
+
+buffalo_status sage_bwd_ffma(const BwdArgs& a, cudaStream_t s) {
+  // TS: dtype of the layer input rows (features at layer 1), TG/TH: activation dtype
+  if (a.in_bf16 && a.act_bf16) return bwd_ffma_t<__nv_bfloat16, __nv_bfloat16, __nv_bfloat16>(a, s);
+  if (a.in_bf16 && !a.act_bf16) return bwd_ffma_t<__nv_bfloat16, float, float>(a, s);
+  if (!a.in_bf16 && a.act_bf16) return bwd_ffma_t<float, __nv_bfloat16, __nv_bfloat16>(a, s);
+  return bwd_ffma_t<float, float, float>(a, s);
+}
+
+}  // namespace buffalo

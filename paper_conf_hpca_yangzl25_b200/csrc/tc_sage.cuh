@@ -1,0 +1,13 @@
+// tc_sage.cuh — tcgen05 (5th-gen tensor core) path of the fused SAGE layer.
+#pragma once
+#include "common.cuh"
+#include "sage.cuh"
+
+namespace buffalo {
+
+int64_t tc_packed_bytes(int64_t d_in, int64_t d_out);
+buffalo_status tc_pack_weights(const float* W, int d_in, int d_out, void* packed, cudaStream_t s);
+bool tc_fwd_supported(const FwdArgs& a);
+buffalo_status tc_sage_fwd(const FwdArgs& a, cudaStream_t s);
+
+}  // namespace buffalo

@@ -1,0 +1,194 @@
+"""Epoch driver: one Buffalo iteration (Alg. 2) through the C ABI.
+
+Python only allocates torch device buffers, marshals arguments and calls NCCL through
+torch.distributed for the single gradient allreduce (R24); every step of the
+path (bucketize, blocks, forward, loss, backward, optimizer) runs in libbuffalo's kernels.
+"""
+import ctypes
+import time
+
+import numpy as np
+import torch
+
+from . import buffalo as B
+
+
+class DeviceGraph:
+    """CSR graph resident in HBM (+ the node_map workspace the relabel kernels use)."""
+
+    def __init__(self, row_ptr, col, device="cuda"):
+        self.row_ptr = torch.as_tensor(np.asarray(row_ptr, np.int64)).to(device)
+        self.col = torch.as_tensor(np.asarray(col, np.int32)).to(device)
+        self.N = self.row_ptr.numel() - 1
+        self.ws = torch.empty(B.graph_workspace_bytes(self.N), dtype=torch.uint8, device=device)
+        self.g = B.Graph()
+        self.g.num_nodes = self.N
+        self.g.nnz = self.col.numel()
+        self.g.row_ptr = self.row_ptr.data_ptr()
+        self.g.col = self.col.data_ptr()
+        B.graph_prepare(self.g, self.ws)
+
+
+class SageParams:
+    """fp32 master weights/biases (Xavier init from synth), flat gradient buffer, packed copies."""
+
+    def __init__(self, model, Ws, bs, device="cuda"):
+        self.model = model
+        self.L = model.num_layers
+        sizes = [w.size for w in Ws] + [b.size for b in bs]
+        self.flat = torch.zeros(sum(sizes), dtype=torch.float32, device=device)
+        self.grad = torch.zeros_like(self.flat)
+        self.W, self.b, self.dW, self.db = [], [], [], []
+        off = 0
+        for w in Ws:
+            self.W.append(self.flat[off:off + w.size].view(w.shape))
+            self.dW.append(self.grad[off:off + w.size].view(w.shape))
+            self.W[-1].copy_(torch.as_tensor(w))
+            off += w.size
+        for b in bs:
+            self.b.append(self.flat[off:off + b.size])
+            self.db.append(self.grad[off:off + b.size])
+            self.b[-1].copy_(torch.as_tensor(b))
+            off += b.size
+        self.packed = [torch.empty(B.packed_weight_bytes(model, l), dtype=torch.uint8, device=device)
+                       for l in range(1, self.L + 1)]
+        self.repack()
+
+    def repack(self):
+        for l in range(1, self.L + 1):
+            B.pack_weights(self.model, l, self.W[l - 1], self.packed[l - 1])
+
+
+class Trainer:
+    def __init__(self, graph, feats, labels, seeds, dims, fanout, F, Ws, bs, feat_dtype=B.FP32,
+                 gemm_mode=B.GEMM_FFMA, mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096,
+                 base_seed=3, rank=0, world=1, process_group=None, device="cuda"):
+        self.graph = graph if isinstance(graph, DeviceGraph) else DeviceGraph(*graph, device=device)
+        self.feats = feats
+        self.labels = labels
+        self.seeds = seeds
+        self.S = seeds.numel()
+        self.dims = list(dims)
+        self.L = len(dims) - 1
+        self.fanout = list(fanout)
+        self.F = F
+        self.base_seed = base_seed
+        self.model = B.make_model(dims, feat_dtype, gemm_mode, feats.shape[1])
+        self.sched = B.make_sched(mem_budget, C_ppm, k_min, k_max, world)
+        self.params = SageParams(self.model, Ws, bs, device)
+        self.rank, self.world, self.pg = rank, world, process_group
+        self.device = device
+        # scheduler outputs
+        self.k_cap = k_max
+        self.group_of_seed = torch.empty(self.S, dtype=torch.int32, device=device)
+        self.group_seeds = torch.empty(self.S, dtype=torch.int32, device=device)
+        self.group_offsets = torch.empty(k_max + 1, dtype=torch.int64, device=device)
+        self.offs_h = np.zeros(k_max + 1, np.int64)
+        self.est_h = np.zeros(k_max, np.int64)
+        self.rank_h = np.zeros(k_max, np.int32)
+        self.hist_h = np.zeros(F + 1, np.int64)
+        self.plan = B.Plan()
+        self.plan.group_of_seed = self.group_of_seed.data_ptr()
+        self.plan.group_seeds = self.group_seeds.data_ptr()
+        self.plan.group_offsets = self.group_offsets.data_ptr()
+        self.plan.group_offsets_h = self.offs_h.ctypes.data
+        self.plan.est_bytes_h = self.est_h.ctypes.data
+        self.plan.rank_of_group_h = self.rank_h.ctypes.data
+        self.plan.hist_h = self.hist_h.ctypes.data
+        sampler = B.make_sampler(self.fanout, F, base_seed)
+        wsb = B.bucketize_workspace_bytes(self.graph.g, self.S, sampler, self.model)
+        self.bucket_ws = torch.empty(wsb, dtype=torch.uint8, device=device)
+        self.arena = torch.empty(0, dtype=torch.uint8, device=device)
+        self.loss = torch.zeros(1, dtype=torch.float32, device=device)
+        self.blocks = B.Blocks()
+        self.last = {}
+
+    # --------------------------------------------------------------- pieces of Alg. 2
+    def sampler(self, epoch):
+        return B.make_sampler(self.fanout, self.F, self.base_seed + epoch)
+
+    def schedule(self, epoch):
+        B.bucketize(self.graph.g, self.seeds, self.sampler(epoch), self.model, self.sched, self.plan,
+                    self.bucket_ws)
+        K = self.plan.k_out
+        return K, self.offs_h[:K + 1].copy(), self.est_h[:K].copy(), self.rank_h[:K].copy()
+
+    def _ensure_arena(self, nbytes):
+        if self.arena.numel() < nbytes:
+            self.arena = torch.empty(int(nbytes), dtype=torch.uint8, device=self.device)
+
+    def build(self, off, n, sampler):
+        while True:
+            try:
+                return B.build_blocks(self.graph.g, self.group_seeds.data_ptr() + 4 * int(off), n, sampler,
+                                      self.model, self.blocks, self.arena)
+            except B.BuffaloError as e:
+                if e.status != B.ERR_CAPACITY:
+                    raise
+                self._ensure_arena(max(int(e.required * 1.25), 2 * self.arena.numel(), 1 << 20))
+
+    def forward(self):
+        m, p, blks = self.model, self.params, self.blocks
+        h, ld = self.feats, self.feats.shape[1]
+        for l in range(1, self.L + 1):
+            b = blks.layer[l - 1]
+            B.sage_fwd(b, l, m, h, ld, p.W[l - 1], p.packed[l - 1], p.b[l - 1], b.out, b.ld_out, b.agg, b.ld_agg)
+            h, ld = b.out, b.ld_out
+
+    def backward(self):
+        m, p, blks = self.model, self.params, self.blocks
+        for l in range(self.L, 0, -1):
+            b = blks.layer[l - 1]
+            if l > 1:
+                prev = blks.layer[l - 2]
+                h_src, ld_src, dh_src, ld_dh_src = prev.out, prev.ld_out, prev.dh, prev.ld_dh
+            else:
+                h_src, ld_src, dh_src, ld_dh_src = self.feats, self.feats.shape[1], None, 0
+            h_dst = b.out if l < self.L else None
+            B.sage_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out,
+                       p.W[l - 1], p.packed[l - 1], p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src,
+                       b.bwd_scratch, b.bwd_scratch_bytes)
+
+    def loss_and_grad(self, off, n):
+        b = self.blocks.layer[self.L - 1]
+        ids = self.group_seeds.data_ptr() + 4 * int(off)
+        B.softmax_ce(b.out, b.ld_out, n, self.dims[-1], self.labels, ids, self.S, self.loss, b.dh, b.ld_dh)
+
+    def microbatch(self, off, n, sampler):
+        self.build(off, n, sampler)
+        self.forward()
+        self.loss_and_grad(off, n)
+        self.backward()
+        blk = self.blocks
+        return dict(edges=sum(blk.layer[l].n_edges for l in range(self.L)),
+                    n=[blk.layer[0].n_src] + [blk.layer[l].n_dst for l in range(self.L)],
+                    e=[blk.layer[l].n_edges for l in range(self.L)],
+                    peak=blk.arena_peak, est_lo=blk.est_lo, est_hi=blk.est_hi)
+
+    def allreduce(self):
+        if self.world > 1:
+            torch.distributed.all_reduce(self.params.grad, group=self.pg)
+
+    def step(self, lr):
+        B.sgd_step(self.params.flat, self.params.grad, lr)
+        self.params.repack()
+
+    def run_epoch(self, epoch=0, lr=0.01, timers=False):
+        """One Buffalo iteration; returns stats (K, own groups, aggregated edges, ...)."""
+        self.loss.zero_()
+        K, offs, est, ranks = self.schedule(epoch)
+        if self.arena.numel() == 0:
+            mine = [est[k] for k in range(K) if ranks[k] == self.rank]
+            self._ensure_arena(max(mine) if mine else 1 << 20)
+        sampler = self.sampler(epoch)
+        groups = []
+        for k in range(K):
+            if ranks[k] != self.rank:
+                continue
+            groups.append(self.microbatch(offs[k], int(offs[k + 1] - offs[k]), sampler))
+        self.allreduce()
+        self.step(lr)
+        self.last = dict(K=K, k_tried=self.plan.k_tried, exploded=self.plan.exploded, est=est,
+                         ranks=ranks, groups=groups, edges=sum(g["edges"] for g in groups),
+                         hist=self.hist_h.copy())
+        return self.last

@@ -1,0 +1,205 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded inputs.
+
+Integer work (buckets, plan, blocks, transposes, heavy lists) must be bit-exact; fp32 (FFMA
+mode) within rel 1e-4 / abs 1e-5; the bf16-GEMM path within rel 2e-2 (+ 2e-2 rms floor,
+Appendix C of SURVEY.md); layer-1 aggregation of k/128 features is bit-exact in both modes.
+Sizes span several tiles, ragged tails, zero-degree seeds and long-tail (heavy) rows.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from synth.graphs import features, labels, random_graph, seed_nodes, xavier_weights
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    from gpu_helpers import (B, act_view, arena_view, assert_bf16_close, assert_close,
+                             blocks_to_numpy, make_trainer)
+
+CASES = {
+    # name: (N, pairs, kind, S, fanout, F, dims)
+    "sampled2": (3000, 20000, "powerlaw", 700, [5, 9], 9, [40, 64, 7]),
+    "full3": (4000, 30000, "powerlaw", 1500, [0, 0, 0], 10, [32, 48, 48, 10]),
+    "mixed3": (5000, 60000, "powerlaw", 900, [3, 0, 25], 25, [24, 40, 56, 12]),
+    "cora": (2708, 5278, "gnm", 2708, [10, 25], 25, [1433, 256, 7]),
+}
+
+
+def _case(name):
+    N, P, kind, S, fan, F, dims = CASES[name]
+    rp, col = random_graph(N, P, kind)
+    X = features(N, dims[0])
+    y = labels(N, dims[-1])
+    seeds = seed_nodes(N, S)
+    Ws, bs = xavier_weights(dims, bias_scale=0.05)
+    return rp, col, X, y, seeds, fan, F, dims, Ws, bs
+
+
+@pytest.mark.parametrize("name", list(CASES))
+def test_blocks_bit_exact(name):
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case(name)
+    g = O.Graph(rp, col)
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs)
+    seed = 11
+    tr.group_seeds.copy_(torch.as_tensor(seeds))
+    tr._ensure_arena(1 << 16)
+    tr.build(0, seeds.size, B.make_sampler(fan, F, seed))
+    got = blocks_to_numpy(tr.arena, tr.blocks, len(fan))
+    ref = O.build_blocks(g, seeds, len(fan), fan, seed)
+    for l, (a, r) in enumerate(zip(got, ref), start=1):
+        assert (a["n_dst"], a["n_src"], a["n_edges"]) == (r["n_dst"], r["n_src"], r["n_edges"]), l
+        np.testing.assert_array_equal(a["row_ptr"], r["row_ptr"])
+        np.testing.assert_array_equal(a["col_local"], r["col_local"])
+        np.testing.assert_array_equal(a["src_global"], r["src_global"])
+        if l == 1:
+            np.testing.assert_array_equal(a["col_global"], r["col_global"])
+        else:
+            np.testing.assert_array_equal(a["t_row_ptr"], r["t_row_ptr"])
+            np.testing.assert_array_equal(a["t_col"], r["t_col"])
+        np.testing.assert_array_equal(a["heavy"], np.nonzero(r["D"] > O.HEAVY_T)[0])
+    if name == "full3":
+        assert got[0]["n_heavy"] > 0          # the long-tail path is exercised
+
+
+@pytest.mark.parametrize("name", ["sampled2", "full3", "mixed3"])
+@pytest.mark.parametrize("variant", ["k4", "budget", "C", "gpus3"])
+def test_bucketize_plan_bit_exact(name, variant):
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case(name)
+    g = O.Graph(rp, col)
+    kw = dict(k_min=1, k_max=4096, num_gpus=1, C_ppm=0, mem_budget=(1 << 63) - 1)
+    if variant == "k4":
+        kw.update(k_min=4, k_max=4)
+    elif variant == "budget":
+        full = O.schedule(g, seeds, len(fan), fan, F, 3, dims, k_min=1, k_max=1)
+        kw.update(mem_budget=int(full["est_bytes"][0] * 0.3))
+    elif variant == "C":
+        full = O.schedule(g, seeds, len(fan), fan, F, 3, dims, k_min=1, k_max=1)
+        kw.update(mem_budget=int(full["est_bytes"][0] * 0.3), C_ppm=226000)
+    else:
+        kw.update(num_gpus=3)
+    ref = O.schedule(g, seeds, len(fan), fan, F, 3, dims, **kw)
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, base_seed=3,
+                      **{k: v for k, v in kw.items() if k != "num_gpus"}, world=kw["num_gpus"])
+    K, offs, est, ranks = tr.schedule(0)
+    assert K == ref["K"] and tr.plan.k_tried == ref["K_tried"]
+    np.testing.assert_array_equal(offs, ref["group_offsets"])
+    np.testing.assert_array_equal(est, ref["est_bytes"])
+    np.testing.assert_array_equal(ranks, ref["rank_of_group"])
+    np.testing.assert_array_equal(tr.group_seeds.cpu().numpy(), ref["group_seeds"])
+    np.testing.assert_array_equal(tr.group_of_seed.cpu().numpy(), ref["group_of_seed"])
+    np.testing.assert_array_equal(tr.hist_h, ref["hist"])
+
+
+def test_bucketize_budget_error():
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case("sampled2")
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, mem_budget=4096, k_max=16)
+    with pytest.raises(B.BuffaloError) as ei:
+        tr.schedule(0)
+    assert ei.value.status == B.ERR_BUDGET
+
+
+def _run_microbatch(tr, seeds, fan, F, seed):
+    tr.group_seeds.copy_(torch.as_tensor(seeds))
+    tr._ensure_arena(1 << 16)
+    tr.loss.zero_()
+    tr.params.grad.zero_()
+    info = tr.microbatch(0, seeds.size, B.make_sampler(fan, F, seed))
+    torch.cuda.synchronize()
+    return info
+
+
+@pytest.mark.parametrize("name", list(CASES))
+@pytest.mark.parametrize("gemm", ["ffma", "bf16"])
+def test_microbatch_fwd_bwd_parity(name, gemm):
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case(name)
+    g = O.Graph(rp, col)
+    L = len(fan)
+    mode = B.GEMM_FFMA if gemm == "ffma" else B.GEMM_BF16
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=mode)
+    S = seeds.size
+    info = _run_microbatch(tr, seeds, fan, F, 7)
+    blocks = O.build_blocks(g, seeds, L, fan, 7)
+    logits, cache = O.sage_forward(blocks, X, Ws, bs)
+    loss, dlog = O.softmax_ce(logits, y[seeds], S)
+    grads = O.sage_backward(blocks, cache, Ws, dlog)
+    adt = torch.float32 if mode == B.GEMM_FFMA else torch.bfloat16
+    # layer-1 aggregation of k/128 features: exact in both modes
+    b1 = tr.blocks.layer[0]
+    agg1 = act_view(tr.arena, b1.agg, b1.n_dst, b1.ld_agg, adt)[:, :dims[0]]
+    if mode == B.GEMM_FFMA:
+        np.testing.assert_array_equal(agg1, cache[0]["agg"].astype(np.float32))
+    else:
+        np.testing.assert_array_equal(agg1, torch.as_tensor(cache[0]["agg"]).to(torch.bfloat16).float().numpy())
+    bl = tr.blocks.layer[L - 1]
+    glog = act_view(tr.arena, bl.out, bl.n_dst, bl.ld_out, torch.float32)[:, :dims[-1]]
+    gW = [w.cpu().numpy() for w in tr.params.dW]
+    gb = [b.cpu().numpy() for b in tr.params.db]
+    if mode == B.GEMM_FFMA:
+        assert_close(glog, logits, 1e-4, 1e-5, "logits")
+        assert abs(tr.loss.item() - loss) <= 1e-5 + 1e-4 * abs(loss)
+        for l in range(L):
+            assert_close(gW[l], grads[l][0], 1e-4, 1e-5, f"dW{l + 1}")
+            assert_close(gb[l], grads[l][1], 1e-4, 1e-5, f"db{l + 1}")
+    else:
+        assert_bf16_close(glog, logits, "logits")
+        assert abs(tr.loss.item() - loss) <= 2e-2 * abs(loss)
+        for l in range(L):
+            assert_bf16_close(gW[l], grads[l][0], f"dW{l + 1}", rel=5e-2)
+            assert_bf16_close(gb[l], grads[l][1], f"db{l + 1}", rel=5e-2)
+    # memory model: the measured arena peak lies in [lo, hi] and equals the oracle's model
+    lo, hi = O.mem_model(info["n"], info["e"], dims, O.FP32 if mode == B.GEMM_FFMA else O.BF16)
+    assert (info["est_lo"], info["est_hi"]) == (lo, hi)
+    assert lo <= info["peak"] <= hi
+
+
+def test_mean_of_constant_is_constant():
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case("full3")
+    Xc = np.full_like(X, 0.5)
+    tr = make_trainer(rp, col, Xc, y, seeds, dims, fan, F, Ws, bs)
+    _run_microbatch(tr, seeds, fan, F, 1)
+    b1 = tr.blocks.layer[0]
+    agg = act_view(tr.arena, b1.agg, b1.n_dst, b1.ld_agg, torch.float32)[:, :dims[0]]
+    D = np.diff(arena_view(tr.arena, b1.row_ptr, b1.n_dst + 1).cpu().numpy())
+    assert np.all(agg[D > 0] == 0.5) and np.all(agg[D == 0] == 0.0)
+
+
+@pytest.mark.parametrize("gemm", ["ffma", "bf16"])
+def test_microbatch_logits_equal_batch_logits(gemm):
+    """micro-batch training is equivalent to batch training; on the GPU the
+    per-seed logits of a group equal the full batch's bit for bit (row-local reductions)."""
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case("mixed3")
+    mode = B.GEMM_FFMA if gemm == "ffma" else B.GEMM_BF16
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=mode)
+    _run_microbatch(tr, seeds, fan, F, 5)
+    bl = tr.blocks.layer[-1 + len(fan)]
+    full = act_view(tr.arena, bl.out, bl.n_dst, bl.ld_out, torch.float32).copy()
+    pos = {int(s): i for i, s in enumerate(seeds)}
+    for part in np.array_split(seeds[::-1].copy(), 3):
+        _run_microbatch(tr, part, fan, F, 5)
+        bl = tr.blocks.layer[len(fan) - 1]
+        sub = act_view(tr.arena, bl.out, bl.n_dst, bl.ld_out, torch.float32)
+        np.testing.assert_array_equal(sub, full[[pos[int(s)] for s in part]])
+
+
+@pytest.mark.parametrize("gemm", ["ffma", "bf16"])
+def test_epoch_parity(gemm):
+    """Alg. 2 end to end: plan, accumulated gradients over K = 4 groups, one SGD step."""
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case("sampled2")
+    g = O.Graph(rp, col)
+    mode = B.GEMM_FFMA if gemm == "ffma" else B.GEMM_BF16
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=mode, k_min=4, k_max=4, base_seed=3)
+    lr = 0.5
+    stats = tr.run_epoch(epoch=2, lr=lr)
+    torch.cuda.synchronize()
+    loss, acc, newW, newb, plan = O.train_epoch(g, seeds, X, y, Ws, bs, len(fan), fan, F, 5, dims, lr=lr,
+                                                k_min=4, k_max=4)
+    assert stats["K"] == plan["K"] == 4
+    for l in range(len(fan)):
+        if mode == B.GEMM_FFMA:
+            assert_close(tr.params.W[l].cpu().numpy(), newW[l], 1e-4, 1e-5, f"W{l + 1}")
+            assert_close(tr.params.b[l].cpu().numpy(), newb[l], 1e-4, 1e-5, f"b{l + 1}")
+        else:
+            assert_bf16_close(tr.params.W[l].cpu().numpy() - Ws[l], newW[l] - Ws[l], f"dW{l + 1}", rel=5e-2)
+    assert float(tr.params.grad.abs().max()) == 0.0       # gradients reset by the step

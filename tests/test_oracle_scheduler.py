@@ -116,14 +116,21 @@ def test_fig9_grouping_structure():
 
 def test_mem_model_hand_instance():
     # L = 1, n = [5, 2], e = [3], dims = [4, 3]; every buffer rounds up to 256 B:
-    # blocks: row_ptr, col_local, src_global, heavy, col_global = 5 * 256 = 1280
-    # build frame: R(4*(2+3+1)) + 8192 = 8448;  acts: agg R(2*8*4) + logits R(2*8*4) = 512
-    # bwd frame l=1: dH_1 R(2*8*4) + dW partials R(1*3*8*4) = 512
-    assert O.mem_model([5, 2], [3], [4, 3], O.FP32) == (1280 + 512 + 512, 1280 + 512 + 8448)
-    # L = 2 adds the transposed block and the dH_{l-1}/aggT buffers of layer 2
-    lo, hi = O.mem_model([300, 100, 10], [400, 50], [16, 8, 4], O.FP32)
-    blocks = (256 * 2 + 1280 + 256 + 1280) + (256 + 1280 + 512 + 256 + 512 + 256 + 256)
-    assert lo > blocks and hi >= lo
+    # blocks: row_ptr, heavy, col_local, src_global, col_global = 5 * 256 = 1280
+    # build frame: totals 256 + scan ws R(4*(ceil(257/16384)+2)) = 256  -> 512
+    # acts: agg R(2*8*4) + logits R(2*8*4) = 512
+    # bwd frame l=1: dH_1 256 + dW partials R(1*3*8*4) 256 + db partials R(1*8*4) 256 = 768
+    assert O.mem_model([5, 2], [3], [4, 3], O.FP32) == (1280 + 512 + 768, 1280 + 512 + 768)
+    # a wide layer: n = [40000, 20000], e = [100000], dims = [64, 32]
+    # blocks: R(80004)=80128, R(80000)=80128, R(400000)=400128, R(160000)=160000, col_global 400128
+    # build: 256 + R(4*(ceil(120001/16384)+2)) = 256 + 256 = 512
+    # acts: agg R(20000*64*4)=5120000, logits R(20000*32*4)=2560000
+    # bwd: dH R(20000*32*4)=2560000; splits: tiles=1*2 -> min(148, 40) = 40;
+    #      dW R(40*32*128*4)=655360; db R(40*32*4)=5120
+    blocks = 80128 + 80128 + 400128 + 160000 + 400128
+    acts = 5120000 + 2560000
+    bwd = 2560000 + 655360 + 5120
+    assert O.mem_model([40000, 20000], [100000], [64, 32], O.FP32) == (blocks + acts + bwd,) * 2
 
 
 def test_mem_model_monotone_and_bf16_smaller():
