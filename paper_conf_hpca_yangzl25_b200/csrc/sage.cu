@@ -444,6 +444,27 @@ __global__ void k_transpose_w(const float* __restrict__ W, int rows, int cols, f
 }
 
 // ================================================================== host launchers
+// Long-tail rows of the tensor-core path: mean written (bf16) into the saved h_agg, which the
+// fused kernel then reads instead of gathering.
+buffalo_status launch_agg_heavy_bf16(const FwdArgs& a, cudaStream_t s) {
+  const buffalo_block* blk = a.blk;
+  const int32_t* col = a.layer1 ? blk->col_global : blk->col_local;
+  const bool wide = a.d_in > 128;
+  __nv_bfloat16* agg = (__nv_bfloat16*)a.agg;
+  const unsigned g = (unsigned)blk->n_heavy;
+  if (a.in_bf16) {
+    const __nv_bfloat16* h = (const __nv_bfloat16*)a.h_src;
+    if (wide) k_agg_heavy<__nv_bfloat16, __nv_bfloat16, 8><<<g, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
+    else k_agg_heavy<__nv_bfloat16, __nv_bfloat16, 4><<<g, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
+  } else {
+    const float* h = (const float*)a.h_src;
+    if (wide) k_agg_heavy<float, __nv_bfloat16, 8><<<g, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
+    else k_agg_heavy<float, __nv_bfloat16, 4><<<g, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
+  }
+  BF_LAUNCHED("k_agg_heavy");
+  return BUFFALO_OK;
+}
+
 buffalo_status launch_softmax_ce(const float* logits, int64_t ld, int64_t n, int classes,
                                  const int32_t* labels, const int32_t* ids, int64_t S,
                                  float* loss, float* dl, int64_t ldd, cudaStream_t s) {

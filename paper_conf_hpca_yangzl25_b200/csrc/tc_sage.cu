@@ -1,13 +1,531 @@
-// tc_sage.cu — placeholder until the tcgen05 kernels land.
+// tc_sage.cu — fused GraphSAGE-mean forward on the 5th-gen tensor cores (sm_100a).
+//
+// One persistent CTA per SM walks tiles of 128 destination rows.  16 gather warps build the
+// A operand [h_self || h_agg] (bf16) of the tile directly in shared memory, in the UMMA
+// K-major SWIZZLE_128B layout, 64 columns (one 128-B swizzle atom) per K-chunk:
+//   * self chunks: the dst rows' own features (row = gidx[i] for layer 1);
+//   * agg chunks:  warp per dst row, 4 lane groups x 8 lanes x 16 B cover 4 neighbours x 64
+//     columns per step; 32 column indices are fetched coalesced once and broadcast by
+//     shuffles, so each lane keeps 8 independent 16-B loads in flight; fp32 accumulation,
+//     one division by D (Alg. 2 l.8, R21); the mean is also written to the saved h_agg.
+// One control warp streams pre-swizzled bf16 weight chunks with cp.async.bulk (mbarrier
+// transaction counts) and one elected thread issues tcgen05.mma (M=128, N=Np, K=16) into a
+// double-buffered TMEM accumulator; the gather warps run the epilogue of tile t-1
+// (tcgen05.ld -> +bias -> ReLU -> store) after gathering tile t, so MMA latency hides under
+// the next gather.  Rows with D > kHeavyT were pre-aggregated by k_agg_heavy (sage.cu).
+#include <algorithm>
+
 #include "tc_sage.cuh"
 
 namespace buffalo {
 
+// ------------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@P1 bra DONE_%=;\n\t"
+      "bra WAIT_%=;\n\t"
+      "DONE_%=:\n\t}" ::"r"(smem_u32(b)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void fence_barrier_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void tmem_alloc(uint32_t* dst_smem, uint32_t ncols) {
+  asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
+               "r"(ncols));
+  asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+}
+__device__ __forceinline__ void tmem_dealloc(uint32_t taddr, uint32_t ncols) {
+  asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols));
+}
+// D[tmem] (+)= A[smem] * B[smem]^T, both K-major; kind::f16 (bf16 in, fp32 accumulate).
+__device__ __forceinline__ void umma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                          uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
+}
+__device__ __forceinline__ void umma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                   smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, float* v) {
+  uint32_t r[8];
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+                 "=r"(r[7])
+               : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 8; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+// UMMA shared-memory descriptor: K-major, SWIZZLE_128B, SBO = 1024 B (8 rows x 128 B).
+__device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)1 << 16;                 // LBO (unused for swizzled K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;       // SBO
+  d |= (uint64_t)1 << 46;                 // descriptor version (sm100)
+  d |= (uint64_t)2 << 61;                 // SWIZZLE_128B
+  return d;
+}
+// Instruction descriptor, kind::f16: D fp32, A/B bf16, both K-major, M = 128, N = n.
+__host__ __device__ constexpr uint32_t idesc_bf16(int n) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+}
+
+__device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+__device__ __forceinline__ void bf16x8_to_f32(const uint4& u, float* v) {
+  const uint32_t w[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    v[2 * i] = __uint_as_float(w[i] << 16);
+    v[2 * i + 1] = __uint_as_float(w[i] & 0xffff0000u);
+  }
+}
+
+// ------------------------------------------------------------------ kernel configuration
+constexpr int kTileM = 128;
+constexpr int kKC = 64;                    // bf16 columns per K-chunk (one 128-B swizzle row)
+constexpr int kChunkBytesA = kTileM * 128; // 16 KB
+constexpr int kSuper = 4;                  // K-chunks per A buffer
+constexpr int kGatherWarps = 16;
+constexpr int kGatherThreads = kGatherWarps * 32;
+constexpr int kThreads = kGatherThreads + 32;
+
+struct TcFwdParams {
+  const int32_t* row_ptr;
+  const int32_t* col;        // neighbour row ids into h (global for layer 1, local otherwise)
+  const int32_t* gidx;       // self row ids (layer 1: src_global) or null (= i)
+  int64_t n_dst;
+  const void* h;             // bf16 or fp32 rows
+  int64_t ldh;               // elements
+  int d_in, pitch_in;        // pitch_in: valid columns readable in a row (multiple of 8)
+  int nkc_self, nkc;         // K-chunks for the self half, total (= 2 nkc_self)
+  const uint8_t* wpk;        // pre-swizzled bf16 W chunks, each Np x 128 B
+  int Np, d_out, ld_out, tmem_cols;
+  const float* bias;
+  int relu, out_f32;
+  void* out;
+  __nv_bfloat16* agg;        // saved h_agg, bf16 [n_dst][ld_agg]
+  int64_t ld_agg;
+};
+
+template <class TI> struct InTraits;
+template <> struct InTraits<__nv_bfloat16> {
+  static constexpr int kElems = 8;     // per 16-B piece
+};
+template <> struct InTraits<float> {
+  static constexpr int kElems = 4;
+};
+
+// Write v (kElems values, columns [piece*kElems, ...)) of row r into the swizzled A chunk.
+template <int E>
+__device__ __forceinline__ void st_swz(uint8_t* chunk, int r, int piece, const float* v) {
+  if constexpr (E == 8) {
+    const int off = r * 128 + (((piece) ^ (r & 7)) << 4);
+    *reinterpret_cast<uint4*>(chunk + off) =
+        make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+                   pack_bf16x2(v[6], v[7]));
+  } else {
+    const int off = r * 128 + (((piece >> 1) ^ (r & 7)) << 4) + ((piece & 1) << 3);
+    *reinterpret_cast<uint2*>(chunk + off) = make_uint2(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]));
+  }
+}
+template <class TI>
+__device__ __forceinline__ void ld_piece(const TI* p, float* v);
+template <> __device__ __forceinline__ void ld_piece<__nv_bfloat16>(const __nv_bfloat16* p, float* v) {
+  bf16x8_to_f32(__ldg(reinterpret_cast<const uint4*>(p)), v);
+}
+template <> __device__ __forceinline__ void ld_piece<float>(const float* p, float* v) {
+  float4 a = __ldg(reinterpret_cast<const float4*>(p));
+  v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+}
+
+template <class TI>
+__device__ __forceinline__ void raw_to_f32(const uint4& u, float* v);
+template <> __device__ __forceinline__ void raw_to_f32<__nv_bfloat16>(const uint4& u, float* v) {
+  bf16x8_to_f32(u, v);
+}
+template <> __device__ __forceinline__ void raw_to_f32<float>(const uint4& u, float* v) {
+  v[0] = __uint_as_float(u.x); v[1] = __uint_as_float(u.y); v[2] = __uint_as_float(u.z); v[3] = __uint_as_float(u.w);
+}
+
+template <class TI>
+__global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p) {
+  constexpr int E = InTraits<TI>::kElems;      // elements per 16-B piece
+  constexpr int P = kKC / E;                   // pieces per 64-column chunk row (8 or 16)
+  constexpr int G = 32 / P;                    // neighbour groups per warp (4 or 2)
+  constexpr int kUnroll = 8;                   // independent 16-B loads in flight per lane
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sA = smem;                                          // 2 x kSuper x 16 KB
+  uint8_t* sB = smem + 2 * kSuper * kChunkBytesA;              // 2 x Np x 128 B
+  const int bbytes = p.Np * 128;
+  uint64_t* bars = (uint64_t*)(sB + 2 * bbytes);
+  uint64_t* a_full = bars;        // [2]
+  uint64_t* a_empty = bars + 2;   // [2]
+  uint64_t* b_full = bars + 4;    // [2]
+  uint64_t* b_empty = bars + 6;   // [2]
+  uint64_t* acc_full = bars + 8;  // [2]
+  uint64_t* acc_empty = bars + 10;// [2]
+  uint32_t* tmem_slot = (uint32_t*)(bars + 12);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t ntiles = (p.n_dst + kTileM - 1) / kTileM;
+  const int nsc = (p.nkc + kSuper - 1) / kSuper;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&a_full[i], kGatherThreads);
+      mbar_init(&a_empty[i], 1);
+      mbar_init(&b_full[i], 1);
+      mbar_init(&b_empty[i], 1);
+      mbar_init(&acc_full[i], 1);
+      mbar_init(&acc_empty[i], kGatherThreads);
+    }
+    fence_barrier_init();
+  }
+  if (warp == kGatherWarps) tmem_alloc(tmem_slot, p.tmem_cols);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == kGatherWarps) {
+    // ===================== control warp: weight chunks + MMA issue (one elected lane)
+    if (lane == 0) {
+      const uint32_t idesc = idesc_bf16(p.Np);
+      int64_t g = 0;           // global chunk counter (B stage = g & 1)
+      int64_t q = 0;           // global super-chunk counter (A buffer = q & 1)
+      int64_t i = 0;           // local tile counter
+      const int64_t total_chunks = ((ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x) * p.nkc;
+      if (total_chunks > 0) {
+        mbar_arrive_expect_tx(&b_full[0], bbytes);
+        bulk_g2s(sB, p.wpk, bbytes, &b_full[0]);
+      }
+      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+        const int acc = (int)(i & 1);
+        if (i >= 2) mbar_wait(&acc_empty[acc], (uint32_t)(((i >> 1) - 1) & 1));
+        tc_fence_after();
+        const uint32_t tmem_d = tmem_base + acc * p.Np;
+        for (int sc = 0; sc < nsc; ++sc, ++q) {
+          const int buf = (int)(q & 1);
+          mbar_wait(&a_full[buf], (uint32_t)((q >> 1) & 1));
+          tc_fence_after();
+          for (int j = 0; j < kSuper; ++j) {
+            const int c = sc * kSuper + j;
+            if (c >= p.nkc) break;
+            const int bs = (int)(g & 1);
+            mbar_wait(&b_full[bs], (uint32_t)((g >> 1) & 1));
+            tc_fence_after();
+            const uint32_t a_addr = smem_u32(sA + (buf * kSuper + j) * kChunkBytesA);
+            const uint32_t b_addr = smem_u32(sB + bs * bbytes);
+#pragma unroll
+            for (int k = 0; k < kKC / 16; ++k)
+              umma_bf16(tmem_d, sw128_desc(a_addr + 32 * k), sw128_desc(b_addr + 32 * k), idesc,
+                        (c > 0 || k > 0) ? 1u : 0u);
+            umma_commit(&b_empty[bs]);
+            // prefetch the next weight chunk into the other stage once its MMAs retired
+            const int64_t gn = g + 1;
+            if (gn < total_chunks) {
+              const int ns = (int)(gn & 1);
+              if (gn >= 2) mbar_wait(&b_empty[ns], (uint32_t)(((gn >> 1) - 1) & 1));
+              const int cn = (int)(gn % p.nkc);
+              mbar_arrive_expect_tx(&b_full[ns], bbytes);
+              bulk_g2s(sB + ns * bbytes, p.wpk + (int64_t)cn * bbytes, bbytes, &b_full[ns]);
+            }
+            ++g;
+          }
+          umma_commit(&a_empty[buf]);
+        }
+        umma_commit(&acc_full[acc]);
+      }
+    }
+    __syncwarp();
+  } else {
+    // ===================== gather + epilogue warps
+    const TI* __restrict__ h = (const TI*)p.h;
+    int64_t q = 0, i = 0;
+    int64_t prev_tile = -1;
+    auto epilogue = [&](int64_t tile, int64_t li) {
+      const int acc = (int)(li & 1);
+      mbar_wait(&acc_full[acc], (uint32_t)((li >> 1) & 1));
+      tc_fence_after();
+      const int quad = warp & 3, part = warp >> 2;
+      const int r = quad * 32 + lane;
+      const int64_t row = tile * kTileM + r;
+      const int ngrp = (int)pitch_of(p.d_out) / 8;
+      for (int grp = part; grp < ngrp; grp += 4) {
+        float v[8];
+        tmem_ld8(tmem_base + ((uint32_t)(quad * 32) << 16) + acc * p.Np + grp * 8, v);
+        if (row < p.n_dst) {
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            const int cidx = grp * 8 + k;
+            float x = v[k] + (cidx < p.d_out ? __ldg(p.bias + cidx) : 0.f);
+            v[k] = p.relu ? fmaxf(x, 0.f) : x;
+          }
+          if (p.out_f32) {
+            float4* o = reinterpret_cast<float4*>((float*)p.out + row * p.ld_out + grp * 8);
+            o[0] = make_float4(v[0], v[1], v[2], v[3]);
+            o[1] = make_float4(v[4], v[5], v[6], v[7]);
+          } else {
+            *reinterpret_cast<uint4*>((__nv_bfloat16*)p.out + row * p.ld_out + grp * 8) =
+                make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+                           pack_bf16x2(v[6], v[7]));
+          }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&acc_empty[acc]);
+    };
+
+    const int grp_id = lane / P, piece = lane % P;
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+      const int64_t row0 = t * kTileM;
+      for (int sc = 0; sc < nsc; ++sc, ++q) {
+        const int buf = (int)(q & 1);
+        if (q >= 2) mbar_wait(&a_empty[buf], (uint32_t)(((q >> 1) - 1) & 1));
+        for (int j = 0; j < kSuper; ++j) {
+          const int c = sc * kSuper + j;
+          if (c >= p.nkc) break;
+          uint8_t* chunk = sA + (buf * kSuper + j) * kChunkBytesA;
+          if (c < p.nkc_self) {
+            // self rows: 128 rows x P pieces, strided over the gather threads
+            for (int u = threadIdx.x; u < kTileM * P; u += kGatherThreads) {
+              const int r = u / P, pc = u % P;
+              const int64_t row = row0 + r;
+              const int col0 = c * kKC + pc * E;
+              float v[E];
+#pragma unroll
+              for (int k = 0; k < E; ++k) v[k] = 0.f;
+              if (row < p.n_dst && col0 < p.pitch_in) {
+                const int64_t hr = p.gidx ? (int64_t)p.gidx[row] : row;
+                ld_piece<TI>(h + hr * p.ldh + col0, v);
+              }
+              st_swz<E>(chunk, r, pc, v);
+            }
+          } else {
+            const int ca = c - p.nkc_self;
+            const int col0 = ca * kKC + piece * E;
+            const bool colok = col0 < p.pitch_in;
+            for (int r = warp; r < kTileM; r += kGatherWarps) {
+              const int64_t row = row0 + r;
+              float acc[E];
+#pragma unroll
+              for (int k = 0; k < E; ++k) acc[k] = 0.f;
+              int32_t b = 0, e_end = 0;
+              if (row < p.n_dst) { b = __ldg(p.row_ptr + row); e_end = __ldg(p.row_ptr + row + 1); }
+              const int32_t D = e_end - b;
+              if (D > kHeavyT) {
+                // long-tail row: pre-aggregated by k_agg_heavy into the saved h_agg (bf16)
+                if (grp_id == 0 && colok) {
+                  float v[E];
+                  const __nv_bfloat16* src = p.agg + row * p.ld_agg + col0;
+                  if constexpr (E == 8) {
+                    bf16x8_to_f32(*reinterpret_cast<const uint4*>(src), v);
+                  } else {
+                    uint2 w = *reinterpret_cast<const uint2*>(src);
+                    v[0] = __uint_as_float(w.x << 16); v[1] = __uint_as_float(w.x & 0xffff0000u);
+                    v[2] = __uint_as_float(w.y << 16); v[3] = __uint_as_float(w.y & 0xffff0000u);
+                  }
+                  st_swz<E>(chunk, r, piece, v);
+                } else if (grp_id == 0) {
+                  st_swz<E>(chunk, r, piece, acc);
+                }
+                continue;
+              }
+              for (int32_t base = b; base < e_end; base += 32) {
+                const int cnt = min(32, e_end - base);
+                const int32_t jj = lane < cnt ? __ldg(p.col + base + lane) : 0;
+                for (int r0 = 0; r0 < cnt; r0 += G * kUnroll) {
+                  uint4 raw[kUnroll];
+#pragma unroll
+                  for (int uu = 0; uu < kUnroll; ++uu) {
+                    const int tt = r0 + grp_id + G * uu;
+                    const int32_t jn = __shfl_sync(0xffffffffu, jj, tt & 31);
+                    raw[uu] = make_uint4(0u, 0u, 0u, 0u);
+                    if (tt < cnt && colok)
+                      raw[uu] = __ldg(reinterpret_cast<const uint4*>(h + (int64_t)jn * p.ldh + col0));
+                  }
+#pragma unroll
+                  for (int uu = 0; uu < kUnroll; ++uu) {
+                    float v[E];
+                    raw_to_f32<TI>(raw[uu], v);
+#pragma unroll
+                    for (int k = 0; k < E; ++k) acc[k] += v[k];
+                  }
+                }
+              }
+              // combine the G neighbour groups (fixed butterfly order: depends only on D)
+#pragma unroll
+              for (int o = P; o < 32; o <<= 1)
+#pragma unroll
+                for (int k = 0; k < E; ++k) acc[k] += __shfl_xor_sync(0xffffffffu, acc[k], o);
+              if (grp_id == 0) {
+                const float fd = (float)D;
+#pragma unroll
+                for (int k = 0; k < E; ++k) acc[k] = D > 0 ? acc[k] / fd : 0.f;
+                st_swz<E>(chunk, r, piece, acc);
+                if (row < p.n_dst && colok) {
+                  __nv_bfloat16* dstp = p.agg + row * p.ld_agg + col0;
+                  if constexpr (E == 8) {
+                    *reinterpret_cast<uint4*>(dstp) =
+                        make_uint4(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]),
+                                   pack_bf16x2(acc[4], acc[5]), pack_bf16x2(acc[6], acc[7]));
+                  } else {
+                    *reinterpret_cast<uint2*>(dstp) = make_uint2(pack_bf16x2(acc[0], acc[1]),
+                                                                 pack_bf16x2(acc[2], acc[3]));
+                  }
+                }
+              }
+            }
+          }
+        }
+        fence_proxy_async_smem();
+        mbar_arrive(&a_full[buf]);
+      }
+      if (prev_tile >= 0) epilogue(prev_tile, i - 1);
+      prev_tile = t;
+    }
+    if (prev_tile >= 0) epilogue(prev_tile, i - 1);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == kGatherWarps) {
+    tc_fence_after();
+    tmem_dealloc(tmem_base, p.tmem_cols);
+  }
+}
+
+// ------------------------------------------------------------------ weight packing
+// packed chunk c (c < nkc_self: W_self columns c*64.., else W_neigh) = Np rows x 128 B,
+// row n, 16-B piece j stored at piece j ^ (n & 7) (the SWIZZLE_128B image).
+__global__ void k_pack_w_tc(const float* __restrict__ W, int d_in, int d_out, int Np, int nkc_self,
+                            __nv_bfloat16* __restrict__ out) {
+  const int64_t total = (int64_t)2 * nkc_self * Np * kKC;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int kk = (int)(t % kKC);
+    const int n = (int)((t / kKC) % Np);
+    const int c = (int)(t / ((int64_t)kKC * Np));
+    const bool self = c < nkc_self;
+    const int col = (self ? c : c - nkc_self) * kKC + kk;
+    float v = 0.f;
+    if (n < d_out && col < d_in) v = W[(int64_t)n * 2 * d_in + (self ? 0 : d_in) + col];
+    const int piece = kk >> 3, e = kk & 7;
+    const int64_t off = (int64_t)c * Np * kKC + (int64_t)n * kKC + (((piece ^ (n & 7)) << 3) | e);
+    out[off] = __float2bfloat16_rn(v);
+  }
+}
+
 int64_t tc_packed_bytes(int64_t d_in, int64_t d_out) {
   return R(round_up(d_out, 16) * 2 * round_up(d_in, 64) * 2);
 }
-buffalo_status tc_pack_weights(const float*, int, int, void*, cudaStream_t) { return BUFFALO_OK; }
-bool tc_fwd_supported(const FwdArgs&) { return false; }
-buffalo_status tc_sage_fwd(const FwdArgs&, cudaStream_t) { return BUFFALO_ERR_UNSUPPORTED; }
+
+buffalo_status tc_pack_weights(const float* W, int d_in, int d_out, void* packed, cudaStream_t s) {
+  const int Np = (int)round_up(d_out, 16), nkc_self = (int)ceil_div(d_in, kKC);
+  k_pack_w_tc<<<grid_for((int64_t)2 * nkc_self * Np * kKC, 256), 256, 0, s>>>(W, d_in, d_out, Np, nkc_self,
+                                                                            (__nv_bfloat16*)packed);
+  BF_LAUNCHED("k_pack_w_tc");
+  return BUFFALO_OK;
+}
+
+static int smem_bytes_for(int Np) { return 2 * kSuper * kChunkBytesA + 2 * Np * 128 + 256 + 1024; }
+
+bool tc_fwd_supported(const FwdArgs& a) {
+  const int Np = (int)round_up(a.d_out, 16);
+  return a.act_bf16 && Np <= 256 && smem_bytes_for(Np) <= 227 * 1024;
+}
+
+buffalo_status launch_agg_heavy_bf16(const FwdArgs& a, cudaStream_t s);
+
+template <class TI>
+static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
+  const buffalo_block* blk = a.blk;
+  if (blk->n_dst <= 0) return BUFFALO_OK;
+  if (blk->n_heavy > 0) BF_CHECK(launch_agg_heavy_bf16(a, s));
+  TcFwdParams p{};
+  p.row_ptr = blk->row_ptr;
+  p.col = a.layer1 ? blk->col_global : blk->col_local;
+  p.gidx = a.layer1 ? blk->src_global : nullptr;
+  p.n_dst = blk->n_dst;
+  p.h = a.h_src;
+  p.ldh = a.ld_src;
+  p.d_in = a.d_in;
+  p.pitch_in = (int)pitch_of(a.d_in);
+  p.nkc_self = (int)ceil_div(a.d_in, kKC);
+  p.nkc = 2 * p.nkc_self;
+  p.wpk = (const uint8_t*)a.W_packed + R((int64_t)2 * a.d_in * a.d_out * 4);
+  p.Np = (int)round_up(a.d_out, 16);
+  p.d_out = a.d_out;
+  p.ld_out = (int)a.ld_out;
+  int cols = 32;
+  while (cols < 2 * p.Np) cols *= 2;
+  p.tmem_cols = cols;
+  p.bias = a.b;
+  p.relu = a.relu;
+  p.out_f32 = a.out_f32;
+  p.out = a.out;
+  p.agg = (__nv_bfloat16*)a.agg;
+  p.ld_agg = a.ld_agg;
+  const int smem = smem_bytes_for(p.Np);
+  static bool attr_set[2] = {false, false};
+  const int which = sizeof(TI) == 2 ? 0 : 1;
+  if (!attr_set[which]) {
+    BF_CUDA(cudaFuncSetAttribute(k_tc_sage_fwd<TI>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    attr_set[which] = true;
+  }
+  const int64_t ntiles = ceil_div(blk->n_dst, kTileM);
+  const int grid = (int)std::min<int64_t>(ntiles, 148);
+  k_tc_sage_fwd<TI><<<grid, kThreads, smem, s>>>(p);
+  BF_LAUNCHED("k_tc_sage_fwd");
+  return BUFFALO_OK;
+}
+
+buffalo_status tc_sage_fwd(const FwdArgs& a, cudaStream_t s) {
+  if (a.in_bf16) return tc_fwd_t<__nv_bfloat16>(a, s);
+  return tc_fwd_t<float>(a, s);
+}
 
 }  // namespace buffalo

@@ -16,7 +16,15 @@ pytestmark = pytest.mark.gpu
 
 if torch.cuda.is_available():
     from gpu_helpers import (B, act_view, arena_view, assert_bf16_close, assert_close,
-                             blocks_to_numpy, make_trainer)
+                             assert_normwise, blocks_to_numpy, make_trainer)
+
+
+def sp_sum(b, H):
+    """Exact neighbour sums of a block (float64; exact for k/128 inputs)."""
+    import scipy.sparse as sp
+    A = sp.csr_matrix((np.ones(b["n_edges"]), b["col_local"], b["row_ptr"].astype(np.int64)),
+                      shape=(b["n_dst"], b["n_src"]))
+    return A @ np.asarray(H, np.float64)
 
 CASES = {
     # name: (N, pairs, kind, S, fanout, F, dims)
@@ -43,7 +51,7 @@ def test_blocks_bit_exact(name):
     g = O.Graph(rp, col)
     tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs)
     seed = 11
-    tr.group_seeds.copy_(torch.as_tensor(seeds))
+    tr.group_seeds[: seeds.size].copy_(torch.as_tensor(seeds))
     tr._ensure_arena(1 << 16)
     tr.build(0, seeds.size, B.make_sampler(fan, F, seed))
     got = blocks_to_numpy(tr.arena, tr.blocks, len(fan))
@@ -101,7 +109,7 @@ def test_bucketize_budget_error():
 
 
 def _run_microbatch(tr, seeds, fan, F, seed):
-    tr.group_seeds.copy_(torch.as_tensor(seeds))
+    tr.group_seeds[: seeds.size].copy_(torch.as_tensor(seeds))
     tr._ensure_arena(1 << 16)
     tr.loss.zero_()
     tr.params.grad.zero_()
@@ -125,13 +133,17 @@ def test_microbatch_fwd_bwd_parity(name, gemm):
     loss, dlog = O.softmax_ce(logits, y[seeds], S)
     grads = O.sage_backward(blocks, cache, Ws, dlog)
     adt = torch.float32 if mode == B.GEMM_FFMA else torch.bfloat16
-    # layer-1 aggregation of k/128 features: exact in both modes
+    # layer-1 aggregation of k/128 features: the neighbour sums are exact in fp32, so h_agg is
+    # the correctly rounded fp32 quotient (then rounded to bf16 in the bf16 mode), bit for bit
     b1 = tr.blocks.layer[0]
     agg1 = act_view(tr.arena, b1.agg, b1.n_dst, b1.ld_agg, adt)[:, :dims[0]]
-    if mode == B.GEMM_FFMA:
-        np.testing.assert_array_equal(agg1, cache[0]["agg"].astype(np.float32))
-    else:
-        np.testing.assert_array_equal(agg1, torch.as_tensor(cache[0]["agg"]).to(torch.bfloat16).float().numpy())
+    rb = blocks[0]
+    S_exact = sp_sum(rb, X[rb["src_global"]])
+    D = rb["D"].astype(np.float32)[:, None]
+    exp = np.where(D > 0, S_exact.astype(np.float32) / np.maximum(D, 1), np.float32(0))
+    if mode == B.GEMM_BF16:
+        exp = torch.as_tensor(exp).to(torch.bfloat16).float().numpy()
+    np.testing.assert_array_equal(agg1, exp)
     bl = tr.blocks.layer[L - 1]
     glog = act_view(tr.arena, bl.out, bl.n_dst, bl.ld_out, torch.float32)[:, :dims[-1]]
     gW = [w.cpu().numpy() for w in tr.params.dW]
@@ -146,8 +158,8 @@ def test_microbatch_fwd_bwd_parity(name, gemm):
         assert_bf16_close(glog, logits, "logits")
         assert abs(tr.loss.item() - loss) <= 2e-2 * abs(loss)
         for l in range(L):
-            assert_bf16_close(gW[l], grads[l][0], f"dW{l + 1}", rel=5e-2)
-            assert_bf16_close(gb[l], grads[l][1], f"db{l + 1}", rel=5e-2)
+            assert_normwise(gW[l], grads[l][0], 2e-2, f"dW{l + 1}")
+            assert_normwise(gb[l], grads[l][1], 2e-2, f"db{l + 1}")
     # memory model: the measured arena peak lies in [lo, hi] and equals the oracle's model
     lo, hi = O.mem_model(info["n"], info["e"], dims, O.FP32 if mode == B.GEMM_FFMA else O.BF16)
     assert (info["est_lo"], info["est_hi"]) == (lo, hi)
@@ -201,5 +213,5 @@ def test_epoch_parity(gemm):
             assert_close(tr.params.W[l].cpu().numpy(), newW[l], 1e-4, 1e-5, f"W{l + 1}")
             assert_close(tr.params.b[l].cpu().numpy(), newb[l], 1e-4, 1e-5, f"b{l + 1}")
         else:
-            assert_bf16_close(tr.params.W[l].cpu().numpy() - Ws[l], newW[l] - Ws[l], f"dW{l + 1}", rel=5e-2)
+            assert_normwise(tr.params.W[l].cpu().numpy() - Ws[l], newW[l] - Ws[l], 2e-2, f"dW{l + 1}")
     assert float(tr.params.grad.abs().max()) == 0.0       # gradients reset by the step
