@@ -19,7 +19,8 @@ Functions and the passages they follow:
   schedule             Alg. 3 PAPER.md:269-280 + :333 (K loop, K=1 special case)
   build_blocks         Alg. 2 l.5 PAPER.md:237 + §IV-E :388-390 (C); transposes by definition
   sage_forward         Alg. 2 l.8-9 PAPER.md:240-241 (Aggregate = mean, Update = W_l) with
-                       GraphSAGE-mean [16]; R20, R21
+                       GraphSAGE-mean [16]; R20, R21; bf16-storage variant R26
+  round_bf16           IEEE round-to-nearest-even to bfloat16 (R26)
   softmax_ce           Alg. 2 l.10 PAPER.md:242; normalisation by the global batch (R19)
   sage_backward        Alg. 2 l.11-12 PAPER.md:243-244 (gradients accumulated over groups)
   train_epoch          Alg. 2 PAPER.md:233-245 end to end (one optimizer step, R18)
@@ -358,24 +359,37 @@ def mean_adjacency(b):
                          shape=(b["n_dst"], b["n_src"]))
 
 
-def sage_forward(blocks, X, Ws, bs):
+def round_bf16(x):
+    """Round to the nearest bfloat16 (ties to even), returned as float64: keep the top 16 bits
+    of the float32 pattern after adding 0x7FFF + lsb (the IEEE round-to-nearest-even rule)."""
+    f = np.ascontiguousarray(np.asarray(x, dtype=np.float32))
+    u = f.view(np.uint32).astype(np.uint64)
+    u = (u + 0x7FFF + ((u >> 16) & 1)) & 0xFFFF0000
+    return u.astype(np.uint32).view(np.float32).astype(np.float64)
+
+
+def sage_forward(blocks, X, Ws, bs, storage="fp64"):
     """GraphSAGE-mean forward over the micro-batch's blocks in float64 (Alg. 2 l.8-9):
     h_agg = D^-1 A H_{l-1};  Z_l = [H_{l-1}[:n_l] || h_agg] W_l^T + b_l;  H_l = ReLU(Z_l)
     for l < L, logits = Z_L.  X is the global feature table (indexed via src_global of
-    block 1).  Returns (logits, cache) with cache for sage_backward."""
+    block 1).  storage="bf16" (reading R26) rounds what the bf16 mode stores to bfloat16 — the
+    Update operands [H_self || h_agg] and W_l, and H_l — and computes everything else in
+    float64, so that the ReLU decisions are taken on the same rounded values as the kernels.
+    Returns (logits, cache) with cache for sage_backward."""
     L = len(blocks)
+    rnd = round_bf16 if storage == "bf16" else (lambda a: a)
     H = np.asarray(X, dtype=np.float64)[blocks[0]["src_global"]]
     cache = []
     for l in range(1, L + 1):
         b = blocks[l - 1]
-        W = np.asarray(Ws[l - 1], dtype=np.float64)
+        W = rnd(np.asarray(Ws[l - 1], dtype=np.float64))
         d_in = H.shape[1]
         A = mean_adjacency(b)
-        agg = A @ H
-        self_ = H[: b["n_dst"]]
+        agg = rnd(A @ H)
+        self_ = rnd(H[: b["n_dst"]])
         Z = self_ @ W[:, :d_in].T + agg @ W[:, d_in:].T + np.asarray(bs[l - 1], dtype=np.float64)
         cache.append(dict(A=A, H_in=H, agg=agg, Z=Z))
-        H = np.maximum(Z, 0.0) if l < L else Z
+        H = rnd(np.maximum(Z, 0.0)) if l < L else Z
     return H, cache
 
 
@@ -416,16 +430,16 @@ def sage_backward(blocks, cache, Ws, dlogits):
     return grads
 
 
-def microbatch_step(g, seeds_k, X, y, Ws, bs, L, fanout, seed, S):
+def microbatch_step(g, seeds_k, X, y, Ws, bs, L, fanout, seed, S, storage="fp64"):
     """One micro-batch of Alg. 2 (l.4-12): blocks, forward, partial loss, gradients."""
     blocks = build_blocks(g, seeds_k, L, fanout, seed)
-    logits, cache = sage_forward(blocks, X, Ws, bs)
+    logits, cache = sage_forward(blocks, X, Ws, bs, storage)
     loss, dlog = softmax_ce(logits, y[np.asarray(seeds_k)], S)
     grads = sage_backward(blocks, cache, Ws, dlog)
     return loss, grads, blocks
 
 
-def train_epoch(g, seeds, X, y, Ws, bs, L, fanout, F, seed, dims, lr=0.0, **sched_kw):
+def train_epoch(g, seeds, X, y, Ws, bs, L, fanout, F, seed, dims, lr=0.0, storage="fp64", **sched_kw):
     """Alg. 2: schedule, then every group's forward/backward with the
     partial gradients accumulated, then ONE optimizer step (SGD with rate lr, R18)."""
     plan = schedule(g, seeds, L, fanout, F, seed, dims, **sched_kw)
@@ -437,7 +451,7 @@ def train_epoch(g, seeds, X, y, Ws, bs, L, fanout, F, seed, dims, lr=0.0, **sche
     off = plan["group_offsets"]
     for k in range(plan["K"]):
         sk = plan["group_seeds"][off[k]:off[k + 1]]
-        loss, grads, _ = microbatch_step(g, sk, X, y, Ws, bs, L, fanout, seed, S)
+        loss, grads, _ = microbatch_step(g, sk, X, y, Ws, bs, L, fanout, seed, S, storage)
         total += loss
         acc = [(a + gw, b + gb) for (a, b), (gw, gb) in zip(acc, grads)]
     newW = [np.asarray(W, np.float64) - lr * gW for W, (gW, _) in zip(Ws, acc)]

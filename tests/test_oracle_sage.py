@@ -143,3 +143,22 @@ def test_train_epoch_runs_and_updates():
                                                 lr=0.1, k_min=3, k_max=3)
     assert plan["K"] == 3 and loss > 0
     np.testing.assert_allclose(newW[0], Ws[0] - 0.1 * acc[0][0], rtol=1e-12)
+
+
+def test_round_bf16_matches_torch_and_ties_to_even():
+    rng = np.random.default_rng(3)
+    x = np.concatenate([rng.standard_normal(10000) * 10.0 ** rng.integers(-8, 8, 10000),
+                        np.array([1.0 + 2.0 ** -8, 1.0 + 3 * 2.0 ** -8, -1.0 - 2.0 ** -8, 0.0, -0.0])])
+    ref = torch.as_tensor(x.astype(np.float32)).to(torch.bfloat16).double().numpy()
+    np.testing.assert_array_equal(O.round_bf16(x), ref)
+    # halfway cases go to the even mantissa
+    assert O.round_bf16(1.0 + 2.0 ** -8) == 1.0 and O.round_bf16(1.0 + 3 * 2.0 ** -8) == 1.0 + 2.0 ** -6
+
+
+def test_bf16_storage_forward_close_to_fp64():
+    g, X, y, seeds, fan, dims, Ws, bs = _setup()
+    blocks = O.build_blocks(g, seeds, 2, fan, 3)
+    a, _ = O.sage_forward(blocks, X, Ws, bs)
+    b, _ = O.sage_forward(blocks, X, Ws, bs, storage="bf16")
+    assert np.linalg.norm(a - b) <= 2e-2 * np.linalg.norm(a)
+    assert not np.array_equal(a, b)
