@@ -195,6 +195,13 @@ def dw_splits(n_l, d_out, d_in):
     return max(1, min(_ceil(296, tiles), _ceil(n_l, 512)))
 
 
+def tc_dw_splits(n_l, d_out, d_in):
+    """Split count of the tensor-core dW reduction (tiles of 128 x 256 over [d_out, 2 Dp])."""
+    Dp = _ceil(d_in, 64) * 64
+    tiles = _ceil(d_out, 128) * _ceil(2 * Dp, 256)
+    return max(1, min(_ceil(296, tiles), _ceil(max(int(n_l), 1), 512)))
+
+
 def _part_count_elems(e):
     return 256 * _ceil(max(int(e), 1), PART_TILE)
 
@@ -236,9 +243,18 @@ def mem_model(n, e, dims, act_dtype=FP32):
         frame = _R(n[l] * pitch(dims[l]) * 4)                   # dH_l (dlogits at l = L)
         if l >= 2:
             frame += _R(n[l - 1] * pitch(dims[l - 1]) * 4)      # dH_{l-1}
-            frame += _R(n[l - 1] * pitch(dims[l]) * 4)          # transposed aggregate of dZ/D
-        S = dw_splits(n[l], dims[l], dims[l - 1])
-        frame += _R(S * dims[l] * 2 * dims[l - 1] * 4) + _R(S * pitch(dims[l]) * 4)  # dW, db partials
+        if act_dtype == FP32:
+            if l >= 2:
+                frame += _R(n[l - 1] * pitch(dims[l]) * 4)      # transposed aggregate of dZ/D
+            S = dw_splits(n[l], dims[l], dims[l - 1])
+            frame += _R(S * dims[l] * 2 * dims[l - 1] * 4) + _R(S * pitch(dims[l]) * 4)  # dW, db partials
+        else:
+            frame += _R(n[l] * pitch(dims[l]) * 2)              # dZ in bf16
+            if l >= 2:
+                frame += _R(n[l] * pitch(dims[l]) * 2)          # dZ / D in bf16
+            S = tc_dw_splits(n[l], dims[l], dims[l - 1])
+            Dp = _ceil(dims[l - 1], 64) * 64
+            frame += _R(S * dims[l] * 2 * Dp * 4) + _R(S * pitch(dims[l]) * 4)          # dW, db partials
         bwd = max(bwd, frame)
     lo = blocks + acts + bwd
     hi = blocks + acts + max(bwd, build)

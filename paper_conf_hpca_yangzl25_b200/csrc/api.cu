@@ -58,6 +58,11 @@ __global__ void k_fill_i32(int32_t* a, int64_t n, int32_t v) {
 
 // ------------------------------------------------------------------ memory model (R15)
 // Restated from DESIGN.md §5; must agree with the arena that buffalo_build_blocks lays out.
+static int64_t bwd_scratch_for(const buffalo_model* m, int64_t n_dst, int64_t n_src, int l) {
+  if (m->gemm_mode == BUFFALO_GEMM_BF16) return tc_bwd_scratch_bytes(n_dst, n_src, l, m->dim[l - 1], m->dim[l]);
+  return bwd_scratch_bytes(n_dst, n_src, l, m->dim[l - 1], m->dim[l]);
+}
+
 static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_model* m,
                       int64_t* lo, int64_t* hi) {
   const int64_t s = m->gemm_mode == BUFFALO_GEMM_BF16 ? 2 : 4;
@@ -76,7 +81,7 @@ static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_m
   for (int l = L; l >= 1; --l) {
     int64_t f = R(n[l] * pitch_of(m->dim[l]) * 4);
     if (l >= 2) f += R(n[l - 1] * pitch_of(m->dim[l - 1]) * 4);
-    f += bwd_scratch_bytes(n[l], n[l - 1], l, m->dim[l - 1], m->dim[l]);
+    f += bwd_scratch_for(m, n[l], n[l - 1], l);
     bwd = std::max(bwd, f);
   }
   *lo = blocks + acts + bwd;
@@ -95,6 +100,12 @@ static buffalo_status validate_model(const buffalo_model* m) {
     }
   if (m->feat_dtype != BUFFALO_FP32 && m->feat_dtype != BUFFALO_BF16) return BUFFALO_ERR_INVALID_ARG;
   if (m->gemm_mode != BUFFALO_GEMM_FFMA && m->gemm_mode != BUFFALO_GEMM_BF16) return BUFFALO_ERR_INVALID_ARG;
+  if (m->gemm_mode == BUFFALO_GEMM_BF16)
+    for (int l = 1; l <= m->num_layers; ++l)
+      if (m->dim[l] > 256) {
+        set_error("model: the bf16 tensor-core path supports dim[l] <= 256 for l >= 1");
+        return BUFFALO_ERR_UNSUPPORTED;
+      }
   if (m->feat_pitch < round_up(m->dim[0], 8) || m->feat_pitch % 8) {
     set_error("model: feat_pitch must be a multiple of 8 and >= round_up(dim[0], 8)");
     return BUFFALO_ERR_INVALID_ARG;
@@ -475,7 +486,7 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
   std::vector<int64_t> ah(L + 1, 0), tmp(L + 1, 0);
   for (int l = 1; l <= L; ++l) ah[l] = R(nn[l] * pitch_of(m->dim[l]) * 4);
   for (int l = L; l >= 1; --l) {
-    tmp[l] = bwd_scratch_bytes(nn[l], nn[l - 1], l, m->dim[l - 1], m->dim[l]);
+    tmp[l] = bwd_scratch_for(m, nn[l], nn[l - 1], l);
     B = std::max(B, ah[l] + (l >= 2 ? ah[l - 1] : 0) + tmp[l]);
   }
   char* region = (char*)A.take(B);
@@ -562,7 +573,7 @@ buffalo_status buffalo_sage_fwd(const buffalo_block* blk, int32_t layer, const b
 
 size_t buffalo_sage_bwd_scratch_bytes(const buffalo_block* blk, int32_t layer, const buffalo_model* m) {
   if (!blk || !m || layer < 1 || layer > m->num_layers) return 0;
-  return (size_t)bwd_scratch_bytes(blk->n_dst, blk->n_src, layer, m->dim[layer - 1], m->dim[layer]);
+  return (size_t)bwd_scratch_for(m, blk->n_dst, blk->n_src, layer);
 }
 
 buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
@@ -610,6 +621,10 @@ buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const b
   a.scratch = scratch;
   a.scratch_bytes = (int64_t)scratch_bytes;
   cudaStream_t s = (cudaStream_t)stream;
+  if (m->gemm_mode == BUFFALO_GEMM_BF16) {
+    if (!tc_bwd_supported(a)) return BUFFALO_ERR_UNSUPPORTED;
+    return tc_sage_bwd(a, s);
+  }
   return sage_bwd_ffma(a, s);
 }
 

@@ -315,7 +315,8 @@ __global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, in
                                                     const TS* __restrict__ self, int64_t lds,
                                                     const int32_t* __restrict__ gidx,
                                                     const TG* __restrict__ agg, int64_t ldg,
-                                                    int64_t rows_per_split, float* __restrict__ part) {
+                                                    int64_t rows_per_split, float* __restrict__ part,
+                                                    float* __restrict__ db_part) {
   __shared__ float Zs[16][64];
   __shared__ float As[16][64];
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
@@ -324,6 +325,8 @@ __global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, in
   const int64_t r_end = min(nrows, r_beg + rows_per_split);
   const int K = 2 * d_in;
   float acc[4][4] = {};
+  float dbs[4] = {0.f, 0.f, 0.f, 0.f};      // column sums of dZ (CTAs of k-tile 0, threads ty == 0)
+  const bool do_db = blockIdx.x == 0 && ty == 0;
   const int lr = tid >> 4, lc = (tid & 15) * 4;
   for (int64_t r0 = r_beg; r0 < r_end; r0 += 16) {
     const int64_t r = r0 + lr;
@@ -344,6 +347,10 @@ __global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, in
       As[lr][lc + q] = a;
     }
     __syncthreads();
+    if (do_db)
+      for (int rr = 0; rr < 16; ++rr)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) dbs[j] += Zs[rr][tx * 4 + j];
 #pragma unroll
     for (int rr = 0; rr < 16; ++rr) {
       float zz[4], aa[4];
@@ -358,6 +365,10 @@ __global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, in
     }
     __syncthreads();
   }
+  if (do_db)
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      if (n0 + tx * 4 + j < d_out) db_part[(int64_t)blockIdx.z * d_out + n0 + tx * 4 + j] = dbs[j];
   float* P = part + (int64_t)blockIdx.z * d_out * K;
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
@@ -368,17 +379,6 @@ __global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, in
       const int k = k0 + tx * 4 + j;
       if (k < K) P[(int64_t)nn * K + k] = acc[i][j];
     }
-  }
-}
-
-__global__ void k_colsum_partial(int64_t nrows, int d, const float* __restrict__ dz, int64_t ldz,
-                                 int64_t rows_per_split, float* __restrict__ part) {
-  const int64_t r_beg = (int64_t)blockIdx.x * rows_per_split;
-  const int64_t r_end = min(nrows, r_beg + rows_per_split);
-  for (int c = threadIdx.x; c < d; c += blockDim.x) {
-    float s = 0.f;
-    for (int64_t r = r_beg; r < r_end; ++r) s += dz[r * ldz + c];
-    part[(int64_t)blockIdx.x * d + c] = s;
   }
 }
 
@@ -553,10 +553,8 @@ static buffalo_status bwd_ffma_t(const BwdArgs& a, cudaStream_t s) {
     dim3 g((unsigned)ceil_div(2 * d_in, 64), (unsigned)ceil_div(d_out, 64), (unsigned)S);
     k_dw_partial<TS, TG><<<g, 256, 0, s>>>(n, d_out, d_in, a.dh, a.ld_dh, (const TS*)a.h_src, a.ld_src,
                                            a.layer1 ? blk->src_global : nullptr, (const TG*)a.agg,
-                                           a.ld_agg, rps, dw_part);
+                                           a.ld_agg, rps, dw_part, db_part);
     BF_LAUNCHED("k_dw_partial");
-    k_colsum_partial<<<S, 256, 0, s>>>(n, d_out, a.dh, a.ld_dh, rps, db_part);
-    BF_LAUNCHED("k_colsum_partial");
     k_reduce_partials<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, (int64_t)d_out * 2 * d_in, a.dW);
     BF_LAUNCHED("k_reduce_partials");
     k_reduce_partials<<<1, 256, 0, s>>>(db_part, S, d_out, a.db);

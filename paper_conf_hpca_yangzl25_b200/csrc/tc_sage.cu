@@ -137,9 +137,12 @@ struct TcFwdParams {
   const int32_t* row_ptr;
   const int32_t* col;        // neighbour row ids into h (global for layer 1, local otherwise)
   const int32_t* gidx;       // self row ids (layer 1: src_global) or null (= i)
-  int64_t n_dst;
-  const void* h;             // bf16 or fp32 rows
+  int64_t n_dst;             // output rows (fwd: dst of the block; bwd: src of the block)
+  int64_t self_rows;         // rows >= self_rows have a zero self half (bwd: n_dst of the block)
+  const void* h;             // neighbour rows, bf16 or fp32
   int64_t ldh;               // elements
+  const void* hs;            // self rows (fwd: = h)
+  int64_t lds;
   int d_in, pitch_in;        // pitch_in: valid columns readable in a row (multiple of 8)
   int nkc_self, nkc;         // K-chunks for the self half, total (= 2 nkc_self)
   const uint8_t* wpk;        // pre-swizzled bf16 W chunks, each Np x 128 B
@@ -191,7 +194,10 @@ template <> __device__ __forceinline__ void raw_to_f32<float>(const uint4& u, fl
   v[0] = __uint_as_float(u.x); v[1] = __uint_as_float(u.y); v[2] = __uint_as_float(u.z); v[3] = __uint_as_float(u.w);
 }
 
-template <class TI>
+// MODE 0: forward (mean of neighbour rows, long-tail rows pre-aggregated, h_agg saved,
+//         + bias, ReLU).  MODE 1: backward dH (plain sum of pre-scaled dZ/D rows over the
+//         transposed block, self half = dZ for rows < self_rows, fp32 output).
+template <class TI, int MODE>
 __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p) {
   constexpr int E = InTraits<TI>::kElems;      // elements per 16-B piece
   constexpr int P = kKC / E;                   // pieces per 64-column chunk row (8 or 16)
@@ -286,6 +292,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
   } else {
     // ===================== gather + epilogue warps
     const TI* __restrict__ h = (const TI*)p.h;
+    const TI* __restrict__ hs = (const TI*)p.hs;
     int64_t q = 0, i = 0;
     int64_t prev_tile = -1;
     auto epilogue = [&](int64_t tile, int64_t li) {
@@ -303,7 +310,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
 #pragma unroll
           for (int k = 0; k < 8; ++k) {
             const int cidx = grp * 8 + k;
-            float x = v[k] + (cidx < p.d_out ? __ldg(p.bias + cidx) : 0.f);
+            float x = v[k] + ((p.bias && cidx < p.d_out) ? __ldg(p.bias + cidx) : 0.f);
             v[k] = p.relu ? fmaxf(x, 0.f) : x;
           }
           if (p.out_f32) {
@@ -340,9 +347,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
               float v[E];
 #pragma unroll
               for (int k = 0; k < E; ++k) v[k] = 0.f;
-              if (row < p.n_dst && col0 < p.pitch_in) {
+              if (row < p.self_rows && col0 < p.pitch_in) {
                 const int64_t hr = p.gidx ? (int64_t)p.gidx[row] : row;
-                ld_piece<TI>(h + hr * p.ldh + col0, v);
+                ld_piece<TI>(hs + hr * p.lds + col0, v);
               }
               st_swz<E>(chunk, r, pc, v);
             }
@@ -358,7 +365,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
               int32_t b = 0, e_end = 0;
               if (row < p.n_dst) { b = __ldg(p.row_ptr + row); e_end = __ldg(p.row_ptr + row + 1); }
               const int32_t D = e_end - b;
-              if (D > kHeavyT) {
+              if (MODE == 0 && D > kHeavyT) {
                 // long-tail row: pre-aggregated by k_agg_heavy into the saved h_agg (bf16)
                 if (grp_id == 0 && colok) {
                   float v[E];
@@ -404,11 +411,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
 #pragma unroll
                 for (int k = 0; k < E; ++k) acc[k] += __shfl_xor_sync(0xffffffffu, acc[k], o);
               if (grp_id == 0) {
-                const float fd = (float)D;
+                if (MODE == 0) {
+                  const float fd = (float)D;
 #pragma unroll
-                for (int k = 0; k < E; ++k) acc[k] = D > 0 ? acc[k] / fd : 0.f;
+                  for (int k = 0; k < E; ++k) acc[k] = D > 0 ? acc[k] / fd : 0.f;
+                }
                 st_swz<E>(chunk, r, piece, acc);
-                if (row < p.n_dst && colok) {
+                if (MODE == 0 && row < p.n_dst && colok) {
                   __nv_bfloat16* dstp = p.agg + row * p.ld_agg + col0;
                   if constexpr (E == 8) {
                     *reinterpret_cast<uint4*>(dstp) =
@@ -459,8 +468,30 @@ __global__ void k_pack_w_tc(const float* __restrict__ W, int d_in, int d_out, in
   }
 }
 
-int64_t tc_packed_bytes(int64_t d_in, int64_t d_out) {
+int64_t tc_fwd_packed_bytes(int64_t d_in, int64_t d_out) {
   return R(round_up(d_out, 16) * 2 * round_up(d_in, 64) * 2);
+}
+int64_t tc_packed_bytes(int64_t d_in, int64_t d_out) {
+  return tc_fwd_packed_bytes(d_in, d_out) + tc_fwd_packed_bytes(d_out, d_in);
+}
+
+// Backward image: B[n][k] over n < d_in (output columns of dH), k in [0, 2 Kp):
+// k < Kp -> W[k][n] (W_self^T), k >= Kp -> W[k - Kp][d_in + n] (W_neigh^T).
+__global__ void k_pack_wt_tc(const float* __restrict__ W, int d_in, int d_out, int Np, int nkc_self,
+                             __nv_bfloat16* __restrict__ out) {
+  const int64_t total = (int64_t)2 * nkc_self * Np * kKC;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int kk = (int)(t % kKC);
+    const int n = (int)((t / kKC) % Np);
+    const int c = (int)(t / ((int64_t)kKC * Np));
+    const bool self = c < nkc_self;
+    const int k = (self ? c : c - nkc_self) * kKC + kk;
+    float v = 0.f;
+    if (n < d_in && k < d_out) v = W[(int64_t)k * 2 * d_in + (self ? 0 : d_in) + n];
+    const int piece = kk >> 3, e = kk & 7;
+    const int64_t off = (int64_t)c * Np * kKC + (int64_t)n * kKC + (((piece ^ (n & 7)) << 3) | e);
+    out[off] = __float2bfloat16_rn(v);
+  }
 }
 
 buffalo_status tc_pack_weights(const float* W, int d_in, int d_out, void* packed, cudaStream_t s) {
@@ -468,6 +499,10 @@ buffalo_status tc_pack_weights(const float* W, int d_in, int d_out, void* packed
   k_pack_w_tc<<<grid_for((int64_t)2 * nkc_self * Np * kKC, 256), 256, 0, s>>>(W, d_in, d_out, Np, nkc_self,
                                                                             (__nv_bfloat16*)packed);
   BF_LAUNCHED("k_pack_w_tc");
+  const int Npb = (int)round_up(d_in, 16), nkb = (int)ceil_div(d_out, kKC);
+  __nv_bfloat16* pb = (__nv_bfloat16*)((char*)packed + tc_fwd_packed_bytes(d_in, d_out));
+  k_pack_wt_tc<<<grid_for((int64_t)2 * nkb * Npb * kKC, 256), 256, 0, s>>>(W, d_in, d_out, Npb, nkb, pb);
+  BF_LAUNCHED("k_pack_wt_tc");
   return BUFFALO_OK;
 }
 
@@ -480,6 +515,27 @@ bool tc_fwd_supported(const FwdArgs& a) {
 
 buffalo_status launch_agg_heavy_bf16(const FwdArgs& a, cudaStream_t s);
 
+template <class TI, int MODE>
+static buffalo_status launch_tc(const TcFwdParams& p, cudaStream_t s) {
+  const int smem = smem_bytes_for(p.Np);
+  static bool attr_set = false;
+  if (!attr_set) {
+    BF_CUDA(cudaFuncSetAttribute(k_tc_sage_fwd<TI, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    attr_set = true;
+  }
+  const int64_t ntiles = ceil_div(p.n_dst, kTileM);
+  const int grid = (int)std::min<int64_t>(ntiles, 148);
+  k_tc_sage_fwd<TI, MODE><<<grid, kThreads, smem, s>>>(p);
+  BF_LAUNCHED(MODE == 0 ? "k_tc_sage_fwd" : "k_tc_sage_bwd_dh");
+  return BUFFALO_OK;
+}
+
+static int tmem_cols_for(int Np) {
+  int cols = 32;
+  while (cols < 2 * Np) cols *= 2;
+  return cols;
+}
+
 template <class TI>
 static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   const buffalo_block* blk = a.blk;
@@ -490,8 +546,11 @@ static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   p.col = a.layer1 ? blk->col_global : blk->col_local;
   p.gidx = a.layer1 ? blk->src_global : nullptr;
   p.n_dst = blk->n_dst;
+  p.self_rows = blk->n_dst;
   p.h = a.h_src;
   p.ldh = a.ld_src;
+  p.hs = a.h_src;
+  p.lds = a.ld_src;
   p.d_in = a.d_in;
   p.pitch_in = (int)pitch_of(a.d_in);
   p.nkc_self = (int)ceil_div(a.d_in, kKC);
@@ -500,32 +559,335 @@ static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   p.Np = (int)round_up(a.d_out, 16);
   p.d_out = a.d_out;
   p.ld_out = (int)a.ld_out;
-  int cols = 32;
-  while (cols < 2 * p.Np) cols *= 2;
-  p.tmem_cols = cols;
+  p.tmem_cols = tmem_cols_for(p.Np);
   p.bias = a.b;
   p.relu = a.relu;
   p.out_f32 = a.out_f32;
   p.out = a.out;
   p.agg = (__nv_bfloat16*)a.agg;
   p.ld_agg = a.ld_agg;
-  const int smem = smem_bytes_for(p.Np);
-  static bool attr_set[2] = {false, false};
-  const int which = sizeof(TI) == 2 ? 0 : 1;
-  if (!attr_set[which]) {
-    BF_CUDA(cudaFuncSetAttribute(k_tc_sage_fwd<TI>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
-    attr_set[which] = true;
-  }
-  const int64_t ntiles = ceil_div(blk->n_dst, kTileM);
-  const int grid = (int)std::min<int64_t>(ntiles, 148);
-  k_tc_sage_fwd<TI><<<grid, kThreads, smem, s>>>(p);
-  BF_LAUNCHED("k_tc_sage_fwd");
-  return BUFFALO_OK;
+  return launch_tc<TI, 0>(p, s);
 }
 
 buffalo_status tc_sage_fwd(const FwdArgs& a, cudaStream_t s) {
   if (a.in_bf16) return tc_fwd_t<__nv_bfloat16>(a, s);
   return tc_fwd_t<float>(a, s);
+}
+
+// ================================================================== backward
+// dZ preparation: dZ = dH * 1[H > 0] in place (l < L); bf16 copies dZ and dZ / D(i).
+template <class TH>
+__global__ void k_dz_prep(float* __restrict__ dz, int64_t ldz, const TH* __restrict__ h, int64_t ldh,
+                          const int32_t* __restrict__ rp, int64_t n, int d, int dp,
+                          __nv_bfloat16* __restrict__ zb, __nv_bfloat16* __restrict__ zs) {
+  const int per_row = dp / 8;
+  const int64_t total = n * per_row;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = t / per_row;
+    const int c0 = (int)(t - i * per_row) * 8;
+    float v[8];
+    const float4 a0 = *reinterpret_cast<const float4*>(dz + i * ldz + c0);
+    const float4 a1 = *reinterpret_cast<const float4*>(dz + i * ldz + c0 + 4);
+    v[0] = a0.x; v[1] = a0.y; v[2] = a0.z; v[3] = a0.w; v[4] = a1.x; v[5] = a1.y; v[6] = a1.z; v[7] = a1.w;
+    if (h) {
+      const uint4 hr = *reinterpret_cast<const uint4*>(reinterpret_cast<const __nv_bfloat16*>(h) + i * ldh + c0);
+      float hv[8];
+      bf16x8_to_f32(hr, hv);
+      bool ch = false;
+#pragma unroll
+      for (int k = 0; k < 8; ++k)
+        if (!(hv[k] > 0.f) && v[k] != 0.f) { v[k] = 0.f; ch = true; }
+      if (ch) {
+        *reinterpret_cast<float4*>(dz + i * ldz + c0) = make_float4(v[0], v[1], v[2], v[3]);
+        *reinterpret_cast<float4*>(dz + i * ldz + c0 + 4) = make_float4(v[4], v[5], v[6], v[7]);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (c0 + k >= d) v[k] = 0.f;
+    *reinterpret_cast<uint4*>(zb + i * dp + c0) = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
+                                                              pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
+    if (zs) {
+      const float fd = (float)(rp[i + 1] - rp[i]);
+#pragma unroll
+      for (int k = 0; k < 8; ++k) v[k] = v[k] / fd;
+      *reinterpret_cast<uint4*>(zs + i * dp + c0) = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
+                                                                pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
+    }
+  }
+}
+
+// dW (tensor cores): D[m][n'] = sum_r dZ[r][m] * Afwd[r][n'] over a row range, both operands
+// MN-major in shared memory (the reduction runs over rows, the slow dimension of both).
+// Afwd columns are padded per half: n' < Dp -> self column n', n' >= Dp -> h_agg column n' - Dp.
+constexpr int kDwThreads = 128;
+constexpr int kDwRows = 64;                       // K per stage
+constexpr int kDwStrip = kDwRows * 128;           // one 64-column MN strip of 64 rows (8 KB)
+constexpr int kDwStages = 2;
+
+struct TcDwParams {
+  const __nv_bfloat16* zb;  int64_t ldz;          // dZ (bf16) [n][ldz]
+  const void* self_; int64_t lds; const int32_t* gidx;  // self rows (feature table for layer 1)
+  const __nv_bfloat16* agg; int64_t lda;          // saved h_agg
+  int64_t n;
+  int d_out, d_in, pitch_in, pz, Dp, NT;          // NT: n' columns per CTA tile (<= 256)
+  int64_t rows_per_split;
+  float* part;                                    // [S][d_out][2 Dp]
+  const float* dz; int64_t lddz;                  // fp32 dZ (for db)
+  float* db_part;                                 // [S][d_out] column sums (CTAs with n-tile 0)
+};
+
+// MN-major SWIZZLE_128B descriptor: LBO = stride between 64-element MN strips, SBO = 8 K-rows.
+__device__ __forceinline__ uint64_t sw128_mn_desc(uint32_t saddr, uint32_t lbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
+  d |= (uint64_t)(1024 >> 4) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)2 << 61;
+  return d;
+}
+__host__ __device__ constexpr uint32_t idesc_bf16_mn(int n) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | (1u << 15) | (1u << 16) | ((uint32_t)(n >> 3) << 17) |
+         ((uint32_t)(128 >> 4) << 24);
+}
+
+template <class TS>
+__global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int nstripA = 2, nstripB = p.NT / 64;
+  const int stage_bytes = (nstripA + nstripB) * kDwStrip;
+  uint64_t* full = (uint64_t*)(smem + kDwStages * stage_bytes);
+  uint64_t* empty = full + kDwStages;
+  uint64_t* done = empty + kDwStages;
+  uint32_t* tmem_slot = (uint32_t*)(done + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int m0 = blockIdx.x * 128, n0 = blockIdx.y * p.NT;
+  const int64_t r_beg = (int64_t)blockIdx.z * p.rows_per_split;
+  const int64_t r_end = min(p.n, r_beg + p.rows_per_split);
+  const int nchunks = r_end > r_beg ? (int)((r_end - r_beg + kDwRows - 1) / kDwRows) : 0;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kDwStages; ++i) { mbar_init(&full[i], kDwThreads); mbar_init(&empty[i], 1); }
+    mbar_init(done, 1);
+    fence_barrier_init();
+  }
+  if (warp == 0) tmem_alloc(tmem_slot, p.NT);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const TS* __restrict__ selfp = (const TS*)p.self_;
+  const uint32_t idesc = idesc_bf16_mn(p.NT);
+  // db: CTAs of n-tile 0 also sum their row range of fp32 dZ column by column (thread = column)
+  const bool do_db = blockIdx.y == 0;
+  const int mcol = m0 + threadIdx.x;
+  float dbs = 0.f;
+  for (int c = 0; c < nchunks; ++c) {
+    const int st = c % kDwStages;
+    if (c >= kDwStages) mbar_wait(&empty[st], (uint32_t)(((c / kDwStages) - 1) & 1));
+    uint8_t* sa = smem + st * stage_bytes;
+    uint8_t* sb = sa + nstripA * kDwStrip;
+    const int64_t rbase = r_beg + (int64_t)c * kDwRows;
+    // A: dZ rows, 128 m-columns = 2 strips x 8 pieces of 16 B per row
+    for (int u = threadIdx.x; u < kDwRows * 16; u += kDwThreads) {
+      const int k = u >> 4, j = u & 15;
+      const int64_t r = rbase + k;
+      const int m = m0 + j * 8;
+      uint4 v = make_uint4(0u, 0u, 0u, 0u);
+      if (r < r_end && m < p.pz) v = *reinterpret_cast<const uint4*>(p.zb + r * p.ldz + m);
+      *reinterpret_cast<uint4*>(sa + (j >> 3) * kDwStrip + k * 128 + (((j & 7) ^ (k & 7)) << 4)) = v;
+    }
+    // B: Afwd rows, NT n'-columns
+    const int pcs = p.NT / 8;
+    for (int u = threadIdx.x; u < kDwRows * pcs; u += kDwThreads) {
+      const int k = u / pcs, j = u % pcs;
+      const int64_t r = rbase + k;
+      const int nn = n0 + j * 8;
+      uint4 v = make_uint4(0u, 0u, 0u, 0u);
+      if (r < r_end) {
+        if (nn < p.Dp) {
+          if (nn < p.pitch_in) {
+            const int64_t rr = p.gidx ? (int64_t)p.gidx[r] : r;
+            if constexpr (sizeof(TS) == 2) {
+              v = *reinterpret_cast<const uint4*>(selfp + rr * p.lds + nn);
+            } else {
+              const float4 a0 = *reinterpret_cast<const float4*>(selfp + rr * p.lds + nn);
+              const float4 a1 = *reinterpret_cast<const float4*>(selfp + rr * p.lds + nn + 4);
+              v = make_uint4(pack_bf16x2(a0.x, a0.y), pack_bf16x2(a0.z, a0.w), pack_bf16x2(a1.x, a1.y),
+                             pack_bf16x2(a1.z, a1.w));
+            }
+          }
+        } else if (nn - p.Dp < p.pitch_in) {
+          v = *reinterpret_cast<const uint4*>(p.agg + r * p.lda + (nn - p.Dp));
+        }
+      }
+      *reinterpret_cast<uint4*>(sb + (j >> 3) * kDwStrip + k * 128 + (((j & 7) ^ (k & 7)) << 4)) = v;
+    }
+    fence_proxy_async_smem();
+    mbar_arrive(&full[st]);
+    if (do_db && mcol < p.d_out) {
+      const int64_t r1 = min(r_end, rbase + kDwRows);
+      for (int64_t r = rbase; r < r1; ++r) dbs += p.dz[r * p.lddz + mcol];
+    }
+    if (threadIdx.x == 0) {
+      mbar_wait(&full[st], (uint32_t)((c / kDwStages) & 1));
+      tc_fence_after();
+      const uint32_t a_addr = smem_u32(sa), b_addr = smem_u32(sb);
+#pragma unroll
+      for (int kk = 0; kk < kDwRows / 16; ++kk)
+        umma_bf16(tmem, sw128_mn_desc(a_addr + kk * 2048, kDwStrip), sw128_mn_desc(b_addr + kk * 2048, kDwStrip),
+                  idesc, (c > 0 || kk > 0) ? 1u : 0u);
+      umma_commit(&empty[st]);
+      if (c == nchunks - 1) umma_commit(done);
+    }
+    __syncwarp();
+  }
+  if (do_db && mcol < p.d_out) p.db_part[(int64_t)blockIdx.z * p.d_out + mcol] = dbs;
+  // epilogue: TMEM lanes = m rows, columns = n'
+  const int64_t K2 = 2 * (int64_t)p.Dp;
+  float* P = p.part + (int64_t)blockIdx.z * p.d_out * K2;
+  const int m = m0 + warp * 32 + lane;
+  if (nchunks > 0) {
+    mbar_wait(done, 0);
+    tc_fence_after();
+  }
+  for (int g = 0; g < p.NT / 8; ++g) {
+    float v[8];
+    if (nchunks > 0) {
+      tmem_ld8(tmem + ((uint32_t)(warp * 32) << 16) + g * 8, v);
+    } else {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) v[k] = 0.f;
+    }
+    const int nn = n0 + g * 8;
+    if (m < p.d_out && nn < K2) {
+      float4* o = reinterpret_cast<float4*>(P + (int64_t)m * K2 + nn);
+      o[0] = make_float4(v[0], v[1], v[2], v[3]);
+      o[1] = make_float4(v[4], v[5], v[6], v[7]);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    tmem_dealloc(tmem, p.NT);
+  }
+}
+
+// dW[m][n] += sum_s part[s][m][n'(n)] in split order (deterministic).
+__global__ void k_reduce_dw(const float* __restrict__ part, int S, int d_out, int d_in, int Dp,
+                            float* __restrict__ dW) {
+  const int64_t total = (int64_t)d_out * 2 * d_in;
+  const int64_t K2 = 2 * (int64_t)Dp;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int m = (int)(t / (2 * d_in)), n = (int)(t % (2 * d_in));
+    const int np = n < d_in ? n : Dp + (n - d_in);
+    float acc = 0.f;
+    for (int q = 0; q < S; ++q) acc += part[(int64_t)q * d_out * K2 + (int64_t)m * K2 + np];
+    dW[t] += acc;
+  }
+}
+
+__global__ void k_reduce_db(const float* __restrict__ part, int S, int d, float* __restrict__ db) {
+  for (int c = threadIdx.x; c < d; c += blockDim.x) {
+    float s = 0.f;
+    for (int q = 0; q < S; ++q) s += part[(int64_t)q * d + c];
+    db[c] += s;
+  }
+}
+
+int tc_dw_splits(int64_t n, int d_out, int d_in) {
+  const int64_t Dp = round_up(d_in, 64);
+  const int64_t tiles = ceil_div(d_out, 128) * ceil_div(2 * Dp, 256);
+  int64_t sp = std::min<int64_t>(ceil_div(296, tiles), ceil_div(n > 0 ? n : 1, 512));
+  return (int)std::max<int64_t>(1, sp);
+}
+
+int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int layer, int d_in, int d_out) {
+  (void)n_src;
+  const int S = tc_dw_splits(n_dst, d_out, d_in);
+  const int64_t Dp = round_up(d_in, 64);
+  int64_t b = R(n_dst * pitch_of(d_out) * 2);                        // dZ bf16
+  if (layer >= 2) b += R(n_dst * pitch_of(d_out) * 2);                // dZ / D bf16
+  b += R((int64_t)S * d_out * 2 * Dp * 4) + R((int64_t)S * pitch_of(d_out) * 4);
+  return b;
+}
+
+bool tc_bwd_supported(const BwdArgs& a) {
+  return a.act_bf16 && round_up(a.d_out, 16) <= 256 && (a.layer1 || round_up(a.d_in, 16) <= 256);
+}
+
+buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
+  const buffalo_block* blk = a.blk;
+  const int64_t n = blk->n_dst;
+  const int d_in = a.d_in, d_out = a.d_out;
+  const int dp = (int)pitch_of(d_out);
+  const int S = tc_dw_splits(n, d_out, d_in);
+  const int64_t Dp = round_up(d_in, 64);
+  char* q = (char*)a.scratch;
+  __nv_bfloat16* zb = (__nv_bfloat16*)q; q += R(n * dp * 2);
+  __nv_bfloat16* zs = nullptr;
+  if (a.dh_src) { zs = (__nv_bfloat16*)q; q += R(n * dp * 2); }
+  float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * Dp * 4);
+  float* db_part = (float*)q;
+  if (n <= 0) return BUFFALO_OK;
+  k_dz_prep<__nv_bfloat16><<<grid_for(n * (dp / 8), 256), 256, 0, s>>>(
+      a.dh, a.ld_dh, a.last ? nullptr : (const __nv_bfloat16*)a.h_dst, a.ld_hdst, blk->row_ptr, n, d_out, dp, zb, zs);
+  BF_LAUNCHED("k_dz_prep");
+  // dW and db
+  TcDwParams w{};
+  w.zb = zb; w.ldz = dp;
+  w.self_ = a.h_src; w.lds = a.ld_src; w.gidx = a.layer1 ? blk->src_global : nullptr;
+  w.agg = (const __nv_bfloat16*)a.agg; w.lda = a.ld_agg;
+  w.n = n; w.d_out = d_out; w.d_in = d_in; w.pitch_in = (int)pitch_of(d_in); w.pz = dp; w.Dp = (int)Dp;
+  w.NT = (int)std::min<int64_t>(256, 2 * Dp);
+  w.rows_per_split = ceil_div(n, S);
+  w.part = dw_part;
+  w.dz = a.dh; w.lddz = a.ld_dh; w.db_part = db_part;
+  const int smem = kDwStages * (2 + w.NT / 64) * kDwStrip + 64 + 1024;
+  dim3 grid((unsigned)ceil_div(d_out, 128), (unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
+  static bool attr[2] = {false, false};
+  if (a.in_bf16) {
+    if (!attr[0]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)); attr[0] = true; }
+    k_tc_dw<__nv_bfloat16><<<grid, kDwThreads, smem, s>>>(w);
+  } else {
+    if (!attr[1]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)); attr[1] = true; }
+    k_tc_dw<float><<<grid, kDwThreads, smem, s>>>(w);
+  }
+  BF_LAUNCHED("k_tc_dw");
+  k_reduce_dw<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, d_out, d_in, (int)Dp, a.dW);
+  BF_LAUNCHED("k_reduce_dw");
+  k_reduce_db<<<1, 256, 0, s>>>(db_part, S, d_out, a.db);
+  BF_LAUNCHED("k_reduce_db");
+  // dH_{l-1} = [dZ (rows < n_dst) || sum_{i in T(j)} dZ[i]/D(i)] [W_self; W_neigh]
+  if (a.dh_src && blk->n_src > 0) {
+    TcFwdParams p{};
+    p.row_ptr = blk->t_row_ptr;
+    p.col = blk->t_col;
+    p.gidx = nullptr;
+    p.n_dst = blk->n_src;
+    p.self_rows = n;
+    p.h = zs; p.ldh = dp;
+    p.hs = zb; p.lds = dp;
+    p.d_in = d_out;
+    p.pitch_in = dp;
+    p.nkc_self = (int)ceil_div(d_out, kKC);
+    p.nkc = 2 * p.nkc_self;
+    p.wpk = (const uint8_t*)a.W_packed + R((int64_t)2 * d_in * d_out * 4) + tc_fwd_packed_bytes(d_in, d_out);
+    p.Np = (int)round_up(d_in, 16);
+    p.d_out = d_in;
+    p.ld_out = (int)a.ld_dh_src;
+    p.tmem_cols = tmem_cols_for(p.Np);
+    p.bias = nullptr;
+    p.relu = 0;
+    p.out_f32 = 1;
+    p.out = a.dh_src;
+    p.agg = nullptr;
+    p.ld_agg = 0;
+    BF_CHECK((launch_tc<__nv_bfloat16, 1>(p, s)));
+  }
+  return BUFFALO_OK;
 }
 
 }  // namespace buffalo

@@ -49,7 +49,8 @@ def test_estimate_mem_equals_oracle(blib, gemm):
     rng = np.random.default_rng(gemm)
     for _ in range(200):
         L = int(rng.integers(1, 4))
-        dims = [int(x) for x in rng.integers(1, 600, L + 1)]
+        dims = [int(x) for x in rng.integers(1, 600 if not gemm else 257, L + 1)]
+        dims[0] = int(rng.integers(1, 2000))
         n = [int(x) for x in rng.integers(0, 300000, L + 1)]
         e = [int(x) for x in rng.integers(0, 3000000, L)]
         m = blib.make_model(dims, gemm_mode=gemm)
