@@ -848,11 +848,12 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   const int smem = kDwStages * (2 + w.NT / 64) * kDwStrip + 64 + 1024;
   dim3 grid((unsigned)ceil_div(d_out, 128), (unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
   static bool attr[2] = {false, false};
+  constexpr int kMaxDwSmem = kDwStages * (2 + 4) * kDwStrip + 64 + 1024;
   if (a.in_bf16) {
-    if (!attr[0]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)); attr[0] = true; }
+    if (!attr[0]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr[0] = true; }
     k_tc_dw<__nv_bfloat16><<<grid, kDwThreads, smem, s>>>(w);
   } else {
-    if (!attr[1]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)); attr[1] = true; }
+    if (!attr[1]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr[1] = true; }
     k_tc_dw<float><<<grid, kDwThreads, smem, s>>>(w);
   }
   BF_LAUNCHED("k_tc_dw");
