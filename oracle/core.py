@@ -222,15 +222,16 @@ def mem_model(n, e, dims, act_dtype=FP32):
     build = 0
     for l in range(1, L + 1):
         nl, nm, el = n[l], n[l - 1], e[l - 1]
-        blocks += _R(4 * (nl + 1)) + _R(4 * nl) + _R(4 * el) + _R(4 * nm)   # row_ptr heavy col src
+        blocks += _R(4 * (nl + 1)) + _R(4 * nl) + _R(4 * el) + _R(4 * nm)   # row_ptr cls_perm col src
         if l == 1:
             blocks += _R(4 * el)                                # col_global kept for layer 1
         else:
             blocks += _R(4 * (nm + 1)) + _R(4 * el)             # transposed block
-        pc = _part_count_elems(el)
-        frame = _R(64) + _scan_ws_bytes(max(nl + el + 1, pc + 1))
+        pc, pn = _part_count_elems(el), _part_count_elems(nl)
+        frame = _R(64) + _scan_ws_bytes(max(nl + el + 1, pc + 1, pn + 1))
+        frame += _R(4 * (max(pc, pn) + 1))                      # partition counts (classes, radix)
         if l >= 2:
-            frame += 6 * _R(4 * el) + _R(4 * (pc + 1))          # col_global + radix buffers
+            frame += 6 * _R(4 * el)                             # col_global + radix buffers
         build = max(build, frame)
     acts = 0
     for l in range(1, L + 1):

@@ -149,11 +149,20 @@ struct HeavyFlag {
     return (rp[i + 1] - rp[i]) > kHeavyT ? 1 : 0;
   }
 };
-struct EmitIndex {
-  int32_t* out;
-  __device__ __forceinline__ void operator()(int64_t i, int32_t excl, int32_t v) const {
-    if (v) out[excl] = (int32_t)i;
+struct NoStore {
+  __device__ __forceinline__ void operator()(int64_t, int32_t, int32_t) const {}
+};
+// Degree class of a dst row (degree bucketing of the block, Alg. 2 l.6): min(D, kHeavyT + 1).
+struct DegClass {
+  const int32_t* rp;
+  __device__ __forceinline__ int operator()(int64_t i) const {
+    const int32_t D = rp[i + 1] - rp[i];
+    return D > kHeavyT ? kHeavyT + 1 : D;
   }
+};
+struct EmitPerm {
+  int32_t* perm;
+  __device__ __forceinline__ void operator()(int64_t i, int32_t pos) const { perm[pos] = (int32_t)i; }
 };
 
 __global__ void k_fill_zero(int32_t* a, int64_t n) {
@@ -195,11 +204,15 @@ static buffalo_status d2h_i32(const int32_t* d, int32_t* h, cudaStream_t s) {
 }
 
 int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only) {
-  int64_t pc = part_count_elems(e);
-  int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pc + 1);
-  int64_t fr = R(64) + R(4 * scan_ws_elems(scan_len));
-  if (sizes_only) return fr + R(4 * e);
-  if (layer >= 2) fr += 6 * R(4 * e) + R(4 * (pc + 1));
+  const int64_t pc = part_count_elems(e);
+  if (sizes_only) {
+    const int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pc + 1);
+    return R(64) + R(4 * scan_ws_elems(scan_len)) + R(4 * e);
+  }
+  const int64_t pn = part_count_elems(n_dst);
+  const int64_t scan_len = std::max<int64_t>(std::max<int64_t>(n_dst + e + 1, pc + 1), pn + 1);
+  int64_t fr = R(64) + R(4 * scan_ws_elems(scan_len)) + R(4 * (std::max(pc, pn) + 1));
+  if (layer >= 2) fr += 6 * R(4 * e);
   return fr;
 }
 
@@ -209,7 +222,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   memset(blk, 0, sizeof(*blk));
   blk->n_dst = n_dst;
   int32_t* rp = (int32_t*)A.take(4 * (n_dst + 1));
-  int32_t* heavy = sizes_only ? nullptr : (int32_t*)A.take(4 * n_dst);
+  int32_t* perm = sizes_only ? nullptr : (int32_t*)A.take(4 * n_dst);
   // frame 1: totals + scan workspace for the count scan and the heavy compaction
   char* fr = A.push_frame(R(64) + R(4 * scan_ws_elems(n_dst + 1)));
   if (A.overflow) return BUFFALO_ERR_CAPACITY;
@@ -222,7 +235,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   BF_CHECK(scan_inplace(rp, n_dst, ws, s));
   int32_t e32 = 0, nh = 0;
   if (!sizes_only) {
-    BF_CHECK(device_scan(HeavyFlag{rp}, EmitIndex{heavy}, n_dst, ws, totals, s));
+    BF_CHECK(device_scan(HeavyFlag{rp}, NoStore{}, n_dst, ws, totals, s));
     BF_CHECK(d2h_i32(totals, &nh, s));
   }
   BF_CHECK(d2h_i32(rp + n_dst, &e32, s));
@@ -231,7 +244,8 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   blk->n_edges = e;
   blk->n_heavy = nh;
   blk->row_ptr = rp;
-  blk->heavy = heavy;
+  blk->cls_perm = perm;
+  blk->heavy = perm ? perm + (n_dst - nh) : nullptr;
 
   // frame 2
   const int64_t pc = part_count_elems(e);
@@ -245,6 +259,13 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   ws = (int32_t*)q; q += R(4 * scan_ws_elems(scan_len));
   int32_t* colg = colg_persist;
   if (!colg) { colg = (int32_t*)q; q += R(4 * e); }
+  int32_t* counts = nullptr;
+  if (!sizes_only) {
+    counts = (int32_t*)q;
+    q += R(4 * (std::max(part_count_elems(e), part_count_elems(n_dst)) + 1));
+    // degree classes of the dst rows: stable counting sort by min(D, kHeavyT + 1)
+    BF_CHECK(stable_partition(DegClass{rp}, EmitPerm{perm}, n_dst, counts, ws, s));
+  }
   if (n_dst > 0) {
     k_sample_fill<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(dst, n_dst, g->row_ptr, g->col, f, hop,
                                                                seed, rp, colg);
@@ -298,7 +319,6 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     int32_t* ed = (int32_t*)q; q += R(4 * e);
     int32_t* bufk[2] = {(int32_t*)q, (int32_t*)(q + R(4 * e))}; q += 2 * R(4 * e);
     int32_t* bufp[2] = {(int32_t*)q, (int32_t*)(q + R(4 * e))}; q += 2 * R(4 * e);
-    int32_t* counts = (int32_t*)q;
     k_fill_zero<<<grid_for(n_src + 1, 256), 256, 0, s>>>(trp, n_src + 1);
     BF_LAUNCHED("k_fill_zero");
     if (e > 0) {

@@ -143,6 +143,7 @@ struct TcFwdParams {
   int64_t ldh;               // elements
   const void* hs;            // self rows (fwd: = h)
   int64_t lds;
+  const int32_t* perm;       // tile row order (degree-sorted dst) or null (natural order)
   int d_in, pitch_in;        // pitch_in: valid columns readable in a row (multiple of 8)
   int nkc_self, nkc;         // K-chunks for the self half, total (= 2 nkc_self)
   const uint8_t* wpk;        // pre-swizzled bf16 W chunks, each Np x 128 B
@@ -197,11 +198,34 @@ template <> __device__ __forceinline__ void raw_to_f32<float>(const uint4& u, fl
 // MODE 0: forward (mean of neighbour rows, long-tail rows pre-aggregated, h_agg saved,
 //         + bias, ReLU).  MODE 1: backward dH (plain sum of pre-scaled dZ/D rows over the
 //         transposed block, self half = dZ for rows < self_rows, fp32 output).
+// Super-chunk schedule of a tile (identical on the gather and the MMA side): the self half in
+// groups of kSuper K-chunks, then the aggregate half in groups of kAggChunks(E) K-chunks
+// (32 lanes x 16 B = one warp-wide row slice).
+template <int E> struct Sched {
+  static constexpr int kAggChunks = (32 * E) / kKC;          // 4 (bf16) or 2 (fp32)
+  int nself_sc, nagg_sc, nkc_self, nkc;
+  __device__ Sched(int nkc_self_, int nkc_) : nkc_self(nkc_self_), nkc(nkc_) {
+    nself_sc = (nkc_self + kSuper - 1) / kSuper;
+    nagg_sc = (nkc - nkc_self + kAggChunks - 1) / kAggChunks;
+  }
+  __device__ int count() const { return nself_sc + nagg_sc; }
+  __device__ int first(int sc) const {
+    return sc < nself_sc ? sc * kSuper : nkc_self + (sc - nself_sc) * kAggChunks;
+  }
+  __device__ int size(int sc) const {
+    const int f = first(sc);
+    return sc < nself_sc ? min(kSuper, nkc_self - f) : min(kAggChunks, nkc - f);
+  }
+};
+
+// MODE 0: forward (mean of neighbour rows, long-tail rows pre-aggregated, h_agg saved,
+//         + bias, ReLU; tile rows taken in degree-sorted order through `perm`).
+// MODE 1: backward dH (plain sum of pre-scaled dZ/D rows over the transposed block, self half
+//         = dZ for rows < self_rows, fp32 output, natural row order).
 template <class TI, int MODE>
 __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p) {
   constexpr int E = InTraits<TI>::kElems;      // elements per 16-B piece
   constexpr int P = kKC / E;                   // pieces per 64-column chunk row (8 or 16)
-  constexpr int G = 32 / P;                    // neighbour groups per warp (4 or 2)
   constexpr int kUnroll = 8;                   // independent 16-B loads in flight per lane
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -219,7 +243,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t ntiles = (p.n_dst + kTileM - 1) / kTileM;
-  const int nsc = (p.nkc + kSuper - 1) / kSuper;
+  const Sched<E> sched(p.nkc_self, p.nkc);
+  const int nsc = sched.count();
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < 2; ++i) {
@@ -259,9 +284,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
           const int buf = (int)(q & 1);
           mbar_wait(&a_full[buf], (uint32_t)((q >> 1) & 1));
           tc_fence_after();
-          for (int j = 0; j < kSuper; ++j) {
-            const int c = sc * kSuper + j;
-            if (c >= p.nkc) break;
+          const int c0 = sched.first(sc), cn_ = sched.size(sc);
+          for (int j = 0; j < cn_; ++j) {
+            const int c = c0 + j;
             const int bs = (int)(g & 1);
             mbar_wait(&b_full[bs], (uint32_t)((g >> 1) & 1));
             tc_fence_after();
@@ -277,9 +302,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
             if (gn < total_chunks) {
               const int ns = (int)(gn & 1);
               if (gn >= 2) mbar_wait(&b_empty[ns], (uint32_t)(((gn >> 1) - 1) & 1));
-              const int cn = (int)(gn % p.nkc);
+              const int cnext = (int)(gn % p.nkc);
               mbar_arrive_expect_tx(&b_full[ns], bbytes);
-              bulk_g2s(sB + ns * bbytes, p.wpk + (int64_t)cn * bbytes, bbytes, &b_full[ns]);
+              bulk_g2s(sB + ns * bbytes, p.wpk + (int64_t)cnext * bbytes, bbytes, &b_full[ns]);
             }
             ++g;
           }
@@ -295,18 +320,20 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
     const TI* __restrict__ hs = (const TI*)p.hs;
     int64_t q = 0, i = 0;
     int64_t prev_tile = -1;
+    auto row_of = [&](int64_t pos) -> int64_t { return p.perm ? (int64_t)__ldg(p.perm + pos) : pos; };
     auto epilogue = [&](int64_t tile, int64_t li) {
       const int acc = (int)(li & 1);
       mbar_wait(&acc_full[acc], (uint32_t)((li >> 1) & 1));
       tc_fence_after();
       const int quad = warp & 3, part = warp >> 2;
       const int r = quad * 32 + lane;
-      const int64_t row = tile * kTileM + r;
+      const int64_t pos = tile * kTileM + r;
+      const int64_t row = pos < p.n_dst ? row_of(pos) : -1;
       const int ngrp = (int)pitch_of(p.d_out) / 8;
       for (int grp = part; grp < ngrp; grp += 4) {
         float v[8];
         tmem_ld8(tmem_base + ((uint32_t)(quad * 32) << 16) + acc * p.Np + grp * 8, v);
-        if (row < p.n_dst) {
+        if (row >= 0) {
 #pragma unroll
           for (int k = 0; k < 8; ++k) {
             const int cidx = grp * 8 + k;
@@ -328,96 +355,96 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
       mbar_arrive(&acc_empty[acc]);
     };
 
-    const int grp_id = lane / P, piece = lane % P;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
-      const int64_t row0 = t * kTileM;
+      const int64_t pos0 = t * kTileM;
       for (int sc = 0; sc < nsc; ++sc, ++q) {
         const int buf = (int)(q & 1);
         if (q >= 2) mbar_wait(&a_empty[buf], (uint32_t)(((q >> 1) - 1) & 1));
-        for (int j = 0; j < kSuper; ++j) {
-          const int c = sc * kSuper + j;
-          if (c >= p.nkc) break;
-          uint8_t* chunk = sA + (buf * kSuper + j) * kChunkBytesA;
-          if (c < p.nkc_self) {
-            // self rows: 128 rows x P pieces, strided over the gather threads
-            for (int u = threadIdx.x; u < kTileM * P; u += kGatherThreads) {
-              const int r = u / P, pc = u % P;
-              const int64_t row = row0 + r;
-              const int col0 = c * kKC + pc * E;
-              float v[E];
+        const int c0 = sched.first(sc), ncs = sched.size(sc);
+        uint8_t* abuf = sA + buf * kSuper * kChunkBytesA;
+        if (c0 < p.nkc_self) {
+          // self rows: 128 rows x (ncs * P) pieces, strided over the gather threads
+          const int pcs = ncs * P;
+          for (int u = threadIdx.x; u < kTileM * pcs; u += kGatherThreads) {
+            const int r = u / pcs, pc = u % pcs;
+            const int64_t pos = pos0 + r;
+            const int col0 = c0 * kKC + pc * E;
+            float v[E];
 #pragma unroll
-              for (int k = 0; k < E; ++k) v[k] = 0.f;
+            for (int k = 0; k < E; ++k) v[k] = 0.f;
+            if (pos < p.n_dst) {
+              const int64_t row = row_of(pos);
               if (row < p.self_rows && col0 < p.pitch_in) {
                 const int64_t hr = p.gidx ? (int64_t)p.gidx[row] : row;
                 ld_piece<TI>(hs + hr * p.lds + col0, v);
               }
-              st_swz<E>(chunk, r, pc, v);
             }
-          } else {
-            const int ca = c - p.nkc_self;
-            const int col0 = ca * kKC + piece * E;
-            const bool colok = col0 < p.pitch_in;
-            for (int r = warp; r < kTileM; r += kGatherWarps) {
-              const int64_t row = row0 + r;
-              float acc[E];
+            st_swz<E>(abuf + (pc / P) * kChunkBytesA, r, pc % P, v);
+          }
+        } else {
+          // aggregate: one lane group per destination row, lane = 16-B column piece
+          const int cbase = (c0 - p.nkc_self) * kKC;                 // first column of this slice
+          const int need = min(ncs * P, (p.pitch_in - cbase + E - 1) / E);
+          int pact = 1;
+          while (pact < need) pact <<= 1;                            // lanes per row (<= 32)
+          const int G = 32 / pact;                                   // rows per warp step
+          const int grp_id = lane / pact, pc = lane % pact;
+          const int col0 = cbase + pc * E;
+          const bool colok = pc < need && col0 < p.pitch_in;
+          for (int rb = warp * G; rb < kTileM; rb += kGatherWarps * G) {
+            const int r = rb + grp_id;
+            const int64_t pos = pos0 + r;
+            const int64_t row = (r < kTileM && pos < p.n_dst) ? row_of(pos) : -1;
+            int32_t b = 0, e_end = 0;
+            if (row >= 0) { b = __ldg(p.row_ptr + row); e_end = __ldg(p.row_ptr + row + 1); }
+            const int32_t D = e_end - b;
+            const bool heavy = MODE == 0 && D > kHeavyT;
+            float acc[E];
 #pragma unroll
-              for (int k = 0; k < E; ++k) acc[k] = 0.f;
-              int32_t b = 0, e_end = 0;
-              if (row < p.n_dst) { b = __ldg(p.row_ptr + row); e_end = __ldg(p.row_ptr + row + 1); }
-              const int32_t D = e_end - b;
-              if (MODE == 0 && D > kHeavyT) {
-                // long-tail row: pre-aggregated by k_agg_heavy into the saved h_agg (bf16)
-                if (grp_id == 0 && colok) {
+            for (int k = 0; k < E; ++k) acc[k] = 0.f;
+            const int32_t Dl = heavy ? 0 : D;
+            const int32_t Dmax = __reduce_max_sync(0xffffffffu, Dl);
+            for (int32_t base = 0; base < Dmax; base += pact) {
+              const int32_t jj = (base + pc < Dl) ? __ldg(p.col + b + base + pc) : 0;
+              for (int u = 0; u < pact; u += kUnroll) {
+                uint4 raw[kUnroll];
+#pragma unroll
+                for (int uu = 0; uu < kUnroll; ++uu) {
+                  const int tt = u + uu;
+                  const int32_t jn = __shfl_sync(0xffffffffu, jj, (grp_id * pact + (tt & (pact - 1))) & 31);
+                  raw[uu] = make_uint4(0u, 0u, 0u, 0u);
+                  if (tt < pact && base + tt < Dl && colok)
+                    raw[uu] = __ldg(reinterpret_cast<const uint4*>(h + (int64_t)jn * p.ldh + col0));
+                }
+#pragma unroll
+                for (int uu = 0; uu < kUnroll; ++uu) {
                   float v[E];
+                  raw_to_f32<TI>(raw[uu], v);
+#pragma unroll
+                  for (int k = 0; k < E; ++k) acc[k] += v[k];
+                }
+              }
+            }
+            if (r < kTileM && pc < ncs * P) {
+              if (heavy) {
+                // long-tail row: pre-aggregated by k_agg_heavy into the saved h_agg (bf16)
+                if (colok) {
                   const __nv_bfloat16* src = p.agg + row * p.ld_agg + col0;
                   if constexpr (E == 8) {
-                    bf16x8_to_f32(*reinterpret_cast<const uint4*>(src), v);
+                    bf16x8_to_f32(*reinterpret_cast<const uint4*>(src), acc);
                   } else {
                     uint2 w = *reinterpret_cast<const uint2*>(src);
-                    v[0] = __uint_as_float(w.x << 16); v[1] = __uint_as_float(w.x & 0xffff0000u);
-                    v[2] = __uint_as_float(w.y << 16); v[3] = __uint_as_float(w.y & 0xffff0000u);
-                  }
-                  st_swz<E>(chunk, r, piece, v);
-                } else if (grp_id == 0) {
-                  st_swz<E>(chunk, r, piece, acc);
-                }
-                continue;
-              }
-              for (int32_t base = b; base < e_end; base += 32) {
-                const int cnt = min(32, e_end - base);
-                const int32_t jj = lane < cnt ? __ldg(p.col + base + lane) : 0;
-                for (int r0 = 0; r0 < cnt; r0 += G * kUnroll) {
-                  uint4 raw[kUnroll];
-#pragma unroll
-                  for (int uu = 0; uu < kUnroll; ++uu) {
-                    const int tt = r0 + grp_id + G * uu;
-                    const int32_t jn = __shfl_sync(0xffffffffu, jj, tt & 31);
-                    raw[uu] = make_uint4(0u, 0u, 0u, 0u);
-                    if (tt < cnt && colok)
-                      raw[uu] = __ldg(reinterpret_cast<const uint4*>(h + (int64_t)jn * p.ldh + col0));
-                  }
-#pragma unroll
-                  for (int uu = 0; uu < kUnroll; ++uu) {
-                    float v[E];
-                    raw_to_f32<TI>(raw[uu], v);
-#pragma unroll
-                    for (int k = 0; k < E; ++k) acc[k] += v[k];
+                    acc[0] = __uint_as_float(w.x << 16); acc[1] = __uint_as_float(w.x & 0xffff0000u);
+                    acc[2] = __uint_as_float(w.y << 16); acc[3] = __uint_as_float(w.y & 0xffff0000u);
                   }
                 }
-              }
-              // combine the G neighbour groups (fixed butterfly order: depends only on D)
-#pragma unroll
-              for (int o = P; o < 32; o <<= 1)
-#pragma unroll
-                for (int k = 0; k < E; ++k) acc[k] += __shfl_xor_sync(0xffffffffu, acc[k], o);
-              if (grp_id == 0) {
+              } else {
                 if (MODE == 0) {
                   const float fd = (float)D;
 #pragma unroll
                   for (int k = 0; k < E; ++k) acc[k] = D > 0 ? acc[k] / fd : 0.f;
                 }
-                st_swz<E>(chunk, r, piece, acc);
-                if (MODE == 0 && row < p.n_dst && colok) {
+                if (MODE == 0 && row >= 0 && colok) {
                   __nv_bfloat16* dstp = p.agg + row * p.ld_agg + col0;
                   if constexpr (E == 8) {
                     *reinterpret_cast<uint4*>(dstp) =
@@ -429,6 +456,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
                   }
                 }
               }
+              st_swz<E>(abuf + (pc / P) * kChunkBytesA, r, pc % P, acc);
+            }
+          }
+          // pieces of this slice beyond pact (zero columns past the row pitch)
+          for (int u = threadIdx.x; u < kTileM * ncs * P; u += kGatherThreads) {
+            const int r = u / (ncs * P), pcz = u % (ncs * P);
+            if (pcz >= pact) {
+              float z[E];
+#pragma unroll
+              for (int k = 0; k < E; ++k) z[k] = 0.f;
+              st_swz<E>(abuf + (pcz / P) * kChunkBytesA, r, pcz % P, z);
             }
           }
         }
@@ -547,6 +585,7 @@ static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   p.gidx = a.layer1 ? blk->src_global : nullptr;
   p.n_dst = blk->n_dst;
   p.self_rows = blk->n_dst;
+  p.perm = blk->cls_perm;
   p.h = a.h_src;
   p.ldh = a.ld_src;
   p.hs = a.h_src;
