@@ -110,13 +110,14 @@ typedef struct {
  * (block >= 2 only, else NULL): for each src j the dst i with an edge to j, ascending.
  * cls_perm int32[n_dst]: the dst sorted by degree class min(D, 129), stable (degree bucketing of
  * the block, Alg. 2 l.6 PAPER.md:238); heavy = cls_perm + n_dst - n_heavy lists the dst with
- * D > 128 (long-tail cooperative path), ascending.
+ * D > 128 (long-tail cooperative path), ascending.  t_perm int32[n_src] (block >= 2 only): the src
+ * sorted by transposed degree class; its last n_heavy_t entries have more than 128 dst.
  * Activations of the standard arena layout: agg (saved h_agg [n_dst][ld_agg]), out (H_l
  * [n_dst][ld_out], act dtype, or logits fp32 at l = L), dh (dH_l / dlogits fp32 [n_dst][ld_dh],
  * valid during the backward of layers l and l+1), bwd_scratch (bwd_scratch_bytes). */
 typedef struct {
-  int64_t n_dst, n_src, n_edges, n_heavy;
-  int32_t *row_ptr, *col_local, *col_global, *src_global, *t_row_ptr, *t_col, *heavy, *cls_perm;
+  int64_t n_dst, n_src, n_edges, n_heavy, n_heavy_t;
+  int32_t *row_ptr, *col_local, *col_global, *src_global, *t_row_ptr, *t_col, *heavy, *cls_perm, *t_perm;
   void* agg;
   void* out;
   float* dh;

@@ -226,10 +226,10 @@ def mem_model(n, e, dims, act_dtype=FP32):
         if l == 1:
             blocks += _R(4 * el)                                # col_global kept for layer 1
         else:
-            blocks += _R(4 * (nm + 1)) + _R(4 * el)             # transposed block
-        pc, pn = _part_count_elems(el), _part_count_elems(nl)
-        frame = _R(64) + _scan_ws_bytes(max(nl + el + 1, pc + 1, pn + 1))
-        frame += _R(4 * (max(pc, pn) + 1))                      # partition counts (classes, radix)
+            blocks += _R(4 * (nm + 1)) + _R(4 * el) + _R(4 * nm)  # transposed block + its classes
+        pne = _part_count_elems(nl + el)
+        frame = _R(64) + _scan_ws_bytes(max(nl + el + 1, pne + 1))
+        frame += _R(4 * (pne + 1))                              # partition counts (classes, radix)
         if l >= 2:
             frame += 6 * _R(4 * el)                             # col_global + radix buffers
         build = max(build, frame)
@@ -253,6 +253,7 @@ def mem_model(n, e, dims, act_dtype=FP32):
             frame += _R(n[l] * pitch(dims[l]) * 2)              # dZ in bf16
             if l >= 2:
                 frame += _R(n[l] * pitch(dims[l]) * 2)          # dZ / D in bf16
+                frame += _R(e[l - 1] // (HEAVY_T + 1) * pitch(dims[l]) * 2)  # long-tail sums
             S = tc_dw_splits(n[l], dims[l], dims[l - 1])
             Dp = _ceil(dims[l - 1], 64) * 64
             frame += _R(S * dims[l] * 2 * Dp * 4) + _R(S * pitch(dims[l]) * 4)          # dW, db partials

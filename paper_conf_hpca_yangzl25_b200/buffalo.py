@@ -66,8 +66,9 @@ class Plan(ctypes.Structure):
 
 class Block(ctypes.Structure):
     _fields_ = [("n_dst", c_i64), ("n_src", c_i64), ("n_edges", c_i64), ("n_heavy", c_i64),
+                ("n_heavy_t", c_i64),
                 ("row_ptr", c_p), ("col_local", c_p), ("col_global", c_p), ("src_global", c_p),
-                ("t_row_ptr", c_p), ("t_col", c_p), ("heavy", c_p), ("cls_perm", c_p),
+                ("t_row_ptr", c_p), ("t_col", c_p), ("heavy", c_p), ("cls_perm", c_p), ("t_perm", c_p),
                 ("agg", c_p), ("out", c_p), ("dh", c_p), ("bwd_scratch", c_p),
                 ("ld_agg", c_i64), ("ld_out", c_i64), ("ld_dh", c_i64), ("bwd_scratch_bytes", c_i64)]
 

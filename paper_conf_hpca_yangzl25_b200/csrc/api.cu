@@ -58,8 +58,8 @@ __global__ void k_fill_i32(int32_t* a, int64_t n, int32_t v) {
 
 // ------------------------------------------------------------------ memory model (R15)
 // Restated from DESIGN.md §5; must agree with the arena that buffalo_build_blocks lays out.
-static int64_t bwd_scratch_for(const buffalo_model* m, int64_t n_dst, int64_t n_src, int l) {
-  if (m->gemm_mode == BUFFALO_GEMM_BF16) return tc_bwd_scratch_bytes(n_dst, n_src, l, m->dim[l - 1], m->dim[l]);
+static int64_t bwd_scratch_for(const buffalo_model* m, int64_t n_dst, int64_t n_src, int64_t e, int l) {
+  if (m->gemm_mode == BUFFALO_GEMM_BF16) return tc_bwd_scratch_bytes(n_dst, n_src, e, l, m->dim[l - 1], m->dim[l]);
   return bwd_scratch_bytes(n_dst, n_src, l, m->dim[l - 1], m->dim[l]);
 }
 
@@ -70,7 +70,7 @@ static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_m
   for (int l = 1; l <= L; ++l) {
     const int64_t nl = n[l], nm = n[l - 1], el = e[l - 1];
     blocks += R(4 * (nl + 1)) + R(4 * nl) + R(4 * el) + R(4 * nm);
-    blocks += (l == 1) ? R(4 * el) : R(4 * (nm + 1)) + R(4 * el);
+    blocks += (l == 1) ? R(4 * el) : R(4 * (nm + 1)) + R(4 * el) + R(4 * nm);
     build = std::max(build, build_frame_bytes(nl, el, l, false));
   }
   for (int l = 1; l <= L; ++l) {
@@ -81,7 +81,7 @@ static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_m
   for (int l = L; l >= 1; --l) {
     int64_t f = R(n[l] * pitch_of(m->dim[l]) * 4);
     if (l >= 2) f += R(n[l - 1] * pitch_of(m->dim[l - 1]) * 4);
-    f += bwd_scratch_for(m, n[l], n[l - 1], l);
+    f += bwd_scratch_for(m, n[l], n[l - 1], e[l - 1], l);
     bwd = std::max(bwd, f);
   }
   *lo = blocks + acts + bwd;
@@ -486,7 +486,7 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
   std::vector<int64_t> ah(L + 1, 0), tmp(L + 1, 0);
   for (int l = 1; l <= L; ++l) ah[l] = R(nn[l] * pitch_of(m->dim[l]) * 4);
   for (int l = L; l >= 1; --l) {
-    tmp[l] = bwd_scratch_for(m, nn[l], nn[l - 1], l);
+    tmp[l] = bwd_scratch_for(m, nn[l], nn[l - 1], ee[l - 1], l);
     B = std::max(B, ah[l] + (l >= 2 ? ah[l - 1] : 0) + tmp[l]);
   }
   char* region = (char*)A.take(B);
@@ -573,7 +573,7 @@ buffalo_status buffalo_sage_fwd(const buffalo_block* blk, int32_t layer, const b
 
 size_t buffalo_sage_bwd_scratch_bytes(const buffalo_block* blk, int32_t layer, const buffalo_model* m) {
   if (!blk || !m || layer < 1 || layer > m->num_layers) return 0;
-  return (size_t)bwd_scratch_for(m, blk->n_dst, blk->n_src, layer);
+  return (size_t)bwd_scratch_for(m, blk->n_dst, blk->n_src, blk->n_edges, layer);
 }
 
 buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,

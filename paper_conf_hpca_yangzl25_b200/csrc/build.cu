@@ -209,9 +209,9 @@ int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only) 
     const int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pc + 1);
     return R(64) + R(4 * scan_ws_elems(scan_len)) + R(4 * e);
   }
-  const int64_t pn = part_count_elems(n_dst);
-  const int64_t scan_len = std::max<int64_t>(std::max<int64_t>(n_dst + e + 1, pc + 1), pn + 1);
-  int64_t fr = R(64) + R(4 * scan_ws_elems(scan_len)) + R(4 * (std::max(pc, pn) + 1));
+  const int64_t pne = part_count_elems(n_dst + e);   // bounds the partitions of n_dst, n_src, e
+  const int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pne + 1);
+  int64_t fr = R(64) + R(4 * scan_ws_elems(scan_len)) + R(4 * (pne + 1));
   if (layer >= 2) fr += 6 * R(4 * e);
   return fr;
 }
@@ -248,7 +248,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   blk->heavy = perm ? perm + (n_dst - nh) : nullptr;
 
   // frame 2
-  const int64_t pc = part_count_elems(e);
+  const int64_t pc = sizes_only ? part_count_elems(e) : part_count_elems(n_dst + e);
   const int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pc + 1);
   int32_t* col_local = (!sizes_only) ? (int32_t*)A.take(4 * e) : nullptr;
   int32_t* colg_persist = (!sizes_only && layer == 1) ? (int32_t*)A.take(4 * e) : nullptr;
@@ -262,7 +262,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   int32_t* counts = nullptr;
   if (!sizes_only) {
     counts = (int32_t*)q;
-    q += R(4 * (std::max(part_count_elems(e), part_count_elems(n_dst)) + 1));
+    q += R(4 * (pc + 1));
     // degree classes of the dst rows: stable counting sort by min(D, kHeavyT + 1)
     BF_CHECK(stable_partition(DegClass{rp}, EmitPerm{perm}, n_dst, counts, ws, s));
   }
@@ -315,6 +315,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     // (dst-ordered) keyed by col_local => each transposed row lists its dst ascending.
     int32_t* trp = (int32_t*)A.take(4 * (n_src + 1));
     int32_t* tcol = (int32_t*)A.take(4 * e);
+    int32_t* tperm = (int32_t*)A.take(4 * n_src);
     if (A.overflow) return BUFFALO_ERR_CAPACITY;
     int32_t* ed = (int32_t*)q; q += R(4 * e);
     int32_t* bufk[2] = {(int32_t*)q, (int32_t*)(q + R(4 * e))}; q += 2 * R(4 * e);
@@ -326,6 +327,11 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
       BF_LAUNCHED("k_tcount");
     }
     BF_CHECK(scan_inplace(trp, n_src, ws, s));
+    // degree classes of the transposed rows (long-tail src go last)
+    BF_CHECK(stable_partition(DegClass{trp}, EmitPerm{tperm}, n_src, counts, ws, s));
+    BF_CHECK(device_scan(HeavyFlag{trp}, NoStore{}, n_src, ws, totals + 1, s));
+    int32_t nht = 0;
+    BF_CHECK(d2h_i32(totals + 1, &nht, s));
     if (e > 0) {
       k_edge_dst<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(rp, n_dst, ed);
       BF_LAUNCHED("k_edge_dst");
@@ -344,6 +350,9 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     }
     blk->t_row_ptr = trp;
     blk->t_col = tcol;
+    blk->t_perm = tperm;
+    BF_CUDA(cudaStreamSynchronize(s));                             // n_heavy_t
+    blk->n_heavy_t = nht;
   }
   A.pop_frame();
   return BUFFALO_OK;

@@ -144,6 +144,9 @@ struct TcFwdParams {
   const void* hs;            // self rows (fwd: = h)
   int64_t lds;
   const int32_t* perm;       // tile row order (degree-sorted dst) or null (natural order)
+  int64_t heavy_base;        // MODE 1: positions >= heavy_base are long-tail rows, pre-summed
+  const __nv_bfloat16* heavy_buf;  // MODE 1: [pos - heavy_base][heavy_ld]
+  int64_t heavy_ld;
   int d_in, pitch_in;        // pitch_in: valid columns readable in a row (multiple of 8)
   int nkc_self, nkc;         // K-chunks for the self half, total (= 2 nkc_self)
   const uint8_t* wpk;        // pre-swizzled bf16 W chunks, each Np x 128 B
@@ -398,7 +401,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
             int32_t b = 0, e_end = 0;
             if (row >= 0) { b = __ldg(p.row_ptr + row); e_end = __ldg(p.row_ptr + row + 1); }
             const int32_t D = e_end - b;
-            const bool heavy = MODE == 0 && D > kHeavyT;
+            const bool heavy = (MODE == 0) ? (D > kHeavyT) : (row >= 0 && pos >= p.heavy_base);
             float acc[E];
 #pragma unroll
             for (int k = 0; k < E; ++k) acc[k] = 0.f;
@@ -406,7 +409,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
             const int32_t Dmax = __reduce_max_sync(0xffffffffu, Dl);
             for (int32_t base = 0; base < Dmax; base += pact) {
               const int32_t jj = (base + pc < Dl) ? __ldg(p.col + b + base + pc) : 0;
-              for (int u = 0; u < pact; u += kUnroll) {
+              const int lim = min(pact, Dmax - base);
+              for (int u = 0; u < lim; u += kUnroll) {
                 uint4 raw[kUnroll];
 #pragma unroll
                 for (int uu = 0; uu < kUnroll; ++uu) {
@@ -429,7 +433,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
               if (heavy) {
                 // long-tail row: pre-aggregated by k_agg_heavy into the saved h_agg (bf16)
                 if (colok) {
-                  const __nv_bfloat16* src = p.agg + row * p.ld_agg + col0;
+                  const __nv_bfloat16* src = (MODE == 0) ? p.agg + row * p.ld_agg + col0
+                                                         : p.heavy_buf + (pos - p.heavy_base) * p.heavy_ld + col0;
                   if constexpr (E == 8) {
                     bf16x8_to_f32(*reinterpret_cast<const uint4*>(src), acc);
                   } else {
@@ -836,6 +841,48 @@ __global__ void k_reduce_db(const float* __restrict__ part, int S, int d, float*
   }
 }
 
+// Long-tail transposed rows (more than kHeavyT dst): out[h] = sum_{t in T(list[h])} z[t_col[t]],
+// 8 warps over the entries (warp w takes t = w, w+8, ...), combined in warp order.
+__global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restrict__ list,
+                                                        const int32_t* __restrict__ rp,
+                                                        const int32_t* __restrict__ col,
+                                                        const __nv_bfloat16* __restrict__ z, int64_t ldz,
+                                                        int dp, __nv_bfloat16* __restrict__ out) {
+  __shared__ float part[8][32][8];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t j = list[blockIdx.x];
+  const int32_t b = rp[j], e_end = rp[j + 1];
+  const int nch = dp / 8;
+  for (int c0 = 0; c0 < nch; c0 += 32) {
+    const int c = c0 + lane;
+    float acc[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) acc[k] = 0.f;
+    if (c < nch)
+      for (int32_t t = b + w; t < e_end; t += 8) {
+        float v[8];
+        bf16x8_to_f32(__ldg(reinterpret_cast<const uint4*>(z + (int64_t)col[t] * ldz + c * 8)), v);
+#pragma unroll
+        for (int k = 0; k < 8; ++k) acc[k] += v[k];
+      }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) part[w][lane][k] = acc[k];
+    __syncthreads();
+    if (w == 0 && c < nch) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        float s = part[0][lane][k];
+        for (int ww = 1; ww < 8; ++ww) s += part[ww][lane][k];
+        acc[k] = s;
+      }
+      *reinterpret_cast<uint4*>(out + (int64_t)blockIdx.x * dp + c * 8) =
+          make_uint4(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]), pack_bf16x2(acc[4], acc[5]),
+                     pack_bf16x2(acc[6], acc[7]));
+    }
+    __syncthreads();
+  }
+}
+
 int tc_dw_splits(int64_t n, int d_out, int d_in) {
   const int64_t Dp = round_up(d_in, 64);
   const int64_t tiles = ceil_div(d_out, 128) * ceil_div(2 * Dp, 256);
@@ -843,12 +890,15 @@ int tc_dw_splits(int64_t n, int d_out, int d_in) {
   return (int)std::max<int64_t>(1, sp);
 }
 
-int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int layer, int d_in, int d_out) {
+int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int64_t e, int layer, int d_in, int d_out) {
   (void)n_src;
   const int S = tc_dw_splits(n_dst, d_out, d_in);
   const int64_t Dp = round_up(d_in, 64);
   int64_t b = R(n_dst * pitch_of(d_out) * 2);                        // dZ bf16
-  if (layer >= 2) b += R(n_dst * pitch_of(d_out) * 2);                // dZ / D bf16
+  if (layer >= 2) {
+    b += R(n_dst * pitch_of(d_out) * 2);                              // dZ / D bf16
+    b += R(e / (kHeavyT + 1) * pitch_of(d_out) * 2);                  // long-tail transposed sums
+  }
   b += R((int64_t)S * d_out * 2 * Dp * 4) + R((int64_t)S * pitch_of(d_out) * 4);
   return b;
 }
@@ -867,7 +917,11 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   char* q = (char*)a.scratch;
   __nv_bfloat16* zb = (__nv_bfloat16*)q; q += R(n * dp * 2);
   __nv_bfloat16* zs = nullptr;
-  if (a.dh_src) { zs = (__nv_bfloat16*)q; q += R(n * dp * 2); }
+  __nv_bfloat16* hbuf = nullptr;
+  if (a.dh_src) {
+    zs = (__nv_bfloat16*)q; q += R(n * dp * 2);
+    hbuf = (__nv_bfloat16*)q; q += R(blk->n_edges / (kHeavyT + 1) * dp * 2);
+  }
   float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * Dp * 4);
   float* db_part = (float*)q;
   if (n <= 0) return BUFFALO_OK;
@@ -902,7 +956,16 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   BF_LAUNCHED("k_reduce_db");
   // dH_{l-1} = [dZ (rows < n_dst) || sum_{i in T(j)} dZ[i]/D(i)] [W_self; W_neigh]
   if (a.dh_src && blk->n_src > 0) {
+    if (blk->n_heavy_t > 0) {
+      k_sum_heavy_rows<<<(unsigned)blk->n_heavy_t, 256, 0, s>>>(blk->t_perm + (blk->n_src - blk->n_heavy_t),
+                                                                blk->t_row_ptr, blk->t_col, zs, dp, dp, hbuf);
+      BF_LAUNCHED("k_sum_heavy_rows");
+    }
     TcFwdParams p{};
+    p.perm = blk->t_perm;
+    p.heavy_base = blk->n_src - blk->n_heavy_t;
+    p.heavy_buf = hbuf;
+    p.heavy_ld = dp;
     p.row_ptr = blk->t_row_ptr;
     p.col = blk->t_col;
     p.gidx = nullptr;

@@ -11,7 +11,7 @@ int64_t tc_fwd_packed_bytes(int64_t d_in, int64_t d_out);
 bool tc_fwd_supported(const FwdArgs& a);
 buffalo_status tc_sage_fwd(const FwdArgs& a, cudaStream_t s);
 int tc_dw_splits(int64_t n, int d_out, int d_in);
-int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int layer, int d_in, int d_out);
+int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int64_t e, int layer, int d_in, int d_out);
 bool tc_bwd_supported(const BwdArgs& a);
 buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s);
 

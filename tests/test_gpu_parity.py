@@ -67,6 +67,13 @@ def test_blocks_bit_exact(name):
             np.testing.assert_array_equal(a["t_row_ptr"], r["t_row_ptr"])
             np.testing.assert_array_equal(a["t_col"], r["t_col"])
         np.testing.assert_array_equal(a["heavy"], np.nonzero(r["D"] > O.HEAVY_T)[0])
+        # degree classes (degree bucketing of the block, Alg. 2 l.6): stable sort by min(D, 129)
+        cls = np.minimum(r["D"], O.HEAVY_T + 1)
+        np.testing.assert_array_equal(a["cls_perm"], np.argsort(cls, kind="stable"))
+        if l >= 2:
+            Dt = np.diff(r["t_row_ptr"])
+            np.testing.assert_array_equal(a["t_perm"], np.argsort(np.minimum(Dt, O.HEAVY_T + 1), kind="stable"))
+            assert a["n_heavy_t"] == int((Dt > O.HEAVY_T).sum())
     if name == "full3":
         assert got[0]["n_heavy"] > 0          # the long-tail path is exercised
 

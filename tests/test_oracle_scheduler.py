@@ -124,7 +124,7 @@ def test_mem_model_hand_instance():
     assert O.mem_model([5, 2], [3], [4, 3], O.FP32) == (1280 + 512 + 768, 1280 + 512 + 1792)
     # a wide layer: n = [40000, 20000], e = [100000], dims = [64, 32]
     # blocks: R(80004)=80128, R(80000)=80128, R(400000)=400128, R(160000)=160000, col_global 400128
-    # build: 256 + R(4*(ceil(120001/16384)+2)) + counts R(4*(256*25+1)) = 256 + 256 + 25856
+    # build: 256 + R(4*(ceil(120001/16384)+2)) + counts R(4*(256*30+1)) = 256 + 256 + 30976
     # acts: agg R(20000*64*4)=5120000, logits R(20000*32*4)=2560000
     # bwd: dH R(20000*32*4)=2560000; splits: tiles=1*2 -> min(148, 40) = 40;
     #      dW R(40*32*128*4)=655360; db R(40*32*4)=5120
