@@ -173,7 +173,7 @@ def degree_bucketing(g, seeds, f_L, F):
 ALIGN = 256
 HEAVY_T = 128          # rows with D > HEAVY_T go through the cooperative long-tail path
 FP32, BF16 = 0, 1
-SCAN_TILE = 16384      # elements per scan tile of the implementation's device-wide scans
+SCAN_TILE = 4096       # elements per tile of the implementation's device-wide scans
 PART_TILE = 4096       # elements per tile of its stable radix/bin partition passes
 
 
@@ -207,7 +207,7 @@ def _part_count_elems(e):
 
 
 def _scan_ws_bytes(length):
-    return _R(4 * (_ceil(max(int(length), 1), SCAN_TILE) + 2))
+    return _R(8 * (_ceil(max(int(length), 1), SCAN_TILE) + 2))
 
 
 def mem_model(n, e, dims, act_dtype=FP32):

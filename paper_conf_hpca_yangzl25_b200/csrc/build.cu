@@ -10,41 +10,6 @@
 
 namespace buffalo {
 
-// ------------------------------------------------------------------ scan tile pass
-__global__ void __launch_bounds__(1024) k_scan_tiles(int32_t* ts, int64_t ntiles, int32_t* total_out) {
-  __shared__ int32_t sw[33];
-  int32_t carry = 0;
-  for (int64_t b = 0; b < ntiles; b += 1024) {
-    int64_t i = b + threadIdx.x;
-    int32_t v = i < ntiles ? ts[i] : 0;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    int32_t x = v;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      int32_t y = __shfl_up_sync(0xffffffffu, x, o);
-      if (lane >= o) x += y;
-    }
-    if (lane == 31) sw[warp] = x;
-    __syncthreads();
-    if (warp == 0) {
-      int32_t w = sw[lane];
-      int32_t s = w;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        int32_t y = __shfl_up_sync(0xffffffffu, s, o);
-        if (lane >= o) s += y;
-      }
-      sw[lane] = s - w;
-      if (lane == 31) sw[32] = s;
-    }
-    __syncthreads();
-    if (i < ntiles) ts[i] = carry + sw[warp] + x - v;
-    carry += sw[32];
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) *total_out = carry;
-}
-
 // ------------------------------------------------------------------ a4: count D per dst
 __global__ void k_count(const int32_t* __restrict__ dst, int64_t n, const int64_t* __restrict__ grow,
                         int32_t f, int32_t* __restrict__ counts) {
@@ -235,7 +200,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   BF_CHECK(scan_inplace(rp, n_dst, ws, s));
   int32_t e32 = 0, nh = 0;
   if (!sizes_only) {
-    BF_CHECK(device_scan(HeavyFlag{rp}, NoStore{}, n_dst, ws, totals, s));
+    BF_CHECK(device_count(HeavyFlag{rp}, n_dst, totals, s));
     BF_CHECK(d2h_i32(totals, &nh, s));
   }
   BF_CHECK(d2h_i32(rp + n_dst, &e32, s));
@@ -279,19 +244,14 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     BF_LAUNCHED("k_relabel_min");
   }
   FirstFlag ff{cand, g->node_map};
-  const int64_t ntiles = ceil_div(total > 0 ? total : 1, kScanTile);
-  k_scan_reduce<<<(unsigned)ntiles, kScanThreads, 0, s>>>(ff, total, ws);
-  BF_LAUNCHED("k_scan_reduce");
-  k_scan_tiles<<<1, 1024, 0, s>>>(ws, ntiles, totals);
-  BF_LAUNCHED("k_scan_tiles");
+  BF_CHECK(device_count(ff, total, totals, s));
   int32_t ns32 = 0;
   BF_CHECK(d2h_i32(totals, &ns32, s));
   BF_CUDA(cudaStreamSynchronize(s));                               // sync 2: n_{l-1}
   const int64_t n_src = ns32;
   int32_t* src = (int32_t*)A.take(4 * n_src);
   if (A.overflow) return BUFFALO_ERR_CAPACITY;
-  k_scan_apply<<<(unsigned)ntiles, kScanThreads, 0, s>>>(ff, EmitSrc{cand, src}, total, ws);
-  BF_LAUNCHED("k_scan_apply");
+  BF_CHECK(device_scan(ff, EmitSrc{cand, src}, total, ws, totals + 2, s));
   blk->n_src = n_src;
   blk->src_global = src;
   blk->col_global = colg_persist;
@@ -329,7 +289,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     BF_CHECK(scan_inplace(trp, n_src, ws, s));
     // degree classes of the transposed rows (long-tail src go last)
     BF_CHECK(stable_partition(DegClass{trp}, EmitPerm{tperm}, n_src, counts, ws, s));
-    BF_CHECK(device_scan(HeavyFlag{trp}, NoStore{}, n_src, ws, totals + 1, s));
+    BF_CHECK(device_count(HeavyFlag{trp}, n_src, totals + 1, s));
     int32_t nht = 0;
     BF_CHECK(d2h_i32(totals + 1, &nht, s));
     if (e > 0) {

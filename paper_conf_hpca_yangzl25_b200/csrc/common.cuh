@@ -12,7 +12,7 @@ namespace buffalo {
 
 constexpr int64_t kAlign = 256;
 constexpr int kHeavyT = 128;          // rows with D > kHeavyT take the cooperative long-tail path
-constexpr int kScanTile = 16384;      // elements per scan tile (512 threads x 32)
+constexpr int kScanTile = 4096;       // elements per scan tile (512 threads x 8)
 
 __host__ __device__ inline int64_t round_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 __host__ __device__ inline int64_t R(int64_t bytes) { return round_up(bytes, kAlign); }

@@ -5,11 +5,17 @@
 
 namespace buffalo {
 
+// Single-pass decoupled look-back scan: each CTA (dynamic tile id) loads its tile with
+// coalesced functor evaluations into shared memory, scans it, publishes its aggregate, looks
+// back over its predecessors' published values and applies the store functor in coalesced
+// order.  Workspace: a zeroed status word (flag | value) per tile + a tile counter.
 constexpr int kScanThreads = 512;
-constexpr int kScanPerThread = kScanTile / kScanThreads;  // 32
-static_assert(kScanPerThread * kScanThreads == kScanTile, "scan tile");
+constexpr int kScanItems = 8;
+static_assert(kScanItems * kScanThreads == kScanTile, "scan tile");
 
-inline int64_t scan_ws_elems(int64_t n) { return ceil_div(n > 0 ? n : 1, kScanTile) + 2; }
+inline int64_t scan_ws_elems(int64_t n) { return 2 * (ceil_div(n > 0 ? n : 1, kScanTile) + 2); }
+
+__device__ __forceinline__ int scan_pad(int i) { return i + (i >> 5); }
 
 template <int NT>
 __device__ __forceinline__ int32_t block_exclusive_sum(int32_t v, int32_t* smem_warp, int32_t* total) {
@@ -40,61 +46,107 @@ __device__ __forceinline__ int32_t block_exclusive_sum(int32_t v, int32_t* smem_
   return r;
 }
 
-// Pass 1: per-tile sums.
-template <class Load>
-__global__ void __launch_bounds__(kScanThreads) k_scan_reduce(Load ld, int64_t n, int32_t* tile_sums) {
-  __shared__ int32_t sw[33];
-  const int64_t base = (int64_t)blockIdx.x * kScanTile + (int64_t)threadIdx.x * kScanPerThread;
-  int32_t s = 0;
-#pragma unroll 4
-  for (int k = 0; k < kScanPerThread; ++k) {
-    int64_t i = base + k;
-    if (i < n) s += ld(i);
-  }
-  int32_t tot;
-  block_exclusive_sum<kScanThreads>(s, sw, &tot);
-  if (threadIdx.x == 0) tile_sums[blockIdx.x] = tot;
-}
+constexpr uint64_t kFlagAgg = 1ull << 32, kFlagPrefix = 2ull << 32;
 
-// Pass 2: exclusive scan of the tile sums (single block); total -> *total_out.
-__global__ void __launch_bounds__(1024) k_scan_tiles(int32_t* tile_sums, int64_t ntiles, int32_t* total_out);
-
-// Pass 3: rescan every tile with its offset; st(i, exclusive_prefix, value).
 template <class Load, class Store>
-__global__ void __launch_bounds__(kScanThreads) k_scan_apply(Load ld, Store st, int64_t n,
-                                                             const int32_t* tile_offsets) {
+__global__ void __launch_bounds__(kScanThreads) k_scan_lookback(Load ld, Store st, int64_t n,
+                                                                unsigned long long* status,
+                                                                unsigned int* counter, int32_t* total_out) {
+  __shared__ int32_t sv[kScanTile + kScanTile / 32];
+  __shared__ int32_t sx[kScanTile + kScanTile / 32];
   __shared__ int32_t sw[33];
-  const int64_t base = (int64_t)blockIdx.x * kScanTile + (int64_t)threadIdx.x * kScanPerThread;
-  int32_t v[kScanPerThread];
-  int32_t s = 0;
+  __shared__ int32_t s_prefix;
+  __shared__ unsigned int s_tile;
+  if (threadIdx.x == 0) s_tile = atomicAdd(counter, 1u);
+  __syncthreads();
+  const int64_t tile = s_tile;
+  const int64_t base = tile * kScanTile;
 #pragma unroll
-  for (int k = 0; k < kScanPerThread; ++k) {
-    int64_t i = base + k;
-    v[k] = i < n ? ld(i) : 0;
-    s += v[k];
+  for (int k = 0; k < kScanItems; ++k) {
+    const int li = k * kScanThreads + threadIdx.x;
+    const int64_t i = base + li;
+    sv[scan_pad(li)] = i < n ? ld(i) : 0;
   }
-  int32_t tot;
-  int32_t run = block_exclusive_sum<kScanThreads>(s, sw, &tot) + tile_offsets[blockIdx.x];
+  __syncthreads();
+  int32_t v[kScanItems];
+  int32_t sum = 0;
 #pragma unroll
-  for (int k = 0; k < kScanPerThread; ++k) {
-    int64_t i = base + k;
-    if (i < n) st(i, run, v[k]);
+  for (int k = 0; k < kScanItems; ++k) {
+    v[k] = sv[scan_pad(threadIdx.x * kScanItems + k)];
+    sum += v[k];
+  }
+  int32_t agg;
+  int32_t run = block_exclusive_sum<kScanThreads>(sum, sw, &agg);
+  if (threadIdx.x == 0) {
+    volatile unsigned long long* vs = status;
+    if (tile == 0) {
+      __threadfence();
+      vs[0] = kFlagPrefix | (uint32_t)agg;
+      s_prefix = 0;
+    } else {
+      vs[tile] = kFlagAgg | (uint32_t)agg;
+      __threadfence();
+      int32_t excl = 0;
+      int64_t p = tile - 1;
+      while (true) {
+        unsigned long long w = vs[p];
+        if ((w >> 32) == 0) continue;        // not yet published: spin
+        excl += (int32_t)(uint32_t)w;
+        if ((w >> 32) == 2) break;
+        --p;
+      }
+      __threadfence();
+      vs[tile] = kFlagPrefix | (uint32_t)(excl + agg);
+      s_prefix = excl;
+    }
+    if (base + kScanTile >= n && total_out) *total_out = s_prefix + agg;
+  }
+  __syncthreads();
+  run += s_prefix;
+#pragma unroll
+  for (int k = 0; k < kScanItems; ++k) {
+    sx[scan_pad(threadIdx.x * kScanItems + k)] = run;
     run += v[k];
   }
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < kScanItems; ++k) {
+    const int li = k * kScanThreads + threadIdx.x;
+    const int64_t i = base + li;
+    if (i < n) st(i, sx[scan_pad(li)], sv[scan_pad(li)]);
+  }
 }
 
-// Device-wide exclusive scan driven by functors.  ws: int32[scan_ws_elems(n)].
+// Device-wide exclusive scan driven by functors.  ws: int32[scan_ws_elems(n)] (any content).
 // The total is written to *total_out (device).
 template <class Load, class Store>
 buffalo_status device_scan(Load ld, Store st, int64_t n, int32_t* ws, int32_t* total_out,
                            cudaStream_t s) {
-  int64_t ntiles = ceil_div(n > 0 ? n : 1, kScanTile);
-  k_scan_reduce<<<(unsigned)ntiles, kScanThreads, 0, s>>>(ld, n, ws);
-  BF_LAUNCHED("k_scan_reduce");
-  k_scan_tiles<<<1, 1024, 0, s>>>(ws, ntiles, total_out);
-  BF_LAUNCHED("k_scan_tiles");
-  k_scan_apply<<<(unsigned)ntiles, kScanThreads, 0, s>>>(ld, st, n, ws);
-  BF_LAUNCHED("k_scan_apply");
+  const int64_t ntiles = ceil_div(n > 0 ? n : 1, kScanTile);
+  BF_CUDA(cudaMemsetAsync(ws, 0, sizeof(unsigned long long) * (ntiles + 1), s));
+  unsigned long long* status = reinterpret_cast<unsigned long long*>(ws);
+  unsigned int* counter = reinterpret_cast<unsigned int*>(status + ntiles);
+  k_scan_lookback<<<(unsigned)ntiles, kScanThreads, 0, s>>>(ld, st, n, status, counter, total_out);
+  BF_LAUNCHED("k_scan_lookback");
+  return BUFFALO_OK;
+}
+
+// Integer count (sum of a 0/1 or small functor) over [0, n) into *total (zeroed first).
+template <class Load>
+__global__ void __launch_bounds__(256) k_count_sum(Load ld, int64_t n, int32_t* total) {
+  int32_t s = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    s += ld(i);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0 && s) atomicAdd(total, s);
+}
+template <class Load>
+buffalo_status device_count(Load ld, int64_t n, int32_t* total, cudaStream_t s) {
+  BF_CUDA(cudaMemsetAsync(total, 0, sizeof(int32_t), s));
+  if (n <= 0) return BUFFALO_OK;
+  k_count_sum<<<grid_for(n, 256), 256, 0, s>>>(ld, n, total);
+  BF_LAUNCHED("k_count_sum");
   return BUFFALO_OK;
 }
 

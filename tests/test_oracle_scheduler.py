@@ -117,14 +117,14 @@ def test_fig9_grouping_structure():
 def test_mem_model_hand_instance():
     # L = 1, n = [5, 2], e = [3], dims = [4, 3]; every buffer rounds up to 256 B:
     # blocks: row_ptr, heavy, col_local, src_global, col_global = 5 * 256 = 1280
-    # build frame: totals 256 + scan ws R(4*(ceil(257/16384)+2)) = 256 + partition counts
+    # build frame: totals 256 + scan ws R(8*(ceil(257/4096)+2)) = 256 + partition counts
     #              R(4*(256+1)) = 1280  -> 1792
     # acts: agg R(2*8*4) + logits R(2*8*4) = 512
     # bwd frame l=1: dH_1 256 + dW partials R(1*3*8*4) 256 + db partials R(1*8*4) 256 = 768
     assert O.mem_model([5, 2], [3], [4, 3], O.FP32) == (1280 + 512 + 768, 1280 + 512 + 1792)
     # a wide layer: n = [40000, 20000], e = [100000], dims = [64, 32]
     # blocks: R(80004)=80128, R(80000)=80128, R(400000)=400128, R(160000)=160000, col_global 400128
-    # build: 256 + R(4*(ceil(120001/16384)+2)) + counts R(4*(256*30+1)) = 256 + 256 + 30976
+    # build: 256 + R(8*(ceil(120001/4096)+2)) + counts R(4*(256*30+1)) = 256 + 256 + 30976
     # acts: agg R(20000*64*4)=5120000, logits R(20000*32*4)=2560000
     # bwd: dH R(20000*32*4)=2560000; splits: tiles=1*2 -> min(148, 40) = 40;
     #      dW R(40*32*128*4)=655360; db R(40*32*4)=5120
