@@ -137,38 +137,35 @@ struct Item {
   int64_t O, E, I, M, w;
 };
 
-// Item statistics (R13): build the item's blocks alone (sizes only) on the GPU.
-static buffalo_status item_stats(const buffalo_graph* g, const int32_t* ids, int64_t count,
-                                 const buffalo_sampler* sp, const buffalo_model* m, char* ws,
-                                 int64_t ws_bytes, Item* it, cudaStream_t s) {
+// Item statistics (R13, R15): exact layer sizes of up to 64 items per pass (mask_stats), then
+// O = #seeds, E = e_L, I = n_{L-1} and M_est = hi of the memory model.
+static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_ids, std::vector<Item>& items,
+                                  size_t first, size_t count, const buffalo_sampler* sp, const buffalo_model* m,
+                                  char* ws, int64_t ws_bytes, bool& masks_clean, cudaStream_t s) {
   const int L = m->num_layers;
-  Arena A;
-  A.base = ws;
-  A.cap = ws_bytes;
-  int64_t n[BUFFALO_MAX_LAYERS + 1], e[BUFFALO_MAX_LAYERS];
-  const int32_t* dst = ids;
-  int64_t nd = count;
-  for (int l = L; l >= 1; --l) {
-    buffalo_block b;
-    buffalo_status st = build_layer(g, dst, nd, sp->fanout[l - 1], (uint32_t)(L - l + 1), sp->seed, l,
-                                    true, A, &b, s);
-    if (st == BUFFALO_ERR_CAPACITY || A.overflow) {
-      set_error("bucketize workspace too small (need > %lld bytes)", (long long)A.need);
-      return BUFFALO_ERR_CAPACITY;
+  for (size_t b0 = first; b0 < first + count; b0 += 64) {
+    const int nit = (int)std::min<size_t>(64, first + count - b0);
+    int64_t starts[65];
+    for (int k = 0; k < nit; ++k) starts[k] = items[b0 + k].start;
+    starts[nit] = items[b0 + nit - 1].start + items[b0 + nit - 1].count;
+    for (int k = 0; k + 1 < nit; ++k)
+      if (items[b0 + k].start + items[b0 + k].count != items[b0 + k + 1].start) {
+        set_error("internal: items of a statistics pass must be adjacent");
+        return BUFFALO_ERR_INVALID_ARG;
+      }
+    static thread_local int64_t nh[64][BUFFALO_MAX_LAYERS + 1], eh[64][BUFFALO_MAX_LAYERS];
+    BF_CHECK(mask_stats(g, sorted_ids, starts, nit, sp, L, ws, ws_bytes, masks_clean, nh, eh, s));
+    masks_clean = true;
+    for (int k = 0; k < nit; ++k) {
+      Item& it = items[b0 + k];
+      int64_t lo, hi;
+      mem_model(L, nh[k], eh[k], m, &lo, &hi);
+      it.O = it.count;
+      it.E = eh[k][L - 1];
+      it.I = nh[k][L - 1];
+      it.M = hi;
     }
-    BF_CHECK(st);
-    n[l] = nd;
-    e[l - 1] = b.n_edges;
-    dst = b.src_global;
-    nd = b.n_src;
   }
-  n[0] = nd;
-  int64_t lo, hi;
-  mem_model(L, n, e, m, &lo, &hi);
-  it->O = count;
-  it->E = e[L - 1];
-  it->I = n[L - 1];
-  it->M = hi;
   return BUFFALO_OK;
 }
 
@@ -190,19 +187,6 @@ __global__ void k_scatter_segments(const int64_t* __restrict__ seg, const int32_
     group_seeds[off + t] = sorted_ids[start + t];
     group_of_seed[order[start + t]] = (int32_t)grp;
   }
-}
-
-static int64_t stats_arena_bound(const buffalo_graph* g, int64_t n_seeds, const buffalo_sampler* sp, int L) {
-  int64_t nl = n_seeds, total = 0, frame = 0;
-  for (int l = L; l >= 1; --l) {
-    const int f = sp->fanout[l - 1];
-    int64_t el = f > 0 ? std::min<int64_t>(g->nnz, nl * f) : g->nnz;
-    int64_t nm = std::min<int64_t>(g->num_nodes, nl + el);
-    total += R(4 * (nl + 1)) + R(4 * nm);
-    frame = std::max(frame, build_frame_bytes(nl, el, l, true));
-    nl = nm;
-  }
-  return total + frame;
 }
 
 static int64_t bucketize_fixed_bytes(int64_t S, int F, int k_max) {
@@ -258,8 +242,7 @@ buffalo_status buffalo_estimate_mem(int32_t num_layers, const int64_t* n, const 
 size_t buffalo_bucketize_workspace_bytes(const buffalo_graph* g, int64_t n_seeds,
                                          const buffalo_sampler* s, const buffalo_model* m) {
   if (!g || !s || !m) return 0;
-  return (size_t)(bucketize_fixed_bytes(n_seeds, s->cutoff_F, 4096) +
-                  stats_arena_bound(g, n_seeds, s, m->num_layers));
+  return (size_t)(bucketize_fixed_bytes(n_seeds, s->cutoff_F, 4096) + mask_stats_bytes(g->num_nodes, m->num_layers));
 }
 
 buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, int64_t S,
@@ -304,16 +287,17 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
   std::vector<int64_t> bstart(F + 2, 0);
   for (int b = 0; b <= F; ++b) bstart[b + 1] = bstart[b] + plan->hist_h[b];
 
-  // a2: per-bucket statistics and estimates (K-independent)
+  // a2: per-bucket statistics and estimates (K-independent); item k = degree bucket k
+  bool masks_clean = false;
   std::vector<Item> bucket_item(F + 1);
+  for (int d = 0; d <= F; ++d) bucket_item[d] = Item{d, 0, bstart[d], plan->hist_h[d], 0, 0, 0, 0, 0};
+  BF_CHECK(items_stats(g, sorted_ids, bucket_item, 0, F + 1, sp, m, stats_ws, stats_bytes, masks_clean, s));
   std::vector<int> non_split;
   int64_t sum_M_all = 0, sum_w = 0, max_w = 0;
   for (int d = 0; d <= F; ++d) {
     if (plan->hist_h[d] == 0) continue;
-    Item it{d, 0, bstart[d], plan->hist_h[d], 0, 0, 0, 0, 0};
-    BF_CHECK(item_stats(g, sorted_ids + it.start, it.count, sp, m, stats_ws, stats_bytes, &it, s));
+    Item& it = bucket_item[d];
     it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
-    bucket_item[d] = it;
     sum_M_all += it.M;
     if (d != F) {
       non_split.push_back(d);
@@ -337,16 +321,17 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
       if (exploded) {
         // SplitExplosionBucket: K contiguous pieces, the first (O mod K) one seed larger (R8)
         const int64_t O = itF.count, base = O / K, extra = O % K;
+        std::vector<Item> pieces;
         int64_t st0 = itF.start;
         for (int k = 0; k < K; ++k) {
           const int64_t len = base + (k < extra ? 1 : 0);
-          if (len > 0) {
-            Item it{F, k, st0, len, 0, 0, 0, 0, 0};
-            BF_CHECK(item_stats(g, sorted_ids + st0, len, sp, m, stats_ws, stats_bytes, &it, s));
-            it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
-            items.push_back(it);
-          }
+          if (len > 0) pieces.push_back(Item{F, k, st0, len, 0, 0, 0, 0, 0});
           st0 += len;
+        }
+        BF_CHECK(items_stats(g, sorted_ids, pieces, 0, pieces.size(), sp, m, stats_ws, stats_bytes, masks_clean, s));
+        for (Item& it : pieces) {
+          it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
+          items.push_back(it);
         }
       } else {
         items.push_back(itF);

@@ -368,4 +368,164 @@ buffalo_status seed_bucketing(const buffalo_graph* g, const int32_t* seeds, int6
   return BUFFALO_OK;
 }
 
+// ------------------------------------------------------------------ a2: item statistics
+// Block sizes of up to 64 items (disjoint seed sets) at once, by propagating item bitmasks
+// top-down: a node's mask at layer l-1 is the OR of the masks of the layer-l nodes that have it
+// as a dst (prefix) or a sampled neighbour.  Because a node's sample depends only on (seed,
+// node, hop) (R2), item k's node set at every layer is exactly the one of its own blocks, so
+// n_l(k) = #nodes with bit k, e_l(k) = sum of D over them — the sizes build_layer would give.
+__device__ __forceinline__ void mask_accumulate(uint64_t mask, int64_t D, unsigned long long* sn,
+                                                unsigned long long* se) {
+  while (mask) {
+    const int k = __ffsll((long long)mask) - 1;
+    mask &= mask - 1;
+    atomicAdd(&sn[k], 1ull);
+    if (se) atomicAdd(&se[k], (unsigned long long)D);
+  }
+}
+
+__global__ void __launch_bounds__(256) k_mask_seed(const int32_t* __restrict__ ids, int64_t n,
+                                                   const int64_t* __restrict__ item_start, int nitems,
+                                                   unsigned long long* __restrict__ m, int32_t* __restrict__ act) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    int k = 0;
+    while (k + 1 < nitems && item_start[k + 1] - item_start[0] <= i) ++k;
+    const int32_t v = ids[i];
+    m[v] = 1ull << k;
+    act[i] = v;
+  }
+}
+
+// One layer: warp per active node v of layer l; accumulates n_l, e_l per item and ORs v's mask
+// into layer l-1 for v itself and its sampled neighbours, appending first touches to act_out.
+__global__ void __launch_bounds__(256) k_mask_layer(const int32_t* __restrict__ act, int64_t n_act,
+                                                    const unsigned long long* __restrict__ m_in,
+                                                    unsigned long long* __restrict__ m_out,
+                                                    int32_t* __restrict__ act_out, int32_t* __restrict__ n_out,
+                                                    const int64_t* __restrict__ grow, const int32_t* __restrict__ gcol,
+                                                    int32_t f, uint32_t hop, uint64_t seed,
+                                                    unsigned long long* __restrict__ gn, unsigned long long* __restrict__ ge) {
+  __shared__ unsigned long long sn[64], se[64];
+  if (threadIdx.x < 64) { sn[threadIdx.x] = 0; se[threadIdx.x] = 0; }
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n_act; i += warps) {
+    const uint32_t v = (uint32_t)act[i];
+    const unsigned long long mask = m_in[v];
+    const int64_t beg = grow[v];
+    const int64_t deg = grow[v + 1] - beg;
+    const int64_t D = (f > 0 && deg > f) ? f : deg;
+    if (lane == 0) {
+      mask_accumulate(mask, D, sn, se);
+      if (atomicOr(&m_out[v], mask) == 0ull) act_out[atomicAdd(n_out, 1)] = (int32_t)v;
+    }
+    if (f <= 0 || deg <= f) {
+      for (int64_t k = lane; k < deg; k += 32) {
+        const int32_t u = gcol[beg + k];
+        if (atomicOr(&m_out[u], mask) == 0ull) act_out[atomicAdd(n_out, 1)] = u;
+      }
+    } else {
+      const uint32_t j = (uint32_t)(deg - f) + (uint32_t)lane;
+      uint32_t r = 0;
+      if (lane < f) r = __umulhi(sample_draw(seed, v, hop, (uint32_t)lane), j + 1u);
+      int32_t S = -1;
+      for (int t = 0; t < f; ++t) {
+        const int32_t cand = (int32_t)__shfl_sync(0xffffffffu, r, t);
+        const unsigned present = __ballot_sync(0xffffffffu, lane < t && S == cand);
+        if (lane == t) S = present ? (int32_t)((uint32_t)(deg - f) + (uint32_t)t) : cand;
+      }
+      if (lane < f) {
+        const int32_t u = gcol[beg + S];
+        if (atomicOr(&m_out[u], mask) == 0ull) act_out[atomicAdd(n_out, 1)] = u;
+      }
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x < 64) {
+    if (sn[threadIdx.x]) atomicAdd(&gn[threadIdx.x], sn[threadIdx.x]);
+    if (se[threadIdx.x]) atomicAdd(&ge[threadIdx.x], se[threadIdx.x]);
+  }
+}
+
+__global__ void __launch_bounds__(256) k_mask_count(const int32_t* __restrict__ act, int64_t n_act,
+                                                    unsigned long long* __restrict__ m,
+                                                    unsigned long long* __restrict__ gn, int clear) {
+  __shared__ unsigned long long sn[64];
+  if (threadIdx.x < 64) sn[threadIdx.x] = 0;
+  __syncthreads();
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_act; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t v = act[i];
+    if (gn) mask_accumulate(m[v], 0, sn, nullptr);
+    if (clear) m[v] = 0ull;
+  }
+  __syncthreads();
+  if (gn && threadIdx.x < 64 && sn[threadIdx.x]) atomicAdd(&gn[threadIdx.x], sn[threadIdx.x]);
+}
+
+int64_t mask_stats_bytes(int64_t N, int L) {
+  return 2 * R(8 * N) + 2 * R(4 * N) + R(8 * 64 * (2 * L + 1)) + R(64) + R(8 * 65);
+}
+
+buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, const int64_t* item_start_h,
+                          int nitems, const buffalo_sampler* sp, int L, char* ws, int64_t ws_bytes,
+                          bool masks_clean, int64_t (*n_h)[BUFFALO_MAX_LAYERS + 1],
+                          int64_t (*e_h)[BUFFALO_MAX_LAYERS], cudaStream_t s) {
+  const int64_t N = g->num_nodes;
+  if (ws_bytes < mask_stats_bytes(N, L)) {
+    set_error("bucketize workspace too small for the item statistics");
+    return BUFFALO_ERR_CAPACITY;
+  }
+  char* q = ws;
+  unsigned long long* m[2] = {(unsigned long long*)q, (unsigned long long*)(q + R(8 * N))};
+  q += 2 * R(8 * N);
+  int32_t* act[2] = {(int32_t*)q, (int32_t*)(q + R(4 * N))};
+  q += 2 * R(4 * N);
+  unsigned long long* acc = (unsigned long long*)q; q += R(8 * 64 * (2 * L + 1));
+  int32_t* cnt = (int32_t*)q; q += R(64);
+  int64_t* starts = (int64_t*)q;
+  if (!masks_clean) {
+    BF_CUDA(cudaMemsetAsync(m[0], 0, 2 * R(8 * N), s));
+  }
+  BF_CUDA(cudaMemsetAsync(acc, 0, sizeof(unsigned long long) * 64 * (2 * L + 1), s));
+  BF_CUDA(cudaMemcpyAsync(starts, item_start_h, sizeof(int64_t) * (nitems + 1), cudaMemcpyHostToDevice, s));
+  const int64_t n_seed = item_start_h[nitems] - item_start_h[0];
+  // acc layout: n[l] at acc + 64*l (l = 0..L), e[l-1] at acc + 64*(L+1) + 64*(l-1)
+  unsigned long long* accn = acc;
+  unsigned long long* acce = acc + 64 * (L + 1);
+  k_mask_seed<<<grid_for(n_seed, 256), 256, 0, s>>>(sorted_ids + item_start_h[0], n_seed, starts, nitems, m[0], act[0]);
+  BF_LAUNCHED("k_mask_seed");
+  int64_t n_act = n_seed;
+  int cur = 0;
+  for (int l = L; l >= 1; --l) {
+    BF_CUDA(cudaMemsetAsync(cnt, 0, sizeof(int32_t), s));
+    if (n_act > 0) {
+      k_mask_layer<<<grid_for(n_act * 32, 256, 16), 256, 0, s>>>(
+          act[cur], n_act, m[cur], m[cur ^ 1], act[cur ^ 1], cnt, g->row_ptr, g->col, sp->fanout[l - 1],
+          (uint32_t)(L - l + 1), sp->seed, accn + 64 * l, acce + 64 * (l - 1));
+      BF_LAUNCHED("k_mask_layer");
+      // masks of layer l are no longer needed: clear them for reuse by layer l-2
+      k_mask_count<<<grid_for(n_act, 256), 256, 0, s>>>(act[cur], n_act, m[cur], nullptr, 1);
+      BF_LAUNCHED("k_mask_count");
+    }
+    int32_t na = 0;
+    BF_CUDA(cudaMemcpyAsync(&na, cnt, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    BF_CUDA(cudaStreamSynchronize(s));
+    n_act = na;
+    cur ^= 1;
+  }
+  if (n_act > 0) {
+    k_mask_count<<<grid_for(n_act, 256), 256, 0, s>>>(act[cur], n_act, m[cur], accn, 1);
+    BF_LAUNCHED("k_mask_count");
+  }
+  unsigned long long host[64 * (2 * BUFFALO_MAX_LAYERS + 1)];
+  BF_CUDA(cudaMemcpyAsync(host, acc, sizeof(unsigned long long) * 64 * (2 * L + 1), cudaMemcpyDeviceToHost, s));
+  BF_CUDA(cudaStreamSynchronize(s));
+  for (int k = 0; k < nitems; ++k) {
+    for (int l = 0; l <= L; ++l) n_h[k][l] = (int64_t)host[64 * l + k];
+    for (int l = 1; l <= L; ++l) e_h[k][l - 1] = (int64_t)host[64 * (L + 1) + 64 * (l - 1) + k];
+  }
+  return BUFFALO_OK;
+}
+
 }  // namespace buffalo
