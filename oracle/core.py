@@ -175,6 +175,7 @@ HEAVY_T = 128          # rows with D > HEAVY_T go through the cooperative long-t
 FP32, BF16 = 0, 1
 SCAN_TILE = 4096       # elements per tile of the implementation's device-wide scans
 PART_TILE = 4096       # elements per tile of its stable radix/bin partition passes
+DB_SPLITS = 296        # row splits of the bf16 path's deterministic db reduction
 
 
 def _R(x):
@@ -256,7 +257,7 @@ def mem_model(n, e, dims, act_dtype=FP32):
                 frame += _R(e[l - 1] // (HEAVY_T + 1) * pitch(dims[l]) * 2)  # long-tail sums
             S = tc_dw_splits(n[l], dims[l], dims[l - 1])
             Dp = _ceil(dims[l - 1], 64) * 64
-            frame += _R(S * dims[l] * 2 * Dp * 4) + _R(S * pitch(dims[l]) * 4)          # dW, db partials
+            frame += _R(S * dims[l] * 2 * Dp * 4) + _R(DB_SPLITS * dims[l] * 4)         # dW, db partials
         bwd = max(bwd, frame)
     lo = blocks + acts + bwd
     hi = blocks + acts + max(bwd, build)

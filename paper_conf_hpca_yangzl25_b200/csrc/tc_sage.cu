@@ -619,16 +619,25 @@ buffalo_status tc_sage_fwd(const FwdArgs& a, cudaStream_t s) {
 }
 
 // ================================================================== backward
-// dZ preparation: dZ = dH * 1[H > 0] in place (l < L); bf16 copies dZ and dZ / D(i).
+// dZ preparation: dZ = dH * 1[H > 0] in place (l < L); bf16 copies of dZ and dZ / D(i); and
+// the column sums of dZ (db) as per-CTA partials over a fixed row split (deterministic).
+constexpr int kDbSplits = 296;
+
 template <class TH>
-__global__ void k_dz_prep(float* __restrict__ dz, int64_t ldz, const TH* __restrict__ h, int64_t ldh,
-                          const int32_t* __restrict__ rp, int64_t n, int d, int dp,
-                          __nv_bfloat16* __restrict__ zb, __nv_bfloat16* __restrict__ zs) {
-  const int per_row = dp / 8;
-  const int64_t total = n * per_row;
-  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t i = t / per_row;
-    const int c0 = (int)(t - i * per_row) * 8;
+__global__ void __launch_bounds__(256) k_dz_prep(float* __restrict__ dz, int64_t ldz, const TH* __restrict__ h,
+                                                 int64_t ldh, const int32_t* __restrict__ rp, int64_t n, int d,
+                                                 int dp, __nv_bfloat16* __restrict__ zb,
+                                                 __nv_bfloat16* __restrict__ zs, float* __restrict__ db_part) {
+  __shared__ float red[256][9];
+  const int per_row = dp / 8;                       // <= 32 column groups of 8
+  const int rows_per_pass = 256 / per_row;
+  const int cg = threadIdx.x % per_row, rsub = threadIdx.x / per_row;
+  const int64_t rows_per_cta = (n + gridDim.x - 1) / gridDim.x;
+  const int64_t r_beg = (int64_t)blockIdx.x * rows_per_cta, r_end = min(n, r_beg + rows_per_cta);
+  float db[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+  const bool active = rsub < rows_per_pass;
+  for (int64_t i = r_beg + rsub; active && i < r_end; i += rows_per_pass) {
+    const int c0 = cg * 8;
     float v[8];
     const float4 a0 = *reinterpret_cast<const float4*>(dz + i * ldz + c0);
     const float4 a1 = *reinterpret_cast<const float4*>(dz + i * ldz + c0 + 4);
@@ -647,8 +656,10 @@ __global__ void k_dz_prep(float* __restrict__ dz, int64_t ldz, const TH* __restr
       }
     }
 #pragma unroll
-    for (int k = 0; k < 8; ++k)
+    for (int k = 0; k < 8; ++k) {
       if (c0 + k >= d) v[k] = 0.f;
+      db[k] += v[k];
+    }
     *reinterpret_cast<uint4*>(zb + i * dp + c0) = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
                                                               pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
     if (zs) {
@@ -659,6 +670,17 @@ __global__ void k_dz_prep(float* __restrict__ dz, int64_t ldz, const TH* __restr
                                                                 pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
     }
   }
+#pragma unroll
+  for (int k = 0; k < 8; ++k) red[threadIdx.x][k] = db[k];
+  __syncthreads();
+  if (threadIdx.x < per_row) {
+    for (int k = 0; k < 8; ++k) {
+      float t = 0.f;
+      for (int r = 0; r < rows_per_pass; ++r) t += red[r * per_row + threadIdx.x][k];
+      const int c = threadIdx.x * 8 + k;
+      if (c < d) db_part[(int64_t)blockIdx.x * d + c] = t;
+    }
+  }
 }
 
 // dW (tensor cores): D[m][n'] = sum_r dZ[r][m] * Afwd[r][n'] over a row range, both operands
@@ -667,7 +689,7 @@ __global__ void k_dz_prep(float* __restrict__ dz, int64_t ldz, const TH* __restr
 constexpr int kDwThreads = 128;
 constexpr int kDwRows = 64;                       // K per stage
 constexpr int kDwStrip = kDwRows * 128;           // one 64-column MN strip of 64 rows (8 KB)
-constexpr int kDwStages = 2;
+constexpr int kDwStages = 3;
 
 struct TcDwParams {
   const __nv_bfloat16* zb;  int64_t ldz;          // dZ (bf16) [n][ldz]
@@ -677,8 +699,6 @@ struct TcDwParams {
   int d_out, d_in, pitch_in, pz, Dp, NT;          // NT: n' columns per CTA tile (<= 256)
   int64_t rows_per_split;
   float* part;                                    // [S][d_out][2 Dp]
-  const float* dz; int64_t lddz;                  // fp32 dZ (for db)
-  float* db_part;                                 // [S][d_out] column sums (CTAs with n-tile 0)
 };
 
 // MN-major SWIZZLE_128B descriptor: LBO = stride between 64-element MN strips, SBO = 8 K-rows.
@@ -696,6 +716,15 @@ __host__ __device__ constexpr uint32_t idesc_bf16_mn(int n) {
          ((uint32_t)(128 >> 4) << 24);
 }
 
+__device__ __forceinline__ void cp_async16(void* dst, const void* src, bool valid) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src),
+               "r"(valid ? 16 : 0)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
 template <class TS>
 __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -706,7 +735,7 @@ __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
   uint64_t* empty = full + kDwStages;
   uint64_t* done = empty + kDwStages;
   uint32_t* tmem_slot = (uint32_t*)(done + 1);
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int warp = threadIdx.x >> 5;
   const int m0 = blockIdx.x * 128, n0 = blockIdx.y * p.NT;
   const int64_t r_beg = (int64_t)blockIdx.z * p.rows_per_split;
   const int64_t r_end = min(p.n, r_beg + p.rows_per_split);
@@ -723,13 +752,10 @@ __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
   const uint32_t tmem = *tmem_slot;
   const TS* __restrict__ selfp = (const TS*)p.self_;
   const uint32_t idesc = idesc_bf16_mn(p.NT);
-  // db: CTAs of n-tile 0 also sum their row range of fp32 dZ column by column (thread = column)
-  const bool do_db = blockIdx.y == 0;
-  const int mcol = m0 + threadIdx.x;
-  float dbs = 0.f;
-  for (int c = 0; c < nchunks; ++c) {
+  const void* dummy = p.zb;            // any global address: zero-fill copies read 0 bytes
+
+  auto load_chunk = [&](int c) {
     const int st = c % kDwStages;
-    if (c >= kDwStages) mbar_wait(&empty[st], (uint32_t)(((c / kDwStages) - 1) & 1));
     uint8_t* sa = smem + st * stage_bytes;
     uint8_t* sb = sa + nstripA * kDwStrip;
     const int64_t rbase = r_beg + (int64_t)c * kDwRows;
@@ -738,9 +764,9 @@ __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
       const int k = u >> 4, j = u & 15;
       const int64_t r = rbase + k;
       const int m = m0 + j * 8;
-      uint4 v = make_uint4(0u, 0u, 0u, 0u);
-      if (r < r_end && m < p.pz) v = *reinterpret_cast<const uint4*>(p.zb + r * p.ldz + m);
-      *reinterpret_cast<uint4*>(sa + (j >> 3) * kDwStrip + k * 128 + (((j & 7) ^ (k & 7)) << 4)) = v;
+      const bool ok = r < r_end && m < p.pz;
+      cp_async16(sa + (j >> 3) * kDwStrip + k * 128 + (((j & 7) ^ (k & 7)) << 4),
+                 ok ? (const void*)(p.zb + r * p.ldz + m) : dummy, ok);
     }
     // B: Afwd rows, NT n'-columns
     const int pcs = p.NT / 8;
@@ -748,47 +774,77 @@ __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
       const int k = u / pcs, j = u % pcs;
       const int64_t r = rbase + k;
       const int nn = n0 + j * 8;
-      uint4 v = make_uint4(0u, 0u, 0u, 0u);
-      if (r < r_end) {
-        if (nn < p.Dp) {
-          if (nn < p.pitch_in) {
-            const int64_t rr = p.gidx ? (int64_t)p.gidx[r] : r;
-            if constexpr (sizeof(TS) == 2) {
-              v = *reinterpret_cast<const uint4*>(selfp + rr * p.lds + nn);
-            } else {
+      uint8_t* dst = sb + (j >> 3) * kDwStrip + k * 128 + (((j & 7) ^ (k & 7)) << 4);
+      if constexpr (sizeof(TS) == 2) {
+        const void* src = dummy;
+        bool ok = false;
+        if (r < r_end) {
+          if (nn < p.Dp) {
+            if (nn < p.pitch_in) {
+              const int64_t rr = p.gidx ? (int64_t)p.gidx[r] : r;
+              src = selfp + rr * p.lds + nn;
+              ok = true;
+            }
+          } else if (nn - p.Dp < p.pitch_in) {
+            src = p.agg + r * p.lda + (nn - p.Dp);
+            ok = true;
+          }
+        }
+        cp_async16(dst, src, ok);
+      } else {
+        uint4 v = make_uint4(0u, 0u, 0u, 0u);
+        if (r < r_end) {
+          if (nn < p.Dp) {
+            if (nn < p.pitch_in) {
+              const int64_t rr = p.gidx ? (int64_t)p.gidx[r] : r;
               const float4 a0 = *reinterpret_cast<const float4*>(selfp + rr * p.lds + nn);
               const float4 a1 = *reinterpret_cast<const float4*>(selfp + rr * p.lds + nn + 4);
               v = make_uint4(pack_bf16x2(a0.x, a0.y), pack_bf16x2(a0.z, a0.w), pack_bf16x2(a1.x, a1.y),
                              pack_bf16x2(a1.z, a1.w));
             }
+          } else if (nn - p.Dp < p.pitch_in) {
+            v = *reinterpret_cast<const uint4*>(p.agg + r * p.lda + (nn - p.Dp));
           }
-        } else if (nn - p.Dp < p.pitch_in) {
-          v = *reinterpret_cast<const uint4*>(p.agg + r * p.lda + (nn - p.Dp));
         }
+        *reinterpret_cast<uint4*>(dst) = v;
       }
-      *reinterpret_cast<uint4*>(sb + (j >> 3) * kDwStrip + k * 128 + (((j & 7) ^ (k & 7)) << 4)) = v;
     }
-    fence_proxy_async_smem();
-    mbar_arrive(&full[st]);
-    if (do_db && mcol < p.d_out) {
-      const int64_t r1 = min(r_end, rbase + kDwRows);
-      for (int64_t r = rbase; r < r1; ++r) dbs += p.dz[r * p.lddz + mcol];
-    }
-    if (threadIdx.x == 0) {
-      mbar_wait(&full[st], (uint32_t)((c / kDwStages) & 1));
-      tc_fence_after();
-      const uint32_t a_addr = smem_u32(sa), b_addr = smem_u32(sb);
+    cp_async_commit();
+  };
+  auto mma_chunk = [&](int c) {
+    const int st = c % kDwStages;
+    mbar_wait(&full[st], (uint32_t)((c / kDwStages) & 1));
+    tc_fence_after();
+    const uint32_t a_addr = smem_u32(smem + st * stage_bytes);
+    const uint32_t b_addr = a_addr + nstripA * kDwStrip;
 #pragma unroll
-      for (int kk = 0; kk < kDwRows / 16; ++kk)
-        umma_bf16(tmem, sw128_mn_desc(a_addr + kk * 2048, kDwStrip), sw128_mn_desc(b_addr + kk * 2048, kDwStrip),
-                  idesc, (c > 0 || kk > 0) ? 1u : 0u);
-      umma_commit(&empty[st]);
-      if (c == nchunks - 1) umma_commit(done);
+    for (int kk = 0; kk < kDwRows / 16; ++kk)
+      umma_bf16(tmem, sw128_mn_desc(a_addr + kk * 2048, kDwStrip), sw128_mn_desc(b_addr + kk * 2048, kDwStrip),
+                idesc, (c > 0 || kk > 0) ? 1u : 0u);
+    umma_commit(&empty[st]);
+    if (c == nchunks - 1) umma_commit(done);
+  };
+  // pipeline: chunk c's copies are in flight while chunk c-1 is completed, fenced and issued
+  for (int c = 0; c < nchunks; ++c) {
+    if (c >= kDwStages) mbar_wait(&empty[c % kDwStages], (uint32_t)(((c / kDwStages) - 1) & 1));
+    load_chunk(c);
+    if (c >= 1) {
+      cp_async_wait<1>();
+      fence_proxy_async_smem();
+      mbar_arrive(&full[(c - 1) % kDwStages]);
+      if (threadIdx.x == 0) mma_chunk(c - 1);
+      __syncwarp();
     }
+  }
+  if (nchunks > 0) {
+    cp_async_wait<0>();
+    fence_proxy_async_smem();
+    mbar_arrive(&full[(nchunks - 1) % kDwStages]);
+    if (threadIdx.x == 0) mma_chunk(nchunks - 1);
     __syncwarp();
   }
-  if (do_db && mcol < p.d_out) p.db_part[(int64_t)blockIdx.z * p.d_out + mcol] = dbs;
   // epilogue: TMEM lanes = m rows, columns = n'
+  const int lane = threadIdx.x & 31;
   const int64_t K2 = 2 * (int64_t)p.Dp;
   float* P = p.part + (int64_t)blockIdx.z * p.d_out * K2;
   const int m = m0 + warp * 32 + lane;
@@ -899,7 +955,7 @@ int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int64_t e, int layer,
     b += R(n_dst * pitch_of(d_out) * 2);                              // dZ / D bf16
     b += R(e / (kHeavyT + 1) * pitch_of(d_out) * 2);                  // long-tail transposed sums
   }
-  b += R((int64_t)S * d_out * 2 * Dp * 4) + R((int64_t)S * pitch_of(d_out) * 4);
+  b += R((int64_t)S * d_out * 2 * Dp * 4) + R((int64_t)kDbSplits * d_out * 4);
   return b;
 }
 
@@ -925,8 +981,9 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * Dp * 4);
   float* db_part = (float*)q;
   if (n <= 0) return BUFFALO_OK;
-  k_dz_prep<__nv_bfloat16><<<grid_for(n * (dp / 8), 256), 256, 0, s>>>(
-      a.dh, a.ld_dh, a.last ? nullptr : (const __nv_bfloat16*)a.h_dst, a.ld_hdst, blk->row_ptr, n, d_out, dp, zb, zs);
+  k_dz_prep<__nv_bfloat16><<<kDbSplits, 256, 0, s>>>(
+      a.dh, a.ld_dh, a.last ? nullptr : (const __nv_bfloat16*)a.h_dst, a.ld_hdst, blk->row_ptr, n, d_out, dp, zb, zs,
+      db_part);
   BF_LAUNCHED("k_dz_prep");
   // dW and db
   TcDwParams w{};
@@ -937,11 +994,10 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   w.NT = (int)std::min<int64_t>(256, 2 * Dp);
   w.rows_per_split = ceil_div(n, S);
   w.part = dw_part;
-  w.dz = a.dh; w.lddz = a.ld_dh; w.db_part = db_part;
-  const int smem = kDwStages * (2 + w.NT / 64) * kDwStrip + 64 + 1024;
+  const int smem = kDwStages * (2 + w.NT / 64) * kDwStrip + 128 + 1024;
   dim3 grid((unsigned)ceil_div(d_out, 128), (unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
   static bool attr[2] = {false, false};
-  constexpr int kMaxDwSmem = kDwStages * (2 + 4) * kDwStrip + 64 + 1024;
+  constexpr int kMaxDwSmem = kDwStages * (2 + 4) * kDwStrip + 128 + 1024;
   if (a.in_bf16) {
     if (!attr[0]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr[0] = true; }
     k_tc_dw<__nv_bfloat16><<<grid, kDwThreads, smem, s>>>(w);
@@ -952,7 +1008,7 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   BF_LAUNCHED("k_tc_dw");
   k_reduce_dw<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, d_out, d_in, (int)Dp, a.dW);
   BF_LAUNCHED("k_reduce_dw");
-  k_reduce_db<<<1, 256, 0, s>>>(db_part, S, d_out, a.db);
+  k_reduce_db<<<1, 256, 0, s>>>(db_part, kDbSplits, d_out, a.db);
   BF_LAUNCHED("k_reduce_db");
   // dH_{l-1} = [dZ (rows < n_dst) || sum_{i in T(j)} dZ[i]/D(i)] [W_self; W_neigh]
   if (a.dh_src && blk->n_src > 0) {
