@@ -13,6 +13,17 @@ import torch
 from . import buffalo as B
 
 
+def own_groups(rank_of_group, rank):
+    """Groups this rank runs: those the scheduler's LPT assignment gave it (R24)."""
+    return [k for k in range(len(rank_of_group)) if int(rank_of_group[k]) == rank]
+
+
+def allreduce_grads(grad, world, group=None):
+    """The one data-path collective: sum of the flat gradient buffer over the ranks."""
+    if world > 1:
+        torch.distributed.all_reduce(grad, group=group)
+
+
 class DeviceGraph:
     """CSR graph resident in HBM (+ the node_map workspace the relabel kernels use)."""
 
@@ -166,8 +177,7 @@ class Trainer:
                     peak=blk.arena_peak, est_lo=blk.est_lo, est_hi=blk.est_hi)
 
     def allreduce(self):
-        if self.world > 1:
-            torch.distributed.all_reduce(self.params.grad, group=self.pg)
+        allreduce_grads(self.params.grad, self.world, self.pg)
 
     def step(self, lr):
         B.sgd_step(self.params.flat, self.params.grad, lr)
@@ -182,9 +192,7 @@ class Trainer:
             self._ensure_arena(max(mine) if mine else 1 << 20)
         sampler = self.sampler(epoch)
         groups = []
-        for k in range(K):
-            if ranks[k] != self.rank:
-                continue
+        for k in own_groups(ranks, self.rank):
             groups.append(self.microbatch(offs[k], int(offs[k + 1] - offs[k]), sampler))
         self.allreduce()
         self.step(lr)
