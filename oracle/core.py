@@ -254,7 +254,7 @@ def mem_model(n, e, dims, act_dtype=FP32):
             frame += _R(n[l] * pitch(dims[l]) * 2)              # dZ in bf16
             if l >= 2:
                 frame += _R(n[l] * pitch(dims[l]) * 2)          # dZ / D in bf16
-                frame += _R(e[l - 1] // (HEAVY_T + 1) * pitch(dims[l]) * 2)  # long-tail sums
+                frame += _R(n[l - 1] * pitch(dims[l]) * 2)      # transposed sums in bf16
             S = tc_dw_splits(n[l], dims[l], dims[l - 1])
             Dp = _ceil(dims[l - 1], 64) * 64
             frame += _R(S * dims[l] * 2 * Dp * 4) + _R(DB_SPLITS * dims[l] * 4)         # dW, db partials

@@ -14,6 +14,7 @@
 // (tcgen05.ld -> +bias -> ReLU -> store) after gathering tile t, so MMA latency hides under
 // the next gather.  Rows with D > kHeavyT were pre-aggregated by k_agg_heavy (sage.cu).
 #include <algorithm>
+#include <cstdlib>
 
 #include "tc_sage.cuh"
 
@@ -124,6 +125,15 @@ __device__ __forceinline__ void bf16x8_to_f32(const uint4& u, float* v) {
   }
 }
 
+__device__ __forceinline__ void cp_async16(void* dst, const void* src, bool valid) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src),
+               "r"(valid ? 16 : 0)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
 // ------------------------------------------------------------------ kernel configuration
 constexpr int kTileM = 128;
 constexpr int kKC = 64;                    // bf16 columns per K-chunk (one 128-B swizzle row)
@@ -144,6 +154,8 @@ struct TcFwdParams {
   const void* hs;            // self rows (fwd: = h)
   int64_t lds;
   const int32_t* perm;       // tile row order (degree-sorted dst) or null (natural order)
+  const __nv_bfloat16* agg_src;  // MODE 2: the aggregate half, bf16 rows [n_dst][ld_agg_src]
+  int64_t ld_agg_src;
   int64_t heavy_base;        // MODE 1: positions >= heavy_base are long-tail rows, pre-summed
   const __nv_bfloat16* heavy_buf;  // MODE 1: [pos - heavy_base][heavy_ld]
   int64_t heavy_ld;
@@ -372,19 +384,37 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
             const int r = u / pcs, pc = u % pcs;
             const int64_t pos = pos0 + r;
             const int col0 = c0 * kKC + pc * E;
-            float v[E];
-#pragma unroll
-            for (int k = 0; k < E; ++k) v[k] = 0.f;
+            int64_t hr = -1;
             if (pos < p.n_dst) {
               const int64_t row = row_of(pos);
-              if (row < p.self_rows && col0 < p.pitch_in) {
-                const int64_t hr = p.gidx ? (int64_t)p.gidx[row] : row;
-                ld_piece<TI>(hs + hr * p.lds + col0, v);
-              }
+              if (row < p.self_rows && col0 < p.pitch_in) hr = p.gidx ? (int64_t)p.gidx[row] : row;
             }
-            st_swz<E>(abuf + (pc / P) * kChunkBytesA, r, pc % P, v);
+            if constexpr (E == 8) {
+              const int off = r * 128 + (((pc % P) ^ (r & 7)) << 4);
+              cp_async16(abuf + (pc / P) * kChunkBytesA + off, hr >= 0 ? (const void*)(hs + hr * p.lds + col0) : p.h,
+                         hr >= 0);
+            } else {
+              float v[E];
+#pragma unroll
+              for (int k = 0; k < E; ++k) v[k] = 0.f;
+              if (hr >= 0) ld_piece<TI>(hs + hr * p.lds + col0, v);
+              st_swz<E>(abuf + (pc / P) * kChunkBytesA, r, pc % P, v);
+            }
           }
-        } else {
+        } else if (MODE == 2) {
+          // aggregate half precomputed (bf16 rows): plain copy
+          const int cb = (c0 - p.nkc_self) * kKC;
+          const int pcs = ncs * 8;
+          for (int u = threadIdx.x; u < kTileM * pcs; u += kGatherThreads) {
+            const int r = u / pcs, pc = u % pcs;
+            const int64_t pos = pos0 + r;
+            const int col0 = cb + pc * 8;
+            const bool ok = pos < p.n_dst && col0 < p.pitch_in;
+            const int off = r * 128 + (((pc & 7) ^ (r & 7)) << 4);
+            cp_async16(abuf + (pc >> 3) * kChunkBytesA + off,
+                       ok ? (const void*)(p.agg_src + row_of(pos) * p.ld_agg_src + col0) : (const void*)p.agg_src, ok);
+          }
+        } else if (MODE != 2) {
           // aggregate: one lane group per destination row, lane = 16-B column piece
           const int cbase = (c0 - p.nkc_self) * kKC;                 // first column of this slice
           const int need = min(ncs * P, (p.pitch_in - cbase + E - 1) / E);
@@ -475,6 +505,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
             }
           }
         }
+        asm volatile("cp.async.wait_all;" ::: "memory");
         fence_proxy_async_smem();
         mbar_arrive(&a_full[buf]);
       }
@@ -558,6 +589,113 @@ bool tc_fwd_supported(const FwdArgs& a) {
 
 buffalo_status launch_agg_heavy_bf16(const FwdArgs& a, cudaStream_t s);
 
+
+// ================================================================== high-occupancy gather
+// Aggregate (Alg. 2 l.8) as its own kernel: lane groups of LPR lanes (16 B each) own one row,
+// rows taken in degree-sorted order (perm) so a warp's rows have equal trip counts; indices of
+// a row are fetched LPR at a time and broadcast with shuffles, kU 16-B loads stay in flight per
+// lane; fp32 accumulation; MODE 0: mean (R21), MODE 1: plain sum (backward, dZ/D rows).
+// Rows with D > kHeavyT are skipped (pre-aggregated by the cooperative kernels).
+constexpr int kGU = 4;
+
+template <class TI, int MODE>
+__global__ void __launch_bounds__(256, 8) k_gather_rows(const int32_t* __restrict__ perm,
+                                                        const int32_t* __restrict__ rp,
+                                                        const int32_t* __restrict__ col, int64_t n,
+                                                        const TI* __restrict__ h, int64_t ldh, int pitch_in,
+                                                        int lpr_log, __nv_bfloat16* __restrict__ out,
+                                                        int64_t ldo) {
+  constexpr int E = InTraits<TI>::kElems;
+  const int lane = threadIdx.x & 31;
+  const int LPR = 1 << lpr_log, G = 32 / LPR;
+  const int g = lane >> lpr_log, pc = lane & (LPR - 1);
+  const int npieces = (pitch_in + E - 1) / E;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n; w += warps) {
+    const int64_t pos = w * G + g;
+    int64_t row = -1;
+    int32_t b = 0, D = 0;
+    if (pos < n) {
+      row = perm ? (int64_t)__ldg(perm + pos) : pos;
+      b = __ldg(rp + row);
+      D = __ldg(rp + row + 1) - b;
+    }
+    const bool skip = row < 0 || D > kHeavyT;
+    const int32_t Dl = skip ? 0 : D;
+    const int32_t Dmax = __reduce_max_sync(0xffffffffu, Dl);
+    for (int p0 = 0; p0 < npieces; p0 += LPR) {
+      const int piece = p0 + pc;
+      const bool colok = piece < npieces;
+      const int col0 = piece * E;
+      float acc[E];
+#pragma unroll
+      for (int k = 0; k < E; ++k) acc[k] = 0.f;
+      for (int32_t base = 0; base < Dmax; base += LPR) {
+        const int32_t jj = (base + pc < Dl) ? __ldg(col + b + base + pc) : 0;
+        const int lim = min(LPR, Dmax - base);
+        for (int u = 0; u < lim; u += kGU) {
+          uint4 raw[kGU];
+#pragma unroll
+          for (int uu = 0; uu < kGU; ++uu) {
+            const int tt = u + uu;
+            const int32_t jn = __shfl_sync(0xffffffffu, jj, ((g << lpr_log) + (tt & (LPR - 1))) & 31);
+            raw[uu] = make_uint4(0u, 0u, 0u, 0u);
+            if (tt < LPR && base + tt < Dl && colok)
+              raw[uu] = __ldg(reinterpret_cast<const uint4*>(h + (int64_t)jn * ldh + col0));
+          }
+#pragma unroll
+          for (int uu = 0; uu < kGU; ++uu) {
+            float v[E];
+            raw_to_f32<TI>(raw[uu], v);
+#pragma unroll
+            for (int k = 0; k < E; ++k) acc[k] += v[k];
+          }
+        }
+      }
+      if (!skip && colok) {
+        if (MODE == 0) {
+          const float fd = (float)D;
+#pragma unroll
+          for (int k = 0; k < E; ++k) acc[k] = D > 0 ? acc[k] / fd : 0.f;
+        }
+        __nv_bfloat16* dst = out + row * ldo + col0;
+        if constexpr (E == 8) {
+          *reinterpret_cast<uint4*>(dst) = make_uint4(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]),
+                                                      pack_bf16x2(acc[4], acc[5]), pack_bf16x2(acc[6], acc[7]));
+        } else {
+          *reinterpret_cast<uint2*>(dst) = make_uint2(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]));
+        }
+      }
+    }
+  }
+}
+
+template <class TI, int MODE>
+static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, const int32_t* col, int64_t n,
+                                    const TI* h, int64_t ldh, int pitch_in, __nv_bfloat16* out, int64_t ldo,
+                                    cudaStream_t s) {
+  if (n <= 0) return BUFFALO_OK;
+  constexpr int E = InTraits<TI>::kElems;
+  const int npieces = (pitch_in + E - 1) / E;
+  int lpr_log = 0;
+  while ((1 << lpr_log) < npieces && lpr_log < 5) ++lpr_log;
+  const int G = 32 >> lpr_log;
+  const int64_t warps = ceil_div(n, G);
+  const int grid = (int)std::min<int64_t>(ceil_div(warps, 8), 148LL * 8 * 4);
+  k_gather_rows<TI, MODE><<<grid, 256, 0, s>>>(perm, rp, col, n, h, ldh, pitch_in, lpr_log, out, ldo);
+  BF_LAUNCHED(MODE == 0 ? "k_gather_mean" : "k_gather_sum");
+  return BUFFALO_OK;
+}
+
+static bool use_fused() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("BUFFALO_FUSED");
+    v = (e && e[0] == '1') ? 1 : 0;
+  }
+  return v == 1;
+}
+
 template <class TI, int MODE>
 static buffalo_status launch_tc(const TcFwdParams& p, cudaStream_t s) {
   const int smem = smem_bytes_for(p.Np);
@@ -569,7 +707,7 @@ static buffalo_status launch_tc(const TcFwdParams& p, cudaStream_t s) {
   const int64_t ntiles = ceil_div(p.n_dst, kTileM);
   const int grid = (int)std::min<int64_t>(ntiles, 148);
   k_tc_sage_fwd<TI, MODE><<<grid, kThreads, smem, s>>>(p);
-  BF_LAUNCHED(MODE == 0 ? "k_tc_sage_fwd" : "k_tc_sage_bwd_dh");
+  BF_LAUNCHED(MODE == 0 ? "k_tc_sage_fwd" : MODE == 1 ? "k_tc_sage_bwd_dh" : "k_tc_update_gemm");
   return BUFFALO_OK;
 }
 
@@ -610,7 +748,14 @@ static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   p.out = a.out;
   p.agg = (__nv_bfloat16*)a.agg;
   p.ld_agg = a.ld_agg;
-  return launch_tc<TI, 0>(p, s);
+  if (use_fused()) return launch_tc<TI, 0>(p, s);
+  // split: high-occupancy gather of the non-heavy rows, then the Update GEMM over copies
+  BF_CHECK((launch_gather<TI, 0>(blk->cls_perm, blk->row_ptr, p.col, blk->n_dst, (const TI*)a.h_src, a.ld_src,
+                                 p.pitch_in, (__nv_bfloat16*)a.agg, a.ld_agg, s)));
+  p.perm = nullptr;
+  p.agg_src = (const __nv_bfloat16*)a.agg;
+  p.ld_agg_src = a.ld_agg;
+  return launch_tc<TI, 2>(p, s);
 }
 
 buffalo_status tc_sage_fwd(const FwdArgs& a, cudaStream_t s) {
@@ -716,14 +861,6 @@ __host__ __device__ constexpr uint32_t idesc_bf16_mn(int n) {
          ((uint32_t)(128 >> 4) << 24);
 }
 
-__device__ __forceinline__ void cp_async16(void* dst, const void* src, bool valid) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src),
-               "r"(valid ? 16 : 0)
-               : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 template <class TS>
 __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
@@ -903,7 +1040,7 @@ __global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restric
                                                         const int32_t* __restrict__ rp,
                                                         const int32_t* __restrict__ col,
                                                         const __nv_bfloat16* __restrict__ z, int64_t ldz,
-                                                        int dp, __nv_bfloat16* __restrict__ out) {
+                                                        int dp, __nv_bfloat16* __restrict__ out, int by_row) {
   __shared__ float part[8][32][8];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t j = list[blockIdx.x];
@@ -931,7 +1068,7 @@ __global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restric
         for (int ww = 1; ww < 8; ++ww) s += part[ww][lane][k];
         acc[k] = s;
       }
-      *reinterpret_cast<uint4*>(out + (int64_t)blockIdx.x * dp + c * 8) =
+      *reinterpret_cast<uint4*>(out + (by_row ? j : (int64_t)blockIdx.x) * dp + c * 8) =
           make_uint4(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]), pack_bf16x2(acc[4], acc[5]),
                      pack_bf16x2(acc[6], acc[7]));
     }
@@ -947,13 +1084,13 @@ int tc_dw_splits(int64_t n, int d_out, int d_in) {
 }
 
 int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int64_t e, int layer, int d_in, int d_out) {
-  (void)n_src;
+  (void)e;
   const int S = tc_dw_splits(n_dst, d_out, d_in);
   const int64_t Dp = round_up(d_in, 64);
   int64_t b = R(n_dst * pitch_of(d_out) * 2);                        // dZ bf16
   if (layer >= 2) {
     b += R(n_dst * pitch_of(d_out) * 2);                              // dZ / D bf16
-    b += R(e / (kHeavyT + 1) * pitch_of(d_out) * 2);                  // long-tail transposed sums
+    b += R(n_src * pitch_of(d_out) * 2);                              // transposed sums (bf16)
   }
   b += R((int64_t)S * d_out * 2 * Dp * 4) + R((int64_t)kDbSplits * d_out * 4);
   return b;
@@ -976,7 +1113,7 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   __nv_bfloat16* hbuf = nullptr;
   if (a.dh_src) {
     zs = (__nv_bfloat16*)q; q += R(n * dp * 2);
-    hbuf = (__nv_bfloat16*)q; q += R(blk->n_edges / (kHeavyT + 1) * dp * 2);
+    hbuf = (__nv_bfloat16*)q; q += R(blk->n_src * dp * 2);
   }
   float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * Dp * 4);
   float* db_part = (float*)q;
@@ -1014,9 +1151,13 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   if (a.dh_src && blk->n_src > 0) {
     if (blk->n_heavy_t > 0) {
       k_sum_heavy_rows<<<(unsigned)blk->n_heavy_t, 256, 0, s>>>(blk->t_perm + (blk->n_src - blk->n_heavy_t),
-                                                                blk->t_row_ptr, blk->t_col, zs, dp, dp, hbuf);
+                                                                blk->t_row_ptr, blk->t_col, zs, dp, dp, hbuf,
+                                                                use_fused() ? 0 : 1);
       BF_LAUNCHED("k_sum_heavy_rows");
     }
+    if (!use_fused())
+      BF_CHECK((launch_gather<__nv_bfloat16, 1>(blk->t_perm, blk->t_row_ptr, blk->t_col, blk->n_src, zs, dp, dp,
+                                                hbuf, dp, s)));
     TcFwdParams p{};
     p.perm = blk->t_perm;
     p.heavy_base = blk->n_src - blk->n_heavy_t;
@@ -1044,6 +1185,13 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     p.out = a.dh_src;
     p.agg = nullptr;
     p.ld_agg = 0;
+    if (!use_fused()) {
+      p.perm = nullptr;
+      p.agg_src = hbuf;
+      p.ld_agg_src = dp;
+      BF_CHECK((launch_tc<__nv_bfloat16, 2>(p, s)));
+      return BUFFALO_OK;
+    }
     BF_CHECK((launch_tc<__nv_bfloat16, 1>(p, s)));
   }
   return BUFFALO_OK;
