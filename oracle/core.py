@@ -197,10 +197,11 @@ def dw_splits(n_l, d_out, d_in):
 
 
 def tc_dw_splits(n_l, d_out, d_in):
-    """Split count of the tensor-core dW reduction (tiles of 128 x 256 over [d_out, 2 Dp])."""
+    """Split count of the tensor-core dW reduction (one CTA per 256-column tile of [2 Dp] and
+    row split, all of d_out per CTA)."""
     Dp = _ceil(d_in, 64) * 64
-    tiles = _ceil(d_out, 128) * _ceil(2 * Dp, 256)
-    return max(1, min(_ceil(296, tiles), _ceil(max(int(n_l), 1), 512)))
+    tiles = _ceil(2 * Dp, 256)
+    return max(1, min(_ceil(148, tiles), _ceil(max(int(n_l), 1), 512)))
 
 
 def _part_count_elems(e):

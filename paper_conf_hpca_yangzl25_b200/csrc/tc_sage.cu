@@ -505,12 +505,28 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
             }
           }
         }
-        asm volatile("cp.async.wait_all;" ::: "memory");
-        fence_proxy_async_smem();
-        mbar_arrive(&a_full[buf]);
+        if (MODE == 2) {
+          // copy-only tiles: keep two super-chunks of cp.async in flight; super-chunk q-1 is
+          // handed to the MMA once its copies landed
+          cp_async_commit();
+          if (q > 0) {
+            cp_async_wait<1>();
+            fence_proxy_async_smem();
+            mbar_arrive(&a_full[(q - 1) & 1]);
+          }
+        } else {
+          asm volatile("cp.async.wait_all;" ::: "memory");
+          fence_proxy_async_smem();
+          mbar_arrive(&a_full[buf]);
+        }
       }
       if (prev_tile >= 0) epilogue(prev_tile, i - 1);
       prev_tile = t;
+    }
+    if (MODE == 2 && q > 0) {
+      cp_async_wait<0>();
+      fence_proxy_async_smem();
+      mbar_arrive(&a_full[(q - 1) & 1]);
     }
     if (prev_tile >= 0) epilogue(prev_tile, i - 1);
   }
@@ -831,7 +847,7 @@ __global__ void __launch_bounds__(256) k_dz_prep(float* __restrict__ dz, int64_t
 // dW (tensor cores): D[m][n'] = sum_r dZ[r][m] * Afwd[r][n'] over a row range, both operands
 // MN-major in shared memory (the reduction runs over rows, the slow dimension of both).
 // Afwd columns are padded per half: n' < Dp -> self column n', n' >= Dp -> h_agg column n' - Dp.
-constexpr int kDwThreads = 128;
+constexpr int kDwThreads = 256;
 constexpr int kDwRows = 64;                       // K per stage
 constexpr int kDwStrip = kDwRows * 128;           // one 64-column MN strip of 64 rows (8 KB)
 constexpr int kDwStages = 3;
@@ -841,7 +857,7 @@ struct TcDwParams {
   const void* self_; int64_t lds; const int32_t* gidx;  // self rows (feature table for layer 1)
   const __nv_bfloat16* agg; int64_t lda;          // saved h_agg
   int64_t n;
-  int d_out, d_in, pitch_in, pz, Dp, NT;          // NT: n' columns per CTA tile (<= 256)
+  int d_out, d_in, pitch_in, pz, Dp, NT, MT;      // NT: n' columns per CTA (<= 256); MT: m-tiles (<= 2)
   int64_t rows_per_split;
   float* part;                                    // [S][d_out][2 Dp]
 };
@@ -861,28 +877,31 @@ __host__ __device__ constexpr uint32_t idesc_bf16_mn(int n) {
          ((uint32_t)(128 >> 4) << 24);
 }
 
-
+// One CTA: all m-tiles of d_out (each 128 TMEM lanes x NT columns) for one n'-tile, over a row
+// split; both operands are read once.  3-stage cp.async pipeline, single-thread MMA issue.
 template <class TS>
 __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  const int nstripA = 2, nstripB = p.NT / 64;
+  const int nstripA = 2 * p.MT, nstripB = p.NT / 64;
   const int stage_bytes = (nstripA + nstripB) * kDwStrip;
   uint64_t* full = (uint64_t*)(smem + kDwStages * stage_bytes);
   uint64_t* empty = full + kDwStages;
   uint64_t* done = empty + kDwStages;
   uint32_t* tmem_slot = (uint32_t*)(done + 1);
   const int warp = threadIdx.x >> 5;
-  const int m0 = blockIdx.x * 128, n0 = blockIdx.y * p.NT;
-  const int64_t r_beg = (int64_t)blockIdx.z * p.rows_per_split;
+  const int n0 = blockIdx.x * p.NT;
+  const int64_t r_beg = (int64_t)blockIdx.y * p.rows_per_split;
   const int64_t r_end = min(p.n, r_beg + p.rows_per_split);
   const int nchunks = r_end > r_beg ? (int)((r_end - r_beg + kDwRows - 1) / kDwRows) : 0;
+  int tcols = 32;
+  while (tcols < p.MT * p.NT) tcols <<= 1;
   if (threadIdx.x == 0) {
     for (int i = 0; i < kDwStages; ++i) { mbar_init(&full[i], kDwThreads); mbar_init(&empty[i], 1); }
     mbar_init(done, 1);
     fence_barrier_init();
   }
-  if (warp == 0) tmem_alloc(tmem_slot, p.NT);
+  if (warp == 0) tmem_alloc(tmem_slot, tcols);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -890,25 +909,24 @@ __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
   const TS* __restrict__ selfp = (const TS*)p.self_;
   const uint32_t idesc = idesc_bf16_mn(p.NT);
   const void* dummy = p.zb;            // any global address: zero-fill copies read 0 bytes
+  const int apcs = p.MT * 16;          // 16-B pieces of a dZ row slice (128 columns per m-tile)
+  const int bpcs = p.NT / 8;
 
   auto load_chunk = [&](int c) {
     const int st = c % kDwStages;
     uint8_t* sa = smem + st * stage_bytes;
     uint8_t* sb = sa + nstripA * kDwStrip;
     const int64_t rbase = r_beg + (int64_t)c * kDwRows;
-    // A: dZ rows, 128 m-columns = 2 strips x 8 pieces of 16 B per row
-    for (int u = threadIdx.x; u < kDwRows * 16; u += kDwThreads) {
-      const int k = u >> 4, j = u & 15;
+    for (int u = threadIdx.x; u < kDwRows * apcs; u += kDwThreads) {
+      const int k = u / apcs, j = u % apcs;
       const int64_t r = rbase + k;
-      const int m = m0 + j * 8;
+      const int m = j * 8;
       const bool ok = r < r_end && m < p.pz;
       cp_async16(sa + (j >> 3) * kDwStrip + k * 128 + (((j & 7) ^ (k & 7)) << 4),
                  ok ? (const void*)(p.zb + r * p.ldz + m) : dummy, ok);
     }
-    // B: Afwd rows, NT n'-columns
-    const int pcs = p.NT / 8;
-    for (int u = threadIdx.x; u < kDwRows * pcs; u += kDwThreads) {
-      const int k = u / pcs, j = u % pcs;
+    for (int u = threadIdx.x; u < kDwRows * bpcs; u += kDwThreads) {
+      const int k = u / bpcs, j = u % bpcs;
       const int64_t r = rbase + k;
       const int nn = n0 + j * 8;
       uint8_t* dst = sb + (j >> 3) * kDwStrip + k * 128 + (((j & 7) ^ (k & 7)) << 4);
@@ -954,10 +972,11 @@ __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
     tc_fence_after();
     const uint32_t a_addr = smem_u32(smem + st * stage_bytes);
     const uint32_t b_addr = a_addr + nstripA * kDwStrip;
+    for (int mt = 0; mt < p.MT; ++mt)
 #pragma unroll
-    for (int kk = 0; kk < kDwRows / 16; ++kk)
-      umma_bf16(tmem, sw128_mn_desc(a_addr + kk * 2048, kDwStrip), sw128_mn_desc(b_addr + kk * 2048, kDwStrip),
-                idesc, (c > 0 || kk > 0) ? 1u : 0u);
+      for (int kk = 0; kk < kDwRows / 16; ++kk)
+        umma_bf16(tmem + mt * p.NT, sw128_mn_desc(a_addr + mt * 2 * kDwStrip + kk * 2048, kDwStrip),
+                  sw128_mn_desc(b_addr + kk * 2048, kDwStrip), idesc, (c > 0 || kk > 0) ? 1u : 0u);
     umma_commit(&empty[st]);
     if (c == nchunks - 1) umma_commit(done);
   };
@@ -980,35 +999,38 @@ __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
     if (threadIdx.x == 0) mma_chunk(nchunks - 1);
     __syncwarp();
   }
-  // epilogue: TMEM lanes = m rows, columns = n'
+  // epilogue: warp w reads TMEM lane quadrant w % 4 of m-tile w / 4
   const int lane = threadIdx.x & 31;
+  const int quad = warp & 3, mt = warp >> 2;
   const int64_t K2 = 2 * (int64_t)p.Dp;
-  float* P = p.part + (int64_t)blockIdx.z * p.d_out * K2;
-  const int m = m0 + warp * 32 + lane;
+  float* P = p.part + (int64_t)blockIdx.y * p.d_out * K2;
+  const int m = mt * 128 + quad * 32 + lane;
   if (nchunks > 0) {
     mbar_wait(done, 0);
     tc_fence_after();
   }
-  for (int g = 0; g < p.NT / 8; ++g) {
-    float v[8];
-    if (nchunks > 0) {
-      tmem_ld8(tmem + ((uint32_t)(warp * 32) << 16) + g * 8, v);
-    } else {
+  if (mt < p.MT) {
+    for (int g = 0; g < p.NT / 8; ++g) {
+      float v[8];
+      if (nchunks > 0) {
+        tmem_ld8(tmem + ((uint32_t)(quad * 32) << 16) + mt * p.NT + g * 8, v);
+      } else {
 #pragma unroll
-      for (int k = 0; k < 8; ++k) v[k] = 0.f;
-    }
-    const int nn = n0 + g * 8;
-    if (m < p.d_out && nn < K2) {
-      float4* o = reinterpret_cast<float4*>(P + (int64_t)m * K2 + nn);
-      o[0] = make_float4(v[0], v[1], v[2], v[3]);
-      o[1] = make_float4(v[4], v[5], v[6], v[7]);
+        for (int k = 0; k < 8; ++k) v[k] = 0.f;
+      }
+      const int nn = n0 + g * 8;
+      if (m < p.d_out && nn < K2) {
+        float4* o = reinterpret_cast<float4*>(P + (int64_t)m * K2 + nn);
+        o[0] = make_float4(v[0], v[1], v[2], v[3]);
+        o[1] = make_float4(v[4], v[5], v[6], v[7]);
+      }
     }
   }
   tc_fence_before();
   __syncthreads();
   if (warp == 0) {
     tc_fence_after();
-    tmem_dealloc(tmem, p.NT);
+    tmem_dealloc(tmem, tcols);
   }
 }
 
@@ -1077,9 +1099,10 @@ __global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restric
 }
 
 int tc_dw_splits(int64_t n, int d_out, int d_in) {
+  (void)d_out;
   const int64_t Dp = round_up(d_in, 64);
-  const int64_t tiles = ceil_div(d_out, 128) * ceil_div(2 * Dp, 256);
-  int64_t sp = std::min<int64_t>(ceil_div(296, tiles), ceil_div(n > 0 ? n : 1, 512));
+  const int64_t tiles = ceil_div(2 * Dp, 256);
+  int64_t sp = std::min<int64_t>(ceil_div(148, tiles), ceil_div(n > 0 ? n : 1, 512));
   return (int)std::max<int64_t>(1, sp);
 }
 
@@ -1129,12 +1152,13 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   w.agg = (const __nv_bfloat16*)a.agg; w.lda = a.ld_agg;
   w.n = n; w.d_out = d_out; w.d_in = d_in; w.pitch_in = (int)pitch_of(d_in); w.pz = dp; w.Dp = (int)Dp;
   w.NT = (int)std::min<int64_t>(256, 2 * Dp);
+  w.MT = (int)ceil_div(d_out, 128);
   w.rows_per_split = ceil_div(n, S);
   w.part = dw_part;
-  const int smem = kDwStages * (2 + w.NT / 64) * kDwStrip + 128 + 1024;
-  dim3 grid((unsigned)ceil_div(d_out, 128), (unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
+  const int smem = kDwStages * (2 * w.MT + w.NT / 64) * kDwStrip + 128 + 1024;
+  dim3 grid((unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
   static bool attr[2] = {false, false};
-  constexpr int kMaxDwSmem = kDwStages * (2 + 4) * kDwStrip + 128 + 1024;
+  constexpr int kMaxDwSmem = kDwStages * (4 + 4) * kDwStrip + 128 + 1024;
   if (a.in_bf16) {
     if (!attr[0]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr[0] = true; }
     k_tc_dw<__nv_bfloat16><<<grid, kDwThreads, smem, s>>>(w);
