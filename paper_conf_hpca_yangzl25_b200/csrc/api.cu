@@ -139,25 +139,22 @@ struct Item {
 
 // Item statistics (R13, R15): exact layer sizes of up to 64 items per pass (mask_stats), then
 // O = #seeds, E = e_L, I = n_{L-1} and M_est = hi of the memory model.
-static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_ids, std::vector<Item>& items,
-                                  size_t first, size_t count, const buffalo_sampler* sp, const buffalo_model* m,
-                                  char* ws, int64_t ws_bytes, bool& masks_clean, cudaStream_t s) {
+static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_ids, std::vector<Item*>& items,
+                                  const buffalo_sampler* sp, const buffalo_model* m, char* ws, int64_t ws_bytes,
+                                  bool& masks_clean, cudaStream_t s) {
   const int L = m->num_layers;
-  for (size_t b0 = first; b0 < first + count; b0 += 64) {
-    const int nit = (int)std::min<size_t>(64, first + count - b0);
-    int64_t starts[65];
-    for (int k = 0; k < nit; ++k) starts[k] = items[b0 + k].start;
-    starts[nit] = items[b0 + nit - 1].start + items[b0 + nit - 1].count;
-    for (int k = 0; k + 1 < nit; ++k)
-      if (items[b0 + k].start + items[b0 + k].count != items[b0 + k + 1].start) {
-        set_error("internal: items of a statistics pass must be adjacent");
-        return BUFFALO_ERR_INVALID_ARG;
-      }
+  for (size_t b0 = 0; b0 < items.size(); b0 += 64) {
+    const int nit = (int)std::min<size_t>(64, items.size() - b0);
+    int64_t starts[64], counts[64];
+    for (int k = 0; k < nit; ++k) {
+      starts[k] = items[b0 + k]->start;
+      counts[k] = items[b0 + k]->count;
+    }
     static thread_local int64_t nh[64][BUFFALO_MAX_LAYERS + 1], eh[64][BUFFALO_MAX_LAYERS];
-    BF_CHECK(mask_stats(g, sorted_ids, starts, nit, sp, L, ws, ws_bytes, masks_clean, nh, eh, s));
+    BF_CHECK(mask_stats(g, sorted_ids, starts, counts, nit, sp, L, ws, ws_bytes, masks_clean, nh, eh, s));
     masks_clean = true;
     for (int k = 0; k < nit; ++k) {
-      Item& it = items[b0 + k];
+      Item& it = *items[b0 + k];
       int64_t lo, hi;
       mem_model(L, nh[k], eh[k], m, &lo, &hi);
       it.O = it.count;
@@ -167,6 +164,19 @@ static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_
     }
   }
   return BUFFALO_OK;
+}
+
+// SplitExplosionBucket (R8): K contiguous pieces of bucket F, the first (O mod K) one seed larger.
+static std::vector<Item> split_pieces(const Item& itF, int F, int K) {
+  std::vector<Item> pieces;
+  const int64_t O = itF.count, base = O / K, extra = O % K;
+  int64_t st0 = itF.start;
+  for (int k = 0; k < K; ++k) {
+    const int64_t len = base + (k < extra ? 1 : 0);
+    if (len > 0) pieces.push_back(Item{F, k, st0, len, 0, 0, 0, 0, 0});
+    st0 += len;
+  }
+  return pieces;
 }
 
 // Eq. 1-2, integer form (R14): floor(M * min(1, I*10^6 / (E*C_ppm))).
@@ -290,8 +300,12 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
   // a2: per-bucket statistics and estimates (K-independent); item k = degree bucket k
   bool masks_clean = false;
   std::vector<Item> bucket_item(F + 1);
-  for (int d = 0; d <= F; ++d) bucket_item[d] = Item{d, 0, bstart[d], plan->hist_h[d], 0, 0, 0, 0, 0};
-  BF_CHECK(items_stats(g, sorted_ids, bucket_item, 0, F + 1, sp, m, stats_ws, stats_bytes, masks_clean, s));
+  std::vector<Item*> todo;
+  for (int d = 0; d <= F; ++d) {
+    bucket_item[d] = Item{d, 0, bstart[d], plan->hist_h[d], 0, 0, 0, 0, 0};
+    if (plan->hist_h[d] > 0) todo.push_back(&bucket_item[d]);
+  }
+  BF_CHECK(items_stats(g, sorted_ids, todo, sp, m, stats_ws, stats_bytes, masks_clean, s));
   std::vector<int> non_split;
   int64_t sum_M_all = 0, sum_w = 0, max_w = 0;
   for (int d = 0; d <= F; ++d) {
@@ -307,8 +321,17 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
   }
   const bool hasF = plan->hist_h[F] > 0;
 
-  // a3: the K loop (Alg. 3) with MemBalancedGrouping (Alg. 4)
+  // a3: the K loop (Alg. 3) with MemBalancedGrouping (Alg. 4).  The micro-bucket statistics
+  // of several consecutive K candidates are computed in one statistics pass (their pieces
+  // overlap, each seed carries one bit per candidate); the loop itself stays sequential.
   const int k_lo = std::max(std::max(sc->k_min, sc->num_gpus), 1);
+  auto needs_split = [&](int K) {
+    if (max_w > sc->mem_budget) return false;
+    if ((__int128)sum_w > (__int128)K * sc->mem_budget) return false;
+    return hasF && K >= 2 && (__int128)bucket_item[F].M * K > (__int128)sum_M_all;
+  };
+  std::vector<std::vector<Item>> piece_cache(sc->k_max + 1);
+  std::vector<char> have(sc->k_max + 1, 0);
   for (int K = k_lo; K <= sc->k_max; ++K) {
     if (max_w > sc->mem_budget) break;                         // R25: fails for every K
     if ((__int128)sum_w > (__int128)K * sc->mem_budget) continue;  // R25: some group exceeds M_ctr
@@ -319,17 +342,27 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
       const Item& itF = bucket_item[F];
       exploded = K >= 2 && (__int128)itF.M * K > (__int128)sum_M_all;   // R7
       if (exploded) {
-        // SplitExplosionBucket: K contiguous pieces, the first (O mod K) one seed larger (R8)
-        const int64_t O = itF.count, base = O / K, extra = O % K;
-        std::vector<Item> pieces;
-        int64_t st0 = itF.start;
-        for (int k = 0; k < K; ++k) {
-          const int64_t len = base + (k < extra ? 1 : 0);
-          if (len > 0) pieces.push_back(Item{F, k, st0, len, 0, 0, 0, 0, 0});
-          st0 += len;
+        if (!have[K]) {
+          // batch this and the following candidates that will need a split (<= 64 pieces)
+          std::vector<int> ks;
+          int total = 0;
+          for (int K2 = K; K2 <= sc->k_max && (int)ks.size() < 64; ++K2) {
+            if (!needs_split(K2)) continue;
+            const int np = (int)std::min<int64_t>(K2, itF.count);
+            if (total + np > 64 && !ks.empty()) break;
+            ks.push_back(K2);
+            total += np;
+          }
+          std::vector<Item*> ptrs;
+          for (int K2 : ks) {
+            piece_cache[K2] = split_pieces(itF, F, K2);
+            have[K2] = 1;
+          }
+          for (int K2 : ks)
+            for (Item& it : piece_cache[K2]) ptrs.push_back(&it);
+          BF_CHECK(items_stats(g, sorted_ids, ptrs, sp, m, stats_ws, stats_bytes, masks_clean, s));
         }
-        BF_CHECK(items_stats(g, sorted_ids, pieces, 0, pieces.size(), sp, m, stats_ws, stats_bytes, masks_clean, s));
-        for (Item& it : pieces) {
+        for (Item it : piece_cache[K]) {
           it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
           items.push_back(it);
         }

@@ -384,14 +384,18 @@ __device__ __forceinline__ void mask_accumulate(uint64_t mask, int64_t D, unsign
   }
 }
 
-__global__ void __launch_bounds__(256) k_mask_seed(const int32_t* __restrict__ ids, int64_t n,
-                                                   const int64_t* __restrict__ item_start, int nitems,
+// Seed masks: position i (of the union range starting at base) gets the bit of every item
+// [start_k, end_k) that contains it (items of different K candidates overlap).
+__global__ void __launch_bounds__(256) k_mask_seed(const int32_t* __restrict__ ids, int64_t base, int64_t n,
+                                                   const int64_t* __restrict__ item_se, int nitems,
                                                    unsigned long long* __restrict__ m, int32_t* __restrict__ act) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    int k = 0;
-    while (k + 1 < nitems && item_start[k + 1] - item_start[0] <= i) ++k;
-    const int32_t v = ids[i];
-    m[v] = 1ull << k;
+    const int64_t pos = base + i;
+    unsigned long long mask = 0;
+    for (int k = 0; k < nitems; ++k)
+      if (pos >= item_se[2 * k] && pos < item_se[2 * k + 1]) mask |= 1ull << k;
+    const int32_t v = ids[pos];
+    m[v] = mask;
     act[i] = v;
   }
 }
@@ -416,10 +420,13 @@ __global__ void __launch_bounds__(256) k_mask_layer(const int32_t* __restrict__ 
     const int64_t beg = grow[v];
     const int64_t deg = grow[v + 1] - beg;
     const int64_t D = (f > 0 && deg > f) ? f : deg;
-    if (lane == 0) {
-      mask_accumulate(mask, D, sn, se);
-      if (atomicOr(&m_out[v], mask) == 0ull) act_out[atomicAdd(n_out, 1)] = (int32_t)v;
+    // per-item sizes: lane k handles items k and k + 32
+    if ((mask >> lane) & 1ull) { atomicAdd(&sn[lane], 1ull); atomicAdd(&se[lane], (unsigned long long)D); }
+    if ((mask >> (lane + 32)) & 1ull) {
+      atomicAdd(&sn[lane + 32], 1ull);
+      atomicAdd(&se[lane + 32], (unsigned long long)D);
     }
+    if (lane == 0 && atomicOr(&m_out[v], mask) == 0ull) act_out[atomicAdd(n_out, 1)] = (int32_t)v;
     if (f <= 0 || deg <= f) {
       for (int64_t k = lane; k < deg; k += 32) {
         const int32_t u = gcol[beg + k];
@@ -454,21 +461,35 @@ __global__ void __launch_bounds__(256) k_mask_count(const int32_t* __restrict__ 
   __shared__ unsigned long long sn[64];
   if (threadIdx.x < 64) sn[threadIdx.x] = 0;
   __syncthreads();
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_act; i += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t v = act[i];
-    if (gn) mask_accumulate(m[v], 0, sn, nullptr);
-    if (clear) m[v] = 0ull;
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i0 = blockIdx.x * (int64_t)blockDim.x; i0 < n_act; i0 += stride) {
+    const int64_t i = i0 + threadIdx.x;
+    unsigned long long mask = 0;
+    if (i < n_act) {
+      const int32_t v = act[i];
+      mask = m[v];
+      if (clear) m[v] = 0ull;
+    }
+    if (gn) {
+      // warp-cooperative per-item counts: one ballot per item bit
+      for (int k = 0; k < 64; ++k) {
+        const unsigned b = __ballot_sync(0xffffffffu, (mask >> k) & 1ull);
+        if (lane == (k & 31) && b) atomicAdd(&sn[k], (unsigned long long)__popc(b));
+      }
+    }
   }
   __syncthreads();
   if (gn && threadIdx.x < 64 && sn[threadIdx.x]) atomicAdd(&gn[threadIdx.x], sn[threadIdx.x]);
 }
 
 int64_t mask_stats_bytes(int64_t N, int L) {
-  return 2 * R(8 * N) + 2 * R(4 * N) + R(8 * 64 * (2 * L + 1)) + R(64) + R(8 * 65);
+  return 2 * R(8 * N) + 2 * R(4 * N) + R(8 * 64 * (2 * L + 1)) + R(64) + R(16 * 64);
 }
 
 buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, const int64_t* item_start_h,
-                          int nitems, const buffalo_sampler* sp, int L, char* ws, int64_t ws_bytes,
+                          const int64_t* item_count_h, int nitems, const buffalo_sampler* sp, int L, char* ws,
+                          int64_t ws_bytes,
                           bool masks_clean, int64_t (*n_h)[BUFFALO_MAX_LAYERS + 1],
                           int64_t (*e_h)[BUFFALO_MAX_LAYERS], cudaStream_t s) {
   const int64_t N = g->num_nodes;
@@ -483,18 +504,31 @@ buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, con
   q += 2 * R(4 * N);
   unsigned long long* acc = (unsigned long long*)q; q += R(8 * 64 * (2 * L + 1));
   int32_t* cnt = (int32_t*)q; q += R(64);
-  int64_t* starts = (int64_t*)q;
+  int64_t* se = (int64_t*)q;
   if (!masks_clean) {
     BF_CUDA(cudaMemsetAsync(m[0], 0, 2 * R(8 * N), s));
   }
   BF_CUDA(cudaMemsetAsync(acc, 0, sizeof(unsigned long long) * 64 * (2 * L + 1), s));
-  BF_CUDA(cudaMemcpyAsync(starts, item_start_h, sizeof(int64_t) * (nitems + 1), cudaMemcpyHostToDevice, s));
-  const int64_t n_seed = item_start_h[nitems] - item_start_h[0];
+  int64_t se_h[128];
+  int64_t lo_pos = INT64_MAX, hi_pos = 0;
+  for (int k = 0; k < nitems; ++k) {
+    se_h[2 * k] = item_start_h[k];
+    se_h[2 * k + 1] = item_start_h[k] + item_count_h[k];
+    if (item_count_h[k] > 0) {
+      lo_pos = std::min(lo_pos, se_h[2 * k]);
+      hi_pos = std::max(hi_pos, se_h[2 * k + 1]);
+    }
+  }
+  if (lo_pos > hi_pos) lo_pos = hi_pos = 0;
+  BF_CUDA(cudaMemcpyAsync(se, se_h, sizeof(int64_t) * 2 * nitems, cudaMemcpyHostToDevice, s));
+  const int64_t n_seed = hi_pos - lo_pos;
   // acc layout: n[l] at acc + 64*l (l = 0..L), e[l-1] at acc + 64*(L+1) + 64*(l-1)
   unsigned long long* accn = acc;
   unsigned long long* acce = acc + 64 * (L + 1);
-  k_mask_seed<<<grid_for(n_seed, 256), 256, 0, s>>>(sorted_ids + item_start_h[0], n_seed, starts, nitems, m[0], act[0]);
-  BF_LAUNCHED("k_mask_seed");
+  if (n_seed > 0) {
+    k_mask_seed<<<grid_for(n_seed, 256), 256, 0, s>>>(sorted_ids, lo_pos, n_seed, se, nitems, m[0], act[0]);
+    BF_LAUNCHED("k_mask_seed");
+  }
   int64_t n_act = n_seed;
   int cur = 0;
   for (int l = L; l >= 1; --l) {

@@ -23,12 +23,13 @@ buffalo_status seed_bucketing(const buffalo_graph* g, const int32_t* seeds, int6
                               int32_t* counts, int32_t* ws, int32_t* starts_dev, int64_t* hist_h,
                               cudaStream_t s);
 
-// Exact per-item block sizes (n[0..L], e[0..L-1]) of up to 64 disjoint items: item k is
-// sorted_ids[item_start_h[k] .. item_start_h[k+1]).  ws: mask_stats_bytes(N, L) bytes; the
+// Exact per-item block sizes (n[0..L], e[0..L-1]) of up to 64 items (they may overlap): item k
+// is sorted_ids[item_start_h[k] .. + item_count_h[k]).  ws: mask_stats_bytes(N, L) bytes; the
 // masks are left zeroed (masks_clean = true on the next call saves a memset).
 int64_t mask_stats_bytes(int64_t N, int L);
 buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, const int64_t* item_start_h,
-                          int nitems, const buffalo_sampler* sp, int L, char* ws, int64_t ws_bytes,
+                          const int64_t* item_count_h, int nitems, const buffalo_sampler* sp, int L, char* ws,
+                          int64_t ws_bytes,
                           bool masks_clean, int64_t (*n_h)[BUFFALO_MAX_LAYERS + 1],
                           int64_t (*e_h)[BUFFALO_MAX_LAYERS], cudaStream_t s);
 
