@@ -156,6 +156,7 @@ struct TcFwdParams {
   const int32_t* perm;       // tile row order (degree-sorted dst) or null (natural order)
   const __nv_bfloat16* agg_src;  // MODE 2: the aggregate half, bf16 rows [n_dst][ld_agg_src]
   int64_t ld_agg_src;
+  int a_chunks, nb;          // K-chunks per A buffer (2 buffers), weight stages
   int64_t heavy_base;        // MODE 1: positions >= heavy_base are long-tail rows, pre-summed
   const __nv_bfloat16* heavy_buf;  // MODE 1: [pos - heavy_base][heavy_ld]
   int64_t heavy_ld;
@@ -218,18 +219,19 @@ template <> __device__ __forceinline__ void raw_to_f32<float>(const uint4& u, fl
 // (32 lanes x 16 B = one warp-wide row slice).
 template <int E> struct Sched {
   static constexpr int kAggChunks = (32 * E) / kKC;          // 4 (bf16) or 2 (fp32)
-  int nself_sc, nagg_sc, nkc_self, nkc;
-  __device__ Sched(int nkc_self_, int nkc_) : nkc_self(nkc_self_), nkc(nkc_) {
-    nself_sc = (nkc_self + kSuper - 1) / kSuper;
-    nagg_sc = (nkc - nkc_self + kAggChunks - 1) / kAggChunks;
+  int nself_sc, nagg_sc, nkc_self, nkc, sup, agg;
+  __device__ Sched(int nkc_self_, int nkc_, int a_chunks, bool copy_mode)
+      : nkc_self(nkc_self_), nkc(nkc_), sup(a_chunks), agg(copy_mode ? a_chunks : kAggChunks) {
+    nself_sc = (nkc_self + sup - 1) / sup;
+    nagg_sc = (nkc - nkc_self + agg - 1) / agg;
   }
   __device__ int count() const { return nself_sc + nagg_sc; }
   __device__ int first(int sc) const {
-    return sc < nself_sc ? sc * kSuper : nkc_self + (sc - nself_sc) * kAggChunks;
+    return sc < nself_sc ? sc * sup : nkc_self + (sc - nself_sc) * agg;
   }
   __device__ int size(int sc) const {
     const int f = first(sc);
-    return sc < nself_sc ? min(kSuper, nkc_self - f) : min(kAggChunks, nkc - f);
+    return sc < nself_sc ? min(sup, nkc_self - f) : min(agg, nkc - f);
   }
 };
 
@@ -244,31 +246,34 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
   constexpr int kUnroll = 8;                   // independent 16-B loads in flight per lane
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint8_t* sA = smem;                                          // 2 x kSuper x 16 KB
-  uint8_t* sB = smem + 2 * kSuper * kChunkBytesA;              // 2 x Np x 128 B
+  const int AC = p.a_chunks, NB = p.nb;                        // chunks per A buffer, B stages
+  uint8_t* sA = smem;                                          // 2 x AC x 16 KB
+  uint8_t* sB = smem + 2 * AC * kChunkBytesA;                  // NB x Np x 128 B
   const int bbytes = p.Np * 128;
-  uint64_t* bars = (uint64_t*)(sB + 2 * bbytes);
+  uint64_t* bars = (uint64_t*)(sB + NB * bbytes);
   uint64_t* a_full = bars;        // [2]
   uint64_t* a_empty = bars + 2;   // [2]
-  uint64_t* b_full = bars + 4;    // [2]
-  uint64_t* b_empty = bars + 6;   // [2]
-  uint64_t* acc_full = bars + 8;  // [2]
-  uint64_t* acc_empty = bars + 10;// [2]
-  uint32_t* tmem_slot = (uint32_t*)(bars + 12);
+  uint64_t* acc_full = bars + 4;  // [2]
+  uint64_t* acc_empty = bars + 6; // [2]
+  uint64_t* b_full = bars + 8;    // [NB]
+  uint64_t* b_empty = bars + 8 + NB;  // [NB]
+  uint32_t* tmem_slot = (uint32_t*)(bars + 8 + 2 * NB);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t ntiles = (p.n_dst + kTileM - 1) / kTileM;
-  const Sched<E> sched(p.nkc_self, p.nkc);
+  const Sched<E> sched(p.nkc_self, p.nkc, AC, MODE == 2);
   const int nsc = sched.count();
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < 2; ++i) {
       mbar_init(&a_full[i], kGatherThreads);
       mbar_init(&a_empty[i], 1);
-      mbar_init(&b_full[i], 1);
-      mbar_init(&b_empty[i], 1);
       mbar_init(&acc_full[i], 1);
       mbar_init(&acc_empty[i], kGatherThreads);
+    }
+    for (int i = 0; i < NB; ++i) {
+      mbar_init(&b_full[i], 1);
+      mbar_init(&b_empty[i], 1);
     }
     fence_barrier_init();
   }
@@ -282,14 +287,23 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
     // ===================== control warp: weight chunks + MMA issue (one elected lane)
     if (lane == 0) {
       const uint32_t idesc = idesc_bf16(p.Np);
-      int64_t g = 0;           // global chunk counter (B stage = g & 1)
+      int64_t g = 0;           // global chunk counter (B stage = g % NB)
+      int64_t issued = 0;      // weight chunks loaded so far (chunk x goes to stage x % NB)
       int64_t q = 0;           // global super-chunk counter (A buffer = q & 1)
       int64_t i = 0;           // local tile counter
       const int64_t total_chunks = ((ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x) * p.nkc;
-      if (total_chunks > 0) {
-        mbar_arrive_expect_tx(&b_full[0], bbytes);
-        bulk_g2s(sB, p.wpk, bbytes, &b_full[0]);
-      }
+      // keep up to NB - 1 weight chunks in flight ahead of the MMAs; a stage is refilled once
+      // the MMAs of the chunk NB positions earlier have retired
+      auto top_up = [&](int64_t upto) {
+        while (issued < total_chunks && issued < upto) {
+          const int st = (int)(issued % NB);
+          if (issued >= NB) mbar_wait(&b_empty[st], (uint32_t)(((issued / NB) - 1) & 1));
+          mbar_arrive_expect_tx(&b_full[st], bbytes);
+          bulk_g2s(sB + st * bbytes, p.wpk + (int64_t)(issued % p.nkc) * bbytes, bbytes, &b_full[st]);
+          ++issued;
+        }
+      };
+      top_up(NB);
       for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
         const int acc = (int)(i & 1);
         if (i >= 2) mbar_wait(&acc_empty[acc], (uint32_t)(((i >> 1) - 1) & 1));
@@ -302,26 +316,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
           const int c0 = sched.first(sc), cn_ = sched.size(sc);
           for (int j = 0; j < cn_; ++j) {
             const int c = c0 + j;
-            const int bs = (int)(g & 1);
-            mbar_wait(&b_full[bs], (uint32_t)((g >> 1) & 1));
+            const int bs = (int)(g % NB);
+            mbar_wait(&b_full[bs], (uint32_t)((g / NB) & 1));
             tc_fence_after();
-            const uint32_t a_addr = smem_u32(sA + (buf * kSuper + j) * kChunkBytesA);
+            const uint32_t a_addr = smem_u32(sA + (buf * AC + j) * kChunkBytesA);
             const uint32_t b_addr = smem_u32(sB + bs * bbytes);
 #pragma unroll
             for (int k = 0; k < kKC / 16; ++k)
               umma_bf16(tmem_d, sw128_desc(a_addr + 32 * k), sw128_desc(b_addr + 32 * k), idesc,
                         (c > 0 || k > 0) ? 1u : 0u);
             umma_commit(&b_empty[bs]);
-            // prefetch the next weight chunk into the other stage once its MMAs retired
-            const int64_t gn = g + 1;
-            if (gn < total_chunks) {
-              const int ns = (int)(gn & 1);
-              if (gn >= 2) mbar_wait(&b_empty[ns], (uint32_t)(((gn >> 1) - 1) & 1));
-              const int cnext = (int)(gn % p.nkc);
-              mbar_arrive_expect_tx(&b_full[ns], bbytes);
-              bulk_g2s(sB + ns * bbytes, p.wpk + (int64_t)cnext * bbytes, bbytes, &b_full[ns]);
-            }
             ++g;
+            top_up(g + NB - 1);
           }
           umma_commit(&a_empty[buf]);
         }
@@ -376,7 +382,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
         const int buf = (int)(q & 1);
         if (q >= 2) mbar_wait(&a_empty[buf], (uint32_t)(((q >> 1) - 1) & 1));
         const int c0 = sched.first(sc), ncs = sched.size(sc);
-        uint8_t* abuf = sA + buf * kSuper * kChunkBytesA;
+        uint8_t* abuf = sA + buf * AC * kChunkBytesA;
         if (c0 < p.nkc_self) {
           // self rows: 128 rows x (ncs * P) pieces, strided over the gather threads
           const int pcs = ncs * P;
@@ -596,7 +602,10 @@ buffalo_status tc_pack_weights(const float* W, int d_in, int d_out, void* packed
   return BUFFALO_OK;
 }
 
-static int smem_bytes_for(int Np) { return 2 * kSuper * kChunkBytesA + 2 * Np * 128 + 256 + 1024; }
+static int smem_bytes_for(int Np, int a_chunks, int nb) {
+  return 2 * a_chunks * kChunkBytesA + nb * Np * 128 + 8 * (8 + 2 * nb) + 64 + 1024;
+}
+static int smem_bytes_for(int Np) { return smem_bytes_for(Np, kSuper, 2); }
 
 bool tc_fwd_supported(const FwdArgs& a) {
   const int Np = (int)round_up(a.d_out, 16);
@@ -713,8 +722,17 @@ static bool use_fused() {
 }
 
 template <class TI, int MODE>
-static buffalo_status launch_tc(const TcFwdParams& p, cudaStream_t s) {
-  const int smem = smem_bytes_for(p.Np);
+static buffalo_status launch_tc(TcFwdParams p, cudaStream_t s) {
+  if (MODE == 2) {
+    // copy mode: small A buffers, deep weight prefetch (the weights stream once per tile)
+    p.a_chunks = 2;
+    const int budget = 220 * 1024 - smem_bytes_for(p.Np, 2, 0);
+    p.nb = std::max(2, std::min(8, budget / (p.Np * 128)));
+  } else {
+    p.a_chunks = kSuper;
+    p.nb = 2;
+  }
+  const int smem = smem_bytes_for(p.Np, p.a_chunks, p.nb);
   static bool attr_set = false;
   if (!attr_set) {
     BF_CUDA(cudaFuncSetAttribute(k_tc_sage_fwd<TI, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
