@@ -1,0 +1,302 @@
+// tc_gemm.cu — the Update GEMM over contiguous operands, TMA-fed (sm_100a).
+//
+//   out[i] = act([self[i] || agg[i]] W^T + b),   i < n_rows
+//
+// self and agg are row-major bf16 matrices whose rows are the tile rows (layers >= 2 of the
+// forward: H_{l-1} and the saved h_agg; the backward dH: dZ and the transposed sums), so both
+// halves of the A operand are plain 2D tiles: one TMA load (box 64 x 128, SWIZZLE_128B) per
+// K-chunk lands them in the UMMA K-major SW128 layout.  The pre-swizzled weight chunk of the
+// same K range comes with a 1D bulk copy into the same pipeline stage.  Roles: warp 4 lane 0
+// produces (TMA), warp 5 lane 0 issues tcgen05.mma into a double-buffered TMEM accumulator,
+// warps 0-3 run the epilogue (tcgen05.ld -> +bias -> ReLU -> store) of the previous tile.
+#include <cuda.h>
+
+#include <algorithm>
+
+#include "tc_sage.cuh"
+
+namespace buffalo {
+
+namespace {
+
+__device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mb_init(uint64_t* b, uint32_t c) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(b)), "r"(c));
+}
+__device__ __forceinline__ void mb_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(b)) : "memory");
+}
+__device__ __forceinline__ void mb_expect(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mb_wait(uint64_t* b, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@P1 bra DONE_%=;\n\t"
+      "bra WAIT_%=;\n\t"
+      "DONE_%=:\n\t}" ::"r"(su32(b)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_2d(void* dst, const CUtensorMap* map, int c0, int c1, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::
+          "r"(su32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(su32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void bulk_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   su32(dst)),
+               "l"(src), "r"(bytes), "r"(su32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ uint64_t desc_sw128(uint32_t saddr) {
+  return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
+         ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+}
+__device__ __forceinline__ void mma_f16(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(su32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void ld32(uint32_t taddr, float* v) {
+  uint32_t r[32];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+      "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+        "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+        "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ __forceinline__ uint32_t pk(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+constexpr int kTM = 128;
+constexpr int kChunkA = kTM * 128;     // 16 KB: 128 rows x 64 bf16
+constexpr int kEpiWarps = 4;
+constexpr int kGemmThreads = (kEpiWarps + 2) * 32;
+
+struct GemmParams {
+  int64_t n_rows;
+  int nkc_self, nkc;          // K-chunks of the self half, total
+  const uint8_t* wpk;         // pre-swizzled weight chunks (Np x 128 B each)
+  int Np, d_out, pitch_out, ld_out, tmem_cols, nstages;
+  const float* bias;
+  int relu, out_f32;
+  void* out;
+};
+
+__global__ void __launch_bounds__(kGemmThreads, 1)
+    k_tc_gemm_tma(const __grid_constant__ CUtensorMap self_map, const __grid_constant__ CUtensorMap agg_map,
+                  const GemmParams p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int NS = p.nstages;
+  const int bbytes = p.Np * 128;
+  uint8_t* sA = smem;                                  // NS x 16 KB
+  uint8_t* sB = smem + NS * kChunkA;                   // NS x Np x 128 B
+  uint64_t* full = (uint64_t*)(sB + NS * bbytes);
+  uint64_t* empty = full + NS;
+  uint64_t* acc_full = empty + NS;
+  uint64_t* acc_empty = acc_full + 2;
+  uint32_t* tmem_slot = (uint32_t*)(acc_empty + 2);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t ntiles = (p.n_rows + kTM - 1) / kTM;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NS; ++i) { mb_init(&full[i], 1); mb_init(&empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mb_init(&acc_full[i], 1); mb_init(&acc_empty[i], kEpiWarps * 32); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == kEpiWarps + 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
+                 "r"(p.tmem_cols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == kEpiWarps) {
+    if (lane == 0) {
+      // ---------------- producer: A chunk (TMA 2D) + weight chunk (bulk) per stage
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&self_map)) : "memory");
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&agg_map)) : "memory");
+      int64_t g = 0;
+      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const int row0 = (int)(t * kTM);
+        for (int c = 0; c < p.nkc; ++c, ++g) {
+          const int st = (int)(g % NS);
+          if (g >= NS) mb_wait(&empty[st], (uint32_t)(((g / NS) - 1) & 1));
+          mb_expect(&full[st], kChunkA + bbytes);
+          if (c < p.nkc_self) tma_2d(sA + st * kChunkA, &self_map, c * 64, row0, &full[st]);
+          else tma_2d(sA + st * kChunkA, &agg_map, (c - p.nkc_self) * 64, row0, &full[st]);
+          bulk_1d(sB + st * bbytes, p.wpk + (int64_t)c * bbytes, bbytes, &full[st]);
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == kEpiWarps + 1) {
+    if (lane == 0) {
+      // ---------------- MMA issuer
+      const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(p.Np >> 3) << 17) |
+                             ((uint32_t)(kTM >> 4) << 24);
+      int64_t g = 0, i = 0;
+      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+        const int acc = (int)(i & 1);
+        if (i >= 2) mb_wait(&acc_empty[acc], (uint32_t)(((i >> 1) - 1) & 1));
+        fence_after();
+        const uint32_t d = tmem + acc * p.Np;
+        for (int c = 0; c < p.nkc; ++c, ++g) {
+          const int st = (int)(g % NS);
+          mb_wait(&full[st], (uint32_t)((g / NS) & 1));
+          fence_after();
+          const uint32_t a = su32(sA + st * kChunkA), b = su32(sB + st * bbytes);
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            mma_f16(d, desc_sw128(a + 32 * k), desc_sw128(b + 32 * k), idesc, (c > 0 || k > 0) ? 1u : 0u);
+          commit(&empty[st]);
+        }
+        commit(&acc_full[acc]);
+      }
+    }
+    __syncwarp();
+  } else {
+    // ---------------- epilogue: warp w owns TMEM lanes (tile rows) 32w .. 32w + 31
+    int64_t i = 0;
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+      const int acc = (int)(i & 1);
+      mb_wait(&acc_full[acc], (uint32_t)((i >> 1) & 1));
+      fence_after();
+      const int64_t row = t * kTM + warp * 32 + lane;
+      for (int c0 = 0; c0 < p.pitch_out; c0 += 32) {
+        float v[32];
+        ld32(tmem + ((uint32_t)(warp * 32) << 16) + acc * p.Np + c0, v);
+        if (row < p.n_rows) {
+#pragma unroll
+          for (int k = 0; k < 32; ++k) {
+            const int cidx = c0 + k;
+            float x = v[k] + ((p.bias && cidx < p.d_out) ? __ldg(p.bias + cidx) : 0.f);
+            v[k] = p.relu ? fmaxf(x, 0.f) : x;
+          }
+          const int ncols = min(32, p.pitch_out - c0);   // multiple of 8
+          if (p.out_f32) {
+            float* o = (float*)p.out + row * p.ld_out + c0;
+#pragma unroll
+            for (int k = 0; k < 32; k += 4)
+              if (k < ncols) *reinterpret_cast<float4*>(o + k) = make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]);
+          } else {
+            __nv_bfloat16* o = (__nv_bfloat16*)p.out + row * p.ld_out + c0;
+#pragma unroll
+            for (int k = 0; k < 32; k += 8)
+              if (k < ncols)
+                *reinterpret_cast<uint4*>(o + k) =
+                    make_uint4(pk(v[k], v[k + 1]), pk(v[k + 2], v[k + 3]), pk(v[k + 4], v[k + 5]), pk(v[k + 6], v[k + 7]));
+          }
+        }
+      }
+      fence_before();
+      mb_arrive(&acc_empty[acc]);
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == kEpiWarps + 1) {
+    fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(p.tmem_cols));
+  }
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+buffalo_status encode_map(CUtensorMap* map, const void* base, int64_t cols, int64_t rows, int64_t ld) {
+  static EncodeTiledFn fn = nullptr;
+  if (!fn) {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    BF_CUDA(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q));
+    if (!f || q != cudaDriverEntryPointSuccess) {
+      set_error("cuTensorMapEncodeTiled unavailable");
+      return BUFFALO_ERR_CUDA;
+    }
+    fn = (EncodeTiledFn)f;
+  }
+  const cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)(rows > 0 ? rows : 1)};
+  const cuuint64_t strides[1] = {(cuuint64_t)ld * 2};
+  const cuuint32_t box[2] = {64, kTM};
+  const cuuint32_t estr[2] = {1, 1};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    set_error("cuTensorMapEncodeTiled failed (%d)", (int)r);
+    return BUFFALO_ERR_CUDA;
+  }
+  return BUFFALO_OK;
+}
+
+}  // namespace
+
+// out[n_rows][ld_out] = act([self || agg] W^T + b); self: bf16 [self_rows][ld_self] (first d_in
+// columns used, columns up to round_up(d_in, 64) read as zero beyond the pitch), agg likewise.
+buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const __nv_bfloat16* self, int64_t ld_self,
+                           const __nv_bfloat16* agg, int64_t ld_agg, int d_in, const uint8_t* wpk, int d_out,
+                           const float* bias, int relu, int out_f32, void* out, int64_t ld_out, cudaStream_t s) {
+  if (n_rows <= 0) return BUFFALO_OK;
+  CUtensorMap sm, am;
+  const int64_t pin = pitch_of(d_in);
+  // rows >= self_rows of the self half read as zero (TMA out-of-bounds fill)
+  BF_CHECK(encode_map(&sm, self, pin, self_rows, ld_self));
+  BF_CHECK(encode_map(&am, agg, pin, n_rows, ld_agg));
+  GemmParams p{};
+  p.n_rows = n_rows;
+  p.nkc_self = (int)ceil_div(d_in, 64);
+  p.nkc = 2 * p.nkc_self;
+  p.wpk = wpk;
+  p.Np = (int)round_up(d_out, 16);
+  p.d_out = d_out;
+  p.pitch_out = (int)pitch_of(d_out);
+  p.ld_out = (int)ld_out;
+  int cols = 32;
+  while (cols < 2 * p.Np) cols *= 2;
+  p.tmem_cols = cols;
+  p.bias = bias;
+  p.relu = relu;
+  p.out_f32 = out_f32;
+  p.out = out;
+  const int stage = kChunkA + p.Np * 128;
+  p.nstages = std::max(2, std::min(8, (200 * 1024) / stage));
+  const int smem = p.nstages * stage + 16 * p.nstages + 64 + 1024;
+  static bool attr = false;
+  if (!attr) {
+    BF_CUDA(cudaFuncSetAttribute(k_tc_gemm_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    attr = true;
+  }
+  const int grid = (int)std::min<int64_t>(ceil_div(n_rows, kTM), 148);
+  k_tc_gemm_tma<<<grid, kGemmThreads, smem, s>>>(sm, am, p);
+  BF_LAUNCHED("k_tc_gemm_tma");
+  return BUFFALO_OK;
+}
+
+}  // namespace buffalo

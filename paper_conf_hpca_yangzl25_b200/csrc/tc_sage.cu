@@ -712,6 +712,15 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   return BUFFALO_OK;
 }
 
+static bool use_cpasync_gemm() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("BUFFALO_CPASYNC_GEMM");
+    v = (e && e[0] == '1') ? 1 : 0;
+  }
+  return v == 1;
+}
+
 static bool use_fused() {
   static int v = -1;
   if (v < 0) {
@@ -786,6 +795,9 @@ static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   // split: high-occupancy gather of the non-heavy rows, then the Update GEMM over copies
   BF_CHECK((launch_gather<TI, 0>(blk->cls_perm, blk->row_ptr, p.col, blk->n_dst, (const TI*)a.h_src, a.ld_src,
                                  p.pitch_in, (__nv_bfloat16*)a.agg, a.ld_agg, s)));
+  if (!a.layer1 && a.in_bf16 && !use_cpasync_gemm())
+    return tc_gemm_tma(blk->n_dst, blk->n_dst, (const __nv_bfloat16*)a.h_src, a.ld_src, (const __nv_bfloat16*)a.agg, a.ld_agg,
+                       a.d_in, p.wpk, a.d_out, a.b, a.relu, a.out_f32, a.out, a.ld_out, s);
   p.perm = nullptr;
   p.agg_src = (const __nv_bfloat16*)a.agg;
   p.ld_agg_src = a.ld_agg;
@@ -1228,6 +1240,11 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     p.agg = nullptr;
     p.ld_agg = 0;
     if (!use_fused()) {
+      if (!use_cpasync_gemm()) {
+        // self half = dZ rows (rows >= n_dst are zero: the map covers n_dst rows only)
+        return tc_gemm_tma(blk->n_src, n, zb, dp, hbuf, dp, d_out, p.wpk, d_in, nullptr, 0, 1, a.dh_src, a.ld_dh_src,
+                           s);
+      }
       p.perm = nullptr;
       p.agg_src = hbuf;
       p.ld_agg_src = dp;
