@@ -47,6 +47,14 @@ __device__ __forceinline__ void tma_2d(void* dst, const CUtensorMap* map, int c0
       "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(su32(bar))
       : "memory");
 }
+__device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, int c0, int r0, int r1, int r2, int r3,
+                                            uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, "
+      "%4, %5, %6}], [%7];" ::"r"(su32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(su32(bar))
+      : "memory");
+}
 __device__ __forceinline__ void bulk_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                    su32(dst)),
@@ -96,6 +104,8 @@ constexpr int kGemmThreads = (kEpiWarps + 2) * 32;
 
 struct GemmParams {
   int64_t n_rows;
+  const int32_t* self_idx;    // null: self rows are rows of the self map; else row i = self_idx[i] (gather4)
+  int32_t self_oob;           // an out-of-bounds row index of the self map (zero rows)
   int nkc_self, nkc;          // K-chunks of the self half, total
   const uint8_t* wpk;         // pre-swizzled weight chunks (Np x 128 B each)
   int Np, d_out, pitch_out, ld_out, tmem_cols, nstages;
@@ -137,24 +147,40 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   const uint32_t tmem = *tmem_slot;
 
   if (warp == kEpiWarps) {
+    // ---------------- producer: A chunk (TMA 2D, or 32 x gather4 for gathered self rows) +
+    // weight chunk (bulk) per stage
     if (lane == 0) {
-      // ---------------- producer: A chunk (TMA 2D) + weight chunk (bulk) per stage
       asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&self_map)) : "memory");
       asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&agg_map)) : "memory");
-      int64_t g = 0;
-      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        const int row0 = (int)(t * kTM);
-        for (int c = 0; c < p.nkc; ++c, ++g) {
-          const int st = (int)(g % NS);
-          if (g >= NS) mb_wait(&empty[st], (uint32_t)(((g / NS) - 1) & 1));
-          mb_expect(&full[st], kChunkA + bbytes);
-          if (c < p.nkc_self) tma_2d(sA + st * kChunkA, &self_map, c * 64, row0, &full[st]);
-          else tma_2d(sA + st * kChunkA, &agg_map, (c - p.nkc_self) * 64, row0, &full[st]);
-          bulk_1d(sB + st * bbytes, p.wpk + (int64_t)c * bbytes, bbytes, &full[st]);
+    }
+    int64_t g = 0;
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      const int row0 = (int)(t * kTM);
+      int32_t idx[4];
+      if (p.self_idx) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int64_t r = (int64_t)row0 + lane * 4 + k;
+          idx[k] = r < p.n_rows ? __ldg(p.self_idx + r) : p.self_oob;
         }
       }
+      for (int c = 0; c < p.nkc; ++c, ++g) {
+        const int st = (int)(g % NS);
+        if (lane == 0) {
+          if (g >= NS) mb_wait(&empty[st], (uint32_t)(((g / NS) - 1) & 1));
+          mb_expect(&full[st], kChunkA + bbytes);
+        }
+        __syncwarp();
+        if (c < p.nkc_self && p.self_idx) {
+          tma_gather4(sA + st * kChunkA + lane * 4 * 128, &self_map, c * 64, idx[0], idx[1], idx[2], idx[3], &full[st]);
+        } else if (lane == 0) {
+          if (c < p.nkc_self) tma_2d(sA + st * kChunkA, &self_map, c * 64, row0, &full[st]);
+          else tma_2d(sA + st * kChunkA, &agg_map, (c - p.nkc_self) * 64, row0, &full[st]);
+        }
+        if (lane == 0) bulk_1d(sB + st * bbytes, p.wpk + (int64_t)c * bbytes, bbytes, &full[st]);
+        __syncwarp();
+      }
     }
-    __syncwarp();
   } else if (warp == kEpiWarps + 1) {
     if (lane == 0) {
       // ---------------- MMA issuer
@@ -230,7 +256,8 @@ typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
-buffalo_status encode_map(CUtensorMap* map, const void* base, int64_t cols, int64_t rows, int64_t ld) {
+buffalo_status encode_map(CUtensorMap* map, const void* base, int64_t cols, int64_t rows, int64_t ld,
+                          int box_rows = kTM) {
   static EncodeTiledFn fn = nullptr;
   if (!fn) {
     void* f = nullptr;
@@ -244,7 +271,7 @@ buffalo_status encode_map(CUtensorMap* map, const void* base, int64_t cols, int6
   }
   const cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)(rows > 0 ? rows : 1)};
   const cuuint64_t strides[1] = {(cuuint64_t)ld * 2};
-  const cuuint32_t box[2] = {64, kTM};
+  const cuuint32_t box[2] = {64, (cuuint32_t)box_rows};
   const cuuint32_t estr[2] = {1, 1};
   CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -260,17 +287,21 @@ buffalo_status encode_map(CUtensorMap* map, const void* base, int64_t cols, int6
 
 // out[n_rows][ld_out] = act([self || agg] W^T + b); self: bf16 [self_rows][ld_self] (first d_in
 // columns used, columns up to round_up(d_in, 64) read as zero beyond the pitch), agg likewise.
-buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const __nv_bfloat16* self, int64_t ld_self,
-                           const __nv_bfloat16* agg, int64_t ld_agg, int d_in, const uint8_t* wpk, int d_out,
-                           const float* bias, int relu, int out_f32, void* out, int64_t ld_out, cudaStream_t s) {
+buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* self_idx, const __nv_bfloat16* self,
+                           int64_t ld_self, const __nv_bfloat16* agg, int64_t ld_agg, int d_in, const uint8_t* wpk,
+                           int d_out, const float* bias, int relu, int out_f32, void* out, int64_t ld_out,
+                           cudaStream_t s) {
   if (n_rows <= 0) return BUFFALO_OK;
   CUtensorMap sm, am;
   const int64_t pin = pitch_of(d_in);
-  // rows >= self_rows of the self half read as zero (TMA out-of-bounds fill)
-  BF_CHECK(encode_map(&sm, self, pin, self_rows, ld_self));
+  // self_idx: self rows gathered (row i = self_idx[i] of a [self_rows] table, box 64 x 1);
+  // else rows >= self_rows of the self half read as zero (TMA out-of-bounds fill)
+  BF_CHECK(encode_map(&sm, self, pin, self_rows, ld_self, self_idx ? 1 : kTM));
   BF_CHECK(encode_map(&am, agg, pin, n_rows, ld_agg));
   GemmParams p{};
   p.n_rows = n_rows;
+  p.self_idx = self_idx;
+  p.self_oob = self_idx ? 0 : (int32_t)self_rows;
   p.nkc_self = (int)ceil_div(d_in, 64);
   p.nkc = 2 * p.nkc_self;
   p.wpk = wpk;

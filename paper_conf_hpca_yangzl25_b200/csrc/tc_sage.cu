@@ -712,6 +712,10 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   return BUFFALO_OK;
 }
 
+// Feature-table rows are addressed through src_global only; the gathered tensor map spans the
+// largest row count TMA accepts and tile padding rows gather row 0 (their outputs are dropped).
+constexpr int64_t kGatherTableRows = 0x7fffffff;
+
 static bool use_cpasync_gemm() {
   static int v = -1;
   if (v < 0) {
@@ -795,8 +799,9 @@ static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   // split: high-occupancy gather of the non-heavy rows, then the Update GEMM over copies
   BF_CHECK((launch_gather<TI, 0>(blk->cls_perm, blk->row_ptr, p.col, blk->n_dst, (const TI*)a.h_src, a.ld_src,
                                  p.pitch_in, (__nv_bfloat16*)a.agg, a.ld_agg, s)));
-  if (!a.layer1 && a.in_bf16 && !use_cpasync_gemm())
-    return tc_gemm_tma(blk->n_dst, blk->n_dst, (const __nv_bfloat16*)a.h_src, a.ld_src, (const __nv_bfloat16*)a.agg, a.ld_agg,
+  if (a.in_bf16 && !use_cpasync_gemm())
+    return tc_gemm_tma(blk->n_dst, a.layer1 ? kGatherTableRows : blk->n_dst, a.layer1 ? blk->src_global : nullptr,
+                       (const __nv_bfloat16*)a.h_src, a.ld_src, (const __nv_bfloat16*)a.agg, a.ld_agg,
                        a.d_in, p.wpk, a.d_out, a.b, a.relu, a.out_f32, a.out, a.ld_out, s);
   p.perm = nullptr;
   p.agg_src = (const __nv_bfloat16*)a.agg;
@@ -1242,8 +1247,8 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     if (!use_fused()) {
       if (!use_cpasync_gemm()) {
         // self half = dZ rows (rows >= n_dst are zero: the map covers n_dst rows only)
-        return tc_gemm_tma(blk->n_src, n, zb, dp, hbuf, dp, d_out, p.wpk, d_in, nullptr, 0, 1, a.dh_src, a.ld_dh_src,
-                           s);
+        return tc_gemm_tma(blk->n_src, n, nullptr, zb, dp, hbuf, dp, d_out, p.wpk, d_in, nullptr, 0, 1, a.dh_src,
+                           a.ld_dh_src, s);
       }
       p.perm = nullptr;
       p.agg_src = hbuf;

@@ -126,13 +126,14 @@ def _run_microbatch(tr, seeds, fan, F, seed):
 
 
 @pytest.mark.parametrize("name", list(CASES))
-@pytest.mark.parametrize("gemm", ["ffma", "bf16"])
+@pytest.mark.parametrize("gemm", ["ffma", "bf16", "bf16feat"])
 def test_microbatch_fwd_bwd_parity(name, gemm):
     rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case(name)
     g = O.Graph(rp, col)
     L = len(fan)
     mode = B.GEMM_FFMA if gemm == "ffma" else B.GEMM_BF16
-    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=mode)
+    fdt = B.BF16 if gemm == "bf16feat" else B.FP32      # bf16 feature table: the bench's configuration
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=mode, feat_dtype=fdt)
     S = seeds.size
     info = _run_microbatch(tr, seeds, fan, F, 7)
     blocks = O.build_blocks(g, seeds, L, fan, 7)
@@ -184,13 +185,14 @@ def test_mean_of_constant_is_constant():
     assert np.all(agg[D > 0] == 0.5) and np.all(agg[D == 0] == 0.0)
 
 
-@pytest.mark.parametrize("gemm", ["ffma", "bf16"])
+@pytest.mark.parametrize("gemm", ["ffma", "bf16", "bf16feat"])
 def test_microbatch_logits_equal_batch_logits(gemm):
     """micro-batch training is equivalent to batch training; on the GPU the
     per-seed logits of a group equal the full batch's bit for bit (row-local reductions)."""
     rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case("mixed3")
     mode = B.GEMM_FFMA if gemm == "ffma" else B.GEMM_BF16
-    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=mode)
+    fdt = B.BF16 if gemm == "bf16feat" else B.FP32
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=mode, feat_dtype=fdt)
     _run_microbatch(tr, seeds, fan, F, 5)
     bl = tr.blocks.layer[-1 + len(fan)]
     full = act_view(tr.arena, bl.out, bl.n_dst, bl.ld_out, torch.float32).copy()
@@ -202,13 +204,15 @@ def test_microbatch_logits_equal_batch_logits(gemm):
         np.testing.assert_array_equal(sub, full[[pos[int(s)] for s in part]])
 
 
-@pytest.mark.parametrize("gemm", ["ffma", "bf16"])
+@pytest.mark.parametrize("gemm", ["ffma", "bf16", "bf16feat"])
 def test_epoch_parity(gemm):
     """Alg. 2 end to end: plan, accumulated gradients over K = 4 groups, one SGD step."""
     rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case("sampled2")
     g = O.Graph(rp, col)
     mode = B.GEMM_FFMA if gemm == "ffma" else B.GEMM_BF16
-    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=mode, k_min=4, k_max=4, base_seed=3)
+    fdt = B.BF16 if gemm == "bf16feat" else B.FP32
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=mode, k_min=4, k_max=4, base_seed=3,
+                      feat_dtype=fdt)
     lr = 0.5
     stats = tr.run_epoch(epoch=2, lr=lr)
     torch.cuda.synchronize()
