@@ -233,7 +233,7 @@ def mem_model(n, e, dims, act_dtype=FP32):
         frame = _R(64) + _scan_ws_bytes(max(nl + el + 1, pne + 1))
         frame += _R(4 * (pne + 1))                              # partition counts (classes, radix)
         if l >= 2:
-            frame += 6 * _R(4 * el)                             # col_global + radix buffers
+            frame += _R(4 * el) + _R(4 * (nl + el))             # col_global + transpose cursors
         build = max(build, frame)
     acts = 0
     for l in range(1, L + 1):

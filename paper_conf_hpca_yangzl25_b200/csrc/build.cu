@@ -138,6 +138,54 @@ __global__ void k_tcount(const int32_t* __restrict__ col_local, int64_t e, int32
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x)
     atomicAdd(&cnt[col_local[k]], 1);
 }
+// Transposed fill: edge (i -> col_local[e]) lands at an atomic cursor of its src row.
+__global__ void __launch_bounds__(256) k_tfill(const int32_t* __restrict__ rp, const int32_t* __restrict__ col_local,
+                                               int64_t n, int32_t* __restrict__ cursor, int32_t* __restrict__ tcol) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n; i += warps)
+    for (int32_t k = rp[i] + lane; k < rp[i + 1]; k += 32) tcol[atomicAdd(&cursor[col_local[k]], 1)] = (int32_t)i;
+}
+// Ascending sort of transposed rows with <= 128 entries (warp per row, up to 4 values per lane,
+// rank = number of smaller entries; entries are distinct).
+__global__ void __launch_bounds__(256) k_tsort_small(const int32_t* __restrict__ rows, int64_t n,
+                                                     const int32_t* __restrict__ trp, int32_t* __restrict__ tcol) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < n; w += warps) {
+    const int32_t j = rows[w];
+    const int32_t b = trp[j], len = trp[j + 1] - b;
+    if (len <= 1) continue;
+    int32_t v[4];
+    int rank[4] = {0, 0, 0, 0};
+#pragma unroll
+    for (int k = 0; k < 4; ++k) v[k] = (lane + 32 * k < len) ? tcol[b + lane + 32 * k] : INT32_MAX;
+    for (int src = 0; src < len; ++src) {
+      const int32_t x = __shfl_sync(0xffffffffu, v[src >> 5], src & 31);
+#pragma unroll
+      for (int k = 0; k < 4; ++k) rank[k] += x < v[k] ? 1 : 0;
+    }
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+      if (lane + 32 * k < len) tcol[b + rank[k]] = v[k];
+  }
+}
+// Long transposed rows (> 128 entries): CTA per row; the row is staged in `stage` (same
+// offsets as t_col), then every entry is written at its rank among the staged values.
+__global__ void __launch_bounds__(256) k_tsort_heavy(const int32_t* __restrict__ rows, const int32_t* __restrict__ trp,
+                                                     int32_t* __restrict__ tcol, int32_t* __restrict__ stage) {
+  const int32_t j = rows[blockIdx.x];
+  const int32_t b = trp[j], len = trp[j + 1] - b;
+  for (int32_t k = threadIdx.x; k < len; k += blockDim.x) stage[b + k] = tcol[b + k];
+  __syncthreads();
+  for (int32_t k = threadIdx.x; k < len; k += blockDim.x) {
+    const int32_t x = stage[b + k];
+    int32_t r = 0;
+    for (int32_t t = 0; t < len; ++t) r += stage[b + t] < x ? 1 : 0;
+    tcol[b + r] = x;
+  }
+}
 // ed[e] = dst index of edge e (warp per dst row).
 __global__ void k_edge_dst(const int32_t* __restrict__ rp, int64_t n, int32_t* __restrict__ ed) {
   const int lane = threadIdx.x & 31;
@@ -177,7 +225,7 @@ int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only) 
   const int64_t pne = part_count_elems(n_dst + e);   // bounds the partitions of n_dst, n_src, e
   const int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pne + 1);
   int64_t fr = R(64) + R(4 * scan_ws_elems(scan_len)) + R(4 * (pne + 1));
-  if (layer >= 2) fr += 6 * R(4 * e);
+  if (layer >= 2) fr += R(4 * e) + R(4 * (n_dst + e));        // col_global + transposed-fill cursors
   return fr;
 }
 
@@ -271,15 +319,14 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     BF_LAUNCHED("k_reset_map");
   }
   if (!sizes_only && layer >= 2) {
-    // transposed block: t_row_ptr by counting, t_col by a stable LSD radix sort of the edges
-    // (dst-ordered) keyed by col_local => each transposed row lists its dst ascending.
+    // transposed block: t_row_ptr by counting; t_col by an atomic-cursor fill followed by an
+    // ascending sort of every transposed row (entries are distinct dst indices, so the sorted
+    // row equals the stable order of the dst-ordered edges); degree classes of the src rows.
     int32_t* trp = (int32_t*)A.take(4 * (n_src + 1));
     int32_t* tcol = (int32_t*)A.take(4 * e);
     int32_t* tperm = (int32_t*)A.take(4 * n_src);
     if (A.overflow) return BUFFALO_ERR_CAPACITY;
-    int32_t* ed = (int32_t*)q; q += R(4 * e);
-    int32_t* bufk[2] = {(int32_t*)q, (int32_t*)(q + R(4 * e))}; q += 2 * R(4 * e);
-    int32_t* bufp[2] = {(int32_t*)q, (int32_t*)(q + R(4 * e))}; q += 2 * R(4 * e);
+    int32_t* cursor = (int32_t*)q; q += R(4 * (n_dst + e));
     k_fill_zero<<<grid_for(n_src + 1, 256), 256, 0, s>>>(trp, n_src + 1);
     BF_LAUNCHED("k_fill_zero");
     if (e > 0) {
@@ -287,31 +334,30 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
       BF_LAUNCHED("k_tcount");
     }
     BF_CHECK(scan_inplace(trp, n_src, ws, s));
-    // degree classes of the transposed rows (long-tail src go last)
     BF_CHECK(stable_partition(DegClass{trp}, EmitPerm{tperm}, n_src, counts, ws, s));
     BF_CHECK(device_count(HeavyFlag{trp}, n_src, totals + 1, s));
     int32_t nht = 0;
     BF_CHECK(d2h_i32(totals + 1, &nht, s));
     if (e > 0) {
-      k_edge_dst<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(rp, n_dst, ed);
-      BF_LAUNCHED("k_edge_dst");
-      int bits = 1;
-      while ((1LL << bits) < n_src) ++bits;
-      const int passes = (bits + 7) / 8;
-      const int32_t* kin = col_local;
-      const int32_t* pin = ed;
-      for (int p = 0; p < passes; ++p) {
-        int32_t* kout = bufk[p & 1];
-        int32_t* pout = (p == passes - 1) ? tcol : bufp[p & 1];
-        BF_CHECK(stable_partition(RadixKey{kin, 8 * p}, RadixEmit{kin, pin, kout, pout}, e, counts, ws, s));
-        kin = kout;
-        pin = pout;
+      BF_CUDA(cudaMemcpyAsync(cursor, trp, sizeof(int32_t) * n_src, cudaMemcpyDeviceToDevice, s));
+      k_tfill<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(rp, col_local, n_dst, cursor, tcol);
+      BF_LAUNCHED("k_tfill");
+    }
+    BF_CUDA(cudaStreamSynchronize(s));                             // n_heavy_t
+    if (e > 0) {
+      const int64_t n_small = n_src - nht;
+      if (n_small > 0) {
+        k_tsort_small<<<grid_for(n_small * 32, 256, 16), 256, 0, s>>>(tperm, n_small, trp, tcol);
+        BF_LAUNCHED("k_tsort_small");
+      }
+      if (nht > 0) {
+        k_tsort_heavy<<<(unsigned)nht, 256, 0, s>>>(tperm + n_small, trp, tcol, cursor);
+        BF_LAUNCHED("k_tsort_heavy");
       }
     }
     blk->t_row_ptr = trp;
     blk->t_col = tcol;
     blk->t_perm = tperm;
-    BF_CUDA(cudaStreamSynchronize(s));                             // n_heavy_t
     blk->n_heavy_t = nht;
   }
   A.pop_frame();
