@@ -252,6 +252,150 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   }
 }
 
+
+// ================================================================== dW on tensor cores, TMA-fed
+// part[split][m][n'] = sum_{r in split} dZ[r][m] * Afwd[r][n'],  Afwd = [self || agg] with n'
+// padded per half to Dp.  Both operands are MN-major in shared memory: a 64-column strip of 64
+// rows is exactly one TMA box {64, 64} with SWIZZLE_128B (gathered self rows: 16 x gather4).
+// One CTA owns all m-tiles (<= 2 x 128 TMEM lanes) of one 256-wide n'-tile and a row split.
+constexpr int kDwR = 64;
+constexpr int kDwStrip2 = kDwR * 128;      // 8 KB
+
+struct DwParams {
+  int64_t n, rows_per_split;
+  int MT, NT, Dp, nself_strips, d_out, tmem_cols, nstages;
+  const int32_t* gidx;                     // layer 1: self row r = gidx[r]
+  float* part;
+};
+
+__device__ __forceinline__ uint64_t desc_mn(uint32_t saddr, uint32_t lbo) {
+  return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+         ((uint64_t)(1024 >> 4) << 32) | ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+}
+
+__global__ void __launch_bounds__(192, 1)
+    k_tc_dw_tma(const __grid_constant__ CUtensorMap z_map, const __grid_constant__ CUtensorMap self_map,
+                const __grid_constant__ CUtensorMap agg_map, const DwParams p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int NS = p.nstages;
+  const int nA = 2 * p.MT, nB = p.NT / 64;
+  const int stage = (nA + nB) * kDwStrip2;
+  uint64_t* full = (uint64_t*)(smem + NS * stage);
+  uint64_t* empty = full + NS;
+  uint64_t* done = empty + NS;
+  uint32_t* tmem_slot = (uint32_t*)(done + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int n0 = blockIdx.x * p.NT;
+  const int64_t r_beg = (int64_t)blockIdx.y * p.rows_per_split;
+  const int64_t r_end = min(p.n, r_beg + p.rows_per_split);
+  const int nchunks = r_end > r_beg ? (int)((r_end - r_beg + kDwR - 1) / kDwR) : 0;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NS; ++i) { mb_init(&full[i], 1); mb_init(&empty[i], 1); }
+    mb_init(done, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 5) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
+                 "r"(p.tmem_cols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *tmem_slot;
+  if (warp == 4) {
+    // ---------------- producer
+    for (int c = 0; c < nchunks; ++c) {
+      const int st = c % NS;
+      const int r0 = (int)(r_beg + (int64_t)c * kDwR);
+      if (lane == 0) {
+        if (c >= NS) mb_wait(&empty[st], (uint32_t)(((c / NS) - 1) & 1));
+        mb_expect(&full[st], stage);
+      }
+      __syncwarp();
+      uint8_t* sa = smem + st * stage;
+      uint8_t* sb = sa + nA * kDwStrip2;
+      if (lane == 0) {
+        for (int j = 0; j < nA; ++j) tma_2d(sa + j * kDwStrip2, &z_map, j * 64, r0, &full[st]);
+      }
+      for (int j = 0; j < nB; ++j) {
+        const int np = n0 + j * 64;               // first n' column of the strip
+        if (np < p.Dp) {
+          if (p.gidx) {
+            // 64 gathered rows = 16 gather4; lanes 0..15 issue one each
+            if (lane < 16) {
+              int32_t rr[4];
+#pragma unroll
+              for (int k = 0; k < 4; ++k) {
+                const int64_t r = (int64_t)r0 + lane * 4 + k;
+                rr[k] = r < p.n ? __ldg(p.gidx + r) : 0;
+              }
+              tma_gather4(sb + j * kDwStrip2 + lane * 4 * 128, &self_map, np, rr[0], rr[1], rr[2], rr[3], &full[st]);
+            }
+          } else if (lane == 0) {
+            tma_2d(sb + j * kDwStrip2, &self_map, np, r0, &full[st]);
+          }
+        } else if (lane == 0) {
+          tma_2d(sb + j * kDwStrip2, &agg_map, np - p.Dp, r0, &full[st]);
+        }
+      }
+      __syncwarp();
+    }
+  } else if (warp == 5) {
+    if (lane == 0) {
+      const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 15) | (1u << 16) |
+                             ((uint32_t)(p.NT >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+      for (int c = 0; c < nchunks; ++c) {
+        const int st = c % NS;
+        mb_wait(&full[st], (uint32_t)((c / NS) & 1));
+        fence_after();
+        const uint32_t a = su32(smem + st * stage), b = a + nA * kDwStrip2;
+        for (int mt = 0; mt < p.MT; ++mt)
+#pragma unroll
+          for (int kk = 0; kk < kDwR / 16; ++kk)
+            mma_f16(tmem + mt * p.NT, desc_mn(a + mt * 2 * kDwStrip2 + kk * 2048, kDwStrip2),
+                    desc_mn(b + kk * 2048, kDwStrip2), idesc, (c > 0 || kk > 0) ? 1u : 0u);
+        commit(&empty[st]);
+      }
+      if (nchunks > 0) commit(done);
+    }
+    __syncwarp();
+  } else {
+    // ---------------- epilogue: warp w -> TMEM lane quadrant w (m rows), all m-tiles
+    if (nchunks > 0) {
+      mb_wait(done, 0);
+      fence_after();
+    }
+    const int64_t K2 = 2 * (int64_t)p.Dp;
+    float* P = p.part + (int64_t)blockIdx.y * p.d_out * K2;
+    for (int mt = 0; mt < p.MT; ++mt) {
+      const int m = mt * 128 + warp * 32 + lane;
+      for (int c0 = 0; c0 < p.NT; c0 += 32) {
+        float v[32];
+        if (nchunks > 0) {
+          ld32(tmem + ((uint32_t)(warp * 32) << 16) + mt * p.NT + c0, v);
+        } else {
+#pragma unroll
+          for (int k = 0; k < 32; ++k) v[k] = 0.f;
+        }
+        const int nn = n0 + c0;
+        if (m < p.d_out && nn < K2) {
+          float* o = P + (int64_t)m * K2 + nn;
+#pragma unroll
+          for (int k = 0; k < 32; k += 4) *reinterpret_cast<float4*>(o + k) = make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]);
+        }
+      }
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 5) {
+    fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(p.tmem_cols));
+  }
+}
+
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -284,6 +428,44 @@ buffalo_status encode_map(CUtensorMap* map, const void* base, int64_t cols, int6
 }
 
 }  // namespace
+
+// dW partials with TMA operands.  z: bf16 dZ [n][ldz] (first d_out columns); self: bf16 rows
+// (gidx: gathered from a table), agg: bf16 saved h_agg [n][lda].  part: [S][d_out][2 Dp].
+buffalo_status tc_dw_tma(int64_t n, int S, const __nv_bfloat16* z, int64_t ldz, int d_out,
+                         const __nv_bfloat16* self, int64_t lds, const int32_t* gidx, int64_t self_table_rows,
+                         const __nv_bfloat16* agg, int64_t lda, int d_in, float* part, cudaStream_t s) {
+  if (n <= 0) return BUFFALO_OK;
+  const int64_t Dp = round_up(d_in, 64);
+  const int64_t pin = pitch_of(d_in), pz = pitch_of(d_out);
+  CUtensorMap zm, sm, am;
+  BF_CHECK(encode_map(&zm, z, pz, n, ldz, kDwR));
+  BF_CHECK(encode_map(&sm, self, pin, gidx ? self_table_rows : n, lds, gidx ? 1 : kDwR));
+  BF_CHECK(encode_map(&am, agg, pin, n, lda, kDwR));
+  DwParams p{};
+  p.n = n;
+  p.MT = (int)ceil_div(d_out, 128);
+  p.NT = (int)std::min<int64_t>(256, 2 * Dp);
+  p.Dp = (int)Dp;
+  p.d_out = d_out;
+  p.gidx = gidx;
+  p.part = part;
+  p.rows_per_split = round_up(ceil_div(n, S), kDwR);
+  int cols = 32;
+  while (cols < p.MT * p.NT) cols *= 2;
+  p.tmem_cols = cols;
+  const int stage = (2 * p.MT + p.NT / 64) * kDwStrip2;
+  p.nstages = std::max(2, std::min(6, (200 * 1024) / stage));
+  const int smem = p.nstages * stage + 16 * p.nstages + 64 + 1024;
+  static bool attr = false;
+  if (!attr) {
+    BF_CUDA(cudaFuncSetAttribute(k_tc_dw_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    attr = true;
+  }
+  dim3 grid((unsigned)ceil_div(2 * Dp, p.NT), (unsigned)S);
+  k_tc_dw_tma<<<grid, 192, smem, s>>>(zm, sm, am, p);
+  BF_LAUNCHED("k_tc_dw_tma");
+  return BUFFALO_OK;
+}
 
 // out[n_rows][ld_out] = act([self || agg] W^T + b); self: bf16 [self_rows][ld_self] (first d_in
 // columns used, columns up to round_up(d_in, 64) read as zero beyond the pitch), agg likewise.

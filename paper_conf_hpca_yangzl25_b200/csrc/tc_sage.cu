@@ -1194,14 +1194,18 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   dim3 grid((unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
   static bool attr[2] = {false, false};
   constexpr int kMaxDwSmem = kDwStages * (4 + 4) * kDwStrip + 128 + 1024;
-  if (a.in_bf16) {
+  if (a.in_bf16 && !use_cpasync_gemm()) {
+    BF_CHECK(tc_dw_tma(n, S, zb, dp, d_out, (const __nv_bfloat16*)a.h_src, a.ld_src, w.gidx, kGatherTableRows,
+                       (const __nv_bfloat16*)a.agg, a.ld_agg, d_in, dw_part, s));
+  } else if (a.in_bf16) {
     if (!attr[0]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr[0] = true; }
     k_tc_dw<__nv_bfloat16><<<grid, kDwThreads, smem, s>>>(w);
+    BF_LAUNCHED("k_tc_dw");
   } else {
     if (!attr[1]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr[1] = true; }
     k_tc_dw<float><<<grid, kDwThreads, smem, s>>>(w);
+    BF_LAUNCHED("k_tc_dw");
   }
-  BF_LAUNCHED("k_tc_dw");
   k_reduce_dw<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, d_out, d_in, (int)Dp, a.dW);
   BF_LAUNCHED("k_reduce_dw");
   k_reduce_db<<<1, 256, 0, s>>>(db_part, kDbSplits, d_out, a.db);
