@@ -195,18 +195,27 @@ BUFFALO_API buffalo_status buffalo_softmax_ce(const float* logits, int64_t ld, i
 /* Scratch bytes buffalo_sage_bwd needs for block blk at layer l. */
 BUFFALO_API size_t buffalo_sage_bwd_scratch_bytes(const buffalo_block* blk, int32_t layer,
                                       const buffalo_model* m);
-/* Backward of layer l (Alg. 2 l.11-12).  dh_dst: dH_l fp32 (l < L; turned
- * into dZ_l = dH_l * 1[H_l > 0] IN PLACE using h_dst) or dlogits (l = L).
+/* Backward of layer l (Alg. 2 l.11-12).
+ *   dZ_l = dH_l * 1[H_l > 0] (l < L) or dlogits (l = L)
  *   dW_accum += dZ^T [H[:n_dst] || h_agg];  db_accum += sum_i dZ[i]   (accumulated, R19)
- *   l > 1: dh_src = pad(dZ W_self) + (sum_{i: j in N(i)} dZ[i] / D(i)) W_neigh   (dH_{l-1})
- * Pass dh_src = NULL for layer 1 (features are not trained). */
+ *   l > 1: dH_{l-1} = pad(dZ W_self) + (sum_{i: j in N(i)} dZ[i] / D(i)) W_neigh
+ * FFMA mode: dh_dst holds dH_l fp32 (l < L; masked IN PLACE using h_dst) or dlogits (l = L);
+ * dh_src receives dH_{l-1} fp32.
+ * BF16 mode: dh_dst holds dlogits fp32 at l = L; for l < L it holds the layer's prepared
+ * backward input as written by the layer above: bf16 dZ_l [n_dst][p(d_l)], then (l >= 2) bf16
+ * dZ_l / D_l [n_dst][p(d_l)], then at byte offset R(4 n_dst p(d_l)) fp32 column-sum partials
+ * of dZ_l [min(ceil(n_dst/128), 148)][d_l]; dh_src receives the same prepared form of layer
+ * l-1 (the Update GEMM's epilogue applies ReLU' with h_src = H_{l-1} and divides by
+ * D_{l-1}(j) = prev_row_ptr[j+1] - prev_row_ptr[j]), so the buffer must hold
+ * R(4 n_src p(d_{l-1})) + R(4 * 148 * d_{l-1}) bytes.  prev_row_ptr: block l-1's row_ptr (l >= 3
+ * in BF16 mode; NULL otherwise).  Pass dh_src = NULL for layer 1 (features are not trained). */
 BUFFALO_API buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
                                 float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
                                 const void* saved_agg, int64_t ld_agg, const void* h_dst,
                                 int64_t ld_hdst, const float* W, const void* W_packed,
                                 float* dW_accum, float* db_accum, float* dh_src,
-                                int64_t ld_dh_src, void* scratch, size_t scratch_bytes,
-                                void* stream);
+                                int64_t ld_dh_src, const int32_t* prev_row_ptr, void* scratch,
+                                size_t scratch_bytes, void* stream);
 
 /* ------------------------------------------------------------------ a10: optimizer */
 /* SGD (Alg. 2 l.13, R18): param -= lr * grad; grad = 0 (ready for the next epoch). */

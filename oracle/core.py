@@ -241,24 +241,34 @@ def mem_model(n, e, dims, act_dtype=FP32):
         if l < L:
             acts += _R(n[l] * pitch(dims[l]) * s)               # H_l
     acts += _R(n[L] * pitch(dims[L]) * 4)                       # logits
+    def dh_slot(l):                                             # dH_l slot of the backward region
+        b = _R(n[l] * pitch(dims[l]) * 4)                       # fp32 dH / dlogits; bf16 dZ + dZ/D
+        if act_dtype == BF16 and l < L:
+            b += _R(4 * 148 * dims[l])                          # GEMM-epilogue db partials
+        return b
+
     bwd = 0
     for l in range(L, 0, -1):
-        frame = _R(n[l] * pitch(dims[l]) * 4)                   # dH_l (dlogits at l = L)
+        frame = dh_slot(l)
         if l >= 2:
-            frame += _R(n[l - 1] * pitch(dims[l - 1]) * 4)      # dH_{l-1}
+            frame += dh_slot(l - 1)
         if act_dtype == FP32:
             if l >= 2:
                 frame += _R(n[l - 1] * pitch(dims[l]) * 4)      # transposed aggregate of dZ/D
             S = dw_splits(n[l], dims[l], dims[l - 1])
             frame += _R(S * dims[l] * 2 * dims[l - 1] * 4) + _R(S * pitch(dims[l]) * 4)  # dW, db partials
         else:
-            frame += _R(n[l] * pitch(dims[l]) * 2)              # dZ in bf16
+            if l == L:
+                frame += _R(n[l] * pitch(dims[l]) * 2)          # dZ in bf16 (from dlogits)
+                if l >= 2:
+                    frame += _R(n[l] * pitch(dims[l]) * 2)      # dZ / D in bf16
             if l >= 2:
-                frame += _R(n[l] * pitch(dims[l]) * 2)          # dZ / D in bf16
                 frame += _R(n[l - 1] * pitch(dims[l]) * 2)      # transposed sums in bf16
             S = tc_dw_splits(n[l], dims[l], dims[l - 1])
             Dp = _ceil(dims[l - 1], 64) * 64
-            frame += _R(S * dims[l] * 2 * Dp * 4) + _R(DB_SPLITS * dims[l] * 4)         # dW, db partials
+            frame += _R(S * dims[l] * 2 * Dp * 4)               # dW partials
+            if l == L:
+                frame += _R(DB_SPLITS * dims[l] * 4)            # db partials
         bwd = max(bwd, frame)
     lo = blocks + acts + bwd
     hi = blocks + acts + max(bwd, build)

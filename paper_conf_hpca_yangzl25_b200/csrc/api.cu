@@ -59,8 +59,17 @@ __global__ void k_fill_i32(int32_t* a, int64_t n, int32_t v) {
 // ------------------------------------------------------------------ memory model (R15)
 // Restated from DESIGN.md §5; must agree with the arena that buffalo_build_blocks lays out.
 static int64_t bwd_scratch_for(const buffalo_model* m, int64_t n_dst, int64_t n_src, int64_t e, int l) {
-  if (m->gemm_mode == BUFFALO_GEMM_BF16) return tc_bwd_scratch_bytes(n_dst, n_src, e, l, m->dim[l - 1], m->dim[l]);
+  if (m->gemm_mode == BUFFALO_GEMM_BF16)
+    return tc_bwd_scratch_bytes(n_dst, n_src, e, l, m->dim[l - 1], m->dim[l], l == m->num_layers);
   return bwd_scratch_bytes(n_dst, n_src, l, m->dim[l - 1], m->dim[l]);
+}
+
+// dH_l slot of the backward region: fp32 dH (FFMA) / dlogits; in BF16 mode layers l < L hold
+// bf16 dZ and dZ/D (same bytes) plus the epilogue's column-sum partials.
+static int64_t dh_slot_bytes(const buffalo_model* m, int64_t n, int l) {
+  int64_t b = R(n * pitch_of(m->dim[l]) * 4);
+  if (m->gemm_mode == BUFFALO_GEMM_BF16 && l < m->num_layers) b += R((int64_t)4 * 148 * m->dim[l]);
+  return b;
 }
 
 static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_model* m,
@@ -79,8 +88,8 @@ static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_m
   }
   acts += R(n[L] * pitch_of(m->dim[L]) * 4);
   for (int l = L; l >= 1; --l) {
-    int64_t f = R(n[l] * pitch_of(m->dim[l]) * 4);
-    if (l >= 2) f += R(n[l - 1] * pitch_of(m->dim[l - 1]) * 4);
+    int64_t f = dh_slot_bytes(m, n[l], l);
+    if (l >= 2) f += dh_slot_bytes(m, n[l - 1], l - 1);
     f += bwd_scratch_for(m, n[l], n[l - 1], e[l - 1], l);
     bwd = std::max(bwd, f);
   }
@@ -502,7 +511,7 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
   // backward region: ping-pong dH buffers at the two ends, scratch in between
   int64_t B = 0;
   std::vector<int64_t> ah(L + 1, 0), tmp(L + 1, 0);
-  for (int l = 1; l <= L; ++l) ah[l] = R(nn[l] * pitch_of(m->dim[l]) * 4);
+  for (int l = 1; l <= L; ++l) ah[l] = dh_slot_bytes(m, nn[l], l);
   for (int l = L; l >= 1; --l) {
     tmp[l] = bwd_scratch_for(m, nn[l], nn[l - 1], ee[l - 1], l);
     B = std::max(B, ah[l] + (l >= 2 ? ah[l - 1] : 0) + tmp[l]);
@@ -598,8 +607,8 @@ buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const b
                                 float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
                                 const void* saved_agg, int64_t ld_agg, const void* h_dst,
                                 int64_t ld_hdst, const float* W, const void* W_packed, float* dW_accum,
-                                float* db_accum, float* dh_src, int64_t ld_dh_src, void* scratch,
-                                size_t scratch_bytes, void* stream) {
+                                float* db_accum, float* dh_src, int64_t ld_dh_src, const int32_t* prev_row_ptr,
+                                void* scratch, size_t scratch_bytes, void* stream) {
   BF_CHECK(require_sm100());
   BF_CHECK(validate_model(m));
   if (!blk || layer < 1 || layer > m->num_layers || !dh_dst || !h_src || !saved_agg || !W ||
@@ -636,6 +645,11 @@ buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const b
   a.db = db_accum;
   a.dh_src = dh_src;
   a.ld_dh_src = ld_dh_src;
+  a.prev_row_ptr = prev_row_ptr;
+  if (m->gemm_mode == BUFFALO_GEMM_BF16 && dh_src && layer >= 3 && !prev_row_ptr) {
+    set_error("sage_bwd: bf16 mode needs block l-1's row_ptr for l >= 3");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
   a.scratch = scratch;
   a.scratch_bytes = (int64_t)scratch_bytes;
   cudaStream_t s = (cudaStream_t)stream;

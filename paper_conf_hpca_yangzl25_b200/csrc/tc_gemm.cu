@@ -112,6 +112,12 @@ struct GemmParams {
   const float* bias;
   int relu, out_f32;
   void* out;
+  // backward epilogue (epi != 0): out = prepared dZ of the layer below
+  int epi;
+  const __nv_bfloat16* H; int64_t ldH;   // ReLU' mask source H_{l-1}
+  const int32_t* rp;                     // block l-1 row_ptr (D for the dZ/D copy) or null
+  __nv_bfloat16* zb; __nv_bfloat16* zs;  // [n_rows][pitch_out] bf16 outputs (zs nullable)
+  float* db_part;                        // [gridDim.x][d_out]
 };
 
 __global__ void __launch_bounds__(kGemmThreads, 1)
@@ -206,6 +212,91 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       }
     }
     __syncwarp();
+  } else if (p.epi) {
+    // ---------------- backward epilogue: dZ = acc * 1[H > 0] -> bf16 dZ, bf16 dZ/D, and
+    // per-warp column sums (fixed row order), combined per CTA at the end
+    float dbacc[8];
+#pragma unroll
+    for (int g = 0; g < 8; ++g) dbacc[g] = 0.f;
+    int64_t i = 0;
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+      const int acc = (int)(i & 1);
+      mb_wait(&acc_full[acc], (uint32_t)((i >> 1) & 1));
+      fence_after();
+      const int64_t row = t * kTM + warp * 32 + lane;
+      const bool rok = row < p.n_rows;
+      float invd = 1.f;
+      if (rok && p.zs) {
+        const int32_t d = __ldg(p.rp + row + 1) - __ldg(p.rp + row);
+        invd = d > 0 ? 1.f / (float)d : 0.f;
+      }
+#pragma unroll
+      for (int g = 0; g < 8; ++g) {
+        const int c0 = g * 32;
+        if (c0 >= p.pitch_out) break;
+        float v[32];
+        ld32(tmem + ((uint32_t)(warp * 32) << 16) + acc * p.Np + c0, v);
+        const int ncols = min(32, p.pitch_out - c0);
+        if (rok) {
+          const __nv_bfloat16* hr = p.H + row * p.ldH + c0;
+#pragma unroll
+          for (int k = 0; k < 32; k += 8) {
+            if (k < ncols) {
+              const uint4 hu = __ldg(reinterpret_cast<const uint4*>(hr + k));
+              const uint32_t hw[4] = {hu.x, hu.y, hu.z, hu.w};
+#pragma unroll
+              for (int q = 0; q < 4; ++q) {
+                const float h0 = __uint_as_float(hw[q] << 16), h1 = __uint_as_float(hw[q] & 0xffff0000u);
+                if (!(h0 > 0.f) || c0 + k + 2 * q >= p.d_out) v[k + 2 * q] = 0.f;
+                if (!(h1 > 0.f) || c0 + k + 2 * q + 1 >= p.d_out) v[k + 2 * q + 1] = 0.f;
+              }
+            } else {
+#pragma unroll
+              for (int q = 0; q < 8; ++q) v[k + q] = 0.f;
+            }
+          }
+          __nv_bfloat16* zo = p.zb + row * p.pitch_out + c0;
+#pragma unroll
+          for (int k = 0; k < 32; k += 8)
+            if (k < ncols)
+              *reinterpret_cast<uint4*>(zo + k) =
+                  make_uint4(pk(v[k], v[k + 1]), pk(v[k + 2], v[k + 3]), pk(v[k + 4], v[k + 5]), pk(v[k + 6], v[k + 7]));
+          if (p.zs) {
+            __nv_bfloat16* so = p.zs + row * p.pitch_out + c0;
+#pragma unroll
+            for (int k = 0; k < 32; k += 8)
+              if (k < ncols)
+                *reinterpret_cast<uint4*>(so + k) =
+                    make_uint4(pk(v[k] * invd, v[k + 1] * invd), pk(v[k + 2] * invd, v[k + 3] * invd),
+                               pk(v[k + 4] * invd, v[k + 5] * invd), pk(v[k + 6] * invd, v[k + 7] * invd));
+          }
+        } else {
+#pragma unroll
+          for (int k = 0; k < 32; ++k) v[k] = 0.f;
+        }
+        // column sums over the warp's 32 rows; lane k keeps column c0 + k
+#pragma unroll
+        for (int k = 0; k < 32; ++k) {
+          float x = v[k];
+#pragma unroll
+          for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+          if (lane == k) dbacc[g] += x;
+        }
+      }
+      fence_before();
+      mb_arrive(&acc_empty[acc]);
+    }
+    // combine the four warps in order -> one partial per CTA
+    float* red = reinterpret_cast<float*>(sA);     // stage 0 A buffer: the producer is done
+    asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
+#pragma unroll
+    for (int g = 0; g < 8; ++g) red[warp * 256 + g * 32 + lane] = dbacc[g];
+    asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
+    for (int c = threadIdx.x; c < p.d_out; c += kEpiWarps * 32) {
+      float t = 0.f;
+      for (int w = 0; w < kEpiWarps; ++w) t += red[w * 256 + c];
+      p.db_part[(int64_t)blockIdx.x * p.d_out + c] = t;
+    }
   } else {
     // ---------------- epilogue: warp w owns TMEM lanes (tile rows) 32w .. 32w + 31
     int64_t i = 0;
@@ -472,7 +563,7 @@ buffalo_status tc_dw_tma(int64_t n, int S, const __nv_bfloat16* z, int64_t ldz, 
 buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* self_idx, const __nv_bfloat16* self,
                            int64_t ld_self, const __nv_bfloat16* agg, int64_t ld_agg, int d_in, const uint8_t* wpk,
                            int d_out, const float* bias, int relu, int out_f32, void* out, int64_t ld_out,
-                           cudaStream_t s) {
+                           cudaStream_t s, const GemmEpi* epi) {
   if (n_rows <= 0) return BUFFALO_OK;
   CUtensorMap sm, am;
   const int64_t pin = pitch_of(d_in);
@@ -498,6 +589,11 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   p.relu = relu;
   p.out_f32 = out_f32;
   p.out = out;
+  if (epi) {
+    p.epi = 1;
+    p.H = epi->H; p.ldH = epi->ldH; p.rp = epi->rp;
+    p.zb = epi->zb; p.zs = epi->zs; p.db_part = epi->db_part;
+  }
   const int stage = kChunkA + p.Np * 128;
   p.nstages = std::max(2, std::min(8, (200 * 1024) / stage));
   const int smem = p.nstages * stage + 16 * p.nstages + 64 + 1024;
@@ -506,7 +602,7 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
     BF_CUDA(cudaFuncSetAttribute(k_tc_gemm_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
     attr = true;
   }
-  const int grid = (int)std::min<int64_t>(ceil_div(n_rows, kTM), 148);
+  const int grid = (int)gemm_grid(n_rows);
   k_tc_gemm_tma<<<grid, kGemmThreads, smem, s>>>(sm, am, p);
   BF_LAUNCHED("k_tc_gemm_tma");
   return BUFFALO_OK;

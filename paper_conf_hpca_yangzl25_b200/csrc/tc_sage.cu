@@ -1141,16 +1141,18 @@ int tc_dw_splits(int64_t n, int d_out, int d_in) {
   return (int)std::max<int64_t>(1, sp);
 }
 
-int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int64_t e, int layer, int d_in, int d_out) {
+int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int64_t e, int layer, int d_in, int d_out, bool last) {
   (void)e;
   const int S = tc_dw_splits(n_dst, d_out, d_in);
   const int64_t Dp = round_up(d_in, 64);
-  int64_t b = R(n_dst * pitch_of(d_out) * 2);                        // dZ bf16
-  if (layer >= 2) {
-    b += R(n_dst * pitch_of(d_out) * 2);                              // dZ / D bf16
-    b += R(n_src * pitch_of(d_out) * 2);                              // transposed sums (bf16)
+  int64_t b = 0;
+  if (last) {
+    b += R(n_dst * pitch_of(d_out) * 2);                              // dZ bf16
+    if (layer >= 2) b += R(n_dst * pitch_of(d_out) * 2);              // dZ / D bf16
   }
-  b += R((int64_t)S * d_out * 2 * Dp * 4) + R((int64_t)kDbSplits * d_out * 4);
+  if (layer >= 2) b += R(n_src * pitch_of(d_out) * 2);                // transposed sums (bf16)
+  b += R((int64_t)S * d_out * 2 * Dp * 4);                            // dW partials
+  if (last) b += R((int64_t)kDbSplits * d_out * 4);                   // db partials (dz_prep)
   return b;
 }
 
@@ -1165,102 +1167,84 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   const int dp = (int)pitch_of(d_out);
   const int S = tc_dw_splits(n, d_out, d_in);
   const int64_t Dp = round_up(d_in, 64);
+  const bool need_zs = a.dh_src != nullptr;
+  // prepared input of this layer: bf16 dZ (+ dZ/D) and db partials
+  __nv_bfloat16 *zb, *zs = nullptr;
+  float* db_part;
+  int nparts;
   char* q = (char*)a.scratch;
-  __nv_bfloat16* zb = (__nv_bfloat16*)q; q += R(n * dp * 2);
-  __nv_bfloat16* zs = nullptr;
-  __nv_bfloat16* hbuf = nullptr;
-  if (a.dh_src) {
-    zs = (__nv_bfloat16*)q; q += R(n * dp * 2);
-    hbuf = (__nv_bfloat16*)q; q += R(blk->n_src * dp * 2);
-  }
-  float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * Dp * 4);
-  float* db_part = (float*)q;
-  if (n <= 0) return BUFFALO_OK;
-  k_dz_prep<__nv_bfloat16><<<kDbSplits, 256, 0, s>>>(
-      a.dh, a.ld_dh, a.last ? nullptr : (const __nv_bfloat16*)a.h_dst, a.ld_hdst, blk->row_ptr, n, d_out, dp, zb, zs,
-      db_part);
-  BF_LAUNCHED("k_dz_prep");
-  // dW and db
-  TcDwParams w{};
-  w.zb = zb; w.ldz = dp;
-  w.self_ = a.h_src; w.lds = a.ld_src; w.gidx = a.layer1 ? blk->src_global : nullptr;
-  w.agg = (const __nv_bfloat16*)a.agg; w.lda = a.ld_agg;
-  w.n = n; w.d_out = d_out; w.d_in = d_in; w.pitch_in = (int)pitch_of(d_in); w.pz = dp; w.Dp = (int)Dp;
-  w.NT = (int)std::min<int64_t>(256, 2 * Dp);
-  w.MT = (int)ceil_div(d_out, 128);
-  w.rows_per_split = ceil_div(n, S);
-  w.part = dw_part;
-  const int smem = kDwStages * (2 * w.MT + w.NT / 64) * kDwStrip + 128 + 1024;
-  dim3 grid((unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
-  static bool attr[2] = {false, false};
-  constexpr int kMaxDwSmem = kDwStages * (4 + 4) * kDwStrip + 128 + 1024;
-  if (a.in_bf16 && !use_cpasync_gemm()) {
-    BF_CHECK(tc_dw_tma(n, S, zb, dp, d_out, (const __nv_bfloat16*)a.h_src, a.ld_src, w.gidx, kGatherTableRows,
-                       (const __nv_bfloat16*)a.agg, a.ld_agg, d_in, dw_part, s));
-  } else if (a.in_bf16) {
-    if (!attr[0]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr[0] = true; }
-    k_tc_dw<__nv_bfloat16><<<grid, kDwThreads, smem, s>>>(w);
-    BF_LAUNCHED("k_tc_dw");
+  if (a.last) {
+    zb = (__nv_bfloat16*)q; q += R(n * dp * 2);
+    if (need_zs) { zs = (__nv_bfloat16*)q; q += R(n * dp * 2); }
   } else {
-    if (!attr[1]) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr[1] = true; }
+    zb = (__nv_bfloat16*)a.dh;
+    if (need_zs) zs = zb + n * dp;
+  }
+  __nv_bfloat16* aggT = nullptr;
+  if (need_zs) { aggT = (__nv_bfloat16*)q; q += R(blk->n_src * dp * 2); }
+  float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * Dp * 4);
+  if (a.last) {
+    db_part = (float*)q;
+    nparts = kDbSplits;
+  } else {
+    db_part = (float*)((char*)a.dh + R(n * dp * 4));
+    nparts = (int)gemm_grid(n);
+  }
+  if (n <= 0) return BUFFALO_OK;
+  if (a.last) {
+    k_dz_prep<__nv_bfloat16><<<kDbSplits, 256, 0, s>>>(a.dh, a.ld_dh, nullptr, 0, blk->row_ptr, n, d_out, dp, zb, zs,
+                                                       db_part);
+    BF_LAUNCHED("k_dz_prep");
+  }
+  // dW (TMA-fed tensor cores, deterministic split reduction) and db
+  if (a.in_bf16) {
+    BF_CHECK(tc_dw_tma(n, S, zb, dp, d_out, (const __nv_bfloat16*)a.h_src, a.ld_src,
+                       a.layer1 ? blk->src_global : nullptr, kGatherTableRows, (const __nv_bfloat16*)a.agg,
+                       a.ld_agg, d_in, dw_part, s));
+  } else {
+    TcDwParams w{};
+    w.zb = zb; w.ldz = dp;
+    w.self_ = a.h_src; w.lds = a.ld_src; w.gidx = a.layer1 ? blk->src_global : nullptr;
+    w.agg = (const __nv_bfloat16*)a.agg; w.lda = a.ld_agg;
+    w.n = n; w.d_out = d_out; w.d_in = d_in; w.pitch_in = (int)pitch_of(d_in); w.pz = dp; w.Dp = (int)Dp;
+    w.NT = (int)std::min<int64_t>(256, 2 * Dp);
+    w.MT = (int)ceil_div(d_out, 128);
+    w.rows_per_split = ceil_div(n, S);
+    w.part = dw_part;
+    const int smem = kDwStages * (2 * w.MT + w.NT / 64) * kDwStrip + 128 + 1024;
+    dim3 grid((unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
+    static bool attr = false;
+    constexpr int kMaxDwSmem = kDwStages * (4 + 4) * kDwStrip + 128 + 1024;
+    if (!attr) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr = true; }
     k_tc_dw<float><<<grid, kDwThreads, smem, s>>>(w);
     BF_LAUNCHED("k_tc_dw");
   }
   k_reduce_dw<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, d_out, d_in, (int)Dp, a.dW);
   BF_LAUNCHED("k_reduce_dw");
-  k_reduce_db<<<1, 256, 0, s>>>(db_part, kDbSplits, d_out, a.db);
+  k_reduce_db<<<1, 256, 0, s>>>(db_part, nparts, d_out, a.db);
   BF_LAUNCHED("k_reduce_db");
-  // dH_{l-1} = [dZ (rows < n_dst) || sum_{i in T(j)} dZ[i]/D(i)] [W_self; W_neigh]
+  // dH_{l-1} = [dZ (rows < n_dst) || sum_{i in T(j)} dZ[i]/D(i)] [W_self; W_neigh], written in the
+  // prepared form of layer l-1 by the GEMM epilogue (ReLU' with H_{l-1}, /D_{l-1}, db partials)
   if (a.dh_src && blk->n_src > 0) {
     if (blk->n_heavy_t > 0) {
       k_sum_heavy_rows<<<(unsigned)blk->n_heavy_t, 256, 0, s>>>(blk->t_perm + (blk->n_src - blk->n_heavy_t),
-                                                                blk->t_row_ptr, blk->t_col, zs, dp, dp, hbuf,
-                                                                use_fused() ? 0 : 1);
+                                                                blk->t_row_ptr, blk->t_col, zs, dp, dp, aggT, 1);
       BF_LAUNCHED("k_sum_heavy_rows");
     }
-    if (!use_fused())
-      BF_CHECK((launch_gather<__nv_bfloat16, 1>(blk->t_perm, blk->t_row_ptr, blk->t_col, blk->n_src, zs, dp, dp,
-                                                hbuf, dp, s)));
-    TcFwdParams p{};
-    p.perm = blk->t_perm;
-    p.heavy_base = blk->n_src - blk->n_heavy_t;
-    p.heavy_buf = hbuf;
-    p.heavy_ld = dp;
-    p.row_ptr = blk->t_row_ptr;
-    p.col = blk->t_col;
-    p.gidx = nullptr;
-    p.n_dst = blk->n_src;
-    p.self_rows = n;
-    p.h = zs; p.ldh = dp;
-    p.hs = zb; p.lds = dp;
-    p.d_in = d_out;
-    p.pitch_in = dp;
-    p.nkc_self = (int)ceil_div(d_out, kKC);
-    p.nkc = 2 * p.nkc_self;
-    p.wpk = (const uint8_t*)a.W_packed + R((int64_t)2 * d_in * d_out * 4) + tc_fwd_packed_bytes(d_in, d_out);
-    p.Np = (int)round_up(d_in, 16);
-    p.d_out = d_in;
-    p.ld_out = (int)a.ld_dh_src;
-    p.tmem_cols = tmem_cols_for(p.Np);
-    p.bias = nullptr;
-    p.relu = 0;
-    p.out_f32 = 1;
-    p.out = a.dh_src;
-    p.agg = nullptr;
-    p.ld_agg = 0;
-    if (!use_fused()) {
-      if (!use_cpasync_gemm()) {
-        // self half = dZ rows (rows >= n_dst are zero: the map covers n_dst rows only)
-        return tc_gemm_tma(blk->n_src, n, nullptr, zb, dp, hbuf, dp, d_out, p.wpk, d_in, nullptr, 0, 1, a.dh_src,
-                           a.ld_dh_src, s);
-      }
-      p.perm = nullptr;
-      p.agg_src = hbuf;
-      p.ld_agg_src = dp;
-      BF_CHECK((launch_tc<__nv_bfloat16, 2>(p, s)));
-      return BUFFALO_OK;
-    }
-    BF_CHECK((launch_tc<__nv_bfloat16, 1>(p, s)));
+    BF_CHECK((launch_gather<__nv_bfloat16, 1>(blk->t_perm, blk->t_row_ptr, blk->t_col, blk->n_src, zs, dp, dp,
+                                              aggT, dp, s)));
+    const int64_t ns = blk->n_src;
+    const int dpp = (int)pitch_of(d_in);
+    GemmEpi epi{};
+    epi.H = (const __nv_bfloat16*)a.h_src;
+    epi.ldH = a.ld_src;
+    epi.zb = (__nv_bfloat16*)a.dh_src;
+    epi.zs = a.prev_row_ptr ? epi.zb + ns * dpp : nullptr;     // layer l-1 >= 2 needs dZ/D
+    epi.rp = a.prev_row_ptr;
+    epi.db_part = (float*)((char*)a.dh_src + R(ns * dpp * 4));
+    const uint8_t* wpk = (const uint8_t*)a.W_packed + R((int64_t)2 * d_in * d_out * 4) + tc_fwd_packed_bytes(d_in, d_out);
+    // self half = dZ rows (rows >= n_dst are zero: the map covers n_dst rows only)
+    BF_CHECK(tc_gemm_tma(ns, n, nullptr, zb, dp, aggT, dp, d_out, wpk, d_in, nullptr, 0, 0, nullptr, 0, s, &epi));
   }
   return BUFFALO_OK;
 }
