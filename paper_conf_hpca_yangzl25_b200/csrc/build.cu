@@ -22,43 +22,77 @@ __global__ void k_count(const int32_t* __restrict__ dst, int64_t n, const int64_
 }
 
 // ------------------------------------------------------------------ a4: sample / slice
-// Warp per dst.  deg <= f or f <= 0: the warp copies the CSR row (coalesced).  Otherwise
-// Floyd's algorithm (R2): lane t computes r_t = floor(x_t (j_t + 1) / 2^32), j_t = deg - f + t;
-// the sequential membership test runs as f ballot steps; the chosen positions are then
-// ranked (sorted ascending) inside the warp and the neighbours gathered.
+// A warp serves 32/SEG destination rows (SEG lanes each, SEG >= f).  deg <= f or f <= 0: the
+// segment copies the CSR row.  Otherwise Floyd's algorithm (R2): lane t of the segment computes
+// r_t = floor(x_t (j_t + 1) / 2^32), j_t = deg - f + t; the sequential membership test runs as
+// f ballot steps (all lanes execute them, so sampling and copying segments may share a warp);
+// the chosen positions are ranked (sorted ascending) inside the segment.
+// emit(slot, k, u): neighbour number k (ascending CSR position) of the warp's row `slot` is u.
+template <int SEG, class RowFn, class Emit>
+__device__ __forceinline__ void sample_warp_rows(int64_t w, int64_t n, RowFn row_of, const int64_t* __restrict__ grow,
+                                                 const int32_t* __restrict__ gcol, int32_t f, uint32_t hop,
+                                                 uint64_t seed, Emit emit) {
+  constexpr int G = 32 / SEG;
+  const int lane = threadIdx.x & 31, g = lane / SEG, sl = lane % SEG;
+  const int64_t slot = w * G + g;
+  uint32_t v = 0;
+  int64_t beg = 0, deg = 0;
+  if (slot < n) {
+    v = (uint32_t)row_of(slot);
+    beg = grow[v];
+    deg = grow[v + 1] - beg;
+  }
+  const bool samp = slot < n && f > 0 && deg > f;
+  if (__any_sync(0xffffffffu, samp)) {
+    const uint32_t j = (uint32_t)(deg - f) + (uint32_t)sl;
+    uint32_t r = 0;
+    if (samp && sl < f) r = __umulhi(sample_draw(seed, v, hop, (uint32_t)sl), j + 1u);
+    int32_t S = -1;
+    const unsigned segmask = (SEG == 32) ? 0xffffffffu : (((1u << SEG) - 1u) << (g * SEG));
+    for (int t = 0; t < f; ++t) {
+      const int32_t cand = (int32_t)__shfl_sync(0xffffffffu, r, g * SEG + t);
+      const unsigned present = __ballot_sync(0xffffffffu, sl < t && S == cand) & segmask;
+      if (sl == t) S = present ? (int32_t)((uint32_t)(deg - f) + (uint32_t)t) : cand;
+    }
+    int rank = 0;
+    for (int u = 0; u < f; ++u) {
+      const int32_t su = __shfl_sync(0xffffffffu, S, g * SEG + u);
+      rank += (su < S) ? 1 : 0;
+    }
+    if (samp && sl < f) emit(slot, rank, gcol[beg + S]);
+  }
+  if (slot < n && !samp)
+    for (int64_t k = sl; k < deg; k += SEG) emit(slot, (int32_t)k, gcol[beg + k]);
+}
+
+struct DstRows {
+  const int32_t* dst;
+  __device__ __forceinline__ int64_t operator()(int64_t i) const { return dst[i]; }
+};
+
+template <int SEG>
 __global__ void __launch_bounds__(256) k_sample_fill(const int32_t* __restrict__ dst, int64_t n,
                                                      const int64_t* __restrict__ grow,
                                                      const int32_t* __restrict__ gcol, int32_t f,
                                                      uint32_t hop, uint64_t seed,
                                                      const int32_t* __restrict__ row_ptr,
                                                      int32_t* __restrict__ out) {
-  const int lane = threadIdx.x & 31;
+  constexpr int G = 32 / SEG;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n; i += warps) {
-    const uint32_t v = (uint32_t)dst[i];
-    const int64_t beg = grow[v];
-    const int64_t deg = grow[v + 1] - beg;
-    int32_t* o = out + row_ptr[i];
-    if (f <= 0 || deg <= f) {
-      for (int64_t k = lane; k < deg; k += 32) o[k] = gcol[beg + k];
-      continue;
-    }
-    const uint32_t j = (uint32_t)(deg - f) + (uint32_t)lane;
-    uint32_t r = 0;
-    if (lane < f) r = __umulhi(sample_draw(seed, v, hop, (uint32_t)lane), j + 1u);
-    int32_t S = -1;
-    for (int t = 0; t < f; ++t) {
-      const int32_t cand = (int32_t)__shfl_sync(0xffffffffu, r, t);
-      const unsigned present = __ballot_sync(0xffffffffu, lane < t && S == cand);
-      if (lane == t) S = present ? (int32_t)((uint32_t)(deg - f) + (uint32_t)t) : cand;
-    }
-    int rank = 0;
-    for (int u = 0; u < f; ++u) {
-      const int32_t su = __shfl_sync(0xffffffffu, S, u);
-      rank += (su < S) ? 1 : 0;
-    }
-    if (lane < f) o[rank] = gcol[beg + S];
-  }
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n; w += warps)
+    sample_warp_rows<SEG>(w, n, DstRows{dst}, grow, gcol, f, hop, seed,
+                          [&](int64_t slot, int32_t k, int32_t u) { out[row_ptr[slot] + k] = u; });
+}
+
+static inline int sample_seg(int32_t f) { return (f > 0 && f <= 8) ? 8 : (f > 0 && f <= 16) ? 16 : 32; }
+
+template <class... Args>
+static void launch_sample_fill(int seg, int64_t n, cudaStream_t s, Args... args) {
+  const int G = 32 / seg;
+  const int grid = grid_for(ceil_div(n, G) * 32, 256, 16);
+  if (seg == 8) k_sample_fill<8><<<grid, 256, 0, s>>>(args...);
+  else if (seg == 16) k_sample_fill<16><<<grid, 256, 0, s>>>(args...);
+  else k_sample_fill<32><<<grid, 256, 0, s>>>(args...);
 }
 
 // ------------------------------------------------------------------ a5: relabel
@@ -280,8 +314,8 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     BF_CHECK(stable_partition(DegClass{rp}, EmitPerm{perm}, n_dst, counts, ws, s));
   }
   if (n_dst > 0) {
-    k_sample_fill<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(dst, n_dst, g->row_ptr, g->col, f, hop,
-                                                               seed, rp, colg);
+    launch_sample_fill(sample_seg(f), n_dst, s, dst, n_dst, g->row_ptr, g->col, f, hop, seed, (const int32_t*)rp,
+                       colg);
     BF_LAUNCHED("k_sample_fill");
   }
   // relabel: first occurrence over the candidate sequence dst ++ col_global
@@ -446,8 +480,10 @@ __global__ void __launch_bounds__(256) k_mask_seed(const int32_t* __restrict__ i
   }
 }
 
-// One layer: warp per active node v of layer l; accumulates n_l, e_l per item and ORs v's mask
-// into layer l-1 for v itself and its sampled neighbours, appending first touches to act_out.
+// One layer: 32/SEG active nodes of layer l per warp; accumulates n_l, e_l per item (lane k
+// handles items k and k+32 of each node) and ORs each node's mask into layer l-1 for the node
+// itself and its sampled neighbours, appending first touches to act_out.
+template <int SEG>
 __global__ void __launch_bounds__(256) k_mask_layer(const int32_t* __restrict__ act, int64_t n_act,
                                                     const unsigned long long* __restrict__ m_in,
                                                     unsigned long long* __restrict__ m_out,
@@ -455,44 +491,35 @@ __global__ void __launch_bounds__(256) k_mask_layer(const int32_t* __restrict__ 
                                                     const int64_t* __restrict__ grow, const int32_t* __restrict__ gcol,
                                                     int32_t f, uint32_t hop, uint64_t seed,
                                                     unsigned long long* __restrict__ gn, unsigned long long* __restrict__ ge) {
+  constexpr int G = 32 / SEG;
   __shared__ unsigned long long sn[64], se[64];
   if (threadIdx.x < 64) { sn[threadIdx.x] = 0; se[threadIdx.x] = 0; }
   __syncthreads();
-  const int lane = threadIdx.x & 31;
+  const int lane = threadIdx.x & 31, g = lane / SEG;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n_act; i += warps) {
-    const uint32_t v = (uint32_t)act[i];
-    const unsigned long long mask = m_in[v];
-    const int64_t beg = grow[v];
-    const int64_t deg = grow[v + 1] - beg;
-    const int64_t D = (f > 0 && deg > f) ? f : deg;
-    // per-item sizes: lane k handles items k and k + 32
-    if ((mask >> lane) & 1ull) { atomicAdd(&sn[lane], 1ull); atomicAdd(&se[lane], (unsigned long long)D); }
-    if ((mask >> (lane + 32)) & 1ull) {
-      atomicAdd(&sn[lane + 32], 1ull);
-      atomicAdd(&se[lane + 32], (unsigned long long)D);
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n_act; w += warps) {
+    const int64_t slot = w * G + g;
+    uint32_t v = 0;
+    unsigned long long mask = 0;
+    int64_t D = 0;
+    if (slot < n_act) {
+      v = (uint32_t)act[slot];
+      mask = m_in[v];
+      const int64_t deg = grow[v + 1] - grow[v];
+      D = (f > 0 && deg > f) ? f : deg;
     }
-    if (lane == 0 && atomicOr(&m_out[v], mask) == 0ull) act_out[atomicAdd(n_out, 1)] = (int32_t)v;
-    if (f <= 0 || deg <= f) {
-      for (int64_t k = lane; k < deg; k += 32) {
-        const int32_t u = gcol[beg + k];
-        if (atomicOr(&m_out[u], mask) == 0ull) act_out[atomicAdd(n_out, 1)] = u;
-      }
-    } else {
-      const uint32_t j = (uint32_t)(deg - f) + (uint32_t)lane;
-      uint32_t r = 0;
-      if (lane < f) r = __umulhi(sample_draw(seed, v, hop, (uint32_t)lane), j + 1u);
-      int32_t S = -1;
-      for (int t = 0; t < f; ++t) {
-        const int32_t cand = (int32_t)__shfl_sync(0xffffffffu, r, t);
-        const unsigned present = __ballot_sync(0xffffffffu, lane < t && S == cand);
-        if (lane == t) S = present ? (int32_t)((uint32_t)(deg - f) + (uint32_t)t) : cand;
-      }
-      if (lane < f) {
-        const int32_t u = gcol[beg + S];
-        if (atomicOr(&m_out[u], mask) == 0ull) act_out[atomicAdd(n_out, 1)] = u;
-      }
+    for (int q = 0; q < G; ++q) {
+      const unsigned long long mq = __shfl_sync(0xffffffffu, mask, q * SEG);
+      const unsigned long long Dq = (unsigned long long)__shfl_sync(0xffffffffu, (long long)D, q * SEG);
+      if ((mq >> lane) & 1ull) { atomicAdd(&sn[lane], 1ull); atomicAdd(&se[lane], Dq); }
+      if ((mq >> (lane + 32)) & 1ull) { atomicAdd(&sn[lane + 32], 1ull); atomicAdd(&se[lane + 32], Dq); }
     }
+    if (slot < n_act && (lane % SEG) == 0 && atomicOr(&m_out[v], mask) == 0ull)
+      act_out[atomicAdd(n_out, 1)] = (int32_t)v;
+    sample_warp_rows<SEG>(w, n_act, DstRows{act}, grow, gcol, f, hop, seed, [&](int64_t s_, int32_t, int32_t u) {
+      const unsigned long long ms = m_in[act[s_]];
+      if (atomicOr(&m_out[u], ms) == 0ull) act_out[atomicAdd(n_out, 1)] = u;
+    });
   }
   __syncthreads();
   if (threadIdx.x < 64) {
@@ -580,9 +607,20 @@ buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, con
   for (int l = L; l >= 1; --l) {
     BF_CUDA(cudaMemsetAsync(cnt, 0, sizeof(int32_t), s));
     if (n_act > 0) {
-      k_mask_layer<<<grid_for(n_act * 32, 256, 16), 256, 0, s>>>(
-          act[cur], n_act, m[cur], m[cur ^ 1], act[cur ^ 1], cnt, g->row_ptr, g->col, sp->fanout[l - 1],
-          (uint32_t)(L - l + 1), sp->seed, accn + 64 * l, acce + 64 * (l - 1));
+      const int32_t fl = sp->fanout[l - 1];
+      const int seg = sample_seg(fl);
+      const int grid = grid_for(ceil_div(n_act, 32 / seg) * 32, 256, 16);
+      if (seg == 8)
+        k_mask_layer<8><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], act[cur ^ 1], cnt, g->row_ptr, g->col,
+                                            fl, (uint32_t)(L - l + 1), sp->seed, accn + 64 * l, acce + 64 * (l - 1));
+      else if (seg == 16)
+        k_mask_layer<16><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], act[cur ^ 1], cnt, g->row_ptr,
+                                             g->col, fl, (uint32_t)(L - l + 1), sp->seed, accn + 64 * l,
+                                             acce + 64 * (l - 1));
+      else
+        k_mask_layer<32><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], act[cur ^ 1], cnt, g->row_ptr,
+                                             g->col, fl, (uint32_t)(L - l + 1), sp->seed, accn + 64 * l,
+                                             acce + 64 * (l - 1));
       BF_LAUNCHED("k_mask_layer");
       // masks of layer l are no longer needed: clear them for reuse by layer l-2
       k_mask_count<<<grid_for(n_act, 256), 256, 0, s>>>(act[cur], n_act, m[cur], nullptr, 1);
