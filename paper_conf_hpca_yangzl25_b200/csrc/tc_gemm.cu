@@ -92,6 +92,43 @@ __device__ __forceinline__ void ld32(uint32_t taddr, float* v) {
 #pragma unroll
   for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
+// Split issue / wait so the next TMEM load overlaps the current group's epilogue math; the
+// wait names the destination registers so no use of them can be scheduled above it.
+__device__ __forceinline__ void ld32_issue(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+      "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+        "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+        "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void ld32_wait(uint32_t (&r)[32]) {
+  asm volatile("tcgen05.wait::ld.sync.aligned;"
+               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]), "+r"(r[7]),
+                 "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]), "+r"(r[14]),
+                 "+r"(r[15]), "+r"(r[16]), "+r"(r[17]), "+r"(r[18]), "+r"(r[19]), "+r"(r[20]), "+r"(r[21]),
+                 "+r"(r[22]), "+r"(r[23]), "+r"(r[24]), "+r"(r[25]), "+r"(r[26]), "+r"(r[27]), "+r"(r[28]),
+                 "+r"(r[29]), "+r"(r[30]), "+r"(r[31])
+               :
+               : "memory");
+}
+// Column sums of a warp's 32 x 32 register tile in 31 shuffles: each step halves the columns a
+// lane keeps and adds its partner's copy; afterwards v[0] of lane k holds the sum of column k.
+__device__ __forceinline__ float warp_colsum32(float (&v)[32], int lane) {
+#pragma unroll
+  for (int o = 16; o >= 1; o >>= 1) {
+    const bool up = (lane & o) != 0;
+#pragma unroll
+    for (int j = 0; j < o; ++j) {
+      const float send = up ? v[j] : v[j + o];
+      const float keep = up ? v[j + o] : v[j];
+      v[j] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+    }
+  }
+  return v[0];
+}
 __device__ __forceinline__ uint32_t pk(float a, float b) {
   __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
   return *reinterpret_cast<uint32_t*>(&h);
@@ -99,11 +136,12 @@ __device__ __forceinline__ uint32_t pk(float a, float b) {
 
 constexpr int kTM = 128;
 constexpr int kChunkA = kTM * 128;     // 16 KB: 128 rows x 64 bf16
-constexpr int kEpiWarps = 4;
+constexpr int kEpiWarps = 8;       // two per TMEM lane quadrant (column groups interleaved)
 constexpr int kGemmThreads = (kEpiWarps + 2) * 32;
 
 struct GemmParams {
   int64_t n_rows;
+  int64_t self_tiles;         // tiles t >= self_tiles have no self rows: their self K-chunks are skipped
   const int32_t* self_idx;    // null: self rows are rows of the self map; else row i = self_idx[i] (gather4)
   int32_t self_oob;           // an out-of-bounds row index of the self map (zero rows)
   int nkc_self, nkc;          // K-chunks of the self half, total
@@ -120,6 +158,7 @@ struct GemmParams {
   float* db_part;                        // [gridDim.x][d_out]
 };
 
+template <bool kBwd>
 __global__ void __launch_bounds__(kGemmThreads, 1)
     k_tc_gemm_tma(const __grid_constant__ CUtensorMap self_map, const __grid_constant__ CUtensorMap agg_map,
                   const GemmParams p) {
@@ -170,7 +209,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
           idx[k] = r < p.n_rows ? __ldg(p.self_idx + r) : p.self_oob;
         }
       }
-      for (int c = 0; c < p.nkc; ++c, ++g) {
+      const int cb = t >= p.self_tiles ? p.nkc_self : 0;
+      for (int c = cb; c < p.nkc; ++c, ++g) {
         const int st = (int)(g % NS);
         if (lane == 0) {
           if (g >= NS) mb_wait(&empty[st], (uint32_t)(((g / NS) - 1) & 1));
@@ -198,141 +238,175 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         if (i >= 2) mb_wait(&acc_empty[acc], (uint32_t)(((i >> 1) - 1) & 1));
         fence_after();
         const uint32_t d = tmem + acc * p.Np;
-        for (int c = 0; c < p.nkc; ++c, ++g) {
+        const int cb = t >= p.self_tiles ? p.nkc_self : 0;
+        for (int c = cb; c < p.nkc; ++c, ++g) {
           const int st = (int)(g % NS);
           mb_wait(&full[st], (uint32_t)((g / NS) & 1));
           fence_after();
           const uint32_t a = su32(sA + st * kChunkA), b = su32(sB + st * bbytes);
 #pragma unroll
           for (int k = 0; k < 4; ++k)
-            mma_f16(d, desc_sw128(a + 32 * k), desc_sw128(b + 32 * k), idesc, (c > 0 || k > 0) ? 1u : 0u);
+            mma_f16(d, desc_sw128(a + 32 * k), desc_sw128(b + 32 * k), idesc, (c > cb || k > 0) ? 1u : 0u);
           commit(&empty[st]);
         }
         commit(&acc_full[acc]);
       }
     }
     __syncwarp();
-  } else if (p.epi) {
-    // ---------------- backward epilogue: dZ = acc * 1[H > 0] -> bf16 dZ, bf16 dZ/D, and
-    // per-warp column sums (fixed row order), combined per CTA at the end
-    float dbacc[8];
+  } else {
+    // ---------------- epilogue: warp e owns TMEM lane quadrant q = e & 3 (tile rows 32q..32q+31)
+    // and the 32-column groups g = 2j + h (h = e >> 2).  Forward: +bias, ReLU, store.  Backward
+    // (kBwd): dZ = acc * 1[H > 0] -> bf16 dZ, bf16 dZ/D, and per-warp column sums (fixed row
+    // order) combined per CTA at the end.  H of the next tile is prefetched into registers while
+    // the current one is processed; the next TMEM load is issued before the current group's math.
+    const int q = warp & 3, h = warp >> 2;
+    float* sbias = reinterpret_cast<float*>(tmem_slot + 4);   // 16-B aligned
+    for (int c = threadIdx.x; c < p.Np; c += kEpiWarps * 32)
+      sbias[c] = (p.bias && c < p.d_out) ? __ldg(p.bias + c) : 0.f;
+    asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
+    const int ng = (p.pitch_out + 31) / 32;
+    const int nj = (ng - h + 1) / 2;              // groups of this warp (<= 4)
+    float dbacc[4] = {0.f, 0.f, 0.f, 0.f};
+    uint4 hreg[4][4];
 #pragma unroll
-    for (int g = 0; g < 8; ++g) dbacc[g] = 0.f;
+    for (int j = 0; j < 4; ++j)
+#pragma unroll
+      for (int k = 0; k < 4; ++k) hreg[j][k] = make_uint4(0u, 0u, 0u, 0u);
+    if (kBwd) {
+      const int64_t row = (int64_t)blockIdx.x * kTM + q * 32 + lane;
+      if (row < p.n_rows) {
+        const __nv_bfloat16* hr = p.H + row * p.ldH;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int c0 = (2 * j + h) * 32;
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            if (j < nj && c0 + 8 * k < p.pitch_out) hreg[j][k] = __ldg(reinterpret_cast<const uint4*>(hr + c0 + 8 * k));
+        }
+      }
+    }
     int64_t i = 0;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
       const int acc = (int)(i & 1);
       mb_wait(&acc_full[acc], (uint32_t)((i >> 1) & 1));
       fence_after();
-      const int64_t row = t * kTM + warp * 32 + lane;
+      const int64_t row = t * kTM + q * 32 + lane;
       const bool rok = row < p.n_rows;
+      const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + acc * p.Np;
       float invd = 1.f;
-      if (rok && p.zs) {
+      if (kBwd && rok && p.zs) {
         const int32_t d = __ldg(p.rp + row + 1) - __ldg(p.rp + row);
         invd = d > 0 ? 1.f / (float)d : 0.f;
       }
+      uint32_t r[2][32];
+      if (nj > 0) {
+        ld32_issue(tbase + h * 32, r[0]);
+        ld32_wait(r[0]);
+      }
 #pragma unroll
-      for (int g = 0; g < 8; ++g) {
-        const int c0 = g * 32;
-        if (c0 >= p.pitch_out) break;
-        float v[32];
-        ld32(tmem + ((uint32_t)(warp * 32) << 16) + acc * p.Np + c0, v);
-        const int ncols = min(32, p.pitch_out - c0);
-        if (rok) {
-          const __nv_bfloat16* hr = p.H + row * p.ldH + c0;
+      for (int j = 0; j < 4; ++j) {
+        if (j < nj) {
+          const int c0 = (2 * j + h) * 32;
+          if (kBwd && j > 0) {                          // backward: registers go to the H prefetch
+            ld32_issue(tbase + c0, r[j & 1]);
+            ld32_wait(r[j & 1]);
+          }
+          if (!kBwd && j + 1 < nj) ld32_issue(tbase + c0 + 64, r[(j + 1) & 1]);
+          const int ncols = min(32, p.pitch_out - c0);   // multiple of 8
+          float v[32];
 #pragma unroll
-          for (int k = 0; k < 32; k += 8) {
-            if (k < ncols) {
-              const uint4 hu = __ldg(reinterpret_cast<const uint4*>(hr + k));
-              const uint32_t hw[4] = {hu.x, hu.y, hu.z, hu.w};
+          for (int k = 0; k < 32; ++k) v[k] = __uint_as_float(r[j & 1][k]);
+          if (kBwd) {
+            if (rok) {
 #pragma unroll
-              for (int q = 0; q < 4; ++q) {
-                const float h0 = __uint_as_float(hw[q] << 16), h1 = __uint_as_float(hw[q] & 0xffff0000u);
-                if (!(h0 > 0.f) || c0 + k + 2 * q >= p.d_out) v[k + 2 * q] = 0.f;
-                if (!(h1 > 0.f) || c0 + k + 2 * q + 1 >= p.d_out) v[k + 2 * q + 1] = 0.f;
+              for (int k = 0; k < 32; k += 8) {
+                if (k < ncols) {
+                  const uint32_t hw[4] = {hreg[j][k / 8].x, hreg[j][k / 8].y, hreg[j][k / 8].z, hreg[j][k / 8].w};
+#pragma unroll
+                  for (int e = 0; e < 4; ++e) {
+                    const float h0 = __uint_as_float(hw[e] << 16), h1 = __uint_as_float(hw[e] & 0xffff0000u);
+                    if (!(h0 > 0.f) || c0 + k + 2 * e >= p.d_out) v[k + 2 * e] = 0.f;
+                    if (!(h1 > 0.f) || c0 + k + 2 * e + 1 >= p.d_out) v[k + 2 * e + 1] = 0.f;
+                  }
+                } else {
+#pragma unroll
+                  for (int e = 0; e < 8; ++e) v[k + e] = 0.f;
+                }
+              }
+              __nv_bfloat16* zo = p.zb + row * p.pitch_out + c0;
+#pragma unroll
+              for (int k = 0; k < 32; k += 8)
+                if (k < ncols)
+                  *reinterpret_cast<uint4*>(zo + k) = make_uint4(pk(v[k], v[k + 1]), pk(v[k + 2], v[k + 3]),
+                                                                 pk(v[k + 4], v[k + 5]), pk(v[k + 6], v[k + 7]));
+              if (p.zs) {
+                __nv_bfloat16* so = p.zs + row * p.pitch_out + c0;
+#pragma unroll
+                for (int k = 0; k < 32; k += 8)
+                  if (k < ncols)
+                    *reinterpret_cast<uint4*>(so + k) =
+                        make_uint4(pk(v[k] * invd, v[k + 1] * invd), pk(v[k + 2] * invd, v[k + 3] * invd),
+                                   pk(v[k + 4] * invd, v[k + 5] * invd), pk(v[k + 6] * invd, v[k + 7] * invd));
               }
             } else {
 #pragma unroll
-              for (int q = 0; q < 8; ++q) v[k + q] = 0.f;
+              for (int k = 0; k < 32; ++k) v[k] = 0.f;
+            }
+            // prefetch this group's H of the next tile (its registers are free now)
+            {
+              const int64_t tn = t + gridDim.x;
+              const int64_t rn = tn * kTM + q * 32 + lane;
+              if (tn < ntiles && rn < p.n_rows) {
+                const __nv_bfloat16* hr = p.H + rn * p.ldH + c0;
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+                  if (8 * k < ncols) hreg[j][k] = __ldg(reinterpret_cast<const uint4*>(hr + 8 * k));
+              }
+            }
+            dbacc[j] += warp_colsum32(v, lane);
+          } else if (rok) {
+#pragma unroll
+            for (int k = 0; k < 32; k += 4) {
+              const float4 bb = *reinterpret_cast<const float4*>(sbias + c0 + k);
+              v[k] += bb.x; v[k + 1] += bb.y; v[k + 2] += bb.z; v[k + 3] += bb.w;
+            }
+            if (p.relu) {
+#pragma unroll
+              for (int k = 0; k < 32; ++k) v[k] = fmaxf(v[k], 0.f);
+            }
+            if (p.out_f32) {
+              float* o = (float*)p.out + row * p.ld_out + c0;
+#pragma unroll
+              for (int k = 0; k < 32; k += 4)
+                if (k < ncols) *reinterpret_cast<float4*>(o + k) = make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]);
+            } else {
+              __nv_bfloat16* o = (__nv_bfloat16*)p.out + row * p.ld_out + c0;
+#pragma unroll
+              for (int k = 0; k < 32; k += 8)
+                if (k < ncols)
+                  *reinterpret_cast<uint4*>(o + k) = make_uint4(pk(v[k], v[k + 1]), pk(v[k + 2], v[k + 3]),
+                                                                pk(v[k + 4], v[k + 5]), pk(v[k + 6], v[k + 7]));
             }
           }
-          __nv_bfloat16* zo = p.zb + row * p.pitch_out + c0;
-#pragma unroll
-          for (int k = 0; k < 32; k += 8)
-            if (k < ncols)
-              *reinterpret_cast<uint4*>(zo + k) =
-                  make_uint4(pk(v[k], v[k + 1]), pk(v[k + 2], v[k + 3]), pk(v[k + 4], v[k + 5]), pk(v[k + 6], v[k + 7]));
-          if (p.zs) {
-            __nv_bfloat16* so = p.zs + row * p.pitch_out + c0;
-#pragma unroll
-            for (int k = 0; k < 32; k += 8)
-              if (k < ncols)
-                *reinterpret_cast<uint4*>(so + k) =
-                    make_uint4(pk(v[k] * invd, v[k + 1] * invd), pk(v[k + 2] * invd, v[k + 3] * invd),
-                               pk(v[k + 4] * invd, v[k + 5] * invd), pk(v[k + 6] * invd, v[k + 7] * invd));
-          }
-        } else {
-#pragma unroll
-          for (int k = 0; k < 32; ++k) v[k] = 0.f;
-        }
-        // column sums over the warp's 32 rows; lane k keeps column c0 + k
-#pragma unroll
-        for (int k = 0; k < 32; ++k) {
-          float x = v[k];
-#pragma unroll
-          for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
-          if (lane == k) dbacc[g] += x;
+          if (!kBwd && j + 1 < nj) ld32_wait(r[(j + 1) & 1]);
         }
       }
       fence_before();
       mb_arrive(&acc_empty[acc]);
     }
-    // combine the four warps in order -> one partial per CTA
-    float* red = reinterpret_cast<float*>(sA);     // stage 0 A buffer: the producer is done
-    asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
+    if (kBwd) {
+      // combine the four lane quadrants in order -> one partial per CTA
+      float* red = reinterpret_cast<float*>(sA);     // stage 0 A buffer: every MMA has completed
+      asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
 #pragma unroll
-    for (int g = 0; g < 8; ++g) red[warp * 256 + g * 32 + lane] = dbacc[g];
-    asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
-    for (int c = threadIdx.x; c < p.d_out; c += kEpiWarps * 32) {
-      float t = 0.f;
-      for (int w = 0; w < kEpiWarps; ++w) t += red[w * 256 + c];
-      p.db_part[(int64_t)blockIdx.x * p.d_out + c] = t;
-    }
-  } else {
-    // ---------------- epilogue: warp w owns TMEM lanes (tile rows) 32w .. 32w + 31
-    int64_t i = 0;
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
-      const int acc = (int)(i & 1);
-      mb_wait(&acc_full[acc], (uint32_t)((i >> 1) & 1));
-      fence_after();
-      const int64_t row = t * kTM + warp * 32 + lane;
-      for (int c0 = 0; c0 < p.pitch_out; c0 += 32) {
-        float v[32];
-        ld32(tmem + ((uint32_t)(warp * 32) << 16) + acc * p.Np + c0, v);
-        if (row < p.n_rows) {
-#pragma unroll
-          for (int k = 0; k < 32; ++k) {
-            const int cidx = c0 + k;
-            float x = v[k] + ((p.bias && cidx < p.d_out) ? __ldg(p.bias + cidx) : 0.f);
-            v[k] = p.relu ? fmaxf(x, 0.f) : x;
-          }
-          const int ncols = min(32, p.pitch_out - c0);   // multiple of 8
-          if (p.out_f32) {
-            float* o = (float*)p.out + row * p.ld_out + c0;
-#pragma unroll
-            for (int k = 0; k < 32; k += 4)
-              if (k < ncols) *reinterpret_cast<float4*>(o + k) = make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]);
-          } else {
-            __nv_bfloat16* o = (__nv_bfloat16*)p.out + row * p.ld_out + c0;
-#pragma unroll
-            for (int k = 0; k < 32; k += 8)
-              if (k < ncols)
-                *reinterpret_cast<uint4*>(o + k) =
-                    make_uint4(pk(v[k], v[k + 1]), pk(v[k + 2], v[k + 3]), pk(v[k + 4], v[k + 5]), pk(v[k + 6], v[k + 7]));
-          }
-        }
+      for (int j = 0; j < 4; ++j)
+        if (j < nj) red[q * 256 + (2 * j + h) * 32 + lane] = dbacc[j];
+      asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
+      for (int c = threadIdx.x; c < p.d_out; c += kEpiWarps * 32) {
+        float tsum = 0.f;
+        for (int w = 0; w < 4; ++w) tsum += red[w * 256 + c];
+        p.db_part[(int64_t)blockIdx.x * p.d_out + c] = tsum;
       }
-      fence_before();
-      mb_arrive(&acc_empty[acc]);
     }
   }
   fence_before();
@@ -573,6 +647,7 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   BF_CHECK(encode_map(&am, agg, pin, n_rows, ld_agg));
   GemmParams p{};
   p.n_rows = n_rows;
+  p.self_tiles = self_idx ? ceil_div(n_rows, kTM) : ceil_div(self_rows, kTM);
   p.self_idx = self_idx;
   p.self_oob = self_idx ? 0 : (int32_t)self_rows;
   p.nkc_self = (int)ceil_div(d_in, 64);
@@ -596,14 +671,16 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   }
   const int stage = kChunkA + p.Np * 128;
   p.nstages = std::max(2, std::min(8, (200 * 1024) / stage));
-  const int smem = p.nstages * stage + 16 * p.nstages + 64 + 1024;
+  const int smem = p.nstages * stage + 16 * p.nstages + 48 + 4 * p.Np + 1024;
   static bool attr = false;
   if (!attr) {
-    BF_CUDA(cudaFuncSetAttribute(k_tc_gemm_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    BF_CUDA(cudaFuncSetAttribute(k_tc_gemm_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    BF_CUDA(cudaFuncSetAttribute(k_tc_gemm_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
     attr = true;
   }
   const int grid = (int)gemm_grid(n_rows);
-  k_tc_gemm_tma<<<grid, kGemmThreads, smem, s>>>(sm, am, p);
+  if (epi) k_tc_gemm_tma<true><<<grid, kGemmThreads, smem, s>>>(sm, am, p);
+  else k_tc_gemm_tma<false><<<grid, kGemmThreads, smem, s>>>(sm, am, p);
   BF_LAUNCHED("k_tc_gemm_tma");
   return BUFFALO_OK;
 }

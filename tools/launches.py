@@ -13,7 +13,8 @@ def summarise(path, top=30):
     for r in rows[hi + 1:]:
         if len(r) <= vi:
             continue
-        name = r[ki].split("(")[0].split("<")[0].replace("void ", "")
+        name = r[ki].replace("<unnamed>::", "").replace("(anonymous namespace)::", "")
+        name = name.split("(")[0].split("<")[0].replace("void ", "")
         try:
             v = float(r[vi].replace(",", ""))
         except ValueError:
