@@ -97,6 +97,8 @@ typedef struct {
   int64_t* est_bytes_h;     /* Eq. 2 estimate per group                       */
   int32_t* rank_of_group_h; /* LPT assignment of groups to num_gpus ranks (R24)              */
   int64_t* hist_h;          /* degree-bucket histogram of the seeds, [cutoff_F + 1]           */
+  int64_t* group_sizes_h;   /* nullable host [k_max][2L+1]: exact block sizes of each group,
+                               n_0..n_L then e_1..e_L (one extra statistics pass over the groups) */
   int32_t k_out;            /* number of non-empty groups                                     */
   int32_t k_tried;          /* the K at which Alg. 4 succeeded                               */
   int32_t exploded;         /* 1 if the degree-F bucket was split (R7)                       */
@@ -109,9 +111,10 @@ typedef struct {
  * col_global (block 1 only, else NULL) int32[n_edges], t_row_ptr/t_col: transposed block
  * (block >= 2 only, else NULL): for each src j the dst i with an edge to j, ascending.
  * cls_perm int32[n_dst]: the dst sorted by degree class min(D, 129), stable (degree bucketing of
- * the block, Alg. 2 l.6 PAPER.md:238); heavy = cls_perm + n_dst - n_heavy lists the dst with
- * D > 128 (long-tail cooperative path), ascending.  t_perm int32[n_src] (block >= 2 only): the src
- * sorted by transposed degree class; its last n_heavy_t entries have more than 128 dst.
+ * the block, Alg. 2 l.6 PAPER.md:238); its tail lists the dst with D > 128 (long-tail cooperative
+ * path): heavy = cls_perm + n_dst - n_heavy when the build read the sizes back, else n_heavy = -1
+ * and heavy = NULL.  t_perm int32[n_src] (block >= 2 only): the src sorted by transposed degree
+ * class; its tail holds those with more than 128 dst (n_heavy_t of them, or -1 if not counted).
  * Activations of the standard arena layout: agg (saved h_agg [n_dst][ld_agg]), out (H_l
  * [n_dst][ld_out], act dtype, or logits fp32 at l = L), dh (dH_l / dlogits fp32 [n_dst][ld_dh],
  * valid during the backward of layers l and l+1), bwd_scratch (bwd_scratch_bytes). */
@@ -158,12 +161,19 @@ BUFFALO_API buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32
 /* MicroBatchGenerator / BlockGenerate (Alg. 2 l.5 PAPER.md:237, §IV-E): the L
  * blocks of the micro-batch whose output nodes are group_seeds[0..n), built top-down, plus the
  * activation and backward buffers of the standard arena layout.  arena: device,
- * 256-B aligned.  Synchronises twice per layer.  BUFFALO_ERR_CAPACITY: *required_bytes_h gets a
- * lower bound of the bytes needed (the exact need once all sizes are known). */
+ * 256-B aligned.
+ * sizes_h (nullable, host [2L+1]): the group's row of plan.group_sizes_h, i.e. the exact sizes
+ *   n_0..n_L, e_1..e_L for this group and sampler.  Given, the arena need is checked up front
+ *   (BUFFALO_ERR_CAPACITY with *required_bytes_h = the exact need) and the build runs without
+ *   any host synchronisation; n_heavy / n_heavy_t / heavy are then left at -1 / NULL (kernels
+ *   find the long rows at the tail of cls_perm / t_perm).  Sizes that do not match the group
+ *   give undefined block contents (writes stay inside the arena).
+ *   NULL: the sizes are read back while building (two to three synchronisations per layer);
+ *   BUFFALO_ERR_CAPACITY then reports a lower bound of the need in *required_bytes_h. */
 BUFFALO_API buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group_seeds, int64_t n,
                                     const buffalo_sampler* s, const buffalo_model* m,
                                     buffalo_blocks* out, void* arena, size_t arena_bytes,
-                                    int64_t* required_bytes_h, void* stream);
+                                    int64_t* required_bytes_h, const int64_t* sizes_h, void* stream);
 
 /* ------------------------------------------------------------------ a7: forward */
 /* Packed copy of W_l [dim[l], 2*dim[l-1]] fp32 for the kernels (transposes / padded bf16). */

@@ -7,6 +7,7 @@ there is no CPU fallback: loading fails loudly without the built library or a GP
 import ctypes
 import os
 
+import numpy as np
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -60,7 +61,7 @@ class Sched(ctypes.Structure):
 class Plan(ctypes.Structure):
     _fields_ = [("group_of_seed", c_p), ("group_seeds", c_p), ("group_offsets", c_p),
                 ("group_offsets_h", c_p), ("est_bytes_h", c_p), ("rank_of_group_h", c_p),
-                ("hist_h", c_p), ("k_out", c_i32), ("k_tried", c_i32), ("exploded", c_i32),
+                ("hist_h", c_p), ("group_sizes_h", c_p), ("k_out", c_i32), ("k_tried", c_i32), ("exploded", c_i32),
                 ("num_items", c_i32)]
 
 
@@ -94,7 +95,7 @@ def lib(require_gpu=True):
             "buffalo_graph_prepare": (c_i32, [P, P, c_sz, P]),
             "buffalo_bucketize_workspace_bytes": (c_sz, [P, c_i64, P, P]),
             "buffalo_bucketize": (c_i32, [P, P, c_i64, P, P, P, P, P, c_sz, P]),
-            "buffalo_build_blocks": (c_i32, [P, P, c_i64, P, P, P, P, c_sz, P, P]),
+            "buffalo_build_blocks": (c_i32, [P, P, c_i64, P, P, P, P, c_sz, P, P, P]),
             "buffalo_packed_weight_bytes": (c_sz, [P, c_i32]),
             "buffalo_pack_weights": (c_i32, [P, c_i32, P, P, P]),
             "buffalo_sage_fwd": (c_i32, [P, c_i32, P, P, c_i64, P, P, P, P, c_i64, P, c_i64, P]),
@@ -160,11 +161,16 @@ def bucketize(graph, seeds, sampler, model, sched, plan, workspace, stream=None)
                                    stream_ptr(stream)))
 
 
-def build_blocks(graph, group_seeds, n, sampler, model, blocks, arena, stream=None):
-    """Returns BUFFALO_OK or raises; on BUFFALO_ERR_CAPACITY the error carries .required."""
+def build_blocks(graph, group_seeds, n, sampler, model, blocks, arena, sizes=None, stream=None):
+    """Returns BUFFALO_OK or raises; on BUFFALO_ERR_CAPACITY the error carries .required.
+    sizes: None or a C-contiguous int64 numpy row [2L+1] of plan.group_sizes_h (sync-free build)."""
     req = c_i64(0)
+    sz = None
+    if sizes is not None:
+        assert sizes.dtype == np.int64 and sizes.flags["C_CONTIGUOUS"]
+        sz = sizes.ctypes.data
     st = lib().buffalo_build_blocks(ref(graph), ptr(group_seeds), n, ref(sampler), ref(model),
-                                    ref(blocks), ptr(arena), arena.numel(), ctypes.byref(req),
+                                    ref(blocks), ptr(arena), arena.numel(), ctypes.byref(req), sz,
                                     stream_ptr(stream))
     if st == ERR_CAPACITY:
         err = BuffaloError(st, lib(False).buffalo_last_error().decode())

@@ -444,6 +444,27 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
       rload[best] += est[k];
     }
     for (int k = 0; k < gk; ++k) plan->est_bytes_h[k] = est[k];
+    if (plan->group_sizes_h) {
+      // exact block sizes of every group (groups as items of the mask statistics), so that
+      // buffalo_build_blocks can lay out the arena up front and run without host round trips
+      const int W = 2 * L + 1;
+      for (int k0 = 0; k0 < gk; k0 += 64) {
+        const int nit = std::min(64, gk - k0);
+        int64_t st[64], ct[64];
+        for (int k = 0; k < nit; ++k) {
+          st[k] = offs[k0 + k];
+          ct[k] = offs[k0 + k + 1] - offs[k0 + k];
+        }
+        static thread_local int64_t nh[64][BUFFALO_MAX_LAYERS + 1], eh[64][BUFFALO_MAX_LAYERS];
+        BF_CHECK(mask_stats(g, plan->group_seeds, st, ct, nit, sp, L, stats_ws, stats_bytes, masks_clean, nh, eh, s));
+        masks_clean = true;
+        for (int k = 0; k < nit; ++k) {
+          int64_t* row = plan->group_sizes_h + (int64_t)(k0 + k) * W;
+          for (int l = 0; l <= L; ++l) row[l] = nh[k][l];
+          for (int l = 1; l <= L; ++l) row[L + l] = eh[k][l - 1];
+        }
+      }
+    }
     plan->k_out = gk;
     plan->k_tried = K;
     plan->exploded = exploded ? 1 : 0;
@@ -459,7 +480,7 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
 buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group_seeds, int64_t n,
                                     const buffalo_sampler* sp, const buffalo_model* m,
                                     buffalo_blocks* out, void* arena, size_t arena_bytes,
-                                    int64_t* required_bytes_h, void* stream) {
+                                    int64_t* required_bytes_h, const int64_t* sizes_h, void* stream) {
   BF_CHECK(require_sm100());
   BF_CHECK(validate_model(m));
   const int L = m->num_layers;
@@ -473,6 +494,25 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
     return BUFFALO_ERR_INVALID_ARG;
   }
   cudaStream_t s = (cudaStream_t)stream;
+  if (sizes_h) {
+    // sizes from the plan: validate, then check the whole arena need (R15: lo = exact) up front
+    if (sizes_h[L] != n) {
+      set_error("build_blocks: sizes_h[L] = %lld != n = %lld", (long long)sizes_h[L], (long long)n);
+      return BUFFALO_ERR_INVALID_ARG;
+    }
+    for (int l = 0; l <= 2 * L; ++l)
+      if (sizes_h[l] < 0 || sizes_h[l] > INT32_MAX) {
+        set_error("build_blocks: bad sizes_h");
+        return BUFFALO_ERR_INVALID_ARG;
+      }
+    int64_t lo, hi;
+    mem_model(L, sizes_h, sizes_h + L + 1, m, &lo, &hi);
+    if (lo > (int64_t)arena_bytes) {
+      if (required_bytes_h) *required_bytes_h = lo;
+      set_error("build_blocks: arena of %lld bytes too small (need %lld)", (long long)arena_bytes, (long long)lo);
+      return BUFFALO_ERR_CAPACITY;
+    }
+  }
   memset(out, 0, sizeof(*out));
   out->num_layers = L;
   Arena A;
@@ -483,8 +523,13 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
   int64_t nn[BUFFALO_MAX_LAYERS + 1], ee[BUFFALO_MAX_LAYERS];
   for (int l = L; l >= 1; --l) {
     buffalo_block* b = &out->layer[l - 1];
+    int64_t known[2];
+    if (sizes_h) {
+      known[0] = sizes_h[L + l];      // e_l
+      known[1] = sizes_h[l - 1];      // n_{l-1}
+    }
     buffalo_status st = build_layer(g, dst, nd, sp->fanout[l - 1], (uint32_t)(L - l + 1), sp->seed, l,
-                                    false, A, b, s);
+                                    false, A, b, s, sizes_h ? known : nullptr);
     if (st == BUFFALO_ERR_CAPACITY || A.overflow) {
       if (required_bytes_h) *required_bytes_h = A.need;
       set_error("build_blocks: arena of %lld bytes too small (need >= %lld)", (long long)A.cap,

@@ -5,6 +5,9 @@
 // in parallel at the node level"): count -> scan -> sample/slice -> relabel into
 // a bipartite block (dst prefix + first occurrence, R3/R4) -> transpose for the backward.
 #include "build.cuh"
+
+#include <cooperative_groups.h>
+namespace cg = cooperative_groups;
 #include "philox.cuh"
 #include "primitives.cuh"
 
@@ -76,12 +79,14 @@ __global__ void __launch_bounds__(256) k_sample_fill(const int32_t* __restrict__
                                                      const int32_t* __restrict__ gcol, int32_t f,
                                                      uint32_t hop, uint64_t seed,
                                                      const int32_t* __restrict__ row_ptr,
-                                                     int32_t* __restrict__ out) {
+                                                     int32_t* __restrict__ out, int64_t cap) {
   constexpr int G = 32 / SEG;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
   for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n; w += warps)
-    sample_warp_rows<SEG>(w, n, DstRows{dst}, grow, gcol, f, hop, seed,
-                          [&](int64_t slot, int32_t k, int32_t u) { out[row_ptr[slot] + k] = u; });
+    sample_warp_rows<SEG>(w, n, DstRows{dst}, grow, gcol, f, hop, seed, [&](int64_t slot, int32_t k, int32_t u) {
+      const int64_t pos = (int64_t)row_ptr[slot] + k;
+      if (pos < cap) out[pos] = u;
+    });
 }
 
 static inline int sample_seg(int32_t f) { return (f > 0 && f <= 8) ? 8 : (f > 0 && f <= 16) ? 16 : 32; }
@@ -122,8 +127,9 @@ struct FirstFlag {
 struct EmitSrc {
   Cand c;
   int32_t* src;
+  int64_t cap;
   __device__ __forceinline__ void operator()(int64_t p, int32_t excl, int32_t v) const {
-    if (v) src[excl] = c(p);
+    if (v && excl < cap) src[excl] = c(p);
   }
 };
 
@@ -189,7 +195,7 @@ __global__ void __launch_bounds__(256) k_tsort_small(const int32_t* __restrict__
   for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < n; w += warps) {
     const int32_t j = rows[w];
     const int32_t b = trp[j], len = trp[j + 1] - b;
-    if (len <= 1) continue;
+    if (len <= 1 || len > kHeavyT) continue;                // heavy rows: k_tsort_heavy
     int32_t v[4];
     int rank[4] = {0, 0, 0, 0};
 #pragma unroll
@@ -207,10 +213,13 @@ __global__ void __launch_bounds__(256) k_tsort_small(const int32_t* __restrict__
 }
 // Long transposed rows (> 128 entries): CTA per row; the row is staged in `stage` (same
 // offsets as t_col), then every entry is written at its rank among the staged values.
-__global__ void __launch_bounds__(256) k_tsort_heavy(const int32_t* __restrict__ rows, const int32_t* __restrict__ trp,
+__global__ void __launch_bounds__(256) k_tsort_heavy(const int32_t* __restrict__ perm, int64_t n,
+                                                     const int32_t* __restrict__ trp,
                                                      int32_t* __restrict__ tcol, int32_t* __restrict__ stage) {
-  const int32_t j = rows[blockIdx.x];
+  for (int64_t hh = blockIdx.x; hh < n; hh += gridDim.x) {
+  const int32_t j = perm[n - 1 - hh];          // heavy rows: the tail of the degree-class perm
   const int32_t b = trp[j], len = trp[j + 1] - b;
+  if (len <= kHeavyT) break;
   for (int32_t k = threadIdx.x; k < len; k += blockDim.x) stage[b + k] = tcol[b + k];
   __syncthreads();
   for (int32_t k = threadIdx.x; k < len; k += blockDim.x) {
@@ -218,6 +227,8 @@ __global__ void __launch_bounds__(256) k_tsort_heavy(const int32_t* __restrict__
     int32_t r = 0;
     for (int32_t t = 0; t < len; ++t) r += stage[b + t] < x ? 1 : 0;
     tcol[b + r] = x;
+  }
+  __syncthreads();
   }
 }
 // ed[e] = dst index of edge e (warp per dst row).
@@ -265,7 +276,7 @@ int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only) 
 
 buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
                            uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
-                           buffalo_block* blk, cudaStream_t s) {
+                           buffalo_block* blk, cudaStream_t s, const int64_t* known) {
   memset(blk, 0, sizeof(*blk));
   blk->n_dst = n_dst;
   int32_t* rp = (int32_t*)A.take(4 * (n_dst + 1));
@@ -280,19 +291,25 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     BF_LAUNCHED("k_count");
   }
   BF_CHECK(scan_inplace(rp, n_dst, ws, s));
-  int32_t e32 = 0, nh = 0;
-  if (!sizes_only) {
-    BF_CHECK(device_count(HeavyFlag{rp}, n_dst, totals, s));
-    BF_CHECK(d2h_i32(totals, &nh, s));
+  int64_t e = 0, nh = -1;
+  if (known) {
+    e = known[0];                                                  // exact sizes from the plan: no sync
+  } else {
+    int32_t e32 = 0, nh32 = 0;
+    if (!sizes_only) {
+      BF_CHECK(device_count(HeavyFlag{rp}, n_dst, totals, s));
+      BF_CHECK(d2h_i32(totals, &nh32, s));
+    }
+    BF_CHECK(d2h_i32(rp + n_dst, &e32, s));
+    BF_CUDA(cudaStreamSynchronize(s));                             // sync 1: e_l, n_heavy
+    e = e32;
+    nh = nh32;
   }
-  BF_CHECK(d2h_i32(rp + n_dst, &e32, s));
-  BF_CUDA(cudaStreamSynchronize(s));                               // sync 1: e_l, n_heavy
-  const int64_t e = e32;
   blk->n_edges = e;
   blk->n_heavy = nh;
   blk->row_ptr = rp;
   blk->cls_perm = perm;
-  blk->heavy = perm ? perm + (n_dst - nh) : nullptr;
+  blk->heavy = (perm && nh >= 0) ? perm + (n_dst - nh) : nullptr;
 
   // frame 2
   const int64_t pc = sizes_only ? part_count_elems(e) : part_count_elems(n_dst + e);
@@ -315,7 +332,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   }
   if (n_dst > 0) {
     launch_sample_fill(sample_seg(f), n_dst, s, dst, n_dst, g->row_ptr, g->col, f, hop, seed, (const int32_t*)rp,
-                       colg);
+                       colg, e);
     BF_LAUNCHED("k_sample_fill");
   }
   // relabel: first occurrence over the candidate sequence dst ++ col_global
@@ -326,14 +343,19 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     BF_LAUNCHED("k_relabel_min");
   }
   FirstFlag ff{cand, g->node_map};
-  BF_CHECK(device_count(ff, total, totals, s));
-  int32_t ns32 = 0;
-  BF_CHECK(d2h_i32(totals, &ns32, s));
-  BF_CUDA(cudaStreamSynchronize(s));                               // sync 2: n_{l-1}
-  const int64_t n_src = ns32;
+  int64_t n_src = 0;
+  if (known) {
+    n_src = known[1];
+  } else {
+    BF_CHECK(device_count(ff, total, totals, s));
+    int32_t ns32 = 0;
+    BF_CHECK(d2h_i32(totals, &ns32, s));
+    BF_CUDA(cudaStreamSynchronize(s));                             // sync 2: n_{l-1}
+    n_src = ns32;
+  }
   int32_t* src = (int32_t*)A.take(4 * n_src);
   if (A.overflow) return BUFFALO_ERR_CAPACITY;
-  BF_CHECK(device_scan(ff, EmitSrc{cand, src}, total, ws, totals + 2, s));
+  BF_CHECK(device_scan(ff, EmitSrc{cand, src, n_src}, total, ws, totals + 2, s));
   blk->n_src = n_src;
   blk->src_global = src;
   blk->col_global = colg_persist;
@@ -352,6 +374,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     k_reset_map<<<grid_for(n_src, 256), 256, 0, s>>>(src, n_src, g->node_map);
     BF_LAUNCHED("k_reset_map");
   }
+  blk->n_heavy_t = -1;
   if (!sizes_only && layer >= 2) {
     // transposed block: t_row_ptr by counting; t_col by an atomic-cursor fill followed by an
     // ascending sort of every transposed row (entries are distinct dst indices, so the sorted
@@ -369,23 +392,25 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     }
     BF_CHECK(scan_inplace(trp, n_src, ws, s));
     BF_CHECK(stable_partition(DegClass{trp}, EmitPerm{tperm}, n_src, counts, ws, s));
-    BF_CHECK(device_count(HeavyFlag{trp}, n_src, totals + 1, s));
-    int32_t nht = 0;
-    BF_CHECK(d2h_i32(totals + 1, &nht, s));
+    int64_t nht = -1;
+    if (!known) {
+      BF_CHECK(device_count(HeavyFlag{trp}, n_src, totals + 1, s));
+      int32_t nht32 = 0;
+      BF_CHECK(d2h_i32(totals + 1, &nht32, s));
+      BF_CUDA(cudaStreamSynchronize(s));                           // n_heavy_t (informational)
+      nht = nht32;
+    }
     if (e > 0) {
       BF_CUDA(cudaMemcpyAsync(cursor, trp, sizeof(int32_t) * n_src, cudaMemcpyDeviceToDevice, s));
       k_tfill<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(rp, col_local, n_dst, cursor, tcol);
       BF_LAUNCHED("k_tfill");
-    }
-    BF_CUDA(cudaStreamSynchronize(s));                             // n_heavy_t
-    if (e > 0) {
-      const int64_t n_small = n_src - nht;
-      if (n_small > 0) {
-        k_tsort_small<<<grid_for(n_small * 32, 256, 16), 256, 0, s>>>(tperm, n_small, trp, tcol);
+      if (n_src > 0) {
+        k_tsort_small<<<grid_for(n_src * 32, 256, 16), 256, 0, s>>>(tperm, n_src, trp, tcol);
         BF_LAUNCHED("k_tsort_small");
       }
-      if (nht > 0) {
-        k_tsort_heavy<<<(unsigned)nht, 256, 0, s>>>(tperm + n_small, trp, tcol, cursor);
+      const int hg = heavy_tail_grid(nht, e);
+      if (hg > 0) {
+        k_tsort_heavy<<<hg, 256, 0, s>>>(tperm, n_src, trp, tcol, cursor);
         BF_LAUNCHED("k_tsort_heavy");
       }
     }
@@ -480,9 +505,42 @@ __global__ void __launch_bounds__(256) k_mask_seed(const int32_t* __restrict__ i
   }
 }
 
-// One layer: 32/SEG active nodes of layer l per warp; accumulates n_l, e_l per item (lane k
-// handles items k and k+32 of each node) and ORs each node's mask into layer l-1 for the node
-// itself and its sampled neighbours, appending first touches to act_out.
+// Appends u to the compacted list with one counter atomic per set of converged threads.
+__device__ __forceinline__ void append_aggregated(int32_t* __restrict__ list, int32_t* __restrict__ n, int32_t u) {
+  cg::coalesced_group grp = cg::coalesced_threads();
+  int32_t base = 0;
+  if (grp.thread_rank() == 0) base = atomicAdd(n, (int32_t)grp.size());
+  base = grp.shfl(base, 0);
+  list[base + (int32_t)grp.thread_rank()] = u;
+}
+
+// Per-item counters of a warp's nodes: lane k accumulates items k and k + 32 in registers; the
+// block's sums are flushed once at the end.
+struct ItemCounters {
+  uint32_t n0 = 0, n1 = 0;
+  unsigned long long e0 = 0, e1 = 0;
+};
+
+__device__ __forceinline__ void flush_item_counters(const ItemCounters& c, unsigned long long* __restrict__ gn,
+                                                    unsigned long long* __restrict__ ge,
+                                                    unsigned long long* sn, unsigned long long* se) {
+  const int lane = threadIdx.x & 31;
+  if (c.n0) atomicAdd(&sn[lane], (unsigned long long)c.n0);
+  if (c.n1) atomicAdd(&sn[lane + 32], (unsigned long long)c.n1);
+  if (ge) {
+    if (c.e0) atomicAdd(&se[lane], c.e0);
+    if (c.e1) atomicAdd(&se[lane + 32], c.e1);
+  }
+  __syncthreads();
+  if (threadIdx.x < 64) {
+    if (sn[threadIdx.x]) atomicAdd(&gn[threadIdx.x], sn[threadIdx.x]);
+    if (ge && se[threadIdx.x]) atomicAdd(&ge[threadIdx.x], se[threadIdx.x]);
+  }
+}
+
+// One layer: 32/SEG active nodes of layer l per warp; accumulates n_l, e_l per item and ORs
+// each node's mask into layer l-1 for the node itself and its sampled neighbours, appending
+// first touches to act_out.
 template <int SEG>
 __global__ void __launch_bounds__(256) k_mask_layer(const int32_t* __restrict__ act, int64_t n_act,
                                                     const unsigned long long* __restrict__ m_in,
@@ -496,6 +554,7 @@ __global__ void __launch_bounds__(256) k_mask_layer(const int32_t* __restrict__ 
   if (threadIdx.x < 64) { sn[threadIdx.x] = 0; se[threadIdx.x] = 0; }
   __syncthreads();
   const int lane = threadIdx.x & 31, g = lane / SEG;
+  ItemCounters cnt;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
   for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n_act; w += warps) {
     const int64_t slot = w * G + g;
@@ -508,26 +567,25 @@ __global__ void __launch_bounds__(256) k_mask_layer(const int32_t* __restrict__ 
       const int64_t deg = grow[v + 1] - grow[v];
       D = (f > 0 && deg > f) ? f : deg;
     }
+#pragma unroll
     for (int q = 0; q < G; ++q) {
       const unsigned long long mq = __shfl_sync(0xffffffffu, mask, q * SEG);
-      const unsigned long long Dq = (unsigned long long)__shfl_sync(0xffffffffu, (long long)D, q * SEG);
-      if ((mq >> lane) & 1ull) { atomicAdd(&sn[lane], 1ull); atomicAdd(&se[lane], Dq); }
-      if ((mq >> (lane + 32)) & 1ull) { atomicAdd(&sn[lane + 32], 1ull); atomicAdd(&se[lane + 32], Dq); }
+      const uint32_t Dq = (uint32_t)__shfl_sync(0xffffffffu, (int32_t)D, q * SEG);
+      if ((mq >> lane) & 1ull) { cnt.n0 += 1; cnt.e0 += Dq; }
+      if ((mq >> (lane + 32)) & 1ull) { cnt.n1 += 1; cnt.e1 += Dq; }
     }
     if (slot < n_act && (lane % SEG) == 0 && atomicOr(&m_out[v], mask) == 0ull)
-      act_out[atomicAdd(n_out, 1)] = (int32_t)v;
+      append_aggregated(act_out, n_out, (int32_t)v);
     sample_warp_rows<SEG>(w, n_act, DstRows{act}, grow, gcol, f, hop, seed, [&](int64_t s_, int32_t, int32_t u) {
       const unsigned long long ms = m_in[act[s_]];
-      if (atomicOr(&m_out[u], ms) == 0ull) act_out[atomicAdd(n_out, 1)] = u;
+      if (atomicOr(&m_out[u], ms) == 0ull) append_aggregated(act_out, n_out, u);
     });
   }
-  __syncthreads();
-  if (threadIdx.x < 64) {
-    if (sn[threadIdx.x]) atomicAdd(&gn[threadIdx.x], sn[threadIdx.x]);
-    if (se[threadIdx.x]) atomicAdd(&ge[threadIdx.x], se[threadIdx.x]);
-  }
+  flush_item_counters(cnt, gn, ge, sn, se);
 }
 
+// Clears the masks of the active list; with gn, first counts per item how many active nodes
+// carry its bit (one ballot per item bit, counted in registers).
 __global__ void __launch_bounds__(256) k_mask_count(const int32_t* __restrict__ act, int64_t n_act,
                                                     unsigned long long* __restrict__ m,
                                                     unsigned long long* __restrict__ gn, int clear) {
@@ -535,6 +593,7 @@ __global__ void __launch_bounds__(256) k_mask_count(const int32_t* __restrict__ 
   if (threadIdx.x < 64) sn[threadIdx.x] = 0;
   __syncthreads();
   const int lane = threadIdx.x & 31;
+  ItemCounters cnt;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i0 = blockIdx.x * (int64_t)blockDim.x; i0 < n_act; i0 += stride) {
     const int64_t i = i0 + threadIdx.x;
@@ -545,15 +604,16 @@ __global__ void __launch_bounds__(256) k_mask_count(const int32_t* __restrict__ 
       if (clear) m[v] = 0ull;
     }
     if (gn) {
-      // warp-cooperative per-item counts: one ballot per item bit
-      for (int k = 0; k < 64; ++k) {
-        const unsigned b = __ballot_sync(0xffffffffu, (mask >> k) & 1ull);
-        if (lane == (k & 31) && b) atomicAdd(&sn[k], (unsigned long long)__popc(b));
+      const unsigned lo = (unsigned)mask, hi = (unsigned)(mask >> 32);
+#pragma unroll
+      for (int k = 0; k < 32; ++k) {
+        const unsigned b0 = __ballot_sync(0xffffffffu, (lo >> k) & 1u);
+        const unsigned b1 = __ballot_sync(0xffffffffu, (hi >> k) & 1u);
+        if (lane == k) { cnt.n0 += __popc(b0); cnt.n1 += __popc(b1); }
       }
     }
   }
-  __syncthreads();
-  if (gn && threadIdx.x < 64 && sn[threadIdx.x]) atomicAdd(&gn[threadIdx.x], sn[threadIdx.x]);
+  if (gn) flush_item_counters(cnt, gn, nullptr, sn, nullptr);
 }
 
 int64_t mask_stats_bytes(int64_t N, int L) {

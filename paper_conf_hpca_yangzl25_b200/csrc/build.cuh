@@ -11,10 +11,12 @@ int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only);
 
 // Builds block `layer` (1-based) whose dst are dst[0..n_dst).  sizes_only: only row_ptr and
 // src_global are produced (scheduler statistics).  Allocates from A (bottom: persistent block
-// arrays; top frame: scratch).  Synchronises the stream twice.
+// arrays; top frame: scratch).  known = {e_l, n_{l-1}} (exact, from the plan): no host
+// synchronisation, n_heavy / n_heavy_t are left at -1; else the stream is synchronised to read
+// the sizes (twice, three times for layers >= 2).
 buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
                            uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
-                           buffalo_block* blk, cudaStream_t s);
+                           buffalo_block* blk, cudaStream_t s, const int64_t* known = nullptr);
 
 // Degree bucketing of the seeds (Alg. 3 l.1): bucket[i] = min(D(seed_i), F); order = seed
 // positions grouped by bucket (stable); sorted_ids = seeds[order]; hist_h[0..F].

@@ -89,4 +89,13 @@ struct Arena {
 __device__ __forceinline__ float bf2f(__nv_bfloat16 v) { return __bfloat162float(v); }
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 
+// Rows with more than kHeavyT entries sit at the tail of a degree-class permutation (stable
+// partition by min(D, kHeavyT + 1)).  Kernels over them walk the permutation from its end and
+// stop at the first light row, so they need no host-side count: the grid is the count when the
+// host knows it (>= 0), else a bound from the entry total (at most e / (kHeavyT + 1) heavy rows).
+inline int heavy_tail_grid(int64_t n_heavy_known, int64_t entries) {
+  if (n_heavy_known >= 0) return (int)std::min<int64_t>(n_heavy_known, 148 * 8);
+  return (int)std::min<int64_t>(entries / (kHeavyT + 1), 148 * 8);
+}
+
 }  // namespace buffalo

@@ -116,15 +116,17 @@ __global__ void __launch_bounds__(256) k_agg_rows(const int32_t* __restrict__ rp
 
 // ------------------------------------------------------------------ aggregate (long tail)
 template <class TI, class TO, int C>
-__global__ void __launch_bounds__(256) k_agg_heavy(const int32_t* __restrict__ heavy,
+__global__ void __launch_bounds__(256) k_agg_heavy(const int32_t* __restrict__ perm, int64_t n,
                                                    const int32_t* __restrict__ rp,
                                                    const int32_t* __restrict__ col,
                                                    const TI* __restrict__ h, int64_t ldh, int d,
                                                    TO* __restrict__ agg, int64_t lda) {
   __shared__ float part[8][32][C];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int64_t i = heavy[blockIdx.x];
+  for (int64_t hh = blockIdx.x; hh < n; hh += gridDim.x) {
+  const int64_t i = perm[n - 1 - hh];        // heavy rows: the tail of the degree-class perm
   const int32_t b = rp[i], e_end = rp[i + 1];
+  if (e_end - b <= kHeavyT) break;
   const float fd = (float)(e_end - b);
   const int nch = (d + C - 1) / C;
   for (int c0 = 0; c0 < nch; c0 += 32) {
@@ -156,6 +158,7 @@ __global__ void __launch_bounds__(256) k_agg_heavy(const int32_t* __restrict__ h
     }
     __syncthreads();
   }
+  }
 }
 
 template <class TI, class TO>
@@ -170,11 +173,12 @@ static buffalo_status launch_agg(const buffalo_block* blk, const int32_t* col, c
     k_agg_rows<TI, TO, 4><<<grid_for(n * 32, 256, 16), 256, 0, s>>>(blk->row_ptr, col, n, h, ldh, d, agg, lda);
   }
   BF_LAUNCHED("k_agg_rows");
-  if (blk->n_heavy > 0) {
+  const int hg = heavy_tail_grid(blk->n_heavy, blk->n_edges);
+  if (hg > 0) {
     if (wide)
-      k_agg_heavy<TI, TO, 8><<<(unsigned)blk->n_heavy, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, ldh, d, agg, lda);
+      k_agg_heavy<TI, TO, 8><<<hg, 256, 0, s>>>(blk->cls_perm, n, blk->row_ptr, col, h, ldh, d, agg, lda);
     else
-      k_agg_heavy<TI, TO, 4><<<(unsigned)blk->n_heavy, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, ldh, d, agg, lda);
+      k_agg_heavy<TI, TO, 4><<<hg, 256, 0, s>>>(blk->cls_perm, n, blk->row_ptr, col, h, ldh, d, agg, lda);
     BF_LAUNCHED("k_agg_heavy");
   }
   return BUFFALO_OK;
@@ -451,15 +455,18 @@ buffalo_status launch_agg_heavy_bf16(const FwdArgs& a, cudaStream_t s) {
   const int32_t* col = a.layer1 ? blk->col_global : blk->col_local;
   const bool wide = a.d_in > 128;
   __nv_bfloat16* agg = (__nv_bfloat16*)a.agg;
-  const unsigned g = (unsigned)blk->n_heavy;
+  const int g = heavy_tail_grid(blk->n_heavy, blk->n_edges);
+  if (g <= 0) return BUFFALO_OK;
+  const int32_t* perm = blk->cls_perm;
+  const int64_t n = blk->n_dst;
   if (a.in_bf16) {
     const __nv_bfloat16* h = (const __nv_bfloat16*)a.h_src;
-    if (wide) k_agg_heavy<__nv_bfloat16, __nv_bfloat16, 8><<<g, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
-    else k_agg_heavy<__nv_bfloat16, __nv_bfloat16, 4><<<g, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
+    if (wide) k_agg_heavy<__nv_bfloat16, __nv_bfloat16, 8><<<g, 256, 0, s>>>(perm, n, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
+    else k_agg_heavy<__nv_bfloat16, __nv_bfloat16, 4><<<g, 256, 0, s>>>(perm, n, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
   } else {
     const float* h = (const float*)a.h_src;
-    if (wide) k_agg_heavy<float, __nv_bfloat16, 8><<<g, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
-    else k_agg_heavy<float, __nv_bfloat16, 4><<<g, 256, 0, s>>>(blk->heavy, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
+    if (wide) k_agg_heavy<float, __nv_bfloat16, 8><<<g, 256, 0, s>>>(perm, n, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
+    else k_agg_heavy<float, __nv_bfloat16, 4><<<g, 256, 0, s>>>(perm, n, blk->row_ptr, col, h, a.ld_src, a.d_in, agg, a.ld_agg);
   }
   BF_LAUNCHED("k_agg_heavy");
   return BUFFALO_OK;

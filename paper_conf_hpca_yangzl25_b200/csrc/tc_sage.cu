@@ -768,7 +768,7 @@ template <class TI>
 static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   const buffalo_block* blk = a.blk;
   if (blk->n_dst <= 0) return BUFFALO_OK;
-  if (blk->n_heavy > 0) BF_CHECK(launch_agg_heavy_bf16(a, s));
+  BF_CHECK(launch_agg_heavy_bf16(a, s));
   TcFwdParams p{};
   p.row_ptr = blk->row_ptr;
   p.col = a.layer1 ? blk->col_global : blk->col_local;
@@ -1093,15 +1093,17 @@ __global__ void k_reduce_db(const float* __restrict__ part, int S, int d, float*
 
 // Long-tail transposed rows (more than kHeavyT dst): out[h] = sum_{t in T(list[h])} z[t_col[t]],
 // 8 warps over the entries (warp w takes t = w, w+8, ...), combined in warp order.
-__global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restrict__ list,
+__global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restrict__ perm, int64_t n,
                                                         const int32_t* __restrict__ rp,
                                                         const int32_t* __restrict__ col,
                                                         const __nv_bfloat16* __restrict__ z, int64_t ldz,
                                                         int dp, __nv_bfloat16* __restrict__ out, int by_row) {
   __shared__ float part[8][32][8];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int64_t j = list[blockIdx.x];
+  for (int64_t hh = blockIdx.x; hh < n; hh += gridDim.x) {
+  const int64_t j = perm[n - 1 - hh];          // heavy rows: the tail of the degree-class perm
   const int32_t b = rp[j], e_end = rp[j + 1];
+  if (e_end - b <= kHeavyT) break;
   const int nch = dp / 8;
   for (int c0 = 0; c0 < nch; c0 += 32) {
     const int c = c0 + lane;
@@ -1125,11 +1127,12 @@ __global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restric
         for (int ww = 1; ww < 8; ++ww) s += part[ww][lane][k];
         acc[k] = s;
       }
-      *reinterpret_cast<uint4*>(out + (by_row ? j : (int64_t)blockIdx.x) * dp + c * 8) =
+      *reinterpret_cast<uint4*>(out + (by_row ? j : hh) * dp + c * 8) =
           make_uint4(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]), pack_bf16x2(acc[4], acc[5]),
                      pack_bf16x2(acc[6], acc[7]));
     }
     __syncthreads();
+  }
   }
 }
 
@@ -1226,9 +1229,9 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   // dH_{l-1} = [dZ (rows < n_dst) || sum_{i in T(j)} dZ[i]/D(i)] [W_self; W_neigh], written in the
   // prepared form of layer l-1 by the GEMM epilogue (ReLU' with H_{l-1}, /D_{l-1}, db partials)
   if (a.dh_src && blk->n_src > 0) {
-    if (blk->n_heavy_t > 0) {
-      k_sum_heavy_rows<<<(unsigned)blk->n_heavy_t, 256, 0, s>>>(blk->t_perm + (blk->n_src - blk->n_heavy_t),
-                                                                blk->t_row_ptr, blk->t_col, zs, dp, dp, aggT, 1);
+    const int hg = heavy_tail_grid(blk->n_heavy_t, blk->n_edges);
+    if (hg > 0) {
+      k_sum_heavy_rows<<<hg, 256, 0, s>>>(blk->t_perm, blk->n_src, blk->t_row_ptr, blk->t_col, zs, dp, dp, aggT, 1);
       BF_LAUNCHED("k_sum_heavy_rows");
     }
     BF_CHECK((launch_gather<__nv_bfloat16, 1>(blk->t_perm, blk->t_row_ptr, blk->t_col, blk->n_src, zs, dp, dp,

@@ -98,6 +98,7 @@ class Trainer:
         self.est_h = np.zeros(k_max, np.int64)
         self.rank_h = np.zeros(k_max, np.int32)
         self.hist_h = np.zeros(F + 1, np.int64)
+        self.sizes_h = np.zeros((k_max, 2 * self.L + 1), np.int64)     # exact per-group block sizes
         self.plan = B.Plan()
         self.plan.group_of_seed = self.group_of_seed.data_ptr()
         self.plan.group_seeds = self.group_seeds.data_ptr()
@@ -106,6 +107,7 @@ class Trainer:
         self.plan.est_bytes_h = self.est_h.ctypes.data
         self.plan.rank_of_group_h = self.rank_h.ctypes.data
         self.plan.hist_h = self.hist_h.ctypes.data
+        self.plan.group_sizes_h = self.sizes_h.ctypes.data
         sampler = B.make_sampler(self.fanout, F, base_seed)
         wsb = B.bucketize_workspace_bytes(self.graph.g, self.S, sampler, self.model)
         self.bucket_ws = torch.empty(wsb, dtype=torch.uint8, device=device)
@@ -128,11 +130,13 @@ class Trainer:
         if self.arena.numel() < nbytes:
             self.arena = torch.empty(int(nbytes), dtype=torch.uint8, device=self.device)
 
-    def build(self, off, n, sampler):
+    def build(self, off, n, sampler, sizes=None):
+        """Blocks of the group at group_seeds[off:off+n]; sizes = its row of the plan's exact
+        block sizes (sync-free build) or None (sizes read back while building)."""
         while True:
             try:
                 return B.build_blocks(self.graph.g, self.group_seeds.data_ptr() + 4 * int(off), n, sampler,
-                                      self.model, self.blocks, self.arena)
+                                      self.model, self.blocks, self.arena, sizes)
             except B.BuffaloError as e:
                 if e.status != B.ERR_CAPACITY:
                     raise
@@ -166,8 +170,8 @@ class Trainer:
         ids = self.group_seeds.data_ptr() + 4 * int(off)
         B.softmax_ce(b.out, b.ld_out, n, self.dims[-1], self.labels, ids, self.S, self.loss, b.dh, b.ld_dh)
 
-    def microbatch(self, off, n, sampler):
-        self.build(off, n, sampler)
+    def microbatch(self, off, n, sampler, sizes=None):
+        self.build(off, n, sampler, sizes)
         self.forward()
         self.loss_and_grad(off, n)
         self.backward()
@@ -188,13 +192,14 @@ class Trainer:
         """One Buffalo iteration; returns stats (K, own groups, aggregated edges, ...)."""
         self.loss.zero_()
         K, offs, est, ranks = self.schedule(epoch)
-        if self.arena.numel() == 0:
-            mine = [est[k] for k in range(K) if ranks[k] == self.rank]
-            self._ensure_arena(max(mine) if mine else 1 << 20)
+        mine = own_groups(ranks, self.rank)
+        L = self.L
+        need = [B.estimate_mem(self.sizes_h[k, :L + 1], self.sizes_h[k, L + 1:], self.model)[0] for k in mine]
+        self._ensure_arena(max(need) if need else 1 << 20)          # exact (R15): no build retries
         sampler = self.sampler(epoch)
         groups = []
-        for k in own_groups(ranks, self.rank):
-            groups.append(self.microbatch(offs[k], int(offs[k + 1] - offs[k]), sampler))
+        for k in mine:
+            groups.append(self.microbatch(offs[k], int(offs[k + 1] - offs[k]), sampler, self.sizes_h[k]))
         self.allreduce()
         self.step(lr)
         self.last = dict(K=K, k_tried=self.plan.k_tried, exploded=self.plan.exploded, est=est,

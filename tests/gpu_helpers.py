@@ -30,7 +30,7 @@ def blocks_to_numpy(arena, blocks, L):
         d["col_global"] = arena_view(arena, b.col_global, b.n_edges).cpu().numpy() if b.col_global else None
         d["t_row_ptr"] = arena_view(arena, b.t_row_ptr, b.n_src + 1).cpu().numpy() if b.t_row_ptr else None
         d["t_col"] = arena_view(arena, b.t_col, b.n_edges).cpu().numpy() if b.t_col else None
-        d["heavy"] = arena_view(arena, b.heavy, b.n_heavy).cpu().numpy()
+        d["heavy"] = arena_view(arena, b.heavy, b.n_heavy).cpu().numpy() if b.heavy else None
         d["cls_perm"] = arena_view(arena, b.cls_perm, b.n_dst).cpu().numpy()
         d["t_perm"] = arena_view(arena, b.t_perm, b.n_src).cpu().numpy() if b.t_perm else None
         d["n_heavy_t"] = b.n_heavy_t

@@ -78,6 +78,42 @@ def test_blocks_bit_exact(name):
         assert got[0]["n_heavy"] > 0          # the long-tail path is exercised
 
 
+@pytest.mark.parametrize("name", list(CASES))
+def test_blocks_sync_free_identical(name):
+    """buffalo_build_blocks with the exact sizes given (no host round trips) builds the same
+    blocks as the read-back build; the long-tail counts are then not reported."""
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case(name)
+    L = len(fan)
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs)
+    tr.group_seeds[: seeds.size].copy_(torch.as_tensor(seeds))
+    tr._ensure_arena(1 << 16)
+    sampler = B.make_sampler(fan, F, 11)
+    tr.build(0, seeds.size, sampler)
+    ref = blocks_to_numpy(tr.arena, tr.blocks, L)
+    peak = tr.blocks.arena_peak
+    sizes = np.array([ref[0]["n_src"]] + [b["n_dst"] for b in ref] + [b["n_edges"] for b in ref], np.int64)
+    tr.arena.fill_(0xAB)
+    small = tr.arena
+    tr.arena = small[: peak - 256]
+    with pytest.raises(B.BuffaloError) as ei:                  # capacity checked up front, exactly
+        B.build_blocks(tr.graph.g, tr.group_seeds.data_ptr(), seeds.size, sampler, tr.model, tr.blocks, tr.arena,
+                       sizes)
+    assert ei.value.status == B.ERR_CAPACITY and ei.value.required == peak
+    tr.arena = small
+    B.build_blocks(tr.graph.g, tr.group_seeds.data_ptr(), seeds.size, sampler, tr.model, tr.blocks, tr.arena, sizes)
+    got = blocks_to_numpy(tr.arena, tr.blocks, L)
+    assert tr.blocks.arena_peak == peak
+    for l, (a, r) in enumerate(zip(got, ref), start=1):
+        assert a["n_heavy"] == -1 and a["heavy"] is None and a["n_heavy_t"] == -1
+        for k in ("n_dst", "n_src", "n_edges"):
+            assert a[k] == r[k], (l, k)
+        for k in ("row_ptr", "col_local", "src_global", "col_global", "t_row_ptr", "t_col", "cls_perm", "t_perm"):
+            if r[k] is None:
+                assert a[k] is None, (l, k)
+            else:
+                np.testing.assert_array_equal(a[k], r[k], err_msg=f"layer {l} {k}")
+
+
 @pytest.mark.parametrize("name", ["sampled2", "full3", "mixed3"])
 @pytest.mark.parametrize("variant", ["k4", "budget", "C", "gpus3"])
 def test_bucketize_plan_bit_exact(name, variant):
@@ -105,6 +141,13 @@ def test_bucketize_plan_bit_exact(name, variant):
     np.testing.assert_array_equal(tr.group_seeds.cpu().numpy(), ref["group_seeds"])
     np.testing.assert_array_equal(tr.group_of_seed.cpu().numpy(), ref["group_of_seed"])
     np.testing.assert_array_equal(tr.hist_h, ref["hist"])
+    # exact block sizes of every group (plan.group_sizes_h) = the oracle's blocks of that group
+    L = len(fan)
+    gs = ref["group_seeds"]
+    for k in range(K):
+        blocks = O.build_blocks(g, gs[offs[k]:offs[k + 1]], L, fan, 3)
+        want = [blocks[0]["n_src"]] + [b["n_dst"] for b in blocks] + [b["n_edges"] for b in blocks]
+        np.testing.assert_array_equal(tr.sizes_h[k], want, err_msg=f"group {k}")
 
 
 def test_bucketize_budget_error():

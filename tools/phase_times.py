@@ -47,12 +47,13 @@ def main():
         tr.loss.zero_()
         K, offs, est, ranks = tr.schedule(ep)
         e1 = ev()
-        if tr.arena.numel() == 0:
-            tr._ensure_arena(max(est))
+        L = tr.L
+        tr._ensure_arena(max(B.estimate_mem(tr.sizes_h[k, :L + 1], tr.sizes_h[k, L + 1:], tr.model)[0]
+                             for k in range(K)))
         sampler = tr.sampler(ep)
         marks = []
         for k in range(K):
-            a = ev(); tr.build(offs[k], int(offs[k + 1] - offs[k]), sampler); b = ev()
+            a = ev(); tr.build(offs[k], int(offs[k + 1] - offs[k]), sampler, tr.sizes_h[k]); b = ev()
             tr.forward(); c = ev()
             tr.loss_and_grad(offs[k], int(offs[k + 1] - offs[k])); d = ev()
             tr.backward(); e = ev()

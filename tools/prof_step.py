@@ -22,7 +22,14 @@ def main():
     tr = Trainer((rp, col), feats, torch.as_tensor(y).cuda(), torch.as_tensor(seeds).cuda(), cfg.dims,
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=B.BF16, gemm_mode=B.GEMM_BF16,
                  k_min=cfg.k_min, k_max=max(cfg.k_min, min(cfg.k_max, 64)))
-    if len(sys.argv) > 3:
+    if len(sys.argv) > 3 and sys.argv[3] == "auto":
+        # bench.py's products calibration: M_ctr = Eq. 2 estimate of K=1 / 8
+        t1 = Trainer((rp, col), feats, torch.as_tensor(y).cuda(), torch.as_tensor(seeds).cuda(), cfg.dims,
+                     cfg.fanout, cfg.F, Ws, bs, feat_dtype=B.BF16, gemm_mode=B.GEMM_BF16, k_min=1, k_max=1)
+        _, _, est1, _ = t1.schedule(0)
+        del t1
+        tr.sched.mem_budget = int(est1[0]) // 8
+    elif len(sys.argv) > 3:
         tr.sched.mem_budget = int(sys.argv[3])
     for e in range(epochs):
         st = tr.run_epoch(epoch=e, lr=0.01)
