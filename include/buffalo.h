@@ -45,8 +45,9 @@ enum { BUFFALO_GEMM_FFMA = 0, BUFFALO_GEMM_BF16 = 1 };  /* Update GEMM: fp32 SIM
 enum { BUFFALO_MAX_LAYERS = 8, BUFFALO_MAX_FANOUT = 32, BUFFALO_MAX_DIM = 4096 };
 
 /* Input graph (the batch's host graph): CSR, rows sorted ascending, symmetric,
- * no self loops or duplicates.  row_ptr int64[num_nodes+1], col int32[nnz].  node_map is a
- * workspace int32[num_nodes] prepared once by buffalo_graph_prepare (all INT32_MAX) and
+ * no self loops or duplicates.  row_ptr int64[num_nodes+1], col int32[nnz].  node_map points
+ * to the graph workspace (buffalo_graph_workspace_bytes): int32[num_nodes] node map, then the
+ * relabel node bitmap and its word prefix; prepared once by buffalo_graph_prepare and
  * restored by every call that uses it. */
 typedef struct {
   int64_t num_nodes, nnz;
@@ -137,9 +138,11 @@ typedef struct {
 } buffalo_blocks;
 
 /* ------------------------------------------------------------------ graph workspace */
-/* Bytes of the node_map workspace (int32 per node, 256-B rounded). */
+/* Bytes of the graph workspace: node map int32[N], bitmap uint32[ceil(N/32)], word prefix
+ * int32[ceil(N/32)+1] and a scan workspace, each 256-B rounded (about 4.2 bytes per node). */
 BUFFALO_API size_t buffalo_graph_workspace_bytes(int64_t num_nodes);
-/* Sets g->node_map = workspace and fills it with INT32_MAX (stream-ordered). */
+/* Sets g->node_map = workspace, fills the node map with INT32_MAX and clears the bitmap
+ * (stream-ordered). */
 BUFFALO_API buffalo_status buffalo_graph_prepare(buffalo_graph* g, void* workspace, size_t bytes, void* stream);
 
 /* ------------------------------------------------------------------ a1-a3: scheduler */

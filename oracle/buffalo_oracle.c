@@ -18,7 +18,8 @@
  *  - oracle_build_blocks  : BlockGenerate / MicroBatchGenerator, Alg. 2 l.5 PAPER.md:237,
  *                           Alg. 3 l.11 PAPER.md:279: the L bipartite blocks of one group,
  *                           built top-down from the output layer; local src ids = dst prefix
- *                           then first occurrence  [DESIGN.md readings R3, R4]
+ *                           then the other neighbours in ascending global id
+ *                           [DESIGN.md readings R3, R4]
  */
 #include <stdint.h>
 #include <stdlib.h>
@@ -84,6 +85,11 @@ int64_t oracle_sample_row(const int64_t* row_ptr, const int32_t* col, int64_t v,
 }
 
 /* ---------------------------------------------------------------- blocks (Alg. 2 l.5) */
+static int cmp_i32(const void* a, const void* b) {
+    int32_t x = *(const int32_t*)a, y = *(const int32_t*)b;
+    return (x > y) - (x < y);
+}
+
 typedef struct {
     int64_t n_dst, n_src, n_edges;
     int32_t* row_ptr;     /* [n_dst + 1] */
@@ -136,16 +142,19 @@ int oracle_build_blocks(int64_t N, const int64_t* row_ptr, const int32_t* col,
             e += d;
             rp[i + 1] = (int32_t)e;
         }
-        /* pass 2: src = dst (prefix, same order), then each new neighbour at first occurrence */
+        /* pass 2: src = dst (prefix, same order), then the distinct neighbours that are not
+           dst, in ascending global id (R3) */
         int32_t* src = (int32_t*)malloc(sizeof(int32_t) * (size_t)(n_dst + e + 1));
         int64_t n_src = 0;
         for (int64_t i = 0; i < n_dst; ++i) { pos[dst[i]] = n_src; src[n_src++] = dst[i]; }
-        int32_t* cl = (int32_t*)malloc(sizeof(int32_t) * (size_t)(e > 0 ? e : 1));
         for (int64_t k = 0; k < e; ++k) {
             int32_t u = cg[k];
-            if (pos[u] < 0) { pos[u] = n_src; src[n_src++] = u; }
-            cl[k] = (int32_t)pos[u];
+            if (pos[u] == -1) { pos[u] = -2; src[n_src++] = u; }   /* -2: seen, not yet placed */
         }
+        qsort(src + n_dst, (size_t)(n_src - n_dst), sizeof(int32_t), cmp_i32);
+        for (int64_t j = n_dst; j < n_src; ++j) pos[src[j]] = j;
+        int32_t* cl = (int32_t*)malloc(sizeof(int32_t) * (size_t)(e > 0 ? e : 1));
+        for (int64_t k = 0; k < e; ++k) cl[k] = (int32_t)pos[cg[k]];
         for (int64_t j = 0; j < n_src; ++j) pos[src[j]] = -1;
         b->n_dst = n_dst; b->n_src = n_src; b->n_edges = e;
         b->row_ptr = rp; b->col_local = cl; b->col_global = cg;

@@ -237,7 +237,7 @@ const char* buffalo_status_str(buffalo_status s) {
 const char* buffalo_last_error(void) { return g_err.c_str(); }
 int64_t buffalo_launch_count(void) { return g_launches.load(); }
 
-size_t buffalo_graph_workspace_bytes(int64_t num_nodes) { return (size_t)R(4 * (num_nodes > 0 ? num_nodes : 1)); }
+size_t buffalo_graph_workspace_bytes(int64_t num_nodes) { return (size_t)graph_ws_bytes(num_nodes); }
 
 buffalo_status buffalo_graph_prepare(buffalo_graph* g, void* workspace, size_t bytes, void* stream) {
   BF_CHECK(require_sm100());
@@ -247,6 +247,8 @@ buffalo_status buffalo_graph_prepare(buffalo_graph* g, void* workspace, size_t b
   cudaStream_t s = (cudaStream_t)stream;
   k_fill_i32<<<grid_for(g->num_nodes, 256), 256, 0, s>>>(g->node_map, g->num_nodes, INT32_MAX);
   BF_LAUNCHED("k_fill_i32");
+  const GraphWs gw = graph_ws(g);
+  BF_CUDA(cudaMemsetAsync(gw.bits, 0, sizeof(uint32_t) * gw.words, s));
   return BUFFALO_OK;
 }
 

@@ -101,38 +101,10 @@ static void launch_sample_fill(int seg, int64_t n, cudaStream_t s, Args... args)
 }
 
 // ------------------------------------------------------------------ a5: relabel
-// Candidate position p: p < n_dst -> dst[p], else col_global[p - n_dst].
-struct Cand {
-  const int32_t* dst;
-  const int32_t* colg;
-  int64_t n_dst;
-  __device__ __forceinline__ int32_t operator()(int64_t p) const {
-    return p < n_dst ? dst[p] : colg[p - n_dst];
-  }
-};
-
-__global__ void k_relabel_min(Cand c, int64_t total, int32_t* __restrict__ node_map) {
-  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < total;
-       p += (int64_t)gridDim.x * blockDim.x)
-    atomicMin(&node_map[c(p)], (int32_t)p);
-}
-
-struct FirstFlag {
-  Cand c;
-  const int32_t* node_map;
-  __device__ __forceinline__ int32_t operator()(int64_t p) const {
-    return node_map[c(p)] == (int32_t)p ? 1 : 0;
-  }
-};
-struct EmitSrc {
-  Cand c;
-  int32_t* src;
-  int64_t cap;
-  __device__ __forceinline__ void operator()(int64_t p, int32_t excl, int32_t v) const {
-    if (v && excl < cap) src[excl] = c(p);
-  }
-};
-
+// Local src ids (R3): the dst keep their positions 0..n_dst-1 (node_map[dst[i]] = i); the other
+// distinct neighbours follow in ascending global id.  They are marked in a node bitmap; an
+// exclusive popcount scan over its words gives each word's first local id, so that
+// local(u) = n_dst + prefix[u / 32] + popc(bits[u / 32] & below(u % 32)).
 __global__ void k_set_map(const int32_t* __restrict__ src, int64_t n, int32_t* __restrict__ node_map) {
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
     node_map[src[j]] = (int32_t)j;
@@ -141,10 +113,47 @@ __global__ void k_reset_map(const int32_t* __restrict__ src, int64_t n, int32_t*
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
     node_map[src[j]] = INT32_MAX;
 }
+__global__ void k_mark_bits(const int32_t* __restrict__ colg, int64_t e, const int32_t* __restrict__ node_map,
+                            uint32_t* __restrict__ bits) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t u = colg[k];
+    if (node_map[u] != INT32_MAX) continue;                      // a dst: keeps its prefix id
+    const uint32_t b = 1u << (u & 31);
+    if (!(bits[u >> 5] & b)) atomicOr(&bits[u >> 5], b);
+  }
+}
+struct PopcWord {
+  const uint32_t* bits;
+  __device__ __forceinline__ int32_t operator()(int64_t w) const { return __popc(bits[w]); }
+};
+// Scan store: the word's exclusive prefix, and its nodes appended to src in ascending id.
+struct EmitWord {
+  const uint32_t* bits;
+  int32_t* prefix;
+  int32_t* src;            // src + n_dst
+  int64_t cap;             // n_src - n_dst
+  __device__ __forceinline__ void operator()(int64_t w, int32_t excl, int32_t v) const {
+    prefix[w] = excl;
+    uint32_t m = v ? bits[w] : 0u;
+    int32_t r = excl;
+    while (m) {
+      const int b = __ffs(m) - 1;
+      m &= m - 1;
+      if (r < cap) src[r] = (int32_t)(w * 32 + b);
+      ++r;
+    }
+  }
+};
 __global__ void k_col_local(const int32_t* __restrict__ colg, int64_t e, const int32_t* __restrict__ node_map,
+                            const uint32_t* __restrict__ bits, const int32_t* __restrict__ prefix, int32_t n_dst,
                             int32_t* __restrict__ col_local) {
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x)
-    col_local[k] = node_map[colg[k]];
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t u = colg[k];
+    const int32_t m = node_map[u];
+    col_local[k] = m != INT32_MAX
+                       ? m
+                       : n_dst + prefix[u >> 5] + __popc(bits[u >> 5] & ((1u << (u & 31)) - 1u));
+  }
 }
 
 // ------------------------------------------------------------------ a6: heavy rows, transpose
@@ -335,45 +344,47 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
                        colg, e);
     BF_LAUNCHED("k_sample_fill");
   }
-  // relabel: first occurrence over the candidate sequence dst ++ col_global
-  Cand cand{dst, colg, n_dst};
-  const int64_t total = n_dst + e;
-  if (total > 0) {
-    k_relabel_min<<<grid_for(total, 256), 256, 0, s>>>(cand, total, g->node_map);
-    BF_LAUNCHED("k_relabel_min");
+  // relabel (R3): dst prefix, then the other neighbours in ascending global id
+  const GraphWs gw = graph_ws(g);
+  if (n_dst > 0) {
+    k_set_map<<<grid_for(n_dst, 256), 256, 0, s>>>(dst, n_dst, g->node_map);
+    BF_LAUNCHED("k_set_map");
   }
-  FirstFlag ff{cand, g->node_map};
+  if (e > 0) {
+    k_mark_bits<<<grid_for(e, 256), 256, 0, s>>>(colg, e, g->node_map, gw.bits);
+    BF_LAUNCHED("k_mark_bits");
+  }
   int64_t n_src = 0;
   if (known) {
     n_src = known[1];
   } else {
-    BF_CHECK(device_count(ff, total, totals, s));
-    int32_t ns32 = 0;
-    BF_CHECK(d2h_i32(totals, &ns32, s));
+    BF_CHECK(device_count(PopcWord{gw.bits}, gw.words, totals, s));
+    int32_t nn32 = 0;
+    BF_CHECK(d2h_i32(totals, &nn32, s));
     BF_CUDA(cudaStreamSynchronize(s));                             // sync 2: n_{l-1}
-    n_src = ns32;
+    n_src = n_dst + nn32;
   }
   int32_t* src = (int32_t*)A.take(4 * n_src);
   if (A.overflow) return BUFFALO_ERR_CAPACITY;
-  BF_CHECK(device_scan(ff, EmitSrc{cand, src, n_src}, total, ws, totals + 2, s));
+  if (n_dst > 0) BF_CUDA(cudaMemcpyAsync(src, dst, sizeof(int32_t) * n_dst, cudaMemcpyDeviceToDevice, s));
+  BF_CHECK(device_scan(PopcWord{gw.bits}, EmitWord{gw.bits, gw.prefix, src + n_dst, n_src - n_dst}, gw.words,
+                       gw.scan_ws, totals + 2, s));
   blk->n_src = n_src;
   blk->src_global = src;
   blk->col_global = colg_persist;
   if (!sizes_only) {
-    if (n_src > 0) {
-      k_set_map<<<grid_for(n_src, 256), 256, 0, s>>>(src, n_src, g->node_map);
-      BF_LAUNCHED("k_set_map");
-    }
     if (e > 0) {
-      k_col_local<<<grid_for(e, 256), 256, 0, s>>>(colg, e, g->node_map, col_local);
+      k_col_local<<<grid_for(e, 256), 256, 0, s>>>(colg, e, g->node_map, gw.bits, gw.prefix, (int32_t)n_dst,
+                                                   col_local);
       BF_LAUNCHED("k_col_local");
     }
     blk->col_local = col_local;
   }
-  if (n_src > 0) {
-    k_reset_map<<<grid_for(n_src, 256), 256, 0, s>>>(src, n_src, g->node_map);
+  if (n_dst > 0) {
+    k_reset_map<<<grid_for(n_dst, 256), 256, 0, s>>>(dst, n_dst, g->node_map);
     BF_LAUNCHED("k_reset_map");
   }
+  BF_CUDA(cudaMemsetAsync(gw.bits, 0, sizeof(uint32_t) * gw.words, s));
   blk->n_heavy_t = -1;
   if (!sizes_only && layer >= 2) {
     // transposed block: t_row_ptr by counting; t_col by an atomic-cursor fill followed by an

@@ -4,10 +4,36 @@
 #include <cstring>
 
 #include "common.cuh"
+#include "primitives.cuh"
 
 namespace buffalo {
 
 int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only);
+
+// Graph workspace (buffalo_graph_workspace_bytes): node_map int32[N] (INT32_MAX when idle), the
+// relabel bitmap uint32[W] (zero when idle), its word prefix int32[W + 1] and a scan workspace,
+// W = ceil(N / 32).
+struct GraphWs {
+  uint32_t* bits;
+  int32_t* prefix;
+  int32_t* scan_ws;
+  int64_t words;
+};
+inline int64_t graph_ws_words(int64_t N) { return ceil_div(N > 0 ? N : 1, 32); }
+inline int64_t graph_ws_bytes(int64_t N) {
+  const int64_t W = graph_ws_words(N);
+  return R(4 * (N > 0 ? N : 1)) + R(4 * W) + R(4 * (W + 1)) + R(4 * scan_ws_elems(W + 1));
+}
+inline GraphWs graph_ws(const buffalo_graph* g) {
+  const int64_t N = g->num_nodes, W = graph_ws_words(N);
+  char* q = (char*)g->node_map + R(4 * (N > 0 ? N : 1));
+  GraphWs w;
+  w.bits = (uint32_t*)q; q += R(4 * W);
+  w.prefix = (int32_t*)q; q += R(4 * (W + 1));
+  w.scan_ws = (int32_t*)q;
+  w.words = W;
+  return w;
+}
 
 // Builds block `layer` (1-based) whose dst are dst[0..n_dst).  sizes_only: only row_ptr and
 // src_global are produced (scheduler statistics).  Allocates from A (bottom: persistent block

@@ -4,7 +4,7 @@ What pins them (not the oracle itself):
 * Floyd sampling: size = min(deg, f), distinct, sorted, inside the row; chi-square uniformity
   over all C(deg, f) subsets (the defining property of sampling without replacement, R2).
 * full-neighbour blocks are exactly the CSR slices (no sampling involved);
-* blocks vs a brute-force set/dict construction (dst prefix, first-occurrence order, R3/R4);
+* blocks vs a brute-force set/dict construction (dst prefix, then ascending global id, R3/R4);
 * invariants of the north star: block edges are a subset of the graph, dst is a prefix of
   src, src unique, n_{l-1} = |dst u N_s(dst)|; transposed block by its definition.
 """
@@ -69,13 +69,8 @@ def _brute_blocks(g, seeds, L, fanout, seed):
     out = [None] * L
     for l in range(L, 0, -1):
         rows = [O.sample_row(g, v, fanout[l - 1], seed, L - l + 1).tolist() for v in dst]
-        src = list(dst)
-        where = {v: i for i, v in enumerate(dst)}
-        for r in rows:
-            for u in r:
-                if u not in where:
-                    where[u] = len(src)
-                    src.append(u)
+        src = list(dst) + sorted({u for r in rows for u in r} - set(dst))      # R3
+        where = {v: i for i, v in enumerate(src)}
         out[l - 1] = dict(dst=list(dst), rows=rows, src=src, where=where)
         dst = src
     return out

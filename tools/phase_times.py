@@ -52,12 +52,18 @@ def main():
                              for k in range(K)))
         sampler = tr.sampler(ep)
         marks = []
+        hb = hf = hk = 0.0
         for k in range(K):
-            a = ev(); tr.build(offs[k], int(offs[k + 1] - offs[k]), sampler, tr.sizes_h[k]); b = ev()
-            tr.forward(); c = ev()
+            a = ev(); t0 = time.perf_counter()
+            tr.build(offs[k], int(offs[k + 1] - offs[k]), sampler, tr.sizes_h[k]); t1 = time.perf_counter(); b = ev()
+            tr.forward(); t2 = time.perf_counter(); c = ev()
             tr.loss_and_grad(offs[k], int(offs[k + 1] - offs[k])); d = ev()
-            tr.backward(); e = ev()
+            t3 = time.perf_counter(); tr.backward(); t4 = time.perf_counter(); e = ev()
+            hb += t1 - t0; hf += t2 - t1; hk += t4 - t3
             marks.append((a, b, c, d, e))
+        if ep >= 2:
+            for nm, v in (("host build", hb), ("host fwd", hf), ("host bwd", hk)):
+                times[nm] = times.get(nm, 0.0) + 1e3 * v
         s0 = ev(); tr.step(0.01); s1 = ev()
         torch.cuda.synchronize()
         wall = (time.perf_counter() - w0) * 1e3
