@@ -126,16 +126,17 @@ struct PopcWord {
   const uint32_t* bits;
   __device__ __forceinline__ int32_t operator()(int64_t w) const { return __popc(bits[w]); }
 };
-// Scan store: the word's exclusive prefix, and its nodes appended to src in ascending id.
-struct EmitWord {
-  const uint32_t* bits;
+// Scan store: the word's exclusive prefix.
+struct StorePrefix {
   int32_t* prefix;
-  int32_t* src;            // src + n_dst
-  int64_t cap;             // n_src - n_dst
-  __device__ __forceinline__ void operator()(int64_t w, int32_t excl, int32_t v) const {
-    prefix[w] = excl;
-    uint32_t m = v ? bits[w] : 0u;
-    int32_t r = excl;
+  __device__ __forceinline__ void operator()(int64_t w, int32_t excl, int32_t) const { prefix[w] = excl; }
+};
+// The marked nodes appended to src (at src + n_dst) in ascending id: thread per bitmap word.
+__global__ void k_emit_bits(const uint32_t* __restrict__ bits, const int32_t* __restrict__ prefix, int64_t words,
+                            int32_t* __restrict__ src, int64_t cap) {
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < words; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t m = bits[w];
+    int32_t r = m ? prefix[w] : 0;
     while (m) {
       const int b = __ffs(m) - 1;
       m &= m - 1;
@@ -143,16 +144,17 @@ struct EmitWord {
       ++r;
     }
   }
-};
+}
+// col_local of every edge; tcnt (layers >= 2, zeroed): transposed row lengths counted on the way.
 __global__ void k_col_local(const int32_t* __restrict__ colg, int64_t e, const int32_t* __restrict__ node_map,
                             const uint32_t* __restrict__ bits, const int32_t* __restrict__ prefix, int32_t n_dst,
-                            int32_t* __restrict__ col_local) {
+                            int32_t* __restrict__ col_local, int32_t* __restrict__ tcnt) {
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x) {
     const int32_t u = colg[k];
     const int32_t m = node_map[u];
-    col_local[k] = m != INT32_MAX
-                       ? m
-                       : n_dst + prefix[u >> 5] + __popc(bits[u >> 5] & ((1u << (u & 31)) - 1u));
+    const int32_t c = m != INT32_MAX ? m : n_dst + prefix[u >> 5] + __popc(bits[u >> 5] & ((1u << (u & 31)) - 1u));
+    col_local[k] = c;
+    if (tcnt) atomicAdd(&tcnt[c], 1);
   }
 }
 
@@ -179,14 +181,6 @@ struct EmitPerm {
   __device__ __forceinline__ void operator()(int64_t i, int32_t pos) const { perm[pos] = (int32_t)i; }
 };
 
-__global__ void k_fill_zero(int32_t* a, int64_t n) {
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
-    a[k] = 0;
-}
-__global__ void k_tcount(const int32_t* __restrict__ col_local, int64_t e, int32_t* __restrict__ cnt) {
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x)
-    atomicAdd(&cnt[col_local[k]], 1);
-}
 // Transposed fill: edge (i -> col_local[e]) lands at an atomic cursor of its src row.
 __global__ void __launch_bounds__(256) k_tfill(const int32_t* __restrict__ rp, const int32_t* __restrict__ col_local,
                                                int64_t n, int32_t* __restrict__ cursor, int32_t* __restrict__ tcol) {
@@ -195,29 +189,58 @@ __global__ void __launch_bounds__(256) k_tfill(const int32_t* __restrict__ rp, c
   for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n; i += warps)
     for (int32_t k = rp[i] + lane; k < rp[i + 1]; k += 32) tcol[atomicAdd(&cursor[col_local[k]], 1)] = (int32_t)i;
 }
-// Ascending sort of transposed rows with <= 128 entries (warp per row, up to 4 values per lane,
-// rank = number of smaller entries; entries are distinct).
-__global__ void __launch_bounds__(256) k_tsort_small(const int32_t* __restrict__ rows, int64_t n,
-                                                     const int32_t* __restrict__ trp, int32_t* __restrict__ tcol) {
+// Ascending sort of the transposed rows with 2..128 entries.  t_perm lists the rows by length
+// (stable partition by min(len, 129); cls_start(c) = first position of class c, read from the
+// scanned partition counts), so rows are taken in bands: len 2..8 eight lanes per row, 9..16
+// sixteen, 17..128 a warp with up to four entries per lane.  rank = number of smaller entries
+// of the row (entries are distinct).
+template <int SEG, int V>
+__device__ __forceinline__ void tsort_segment(const int32_t* __restrict__ trp, int32_t* __restrict__ tcol, int32_t j,
+                                              bool valid) {
+  const int lane = threadIdx.x & 31, g = lane / SEG, sl = lane % SEG;
+  int32_t b = 0, len = 0;
+  if (valid) {
+    b = trp[j];
+    len = trp[j + 1] - b;
+  }
+  int32_t v[V];
+  int rank[V];
+#pragma unroll
+  for (int k = 0; k < V; ++k) {
+    v[k] = (sl + SEG * k < len) ? tcol[b + sl + SEG * k] : INT32_MAX;
+    rank[k] = 0;
+  }
+  const int tmax = SEG == 32 ? len : SEG * V;      // one row per warp at SEG = 32: len is uniform
+  for (int t = 0; t < tmax; ++t) {
+    const int32_t x = __shfl_sync(0xffffffffu, v[t / SEG], g * SEG + (t % SEG));
+#pragma unroll
+    for (int k = 0; k < V; ++k) rank[k] += x < v[k] ? 1 : 0;
+  }
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < V; ++k)
+    if (sl + SEG * k < len) tcol[b + rank[k]] = v[k];
+}
+
+__global__ void __launch_bounds__(256) k_tsort_banded(const int32_t* __restrict__ perm, const int32_t* __restrict__ trp,
+                                                      int32_t* __restrict__ tcol, const int32_t* __restrict__ cls_off,
+                                                      int64_t ntiles) {
+  const int64_t sA = cls_off[2 * ntiles], sB = cls_off[9 * ntiles], sC = cls_off[17 * ntiles];
+  const int64_t sH = cls_off[(kHeavyT + 1) * ntiles];
+  const int64_t wA = (sB - sA + 3) / 4, wB = (sC - sB + 1) / 2, wC = sH - sC;
   const int lane = threadIdx.x & 31;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < n; w += warps) {
-    const int32_t j = rows[w];
-    const int32_t b = trp[j], len = trp[j + 1] - b;
-    if (len <= 1 || len > kHeavyT) continue;                // heavy rows: k_tsort_heavy
-    int32_t v[4];
-    int rank[4] = {0, 0, 0, 0};
-#pragma unroll
-    for (int k = 0; k < 4; ++k) v[k] = (lane + 32 * k < len) ? tcol[b + lane + 32 * k] : INT32_MAX;
-    for (int src = 0; src < len; ++src) {
-      const int32_t x = __shfl_sync(0xffffffffu, v[src >> 5], src & 31);
-#pragma unroll
-      for (int k = 0; k < 4; ++k) rank[k] += x < v[k] ? 1 : 0;
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < wA + wB + wC; w += warps) {
+    if (w < wA) {
+      const int64_t p = sA + w * 4 + lane / 8;
+      tsort_segment<8, 1>(trp, tcol, p < sB ? perm[p] : 0, p < sB);
+    } else if (w < wA + wB) {
+      const int64_t p = sB + (w - wA) * 2 + lane / 16;
+      tsort_segment<16, 1>(trp, tcol, p < sC ? perm[p] : 0, p < sC);
+    } else {
+      const int64_t p = sC + (w - wA - wB);
+      tsort_segment<32, 4>(trp, tcol, perm[p], true);
     }
-    __syncwarp();
-#pragma unroll
-    for (int k = 0; k < 4; ++k)
-      if (lane + 32 * k < len) tcol[b + rank[k]] = v[k];
   }
 }
 // Long transposed rows (> 128 entries): CTA per row; the row is staged in `stage` (same
@@ -240,30 +263,43 @@ __global__ void __launch_bounds__(256) k_tsort_heavy(const int32_t* __restrict__
   __syncthreads();
   }
 }
-// ed[e] = dst index of edge e (warp per dst row).
-__global__ void k_edge_dst(const int32_t* __restrict__ rp, int64_t n, int32_t* __restrict__ ed) {
-  const int lane = threadIdx.x & 31;
-  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n; i += warps)
-    for (int32_t k = rp[i] + lane; k < rp[i + 1]; k += 32) ed[k] = (int32_t)i;
-}
-
-struct RadixKey {
-  const int32_t* keys;
-  int shift;
-  __device__ __forceinline__ int operator()(int64_t i) const { return (keys[i] >> shift) & 255; }
-};
-struct RadixEmit {
-  const int32_t* kin;
-  const int32_t* pin;
-  int32_t* kout;
-  int32_t* pout;
-  __device__ __forceinline__ void operator()(int64_t i, int32_t pos) const {
-    kout[pos] = kin[i];
-    pout[pos] = pin[i];
+// Long transposed rows, counting sort through a shared-memory bitmap over the dst range (the
+// entries are distinct dst indices < n_dst): set the bits, then every thread emits its slice
+// of words at the slice's popcount prefix.  O(len + n_dst / 32) per row.
+constexpr int kBitsortMaxWords = 40 * 1024;      // 160 KB of shared memory (n_dst <= 1.31 M)
+__global__ void __launch_bounds__(256) k_tsort_heavy_bits(const int32_t* __restrict__ perm, int64_t n,
+                                                          const int32_t* __restrict__ trp,
+                                                          int32_t* __restrict__ tcol, int32_t words) {
+  extern __shared__ uint32_t bm[];
+  __shared__ int32_t sw[33];
+  const int per = (words + blockDim.x - 1) / blockDim.x;
+  const int w0 = min(words, (int)threadIdx.x * per), w1 = min(words, w0 + per);
+  for (int64_t hh = blockIdx.x; hh < n; hh += gridDim.x) {
+    const int32_t j = perm[n - 1 - hh];          // heavy rows: the tail of the degree-class perm
+    const int32_t b = trp[j], len = trp[j + 1] - b;
+    if (len <= kHeavyT) break;
+    for (int w = threadIdx.x; w < words; w += blockDim.x) bm[w] = 0u;
+    __syncthreads();
+    for (int32_t k = threadIdx.x; k < len; k += blockDim.x) {
+      const int32_t x = tcol[b + k];
+      atomicOr(&bm[x >> 5], 1u << (x & 31));
+    }
+    __syncthreads();
+    int32_t cnt = 0;
+    for (int w = w0; w < w1; ++w) cnt += __popc(bm[w]);
+    int32_t total;
+    int32_t r = block_exclusive_sum<256>(cnt, sw, &total);
+    for (int w = w0; w < w1; ++w) {
+      uint32_t m = bm[w];
+      while (m) {
+        const int bit = __ffs(m) - 1;
+        m &= m - 1;
+        tcol[b + r++] = w * 32 + bit;
+      }
+    }
+    __syncthreads();
   }
-};
-
+}
 // ------------------------------------------------------------------ host side
 static buffalo_status d2h_i32(const int32_t* d, int32_t* h, cudaStream_t s) {
   BF_CUDA(cudaMemcpyAsync(h, d, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
@@ -364,43 +400,55 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     BF_CUDA(cudaStreamSynchronize(s));                             // sync 2: n_{l-1}
     n_src = n_dst + nn32;
   }
+  // from here on the graph workspace is dirty: an early return must restore it
+  auto restore_ws = [&]() -> buffalo_status {
+    if (n_dst > 0) {
+      k_reset_map<<<grid_for(n_dst, 256), 256, 0, s>>>(dst, n_dst, g->node_map);
+      BF_LAUNCHED("k_reset_map");
+    }
+    BF_CUDA(cudaMemsetAsync(gw.bits, 0, sizeof(uint32_t) * gw.words, s));
+    return BUFFALO_OK;
+  };
   int32_t* src = (int32_t*)A.take(4 * n_src);
-  if (A.overflow) return BUFFALO_ERR_CAPACITY;
+  if (A.overflow) {
+    BF_CHECK(restore_ws());
+    return BUFFALO_ERR_CAPACITY;
+  }
   if (n_dst > 0) BF_CUDA(cudaMemcpyAsync(src, dst, sizeof(int32_t) * n_dst, cudaMemcpyDeviceToDevice, s));
-  BF_CHECK(device_scan(PopcWord{gw.bits}, EmitWord{gw.bits, gw.prefix, src + n_dst, n_src - n_dst}, gw.words,
-                       gw.scan_ws, totals + 2, s));
+  BF_CHECK(device_scan(PopcWord{gw.bits}, StorePrefix{gw.prefix}, gw.words, gw.scan_ws, totals + 2, s));
+  k_emit_bits<<<grid_for(gw.words, 256), 256, 0, s>>>(gw.bits, gw.prefix, gw.words, src + n_dst, n_src - n_dst);
+  BF_LAUNCHED("k_emit_bits");
   blk->n_src = n_src;
   blk->src_global = src;
   blk->col_global = colg_persist;
+  const bool transpose = !sizes_only && layer >= 2;
+  int32_t *trp = nullptr, *tcol = nullptr, *tperm = nullptr;
+  if (transpose) {
+    trp = (int32_t*)A.take(4 * (n_src + 1));
+    tcol = (int32_t*)A.take(4 * e);
+    tperm = (int32_t*)A.take(4 * n_src);
+    if (A.overflow) {
+      BF_CHECK(restore_ws());
+      return BUFFALO_ERR_CAPACITY;
+    }
+    BF_CUDA(cudaMemsetAsync(trp, 0, sizeof(int32_t) * (n_src + 1), s));
+  }
   if (!sizes_only) {
     if (e > 0) {
       k_col_local<<<grid_for(e, 256), 256, 0, s>>>(colg, e, g->node_map, gw.bits, gw.prefix, (int32_t)n_dst,
-                                                   col_local);
+                                                   col_local, trp);
       BF_LAUNCHED("k_col_local");
     }
     blk->col_local = col_local;
   }
-  if (n_dst > 0) {
-    k_reset_map<<<grid_for(n_dst, 256), 256, 0, s>>>(dst, n_dst, g->node_map);
-    BF_LAUNCHED("k_reset_map");
-  }
-  BF_CUDA(cudaMemsetAsync(gw.bits, 0, sizeof(uint32_t) * gw.words, s));
+  BF_CHECK(restore_ws());
   blk->n_heavy_t = -1;
-  if (!sizes_only && layer >= 2) {
-    // transposed block: t_row_ptr by counting; t_col by an atomic-cursor fill followed by an
-    // ascending sort of every transposed row (entries are distinct dst indices, so the sorted
-    // row equals the stable order of the dst-ordered edges); degree classes of the src rows.
-    int32_t* trp = (int32_t*)A.take(4 * (n_src + 1));
-    int32_t* tcol = (int32_t*)A.take(4 * e);
-    int32_t* tperm = (int32_t*)A.take(4 * n_src);
-    if (A.overflow) return BUFFALO_ERR_CAPACITY;
+  if (transpose) {
+    // transposed block: t_row_ptr from the counts taken in k_col_local; t_col by an
+    // atomic-cursor fill followed by an ascending sort of every transposed row (entries are
+    // distinct dst indices, so the sorted row equals the stable order of the dst-ordered
+    // edges); degree classes of the src rows.
     int32_t* cursor = (int32_t*)q; q += R(4 * (n_dst + e));
-    k_fill_zero<<<grid_for(n_src + 1, 256), 256, 0, s>>>(trp, n_src + 1);
-    BF_LAUNCHED("k_fill_zero");
-    if (e > 0) {
-      k_tcount<<<grid_for(e, 256), 256, 0, s>>>(col_local, e, trp);
-      BF_LAUNCHED("k_tcount");
-    }
     BF_CHECK(scan_inplace(trp, n_src, ws, s));
     BF_CHECK(stable_partition(DegClass{trp}, EmitPerm{tperm}, n_src, counts, ws, s));
     int64_t nht = -1;
@@ -416,13 +464,25 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
       k_tfill<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(rp, col_local, n_dst, cursor, tcol);
       BF_LAUNCHED("k_tfill");
       if (n_src > 0) {
-        k_tsort_small<<<grid_for(n_src * 32, 256, 16), 256, 0, s>>>(tperm, n_src, trp, tcol);
-        BF_LAUNCHED("k_tsort_small");
+        k_tsort_banded<<<grid_for(n_src * 8, 256, 16), 256, 0, s>>>(tperm, trp, tcol, counts, part_tiles(n_src));
+        BF_LAUNCHED("k_tsort_banded");
       }
       const int hg = heavy_tail_grid(nht, e);
       if (hg > 0) {
-        k_tsort_heavy<<<hg, 256, 0, s>>>(tperm, n_src, trp, tcol, cursor);
-        BF_LAUNCHED("k_tsort_heavy");
+        const int64_t words = ceil_div(n_dst, 32);
+        if (words <= kBitsortMaxWords) {
+          static bool attr = false;
+          if (!attr) {
+            BF_CUDA(cudaFuncSetAttribute(k_tsort_heavy_bits, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         kBitsortMaxWords * 4));
+            attr = true;
+          }
+          k_tsort_heavy_bits<<<hg, 256, words * 4, s>>>(tperm, n_src, trp, tcol, (int32_t)words);
+          BF_LAUNCHED("k_tsort_heavy_bits");
+        } else {
+          k_tsort_heavy<<<hg, 256, 0, s>>>(tperm, n_src, trp, tcol, cursor);
+          BF_LAUNCHED("k_tsort_heavy");
+        }
       }
     }
     blk->t_row_ptr = trp;

@@ -165,8 +165,9 @@ inline buffalo_status scan_inplace(int32_t* a, int64_t n, int32_t* ws, cudaStrea
 }
 
 // ------------------------------------------------------------------ stable bin partition
-// Stable counting partition of n items into <= 256 bins (one LSD radix pass).
-constexpr int kPartThreads = 256;
+// Stable counting partition of n items into <= 256 bins (one LSD radix pass).  Tiles of
+// kPartTile items, one 1024-thread CTA each (four rounds of 1024 items per tile).
+constexpr int kPartThreads = 1024;
 constexpr int kPartTile = 4096;
 
 inline int64_t part_tiles(int64_t n) { return ceil_div(n > 0 ? n : 1, kPartTile); }
@@ -176,7 +177,7 @@ template <class Key>
 __global__ void __launch_bounds__(kPartThreads) k_part_hist(Key key, int64_t n, int32_t* counts,
                                                             int64_t ntiles) {
   __shared__ int32_t h[256];
-  h[threadIdx.x] = 0;
+  if (threadIdx.x < 256) h[threadIdx.x] = 0;
   __syncthreads();
   const int64_t t0 = (int64_t)blockIdx.x * kPartTile;
   for (int k = threadIdx.x; k < kPartTile; k += kPartThreads) {
@@ -184,7 +185,7 @@ __global__ void __launch_bounds__(kPartThreads) k_part_hist(Key key, int64_t n, 
     if (i < n) atomicAdd(&h[key(i)], 1);
   }
   __syncthreads();
-  counts[(int64_t)threadIdx.x * ntiles + blockIdx.x] = h[threadIdx.x];
+  if (threadIdx.x < 256) counts[(int64_t)threadIdx.x * ntiles + blockIdx.x] = h[threadIdx.x];
 }
 
 // emit(i, pos): item i goes to position pos (stable: input order inside a bin).
@@ -195,11 +196,10 @@ __global__ void __launch_bounds__(kPartThreads) k_part_scatter(Key key, Emit emi
   __shared__ int32_t base[256];
   __shared__ int32_t wcnt[NW][256];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  base[threadIdx.x] = offsets[(int64_t)threadIdx.x * ntiles + blockIdx.x];
+  if (threadIdx.x < 256) base[threadIdx.x] = offsets[(int64_t)threadIdx.x * ntiles + blockIdx.x];
   const int64_t t0 = (int64_t)blockIdx.x * kPartTile;
   for (int r = 0; r < kPartTile / kPartThreads; ++r) {
-#pragma unroll
-    for (int w = 0; w < NW; ++w) wcnt[w][threadIdx.x] = 0;
+    for (int k = threadIdx.x; k < NW * 256; k += kPartThreads) (&wcnt[0][0])[k] = 0;
     __syncthreads();
     const int64_t i = t0 + (int64_t)r * kPartThreads + threadIdx.x;
     const bool valid = i < n;
@@ -214,10 +214,12 @@ __global__ void __launch_bounds__(kPartThreads) k_part_scatter(Key key, Emit emi
       emit(i, off);
     }
     __syncthreads();
-    int32_t add = 0;
-#pragma unroll
-    for (int w = 0; w < NW; ++w) add += wcnt[w][threadIdx.x];
-    base[threadIdx.x] += add;
+    if (threadIdx.x < 256) {
+      int32_t add = 0;
+#pragma unroll 8
+      for (int w = 0; w < NW; ++w) add += wcnt[w][threadIdx.x];
+      base[threadIdx.x] += add;
+    }
     __syncthreads();
   }
 }
