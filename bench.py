@@ -40,8 +40,8 @@ WORKLOADS = {
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
-    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="arxiv", choices=list(WORKLOADS))
     ap.add_argument("--gemm", default="bf16", choices=["bf16", "ffma"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -121,63 +121,73 @@ def run_reference(args, cfg):
 
 # ----------------------------------------------------------------------------- clocks
 class Clocks:
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    """SM clock and throttle reasons sampled every 5 ms during the timed region (NVML in a
+    thread; nvidia-smi -lms 20 if NVML is unavailable)."""
+    REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+               "hw_power_brake_slowdown": 0x80, "sw_power_cap": 0x4}
 
     def __init__(self, index):
         self.index = index
-        self.p = None
+        self.samples, self.reasons, self.max_mhz = [], set(), 0.0
+        self.thread = self.proc = None
+        self.stop_flag = False
+
+    def _poll(self, nv, h):
+        while not self.stop_flag:
+            try:
+                self.samples.append(float(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+                for name, bit in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.005)
 
     def start(self):
         try:
-            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                                       "-i", str(self.index), "-lms", "200"], stdout=subprocess.PIPE,
-                                      stderr=subprocess.DEVNULL, text=True)
-        except OSError:
-            self.p = None
+            import threading
+            import pynvml as nv
+            nv.nvmlInit()
+            h = nv.nvmlDeviceGetHandleByIndex(self.index)
+            self.max_mhz = float(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM))
+            self.thread = threading.Thread(target=self._poll, args=(nv, h), daemon=True)
+            self.thread.start()
+        except Exception:
+            q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+            try:
+                self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                              "-i", str(self.index), "-lms", "20"], stdout=subprocess.PIPE,
+                                             stderr=subprocess.DEVNULL, text=True)
+            except OSError:
+                self.proc = None
 
     def stop(self):
-        if self.p is None:
+        if self.thread is not None:
+            self.stop_flag = True
+            self.thread.join()
+        elif self.proc is not None:
+            self.proc.terminate()
+            out, _ = self.proc.communicate()
+            names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+            for ln in out.strip().splitlines():
+                f = [x.strip() for x in ln.split(",")]
+                try:
+                    self.samples.append(float(f[0]))
+                    self.max_mhz = max(self.max_mhz, float(f[1]))
+                except (ValueError, IndexError):
+                    continue
+                for n, v in zip(names, f[2:6]):
+                    if v.lower() == "active":
+                        self.reasons.add(n)
+        if not self.samples:
             return None
-        self.p.terminate()
-        out, _ = self.p.communicate()
-        sm, mx, reasons = [], 0.0, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in out.strip().splitlines():
-            f = [x.strip() for x in ln.split(",")]
-            if len(f) < 9:
-                continue
-            try:
-                sm.append(float(f[1]))
-                mx = max(mx, float(f[2]))
-            except ValueError:
-                continue
-            for n, v in zip(names, f[5:9]):
-                if v.lower() == "active":
-                    reasons.add(n)
-        if not sm:
-            return None
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
-                "samples": len(sm)}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
 # ----------------------------------------------------------------------------- our arm
-def fwd_bytes(tr, groups_sizes, cfg, act_bytes, feat_bytes):
-    """Algorithmic bytes of the fused forward: per block edge one source row
-    + its 4-B index; per dst row_ptr, self row, saved h_agg and output row."""
-    from paper_conf_hpca_yangzl25_b200.buffalo import pitch
-    total = 0
-    for n, e in groups_sizes:
-        for l in range(1, cfg.L + 1):
-            s_in = feat_bytes if l == 1 else act_bytes
-            s_out = 4 if l == cfg.L else act_bytes
-            pin, pout = pitch(cfg.dims[l - 1]), pitch(cfg.dims[l])
-            total += e[l - 1] * (pin * s_in + 4)
-            total += n[l] * (4 + pin * s_in + pin * act_bytes + pout * s_out)
-    return total
-
-
 def run_ours(args, cfg):
     import torch
     rank, world, local = dist_env()
@@ -211,17 +221,7 @@ def run_ours(args, cfg):
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
 
-    fwd_events = []
-    orig_forward = tr.forward
-
-    def timed_forward():
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        orig_forward()
-        e1.record(stream)
-        fwd_events.append((e0, e1))
-
+    prof_counters = torch.zeros(1 << 16, dtype=torch.int64, device="cuda")
     lr = 0.01
     for i in range(args.warmup):
         tr.run_epoch(epoch=i, lr=lr)
@@ -230,7 +230,9 @@ def run_ours(args, cfg):
         torch.distributed.barrier()
     clocks = Clocks(local)
     clocks.start()
-    tr.forward = timed_forward
+    # live roofline of the dominant kernel (k_gather_rows, the Aggregate): CUDA events around
+    # each of its launches on its stream, algorithmic bytes from the edges it aggregated
+    B.profile_begin("gather", prof_counters)
     l0 = B.launch_count()
     step_ms, edges, sizes, ks = [], 0, [], []
     torch.cuda.synchronize()
@@ -253,14 +255,10 @@ def run_ours(args, cfg):
         torch.distributed.barrier()
     launches = B.launch_count() - l0
     clk = clocks.stop()
-    tr.forward = orig_forward
+    g_ms, g_launches, g_bytes = B.profile_end()
     total_ms = sum(step_ms)
-    fwd_ms = sum(a.elapsed_time(b) for a, b in fwd_events)
-    act_bytes = 2 if gemm == B.GEMM_BF16 else 4
-    fbytes = fwd_bytes(tr, sizes, cfg, act_bytes, 2 if feat_dtype == B.BF16 else 4)
-    n_fwd = len(fwd_events)
     if world > 1:
-        t = torch.tensor([total_ms, edges, fwd_ms, fbytes], dtype=torch.float64, device="cuda")
+        t = torch.tensor([total_ms, edges], dtype=torch.float64, device="cuda")
         mx = t.clone()
         torch.distributed.all_reduce(mx, op=torch.distributed.ReduceOp.MAX)
         sm = t.clone()
@@ -296,10 +294,10 @@ def run_ours(args, cfg):
 
     peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(peaks_path):
-        peak, peak_src = json.load(open(peaks_path))["hbm_gbs"], "measured (MEASURED_PEAKS.json hbm_gbs)"
+        peak, peak_src = json.load(open(peaks_path))["hbm_gbs"], "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
     else:
         peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
-    achieved = fbytes / (fwd_ms / 1e3) / 1e9 if fwd_ms > 0 else 0.0
+    achieved = g_bytes / (g_ms / 1e3) / 1e9 if g_ms > 0 else 0.0
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
@@ -317,11 +315,12 @@ def run_ours(args, cfg):
                     "gemm": args.gemm, "l2": "flushed (512 MiB write) between timed steps",
                     "epoch_ms": total_ms / args.steps, "edges_per_epoch": edges / args.steps,
                     "parallelism": f"dp{world} over bucket groups"},
-            roofline={"bound": "hbm", "kernel": "buffalo_sage_fwd (fused gather-mean + Update GEMM)",
+            roofline={"bound": "hbm", "kernel": "k_gather_rows (Aggregate: fwd neighbour mean, bwd transposed sum)",
                       "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                       "traffic": traffic, "peak_source": peak_src,
-                      "algorithmic_bytes_per_launch": fbytes / max(1, n_fwd),
-                      "launch_ms": fwd_ms / max(1, n_fwd), "share_of_step": fwd_ms / total_ms},
+                      "algorithmic_bytes_per_launch": g_bytes / max(1, g_launches),
+                      "launch_ms": g_ms / max(1, g_launches), "launches": g_launches,
+                      "share_of_step": g_ms / total_ms},
             cpu_baseline=cpu,
             e2e={"value": e2e_val, "unit": "edges/s", "h2d_bytes_per_step": 4 * len(seeds),
                  "d2h_bytes_per_step": 4},

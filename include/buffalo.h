@@ -245,6 +245,19 @@ BUFFALO_API buffalo_status buffalo_estimate_mem(int32_t num_layers, const int64_
 
 /* Number of kernels this thread has launched through the library (for bench accounting). */
 BUFFALO_API int64_t buffalo_launch_count(void);
+
+/* Diagnostics (bench roofline): time every launch of one kernel family with CUDA events on the
+ * stream it is launched on.  family "gather": k_gather_rows, the Aggregate of the forward (mean
+ * of neighbour rows) and of the backward (sum of dZ/D rows over the transposed block).
+ * counters: caller's device buffer of max_launches uint64 (edges each launch aggregated);
+ * launches beyond max_launches are not timed.  Not thread-safe; one family at a time.
+ * buffalo_profile_end synchronises the device and returns the summed launch time, the number of
+ * timed launches and their algorithmic bytes: per aggregated edge the 4-B index and the source
+ * row (pitch x element size), per row the 4-B permutation entry, two 4-B row_ptr reads and the
+ * bf16 output row. */
+BUFFALO_API buffalo_status buffalo_profile_begin(const char* family, void* counters, int64_t max_launches,
+                                     void* stream);
+BUFFALO_API buffalo_status buffalo_profile_end(double* ms_total_h, int64_t* launches_h, double* algo_bytes_h);
 BUFFALO_API const char* buffalo_status_str(buffalo_status s);
 BUFFALO_API const char* buffalo_last_error(void);
 

@@ -26,7 +26,8 @@ EXPORTS = [
     "buffalo_bucketize", "buffalo_build_blocks", "buffalo_packed_weight_bytes",
     "buffalo_pack_weights", "buffalo_sage_fwd", "buffalo_softmax_ce",
     "buffalo_sage_bwd_scratch_bytes", "buffalo_sage_bwd", "buffalo_sgd_step",
-    "buffalo_estimate_mem", "buffalo_launch_count", "buffalo_status_str", "buffalo_last_error",
+    "buffalo_estimate_mem", "buffalo_launch_count", "buffalo_profile_begin", "buffalo_profile_end",
+    "buffalo_status_str", "buffalo_last_error",
 ]
 
 
@@ -106,6 +107,8 @@ def lib(require_gpu=True):
             "buffalo_sgd_step": (c_i32, [P, P, c_i64, c_f, P]),
             "buffalo_estimate_mem": (c_i32, [c_i32, P, P, P, P, P]),
             "buffalo_launch_count": (c_i64, []),
+            "buffalo_profile_begin": (c_i32, [ctypes.c_char_p, P, c_i64, P]),
+            "buffalo_profile_end": (c_i32, [P, P, P]),
             "buffalo_status_str": (ctypes.c_char_p, [c_i32]),
             "buffalo_last_error": (ctypes.c_char_p, []),
         }
@@ -225,6 +228,18 @@ def estimate_mem(n, e, model):
 
 def launch_count():
     return lib(False).buffalo_launch_count()
+
+
+def profile_begin(family, counters, stream=None):
+    """Times every launch of a kernel family (diagnostic; counters: int64 CUDA tensor)."""
+    _check(lib().buffalo_profile_begin(family.encode(), ptr(counters), counters.numel(), stream_ptr(stream)))
+
+
+def profile_end():
+    """(summed launch ms, number of launches, algorithmic bytes) of the profiled family."""
+    ms, n, by = ctypes.c_double(0), c_i64(0), ctypes.c_double(0)
+    _check(lib().buffalo_profile_end(ctypes.byref(ms), ctypes.byref(n), ctypes.byref(by)))
+    return ms.value, n.value, by.value
 
 
 # ------------------------------------------------------------------------- struct helpers

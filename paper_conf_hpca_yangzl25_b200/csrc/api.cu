@@ -29,6 +29,41 @@ void set_error(const char* fmt, ...) {
 }
 void count_launch(int n) { g_launches += n; }
 
+// ------------------------------------------------------------------ kernel timing (diagnostic)
+namespace {
+struct Profiler {
+  bool on = false;
+  std::string family;
+  unsigned long long* counters = nullptr;   // caller's device buffer, one per launch
+  int64_t max_launches = 0;
+  std::vector<cudaEvent_t> ev;
+  std::vector<double> fixed, per_edge;
+};
+Profiler g_prof;
+}  // namespace
+
+ProfSlot prof_begin_launch(const char* family, cudaStream_t s) {
+  ProfSlot slot{nullptr, -1};
+  if (!g_prof.on || g_prof.family != family || (int64_t)g_prof.fixed.size() >= g_prof.max_launches) return slot;
+  slot.index = (int)g_prof.fixed.size();
+  slot.edges_dev = g_prof.counters + slot.index;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  g_prof.ev.push_back(a);
+  g_prof.ev.push_back(b);
+  g_prof.fixed.push_back(0.0);
+  g_prof.per_edge.push_back(0.0);
+  cudaEventRecord(a, s);
+  return slot;
+}
+void prof_end_launch(const ProfSlot& slot, cudaStream_t s, double fixed_bytes, double bytes_per_edge) {
+  if (slot.index < 0) return;
+  cudaEventRecord(g_prof.ev[2 * slot.index + 1], s);
+  g_prof.fixed[slot.index] = fixed_bytes;
+  g_prof.per_edge[slot.index] = bytes_per_edge;
+}
+
 buffalo_status check_cuda(const char* what) {
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) {
@@ -236,6 +271,42 @@ const char* buffalo_status_str(buffalo_status s) {
 
 const char* buffalo_last_error(void) { return g_err.c_str(); }
 int64_t buffalo_launch_count(void) { return g_launches.load(); }
+
+buffalo_status buffalo_profile_begin(const char* family, void* counters, int64_t max_launches, void* stream) {
+  if (!family || (std::string(family) != "gather") || !counters || max_launches <= 0) {
+    set_error("profile_begin: unknown kernel family or no counter buffer");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  for (cudaEvent_t e : g_prof.ev) cudaEventDestroy(e);
+  g_prof = Profiler();
+  g_prof.on = true;
+  g_prof.family = family;
+  g_prof.counters = (unsigned long long*)counters;
+  g_prof.max_launches = max_launches;
+  BF_CUDA(cudaMemsetAsync(counters, 0, sizeof(unsigned long long) * max_launches, (cudaStream_t)stream));
+  return BUFFALO_OK;
+}
+
+buffalo_status buffalo_profile_end(double* ms_total_h, int64_t* launches_h, double* algo_bytes_h) {
+  if (!g_prof.on) return BUFFALO_ERR_INVALID_ARG;
+  const int64_t n = (int64_t)g_prof.fixed.size();
+  std::vector<unsigned long long> edges(n > 0 ? n : 1, 0);
+  BF_CUDA(cudaDeviceSynchronize());
+  if (n > 0) BF_CUDA(cudaMemcpy(edges.data(), g_prof.counters, sizeof(unsigned long long) * n, cudaMemcpyDeviceToHost));
+  double ms = 0.0, bytes = 0.0;
+  for (int64_t i = 0; i < n; ++i) {
+    float t = 0.f;
+    BF_CUDA(cudaEventElapsedTime(&t, g_prof.ev[2 * i], g_prof.ev[2 * i + 1]));
+    ms += t;
+    bytes += g_prof.fixed[i] + g_prof.per_edge[i] * (double)edges[i];
+  }
+  if (ms_total_h) *ms_total_h = ms;
+  if (launches_h) *launches_h = n;
+  if (algo_bytes_h) *algo_bytes_h = bytes;
+  for (cudaEvent_t e : g_prof.ev) cudaEventDestroy(e);
+  g_prof = Profiler();
+  return BUFFALO_OK;
+}
 
 size_t buffalo_graph_workspace_bytes(int64_t num_nodes) { return (size_t)graph_ws_bytes(num_nodes); }
 

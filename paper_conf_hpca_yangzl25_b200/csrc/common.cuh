@@ -21,6 +21,16 @@ __host__ __device__ inline int64_t pitch_of(int64_t d) { return round_up(d, 8); 
 void set_error(const char* fmt, ...);
 void count_launch(int n = 1);
 
+// Live timing of one kernel family (buffalo_profile_begin/end): the launch site asks for a
+// slot; with one, it records CUDA events around the launch on its stream, passes the slot's
+// device counter (edges actually aggregated) and notes the launch's fixed and per-edge bytes.
+struct ProfSlot {
+  unsigned long long* edges_dev;   // null: not profiled
+  int index;
+};
+ProfSlot prof_begin_launch(const char* family, cudaStream_t s);
+void prof_end_launch(const ProfSlot& slot, cudaStream_t s, double fixed_bytes, double bytes_per_edge);
+
 // Returns BUFFALO_ERR_CUDA with the message if the last launch failed.
 buffalo_status check_cuda(const char* what);
 

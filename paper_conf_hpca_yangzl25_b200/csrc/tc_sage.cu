@@ -629,7 +629,7 @@ __global__ void __launch_bounds__(256, 8) k_gather_rows(const int32_t* __restric
                                                         const int32_t* __restrict__ col, int64_t n,
                                                         const TI* __restrict__ h, int64_t ldh, int pitch_in,
                                                         int lpr_log, __nv_bfloat16* __restrict__ out,
-                                                        int64_t ldo) {
+                                                        int64_t ldo, unsigned long long* __restrict__ edges_dev) {
   constexpr int E = InTraits<TI>::kElems;
   const int lane = threadIdx.x & 31;
   const int LPR = 1 << lpr_log, G = 32 / LPR;
@@ -648,6 +648,10 @@ __global__ void __launch_bounds__(256, 8) k_gather_rows(const int32_t* __restric
     const bool skip = row < 0 || D > kHeavyT;
     const int32_t Dl = skip ? 0 : D;
     const int32_t Dmax = __reduce_max_sync(0xffffffffu, Dl);
+    if (edges_dev) {                                    // profiling: edges this warp aggregates
+      const unsigned tot = __reduce_add_sync(0xffffffffu, pc == 0 ? (unsigned)Dl : 0u);
+      if (lane == 0 && tot) atomicAdd(edges_dev, (unsigned long long)tot);
+    }
     for (int p0 = 0; p0 < npieces; p0 += LPR) {
       const int piece = p0 + pc;
       const bool colok = piece < npieces;
@@ -707,8 +711,11 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   const int G = 32 >> lpr_log;
   const int64_t warps = ceil_div(n, G);
   const int grid = (int)std::min<int64_t>(ceil_div(warps, 8), 148LL * 8 * 4);
-  k_gather_rows<TI, MODE><<<grid, 256, 0, s>>>(perm, rp, col, n, h, ldh, pitch_in, lpr_log, out, ldo);
+  const ProfSlot ps = prof_begin_launch("gather", s);
+  k_gather_rows<TI, MODE><<<grid, 256, 0, s>>>(perm, rp, col, n, h, ldh, pitch_in, lpr_log, out, ldo, ps.edges_dev);
   BF_LAUNCHED(MODE == 0 ? "k_gather_mean" : "k_gather_sum");
+  // algorithmic bytes: per row perm + row_ptr pair + bf16 output row; per edge index + source row
+  prof_end_launch(ps, s, (double)n * (12.0 + 2.0 * pitch_in), 4.0 + (double)pitch_in * sizeof(TI));
   return BUFFALO_OK;
 }
 
