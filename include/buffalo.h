@@ -250,7 +250,7 @@ BUFFALO_API int64_t buffalo_launch_count(void);
  * stream it is launched on.  family "gather": k_gather_rows, the Aggregate of the forward (mean
  * of neighbour rows) and of the backward (sum of dZ/D rows over the transposed block).
  * counters: caller's device buffer of max_launches uint64 (edges each launch aggregated);
- * launches beyond max_launches are not timed.  Not thread-safe; one family at a time.
+ * launches beyond min(max_launches, 4096) are not timed.  Not thread-safe; one family at a time.
  * buffalo_profile_end synchronises the device and returns the summed launch time, the number of
  * timed launches and their algorithmic bytes: per aggregated edge the 4-B index and the source
  * row (pitch x element size), per row the 4-B permutation entry, two 4-B row_ptr reads and the

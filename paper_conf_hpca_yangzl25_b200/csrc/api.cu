@@ -45,16 +45,12 @@ Profiler g_prof;
 ProfSlot prof_begin_launch(const char* family, cudaStream_t s) {
   ProfSlot slot{nullptr, -1};
   if (!g_prof.on || g_prof.family != family || (int64_t)g_prof.fixed.size() >= g_prof.max_launches) return slot;
+  if (2 * g_prof.fixed.size() >= g_prof.ev.size()) return slot;   // event pool exhausted
   slot.index = (int)g_prof.fixed.size();
   slot.edges_dev = g_prof.counters + slot.index;
-  cudaEvent_t a, b;
-  cudaEventCreate(&a);
-  cudaEventCreate(&b);
-  g_prof.ev.push_back(a);
-  g_prof.ev.push_back(b);
   g_prof.fixed.push_back(0.0);
   g_prof.per_edge.push_back(0.0);
-  cudaEventRecord(a, s);
+  cudaEventRecord(g_prof.ev[2 * slot.index], s);
   return slot;
 }
 void prof_end_launch(const ProfSlot& slot, cudaStream_t s, double fixed_bytes, double bytes_per_edge) {
@@ -283,6 +279,9 @@ buffalo_status buffalo_profile_begin(const char* family, void* counters, int64_t
   g_prof.family = family;
   g_prof.counters = (unsigned long long*)counters;
   g_prof.max_launches = max_launches;
+  // events are created here, outside the timed region (at most 4096 timed launches)
+  g_prof.ev.resize(2 * std::min<int64_t>(max_launches, 4096));
+  for (cudaEvent_t& e : g_prof.ev) BF_CUDA(cudaEventCreate(&e));
   BF_CUDA(cudaMemsetAsync(counters, 0, sizeof(unsigned long long) * max_launches, (cudaStream_t)stream));
   return BUFFALO_OK;
 }
