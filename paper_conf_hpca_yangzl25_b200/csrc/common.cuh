@@ -99,6 +99,16 @@ struct Arena {
 __device__ __forceinline__ float bf2f(__nv_bfloat16 v) { return __bfloat162float(v); }
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 
+// a0 += low bf16 of w, a1 += high bf16 of w: one mixed-precision add per element
+// (add.rn.f32.bf16: exact widening of the bf16 half-register, one fp32 rounding), the same
+// result as widening then adding, at half the instructions.
+__device__ __forceinline__ void add_bf16x2(float& a0, float& a1, uint32_t w) {
+  asm("{\n\t.reg .b16 lo, hi;\n\tmov.b32 {lo, hi}, %2;\n\t"
+      "add.rn.f32.bf16 %0, lo, %0;\n\tadd.rn.f32.bf16 %1, hi, %1;\n\t}"
+      : "+f"(a0), "+f"(a1)
+      : "r"(w));
+}
+
 // Rows with more than kHeavyT entries sit at the tail of a degree-class permutation (stable
 // partition by min(D, kHeavyT + 1)).  Kernels over them walk the permutation from its end and
 // stop at the first light row, so they need no host-side count: the grid is the count when the

@@ -7,6 +7,8 @@
 // Update (Alg. 2 l.9): fp32 SIMT GEMM over [h_self || h_agg] (gemm_mode FFMA, the parity
 // path); the tensor-core path is in tc_sage.cu.
 #include "common.cuh"
+#include <type_traits>
+
 #include "sage.cuh"
 
 namespace buffalo {
@@ -135,7 +137,30 @@ __global__ void __launch_bounds__(256) k_agg_heavy(const int32_t* __restrict__ p
 #pragma unroll
     for (int k = 0; k < C; ++k) acc[k] = 0.f;
     if (c < nch) {
-      for (int32_t e = b + w; e < e_end; e += 8) {
+      int32_t e = b + w;
+      if constexpr (std::is_same<TI, __nv_bfloat16>::value && C == 8) {
+        for (; e + 24 < e_end; e += 32) {                // four rows in flight per lane
+          uint4 r[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) r[u] = __ldg(reinterpret_cast<const uint4*>(h + (int64_t)col[e + 8 * u] * ldh + c * C));
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            add_bf16x2(acc[0], acc[1], r[u].x); add_bf16x2(acc[2], acc[3], r[u].y);
+            add_bf16x2(acc[4], acc[5], r[u].z); add_bf16x2(acc[6], acc[7], r[u].w);
+          }
+        }
+      } else {
+        for (; e + 24 < e_end; e += 32) {
+          float v[4][C];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) VecIO<TI, C>::load(h + (int64_t)col[e + 8 * u] * ldh + c * C, v[u]);
+#pragma unroll
+          for (int u = 0; u < 4; ++u)
+#pragma unroll
+            for (int k = 0; k < C; ++k) acc[k] += v[u][k];
+        }
+      }
+      for (; e < e_end; e += 8) {
         float v[C];
         VecIO<TI, C>::load(h + (int64_t)col[e] * ldh + c * C, v);
 #pragma unroll

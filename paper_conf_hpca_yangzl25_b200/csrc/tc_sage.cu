@@ -211,6 +211,20 @@ template <> __device__ __forceinline__ void raw_to_f32<float>(const uint4& u, fl
   v[0] = __uint_as_float(u.x); v[1] = __uint_as_float(u.y); v[2] = __uint_as_float(u.z); v[3] = __uint_as_float(u.w);
 }
 
+// acc[k] += element k of a 16-B piece (bf16: add_bf16x2, common.cuh).
+template <class TI>
+__device__ __forceinline__ void acc_piece(float* acc, const uint4& u);
+template <> __device__ __forceinline__ void acc_piece<__nv_bfloat16>(float* acc, const uint4& u) {
+  add_bf16x2(acc[0], acc[1], u.x);
+  add_bf16x2(acc[2], acc[3], u.y);
+  add_bf16x2(acc[4], acc[5], u.z);
+  add_bf16x2(acc[6], acc[7], u.w);
+}
+template <> __device__ __forceinline__ void acc_piece<float>(float* acc, const uint4& u) {
+  acc[0] += __uint_as_float(u.x); acc[1] += __uint_as_float(u.y);
+  acc[2] += __uint_as_float(u.z); acc[3] += __uint_as_float(u.w);
+}
+
 // MODE 0: forward (mean of neighbour rows, long-tail rows pre-aggregated, h_agg saved,
 //         + bias, ReLU).  MODE 1: backward dH (plain sum of pre-scaled dZ/D rows over the
 //         transposed block, self half = dZ for rows < self_rows, fp32 output).
@@ -673,12 +687,7 @@ __global__ void __launch_bounds__(256, 8) k_gather_rows(const int32_t* __restric
               raw[uu] = __ldg(reinterpret_cast<const uint4*>(h + (int64_t)jn * ldh + col0));
           }
 #pragma unroll
-          for (int uu = 0; uu < kGU; ++uu) {
-            float v[E];
-            raw_to_f32<TI>(raw[uu], v);
-#pragma unroll
-            for (int k = 0; k < E; ++k) acc[k] += v[k];
-          }
+          for (int uu = 0; uu < kGU; ++uu) acc_piece<TI>(acc, raw[uu]);
         }
       }
       if (!skip && colok) {
@@ -1117,13 +1126,18 @@ __global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restric
     float acc[8];
 #pragma unroll
     for (int k = 0; k < 8; ++k) acc[k] = 0.f;
-    if (c < nch)
-      for (int32_t t = b + w; t < e_end; t += 8) {
-        float v[8];
-        bf16x8_to_f32(__ldg(reinterpret_cast<const uint4*>(z + (int64_t)col[t] * ldz + c * 8)), v);
+    if (c < nch) {
+      int32_t t = b + w;
+      for (; t + 24 < e_end; t += 32) {                  // four rows in flight per lane
+        uint4 r[4];
 #pragma unroll
-        for (int k = 0; k < 8; ++k) acc[k] += v[k];
+        for (int u = 0; u < 4; ++u) r[u] = __ldg(reinterpret_cast<const uint4*>(z + (int64_t)col[t + 8 * u] * ldz + c * 8));
+#pragma unroll
+        for (int u = 0; u < 4; ++u) acc_piece<__nv_bfloat16>(acc, r[u]);
       }
+      for (; t < e_end; t += 8)
+        acc_piece<__nv_bfloat16>(acc, __ldg(reinterpret_cast<const uint4*>(z + (int64_t)col[t] * ldz + c * 8)));
+    }
 #pragma unroll
     for (int k = 0; k < 8; ++k) part[w][lane][k] = acc[k];
     __syncthreads();
