@@ -177,20 +177,22 @@ struct Item {
   int64_t O, E, I, M, w;
 };
 
-// Item statistics (R13, R15): exact layer sizes of up to 64 items per pass (mask_stats), then
+constexpr int kStatsBatch = 256;       // items per statistics pass (mask_stats)
+
+// Item statistics (R13, R15): exact layer sizes of up to 256 items per pass (mask_stats), then
 // O = #seeds, E = e_L, I = n_{L-1} and M_est = hi of the memory model.
 static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_ids, std::vector<Item*>& items,
                                   const buffalo_sampler* sp, const buffalo_model* m, char* ws, int64_t ws_bytes,
                                   bool& masks_clean, cudaStream_t s) {
   const int L = m->num_layers;
-  for (size_t b0 = 0; b0 < items.size(); b0 += 64) {
-    const int nit = (int)std::min<size_t>(64, items.size() - b0);
-    int64_t starts[64], counts[64];
+  for (size_t b0 = 0; b0 < items.size(); b0 += kStatsBatch) {
+    const int nit = (int)std::min<size_t>(kStatsBatch, items.size() - b0);
+    int64_t starts[kStatsBatch], counts[kStatsBatch];
     for (int k = 0; k < nit; ++k) {
       starts[k] = items[b0 + k]->start;
       counts[k] = items[b0 + k]->count;
     }
-    static thread_local int64_t nh[64][BUFFALO_MAX_LAYERS + 1], eh[64][BUFFALO_MAX_LAYERS];
+    static thread_local int64_t nh[kStatsBatch][BUFFALO_MAX_LAYERS + 1], eh[kStatsBatch][BUFFALO_MAX_LAYERS];
     BF_CHECK(mask_stats(g, sorted_ids, starts, counts, nit, sp, L, ws, ws_bytes, masks_clean, nh, eh, s));
     masks_clean = true;
     for (int k = 0; k < nit; ++k) {
@@ -424,13 +426,13 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
       exploded = K >= 2 && (__int128)itF.M * K > (__int128)sum_M_all;   // R7
       if (exploded) {
         if (!have[K]) {
-          // batch this and the following candidates that will need a split (<= 64 pieces)
+          // batch this and the following candidates that will need a split (<= 256 pieces)
           std::vector<int> ks;
           int total = 0;
-          for (int K2 = K; K2 <= sc->k_max && (int)ks.size() < 64; ++K2) {
+          for (int K2 = K; K2 <= sc->k_max && total < kStatsBatch; ++K2) {
             if (!needs_split(K2)) continue;
             const int np = (int)std::min<int64_t>(K2, itF.count);
-            if (total + np > 64 && !ks.empty()) break;
+            if (total + np > kStatsBatch && !ks.empty()) break;
             ks.push_back(K2);
             total += np;
           }
@@ -520,14 +522,14 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
       // exact block sizes of every group (groups as items of the mask statistics), so that
       // buffalo_build_blocks can lay out the arena up front and run without host round trips
       const int W = 2 * L + 1;
-      for (int k0 = 0; k0 < gk; k0 += 64) {
-        const int nit = std::min(64, gk - k0);
-        int64_t st[64], ct[64];
+      for (int k0 = 0; k0 < gk; k0 += kStatsBatch) {
+        const int nit = std::min(kStatsBatch, gk - k0);
+        int64_t st[kStatsBatch], ct[kStatsBatch];
         for (int k = 0; k < nit; ++k) {
           st[k] = offs[k0 + k];
           ct[k] = offs[k0 + k + 1] - offs[k0 + k];
         }
-        static thread_local int64_t nh[64][BUFFALO_MAX_LAYERS + 1], eh[64][BUFFALO_MAX_LAYERS];
+        static thread_local int64_t nh[kStatsBatch][BUFFALO_MAX_LAYERS + 1], eh[kStatsBatch][BUFFALO_MAX_LAYERS];
         BF_CHECK(mask_stats(g, plan->group_seeds, st, ct, nit, sp, L, stats_ws, stats_bytes, masks_clean, nh, eh, s));
         masks_clean = true;
         for (int k = 0; k < nit; ++k) {

@@ -545,150 +545,221 @@ buffalo_status seed_bucketing(const buffalo_graph* g, const int32_t* seeds, int6
 }
 
 // ------------------------------------------------------------------ a2: item statistics
-// Block sizes of up to 64 items (disjoint seed sets) at once, by propagating item bitmasks
-// top-down: a node's mask at layer l-1 is the OR of the masks of the layer-l nodes that have it
-// as a dst (prefix) or a sampled neighbour.  Because a node's sample depends only on (seed,
-// node, hop) (R2), item k's node set at every layer is exactly the one of its own blocks, so
-// n_l(k) = #nodes with bit k, e_l(k) = sum of D over them — the sizes build_layer would give.
-__device__ __forceinline__ void mask_accumulate(uint64_t mask, int64_t D, unsigned long long* sn,
-                                                unsigned long long* se) {
-  while (mask) {
-    const int k = __ffsll((long long)mask) - 1;
-    mask &= mask - 1;
-    atomicAdd(&sn[k], 1ull);
-    if (se) atomicAdd(&se[k], (unsigned long long)D);
-  }
-}
+// Block sizes of up to 256 items (seed ranges, possibly overlapping) at once, by propagating
+// item bitmasks top-down: a node's mask at layer l-1 is the OR of the masks of the layer-l
+// nodes that have it as a dst (prefix) or a sampled neighbour.  Because a node's sample depends
+// only on (seed, node, hop) (R2), item k's node set at every layer is exactly the one of its own
+// blocks, so n_l(k) = #nodes with bit k, e_l(k) = sum of D over them — the sizes build_layer
+// would give.  A mask is W 64-bit words per node (W = 1, 2 or 4 by the item count); the nodes
+// of each layer are collected through the graph workspace's node bitmap (ascending ids).
 
 // Seed masks: position i (of the union range starting at base) gets the bit of every item
 // [start_k, end_k) that contains it (items of different K candidates overlap).
+template <int W>
 __global__ void __launch_bounds__(256) k_mask_seed(const int32_t* __restrict__ ids, int64_t base, int64_t n,
                                                    const int64_t* __restrict__ item_se, int nitems,
                                                    unsigned long long* __restrict__ m, int32_t* __restrict__ act) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t pos = base + i;
-    unsigned long long mask = 0;
+    unsigned long long mask[W];
+#pragma unroll
+    for (int w = 0; w < W; ++w) mask[w] = 0;
     for (int k = 0; k < nitems; ++k)
-      if (pos >= item_se[2 * k] && pos < item_se[2 * k + 1]) mask |= 1ull << k;
+      if (pos >= item_se[2 * k] && pos < item_se[2 * k + 1]) mask[k >> 6] |= 1ull << (k & 63);
     const int32_t v = ids[pos];
-    m[v] = mask;
+#pragma unroll
+    for (int w = 0; w < W; ++w) m[(int64_t)v * W + w] = mask[w];
     act[i] = v;
   }
 }
 
-// Appends u to the compacted list with one counter atomic per set of converged threads.
-__device__ __forceinline__ void append_aggregated(int32_t* __restrict__ list, int32_t* __restrict__ n, int32_t u) {
-  cg::coalesced_group grp = cg::coalesced_threads();
-  int32_t base = 0;
-  if (grp.thread_rank() == 0) base = atomicAdd(n, (int32_t)grp.size());
-  base = grp.shfl(base, 0);
-  list[base + (int32_t)grp.thread_rank()] = u;
-}
-
-// Per-item counters of a warp's nodes: lane k accumulates items k and k + 32 in registers; the
-// block's sums are flushed once at the end.
+// Per-item counters of a warp's nodes: lane k accumulates items k + 32 j (j < 2W) in registers;
+// the block's sums are flushed once at the end.
+template <int W>
 struct ItemCounters {
-  uint32_t n0 = 0, n1 = 0;
-  unsigned long long e0 = 0, e1 = 0;
+  uint32_t n[2 * W];
+  unsigned long long e[2 * W];
+  __device__ ItemCounters() {
+#pragma unroll
+    for (int j = 0; j < 2 * W; ++j) { n[j] = 0; e[j] = 0; }
+  }
 };
 
-__device__ __forceinline__ void flush_item_counters(const ItemCounters& c, unsigned long long* __restrict__ gn,
+template <int W>
+__device__ __forceinline__ void flush_item_counters(const ItemCounters<W>& c, unsigned long long* __restrict__ gn,
                                                     unsigned long long* __restrict__ ge,
                                                     unsigned long long* sn, unsigned long long* se) {
   const int lane = threadIdx.x & 31;
-  if (c.n0) atomicAdd(&sn[lane], (unsigned long long)c.n0);
-  if (c.n1) atomicAdd(&sn[lane + 32], (unsigned long long)c.n1);
-  if (ge) {
-    if (c.e0) atomicAdd(&se[lane], c.e0);
-    if (c.e1) atomicAdd(&se[lane + 32], c.e1);
+#pragma unroll
+  for (int j = 0; j < 2 * W; ++j) {
+    if (c.n[j]) atomicAdd(&sn[lane + 32 * j], (unsigned long long)c.n[j]);
+    if (ge && c.e[j]) atomicAdd(&se[lane + 32 * j], c.e[j]);
   }
   __syncthreads();
-  if (threadIdx.x < 64) {
-    if (sn[threadIdx.x]) atomicAdd(&gn[threadIdx.x], sn[threadIdx.x]);
-    if (ge && se[threadIdx.x]) atomicAdd(&ge[threadIdx.x], se[threadIdx.x]);
+  for (int k = threadIdx.x; k < 64 * W; k += blockDim.x) {
+    if (sn[k]) atomicAdd(&gn[k], sn[k]);
+    if (ge && se[k]) atomicAdd(&ge[k], se[k]);
   }
 }
 
+// ORs the nonzero words of mask into node u's mask and marks u in the layer's node bitmap.
+template <int W>
+__device__ __forceinline__ void mask_or(unsigned long long* __restrict__ m_out, uint32_t* __restrict__ bits, int32_t u,
+                                        const unsigned long long (&mask)[W]) {
+#pragma unroll
+  for (int w = 0; w < W; ++w)
+    if (mask[w]) atomicOr(&m_out[(int64_t)u * W + w], mask[w]);
+  const uint32_t b = 1u << (u & 31);
+  if (!(bits[u >> 5] & b)) atomicOr(&bits[u >> 5], b);
+}
+
 // One layer: 32/SEG active nodes of layer l per warp; accumulates n_l, e_l per item and ORs
-// each node's mask into layer l-1 for the node itself and its sampled neighbours, appending
-// first touches to act_out.
-template <int SEG>
+// each node's mask into layer l-1 for the node itself and its sampled neighbours.
+template <int SEG, int W>
 __global__ void __launch_bounds__(256) k_mask_layer(const int32_t* __restrict__ act, int64_t n_act,
                                                     const unsigned long long* __restrict__ m_in,
-                                                    unsigned long long* __restrict__ m_out,
-                                                    int32_t* __restrict__ act_out, int32_t* __restrict__ n_out,
+                                                    unsigned long long* __restrict__ m_out, uint32_t* __restrict__ bits,
                                                     const int64_t* __restrict__ grow, const int32_t* __restrict__ gcol,
                                                     int32_t f, uint32_t hop, uint64_t seed,
                                                     unsigned long long* __restrict__ gn, unsigned long long* __restrict__ ge) {
   constexpr int G = 32 / SEG;
-  __shared__ unsigned long long sn[64], se[64];
-  if (threadIdx.x < 64) { sn[threadIdx.x] = 0; se[threadIdx.x] = 0; }
+  __shared__ unsigned long long sn[64 * W], se[64 * W];
+  for (int k = threadIdx.x; k < 64 * W; k += blockDim.x) { sn[k] = 0; se[k] = 0; }
   __syncthreads();
   const int lane = threadIdx.x & 31, g = lane / SEG;
-  ItemCounters cnt;
+  ItemCounters<W> cnt;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
   for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n_act; w += warps) {
     const int64_t slot = w * G + g;
-    uint32_t v = 0;
-    unsigned long long mask = 0;
-    int64_t D = 0;
+    int32_t v = 0;
+    unsigned long long mask[W];
+#pragma unroll
+    for (int q = 0; q < W; ++q) mask[q] = 0;
+    int32_t D = 0;
     if (slot < n_act) {
-      v = (uint32_t)act[slot];
-      mask = m_in[v];
+      v = act[slot];
+#pragma unroll
+      for (int q = 0; q < W; ++q) mask[q] = m_in[(int64_t)v * W + q];
       const int64_t deg = grow[v + 1] - grow[v];
-      D = (f > 0 && deg > f) ? f : deg;
+      D = (int32_t)((f > 0 && deg > f) ? f : deg);
     }
 #pragma unroll
     for (int q = 0; q < G; ++q) {
-      const unsigned long long mq = __shfl_sync(0xffffffffu, mask, q * SEG);
-      const uint32_t Dq = (uint32_t)__shfl_sync(0xffffffffu, (int32_t)D, q * SEG);
-      if ((mq >> lane) & 1ull) { cnt.n0 += 1; cnt.e0 += Dq; }
-      if ((mq >> (lane + 32)) & 1ull) { cnt.n1 += 1; cnt.e1 += Dq; }
+      const uint32_t Dq = (uint32_t)__shfl_sync(0xffffffffu, D, q * SEG);
+#pragma unroll
+      for (int j = 0; j < 2 * W; ++j) {
+        const unsigned long long mq = __shfl_sync(0xffffffffu, mask[j >> 1], q * SEG);
+        if ((mq >> (lane + 32 * (j & 1))) & 1ull) { cnt.n[j] += 1; cnt.e[j] += Dq; }
+      }
     }
-    if (slot < n_act && (lane % SEG) == 0 && atomicOr(&m_out[v], mask) == 0ull)
-      append_aggregated(act_out, n_out, (int32_t)v);
+    if (slot < n_act && (lane % SEG) == 0) mask_or<W>(m_out, bits, v, mask);
     sample_warp_rows<SEG>(w, n_act, DstRows{act}, grow, gcol, f, hop, seed, [&](int64_t s_, int32_t, int32_t u) {
-      const unsigned long long ms = m_in[act[s_]];
-      if (atomicOr(&m_out[u], ms) == 0ull) append_aggregated(act_out, n_out, u);
+      unsigned long long ms[W];
+#pragma unroll
+      for (int q = 0; q < W; ++q) ms[q] = m_in[(int64_t)act[s_] * W + q];
+      mask_or<W>(m_out, bits, u, ms);
     });
   }
-  flush_item_counters(cnt, gn, ge, sn, se);
+  flush_item_counters<W>(cnt, gn, ge, sn, se);
 }
 
 // Clears the masks of the active list; with gn, first counts per item how many active nodes
 // carry its bit (one ballot per item bit, counted in registers).
+template <int W>
 __global__ void __launch_bounds__(256) k_mask_count(const int32_t* __restrict__ act, int64_t n_act,
                                                     unsigned long long* __restrict__ m,
-                                                    unsigned long long* __restrict__ gn, int clear) {
-  __shared__ unsigned long long sn[64];
-  if (threadIdx.x < 64) sn[threadIdx.x] = 0;
+                                                    unsigned long long* __restrict__ gn) {
+  __shared__ unsigned long long sn[64 * W];
+  for (int k = threadIdx.x; k < 64 * W; k += blockDim.x) sn[k] = 0;
   __syncthreads();
   const int lane = threadIdx.x & 31;
-  ItemCounters cnt;
+  ItemCounters<W> cnt;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i0 = blockIdx.x * (int64_t)blockDim.x; i0 < n_act; i0 += stride) {
     const int64_t i = i0 + threadIdx.x;
-    unsigned long long mask = 0;
+    unsigned long long mask[W];
+#pragma unroll
+    for (int q = 0; q < W; ++q) mask[q] = 0;
     if (i < n_act) {
       const int32_t v = act[i];
-      mask = m[v];
-      if (clear) m[v] = 0ull;
+#pragma unroll
+      for (int q = 0; q < W; ++q) {
+        mask[q] = m[(int64_t)v * W + q];
+        m[(int64_t)v * W + q] = 0ull;
+      }
     }
     if (gn) {
-      const unsigned lo = (unsigned)mask, hi = (unsigned)(mask >> 32);
 #pragma unroll
-      for (int k = 0; k < 32; ++k) {
-        const unsigned b0 = __ballot_sync(0xffffffffu, (lo >> k) & 1u);
-        const unsigned b1 = __ballot_sync(0xffffffffu, (hi >> k) & 1u);
-        if (lane == k) { cnt.n0 += __popc(b0); cnt.n1 += __popc(b1); }
+      for (int j = 0; j < 2 * W; ++j) {
+        const unsigned word = (unsigned)(mask[j >> 1] >> (32 * (j & 1)));
+#pragma unroll
+        for (int k = 0; k < 32; ++k) {
+          const unsigned b = __ballot_sync(0xffffffffu, (word >> k) & 1u);
+          if (lane == k) cnt.n[j] += __popc(b);
+        }
       }
     }
   }
-  if (gn) flush_item_counters(cnt, gn, nullptr, sn, nullptr);
+  if (gn) flush_item_counters<W>(cnt, gn, nullptr, sn, nullptr);
 }
 
+constexpr int kMaskMaxItems = 256;
+constexpr int kMaskMaxW = kMaskMaxItems / 64;
+
 int64_t mask_stats_bytes(int64_t N, int L) {
-  return 2 * R(8 * N) + 2 * R(4 * N) + R(8 * 64 * (2 * L + 1)) + R(64) + R(16 * 64);
+  return 2 * R(8 * kMaskMaxW * N) + 2 * R(4 * N) + R(8 * kMaskMaxItems * (2 * L + 1)) + R(64) +
+         R(16 * kMaskMaxItems);
+}
+
+template <int W>
+static buffalo_status mask_stats_w(const buffalo_graph* g, const int32_t* sorted_ids, int64_t lo_pos, int64_t n_seed,
+                                   const int64_t* se, int nitems, const buffalo_sampler* sp, int L,
+                                   unsigned long long* const* m, int32_t* const* act, unsigned long long* accn,
+                                   unsigned long long* acce, cudaStream_t s) {
+  const GraphWs gw = graph_ws(g);
+  if (n_seed > 0) {
+    k_mask_seed<W><<<grid_for(n_seed, 256), 256, 0, s>>>(sorted_ids, lo_pos, n_seed, se, nitems, m[0], act[0]);
+    BF_LAUNCHED("k_mask_seed");
+  }
+  int64_t n_act = n_seed;
+  int cur = 0;
+  int32_t* total = gw.prefix + gw.words;          // the prefix array's spare last element
+  for (int l = L; l >= 1; --l) {
+    int32_t na = 0;
+    if (n_act > 0) {
+      const int32_t fl = sp->fanout[l - 1];
+      const int seg = sample_seg(fl);
+      const int grid = grid_for(ceil_div(n_act, 32 / seg) * 32, 256, 16);
+      const uint32_t hop = (uint32_t)(L - l + 1);
+      if (seg == 8)
+        k_mask_layer<8, W><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], gw.bits, g->row_ptr, g->col, fl,
+                                               hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1));
+      else if (seg == 16)
+        k_mask_layer<16, W><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], gw.bits, g->row_ptr, g->col, fl,
+                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1));
+      else
+        k_mask_layer<32, W><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], gw.bits, g->row_ptr, g->col, fl,
+                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1));
+      BF_LAUNCHED("k_mask_layer");
+      // masks of layer l are no longer needed: clear them for reuse by layer l-2
+      k_mask_count<W><<<grid_for(n_act, 256), 256, 0, s>>>(act[cur], n_act, m[cur], nullptr);
+      BF_LAUNCHED("k_mask_count");
+      // layer l-1's nodes, ascending: popcount scan of the node bitmap, emit, clear
+      BF_CHECK(device_scan(PopcWord{gw.bits}, StorePrefix{gw.prefix}, gw.words, gw.scan_ws, total, s));
+      k_emit_bits<<<grid_for(gw.words, 256), 256, 0, s>>>(gw.bits, gw.prefix, gw.words, act[cur ^ 1], g->num_nodes);
+      BF_LAUNCHED("k_emit_bits");
+      BF_CUDA(cudaMemsetAsync(gw.bits, 0, sizeof(uint32_t) * gw.words, s));
+      BF_CUDA(cudaMemcpyAsync(&na, total, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+      BF_CUDA(cudaStreamSynchronize(s));
+    }
+    n_act = na;
+    cur ^= 1;
+  }
+  if (n_act > 0) {
+    k_mask_count<W><<<grid_for(n_act, 256), 256, 0, s>>>(act[cur], n_act, m[cur], accn);
+    BF_LAUNCHED("k_mask_count");
+  }
+  return BUFFALO_OK;
 }
 
 buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, const int64_t* item_start_h,
@@ -701,19 +772,25 @@ buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, con
     set_error("bucketize workspace too small for the item statistics");
     return BUFFALO_ERR_CAPACITY;
   }
+  if (nitems < 1 || nitems > kMaskMaxItems) {
+    set_error("mask_stats: %d items (1..%d)", nitems, kMaskMaxItems);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  const int W = nitems <= 64 ? 1 : nitems <= 128 ? 2 : 4;
   char* q = ws;
-  unsigned long long* m[2] = {(unsigned long long*)q, (unsigned long long*)(q + R(8 * N))};
-  q += 2 * R(8 * N);
+  unsigned long long* m[2] = {(unsigned long long*)q, (unsigned long long*)(q + R(8 * kMaskMaxW * N))};
+  q += 2 * R(8 * kMaskMaxW * N);
   int32_t* act[2] = {(int32_t*)q, (int32_t*)(q + R(4 * N))};
   q += 2 * R(4 * N);
-  unsigned long long* acc = (unsigned long long*)q; q += R(8 * 64 * (2 * L + 1));
-  int32_t* cnt = (int32_t*)q; q += R(64);
+  unsigned long long* acc = (unsigned long long*)q; q += R(8 * kMaskMaxItems * (2 * L + 1));
+  q += R(64);
   int64_t* se = (int64_t*)q;
   if (!masks_clean) {
-    BF_CUDA(cudaMemsetAsync(m[0], 0, 2 * R(8 * N), s));
+    BF_CUDA(cudaMemsetAsync(m[0], 0, 2 * R(8 * kMaskMaxW * N), s));
   }
-  BF_CUDA(cudaMemsetAsync(acc, 0, sizeof(unsigned long long) * 64 * (2 * L + 1), s));
-  int64_t se_h[128];
+  const int stride = 64 * W;                      // items per accumulator row
+  BF_CUDA(cudaMemsetAsync(acc, 0, sizeof(unsigned long long) * stride * (2 * L + 1), s));
+  int64_t se_h[2 * kMaskMaxItems];
   int64_t lo_pos = INT64_MAX, hi_pos = 0;
   for (int k = 0; k < nitems; ++k) {
     se_h[2 * k] = item_start_h[k];
@@ -726,53 +803,21 @@ buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, con
   if (lo_pos > hi_pos) lo_pos = hi_pos = 0;
   BF_CUDA(cudaMemcpyAsync(se, se_h, sizeof(int64_t) * 2 * nitems, cudaMemcpyHostToDevice, s));
   const int64_t n_seed = hi_pos - lo_pos;
-  // acc layout: n[l] at acc + 64*l (l = 0..L), e[l-1] at acc + 64*(L+1) + 64*(l-1)
+  // acc layout: n[l] at acc + stride*l (l = 0..L), e[l-1] at acc + stride*(L+1) + stride*(l-1)
   unsigned long long* accn = acc;
-  unsigned long long* acce = acc + 64 * (L + 1);
-  if (n_seed > 0) {
-    k_mask_seed<<<grid_for(n_seed, 256), 256, 0, s>>>(sorted_ids, lo_pos, n_seed, se, nitems, m[0], act[0]);
-    BF_LAUNCHED("k_mask_seed");
-  }
-  int64_t n_act = n_seed;
-  int cur = 0;
-  for (int l = L; l >= 1; --l) {
-    BF_CUDA(cudaMemsetAsync(cnt, 0, sizeof(int32_t), s));
-    if (n_act > 0) {
-      const int32_t fl = sp->fanout[l - 1];
-      const int seg = sample_seg(fl);
-      const int grid = grid_for(ceil_div(n_act, 32 / seg) * 32, 256, 16);
-      if (seg == 8)
-        k_mask_layer<8><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], act[cur ^ 1], cnt, g->row_ptr, g->col,
-                                            fl, (uint32_t)(L - l + 1), sp->seed, accn + 64 * l, acce + 64 * (l - 1));
-      else if (seg == 16)
-        k_mask_layer<16><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], act[cur ^ 1], cnt, g->row_ptr,
-                                             g->col, fl, (uint32_t)(L - l + 1), sp->seed, accn + 64 * l,
-                                             acce + 64 * (l - 1));
-      else
-        k_mask_layer<32><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], act[cur ^ 1], cnt, g->row_ptr,
-                                             g->col, fl, (uint32_t)(L - l + 1), sp->seed, accn + 64 * l,
-                                             acce + 64 * (l - 1));
-      BF_LAUNCHED("k_mask_layer");
-      // masks of layer l are no longer needed: clear them for reuse by layer l-2
-      k_mask_count<<<grid_for(n_act, 256), 256, 0, s>>>(act[cur], n_act, m[cur], nullptr, 1);
-      BF_LAUNCHED("k_mask_count");
-    }
-    int32_t na = 0;
-    BF_CUDA(cudaMemcpyAsync(&na, cnt, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-    BF_CUDA(cudaStreamSynchronize(s));
-    n_act = na;
-    cur ^= 1;
-  }
-  if (n_act > 0) {
-    k_mask_count<<<grid_for(n_act, 256), 256, 0, s>>>(act[cur], n_act, m[cur], accn, 1);
-    BF_LAUNCHED("k_mask_count");
-  }
-  unsigned long long host[64 * (2 * BUFFALO_MAX_LAYERS + 1)];
-  BF_CUDA(cudaMemcpyAsync(host, acc, sizeof(unsigned long long) * 64 * (2 * L + 1), cudaMemcpyDeviceToHost, s));
+  unsigned long long* acce = acc + stride * (L + 1);
+  if (W == 1)
+    BF_CHECK(mask_stats_w<1>(g, sorted_ids, lo_pos, n_seed, se, nitems, sp, L, m, act, accn, acce, s));
+  else if (W == 2)
+    BF_CHECK(mask_stats_w<2>(g, sorted_ids, lo_pos, n_seed, se, nitems, sp, L, m, act, accn, acce, s));
+  else
+    BF_CHECK(mask_stats_w<4>(g, sorted_ids, lo_pos, n_seed, se, nitems, sp, L, m, act, accn, acce, s));
+  static thread_local unsigned long long host[kMaskMaxItems * (2 * BUFFALO_MAX_LAYERS + 1)];
+  BF_CUDA(cudaMemcpyAsync(host, acc, sizeof(unsigned long long) * stride * (2 * L + 1), cudaMemcpyDeviceToHost, s));
   BF_CUDA(cudaStreamSynchronize(s));
   for (int k = 0; k < nitems; ++k) {
-    for (int l = 0; l <= L; ++l) n_h[k][l] = (int64_t)host[64 * l + k];
-    for (int l = 1; l <= L; ++l) e_h[k][l - 1] = (int64_t)host[64 * (L + 1) + 64 * (l - 1) + k];
+    for (int l = 0; l <= L; ++l) n_h[k][l] = (int64_t)host[stride * l + k];
+    for (int l = 1; l <= L; ++l) e_h[k][l - 1] = (int64_t)host[stride * (L + 1) + stride * (l - 1) + k];
   }
   return BUFFALO_OK;
 }

@@ -51,9 +51,10 @@ buffalo_status seed_bucketing(const buffalo_graph* g, const int32_t* seeds, int6
                               int32_t* counts, int32_t* ws, int32_t* starts_dev, int64_t* hist_h,
                               cudaStream_t s);
 
-// Exact per-item block sizes (n[0..L], e[0..L-1]) of up to 64 items (they may overlap): item k
-// is sorted_ids[item_start_h[k] .. + item_count_h[k]).  ws: mask_stats_bytes(N, L) bytes; the
-// masks are left zeroed (masks_clean = true on the next call saves a memset).
+// Exact per-item block sizes (n[0..L], e[0..L-1]) of up to 256 items (they may overlap): item
+// k is sorted_ids[item_start_h[k] .. + item_count_h[k]).  ws: mask_stats_bytes(N, L) bytes; the
+// masks are left zeroed (masks_clean = true on the next call saves a memset).  Uses (and
+// leaves cleared) the graph workspace's node bitmap.  Synchronises once per layer.
 int64_t mask_stats_bytes(int64_t N, int L);
 buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, const int64_t* item_start_h,
                           const int64_t* item_count_h, int nitems, const buffalo_sampler* sp, int L, char* ws,

@@ -127,8 +127,11 @@ class Trainer:
         return K, self.offs_h[:K + 1].copy(), self.est_h[:K].copy(), self.rank_h[:K].copy()
 
     def _ensure_arena(self, nbytes):
+        """Grows the micro-batch arena (with 1/8 headroom, so that the need drifting between
+        epochs does not reallocate it every time)."""
         if self.arena.numel() < nbytes:
-            self.arena = torch.empty(int(nbytes), dtype=torch.uint8, device=self.device)
+            self.arena = None
+            self.arena = torch.empty(int(nbytes + nbytes // 8), dtype=torch.uint8, device=self.device)
 
     def build(self, off, n, sampler, sizes=None):
         """Blocks of the group at group_seeds[off:off+n]; sizes = its row of the plan's exact

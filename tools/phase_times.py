@@ -48,8 +48,10 @@ def main():
         K, offs, est, ranks = tr.schedule(ep)
         e1 = ev()
         L = tr.L
+        ea = ev()
         tr._ensure_arena(max(B.estimate_mem(tr.sizes_h[k, :L + 1], tr.sizes_h[k, L + 1:], tr.model)[0]
                              for k in range(K)))
+        eb = ev()
         sampler = tr.sampler(ep)
         marks = []
         hb = hf = hk = 0.0
@@ -69,6 +71,7 @@ def main():
         wall = (time.perf_counter() - w0) * 1e3
         if ep >= 2:
             add("schedule", e0, e1)
+            add("arena", ea, eb)
             for a, b, c, d, e in marks:
                 add("build", a, b); add("fwd", b, c); add("loss", c, d); add("bwd", d, e)
             add("step", s0, s1)
