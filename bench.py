@@ -7,7 +7,10 @@ bucketize (Alg. 3/4 + Eq. 1-2) + for every own bucket group: block generation, L
 SAGE-mean forward layers, loss, L backward layers + NCCL gradient allreduce (N > 1) + SGD.
 value = aggregated block edges of all ranks / max-over-ranks device time (edges/s).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config arxiv|cora|products]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config products|arxiv|cora]
+
+The default workload is BASELINE.json configs[2] (products-shaped, fixed memory budget, the
+config the metric is quoted on at 1/2/4/8 GPUs); arxiv and Cora are selectable.
                   [--gemm bf16|ffma] [--impl ours|reference]
 
 Under torchrun (N > 1) every rank runs its own groups (k_min = N, LPT by estimate).
@@ -42,7 +45,7 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=30)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--config", default="arxiv", choices=list(WORKLOADS))
+    ap.add_argument("--config", default="products", choices=list(WORKLOADS))
     ap.add_argument("--gemm", default="bf16", choices=["bf16", "ffma"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-baseline-seconds", type=float, default=20.0)
@@ -55,6 +58,24 @@ def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     return rank, world, local
+
+
+def make_inputs_device(cfg):
+    """The same inputs as make_inputs, generated on the GPU by synth.device (bit-identical to
+    the numpy recipe; a products-shaped graph takes seconds instead of minutes on one core)."""
+    import torch
+    from synth import device as SD
+    rp, col = SD.random_graph(cfg.N, cfg.pairs, cfg.kind)
+    X = SD.features(cfg.N, cfg.d0, ((cfg.d0 + 31) // 32) * 32)
+    y = SD.labels(cfg.N, cfg.classes)
+    seeds = SD.seed_nodes(cfg.N, cfg.S)
+    Ws, bs = xavier_weights(cfg.dims)
+    torch.cuda.synchronize()
+    return rp, col, X, y, seeds, Ws, bs
+
+
+def host_copies(*ts):
+    return [t.cpu().numpy() if hasattr(t, "cpu") else t for t in ts]
 
 
 def make_inputs(cfg):
@@ -95,10 +116,20 @@ def run_reference(args, cfg):
     rank, world, _ = dist_env()
     if rank != 0:
         return
-    rp, col, X, y, seeds, Ws, bs = make_inputs(cfg)
+    try:
+        import torch
+        on_gpu = torch.cuda.is_available()
+    except ImportError:
+        on_gpu = False
+    if on_gpu:       # same inputs, generated on the device (synth.device), then copied to the host
+        rp, col, X, y, seeds, Ws, bs = make_inputs_device(cfg)
+        rp, col, X, y, seeds = host_copies(rp, col, X, y, seeds)
+    else:
+        rp, col, X, y, seeds, Ws, bs = make_inputs(cfg)
     import oracle as O
     g = O.Graph(rp, col)
-    part = seeds[: max(1, len(seeds) // 16)]
+    # bounded sample per step (~1-5 s of oracle work; 35 steps end within a few minutes)
+    part = seeds[: max(1, len(seeds) // {"products": 150, "cora": 1}.get(args.config, 16))]
     times, edges = [], 0
     for i in range(args.warmup + args.steps):
         t = time.perf_counter()
@@ -197,23 +228,26 @@ def run_ours(args, cfg):
         torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local))
         pg = torch.distributed.group.WORLD
     from paper_conf_hpca_yangzl25_b200 import buffalo as B
-    from paper_conf_hpca_yangzl25_b200.train import Trainer
+    from paper_conf_hpca_yangzl25_b200.train import DeviceGraph, Trainer
 
     B.lib()
-    rp, col, X, y, seeds, Ws, bs = make_inputs(cfg)
+    t_gen = time.perf_counter()
+    rp, col, X, y, seeds, Ws, bs = make_inputs_device(cfg)
+    t_gen = time.perf_counter() - t_gen
     gemm = B.GEMM_BF16 if args.gemm == "bf16" else B.GEMM_FFMA
     feat_dtype = B.BF16 if args.gemm == "bf16" else B.FP32
-    feats = torch.as_tensor(X).cuda()
+    feats = X
     if feat_dtype == B.BF16:
         feats = feats.to(torch.bfloat16).contiguous()      # k/128 features are exact in bf16
     kmin = max(cfg.k_min, world)
     budget = cfg.mem_budget
-    tr = Trainer((rp, col), feats, torch.as_tensor(y).cuda(), torch.as_tensor(seeds).cuda(), cfg.dims,
+    graph = DeviceGraph(rp, col)
+    tr = Trainer(graph, feats, y, seeds, cfg.dims,
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, mem_budget=budget,
                  k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg)
     if args.config == "products":
         # calibrate M_ctr once so that one GPU needs >= 8 groups, then freeze it for every N
-        B_full = Trainer((rp, col), feats, torch.as_tensor(y).cuda(), torch.as_tensor(seeds).cuda(), cfg.dims,
+        B_full = Trainer(graph, feats, y, seeds, cfg.dims,
                          cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, k_min=1, k_max=1)
         _, _, est1, _ = B_full.schedule(0)
         del B_full
@@ -268,7 +302,7 @@ def run_ours(args, cfg):
 
     # end to end through the public API with host buffers: H2D of the step's seed batch from
     # pinned memory, D2H of the loss, copies inside the timed region
-    seeds_h = torch.as_tensor(seeds).pin_memory()
+    seeds_h = seeds.cpu().pin_memory()
     loss_h = torch.empty(1, dtype=torch.float32).pin_memory()
     e2e_ms, e2e_edges = [], 0
     for i in range(max(1, args.steps)):
@@ -305,7 +339,8 @@ def run_ours(args, cfg):
     if rank == 0:
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
-            cpu = oracle_sample(cfg, rp, col, X, y, seeds, Ws, bs, args.cpu_baseline_seconds)
+            rp_h, col_h, X_h, y_h, seeds_h = host_copies(rp, col, X, y, tr.seeds)
+            cpu = oracle_sample(cfg, rp_h, col_h, X_h, y_h, seeds_h, Ws, bs, args.cpu_baseline_seconds)
         line = dict(
             metric="aggregated edges/s (epoch of Buffalo hot path)", value=value, unit="edges/s",
             n_gpus=world, steps=args.steps, warmup=args.warmup, ms_per_step=total_ms / args.steps,

@@ -281,8 +281,8 @@ buffalo_status buffalo_profile_begin(const char* family, void* counters, int64_t
   g_prof.family = family;
   g_prof.counters = (unsigned long long*)counters;
   g_prof.max_launches = max_launches;
-  // events are created here, outside the timed region (at most 4096 timed launches)
-  g_prof.ev.resize(2 * std::min<int64_t>(max_launches, 4096));
+  // events are created here, outside the timed region (at most 16384 timed launches)
+  g_prof.ev.resize(2 * std::min<int64_t>(max_launches, 16384));
   for (cudaEvent_t& e : g_prof.ev) BF_CUDA(cudaEventCreate(&e));
   BF_CUDA(cudaMemsetAsync(counters, 0, sizeof(unsigned long long) * max_launches, (cudaStream_t)stream));
   return BUFFALO_OK;

@@ -630,81 +630,127 @@ buffalo_status launch_agg_heavy_bf16(const FwdArgs& a, cudaStream_t s);
 
 
 // ================================================================== high-occupancy gather
-// Aggregate (Alg. 2 l.8) as its own kernel: lane groups of LPR lanes (16 B each) own one row,
-// rows taken in degree-sorted order (perm) so a warp's rows have equal trip counts; indices of
-// a row are fetched LPR at a time and broadcast with shuffles, kU 16-B loads stay in flight per
-// lane; fp32 accumulation; MODE 0: mean (R21), MODE 1: plain sum (backward, dZ/D rows).
-// Rows with D > kHeavyT are skipped (pre-aggregated by the cooperative kernels).
-constexpr int kGU = 4;
-
-template <class TI, int MODE>
-__global__ void __launch_bounds__(256, 8) k_gather_rows(const int32_t* __restrict__ perm,
-                                                        const int32_t* __restrict__ rp,
-                                                        const int32_t* __restrict__ col, int64_t n,
-                                                        const TI* __restrict__ h, int64_t ldh, int pitch_in,
-                                                        int lpr_log, __nv_bfloat16* __restrict__ out,
-                                                        int64_t ldo, unsigned long long* __restrict__ edges_dev) {
+// Aggregate kernel used by launch_gather.  Lane groups of LPR lanes (one 16-B piece each,
+// LPR a compile-time power of two covering the row) own one row each, rows taken in the
+// degree-class order so the G = 32/LPR rows of a warp have (nearly) equal trip counts.  Per
+// chunk of LPR edges every lane fetches one column index, then the group issues kU 16-B row
+// loads per lane at once (indices broadcast by shuffles, -1 marks an absent edge).  Written for
+// few instructions per loaded byte (the earlier row kernel ran ~75 instructions per 16-B load
+// and was issue-bound): compile-time lane geometry, no spills (<= 40 registers, 48 warps per
+// SM), and the next row's perm / row_ptr entries fetched one iteration ahead so short rows do
+// not pay the whole perm -> row_ptr -> col -> row dependency chain each.  MODE 0 writes the
+// mean as x * (1/D) corrected by one FMA residual step (Markstein), MODE 1 the plain sum; the
+// per-row sum order is the CSR order (R21).
+template <class TI, int MODE, int LPR, int kU, int MINB>
+__global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restrict__ perm,
+                                                         const int32_t* __restrict__ rp,
+                                                         const int32_t* __restrict__ col, int32_t n,
+                                                         const TI* __restrict__ h, int32_t ldb, int npieces,
+                                                         __nv_bfloat16* __restrict__ out, int64_t ldo,
+                                                         unsigned long long* __restrict__ edges_dev) {
   constexpr int E = InTraits<TI>::kElems;
+  constexpr int G = 32 / LPR;
+  constexpr unsigned kFull = 0xffffffffu;
   const int lane = threadIdx.x & 31;
-  const int LPR = 1 << lpr_log, G = 32 / LPR;
-  const int g = lane >> lpr_log, pc = lane & (LPR - 1);
-  const int npieces = (pitch_in + E - 1) / E;
-  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n; w += warps) {
-    const int64_t pos = w * G + g;
-    int64_t row = -1;
-    int32_t b = 0, D = 0;
+  const int g = lane / LPR, pc = lane & (LPR - 1);
+  const int gbase = g * LPR;
+  const int32_t warps = (int32_t)(gridDim.x * (blockDim.x >> 5));
+  int32_t w = (int32_t)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+  unsigned my_edges = 0;
+  // row metadata of the first iteration
+  int32_t row = -1, b = 0, e = 0;
+  {
+    const int32_t pos = w * G + g;
     if (pos < n) {
-      row = perm ? (int64_t)__ldg(perm + pos) : pos;
+      row = perm ? __ldg(perm + pos) : pos;
       b = __ldg(rp + row);
-      D = __ldg(rp + row + 1) - b;
+      e = __ldg(rp + row + 1);
     }
-    const bool skip = row < 0 || D > kHeavyT;
-    const int32_t Dl = skip ? 0 : D;
-    const int32_t Dmax = __reduce_max_sync(0xffffffffu, Dl);
-    if (edges_dev) {                                    // profiling: edges this warp aggregates
-      const unsigned tot = __reduce_add_sync(0xffffffffu, pc == 0 ? (unsigned)Dl : 0u);
-      if (lane == 0 && tot) atomicAdd(edges_dev, (unsigned long long)tot);
+  }
+  for (; w * G < n; w += warps) {
+    // next iteration's metadata, in flight while this row is gathered
+    int32_t row_n = -1, b_n = 0, e_n = 0;
+    {
+      const int32_t pos = (w + warps) * G + g;
+      if (pos < n) {
+        row_n = perm ? __ldg(perm + pos) : pos;
+        b_n = __ldg(rp + row_n);
+        e_n = __ldg(rp + row_n + 1);
+      }
     }
+    const int32_t D = e - b;
+    const int32_t Dl = (row < 0 || D > kHeavyT) ? 0 : D;
+    const int32_t Dmax = __reduce_max_sync(kFull, Dl);
+    if (edges_dev && pc == 0) my_edges += (unsigned)Dl;
+    const bool uni = __reduce_min_sync(kFull, Dl) == Dmax;   // all rows of the warp equally long
     for (int p0 = 0; p0 < npieces; p0 += LPR) {
       const int piece = p0 + pc;
       const bool colok = piece < npieces;
-      const int col0 = piece * E;
+      // lanes past the row read piece 0 again (same sectors, in bounds) and store nothing
+      const char* hb = reinterpret_cast<const char*>(h) + (colok ? piece : 0) * 16;
       float acc[E];
 #pragma unroll
       for (int k = 0; k < E; ++k) acc[k] = 0.f;
       for (int32_t base = 0; base < Dmax; base += LPR) {
-        const int32_t jj = (base + pc < Dl) ? __ldg(col + b + base + pc) : 0;
-        const int lim = min(LPR, Dmax - base);
-        for (int u = 0; u < lim; u += kGU) {
-          uint4 raw[kGU];
+        const int32_t jj = (base + pc < Dl) ? __ldg(col + b + base + pc) : -1;
+        const int m = min(LPR, Dmax - base);
+        int k = 0;
+        if (uni) {                                      // full groups of kU edges: no predicates
+          for (; k + kU <= m; k += kU) {
+            uint4 raw[kU];
 #pragma unroll
-          for (int uu = 0; uu < kGU; ++uu) {
-            const int tt = u + uu;
-            const int32_t jn = __shfl_sync(0xffffffffu, jj, ((g << lpr_log) + (tt & (LPR - 1))) & 31);
-            raw[uu] = make_uint4(0u, 0u, 0u, 0u);
-            if (tt < LPR && base + tt < Dl && colok)
-              raw[uu] = __ldg(reinterpret_cast<const uint4*>(h + (int64_t)jn * ldh + col0));
+            for (int uu = 0; uu < kU; ++uu) {
+              const int32_t jn = __shfl_sync(kFull, jj, gbase + k + uu);
+              raw[uu] = __ldg(reinterpret_cast<const uint4*>(hb + (int64_t)jn * ldb));
+            }
+#pragma unroll
+            for (int uu = 0; uu < kU; ++uu) acc_piece<TI>(acc, raw[uu]);
+          }
+        }
+        for (; k < m; k += kU) {                        // ragged rows / tail
+          uint4 raw[kU];
+          bool ok[kU];
+#pragma unroll
+          for (int uu = 0; uu < kU; ++uu) {
+            const int32_t jn = __shfl_sync(kFull, jj, gbase + ((k + uu) & (LPR - 1)));
+            ok[uu] = k + uu < m && jn >= 0;
+            if (ok[uu]) raw[uu] = __ldg(reinterpret_cast<const uint4*>(hb + (int64_t)jn * ldb));
           }
 #pragma unroll
-          for (int uu = 0; uu < kGU; ++uu) acc_piece<TI>(acc, raw[uu]);
+          for (int uu = 0; uu < kU; ++uu)
+            if (ok[uu]) acc_piece<TI>(acc, raw[uu]);
         }
       }
-      if (!skip && colok) {
-        if (MODE == 0) {
+      if (row >= 0 && D <= kHeavyT && colok) {
+        float v[E];
+        if (MODE == 0 && D > 0) {
           const float fd = (float)D;
+          const float y = 1.0f / fd;                    // once per row
 #pragma unroll
-          for (int k = 0; k < E; ++k) acc[k] = D > 0 ? acc[k] / fd : 0.f;
-        }
-        __nv_bfloat16* dst = out + row * ldo + col0;
-        if constexpr (E == 8) {
-          *reinterpret_cast<uint4*>(dst) = make_uint4(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]),
-                                                      pack_bf16x2(acc[4], acc[5]), pack_bf16x2(acc[6], acc[7]));
+          for (int k = 0; k < E; ++k) {
+            const float q = acc[k] * y;
+            v[k] = fmaf(fmaf(-q, fd, acc[k]), y, q);
+          }
         } else {
-          *reinterpret_cast<uint2*>(dst) = make_uint2(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]));
+#pragma unroll
+          for (int k = 0; k < E; ++k) v[k] = acc[k];
+        }
+        __nv_bfloat16* dst = out + (int64_t)row * ldo + piece * E;
+        if constexpr (E == 8) {
+          *reinterpret_cast<uint4*>(dst) = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
+                                                      pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
+        } else {
+          *reinterpret_cast<uint2*>(dst) = make_uint2(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]));
         }
       }
     }
+    row = row_n;
+    b = b_n;
+    e = e_n;
+  }
+  if (edges_dev) {                                      // one atomic per warp per launch
+    my_edges = __reduce_add_sync(kFull, my_edges);
+    if (lane == 0 && my_edges) atomicAdd(edges_dev, (unsigned long long)my_edges);
   }
 }
 
@@ -717,11 +763,25 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   const int npieces = (pitch_in + E - 1) / E;
   int lpr_log = 0;
   while ((1 << lpr_log) < npieces && lpr_log < 5) ++lpr_log;
-  const int G = 32 >> lpr_log;
-  const int64_t warps = ceil_div(n, G);
-  const int grid = (int)std::min<int64_t>(ceil_div(warps, 8), 148LL * 8 * 4);
+  if (n > INT32_MAX || ldh * (int64_t)sizeof(TI) > INT32_MAX) {
+    set_error("gather: %lld rows of stride %lld elements exceed the 32-bit row / byte-stride range",
+              (long long)n, (long long)ldh);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
   const ProfSlot ps = prof_begin_launch("gather", s);
-  k_gather_rows<TI, MODE><<<grid, 256, 0, s>>>(perm, rp, col, n, h, ldh, pitch_in, lpr_log, out, ldo, ps.edges_dev);
+  // 2 row loads in flight per lane at 40 registers (6 CTAs, 48 warps per SM) measured best on
+  // products-shaped blocks: occupancy hides the per-row index chain better than deeper unrolling
+  constexpr int kU = 2, kMinB = 6;
+  const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
+  const int32_t n32 = (int32_t)n;
+  const int32_t ldb = (int32_t)(ldh * (int64_t)sizeof(TI));             // row stride in bytes
+#define BF_V2(L) k_gather_v2<TI, MODE, L, kU, kMinB><<<fgrid, 256, 0, s>>>(perm, rp, col, n32, h, ldb, npieces, out, \
+                                                                          ldo, ps.edges_dev)
+  if (lpr_log <= 2) BF_V2(4);
+  else if (lpr_log == 3) BF_V2(8);
+  else if (lpr_log == 4) BF_V2(16);
+  else BF_V2(32);
+#undef BF_V2
   BF_LAUNCHED(MODE == 0 ? "k_gather_mean" : "k_gather_sum");
   // algorithmic bytes: per row perm + row_ptr pair + bf16 output row; per edge index + source row
   prof_end_launch(ps, s, (double)n * (12.0 + 2.0 * pitch_in), 4.0 + (double)pitch_in * sizeof(TI));

@@ -28,8 +28,12 @@ class DeviceGraph:
     """CSR graph resident in HBM (+ the node_map workspace the relabel kernels use)."""
 
     def __init__(self, row_ptr, col, device="cuda"):
-        self.row_ptr = torch.as_tensor(np.asarray(row_ptr, np.int64)).to(device)
-        self.col = torch.as_tensor(np.asarray(col, np.int32)).to(device)
+        if torch.is_tensor(row_ptr):
+            self.row_ptr = row_ptr.to(device=device, dtype=torch.int64).contiguous()
+            self.col = col.to(device=device, dtype=torch.int32).contiguous()
+        else:
+            self.row_ptr = torch.as_tensor(np.asarray(row_ptr, np.int64)).to(device)
+            self.col = torch.as_tensor(np.asarray(col, np.int32)).to(device)
         self.N = self.row_ptr.numel() - 1
         self.ws = torch.empty(B.graph_workspace_bytes(self.N), dtype=torch.uint8, device=device)
         self.g = B.Graph()

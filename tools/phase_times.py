@@ -18,13 +18,13 @@ def main():
     cfg = CONFIGS[name]
     from paper_conf_hpca_yangzl25_b200 import buffalo as B
     from paper_conf_hpca_yangzl25_b200.train import Trainer
-    rp, col, X, y, seeds, Ws, bs = bench.make_inputs(cfg)
-    feats = torch.as_tensor(X).cuda().to(torch.bfloat16).contiguous()
-    tr = Trainer((rp, col), feats, torch.as_tensor(y).cuda(), torch.as_tensor(seeds).cuda(), cfg.dims,
+    rp, col, X, y, seeds, Ws, bs = bench.make_inputs_device(cfg)
+    feats = X.to(torch.bfloat16).contiguous()
+    tr = Trainer((rp, col), feats, y, seeds, cfg.dims,
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=B.BF16, gemm_mode=B.GEMM_BF16,
                  k_min=cfg.k_min, k_max=max(cfg.k_min, min(cfg.k_max, 64)))
     if name == "products":
-        t2 = Trainer((rp, col), feats, torch.as_tensor(y).cuda(), torch.as_tensor(seeds).cuda(), cfg.dims,
+        t2 = Trainer((rp, col), feats, y, seeds, cfg.dims,
                      cfg.fanout, cfg.F, Ws, bs, feat_dtype=B.BF16, gemm_mode=B.GEMM_BF16, k_min=1, k_max=1)
         _, _, est1, _ = t2.schedule(0)
         del t2
