@@ -11,7 +11,8 @@ import numpy as np
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbuffalo.so")
+# BUFFALO_LIB: load an experimental build instead (diagnostics only; tools/exp_build.sh)
+LIB_PATH = os.environ.get("BUFFALO_LIB") or os.path.join(_HERE, "libbuffalo.so")
 
 c_i32, c_i64, c_u64, c_p, c_sz, c_f = (ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64,
                                        ctypes.c_void_p, ctypes.c_size_t, ctypes.c_float)

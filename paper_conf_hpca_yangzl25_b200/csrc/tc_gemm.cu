@@ -55,6 +55,22 @@ __device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, i
       "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(su32(bar))
       : "memory");
 }
+// TMA store of a {32 col, 32 row} bf16 box from SWIZZLE_64B-staged shared memory (bulk group).
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void* src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(su32(src)), "r"(c0), "r"(c1)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
+__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+// Row `lane` of a 32 x 64-B staging box, 16-B chunk k, in the SWIZZLE_64B layout (chunk ^= row>>1 & 3).
+__device__ __forceinline__ void st_stage64(uint8_t* box, int lane, int k, uint4 v) {
+  *reinterpret_cast<uint4*>(box + lane * 64 + ((k ^ ((lane >> 1) & 3)) << 4)) = v;
+}
+
 __device__ __forceinline__ void bulk_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                    su32(dst)),
@@ -137,7 +153,12 @@ __device__ __forceinline__ uint32_t pk(float a, float b) {
 constexpr int kTM = 128;
 constexpr int kChunkA = kTM * 128;     // 16 KB: 128 rows x 64 bf16
 constexpr int kEpiWarps = 8;       // two per TMEM lane quadrant (column groups interleaved)
-constexpr int kGemmThreads = (kEpiWarps + 2) * 32;
+// Producer warps: TMA issue is throughput-limited per issuing warp (tools/tma_bench.cu: one
+// issuer reaches ~1.6 TB/s with gather4 and ~4.8 TB/s with 2D boxes, four reach 4.5 / 6.1 TB/s),
+// so chunk g of the CTA's sequence is loaded by producer warp g % kProducers.
+constexpr int kProducers = 2;
+constexpr int kMmaWarp = kEpiWarps + kProducers;
+constexpr int kGemmThreads = (kEpiWarps + kProducers + 1) * 32;
 
 struct GemmParams {
   int64_t n_rows;
@@ -147,6 +168,12 @@ struct GemmParams {
   int nkc_self, nkc;          // K-chunks of the self half, total
   const uint8_t* wpk;         // pre-swizzled weight chunks (Np x 128 B each)
   int Np, d_out, pitch_out, ld_out, tmem_cols, nstages;
+  // Resident weights (w_res): the CTA keeps the rows [half * Nsub, (half + 1) * Nsub) of every
+  // weight chunk in shared memory for the whole launch (one 1D bulk copy per chunk at start), so
+  // the pipeline stages carry A tiles only; with nsplit = 2 the two CTAs of a tile set compute
+  // the two column halves of the same tiles (A is read twice, the second time from L2).
+  int w_res, nsplit, Nsub, db_parts;
+  int stage_off, stage_bytes; // epilogue staging area (8 warps x 2 x 2 KB; 0 for the backward)
   const float* bias;
   int relu, out_f32;
   void* out;
@@ -161,27 +188,35 @@ struct GemmParams {
 template <bool kBwd>
 __global__ void __launch_bounds__(kGemmThreads, 1)
     k_tc_gemm_tma(const __grid_constant__ CUtensorMap self_map, const __grid_constant__ CUtensorMap agg_map,
+                  const __grid_constant__ CUtensorMap out_map, const __grid_constant__ CUtensorMap out2_map,
                   const GemmParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  // 1024-B alignment by offset (keeps the shared address space visible to the compiler)
+  uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
   const int NS = p.nstages;
-  const int bbytes = p.Np * 128;
+  const int bbytes = p.Np * 128;                       // one packed weight chunk
+  const int wsz = p.Nsub * 128;                        // this CTA's rows of a chunk
+  const int half = (int)(blockIdx.x % p.nsplit);
+  const int64_t set0 = blockIdx.x / p.nsplit, nsets = gridDim.x / p.nsplit;
   uint8_t* sA = smem;                                  // NS x 16 KB
-  uint8_t* sB = smem + NS * kChunkA;                   // NS x Np x 128 B
-  uint64_t* full = (uint64_t*)(sB + NS * bbytes);
+  uint8_t* sB = smem + NS * kChunkA;                   // streamed: NS x Np x 128 B; resident: nkc x wsz
+  uint64_t* full = (uint64_t*)(smem + p.stage_off + p.stage_bytes);   // after the store staging
   uint64_t* empty = full + NS;
   uint64_t* acc_full = empty + NS;
   uint64_t* acc_empty = acc_full + 2;
-  uint32_t* tmem_slot = (uint32_t*)(acc_empty + 2);
+  uint64_t* wbar = acc_empty + 2;
+  uint32_t* tmem_slot = (uint32_t*)(wbar + 2);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t ntiles = (p.n_rows + kTM - 1) / kTM;
+  const int col_base = half * p.Nsub;                  // first output column of this CTA
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < NS; ++i) { mb_init(&full[i], 1); mb_init(&empty[i], 1); }
     for (int i = 0; i < 2; ++i) { mb_init(&acc_full[i], 1); mb_init(&acc_empty[i], kEpiWarps * 32); }
+    mb_init(wbar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == kEpiWarps + 1) {
+  if (warp == kMmaWarp) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
                  "r"(p.tmem_cols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -191,15 +226,22 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   fence_after();
   const uint32_t tmem = *tmem_slot;
 
-  if (warp == kEpiWarps) {
+  if (warp >= kEpiWarps && warp < kMmaWarp) {
     // ---------------- producer: A chunk (TMA 2D, or 32 x gather4 for gathered self rows) +
     // weight chunk (bulk) per stage
+    const int pw = warp - kEpiWarps;                 // this producer's share: chunks g % kProducers == pw
     if (lane == 0) {
       asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&self_map)) : "memory");
       asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&agg_map)) : "memory");
+      if (p.w_res && pw == 0) {                                   // the CTA's weight rows, once
+        const int c_lo = p.self_tiles > 0 ? 0 : p.nkc_self;
+        mb_expect(wbar, (uint32_t)((p.nkc - c_lo) * wsz));
+        for (int c = c_lo; c < p.nkc; ++c)
+          bulk_1d(sB + c * wsz, p.wpk + (int64_t)c * bbytes + (int64_t)col_base * 128, wsz, wbar);
+      }
     }
     int64_t g = 0;
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (int64_t t = set0; t < ntiles; t += nsets) {
       const int row0 = (int)(t * kTM);
       int32_t idx[4];
       if (p.self_idx) {
@@ -211,10 +253,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       }
       const int cb = t >= p.self_tiles ? p.nkc_self : 0;
       for (int c = cb; c < p.nkc; ++c, ++g) {
+        if ((int)(g % kProducers) != pw) continue;
         const int st = (int)(g % NS);
         if (lane == 0) {
           if (g >= NS) mb_wait(&empty[st], (uint32_t)(((g / NS) - 1) & 1));
-          mb_expect(&full[st], kChunkA + bbytes);
+          mb_expect(&full[st], kChunkA + (p.w_res ? 0 : bbytes));
         }
         __syncwarp();
         if (c < p.nkc_self && p.self_idx) {
@@ -223,27 +266,28 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
           if (c < p.nkc_self) tma_2d(sA + st * kChunkA, &self_map, c * 64, row0, &full[st]);
           else tma_2d(sA + st * kChunkA, &agg_map, (c - p.nkc_self) * 64, row0, &full[st]);
         }
-        if (lane == 0) bulk_1d(sB + st * bbytes, p.wpk + (int64_t)c * bbytes, bbytes, &full[st]);
+        if (lane == 0 && !p.w_res) bulk_1d(sB + st * bbytes, p.wpk + (int64_t)c * bbytes, bbytes, &full[st]);
         __syncwarp();
       }
     }
-  } else if (warp == kEpiWarps + 1) {
+  } else if (warp == kMmaWarp) {
     if (lane == 0) {
       // ---------------- MMA issuer
-      const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(p.Np >> 3) << 17) |
+      const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(p.Nsub >> 3) << 17) |
                              ((uint32_t)(kTM >> 4) << 24);
+      if (p.w_res) mb_wait(wbar, 0);
       int64_t g = 0, i = 0;
-      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+      for (int64_t t = set0; t < ntiles; t += nsets, ++i) {
         const int acc = (int)(i & 1);
         if (i >= 2) mb_wait(&acc_empty[acc], (uint32_t)(((i >> 1) - 1) & 1));
         fence_after();
-        const uint32_t d = tmem + acc * p.Np;
+        const uint32_t d = tmem + acc * p.Nsub;
         const int cb = t >= p.self_tiles ? p.nkc_self : 0;
         for (int c = cb; c < p.nkc; ++c, ++g) {
           const int st = (int)(g % NS);
           mb_wait(&full[st], (uint32_t)((g / NS) & 1));
           fence_after();
-          const uint32_t a = su32(sA + st * kChunkA), b = su32(sB + st * bbytes);
+          const uint32_t a = su32(sA + st * kChunkA), b = su32(p.w_res ? sB + c * wsz : sB + st * bbytes);
 #pragma unroll
           for (int k = 0; k < 4; ++k)
             mma_f16(d, desc_sw128(a + 32 * k), desc_sw128(b + 32 * k), idesc, (c > cb || k > 0) ? 1u : 0u);
@@ -261,10 +305,13 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     // the current one is processed; the next TMEM load is issued before the current group's math.
     const int q = warp & 3, h = warp >> 2;
     float* sbias = reinterpret_cast<float*>(tmem_slot + 4);   // 16-B aligned
-    for (int c = threadIdx.x; c < p.Np; c += kEpiWarps * 32)
-      sbias[c] = (p.bias && c < p.d_out) ? __ldg(p.bias + c) : 0.f;
+    uint8_t* stg = smem + p.stage_off + warp * 4096;          // this warp's two 2-KB staging boxes
+    int sbuf = 0;
+    for (int c = threadIdx.x; c < p.Nsub; c += kEpiWarps * 32)
+      sbias[c] = (p.bias && col_base + c < p.d_out) ? __ldg(p.bias + col_base + c) : 0.f;
     asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
-    const int ng = (p.pitch_out + 31) / 32;
+    const int ncol_cta = min(p.Nsub, p.pitch_out - col_base);   // output columns of this CTA
+    const int ng = (ncol_cta + 31) / 32;
     const int nj = (ng - h + 1) / 2;              // groups of this warp (<= 4)
     float dbacc[4] = {0.f, 0.f, 0.f, 0.f};
     uint4 hreg[4][4];
@@ -273,26 +320,26 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
 #pragma unroll
       for (int k = 0; k < 4; ++k) hreg[j][k] = make_uint4(0u, 0u, 0u, 0u);
     if (kBwd) {
-      const int64_t row = (int64_t)blockIdx.x * kTM + q * 32 + lane;
+      const int64_t row = set0 * kTM + q * 32 + lane;
       if (row < p.n_rows) {
-        const __nv_bfloat16* hr = p.H + row * p.ldH;
+        const __nv_bfloat16* hr = p.H + row * p.ldH + col_base;
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
           const int c0 = (2 * j + h) * 32;
 #pragma unroll
           for (int k = 0; k < 4; ++k)
-            if (j < nj && c0 + 8 * k < p.pitch_out) hreg[j][k] = __ldg(reinterpret_cast<const uint4*>(hr + c0 + 8 * k));
+            if (j < nj && c0 + 8 * k < ncol_cta) hreg[j][k] = __ldg(reinterpret_cast<const uint4*>(hr + c0 + 8 * k));
         }
       }
     }
     int64_t i = 0;
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+    for (int64_t t = set0; t < ntiles; t += nsets, ++i) {
       const int acc = (int)(i & 1);
       mb_wait(&acc_full[acc], (uint32_t)((i >> 1) & 1));
       fence_after();
       const int64_t row = t * kTM + q * 32 + lane;
       const bool rok = row < p.n_rows;
-      const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + acc * p.Np;
+      const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + acc * p.Nsub;
       float invd = 1.f;
       if (kBwd && rok && p.zs) {
         const int32_t d = __ldg(p.rp + row + 1) - __ldg(p.rp + row);
@@ -312,7 +359,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             ld32_wait(r[j & 1]);
           }
           if (!kBwd && j + 1 < nj) ld32_issue(tbase + c0 + 64, r[(j + 1) & 1]);
-          const int ncols = min(32, p.pitch_out - c0);   // multiple of 8
+          const int ncols = min(32, ncol_cta - c0);      // multiple of 8
+          const int gc0 = col_base + c0;                 // global output column
           float v[32];
 #pragma unroll
           for (int k = 0; k < 32; ++k) v[k] = __uint_as_float(r[j & 1][k]);
@@ -325,22 +373,24 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
 #pragma unroll
                   for (int e = 0; e < 4; ++e) {
                     const float h0 = __uint_as_float(hw[e] << 16), h1 = __uint_as_float(hw[e] & 0xffff0000u);
-                    if (!(h0 > 0.f) || c0 + k + 2 * e >= p.d_out) v[k + 2 * e] = 0.f;
-                    if (!(h1 > 0.f) || c0 + k + 2 * e + 1 >= p.d_out) v[k + 2 * e + 1] = 0.f;
+                    if (!(h0 > 0.f) || gc0 + k + 2 * e >= p.d_out) v[k + 2 * e] = 0.f;
+                    if (!(h1 > 0.f) || gc0 + k + 2 * e + 1 >= p.d_out) v[k + 2 * e + 1] = 0.f;
                   }
                 } else {
 #pragma unroll
                   for (int e = 0; e < 8; ++e) v[k + e] = 0.f;
                 }
               }
-              __nv_bfloat16* zo = p.zb + row * p.pitch_out + c0;
+              // bf16 dZ and dZ/D rows (direct stores: measured faster here than staging two
+              // boxes per group through the TMA-store path)
+              __nv_bfloat16* zo = p.zb + row * p.pitch_out + gc0;
 #pragma unroll
               for (int k = 0; k < 32; k += 8)
                 if (k < ncols)
                   *reinterpret_cast<uint4*>(zo + k) = make_uint4(pk(v[k], v[k + 1]), pk(v[k + 2], v[k + 3]),
                                                                  pk(v[k + 4], v[k + 5]), pk(v[k + 6], v[k + 7]));
               if (p.zs) {
-                __nv_bfloat16* so = p.zs + row * p.pitch_out + c0;
+                __nv_bfloat16* so = p.zs + row * p.pitch_out + gc0;
 #pragma unroll
                 for (int k = 0; k < 32; k += 8)
                   if (k < ncols)
@@ -354,17 +404,17 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             }
             // prefetch this group's H of the next tile (its registers are free now)
             {
-              const int64_t tn = t + gridDim.x;
+              const int64_t tn = t + nsets;
               const int64_t rn = tn * kTM + q * 32 + lane;
               if (tn < ntiles && rn < p.n_rows) {
-                const __nv_bfloat16* hr = p.H + rn * p.ldH + c0;
+                const __nv_bfloat16* hr = p.H + rn * p.ldH + gc0;
 #pragma unroll
                 for (int k = 0; k < 4; ++k)
                   if (8 * k < ncols) hreg[j][k] = __ldg(reinterpret_cast<const uint4*>(hr + 8 * k));
               }
             }
             dbacc[j] += warp_colsum32(v, lane);
-          } else if (rok) {
+          } else {
 #pragma unroll
             for (int k = 0; k < 32; k += 4) {
               const float4 bb = *reinterpret_cast<const float4*>(sbias + c0 + k);
@@ -375,17 +425,29 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
               for (int k = 0; k < 32; ++k) v[k] = fmaxf(v[k], 0.f);
             }
             if (p.out_f32) {
-              float* o = (float*)p.out + row * p.ld_out + c0;
+              if (rok) {
+                float* o = (float*)p.out + row * p.ld_out + gc0;
 #pragma unroll
-              for (int k = 0; k < 32; k += 4)
-                if (k < ncols) *reinterpret_cast<float4*>(o + k) = make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]);
+                for (int k = 0; k < 32; k += 4)
+                  if (k < ncols) *reinterpret_cast<float4*>(o + k) = make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]);
+              }
             } else {
-              __nv_bfloat16* o = (__nv_bfloat16*)p.out + row * p.ld_out + c0;
+              // bf16 rows through a staging box and one TMA store per warp and column group
+              // (coalesced, asynchronous; rows past n_rows are clipped by the map)
+              uint8_t* box = stg + sbuf * 2048;
+              sbuf ^= 1;
+              if (lane == 0) bulk_wait_read<1>();       // the store that used this box has read it
+              __syncwarp();
 #pragma unroll
-              for (int k = 0; k < 32; k += 8)
-                if (k < ncols)
-                  *reinterpret_cast<uint4*>(o + k) = make_uint4(pk(v[k], v[k + 1]), pk(v[k + 2], v[k + 3]),
-                                                                pk(v[k + 4], v[k + 5]), pk(v[k + 6], v[k + 7]));
+              for (int k = 0; k < 4; ++k)
+                st_stage64(box, lane, k, make_uint4(pk(v[8 * k], v[8 * k + 1]), pk(v[8 * k + 2], v[8 * k + 3]),
+                                                     pk(v[8 * k + 4], v[8 * k + 5]), pk(v[8 * k + 6], v[8 * k + 7])));
+              fence_async_smem();
+              __syncwarp();
+              if (lane == 0) {
+                tma_store_2d(&out_map, box, gc0, (int)(t * kTM + q * 32));
+                bulk_commit();
+              }
             }
           }
           if (!kBwd && j + 1 < nj) ld32_wait(r[(j + 1) & 1]);
@@ -394,6 +456,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       fence_before();
       mb_arrive(&acc_empty[acc]);
     }
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    __syncwarp();
     if (kBwd) {
       // combine the four lane quadrants in order -> one partial per CTA
       float* red = reinterpret_cast<float*>(sA);     // stage 0 A buffer: every MMA has completed
@@ -402,16 +466,20 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       for (int j = 0; j < 4; ++j)
         if (j < nj) red[q * 256 + (2 * j + h) * 32 + lane] = dbacc[j];
       asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
-      for (int c = threadIdx.x; c < p.d_out; c += kEpiWarps * 32) {
+      const int ncd = min(p.Nsub, p.d_out - col_base);
+      for (int c = threadIdx.x; c < ncd; c += kEpiWarps * 32) {
         float tsum = 0.f;
         for (int w = 0; w < 4; ++w) tsum += red[w * 256 + c];
-        p.db_part[(int64_t)blockIdx.x * p.d_out + c] = tsum;
+        p.db_part[set0 * p.d_out + col_base + c] = tsum;
       }
+      // the reader sums db_parts rows: rows no tile set wrote are zero
+      for (int64_t r = nsets + set0; r < p.db_parts; r += nsets)
+        for (int c = threadIdx.x; c < ncd; c += kEpiWarps * 32) p.db_part[r * p.d_out + col_base + c] = 0.f;
     }
   }
   fence_before();
   __syncthreads();
-  if (warp == kEpiWarps + 1) {
+  if (warp == kMmaWarp) {
     fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(p.tmem_cols));
   }
@@ -566,7 +634,8 @@ typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
 buffalo_status encode_map(CUtensorMap* map, const void* base, int64_t cols, int64_t rows, int64_t ld,
-                          int box_rows = kTM) {
+                          int box_rows = kTM, int box_cols = 64,
+                          CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B) {
   static EncodeTiledFn fn = nullptr;
   if (!fn) {
     void* f = nullptr;
@@ -580,10 +649,10 @@ buffalo_status encode_map(CUtensorMap* map, const void* base, int64_t cols, int6
   }
   const cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)(rows > 0 ? rows : 1)};
   const cuuint64_t strides[1] = {(cuuint64_t)ld * 2};
-  const cuuint32_t box[2] = {64, (cuuint32_t)box_rows};
+  const cuuint32_t box[2] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows};
   const cuuint32_t estr[2] = {1, 1};
   CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
-                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     set_error("cuTensorMapEncodeTiled failed (%d)", (int)r);
@@ -657,8 +726,18 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   p.d_out = d_out;
   p.pitch_out = (int)pitch_of(d_out);
   p.ld_out = (int)ld_out;
+  // resident weights when all weight chunks fit next to >= 4 A stages and the store staging
+  // (a CTA-pair column split, nsplit = 2, is supported by the kernel but measured slower)
+  const int64_t w_all = (int64_t)p.nkc * p.Np * 128;
+  const int64_t kStaging = epi ? 0 : kEpiWarps * 4096;
+  const int misc = 16 * 8 + 48 + 4 * p.Np + 1024;                    // barriers, slot, bias, alignment
+  p.nsplit = 1;
+  p.w_res = (227 * 1024 - w_all - kStaging - misc) / kChunkA >= 4 ? 1 : 0;
+  if (getenv("BUFFALO_GEMM_STREAM_W")) p.w_res = 0;                  // A/B switch (diagnostic)
+  p.Nsub = p.Np / p.nsplit;
+  p.db_parts = (int)gemm_grid(n_rows);
   int cols = 32;
-  while (cols < 2 * p.Np) cols *= 2;
+  while (cols < 2 * p.Nsub) cols *= 2;
   p.tmem_cols = cols;
   p.bias = bias;
   p.relu = relu;
@@ -669,18 +748,37 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
     p.H = epi->H; p.ldH = epi->ldH; p.rp = epi->rp;
     p.zb = epi->zb; p.zs = epi->zs; p.db_part = epi->db_part;
   }
-  const int stage = kChunkA + p.Np * 128;
-  p.nstages = std::max(2, std::min(8, (200 * 1024) / stage));
-  const int smem = p.nstages * stage + 16 * p.nstages + 48 + 4 * p.Np + 1024;
+  int smem;
+  if (p.w_res) {
+    const int64_t wres = (int64_t)p.nkc * p.Nsub * 128;               // chunks < c_lo stay unused
+    p.nstages = (int)std::min<int64_t>(8, (227 * 1024 - wres - kStaging - misc) / kChunkA);
+    p.stage_off = (int)(p.nstages * kChunkA + wres);
+  } else {
+    const int stage = kChunkA + p.Np * 128;
+    p.nstages = std::max(2, std::min<int>(8, (int)((227 * 1024 - kStaging - misc) / stage)));
+    p.stage_off = p.nstages * stage;
+  }
+  p.stage_bytes = (int)kStaging;
+  smem = (int)(p.stage_off + kStaging + misc);
+  // output maps for the TMA-store epilogue: {32 col, 32 row} boxes, SWIZZLE_64B staging
+  CUtensorMap om, om2;
+  if (!epi && !out_f32) {
+    BF_CHECK(encode_map(&om, out, p.pitch_out, n_rows, ld_out, 32, 32, CU_TENSOR_MAP_SWIZZLE_64B));
+    om2 = om;
+  } else {
+    om = am;                                                          // unused (fp32 rows stored directly)
+    om2 = am;
+  }
   static bool attr = false;
   if (!attr) {
     BF_CUDA(cudaFuncSetAttribute(k_tc_gemm_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
     BF_CUDA(cudaFuncSetAttribute(k_tc_gemm_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
     attr = true;
   }
-  const int grid = (int)gemm_grid(n_rows);
-  if (epi) k_tc_gemm_tma<true><<<grid, kGemmThreads, smem, s>>>(sm, am, p);
-  else k_tc_gemm_tma<false><<<grid, kGemmThreads, smem, s>>>(sm, am, p);
+  const int64_t sets = std::min<int64_t>(ceil_div(n_rows, kTM), 148 / p.nsplit);
+  const int grid = (int)(sets * p.nsplit);
+  if (epi) k_tc_gemm_tma<true><<<grid, kGemmThreads, smem, s>>>(sm, am, om, om2, p);
+  else k_tc_gemm_tma<false><<<grid, kGemmThreads, smem, s>>>(sm, am, om, om2, p);
   BF_LAUNCHED("k_tc_gemm_tma");
   return BUFFALO_OK;
 }
