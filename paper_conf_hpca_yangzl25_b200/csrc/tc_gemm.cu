@@ -506,11 +506,15 @@ __device__ __forceinline__ uint64_t desc_mn(uint32_t saddr, uint32_t lbo) {
          ((uint64_t)(1024 >> 4) << 32) | ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
 }
 
-__global__ void __launch_bounds__(192, 1)
+constexpr int kDwProducers = 2;                 // chunk c is loaded by producer warp 4 + c % 2
+constexpr int kDwMmaWarp = 4 + kDwProducers;
+constexpr int kDwThreads2 = (kDwMmaWarp + 1) * 32;
+
+__global__ void __launch_bounds__(kDwThreads2, 1)
     k_tc_dw_tma(const __grid_constant__ CUtensorMap z_map, const __grid_constant__ CUtensorMap self_map,
                 const __grid_constant__ CUtensorMap agg_map, const DwParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
   const int NS = p.nstages;
   const int nA = 2 * p.MT, nB = p.NT / 64;
   const int stage = (nA + nB) * kDwStrip2;
@@ -528,7 +532,7 @@ __global__ void __launch_bounds__(192, 1)
     mb_init(done, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 5) {
+  if (warp == kDwMmaWarp) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
                  "r"(p.tmem_cols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -537,9 +541,9 @@ __global__ void __launch_bounds__(192, 1)
   __syncthreads();
   fence_after();
   const uint32_t tmem = *tmem_slot;
-  if (warp == 4) {
-    // ---------------- producer
-    for (int c = 0; c < nchunks; ++c) {
+  if (warp >= 4 && warp < kDwMmaWarp) {
+    // ---------------- producers
+    for (int c = warp - 4; c < nchunks; c += kDwProducers) {
       const int st = c % NS;
       const int r0 = (int)(r_beg + (int64_t)c * kDwR);
       if (lane == 0) {
@@ -575,7 +579,7 @@ __global__ void __launch_bounds__(192, 1)
       }
       __syncwarp();
     }
-  } else if (warp == 5) {
+  } else if (warp == kDwMmaWarp) {
     if (lane == 0) {
       const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 15) | (1u << 16) |
                              ((uint32_t)(p.NT >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
@@ -623,7 +627,7 @@ __global__ void __launch_bounds__(192, 1)
   }
   fence_before();
   __syncthreads();
-  if (warp == 5) {
+  if (warp == kDwMmaWarp) {
     fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(p.tmem_cols));
   }
@@ -696,7 +700,7 @@ buffalo_status tc_dw_tma(int64_t n, int S, const __nv_bfloat16* z, int64_t ldz, 
     attr = true;
   }
   dim3 grid((unsigned)ceil_div(2 * Dp, p.NT), (unsigned)S);
-  k_tc_dw_tma<<<grid, 192, smem, s>>>(zm, sm, am, p);
+  k_tc_dw_tma<<<grid, kDwThreads2, smem, s>>>(zm, sm, am, p);
   BF_LAUNCHED("k_tc_dw_tma");
   return BUFFALO_OK;
 }
