@@ -350,7 +350,7 @@ def run_ours(args, cfg):
                     "gemm": args.gemm, "l2": "flushed (512 MiB write) between timed steps",
                     "epoch_ms": total_ms / args.steps, "edges_per_epoch": edges / args.steps,
                     "parallelism": f"dp{world} over bucket groups"},
-            roofline={"bound": "hbm", "kernel": "k_gather_rows (Aggregate: fwd neighbour mean, bwd transposed sum)",
+            roofline={"bound": "hbm", "kernel": "k_gather_v2 (Aggregate: fwd neighbour mean, bwd transposed sum)",
                       "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                       "traffic": traffic, "peak_source": peak_src,
                       "algorithmic_bytes_per_launch": g_bytes / max(1, g_launches),
