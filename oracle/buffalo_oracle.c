@@ -20,6 +20,12 @@
  *                           built top-down from the output layer; local src ids = dst prefix
  *                           then the other neighbours in ascending global id
  *                           [DESIGN.md readings R3, R4]
+ *  - oracle_triangles     : the average clustering coefficient C of Eq. 1 (PAPER.md:363,
+ *                           :384-386: "C ... obtained by offline graph analysis, utilizing the
+ *                           equation presented on page 142 of reference [27]"): the number of
+ *                           triangles through every node, T_v = #{(u, w): u < w, u, w in N(v),
+ *                           w in N(u)}, by definition (every neighbour pair tested with a binary
+ *                           search of the sorted row) [DESIGN.md reading R27]
  */
 #include <stdint.h>
 #include <stdlib.h>
@@ -186,4 +192,25 @@ int oracle_block_sizes(int64_t N, const int64_t* row_ptr, const int32_t* col,
     oracle_free_blocks(b, L);
     free(b);
     return rc;
+}
+
+/* ---------------------------------------------------------------- triangles per node (C, R27) */
+static int has_edge(const int64_t* row_ptr, const int32_t* col, int32_t u, int32_t w) {
+    int64_t lo = row_ptr[u], hi = row_ptr[u + 1];          /* sorted row: binary search */
+    while (lo < hi) {
+        const int64_t mid = lo + (hi - lo) / 2;
+        if (col[mid] < w) lo = mid + 1; else hi = mid;
+    }
+    return lo < row_ptr[u + 1] && col[lo] == w;
+}
+
+/* T[v] for v in [v0, v1): pairs of neighbours of v that are adjacent (each pair once). */
+void oracle_triangles(const int64_t* row_ptr, const int32_t* col, int64_t v0, int64_t v1, int64_t* T) {
+    for (int64_t v = v0; v < v1; ++v) {
+        int64_t t = 0;
+        for (int64_t a = row_ptr[v]; a < row_ptr[v + 1]; ++a)
+            for (int64_t b = a + 1; b < row_ptr[v + 1]; ++b)
+                t += has_edge(row_ptr, col, col[a], col[b]);
+        T[v - v0] = t;
+    }
 }

@@ -24,6 +24,10 @@ Functions and the passages they follow:
   softmax_ce           Alg. 2 l.10 PAPER.md:242; normalisation by the global batch (R19)
   sage_backward        Alg. 2 l.11-12 PAPER.md:243-244 (gradients accumulated over groups)
   train_epoch          Alg. 2 PAPER.md:233-245 end to end (one optimizer step, R18)
+  triangles, avg_clustering
+                       C of Eq. 1 (Newman's local clustering
+                       coefficient, "page 142 of reference [27]"): T_v by definition (C),
+                       C = mean over all nodes of 2 T_v / (d_v (d_v - 1)), 0 for d_v < 2 (R27)
 """
 import ctypes
 import math
@@ -70,6 +74,8 @@ def lib():
         _lib.oracle_build_blocks.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int64,
                                              ctypes.c_int32, P, ctypes.c_uint64, P]
         _lib.oracle_build_blocks.restype = ctypes.c_int
+        _lib.oracle_triangles.argtypes = [P, P, ctypes.c_int64, ctypes.c_int64, P]
+        _lib.oracle_triangles.restype = None
         _lib.oracle_block_sizes.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int64,
                                             ctypes.c_int32, P, ctypes.c_uint64, P, P]
         _lib.oracle_block_sizes.restype = ctypes.c_int
@@ -487,3 +493,34 @@ def train_epoch(g, seeds, X, y, Ws, bs, L, fanout, F, seed, dims, lr=0.0, storag
     newW = [np.asarray(W, np.float64) - lr * gW for W, (gW, _) in zip(Ws, acc)]
     newb = [np.asarray(b, np.float64) - lr * gb for b, (_, gb) in zip(bs, acc)]
     return total, acc, newW, newb, plan
+
+
+# ============================================================================ clustering (Eq. 1's C)
+def triangles(g, nodes=None):
+    """T_v = number of adjacent pairs among the neighbours of v (triangles through v), by
+    definition (oracle_triangles, every neighbour pair tested).  nodes=None: all nodes."""
+    if nodes is None:
+        T = np.zeros(g.N, dtype=np.int64)
+        lib().oracle_triangles(_p(g.row_ptr), _p(g.col), 0, g.N, _p(T))
+        return T
+    out = np.zeros(len(nodes), dtype=np.int64)
+    one = np.zeros(1, dtype=np.int64)
+    for i, v in enumerate(nodes):
+        lib().oracle_triangles(_p(g.row_ptr), _p(g.col), int(v), int(v) + 1, _p(one))
+        out[i] = one[0]
+    return out
+
+
+def avg_clustering(g, T=None):
+    """Average clustering coefficient C (reading R27): the mean over ALL nodes of the local
+    coefficient 2 T_v / (d_v (d_v - 1)), taken as 0 for d_v < 2 (Newman [27]; networkx's
+    average_clustering with count_zeros=True).  float64, summed in node order."""
+    T = triangles(g) if T is None else np.asarray(T, np.int64)
+    d = np.diff(np.asarray(g.row_ptr, np.int64)).astype(np.float64)
+    loc = np.zeros(g.N, dtype=np.float64)
+    ok = d >= 2
+    loc[ok] = 2.0 * T[ok] / (d[ok] * (d[ok] - 1.0))
+    total = 0.0
+    for x in loc:                      # plain sequential sum (node order)
+        total += x
+    return total / g.N
