@@ -243,6 +243,27 @@ BUFFALO_API buffalo_status buffalo_estimate_mem(int32_t num_layers, const int64_
                                     const buffalo_model* m, int64_t* lo_bytes_h,
                                     int64_t* hi_bytes_h);
 
+/* ------------------------------------------------------------------ C of Eq. 1 */
+/* The average clustering coefficient C of Eq. 1 (PAPER.md:363 R = min(1, I / (D * O * C));
+ * an offline property of the input graph, "page 142 of [27]"), exactly, by
+ * triangle counting (reading R27: C = (1/N) * sum_v 2 T_v / (d_v (d_v - 1)), 0 for d_v < 2).
+ * Graph as for every call (symmetric, sorted, simple CSR); node_map is not used.  Workspace:
+ * caller-owned device buffer of buffalo_clustering_workspace_bytes(g) bytes (the degree-oriented
+ * graph: int32[N+1] + int32[nnz/2+1], scan state, 593 doubles), any content.
+ * Errors: INVALID_ARG (null pointers, N <= 0), CAPACITY (workspace too small),
+ * UNSUPPORTED (nnz/2 or N >= 2^31: the oriented graph uses int32 offsets). */
+BUFFALO_API size_t buffalo_clustering_workspace_bytes(const buffalo_graph* g);
+/* T int64[num_nodes] (device, overwritten): T[v] = number of triangles through v, i.e. of
+ * adjacent pairs among v's neighbours.  Exact integers (bit-exact, any launch order). */
+BUFFALO_API buffalo_status buffalo_triangles(const buffalo_graph* g, int64_t* T, void* workspace,
+                                 size_t workspace_bytes, void* stream);
+/* *C_h = C from T (device, as written by buffalo_triangles), float64 summed in a fixed order
+ * (deterministic); *C_ppm_h (nullable) = llround(C * 10^6), the buffalo_sched.C_ppm input.
+ * Synchronises the stream once (the 8-byte result). */
+BUFFALO_API buffalo_status buffalo_avg_clustering(const buffalo_graph* g, const int64_t* T, double* C_h,
+                                      int64_t* C_ppm_h, void* workspace, size_t workspace_bytes,
+                                      void* stream);
+
 /* Number of kernels this thread has launched through the library (for bench accounting). */
 BUFFALO_API int64_t buffalo_launch_count(void);
 

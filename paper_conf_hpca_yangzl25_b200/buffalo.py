@@ -29,6 +29,7 @@ EXPORTS = [
     "buffalo_sage_bwd_scratch_bytes", "buffalo_sage_bwd", "buffalo_sgd_step",
     "buffalo_estimate_mem", "buffalo_launch_count", "buffalo_profile_begin", "buffalo_profile_end",
     "buffalo_status_str", "buffalo_last_error",
+    "buffalo_clustering_workspace_bytes", "buffalo_triangles", "buffalo_avg_clustering",
 ]
 
 
@@ -110,6 +111,9 @@ def lib(require_gpu=True):
             "buffalo_launch_count": (c_i64, []),
             "buffalo_profile_begin": (c_i32, [ctypes.c_char_p, P, c_i64, P]),
             "buffalo_profile_end": (c_i32, [P, P, P]),
+            "buffalo_clustering_workspace_bytes": (c_sz, [P]),
+            "buffalo_triangles": (c_i32, [P, P, P, c_sz, P]),
+            "buffalo_avg_clustering": (c_i32, [P, P, P, P, P, c_sz, P]),
             "buffalo_status_str": (ctypes.c_char_p, [c_i32]),
             "buffalo_last_error": (ctypes.c_char_p, []),
         }
@@ -225,6 +229,34 @@ def estimate_mem(n, e, model):
     lo, hi = c_i64(0), c_i64(0)
     _check(lib(False).buffalo_estimate_mem(L, na, ea, ref(model), ctypes.byref(lo), ctypes.byref(hi)))
     return lo.value, hi.value
+
+
+def clustering_workspace_bytes(graph):
+    return lib(False).buffalo_clustering_workspace_bytes(ref(graph))
+
+
+def triangles(graph, T, workspace, stream=None):
+    """T (int64 CUDA tensor [N]) = triangles through each node (C of Eq. 1, R27)."""
+    _check(lib().buffalo_triangles(ref(graph), ptr(T), ptr(workspace), workspace.numel() * workspace.element_size(),
+                                   stream_ptr(stream)))
+
+
+def avg_clustering(graph, T, workspace, stream=None):
+    """(C, C_ppm) from T (synchronises once)."""
+    C, ppm = ctypes.c_double(0), c_i64(0)
+    _check(lib().buffalo_avg_clustering(ref(graph), ptr(T), ctypes.byref(C), ctypes.byref(ppm), ptr(workspace),
+                                        workspace.numel() * workspace.element_size(), stream_ptr(stream)))
+    return C.value, ppm.value
+
+
+def clustering(graph, stream=None):
+    """Triangles per node and C for a buffalo Graph struct: (T tensor, C, C_ppm).  Allocates the
+    workspace and T with torch (device memory only)."""
+    ws = torch.empty(clustering_workspace_bytes(graph), dtype=torch.uint8, device="cuda")
+    T = torch.empty(graph.num_nodes, dtype=torch.int64, device="cuda")
+    triangles(graph, T, ws, stream)
+    C, ppm = avg_clustering(graph, T, ws, stream)
+    return T, C, ppm
 
 
 def launch_count():
