@@ -24,6 +24,12 @@ Functions and the passages they follow:
   softmax_ce           Alg. 2 l.10 PAPER.md:242; normalisation by the global batch (R19)
   sage_backward        Alg. 2 l.11-12 PAPER.md:243-244 (gradients accumulated over groups)
   train_epoch          Alg. 2 PAPER.md:233-245 end to end (one optimizer step, R18)
+  pool_forward, pool_backward
+                       GraphSAGE-pool (the paper's aggregators "mean, pool
+                       or LSTM", "Our method is general and applicable to any
+                       aggregators", :386; pool as defined by GraphSAGE [16]): P = ReLU(H W_pool^T
+                       + b_pool), h_agg = element-wise max over the sampled neighbours, then the
+                       same Update as mean (R28)
   triangles, avg_clustering
                        C of Eq. 1 (Newman's local clustering
                        coefficient, "page 142 of reference [27]"): T_v by definition (C),
@@ -218,7 +224,13 @@ def _scan_ws_bytes(length):
     return _R(8 * (_ceil(max(int(length), 1), SCAN_TILE) + 2))
 
 
-def mem_model(n, e, dims, act_dtype=FP32):
+def pool_dw_splits(n_rows, d):
+    """Split count of the pool weight's dW reduction (K = d columns, d rows)."""
+    tiles = _ceil(d, 64) * _ceil(d, 64)
+    return max(1, min(_ceil(296, tiles), _ceil(n_rows, 512)))
+
+
+def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
     """BucketMemEstimator reading R15: the exact arena bytes of one
     micro-batch with layer sizes n[0..L], e[1..L] (e indexed l-1) and widths dims[0..L].
     Returns (lo, hi): hi = capacity that always suffices (used as M_est), lo = bytes the
@@ -226,6 +238,7 @@ def mem_model(n, e, dims, act_dtype=FP32):
     Every buffer is rounded up to 256 B.  Restated from DESIGN.md §5 "Arena"."""
     L = len(e)
     s = 4 if act_dtype == FP32 else 2
+    pool = aggregator == "pool"                  # R28: fp32 only; block 1 keeps a transpose too
     blocks = 0
     build = 0
     for l in range(1, L + 1):
@@ -233,6 +246,8 @@ def mem_model(n, e, dims, act_dtype=FP32):
         blocks += _R(4 * (nl + 1)) + _R(4 * nl) + _R(4 * el) + _R(4 * nm)   # row_ptr cls_perm col src
         if l == 1:
             blocks += _R(4 * el)                                # col_global kept for layer 1
+            if pool:
+                blocks += _R(4 * (nm + 1)) + _R(4 * el) + _R(4 * nm)
         else:
             blocks += _R(4 * (nm + 1)) + _R(4 * el) + _R(4 * nm)  # transposed block + its classes
         pne = _part_count_elems(nl + el)
@@ -240,6 +255,8 @@ def mem_model(n, e, dims, act_dtype=FP32):
         frame += _R(4 * (pne + 1))                              # partition counts (classes, radix)
         if l >= 2:
             frame += _R(4 * el) + _R(4 * (nl + el))             # col_global + transpose cursors
+        elif pool:
+            frame += _R(4 * (nl + el))                          # transpose cursors of block 1
         build = max(build, frame)
     acts = 0
     for l in range(1, L + 1):
@@ -247,6 +264,11 @@ def mem_model(n, e, dims, act_dtype=FP32):
         if l < L:
             acts += _R(n[l] * pitch(dims[l]) * s)               # H_l
     acts += _R(n[L] * pitch(dims[L]) * 4)                       # logits
+    if pool:
+        for l in range(1, L + 1):
+            acts += _R(n[l - 1] * pitch(dims[l - 1]) * 4)       # P = ReLU(H W_pool^T + b_pool)
+            acts += _R(n[l] * pitch(dims[l - 1]) * 4)           # argmax (local src index)
+
     def dh_slot(l):                                             # dH_l slot of the backward region
         b = _R(n[l] * pitch(dims[l]) * 4)                       # fp32 dH / dlogits; bf16 dZ + dZ/D
         if act_dtype == BF16 and l < L:
@@ -258,8 +280,13 @@ def mem_model(n, e, dims, act_dtype=FP32):
         frame = dh_slot(l)
         if l >= 2:
             frame += dh_slot(l - 1)
+        if pool:
+            d = dims[l - 1]
+            frame += _R(n[l] * pitch(d) * 4) + _R(n[l - 1] * pitch(d) * 4)     # dh_agg, dQ
+            S2 = pool_dw_splits(n[l - 1], d)
+            frame += _R(S2 * d * d * 4) + _R(S2 * pitch(d) * 4)               # dW_pool, db_pool partials
         if act_dtype == FP32:
-            if l >= 2:
+            if l >= 2 and not pool:
                 frame += _R(n[l - 1] * pitch(dims[l]) * 4)      # transposed aggregate of dZ/D
             S = dw_splits(n[l], dims[l], dims[l - 1])
             frame += _R(S * dims[l] * 2 * dims[l - 1] * 4) + _R(S * pitch(dims[l]) * 4)  # dW, db partials
@@ -462,6 +489,76 @@ def sage_backward(blocks, cache, Ws, dlogits):
         if l > 1:
             dHin = c["A"].T @ (dZ @ W[:, d_in:])
             dHin[:n_dst] += dZ @ W[:, :d_in]
+            dH = dHin
+    return grads
+
+
+def pool_forward(blocks, X, Ws, bs, Wps, bps):
+    """GraphSAGE-pool forward in float64 (R28; GraphSAGE [16] "pooling aggregator", the
+    paper's aggregator list PAPER.md:63).  For block l with input rows H (its src, in local
+    order):  Q = H W_pool_l^T + b_pool_l,  P = ReLU(Q);  for dst i and column k,
+    h_agg[i,k] = max over the sampled neighbours j of P[j,k] (0 if D(i) = 0), arg[i,k] = the
+    neighbour attaining it, the first in CSR order (-1 when the max is 0: no gradient can flow
+    there, P = 0 means Q <= 0);  Z = [H[:n_dst] || h_agg] W_l^T + b_l;  H_l = ReLU(Z) for l < L.
+    Returns (logits, cache)."""
+    L = len(blocks)
+    H = np.asarray(X, dtype=np.float64)[blocks[0]["src_global"]]
+    cache = []
+    for l in range(1, L + 1):
+        b = blocks[l - 1]
+        W = np.asarray(Ws[l - 1], dtype=np.float64)
+        Wp = np.asarray(Wps[l - 1], dtype=np.float64)
+        d_in = H.shape[1]
+        Q = H @ Wp.T + np.asarray(bps[l - 1], dtype=np.float64)
+        P = np.maximum(Q, 0.0)
+        n = b["n_dst"]
+        agg = np.zeros((n, d_in))
+        arg = np.full((n, d_in), -1, dtype=np.int64)
+        rp, col = b["row_ptr"], b["col_local"]
+        for i in range(n):
+            nb = col[rp[i]:rp[i + 1]]
+            if len(nb) == 0:
+                continue
+            vals = P[nb]                                   # [D, d_in]
+            first = np.argmax(vals, axis=0)                # first occurrence of the max
+            agg[i] = vals[first, np.arange(d_in)]
+            arg[i] = np.where(agg[i] > 0, nb[first], -1)
+        Z = H[:n] @ W[:, :d_in].T + agg @ W[:, d_in:].T + np.asarray(bs[l - 1], dtype=np.float64)
+        cache.append(dict(H_in=H, Q=Q, P=P, agg=agg, arg=arg, Z=Z))
+        H = np.maximum(Z, 0.0) if l < L else Z
+    return H, cache
+
+
+def pool_backward(blocks, cache, Ws, Wps, dlogits):
+    """Backward of pool_forward: per layer (dW_l, db_l, dW_pool_l, db_pool_l).
+    dZ_l = dH_l * 1[Z_l > 0] (dZ_L = dlogits); dW_l = dZ^T [H_self || h_agg]; db_l = sum dZ;
+    dh_agg = dZ W_neigh;  dP[j,k] = sum of dh_agg[i,k] over the dst i with arg[i,k] = j;
+    dQ = dP * 1[Q > 0];  dW_pool = dQ^T H;  db_pool = sum dQ;
+    dH_{l-1} = dQ W_pool + pad(dZ W_self)."""
+    L = len(blocks)
+    grads = [None] * L
+    dH = np.asarray(dlogits, dtype=np.float64)
+    for l in range(L, 0, -1):
+        c = cache[l - 1]
+        W = np.asarray(Ws[l - 1], dtype=np.float64)
+        Wp = np.asarray(Wps[l - 1], dtype=np.float64)
+        H = c["H_in"]
+        d_in = H.shape[1]
+        dZ = dH if l == L else dH * (c["Z"] > 0)
+        n = dZ.shape[0]
+        dW = dZ.T @ np.concatenate([H[:n], c["agg"]], axis=1)
+        dagg = dZ @ W[:, d_in:]
+        dP = np.zeros_like(c["P"])
+        arg = c["arg"]
+        for i in range(n):
+            for k in range(d_in):
+                if arg[i, k] >= 0:
+                    dP[arg[i, k], k] += dagg[i, k]
+        dQ = dP * (c["Q"] > 0)
+        grads[l - 1] = (dW, dZ.sum(axis=0), dQ.T @ H, dQ.sum(axis=0))
+        if l > 1:
+            dHin = dQ @ Wp
+            dHin[:n] += dZ @ W[:, :d_in]
             dH = dHin
     return grads
 

@@ -198,6 +198,34 @@ def xavier_weights(dims, seed=WEIGHT_SEED, bias_scale=0.0):
     return Ws, bs
 
 
+def pool_weights(dims, seed=WEIGHT_SEED, bias_scale=0.0, dyadic=False):
+    """GraphSAGE-pool weights per layer l = 1..L: W_pool_l float32 [d_{l-1}, d_{l-1}]
+    (Xavier-uniform, Philox counter c0 = 64 + l so the stream is disjoint from the layer
+    weights) and b_pool_l [d_{l-1}].  dyadic=True rounds every value to a multiple of 2^-8
+    (exact products with k/128 features: the pool transform is then exact in fp32 for
+    d_{l-1} <= 256, so float-decided argmaxes agree with the oracle)."""
+    Wps, bps = [], []
+    for l in range(1, len(dims)):
+        d = dims[l - 1]
+        a = math.sqrt(6.0 / (2 * d))
+        r = np.arange(d, dtype=np.uint64)[:, None]
+        c = np.arange(d, dtype=np.uint64)[None, :]
+        w = words(seed, 64 + l, r, c >> np.uint64(2), TAG_WEIGHT)
+        sel = np.choose((c & np.uint64(3)).astype(np.int64), w)
+        u = (sel.astype(np.float64) + 0.5) / 4294967296.0
+        W = (2.0 * u - 1.0) * a
+        if bias_scale:
+            wb = words(seed, 64 + l, d + 7, np.arange(d, dtype=np.uint64), TAG_WEIGHT)[0]
+            b = ((wb.astype(np.float64) + 0.5) / 4294967296.0 * 2.0 - 1.0) * bias_scale
+        else:
+            b = np.zeros(d)
+        if dyadic:
+            W, b = np.round(W * 256.0) / 256.0, np.round(b * 256.0) / 256.0
+        Wps.append(W.astype(np.float32))
+        bps.append(b.astype(np.float32))
+    return Wps, bps
+
+
 # ----------------------------------------------------------------------------- configs
 @dataclass
 class Config:
