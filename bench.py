@@ -52,6 +52,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="products", choices=list(WORKLOADS))
     ap.add_argument("--gemm", default="bf16", choices=["bf16", "ffma"])
+    ap.add_argument("--aggregator", default="mean", choices=["mean", "pool"],
+                    help="pool: GraphSAGE-pool (SURVEY §8(f) NEXT 2), fp32 FFMA path only")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-baseline-seconds", type=float, default=20.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -239,7 +241,15 @@ def run_ours(args, cfg):
     t_gen = time.perf_counter()
     rp, col, X, y, seeds, Ws, bs = make_inputs_device(cfg)
     t_gen = time.perf_counter() - t_gen
+    pool = args.aggregator == "pool"
+    if pool:
+        args.gemm = "ffma"                             # the pool aggregator is built for fp32 only
     gemm = B.GEMM_BF16 if args.gemm == "bf16" else B.GEMM_FFMA
+    agg_kw = {}
+    if pool:
+        from synth.graphs import pool_weights
+        Wps, bps = pool_weights(cfg.dims)
+        agg_kw = dict(aggregator=B.AGG_POOL, Wps=Wps, bps=bps)
     feat_dtype = B.BF16 if args.gemm == "bf16" else B.FP32
     feats = X
     if feat_dtype == B.BF16:
@@ -254,12 +264,13 @@ def run_ours(args, cfg):
     t_c = time.perf_counter() - t_c
     tr = Trainer(graph, feats, y, seeds, cfg.dims,
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, mem_budget=budget,
-                 C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg)
+                 C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg,
+                 **agg_kw)
     if args.config == "products":
         # calibrate M_ctr once so that one GPU needs >= 8 groups, then freeze it for every N
         B_full = Trainer(graph, feats, y, seeds, cfg.dims,
                          cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, C_ppm=C_ppm,
-                         k_min=1, k_max=1)
+                         k_min=1, k_max=1, **agg_kw)
         _, _, est1, _ = B_full.schedule(0)
         del B_full
         tr.sched.mem_budget = int(est1[0]) // 8
@@ -277,7 +288,7 @@ def run_ours(args, cfg):
     clocks.start()
     # live roofline of the dominant kernel (k_gather_rows, the Aggregate): CUDA events around
     # each of its launches on its stream, algorithmic bytes from the edges it aggregated
-    B.profile_begin("gather", prof_counters)
+    B.profile_begin("pool_max" if pool else "gather", prof_counters)
     l0 = B.launch_count()
     step_ms, edges, sizes, ks = [], 0, [], []
     torch.cuda.synchronize()
@@ -346,10 +357,10 @@ def run_ours(args, cfg):
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
-        traffic = json.load(open(tpath)).get(f"{args.config}/{args.gemm}")
+        traffic = json.load(open(tpath)).get(f"{args.config}/{args.gemm}" + ("/pool" if pool else ""))
     if rank == 0:
         cpu = None
-        if world == 1 and not args.no_cpu_baseline:
+        if world == 1 and not args.no_cpu_baseline and not pool:   # (the pool oracle is loop-plain: tests only)
             rp_h, col_h, X_h, y_h, seeds_h = host_copies(rp, col, X, y, tr.seeds)
             cpu = oracle_sample(cfg, rp_h, col_h, X_h, y_h, seeds_h, Ws, bs, args.cpu_baseline_seconds)
         line = dict(
@@ -358,12 +369,15 @@ def run_ours(args, cfg):
             higher_is_better=True, scaling="strong", vs_baseline=None,
             dtype="bf16" if gemm == B.GEMM_BF16 else "f32", data="synthetic",
             config={"workload": WORKLOADS[args.config], "config": args.config, "K": ks[-1],
-                    "gemm": args.gemm, "l2": "flushed (512 MiB write) between timed steps",
+                    "gemm": args.gemm, "aggregator": args.aggregator,
+                    "l2": "flushed (512 MiB write) between timed steps",
                     "epoch_ms": total_ms / args.steps, "edges_per_epoch": edges / args.steps,
                     "parallelism": f"dp{world} over bucket groups",
                     "C_eq1": C_eq1, "C_ppm": C_ppm, "C_table2": C_TABLE2.get(args.config),
                     "C_seconds": t_c},
-            roofline={"bound": "hbm", "kernel": "k_gather_v2 (Aggregate: fwd neighbour mean, bwd transposed sum)",
+            roofline={"bound": "hbm",
+                      "kernel": ("k_pool_max (GraphSAGE-pool neighbour max + argmax)" if pool else
+                                 "k_gather_v2 (Aggregate: fwd neighbour mean, bwd transposed sum)"),
                       "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                       "traffic": traffic, "peak_source": peak_src,
                       "algorithmic_bytes_per_launch": g_bytes / max(1, g_launches),

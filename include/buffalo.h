@@ -42,6 +42,7 @@ typedef enum {
 
 enum { BUFFALO_FP32 = 0, BUFFALO_BF16 = 1 };            /* storage dtypes                  */
 enum { BUFFALO_GEMM_FFMA = 0, BUFFALO_GEMM_BF16 = 1 };  /* Update GEMM: fp32 SIMT | tcgen05 */
+enum { BUFFALO_AGG_MEAN = 0, BUFFALO_AGG_POOL = 1 };    /* GraphSAGE aggregator (R20, R28)  */
 enum { BUFFALO_MAX_LAYERS = 8, BUFFALO_MAX_FANOUT = 32, BUFFALO_MAX_DIM = 4096 };
 
 /* Input graph (the batch's host graph): CSR, rows sorted ascending, symmetric,
@@ -76,6 +77,7 @@ typedef struct {
   int32_t feat_dtype;
   int32_t gemm_mode;
   int64_t feat_pitch;
+  int32_t aggregator;       /* BUFFALO_AGG_MEAN (default) | BUFFALO_AGG_POOL (gemm_mode FFMA only) */
 } buffalo_model;
 
 /* Scheduler parameters (Alg. 3): mem_budget = M_ctr in bytes (arena bytes
@@ -127,6 +129,12 @@ typedef struct {
   float* dh;
   void* bwd_scratch;
   int64_t ld_agg, ld_out, ld_dh, bwd_scratch_bytes;
+  /* aggregator POOL only (else NULL / 0): P = ReLU(H_{l-1} W_pool^T + b_pool) fp32 [n_src][ld_pool]
+   * and the argmax of the neighbour max, int32 [n_dst][ld_pool] (local src index, -1 where
+   * the max is 0); block 1 then also carries its transpose (t_row_ptr, t_col, t_perm). */
+  float* pool_P;
+  int32_t* pool_arg;
+  int64_t ld_pool;
 } buffalo_block;
 
 typedef struct {
@@ -230,6 +238,40 @@ BUFFALO_API buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t la
                                 int64_t ld_dh_src, const int32_t* prev_row_ptr, void* scratch,
                                 size_t scratch_bytes, void* stream);
 
+/* ------------------------------------------------------------------ GraphSAGE-pool */
+/* the pooling aggregator (the paper's aggregator list "mean, pool or
+ * LSTM"; "applicable to any aggregators", :386; GraphSAGE [16]), reading R28.
+ * Forward of block `layer` (model.aggregator = BUFFALO_AGG_POOL, gemm_mode FFMA, fp32):
+ *   P = ReLU(H_{l-1} W_pool^T + b_pool) over the block's n_src input rows (layer 1: feature rows
+ *   via src_global), h_agg[i][k] = max over i's sampled neighbours j of P[j][k] (0 if D = 0),
+ *   arg[i][k] = that j, the first in CSR order (-1 where the max is 0), then the Update of
+ *   buffalo_sage_fwd: out = [H_self || h_agg] W^T + b (ReLU for l < L).
+ * W_pool fp32 [d_{l-1}][d_{l-1}] row-major, b_pool fp32 [d_{l-1}]; W / W_packed / b / out /
+ * saved_agg as buffalo_sage_fwd; P, arg: the block's pool_P / pool_arg (ld_pool >= pitch).
+ * Deterministic (every reduction order depends only on the row).  Errors: INVALID_ARG (nulls,
+ * leading dimensions), UNSUPPORTED (aggregator != POOL or gemm_mode != FFMA). */
+BUFFALO_API buffalo_status buffalo_pool_fwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                const void* h_src, int64_t ld_src, const float* W_pool,
+                                const float* b_pool, const float* W, const void* W_packed,
+                                const float* b, void* out, int64_t ld_out, void* saved_agg,
+                                int64_t ld_agg, float* P, int32_t* arg, int64_t ld_pool,
+                                void* stream);
+/* Backward of buffalo_pool_fwd (gradients accumulated in place, +=):
+ *   dZ = dh_dst * 1[h_dst > 0] (l < L, in place; l = L: dh_dst = dlogits);
+ *   dW += dZ^T [H_self || h_agg], db += sum dZ;  dh_agg = dZ W_neigh;
+ *   dP[j][k] = sum of dh_agg[i][k] over the dst i with arg[i][k] = j, ascending i through the
+ *   transposed block (deterministic);  dQ = dP * 1[P > 0];  dW_pool += dQ^T H_{l-1},
+ *   db_pool += sum dQ;  dh_src (l >= 2, NULL at l = 1) = dQ W_pool + pad(dZ W_self).
+ * scratch: the block's bwd_scratch (buffalo_sage_bwd_scratch_bytes). */
+BUFFALO_API buffalo_status buffalo_pool_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
+                                const void* saved_agg, int64_t ld_agg, const void* h_dst,
+                                int64_t ld_hdst, const float* P, const int32_t* arg, int64_t ld_pool,
+                                const float* W_pool, const float* W, float* dW_pool_accum,
+                                float* db_pool_accum, float* dW_accum, float* db_accum,
+                                float* dh_src, int64_t ld_dh_src, void* scratch,
+                                size_t scratch_bytes, void* stream);
+
 /* ------------------------------------------------------------------ a10: optimizer */
 /* SGD (Alg. 2 l.13, R18): param -= lr * grad; grad = 0 (ready for the next epoch). */
 BUFFALO_API buffalo_status buffalo_sgd_step(float* param, float* grad, int64_t n, float lr, void* stream);
@@ -268,7 +310,9 @@ BUFFALO_API buffalo_status buffalo_avg_clustering(const buffalo_graph* g, const 
 BUFFALO_API int64_t buffalo_launch_count(void);
 
 /* Diagnostics (bench roofline): time every launch of one kernel family with CUDA events on the
- * stream it is launched on.  family "gather": k_gather_rows, the Aggregate of the forward (mean
+ * stream it is launched on.  family "pool_max": k_pool_max, the GraphSAGE-pool neighbour max
+ * (per row 12 B + the max and argmax rows, per edge the index and the pooled fp32 row).
+ * family "gather": k_gather_rows, the Aggregate of the forward (mean
  * of neighbour rows) and of the backward (sum of dZ/D rows over the transposed block).
  * counters: caller's device buffer of max_launches uint64 (edges each launch aggregated);
  * launches beyond min(max_launches, 4096) are not timed.  Not thread-safe; one family at a time.

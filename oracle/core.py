@@ -319,11 +319,11 @@ def grouping_weight(M, I, E, C_ppm):
     return min(M, (M * I * 1_000_000) // (E * C_ppm))
 
 
-def item_stats(g, seeds, L, fanout, seed, dims, act_dtype):
+def item_stats(g, seeds, L, fanout, seed, dims, act_dtype, aggregator="mean"):
     """O, E = sum D, I = unique src of the item's own output block, sizes, M_est (R13, R15)."""
     seeds = np.asarray(seeds, dtype=np.int32)
     n, e = block_sizes(g, seeds, L, fanout, seed)
-    lo, hi = mem_model(n, e, dims, act_dtype)
+    lo, hi = mem_model(n, e, dims, act_dtype, aggregator)
     return dict(O=int(seeds.size), E=int(e[L - 1]), I=int(n[L - 1]), n=n, e=e, M=hi)
 
 
@@ -349,7 +349,7 @@ def mem_balanced_grouping(items, K, M_ctr):
 
 
 def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT64_MAX,
-             C_ppm=0, k_min=1, k_max=4096, num_gpus=1):
+             C_ppm=0, k_min=1, k_max=4096, num_gpus=1, aggregator="mean"):
     """Alg. 3 Buffalo_Scheduler with the readings of DESIGN.md
     (R7 explosion test, R11 sort/placement keys, R16 K_max, R17 empty groups dropped,
     R27 k_min = #GPUs and LPT rank assignment).  Returns a dict plan or None (budget)."""
@@ -360,7 +360,7 @@ def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT6
     stats = {}
     for d in range(F + 1):
         if pos_of[d].size:
-            st = item_stats(g, seeds[pos_of[d]], L, fanout, seed, dims, act_dtype)
+            st = item_stats(g, seeds[pos_of[d]], L, fanout, seed, dims, act_dtype, aggregator)
             st["w"] = grouping_weight(st["M"], st["I"], st["E"], C_ppm)
             stats[d] = st
     non_split = [d for d in stats if d != F]
@@ -380,7 +380,7 @@ def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT6
                 for k, piece in enumerate(split_explosion(pos_of[F], K)):
                     if piece.size == 0:
                         continue
-                    st = item_stats(g, seeds[piece], L, fanout, seed, dims, act_dtype)
+                    st = item_stats(g, seeds[piece], L, fanout, seed, dims, act_dtype, aggregator)
                     st["w"] = grouping_weight(st["M"], st["I"], st["E"], C_ppm)
                     items.append(dict(d=F, k=k, pos=piece, **st))
             else:

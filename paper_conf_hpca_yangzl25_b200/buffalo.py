@@ -20,6 +20,7 @@ c_i32, c_i64, c_u64, c_p, c_sz, c_f = (ctypes.c_int32, ctypes.c_int64, ctypes.c_
 OK, ERR_INVALID_ARG, ERR_BUDGET, ERR_CAPACITY, ERR_CUDA, ERR_UNSUPPORTED = range(6)
 FP32, BF16 = 0, 1
 GEMM_FFMA, GEMM_BF16 = 0, 1
+AGG_MEAN, AGG_POOL = 0, 1
 MAX_LAYERS = 8
 
 EXPORTS = [
@@ -30,6 +31,7 @@ EXPORTS = [
     "buffalo_estimate_mem", "buffalo_launch_count", "buffalo_profile_begin", "buffalo_profile_end",
     "buffalo_status_str", "buffalo_last_error",
     "buffalo_clustering_workspace_bytes", "buffalo_triangles", "buffalo_avg_clustering",
+    "buffalo_pool_fwd", "buffalo_pool_bwd",
 ]
 
 
@@ -53,7 +55,7 @@ class Sampler(ctypes.Structure):
 
 class Model(ctypes.Structure):
     _fields_ = [("num_layers", c_i32), ("dim", c_i32 * (MAX_LAYERS + 1)), ("feat_dtype", c_i32),
-                ("gemm_mode", c_i32), ("feat_pitch", c_i64)]
+                ("gemm_mode", c_i32), ("feat_pitch", c_i64), ("aggregator", c_i32)]
 
 
 class Sched(ctypes.Structure):
@@ -74,7 +76,8 @@ class Block(ctypes.Structure):
                 ("row_ptr", c_p), ("col_local", c_p), ("col_global", c_p), ("src_global", c_p),
                 ("t_row_ptr", c_p), ("t_col", c_p), ("heavy", c_p), ("cls_perm", c_p), ("t_perm", c_p),
                 ("agg", c_p), ("out", c_p), ("dh", c_p), ("bwd_scratch", c_p),
-                ("ld_agg", c_i64), ("ld_out", c_i64), ("ld_dh", c_i64), ("bwd_scratch_bytes", c_i64)]
+                ("ld_agg", c_i64), ("ld_out", c_i64), ("ld_dh", c_i64), ("bwd_scratch_bytes", c_i64),
+                ("pool_P", c_p), ("pool_arg", c_p), ("ld_pool", c_i64)]
 
 
 class Blocks(ctypes.Structure):
@@ -114,6 +117,9 @@ def lib(require_gpu=True):
             "buffalo_clustering_workspace_bytes": (c_sz, [P]),
             "buffalo_triangles": (c_i32, [P, P, P, c_sz, P]),
             "buffalo_avg_clustering": (c_i32, [P, P, P, P, P, c_sz, P]),
+            "buffalo_pool_fwd": (c_i32, [P, c_i32, P, P, c_i64, P, P, P, P, P, P, c_i64, P, c_i64, P, P, c_i64, P]),
+            "buffalo_pool_bwd": (c_i32, [P, c_i32, P, P, c_i64, P, c_i64, P, c_i64, P, c_i64, P, P, c_i64, P, P,
+                                         P, P, P, P, P, c_i64, P, c_sz, P]),
             "buffalo_status_str": (ctypes.c_char_p, [c_i32]),
             "buffalo_last_error": (ctypes.c_char_p, []),
         }
@@ -218,6 +224,21 @@ def sage_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg,
                                   scratch_bytes, stream_ptr(stream)))
 
 
+def pool_fwd(blk, layer, model, h_src, ld_src, W_pool, b_pool, W, W_packed, b, out, ld_out, saved_agg, ld_agg,
+             P, arg, ld_pool, stream=None):
+    _check(lib().buffalo_pool_fwd(ref(blk), layer, ref(model), ptr(h_src), ld_src, ptr(W_pool), ptr(b_pool), ptr(W),
+                                  ptr(W_packed), ptr(b), ptr(out), ld_out, ptr(saved_agg), ld_agg, ptr(P), ptr(arg),
+                                  ld_pool, stream_ptr(stream)))
+
+
+def pool_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg, h_dst, ld_hdst, P, arg, ld_pool,
+             W_pool, W, dW_pool, db_pool, dW, db, dh_src, ld_dh_src, scratch, scratch_bytes, stream=None):
+    _check(lib().buffalo_pool_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh, ptr(h_src), ld_src,
+                                  ptr(saved_agg), ld_agg, ptr(h_dst), ld_hdst, ptr(P), ptr(arg), ld_pool,
+                                  ptr(W_pool), ptr(W), ptr(dW_pool), ptr(db_pool), ptr(dW), ptr(db), ptr(dh_src),
+                                  ld_dh_src, ptr(scratch), scratch_bytes, stream_ptr(stream)))
+
+
 def sgd_step(param, grad, lr, stream=None):
     _check(lib().buffalo_sgd_step(ptr(param), ptr(grad), param.numel(), lr, stream_ptr(stream)))
 
@@ -286,7 +307,7 @@ def make_sampler(fanout, F, seed):
     return s
 
 
-def make_model(dims, feat_dtype=FP32, gemm_mode=GEMM_FFMA, feat_pitch=None):
+def make_model(dims, feat_dtype=FP32, gemm_mode=GEMM_FFMA, feat_pitch=None, aggregator=AGG_MEAN):
     m = Model()
     m.num_layers = len(dims) - 1
     for i, d in enumerate(dims):
@@ -294,6 +315,7 @@ def make_model(dims, feat_dtype=FP32, gemm_mode=GEMM_FFMA, feat_pitch=None):
     m.feat_dtype = feat_dtype
     m.gemm_mode = gemm_mode
     m.feat_pitch = int(feat_pitch if feat_pitch else ((dims[0] + 7) // 8) * 8)
+    m.aggregator = int(aggregator)
     return m
 
 

@@ -90,6 +90,7 @@ __global__ void k_fill_i32(int32_t* a, int64_t n, int32_t v) {
 // ------------------------------------------------------------------ memory model (R15)
 // Restated from DESIGN.md §5; must agree with the arena that buffalo_build_blocks lays out.
 static int64_t bwd_scratch_for(const buffalo_model* m, int64_t n_dst, int64_t n_src, int64_t e, int l) {
+  if (m->aggregator == BUFFALO_AGG_POOL) return pool_bwd_scratch_bytes(n_dst, n_src, m->dim[l - 1], m->dim[l]);
   if (m->gemm_mode == BUFFALO_GEMM_BF16)
     return tc_bwd_scratch_bytes(n_dst, n_src, e, l, m->dim[l - 1], m->dim[l], l == m->num_layers);
   return bwd_scratch_bytes(n_dst, n_src, l, m->dim[l - 1], m->dim[l]);
@@ -106,18 +107,23 @@ static int64_t dh_slot_bytes(const buffalo_model* m, int64_t n, int l) {
 static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_model* m,
                       int64_t* lo, int64_t* hi) {
   const int64_t s = m->gemm_mode == BUFFALO_GEMM_BF16 ? 2 : 4;
+  const bool pool = m->aggregator == BUFFALO_AGG_POOL;    // R28: block 1 keeps a transpose too
   int64_t blocks = 0, build = 0, acts = 0, bwd = 0;
   for (int l = 1; l <= L; ++l) {
     const int64_t nl = n[l], nm = n[l - 1], el = e[l - 1];
     blocks += R(4 * (nl + 1)) + R(4 * nl) + R(4 * el) + R(4 * nm);
     blocks += (l == 1) ? R(4 * el) : R(4 * (nm + 1)) + R(4 * el) + R(4 * nm);
-    build = std::max(build, build_frame_bytes(nl, el, l, false));
+    if (l == 1 && pool) blocks += R(4 * (nm + 1)) + R(4 * el) + R(4 * nm);
+    build = std::max(build, build_frame_bytes(nl, el, l, false, pool));
   }
   for (int l = 1; l <= L; ++l) {
     acts += R(n[l] * pitch_of(m->dim[l - 1]) * s);
     if (l < L) acts += R(n[l] * pitch_of(m->dim[l]) * s);
   }
   acts += R(n[L] * pitch_of(m->dim[L]) * 4);
+  if (pool)
+    for (int l = 1; l <= L; ++l)   // P [n_{l-1}] and argmax [n_l] rows of width pitch(d_{l-1})
+      acts += R(n[l - 1] * pitch_of(m->dim[l - 1]) * 4) + R(n[l] * pitch_of(m->dim[l - 1]) * 4);
   for (int l = L; l >= 1; --l) {
     int64_t f = dh_slot_bytes(m, n[l], l);
     if (l >= 2) f += dh_slot_bytes(m, n[l - 1], l - 1);
@@ -146,6 +152,14 @@ static buffalo_status validate_model(const buffalo_model* m) {
         set_error("model: the bf16 tensor-core path supports dim[l] <= 256 for l >= 1");
         return BUFFALO_ERR_UNSUPPORTED;
       }
+  if (m->aggregator != BUFFALO_AGG_MEAN && m->aggregator != BUFFALO_AGG_POOL) {
+    set_error("model: unknown aggregator %d", m->aggregator);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (m->aggregator == BUFFALO_AGG_POOL && m->gemm_mode != BUFFALO_GEMM_FFMA) {
+    set_error("model: the pool aggregator is built for gemm_mode FFMA (fp32) only");
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
   if (m->feat_pitch < round_up(m->dim[0], 8) || m->feat_pitch % 8) {
     set_error("model: feat_pitch must be a multiple of 8 and >= round_up(dim[0], 8)");
     return BUFFALO_ERR_INVALID_ARG;
@@ -271,7 +285,8 @@ const char* buffalo_last_error(void) { return g_err.c_str(); }
 int64_t buffalo_launch_count(void) { return g_launches.load(); }
 
 buffalo_status buffalo_profile_begin(const char* family, void* counters, int64_t max_launches, void* stream) {
-  if (!family || (std::string(family) != "gather") || !counters || max_launches <= 0) {
+  if (!family || (std::string(family) != "gather" && std::string(family) != "pool_max") || !counters ||
+      max_launches <= 0) {
     set_error("profile_begin: unknown kernel family or no counter buffer");
     return BUFFALO_ERR_INVALID_ARG;
   }
@@ -603,7 +618,8 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
       known[1] = sizes_h[l - 1];      // n_{l-1}
     }
     buffalo_status st = build_layer(g, dst, nd, sp->fanout[l - 1], (uint32_t)(L - l + 1), sp->seed, l,
-                                    false, A, b, s, sizes_h ? known : nullptr);
+                                    false, A, b, s, sizes_h ? known : nullptr,
+                                    m->aggregator == BUFFALO_AGG_POOL);
     if (st == BUFFALO_ERR_CAPACITY || A.overflow) {
       if (required_bytes_h) *required_bytes_h = A.need;
       set_error("build_blocks: arena of %lld bytes too small (need >= %lld)", (long long)A.cap,
@@ -627,6 +643,13 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
     b->ld_out = pitch_of(m->dim[l]);
     b->out = A.take(b->n_dst * b->ld_out * (l < L ? sa : 4));
   }
+  if (m->aggregator == BUFFALO_AGG_POOL)
+    for (int l = 1; l <= L; ++l) {
+      buffalo_block* b = &out->layer[l - 1];
+      b->ld_pool = pitch_of(m->dim[l - 1]);
+      b->pool_P = (float*)A.take(b->n_src * b->ld_pool * 4);
+      b->pool_arg = (int32_t*)A.take(b->n_dst * b->ld_pool * 4);
+    }
   // backward region: ping-pong dH buffers at the two ends, scratch in between
   int64_t B = 0;
   std::vector<int64_t> ah(L + 1, 0), tmp(L + 1, 0);
@@ -683,6 +706,10 @@ buffalo_status buffalo_sage_fwd(const buffalo_block* blk, int32_t layer, const b
                                 int64_t ld_agg, void* stream) {
   BF_CHECK(require_sm100());
   BF_CHECK(validate_model(m));
+  if (m->aggregator != BUFFALO_AGG_MEAN) {
+    set_error("sage_fwd: model.aggregator is not MEAN (use buffalo_pool_fwd)");
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
   if (!blk || layer < 1 || layer > m->num_layers || !h_src || !W || !W_packed || !out || !saved_agg) {
     set_error("sage_fwd: null argument or bad layer");
     return BUFFALO_ERR_INVALID_ARG;
@@ -730,6 +757,10 @@ buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const b
                                 void* scratch, size_t scratch_bytes, void* stream) {
   BF_CHECK(require_sm100());
   BF_CHECK(validate_model(m));
+  if (m->aggregator != BUFFALO_AGG_MEAN) {
+    set_error("sage_bwd: model.aggregator is not MEAN (use buffalo_pool_bwd)");
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
   if (!blk || layer < 1 || layer > m->num_layers || !dh_dst || !h_src || !saved_agg || !W ||
       !dW_accum || !db_accum || !scratch) {
     set_error("sage_bwd: null argument or bad layer");
@@ -777,6 +808,113 @@ buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const b
     return tc_sage_bwd(a, s);
   }
   return sage_bwd_ffma(a, s);
+}
+
+static buffalo_status pool_args(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                 const void* h_src, int64_t ld_src, PoolArgs& a, const char* who) {
+  BF_CHECK(require_sm100());
+  BF_CHECK(validate_model(m));
+  if (m->aggregator != BUFFALO_AGG_POOL) {
+    set_error("%s: model.aggregator is not BUFFALO_AGG_POOL", who);
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
+  if (!blk || layer < 1 || layer > m->num_layers || !h_src) {
+    set_error("%s: null argument or bad layer", who);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  a = PoolArgs{};
+  a.blk = blk;
+  a.layer1 = layer == 1;
+  a.in_bf16 = a.layer1 && m->feat_dtype == BUFFALO_BF16;
+  a.last = layer == m->num_layers;
+  a.d_in = m->dim[layer - 1];
+  a.d_out = m->dim[layer];
+  a.h_src = h_src;
+  a.ld_src = a.layer1 ? m->feat_pitch : ld_src;
+  if (a.ld_src < pitch_of(a.d_in) || a.ld_src % 8) {
+    set_error("%s: ld_src must be a multiple of 8 and >= pitch(d_in)", who);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  return BUFFALO_OK;
+}
+
+buffalo_status buffalo_pool_fwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                const void* h_src, int64_t ld_src, const float* W_pool, const float* b_pool,
+                                const float* W, const void* W_packed, const float* b, void* out, int64_t ld_out,
+                                void* saved_agg, int64_t ld_agg, float* P, int32_t* arg, int64_t ld_pool,
+                                void* stream) {
+  PoolArgs a;
+  BF_CHECK(pool_args(blk, layer, m, h_src, ld_src, a, "pool_fwd"));
+  if (!W_pool || !b_pool || !W || !W_packed || !b || !out || !saved_agg || !P || !arg) {
+    set_error("pool_fwd: null argument");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (ld_out < pitch_of(a.d_out) || ld_agg < pitch_of(a.d_in) || ld_pool < pitch_of(a.d_in) || ld_out % 8 ||
+      ld_agg % 8 || ld_pool % 8) {
+    set_error("pool_fwd: leading dimensions must be multiples of 8 and >= the padded widths");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  a.W_pool = W_pool;
+  a.b_pool = b_pool;
+  a.W = W;
+  a.W_packed = (const float*)W_packed;
+  a.b = b;
+  a.out = (float*)out;
+  a.ld_out = ld_out;
+  a.agg = (float*)saved_agg;
+  a.ld_agg = ld_agg;
+  a.P = P;
+  a.arg = arg;
+  a.ld_pool = ld_pool;
+  return pool_fwd_ffma(a, (cudaStream_t)stream);
+}
+
+buffalo_status buffalo_pool_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
+                                const void* saved_agg, int64_t ld_agg, const void* h_dst, int64_t ld_hdst,
+                                const float* P, const int32_t* arg, int64_t ld_pool, const float* W_pool,
+                                const float* W, float* dW_pool_accum, float* db_pool_accum, float* dW_accum,
+                                float* db_accum, float* dh_src, int64_t ld_dh_src, void* scratch,
+                                size_t scratch_bytes, void* stream) {
+  PoolArgs a;
+  BF_CHECK(pool_args(blk, layer, m, h_src, ld_src, a, "pool_bwd"));
+  if (!dh_dst || !saved_agg || !P || !arg || !W_pool || !W || !dW_pool_accum || !db_pool_accum || !dW_accum ||
+      !db_accum || !scratch || (!a.last && !h_dst)) {
+    set_error("pool_bwd: null argument");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (!blk->t_row_ptr || !blk->t_col) {
+    set_error("pool_bwd: the block has no transpose (build it with model.aggregator = POOL)");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (dh_src && layer == 1) {
+    set_error("pool_bwd: no dh_src at layer 1 (features are not trained)");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if ((int64_t)scratch_bytes < pool_bwd_scratch_bytes(blk->n_dst, blk->n_src, a.d_in, a.d_out)) {
+    set_error("pool_bwd: scratch too small");
+    return BUFFALO_ERR_CAPACITY;
+  }
+  a.dh = dh_dst;
+  a.ld_dh = ld_dh;
+  a.agg = (float*)saved_agg;
+  a.ld_agg = ld_agg;
+  a.h_dst = (const float*)h_dst;
+  a.ld_hdst = ld_hdst;
+  a.P = (float*)P;
+  a.arg = (int32_t*)arg;
+  a.ld_pool = ld_pool;
+  a.W_pool = W_pool;
+  a.W = W;
+  a.dW_pool = dW_pool_accum;
+  a.db_pool = db_pool_accum;
+  a.dW = dW_accum;
+  a.db = db_accum;
+  a.dh_src = dh_src;
+  a.ld_dh_src = ld_dh_src;
+  a.scratch = scratch;
+  a.scratch_bytes = (int64_t)scratch_bytes;
+  return pool_bwd_ffma(a, (cudaStream_t)stream);
 }
 
 buffalo_status buffalo_softmax_ce(const float* logits, int64_t ld, int64_t n, int32_t classes,

@@ -306,7 +306,7 @@ static buffalo_status d2h_i32(const int32_t* d, int32_t* h, cudaStream_t s) {
   return BUFFALO_OK;
 }
 
-int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only) {
+int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only, bool t1) {
   const int64_t pc = part_count_elems(e);
   if (sizes_only) {
     const int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pc + 1);
@@ -316,12 +316,13 @@ int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only) 
   const int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pne + 1);
   int64_t fr = R(64) + R(4 * scan_ws_elems(scan_len)) + R(4 * (pne + 1));
   if (layer >= 2) fr += R(4 * e) + R(4 * (n_dst + e));        // col_global + transposed-fill cursors
+  else if (t1) fr += R(4 * (n_dst + e));                       // block 1: cursors (col_global persists)
   return fr;
 }
 
 buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
                            uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
-                           buffalo_block* blk, cudaStream_t s, const int64_t* known) {
+                           buffalo_block* blk, cudaStream_t s, const int64_t* known, bool t1) {
   memset(blk, 0, sizeof(*blk));
   blk->n_dst = n_dst;
   int32_t* rp = (int32_t*)A.take(4 * (n_dst + 1));
@@ -361,7 +362,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   const int64_t scan_len = std::max<int64_t>(n_dst + e + 1, pc + 1);
   int32_t* col_local = (!sizes_only) ? (int32_t*)A.take(4 * e) : nullptr;
   int32_t* colg_persist = (!sizes_only && layer == 1) ? (int32_t*)A.take(4 * e) : nullptr;
-  fr = A.push_frame(build_frame_bytes(n_dst, e, layer, sizes_only));
+  fr = A.push_frame(build_frame_bytes(n_dst, e, layer, sizes_only, t1));
   if (A.overflow) return BUFFALO_ERR_CAPACITY;
   totals = (int32_t*)fr;
   char* q = fr + R(64);
@@ -421,7 +422,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   blk->n_src = n_src;
   blk->src_global = src;
   blk->col_global = colg_persist;
-  const bool transpose = !sizes_only && layer >= 2;
+  const bool transpose = !sizes_only && (layer >= 2 || t1);
   int32_t *trp = nullptr, *tcol = nullptr, *tperm = nullptr;
   if (transpose) {
     trp = (int32_t*)A.take(4 * (n_src + 1));

@@ -8,7 +8,8 @@
 
 namespace buffalo {
 
-int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only);
+// t1: block 1 also gets its transpose (GraphSAGE-pool's backward scatters through it, R28).
+int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only, bool t1 = false);
 
 // Graph workspace (buffalo_graph_workspace_bytes): node_map int32[N] (INT32_MAX when idle), the
 // relabel bitmap uint32[W] (zero when idle), its word prefix int32[W + 1] and a scan workspace,
@@ -42,7 +43,8 @@ inline GraphWs graph_ws(const buffalo_graph* g) {
 // the sizes (twice, three times for layers >= 2).
 buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
                            uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
-                           buffalo_block* blk, cudaStream_t s, const int64_t* known = nullptr);
+                           buffalo_block* blk, cudaStream_t s, const int64_t* known = nullptr,
+                           bool t1 = false);
 
 // Degree bucketing of the seeds (Alg. 3 l.1): bucket[i] = min(D(seed_i), F); order = seed
 // positions grouped by bucket (stable); sorted_ids = seeds[order]; hist_h[0..F].

@@ -214,7 +214,8 @@ static buffalo_status launch_agg(const buffalo_block* blk, const int32_t* col, c
 // A1 row r is A1[gidx ? gidx[r] : r] and is zero for r >= m1.
 constexpr int GB_M = 64, GB_N = 64, GB_K = 16;
 
-template <class TA1, class TA2, class TO>
+// TB: B1 is read transposed (B1[k][n] = B1t[n][k], ldb1 = row pitch of B1t).
+template <class TA1, class TA2, class TO, bool TB = false>
 __global__ void __launch_bounds__(256) k_gemm2(int64_t M, int N, int Np, int K1, int K2,
                                                const TA1* __restrict__ A1, int64_t lda1,
                                                const int32_t* __restrict__ gidx, int64_t m1,
@@ -260,7 +261,8 @@ __global__ void __launch_bounds__(256) k_gemm2(int64_t M, int N, int Np, int K1,
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const int nn = n0 + bn + q;
-        Bs[bk][bn + q] = (k < K && nn < N) ? __ldg(B + (int64_t)k * ldb + nn) : 0.f;
+        Bs[bk][bn + q] = (k < K && nn < N) ? __ldg(TB && first ? B + (int64_t)nn * ldb + k : B + (int64_t)k * ldb + nn)
+                                           : 0.f;
       }
     }
     __syncthreads();
@@ -338,8 +340,9 @@ __global__ void __launch_bounds__(256) k_aggT(const int32_t* __restrict__ trp, c
 
 // dW partial of split s: part[s][n][k] = sum_{r in split s} dZ[r][n] * Afwd[r][k],
 // Afwd[r] = [self(r) || agg(r)].
+// K = 2 d_in (Update weight: [self || agg]) or d_in (pool weight: self rows only).
 template <class TS, class TG>
-__global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, int d_in,
+__global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, int d_in, int K,
                                                     const float* __restrict__ dz, int64_t ldz,
                                                     const TS* __restrict__ self, int64_t lds,
                                                     const int32_t* __restrict__ gidx,
@@ -352,7 +355,6 @@ __global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, in
   const int k0 = blockIdx.x * 64, n0 = blockIdx.y * 64;
   const int64_t r_beg = (int64_t)blockIdx.z * rows_per_split;
   const int64_t r_end = min(nrows, r_beg + rows_per_split);
-  const int K = 2 * d_in;
   float acc[4][4] = {};
   float dbs[4] = {0.f, 0.f, 0.f, 0.f};      // column sums of dZ (CTAs of k-tile 0, threads ty == 0)
   const bool do_db = blockIdx.x == 0 && ty == 0;
@@ -583,7 +585,7 @@ static buffalo_status bwd_ffma_t(const BwdArgs& a, cudaStream_t s) {
   const int64_t rps = ceil_div(n > 0 ? n : 1, S);
   if (n > 0) {
     dim3 g((unsigned)ceil_div(2 * d_in, 64), (unsigned)ceil_div(d_out, 64), (unsigned)S);
-    k_dw_partial<TS, TG><<<g, 256, 0, s>>>(n, d_out, d_in, a.dh, a.ld_dh, (const TS*)a.h_src, a.ld_src,
+    k_dw_partial<TS, TG><<<g, 256, 0, s>>>(n, d_out, d_in, 2 * d_in, a.dh, a.ld_dh, (const TS*)a.h_src, a.ld_src,
                                            a.layer1 ? blk->src_global : nullptr, (const TG*)a.agg,
                                            a.ld_agg, rps, dw_part, db_part);
     BF_LAUNCHED("k_dw_partial");
@@ -615,6 +617,189 @@ buffalo_status sage_bwd_ffma(const BwdArgs& a, cudaStream_t s) {
   if (a.in_bf16 && !a.act_bf16) return bwd_ffma_t<__nv_bfloat16, float, float>(a, s);
   if (!a.in_bf16 && a.act_bf16) return bwd_ffma_t<float, __nv_bfloat16, __nv_bfloat16>(a, s);
   return bwd_ffma_t<float, float, float>(a, s);
+}
+
+// ================================================================== GraphSAGE-pool (R28)
+// Neighbour max of the pooled rows: warp per dst row (degree-class order), each lane owns
+// 4-column chunks; strict '>' keeps the first neighbour (CSR order) attaining the max; the
+// running max starts at 0 (P >= 0), so arg = -1 exactly where the max is 0 (or D = 0).
+__global__ void __launch_bounds__(256) k_pool_max(const int32_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                                  const int32_t* __restrict__ perm, int64_t n,
+                                                  const float* __restrict__ P, int64_t ldp, int d,
+                                                  float* __restrict__ agg, int64_t ld_agg,
+                                                  int32_t* __restrict__ arg, int64_t ld_arg) {
+  const int lane = threadIdx.x & 31;
+  const int nch = (int)(pitch_of(d) / 4);
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < n; w += warps) {
+    const int64_t i = perm ? perm[w] : w;
+    const int32_t e0 = rp[i], e1 = rp[i + 1];
+    for (int c = lane; c < nch; c += 32) {
+      float best[4] = {0.f, 0.f, 0.f, 0.f};
+      int32_t am[4] = {-1, -1, -1, -1};
+      for (int32_t e = e0; e < e1; ++e) {
+        const int32_t j = col[e];
+        float v[4];
+        VecIO<float, 4>::load(P + (int64_t)j * ldp + c * 4, v);
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (v[q] > best[q]) { best[q] = v[q]; am[q] = j; }
+      }
+      VecIO<float, 4>::store(agg + i * ld_agg + c * 4, best);
+      *reinterpret_cast<int4*>(arg + i * ld_arg + c * 4) = make_int4(am[0], am[1], am[2], am[3]);
+    }
+  }
+}
+
+// dQ[j] = 1[P[j] > 0] * sum over the dst i of src j (transposed block, ascending i) of
+// dh_agg[i] restricted to the columns whose argmax is j.  Warp per src row.
+__global__ void __launch_bounds__(256) k_pool_scatterT(const int32_t* __restrict__ trp, const int32_t* __restrict__ tcol,
+                                                       int64_t n_src, const int32_t* __restrict__ arg, int64_t ld_arg,
+                                                       const float* __restrict__ dagg, int64_t ld_dagg,
+                                                       const float* __restrict__ P, int64_t ldp, int d,
+                                                       float* __restrict__ dq, int64_t ldq) {
+  const int lane = threadIdx.x & 31;
+  const int nch = (int)(pitch_of(d) / 4);
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t j = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; j < n_src; j += warps) {
+    const int32_t t0 = trp[j], t1 = trp[j + 1];
+    for (int c = lane; c < nch; c += 32) {
+      float acc[4] = {0.f, 0.f, 0.f, 0.f};
+      for (int32_t t = t0; t < t1; ++t) {
+        const int64_t i = tcol[t];
+        const int4 a4 = __ldg(reinterpret_cast<const int4*>(arg + i * ld_arg + c * 4));
+        float g[4];
+        VecIO<float, 4>::load(dagg + i * ld_dagg + c * 4, g);
+        acc[0] += a4.x == (int32_t)j ? g[0] : 0.f;
+        acc[1] += a4.y == (int32_t)j ? g[1] : 0.f;
+        acc[2] += a4.z == (int32_t)j ? g[2] : 0.f;
+        acc[3] += a4.w == (int32_t)j ? g[3] : 0.f;
+      }
+      float p[4];
+      VecIO<float, 4>::load(P + j * ldp + c * 4, p);
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        if (!(p[q] > 0.f) || c * 4 + q >= d) acc[q] = 0.f;
+      VecIO<float, 4>::store(dq + j * ldq + c * 4, acc);
+    }
+  }
+}
+
+int pool_dw_splits(int64_t n_rows, int d) {
+  const int64_t tiles = ceil_div(d, 64) * ceil_div(d, 64);
+  const int64_t a = ceil_div(296, tiles), b = ceil_div(n_rows, 512);
+  const int64_t sp = a < b ? a : b;
+  return (int)(sp < 1 ? 1 : sp);
+}
+
+// Layout of the pool backward scratch (R15 restated in DESIGN.md §5): dW/db partials of the
+// Update weight, dh_agg, dQ, dW_pool/db_pool partials.
+int64_t pool_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int d_in, int d_out) {
+  const int S = dw_splits(n_dst, d_out, d_in), S2 = pool_dw_splits(n_src, d_in);
+  return R((int64_t)S * d_out * 2 * d_in * 4) + R((int64_t)S * pitch_of(d_out) * 4) +
+         R(n_dst * pitch_of(d_in) * 4) + R(n_src * pitch_of(d_in) * 4) +
+         R((int64_t)S2 * d_in * d_in * 4) + R((int64_t)S2 * pitch_of(d_in) * 4);
+}
+
+template <class TI>
+static buffalo_status pool_fwd_t(const PoolArgs& a, cudaStream_t s) {
+  const buffalo_block* blk = a.blk;
+  const int64_t ns = blk->n_src, nd = blk->n_dst;
+  const int dp = (int)pitch_of(a.d_in);
+  const int32_t* gidx = a.layer1 ? blk->src_global : nullptr;
+  if (ns > 0) {   // P = ReLU(H W_pool^T + b_pool)
+    dim3 grid((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dp, GB_N));
+    k_gemm2<TI, float, float, true><<<grid, 256, 0, s>>>(ns, a.d_in, dp, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
+                                                        gidx, ns, nullptr, 0, a.W_pool, a.d_in, nullptr, 0,
+                                                        a.b_pool, 1, a.P, a.ld_pool);
+    BF_LAUNCHED("k_gemm2");
+  }
+  if (nd <= 0) return BUFFALO_OK;
+  const ProfSlot ps = prof_begin_launch("pool_max", s);
+  k_pool_max<<<grid_for(nd * 32, 256, 16), 256, 0, s>>>(blk->row_ptr, blk->col_local, blk->cls_perm, nd, a.P,
+                                                        a.ld_pool, a.d_in, a.agg, a.ld_agg, a.arg, a.ld_pool);
+  BF_LAUNCHED("k_pool_max");
+  // algorithmic bytes: per row perm + row_ptr pair + the max and argmax rows written; per edge
+  // the index and the pooled source row (the edge count is known on the host: no counter)
+  prof_end_launch(ps, s, (double)nd * (12.0 + 8.0 * dp) + (double)blk->n_edges * (4.0 + 4.0 * dp), 0.0);
+  const int Np = (int)pitch_of(a.d_out);
+  dim3 grid((unsigned)ceil_div(nd, GB_M), (unsigned)ceil_div(Np, GB_N));
+  const float* Wt = a.W_packed;   // [2 d_in][d_out]
+  k_gemm2<TI, float, float><<<grid, 256, 0, s>>>(nd, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
+                                                gidx, nd, a.agg, a.ld_agg, Wt, a.d_out,
+                                                Wt + (int64_t)a.d_in * a.d_out, a.d_out, a.b, !a.last, a.out,
+                                                a.ld_out);
+  BF_LAUNCHED("k_gemm2");
+  return BUFFALO_OK;
+}
+
+buffalo_status pool_fwd_ffma(const PoolArgs& a, cudaStream_t s) {
+  return a.in_bf16 ? pool_fwd_t<__nv_bfloat16>(a, s) : pool_fwd_t<float>(a, s);
+}
+
+template <class TI>
+static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
+  const buffalo_block* blk = a.blk;
+  const int64_t n = blk->n_dst, ns = blk->n_src;
+  const int d_in = a.d_in, d_out = a.d_out, dp = (int)pitch_of(d_in);
+  const int32_t* gidx = a.layer1 ? blk->src_global : nullptr;
+  if (!a.last && n > 0) {
+    k_dz_mask<float><<<grid_for(n * d_out, 256), 256, 0, s>>>(a.dh, a.ld_dh, a.h_dst, a.ld_hdst, n, d_out);
+    BF_LAUNCHED("k_dz_mask");
+  }
+  const int S = dw_splits(n, d_out, d_in), S2 = pool_dw_splits(ns, d_in);
+  char* q = (char*)a.scratch;
+  float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * d_in * 4);
+  float* db_part = (float*)q; q += R((int64_t)S * pitch_of(d_out) * 4);
+  float* dagg = (float*)q; q += R(n * dp * 4);
+  float* dq = (float*)q; q += R(ns * dp * 4);
+  float* dwp_part = (float*)q; q += R((int64_t)S2 * d_in * d_in * 4);
+  float* dbp_part = (float*)q;
+  if (n > 0) {
+    // dW, db of the Update weight (as the mean path)
+    dim3 g((unsigned)ceil_div(2 * d_in, 64), (unsigned)ceil_div(d_out, 64), (unsigned)S);
+    k_dw_partial<TI, float><<<g, 256, 0, s>>>(n, d_out, d_in, 2 * d_in, a.dh, a.ld_dh, (const TI*)a.h_src,
+                                              a.ld_src, gidx, a.agg, a.ld_agg, ceil_div(n, S), dw_part, db_part);
+    BF_LAUNCHED("k_dw_partial");
+    k_reduce_partials<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, (int64_t)d_out * 2 * d_in, a.dW);
+    BF_LAUNCHED("k_reduce_partials");
+    k_reduce_partials<<<1, 256, 0, s>>>(db_part, S, d_out, a.db);
+    BF_LAUNCHED("k_reduce_partials");
+    // dh_agg = dZ W_neigh  (B[k][n] = W[k][d_in + n])
+    dim3 gg((unsigned)ceil_div(n, GB_M), (unsigned)ceil_div(dp, GB_N));
+    k_gemm2<float, float, float><<<gg, 256, 0, s>>>(n, d_in, dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
+                                                   a.W + d_in, 2 * d_in, nullptr, 0, nullptr, 0, dagg, dp);
+    BF_LAUNCHED("k_gemm2");
+  }
+  if (ns <= 0) return BUFFALO_OK;
+  if (n > 0) {
+    k_pool_scatterT<<<grid_for(ns * 32, 256, 16), 256, 0, s>>>(blk->t_row_ptr, blk->t_col, ns, a.arg, a.ld_pool,
+                                                               dagg, dp, a.P, a.ld_pool, d_in, dq, dp);
+    BF_LAUNCHED("k_pool_scatterT");
+  } else {
+    BF_CUDA(cudaMemsetAsync(dq, 0, sizeof(float) * ns * dp, s));
+  }
+  // dW_pool, db_pool over the src rows
+  dim3 g2((unsigned)ceil_div(d_in, 64), (unsigned)ceil_div(d_in, 64), (unsigned)S2);
+  k_dw_partial<TI, float><<<g2, 256, 0, s>>>(ns, d_in, d_in, d_in, dq, dp, (const TI*)a.h_src, a.ld_src, gidx,
+                                             nullptr, 0, ceil_div(ns, S2), dwp_part, dbp_part);
+  BF_LAUNCHED("k_dw_partial");
+  k_reduce_partials<<<grid_for((int64_t)d_in * d_in, 256), 256, 0, s>>>(dwp_part, S2, (int64_t)d_in * d_in, a.dW_pool);
+  BF_LAUNCHED("k_reduce_partials");
+  k_reduce_partials<<<1, 256, 0, s>>>(dbp_part, S2, d_in, a.db_pool);
+  BF_LAUNCHED("k_reduce_partials");
+  if (a.dh_src) {   // dH_{l-1} = pad(dZ W_self) + dQ W_pool
+    dim3 gg((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dp, GB_N));
+    k_gemm2<float, float, float><<<gg, 256, 0, s>>>(ns, d_in, dp, d_out, d_in, a.dh, a.ld_dh, nullptr, n, dq, dp,
+                                                   a.W, 2 * d_in, a.W_pool, d_in, nullptr, 0, a.dh_src,
+                                                   a.ld_dh_src);
+    BF_LAUNCHED("k_gemm2");
+  }
+  return BUFFALO_OK;
+}
+
+buffalo_status pool_bwd_ffma(const PoolArgs& a, cudaStream_t s) {
+  return a.in_bf16 ? pool_bwd_t<__nv_bfloat16>(a, s) : pool_bwd_t<float>(a, s);
 }
 
 }  // namespace buffalo

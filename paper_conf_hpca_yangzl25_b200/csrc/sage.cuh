@@ -33,6 +33,29 @@ struct BwdArgs {
   void* scratch; int64_t scratch_bytes;
 };
 
+// GraphSAGE-pool (R28): FFMA path, fp32 activations.
+struct PoolArgs {
+  const buffalo_block* blk;
+  bool layer1, in_bf16, last;
+  int d_in, d_out;
+  const void* h_src; int64_t ld_src;
+  const float* W_pool; const float* b_pool;
+  const float* W; const float* W_packed; const float* b;
+  float* out; int64_t ld_out;
+  float* agg; int64_t ld_agg;
+  float* P; int32_t* arg; int64_t ld_pool;
+  // backward
+  float* dh; int64_t ld_dh;
+  const float* h_dst; int64_t ld_hdst;
+  float* dW_pool; float* db_pool; float* dW; float* db;
+  float* dh_src; int64_t ld_dh_src;
+  void* scratch; int64_t scratch_bytes;
+};
+int pool_dw_splits(int64_t n_rows, int d);
+int64_t pool_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int d_in, int d_out);
+buffalo_status pool_fwd_ffma(const PoolArgs& a, cudaStream_t s);
+buffalo_status pool_bwd_ffma(const PoolArgs& a, cudaStream_t s);
+
 int dw_splits(int64_t n_l, int d_out, int d_in);
 int64_t bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int layer, int d_in, int d_out);
 

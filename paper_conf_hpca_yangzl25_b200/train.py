@@ -47,10 +47,11 @@ class DeviceGraph:
 class SageParams:
     """fp32 master weights/biases (Xavier init from synth), flat gradient buffer, packed copies."""
 
-    def __init__(self, model, Ws, bs, device="cuda"):
+    def __init__(self, model, Ws, bs, device="cuda", Wps=None, bps=None):
         self.model = model
         self.L = model.num_layers
-        sizes = [w.size for w in Ws] + [b.size for b in bs]
+        Wps, bps = list(Wps or []), list(bps or [])
+        sizes = [w.size for w in Ws] + [b.size for b in bs] + [w.size for w in Wps] + [b.size for b in bps]
         self.flat = torch.zeros(sum(sizes), dtype=torch.float32, device=device)
         self.grad = torch.zeros_like(self.flat)
         self.W, self.b, self.dW, self.db = [], [], [], []
@@ -65,6 +66,18 @@ class SageParams:
             self.db.append(self.grad[off:off + b.size])
             self.b[-1].copy_(torch.as_tensor(b))
             off += b.size
+        # GraphSAGE-pool weights (R28), in the same flat buffers (one allreduce, one SGD step)
+        self.Wp, self.bp, self.dWp, self.dbp = [], [], [], []
+        for w in Wps:
+            self.Wp.append(self.flat[off:off + w.size].view(w.shape))
+            self.dWp.append(self.grad[off:off + w.size].view(w.shape))
+            self.Wp[-1].copy_(torch.as_tensor(w))
+            off += w.size
+        for b in bps:
+            self.bp.append(self.flat[off:off + b.size])
+            self.dbp.append(self.grad[off:off + b.size])
+            self.bp[-1].copy_(torch.as_tensor(b))
+            off += b.size
         self.packed = [torch.empty(B.packed_weight_bytes(model, l), dtype=torch.uint8, device=device)
                        for l in range(1, self.L + 1)]
         self.repack()
@@ -77,7 +90,8 @@ class SageParams:
 class Trainer:
     def __init__(self, graph, feats, labels, seeds, dims, fanout, F, Ws, bs, feat_dtype=B.FP32,
                  gemm_mode=B.GEMM_FFMA, mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096,
-                 base_seed=3, rank=0, world=1, process_group=None, device="cuda"):
+                 base_seed=3, rank=0, world=1, process_group=None, device="cuda", aggregator=B.AGG_MEAN,
+                 Wps=None, bps=None):
         self.graph = graph if isinstance(graph, DeviceGraph) else DeviceGraph(*graph, device=device)
         self.feats = feats
         self.labels = labels
@@ -88,9 +102,12 @@ class Trainer:
         self.fanout = list(fanout)
         self.F = F
         self.base_seed = base_seed
-        self.model = B.make_model(dims, feat_dtype, gemm_mode, feats.shape[1])
+        self.pool = aggregator == B.AGG_POOL
+        if self.pool and Wps is None:
+            raise ValueError("the pool aggregator needs its weights (Wps, bps)")
+        self.model = B.make_model(dims, feat_dtype, gemm_mode, feats.shape[1], aggregator)
         self.sched = B.make_sched(mem_budget, C_ppm, k_min, k_max, world)
-        self.params = SageParams(self.model, Ws, bs, device)
+        self.params = SageParams(self.model, Ws, bs, device, Wps, bps)
         self.rank, self.world, self.pg = rank, world, process_group
         self.device = device
         # scheduler outputs
@@ -154,7 +171,12 @@ class Trainer:
         h, ld = self.feats, self.feats.shape[1]
         for l in range(1, self.L + 1):
             b = blks.layer[l - 1]
-            B.sage_fwd(b, l, m, h, ld, p.W[l - 1], p.packed[l - 1], p.b[l - 1], b.out, b.ld_out, b.agg, b.ld_agg)
+            if self.pool:
+                B.pool_fwd(b, l, m, h, ld, p.Wp[l - 1], p.bp[l - 1], p.W[l - 1], p.packed[l - 1], p.b[l - 1],
+                           b.out, b.ld_out, b.agg, b.ld_agg, b.pool_P, b.pool_arg, b.ld_pool)
+            else:
+                B.sage_fwd(b, l, m, h, ld, p.W[l - 1], p.packed[l - 1], p.b[l - 1], b.out, b.ld_out, b.agg,
+                           b.ld_agg)
             h, ld = b.out, b.ld_out
 
     def backward(self):
@@ -168,6 +190,11 @@ class Trainer:
             else:
                 h_src, ld_src, dh_src, ld_dh_src, prev_rp = self.feats, self.feats.shape[1], None, 0, None
             h_dst = b.out if l < self.L else None
+            if self.pool:
+                B.pool_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out, b.pool_P,
+                           b.pool_arg, b.ld_pool, p.Wp[l - 1], p.W[l - 1], p.dWp[l - 1], p.dbp[l - 1],
+                           p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src, b.bwd_scratch, b.bwd_scratch_bytes)
+                continue
             B.sage_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out,
                        p.W[l - 1], p.packed[l - 1], p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src, prev_rp,
                        b.bwd_scratch, b.bwd_scratch_bytes)
