@@ -30,6 +30,11 @@ Functions and the passages they follow:
                        aggregators", :386; pool as defined by GraphSAGE [16]): P = ReLU(H W_pool^T
                        + b_pool), h_agg = element-wise max over the sampled neighbours, then the
                        same Update as mean (R28)
+  lstm_forward, lstm_backward
+                       GraphSAGE-LSTM (the paper's memory-intensive
+                       aggregator, Table III :479-497): an LSTM with
+                       hidden size d_{l-1} run over each destination's sampled neighbours in CSR
+                       order, h_agg = its last hidden state (R29)
   triangles, avg_clustering
                        C of Eq. 1 (Newman's local clustering
                        coefficient, "page 142 of reference [27]"): T_v by definition (C),
@@ -230,6 +235,12 @@ def pool_dw_splits(n_rows, d):
     return max(1, min(_ceil(296, tiles), _ceil(n_rows, 512)))
 
 
+def lstm_dw_splits(n_rows, d):
+    """Split count of the LSTM weights' dW reduction (4d rows, K = d columns)."""
+    tiles = _ceil(4 * d, 64) * _ceil(d, 64)
+    return max(1, min(_ceil(296, tiles), _ceil(max(int(n_rows), 1), 512)))
+
+
 def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
     """BucketMemEstimator reading R15: the exact arena bytes of one
     micro-batch with layer sizes n[0..L], e[1..L] (e indexed l-1) and widths dims[0..L].
@@ -239,6 +250,7 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
     L = len(e)
     s = 4 if act_dtype == FP32 else 2
     pool = aggregator == "pool"                  # R28: fp32 only; block 1 keeps a transpose too
+    lstm = aggregator == "lstm"                  # R29: fp32 only
     blocks = 0
     build = 0
     for l in range(1, L + 1):
@@ -264,6 +276,14 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
         if l < L:
             acts += _R(n[l] * pitch(dims[l]) * s)               # H_l
     acts += _R(n[L] * pitch(dims[L]) * 4)                       # logits
+    if lstm:
+        for l in range(1, L + 1):
+            d, el, nl = dims[l - 1], e[l - 1], n[l]
+            acts += _R(el * pitch(4 * d) * 4)                   # gates (i, f, u, o), later their gradients
+            acts += _R(el * pitch(d) * 4)                       # cell state c_t per (dst, step)
+            acts += 2 * _R(el * 4)                              # source row and packed position per edge
+            acts += 2 * _R(nl * pitch(d) * 4)                   # running h, c (backward: dh, dc)
+            acts += _R(4 * 256)                                 # degree-class counts, max degree
     if pool:
         for l in range(1, L + 1):
             acts += _R(n[l - 1] * pitch(dims[l - 1]) * 4)       # P = ReLU(H W_pool^T + b_pool)
@@ -285,8 +305,16 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
             frame += _R(n[l] * pitch(d) * 4) + _R(n[l - 1] * pitch(d) * 4)     # dh_agg, dQ
             S2 = pool_dw_splits(n[l - 1], d)
             frame += _R(S2 * d * d * 4) + _R(S2 * pitch(d) * 4)               # dW_pool, db_pool partials
+        if lstm:
+            d, el = dims[l - 1], e[l - 1]
+            frame += 2 * _R(n[l] * pitch(d) * 4)                 # dh_agg, dh_prev staging
+            frame += _R(el * pitch(d) * 4)                       # h_{t-1} per (dst, step)
+            if l >= 2:
+                frame += _R(el * pitch(d) * 4)                   # dx per (dst, step)
+            S3 = lstm_dw_splits(el, d)
+            frame += _R(S3 * 4 * d * d * 4) + _R(S3 * pitch(4 * d) * 4)   # dW_ih / dW_hh partials
         if act_dtype == FP32:
-            if l >= 2 and not pool:
+            if l >= 2 and not (pool or lstm):
                 frame += _R(n[l - 1] * pitch(dims[l]) * 4)      # transposed aggregate of dZ/D
             S = dw_splits(n[l], dims[l], dims[l - 1])
             frame += _R(S * dims[l] * 2 * dims[l - 1] * 4) + _R(S * pitch(dims[l]) * 4)  # dW, db partials
@@ -559,6 +587,102 @@ def pool_backward(blocks, cache, Ws, Wps, dlogits):
         if l > 1:
             dHin = dQ @ Wp
             dHin[:n] += dZ @ W[:, :d_in]
+            dH = dHin
+    return grads
+
+
+def _sigmoid(x):
+    return 1.0 / (1.0 + np.exp(-x))
+
+
+def lstm_forward(blocks, X, Ws, bs, Wihs, Whhs, bls):
+    """GraphSAGE-LSTM forward in float64 (R29; GraphSAGE [16] LSTM aggregator as DGL's SAGEConv
+    'lstm' computes it, PyTorch gate order i, f, g, o).  For block l with input rows H and dst i
+    with sampled neighbours j_1..j_D in CSR order: h_0 = c_0 = 0;
+    for t = 1..D:  g = W_ih H[j_t] + W_hh h_{t-1} + b;  i = s(g_i), f = s(g_f), u = tanh(g_g),
+    o = s(g_o);  c_t = f c_{t-1} + i u;  h_t = o tanh(c_t);   h_agg[i] = h_D (0 if D = 0);
+    Z = [H[:n_dst] || h_agg] W_l^T + b_l;  H_l = ReLU(Z) for l < L.
+    W_ih, W_hh: [4 d_{l-1}, d_{l-1}], b: [4 d_{l-1}] (= b_ih + b_hh of nn.LSTM)."""
+    L = len(blocks)
+    H = np.asarray(X, dtype=np.float64)[blocks[0]["src_global"]]
+    cache = []
+    for l in range(1, L + 1):
+        b = blocks[l - 1]
+        W = np.asarray(Ws[l - 1], dtype=np.float64)
+        Wih = np.asarray(Wihs[l - 1], dtype=np.float64)
+        Whh = np.asarray(Whhs[l - 1], dtype=np.float64)
+        bl = np.asarray(bls[l - 1], dtype=np.float64)
+        d = H.shape[1]
+        n = b["n_dst"]
+        agg = np.zeros((n, d))
+        steps = []                                   # per dst: list of (i, f, u, o, c_prev, c, h_prev)
+        rp, col = b["row_ptr"], b["col_local"]
+        for r in range(n):
+            h = np.zeros(d)
+            c = np.zeros(d)
+            st = []
+            for e in range(rp[r], rp[r + 1]):
+                g = Wih @ H[col[e]] + Whh @ h + bl
+                gi, gf, gu, go = _sigmoid(g[:d]), _sigmoid(g[d:2 * d]), np.tanh(g[2 * d:3 * d]), _sigmoid(g[3 * d:])
+                c_new = gf * c + gi * gu
+                h_new = go * np.tanh(c_new)
+                st.append((gi, gf, gu, go, c, c_new, h))
+                h, c = h_new, c_new
+            agg[r] = h
+            steps.append(st)
+        Z = H[:n] @ W[:, :d].T + agg @ W[:, d:].T + np.asarray(bs[l - 1], dtype=np.float64)
+        cache.append(dict(H_in=H, agg=agg, steps=steps, Z=Z))
+        H = np.maximum(Z, 0.0) if l < L else Z
+    return H, cache
+
+
+def lstm_backward(blocks, cache, Ws, Wihs, Whhs, dlogits):
+    """Backward of lstm_forward (back-propagation through the neighbour sequence): per layer
+    (dW_l, db_l, dW_ih_l, dW_hh_l, db_lstm_l).  dZ as for mean; dh_agg = dZ W_neigh; per dst,
+    for t = D..1: dc += dh o (1 - tanh^2 c_t); gate pre-activation gradients
+    di = dc u i(1-i), df = dc c_{t-1} f(1-f), du = dc i (1-u^2), do = dh tanh(c_t) o(1-o);
+    dW_ih += dg x_t^T, dW_hh += dg h_{t-1}^T, db += dg;  dx_t = W_ih^T dg (into dH_{l-1}[j_t]);
+    dh <- W_hh^T dg, dc <- dc f.   dH_{l-1} = (sum of dx over edges) + pad(dZ W_self)."""
+    L = len(blocks)
+    grads = [None] * L
+    dH = np.asarray(dlogits, dtype=np.float64)
+    for l in range(L, 0, -1):
+        c_ = cache[l - 1]
+        b = blocks[l - 1]
+        W = np.asarray(Ws[l - 1], dtype=np.float64)
+        Wih = np.asarray(Wihs[l - 1], dtype=np.float64)
+        Whh = np.asarray(Whhs[l - 1], dtype=np.float64)
+        H = c_["H_in"]
+        d = H.shape[1]
+        dZ = dH if l == L else dH * (c_["Z"] > 0)
+        n = dZ.shape[0]
+        dW = dZ.T @ np.concatenate([H[:n], c_["agg"]], axis=1)
+        dagg = dZ @ W[:, d:]
+        dWih = np.zeros_like(Wih)
+        dWhh = np.zeros_like(Whh)
+        dbl = np.zeros(4 * d)
+        dHin = np.zeros_like(H)
+        rp, col = b["row_ptr"], b["col_local"]
+        for r in range(n):
+            dh = dagg[r].copy()
+            dc = np.zeros(d)
+            st = c_["steps"][r]
+            for t in range(len(st) - 1, -1, -1):
+                gi, gf, gu, go, c_prev, c_t, h_prev = st[t]
+                tc = np.tanh(c_t)
+                dc = dc + dh * go * (1.0 - tc * tc)
+                dg = np.concatenate([dc * gu * gi * (1.0 - gi), dc * c_prev * gf * (1.0 - gf),
+                                     dc * gi * (1.0 - gu * gu), dh * tc * go * (1.0 - go)])
+                x = H[col[rp[r] + t]]
+                dWih += np.outer(dg, x)
+                dWhh += np.outer(dg, h_prev)
+                dbl += dg
+                dHin[col[rp[r] + t]] += Wih.T @ dg
+                dh = Whh.T @ dg
+                dc = dc * gf
+        grads[l - 1] = (dW, dZ.sum(axis=0), dWih, dWhh, dbl)
+        if l > 1:
+            dHin[:n] += dZ @ W[:, :d]
             dH = dHin
     return grads
 

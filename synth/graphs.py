@@ -226,6 +226,30 @@ def pool_weights(dims, seed=WEIGHT_SEED, bias_scale=0.0, dyadic=False):
     return Wps, bps
 
 
+def lstm_weights(dims, seed=WEIGHT_SEED):
+    """GraphSAGE-LSTM weights per layer l = 1..L (hidden size d = d_{l-1}): W_ih, W_hh float32
+    [4d, d] and b [4d] (b_ih + b_hh of nn.LSTM), uniform on +-1/sqrt(d) as nn.LSTM initialises
+    them; Philox counters c0 = 128 + l (W_ih), 160 + l (W_hh), 192 + l (b)."""
+    Wih, Whh, bl = [], [], []
+    for l in range(1, len(dims)):
+        d = dims[l - 1]
+        a = 1.0 / math.sqrt(d)
+        r = np.arange(4 * d, dtype=np.uint64)[:, None]
+        c = np.arange(d, dtype=np.uint64)[None, :]
+        out = []
+        for c0 in (128 + l, 160 + l):
+            w = words(seed, c0, r, c >> np.uint64(2), TAG_WEIGHT)
+            sel = np.choose((c & np.uint64(3)).astype(np.int64), w)
+            u = (sel.astype(np.float64) + 0.5) / 4294967296.0
+            out.append(((2.0 * u - 1.0) * a).astype(np.float32))
+        wb = words(seed, 192 + l, 0, np.arange(4 * d, dtype=np.uint64), TAG_WEIGHT)[0]
+        ub = (wb.astype(np.float64) + 0.5) / 4294967296.0
+        Wih.append(out[0])
+        Whh.append(out[1])
+        bl.append(((2.0 * ub - 1.0) * a).astype(np.float32))
+    return Wih, Whh, bl
+
+
 # ----------------------------------------------------------------------------- configs
 @dataclass
 class Config:
