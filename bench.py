@@ -35,6 +35,9 @@ WORKLOADS = {
               "3-layer SAGE-mean 128-256-256-40, full-neighbour blocks, F=10, 90,941 seeds, K=4 bucket groups"),
     "cora": ("Cora-sized synthetic graph (2,708 nodes, 5,278 edges, 1,433-d), 2-layer SAGE-mean "
              "1433-256-7, fanout (10,25), 4 partitions"),
+    "arxiv_lstm": ("ogbn-arxiv-shaped power-law graph (169,343 nodes, 1,166,243 undirected edges, 128-d), "
+                   "2-layer SAGE-LSTM 128-128-40 (LSTM hidden 128, PAPER.md:351), fanout (10,25), F=25, "
+                   "90,941 seeds, budget forcing >= 2 bucket groups"),
     "products": ("ogbn-products-shaped power-law graph (2,449,029 nodes, 61,859,140 edges, 100-d), 3-layer "
                  "SAGE-mean 100-256-256-47, fanout (10,25,30), budget forcing >= 8 bucket groups"),
 }
@@ -42,7 +45,8 @@ WORKLOADS = {
 
 # Table II's average clustering coefficients, logged beside the C measured
 # on the synthetic graph (reading R27; the Chung-Lu graphs have far fewer triangles)
-C_TABLE2 = {"cora": 0.24, "arxiv": 0.226, "products": 0.411, "papers": 0.085}
+FP32_PEAK_TFLOPS = 148 * 128 * 2 * 1.965e9 / 1e12     # FP32 FMA pipes at the max SM clock
+C_TABLE2 = {"cora": 0.24, "arxiv": 0.226, "arxiv_lstm": 0.226, "products": 0.411, "papers": 0.085}
 
 
 def parse():
@@ -52,8 +56,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="products", choices=list(WORKLOADS))
     ap.add_argument("--gemm", default="bf16", choices=["bf16", "ffma"])
-    ap.add_argument("--aggregator", default="mean", choices=["mean", "pool"],
-                    help="pool: GraphSAGE-pool (SURVEY §8(f) NEXT 2), fp32 FFMA path only")
+    ap.add_argument("--aggregator", default="mean", choices=["mean", "pool", "lstm"],
+                    help="pool / lstm: GraphSAGE-pool / -LSTM (SURVEY §8(f) NEXT 2 / 1), fp32 FFMA path only")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-baseline-seconds", type=float, default=20.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -242,14 +246,18 @@ def run_ours(args, cfg):
     rp, col, X, y, seeds, Ws, bs = make_inputs_device(cfg)
     t_gen = time.perf_counter() - t_gen
     pool = args.aggregator == "pool"
-    if pool:
-        args.gemm = "ffma"                             # the pool aggregator is built for fp32 only
+    lstm = args.aggregator == "lstm"
+    if pool or lstm:
+        args.gemm = "ffma"                             # the pool / LSTM aggregators are built for fp32 only
     gemm = B.GEMM_BF16 if args.gemm == "bf16" else B.GEMM_FFMA
     agg_kw = {}
     if pool:
         from synth.graphs import pool_weights
         Wps, bps = pool_weights(cfg.dims)
         agg_kw = dict(aggregator=B.AGG_POOL, Wps=Wps, bps=bps)
+    if lstm:
+        from synth.graphs import lstm_weights
+        agg_kw = dict(aggregator=B.AGG_LSTM, lstm=lstm_weights(cfg.dims))
     feat_dtype = B.BF16 if args.gemm == "bf16" else B.FP32
     feats = X
     if feat_dtype == B.BF16:
@@ -266,14 +274,15 @@ def run_ours(args, cfg):
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, mem_budget=budget,
                  C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg,
                  **agg_kw)
-    if args.config == "products":
-        # calibrate M_ctr once so that one GPU needs >= 8 groups, then freeze it for every N
+    if args.config in ("products", "arxiv_lstm"):
+        # calibrate M_ctr once so that one GPU needs >= 8 groups (products; 2 for the LSTM
+        # workload), then freeze it for every N
         B_full = Trainer(graph, feats, y, seeds, cfg.dims,
                          cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, C_ppm=C_ppm,
                          k_min=1, k_max=1, **agg_kw)
         _, _, est1, _ = B_full.schedule(0)
         del B_full
-        tr.sched.mem_budget = int(est1[0]) // 8
+        tr.sched.mem_budget = int(est1[0]) // (8 if args.config == "products" else 2)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
 
@@ -288,7 +297,7 @@ def run_ours(args, cfg):
     clocks.start()
     # live roofline of the dominant kernel (k_gather_rows, the Aggregate): CUDA events around
     # each of its launches on its stream, algorithmic bytes from the edges it aggregated
-    B.profile_begin("pool_max" if pool else "gather", prof_counters)
+    B.profile_begin("lstm_gates" if lstm else "pool_max" if pool else "gather", prof_counters)
     l0 = B.launch_count()
     step_ms, edges, sizes, ks = [], 0, [], []
     torch.cuda.synchronize()
@@ -358,9 +367,27 @@ def run_ours(args, cfg):
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
         traffic = json.load(open(tpath)).get(f"{args.config}/{args.gemm}" + ("/pool" if pool else ""))
+    if lstm:   # the LSTM path is bound by its fp32 SIMT gate GEMMs: FLOP roofline ("alu")
+        tf = g_bytes / (g_ms / 1e3) / 1e12 if g_ms > 0 else 0.0
+        roof = {"bound": "alu", "kernel": "k_gemm2 (LSTM gate GEMM of every step, fp32 SIMT)",
+                "achieved": tf, "peak": FP32_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": tf / FP32_PEAK_TFLOPS,
+                "traffic": None,
+                "peak_source": "derived: 148 SMs x 128 FP32 FMA/clk x 2 flop x 1.965 GHz (no FP32 figure in "
+                               "B200_PROFILING.md)",
+                "flops_per_launch": g_bytes / max(1, g_launches), "launch_ms": g_ms / max(1, g_launches),
+                "launches": g_launches, "share_of_step": g_ms / total_ms}
+    else:
+        roof = {"bound": "hbm",
+                "kernel": ("k_pool_max (GraphSAGE-pool neighbour max + argmax)" if pool else
+                           "k_gather_v2 (Aggregate: fwd neighbour mean, bwd transposed sum)"),
+                "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": traffic, "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": g_bytes / max(1, g_launches),
+                "launch_ms": g_ms / max(1, g_launches), "launches": g_launches,
+                "share_of_step": g_ms / total_ms}
     if rank == 0:
         cpu = None
-        if world == 1 and not args.no_cpu_baseline and not pool:   # (the pool oracle is loop-plain: tests only)
+        if world == 1 and not args.no_cpu_baseline and not (pool or lstm):   # (the pool oracle is loop-plain: tests only)
             rp_h, col_h, X_h, y_h, seeds_h = host_copies(rp, col, X, y, tr.seeds)
             cpu = oracle_sample(cfg, rp_h, col_h, X_h, y_h, seeds_h, Ws, bs, args.cpu_baseline_seconds)
         line = dict(
@@ -375,14 +402,7 @@ def run_ours(args, cfg):
                     "parallelism": f"dp{world} over bucket groups",
                     "C_eq1": C_eq1, "C_ppm": C_ppm, "C_table2": C_TABLE2.get(args.config),
                     "C_seconds": t_c},
-            roofline={"bound": "hbm",
-                      "kernel": ("k_pool_max (GraphSAGE-pool neighbour max + argmax)" if pool else
-                                 "k_gather_v2 (Aggregate: fwd neighbour mean, bwd transposed sum)"),
-                      "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                      "traffic": traffic, "peak_source": peak_src,
-                      "algorithmic_bytes_per_launch": g_bytes / max(1, g_launches),
-                      "launch_ms": g_ms / max(1, g_launches), "launches": g_launches,
-                      "share_of_step": g_ms / total_ms},
+            roofline=roof,
             cpu_baseline=cpu,
             e2e={"value": e2e_val, "unit": "edges/s", "h2d_bytes_per_step": 4 * len(seeds),
                  "d2h_bytes_per_step": 4},

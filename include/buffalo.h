@@ -42,7 +42,7 @@ typedef enum {
 
 enum { BUFFALO_FP32 = 0, BUFFALO_BF16 = 1 };            /* storage dtypes                  */
 enum { BUFFALO_GEMM_FFMA = 0, BUFFALO_GEMM_BF16 = 1 };  /* Update GEMM: fp32 SIMT | tcgen05 */
-enum { BUFFALO_AGG_MEAN = 0, BUFFALO_AGG_POOL = 1 };    /* GraphSAGE aggregator (R20, R28)  */
+enum { BUFFALO_AGG_MEAN = 0, BUFFALO_AGG_POOL = 1, BUFFALO_AGG_LSTM = 2 }; /* aggregator (R20, R28, R29) */
 enum { BUFFALO_MAX_LAYERS = 8, BUFFALO_MAX_FANOUT = 32, BUFFALO_MAX_DIM = 4096 };
 
 /* Input graph (the batch's host graph): CSR, rows sorted ascending, symmetric,
@@ -77,7 +77,7 @@ typedef struct {
   int32_t feat_dtype;
   int32_t gemm_mode;
   int64_t feat_pitch;
-  int32_t aggregator;       /* BUFFALO_AGG_MEAN (default) | BUFFALO_AGG_POOL (gemm_mode FFMA only) */
+  int32_t aggregator;       /* BUFFALO_AGG_MEAN (default) | _POOL | _LSTM (the last two: gemm_mode FFMA) */
 } buffalo_model;
 
 /* Scheduler parameters (Alg. 3): mem_budget = M_ctr in bytes (arena bytes
@@ -135,6 +135,10 @@ typedef struct {
   float* pool_P;
   int32_t* pool_arg;
   int64_t ld_pool;
+  /* aggregator LSTM only (else NULL / 0): the layer's saved sequence state (gates, cell states,
+   * per-edge source rows and packed positions, running h/c, degree-class counts), R29. */
+  void* lstm_saved;
+  int64_t lstm_saved_bytes;
 } buffalo_block;
 
 typedef struct {
@@ -272,6 +276,38 @@ BUFFALO_API buffalo_status buffalo_pool_bwd(const buffalo_block* blk, int32_t la
                                 float* dh_src, int64_t ld_dh_src, void* scratch,
                                 size_t scratch_bytes, void* stream);
 
+/* ------------------------------------------------------------------ GraphSAGE-LSTM */
+/* the LSTM aggregator, the paper's memory-intensive case (PAPER.md:56,
+ * :63, :125 "degree bucketing ... is crucial for memory-intensive aggregators (e.g., LSTM)",
+ * :351, Table III :479-497), reading R29.  For block `layer` (model.aggregator = LSTM, gemm_mode
+ * FFMA, fp32): an LSTM of hidden size d = d_{l-1} (gates i, f, g, o; W_ih, W_hh fp32 [4d][d]
+ * row-major, b_lstm fp32 [4d] = b_ih + b_hh) runs over each dst row's sampled neighbours in CSR
+ * order from zero state; h_agg = its last hidden state (0 for D = 0); then the Update of
+ * buffalo_sage_fwd.  The dst rows are processed in degree-class order (the block's cls_perm:
+ * the degree buckets of Alg. 2 l.6), so step t is one batched gate GEMM over the rows with
+ * D > t.  saved = the block's lstm_saved (kept for the backward).  Synchronises the stream once
+ * (an 520-byte read of the degree-class counts sizes the per-step launches).  Errors:
+ * UNSUPPORTED (a row with more than 128 neighbours; aggregator/gemm_mode), INVALID_ARG. */
+BUFFALO_API buffalo_status buffalo_lstm_fwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                const void* h_src, int64_t ld_src, const float* W_ih,
+                                const float* W_hh, const float* b_lstm, const float* W,
+                                const void* W_packed, const float* b, void* out, int64_t ld_out,
+                                void* saved_agg, int64_t ld_agg, void* lstm_saved,
+                                size_t lstm_saved_bytes, void* stream);
+/* Backward (back-propagation through the neighbour sequences; gradients accumulated, +=):
+ * dZ, dW, db as buffalo_sage_bwd; dh_agg = dZ W_neigh; per step t = T-1..0 the gate gradients,
+ * dW_ih += sum dG x^T, dW_hh += sum dG h_{t-1}^T, db_lstm += sum dG (deterministic split
+ * reductions); dh_src (l >= 2) = pad(dZ W_self) + sum over each src's edges (ascending dst) of
+ * W_ih^T dG.  Synchronises once (the step table).  scratch: the block's bwd_scratch. */
+BUFFALO_API buffalo_status buffalo_lstm_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
+                                const void* saved_agg, int64_t ld_agg, const void* h_dst,
+                                int64_t ld_hdst, void* lstm_saved, size_t lstm_saved_bytes,
+                                const float* W_ih, const float* W_hh, const float* W,
+                                float* dW_ih_accum, float* dW_hh_accum, float* db_lstm_accum,
+                                float* dW_accum, float* db_accum, float* dh_src, int64_t ld_dh_src,
+                                void* scratch, size_t scratch_bytes, void* stream);
+
 /* ------------------------------------------------------------------ a10: optimizer */
 /* SGD (Alg. 2 l.13, R18): param -= lr * grad; grad = 0 (ready for the next epoch). */
 BUFFALO_API buffalo_status buffalo_sgd_step(float* param, float* grad, int64_t n, float lr, void* stream);
@@ -310,7 +346,8 @@ BUFFALO_API buffalo_status buffalo_avg_clustering(const buffalo_graph* g, const 
 BUFFALO_API int64_t buffalo_launch_count(void);
 
 /* Diagnostics (bench roofline): time every launch of one kernel family with CUDA events on the
- * stream it is launched on.  family "pool_max": k_pool_max, the GraphSAGE-pool neighbour max
+ * stream it is launched on.  family "lstm_gates": the LSTM gate GEMM of every step; its
+ * "algorithmic bytes" are FLOPs (2 x rows x 4d x (d + d)).  family "pool_max": k_pool_max, the GraphSAGE-pool neighbour max
  * (per row 12 B + the max and argmax rows, per edge the index and the pooled fp32 row).
  * family "gather": k_gather_rows, the Aggregate of the forward (mean
  * of neighbour rows) and of the backward (sum of dZ/D rows over the transposed block).

@@ -307,7 +307,7 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
             frame += _R(S2 * d * d * 4) + _R(S2 * pitch(d) * 4)               # dW_pool, db_pool partials
         if lstm:
             d, el = dims[l - 1], e[l - 1]
-            frame += 2 * _R(n[l] * pitch(d) * 4)                 # dh_agg, dh_prev staging
+            frame += _R(n[l] * pitch(d) * 4)                     # dh_agg
             frame += _R(el * pitch(d) * 4)                       # h_{t-1} per (dst, step)
             if l >= 2:
                 frame += _R(el * pitch(d) * 4)                   # dx per (dst, step)

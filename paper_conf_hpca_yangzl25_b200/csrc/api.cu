@@ -91,6 +91,7 @@ __global__ void k_fill_i32(int32_t* a, int64_t n, int32_t v) {
 // Restated from DESIGN.md §5; must agree with the arena that buffalo_build_blocks lays out.
 static int64_t bwd_scratch_for(const buffalo_model* m, int64_t n_dst, int64_t n_src, int64_t e, int l) {
   if (m->aggregator == BUFFALO_AGG_POOL) return pool_bwd_scratch_bytes(n_dst, n_src, m->dim[l - 1], m->dim[l]);
+  if (m->aggregator == BUFFALO_AGG_LSTM) return lstm_bwd_scratch_bytes(n_dst, e, l, m->dim[l - 1], m->dim[l]);
   if (m->gemm_mode == BUFFALO_GEMM_BF16)
     return tc_bwd_scratch_bytes(n_dst, n_src, e, l, m->dim[l - 1], m->dim[l], l == m->num_layers);
   return bwd_scratch_bytes(n_dst, n_src, l, m->dim[l - 1], m->dim[l]);
@@ -121,6 +122,8 @@ static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_m
     if (l < L) acts += R(n[l] * pitch_of(m->dim[l]) * s);
   }
   acts += R(n[L] * pitch_of(m->dim[L]) * 4);
+  if (m->aggregator == BUFFALO_AGG_LSTM)
+    for (int l = 1; l <= L; ++l) acts += R(lstm_saved_bytes(n[l], e[l - 1], m->dim[l - 1]));
   if (pool)
     for (int l = 1; l <= L; ++l)   // P [n_{l-1}] and argmax [n_l] rows of width pitch(d_{l-1})
       acts += R(n[l - 1] * pitch_of(m->dim[l - 1]) * 4) + R(n[l] * pitch_of(m->dim[l - 1]) * 4);
@@ -152,12 +155,12 @@ static buffalo_status validate_model(const buffalo_model* m) {
         set_error("model: the bf16 tensor-core path supports dim[l] <= 256 for l >= 1");
         return BUFFALO_ERR_UNSUPPORTED;
       }
-  if (m->aggregator != BUFFALO_AGG_MEAN && m->aggregator != BUFFALO_AGG_POOL) {
+  if (m->aggregator != BUFFALO_AGG_MEAN && m->aggregator != BUFFALO_AGG_POOL && m->aggregator != BUFFALO_AGG_LSTM) {
     set_error("model: unknown aggregator %d", m->aggregator);
     return BUFFALO_ERR_INVALID_ARG;
   }
-  if (m->aggregator == BUFFALO_AGG_POOL && m->gemm_mode != BUFFALO_GEMM_FFMA) {
-    set_error("model: the pool aggregator is built for gemm_mode FFMA (fp32) only");
+  if (m->aggregator != BUFFALO_AGG_MEAN && m->gemm_mode != BUFFALO_GEMM_FFMA) {
+    set_error("model: the pool and LSTM aggregators are built for gemm_mode FFMA (fp32) only");
     return BUFFALO_ERR_UNSUPPORTED;
   }
   if (m->feat_pitch < round_up(m->dim[0], 8) || m->feat_pitch % 8) {
@@ -285,7 +288,8 @@ const char* buffalo_last_error(void) { return g_err.c_str(); }
 int64_t buffalo_launch_count(void) { return g_launches.load(); }
 
 buffalo_status buffalo_profile_begin(const char* family, void* counters, int64_t max_launches, void* stream) {
-  if (!family || (std::string(family) != "gather" && std::string(family) != "pool_max") || !counters ||
+  const std::string fam = family ? family : "";
+  if (!family || (fam != "gather" && fam != "pool_max" && fam != "lstm_gates") || !counters ||
       max_launches <= 0) {
     set_error("profile_begin: unknown kernel family or no counter buffer");
     return BUFFALO_ERR_INVALID_ARG;
@@ -650,6 +654,12 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
       b->pool_P = (float*)A.take(b->n_src * b->ld_pool * 4);
       b->pool_arg = (int32_t*)A.take(b->n_dst * b->ld_pool * 4);
     }
+  if (m->aggregator == BUFFALO_AGG_LSTM)
+    for (int l = 1; l <= L; ++l) {
+      buffalo_block* b = &out->layer[l - 1];
+      b->lstm_saved_bytes = R(lstm_saved_bytes(b->n_dst, b->n_edges, m->dim[l - 1]));
+      b->lstm_saved = A.take(b->lstm_saved_bytes);
+    }
   // backward region: ping-pong dH buffers at the two ends, scratch in between
   int64_t B = 0;
   std::vector<int64_t> ah(L + 1, 0), tmp(L + 1, 0);
@@ -915,6 +925,111 @@ buffalo_status buffalo_pool_bwd(const buffalo_block* blk, int32_t layer, const b
   a.scratch = scratch;
   a.scratch_bytes = (int64_t)scratch_bytes;
   return pool_bwd_ffma(a, (cudaStream_t)stream);
+}
+
+static buffalo_status lstm_args(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                                 const void* h_src, int64_t ld_src, void* saved, size_t saved_bytes, LstmArgs& a,
+                                 const char* who) {
+  BF_CHECK(require_sm100());
+  BF_CHECK(validate_model(m));
+  if (m->aggregator != BUFFALO_AGG_LSTM) {
+    set_error("%s: model.aggregator is not BUFFALO_AGG_LSTM", who);
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
+  if (!blk || layer < 1 || layer > m->num_layers || !h_src || !saved || !blk->cls_perm) {
+    set_error("%s: null argument or bad layer", who);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if ((int64_t)saved_bytes < lstm_saved_bytes(blk->n_dst, blk->n_edges, m->dim[layer - 1])) {
+    set_error("%s: lstm_saved too small", who);
+    return BUFFALO_ERR_CAPACITY;
+  }
+  a = LstmArgs{};
+  a.blk = blk;
+  a.layer1 = layer == 1;
+  a.in_bf16 = a.layer1 && m->feat_dtype == BUFFALO_BF16;
+  a.last = layer == m->num_layers;
+  a.d_in = m->dim[layer - 1];
+  a.d_out = m->dim[layer];
+  a.h_src = h_src;
+  a.ld_src = a.layer1 ? m->feat_pitch : ld_src;
+  a.saved = saved;
+  if (a.ld_src < pitch_of(a.d_in) || a.ld_src % 8) {
+    set_error("%s: ld_src must be a multiple of 8 and >= pitch(d_in)", who);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (a.layer1 && !blk->col_global) return BUFFALO_ERR_INVALID_ARG;
+  return BUFFALO_OK;
+}
+
+buffalo_status buffalo_lstm_fwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m, const void* h_src,
+                                int64_t ld_src, const float* W_ih, const float* W_hh, const float* b_lstm,
+                                const float* W, const void* W_packed, const float* b, void* out, int64_t ld_out,
+                                void* saved_agg, int64_t ld_agg, void* lstm_saved, size_t lstm_saved_bytes,
+                                void* stream) {
+  LstmArgs a;
+  BF_CHECK(lstm_args(blk, layer, m, h_src, ld_src, lstm_saved, lstm_saved_bytes, a, "lstm_fwd"));
+  if (!W_ih || !W_hh || !b_lstm || !W || !W_packed || !b || !out || !saved_agg) {
+    set_error("lstm_fwd: null argument");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (ld_out < pitch_of(a.d_out) || ld_agg < pitch_of(a.d_in) || ld_out % 8 || ld_agg % 8) {
+    set_error("lstm_fwd: leading dimensions must be multiples of 8 and >= the padded widths");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  a.W_ih = W_ih;
+  a.W_hh = W_hh;
+  a.b_lstm = b_lstm;
+  a.W = W;
+  a.W_packed = (const float*)W_packed;
+  a.b = b;
+  a.out = (float*)out;
+  a.ld_out = ld_out;
+  a.agg = (float*)saved_agg;
+  a.ld_agg = ld_agg;
+  return lstm_fwd_ffma(a, (cudaStream_t)stream);
+}
+
+buffalo_status buffalo_lstm_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m, float* dh_dst,
+                                int64_t ld_dh, const void* h_src, int64_t ld_src, const void* saved_agg,
+                                int64_t ld_agg, const void* h_dst, int64_t ld_hdst, void* lstm_saved,
+                                size_t lstm_saved_bytes, const float* W_ih, const float* W_hh, const float* W,
+                                float* dW_ih_accum, float* dW_hh_accum, float* db_lstm_accum, float* dW_accum,
+                                float* db_accum, float* dh_src, int64_t ld_dh_src, void* scratch,
+                                size_t scratch_bytes, void* stream) {
+  LstmArgs a;
+  BF_CHECK(lstm_args(blk, layer, m, h_src, ld_src, lstm_saved, lstm_saved_bytes, a, "lstm_bwd"));
+  if (!dh_dst || !saved_agg || !W_ih || !W_hh || !W || !dW_ih_accum || !dW_hh_accum || !db_lstm_accum ||
+      !dW_accum || !db_accum || !scratch || (!a.last && !h_dst)) {
+    set_error("lstm_bwd: null argument");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (dh_src && (layer == 1 || !blk->t_row_ptr)) {
+    set_error("lstm_bwd: dh_src needs a transposed block (layer >= 2)");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if ((int64_t)scratch_bytes < lstm_bwd_scratch_bytes(blk->n_dst, blk->n_edges, layer, a.d_in, a.d_out)) {
+    set_error("lstm_bwd: scratch too small");
+    return BUFFALO_ERR_CAPACITY;
+  }
+  a.dh = dh_dst;
+  a.ld_dh = ld_dh;
+  a.agg = (float*)saved_agg;
+  a.ld_agg = ld_agg;
+  a.h_dst = (const float*)h_dst;
+  a.ld_hdst = ld_hdst;
+  a.W_ih = W_ih;
+  a.W_hh = W_hh;
+  a.W = W;
+  a.dW_ih = dW_ih_accum;
+  a.dW_hh = dW_hh_accum;
+  a.db_lstm = db_lstm_accum;
+  a.dW = dW_accum;
+  a.db = db_accum;
+  a.dh_src = dh_src;
+  a.ld_dh_src = ld_dh_src;
+  a.scratch = scratch;
+  return lstm_bwd_ffma(a, (cudaStream_t)stream);
 }
 
 buffalo_status buffalo_softmax_ce(const float* logits, int64_t ld, int64_t n, int32_t classes,

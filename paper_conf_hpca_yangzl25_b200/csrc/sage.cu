@@ -9,6 +9,8 @@
 #include "common.cuh"
 #include <type_traits>
 
+#include <vector>
+
 #include "sage.cuh"
 
 namespace buffalo {
@@ -214,7 +216,7 @@ static buffalo_status launch_agg(const buffalo_block* blk, const int32_t* col, c
 // A1 row r is A1[gidx ? gidx[r] : r] and is zero for r >= m1.
 constexpr int GB_M = 64, GB_N = 64, GB_K = 16;
 
-// TB: B1 is read transposed (B1[k][n] = B1t[n][k], ldb1 = row pitch of B1t).
+// TB: B1 and B2 are read transposed (B[k][n] = Bt[n][k], ldb = row pitch of Bt).
 template <class TA1, class TA2, class TO, bool TB = false>
 __global__ void __launch_bounds__(256) k_gemm2(int64_t M, int N, int Np, int K1, int K2,
                                                const TA1* __restrict__ A1, int64_t lda1,
@@ -261,7 +263,7 @@ __global__ void __launch_bounds__(256) k_gemm2(int64_t M, int N, int Np, int K1,
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const int nn = n0 + bn + q;
-        Bs[bk][bn + q] = (k < K && nn < N) ? __ldg(TB && first ? B + (int64_t)nn * ldb + k : B + (int64_t)k * ldb + nn)
+        Bs[bk][bn + q] = (k < K && nn < N) ? __ldg(TB ? B + (int64_t)nn * ldb + k : B + (int64_t)k * ldb + nn)
                                            : 0.f;
       }
     }
@@ -800,6 +802,381 @@ static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
 
 buffalo_status pool_bwd_ffma(const PoolArgs& a, cudaStream_t s) {
   return a.in_bf16 ? pool_bwd_t<__nv_bfloat16>(a, s) : pool_bwd_t<float>(a, s);
+}
+
+// ================================================================== GraphSAGE-LSTM (R29)
+// An LSTM (hidden size d = d_{l-1}, gate order i, f, u, o) over each dst row's sampled
+// neighbours in CSR order.  The rows are walked in degree-class order (cls_perm, ascending D),
+// so the rows still running at step t are a suffix [s_t, n) of the permutation (the packed-
+// sequence layout): step t is one gate GEMM over c_t = n - s_t rows plus one cell kernel, and
+// the per-step tensors are stored packed, step after step (off_t = sum of earlier c_t'), e rows
+// in all.  Rows with D > kHeavyT are not supported here (sampled fanouts are <= 32).
+__device__ __forceinline__ float sigm(float x) { return 1.f / (1.f + expf(-x)); }
+
+// counts of rows per degree class min(D, kHeavyT + 1) and the maximum degree (cnt[kHeavyT + 2])
+__global__ void __launch_bounds__(256) k_lstm_hist(const int32_t* __restrict__ rp, int64_t n, int32_t* __restrict__ cnt) {
+  __shared__ int32_t sh[kHeavyT + 3];
+  for (int i = threadIdx.x; i < kHeavyT + 3; i += blockDim.x) sh[i] = 0;
+  __syncthreads();
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t D = rp[i + 1] - rp[i];
+    atomicAdd(&sh[D > kHeavyT ? kHeavyT + 1 : D], 1);
+    atomicMax(&sh[kHeavyT + 2], D);
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < kHeavyT + 2; i += blockDim.x)
+    if (sh[i]) atomicAdd(&cnt[i], sh[i]);
+  if (threadIdx.x == 0) atomicMax(&cnt[kHeavyT + 2], sh[kHeavyT + 2]);
+}
+
+// step t: source row (gix) of each running row's t-th neighbour, packed position of the edge
+__global__ void k_lstm_gix(const int32_t* __restrict__ perm, const int32_t* __restrict__ rp,
+                           const int32_t* __restrict__ colsrc, int64_t s_t, int64_t c_t, int t, int64_t off_t,
+                           int32_t* __restrict__ gix, int32_t* __restrict__ ppos) {
+  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < c_t; q += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t e = rp[perm[s_t + q]] + t;
+    gix[off_t + q] = colsrc[e];
+    ppos[e] = (int32_t)(off_t + q);
+  }
+}
+
+// step t cell: gates (pre-activation, from the GEMM) -> i, f, u, o saved in place; c_t saved
+// packed; running state (h, c) of row r = s_t + q updated.
+__global__ void k_lstm_cell(float* __restrict__ G, int64_t ldg, float* __restrict__ Cs, float* __restrict__ Hs,
+                            float* __restrict__ Cst, int64_t s_t, int64_t c_t, int t, int d, int64_t dp) {
+  const int64_t total = c_t * d;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total; x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t q = x / d;
+    const int k = (int)(x - q * d);
+    const int64_t r = s_t + q;
+    float* g = G + q * ldg;
+    const float gi = sigm(g[k]), gf = sigm(g[d + k]), gu = tanhf(g[2 * d + k]), go = sigm(g[3 * d + k]);
+    const float cp = t ? Cst[r * dp + k] : 0.f;
+    const float c = gf * cp + gi * gu;
+    g[k] = gi;
+    g[d + k] = gf;
+    g[2 * d + k] = gu;
+    g[3 * d + k] = go;
+    Cs[q * dp + k] = c;
+    Cst[r * dp + k] = c;
+    Hs[r * dp + k] = go * tanhf(c);
+  }
+}
+
+// h_agg[perm[r]] = last hidden state (0 for D = 0), padding columns 0
+__global__ void k_lstm_final(const int32_t* __restrict__ perm, const int32_t* __restrict__ rp,
+                             const float* __restrict__ Hs, int64_t n, int d, int64_t dp, float* __restrict__ agg,
+                             int64_t ld_agg) {
+  const int64_t total = n * dp;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total; x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = x / dp;
+    const int k = (int)(x - r * dp);
+    const int32_t i = perm[r];
+    agg[(int64_t)i * ld_agg + k] = (k < d && rp[i + 1] > rp[i]) ? Hs[r * dp + k] : 0.f;
+  }
+}
+
+// backward state: dh = dh_agg of the row, dc = 0
+__global__ void k_lstm_bwd_init(const int32_t* __restrict__ perm, const float* __restrict__ dagg, int64_t n,
+                                int64_t dp, float* __restrict__ dhs, float* __restrict__ dcs) {
+  const int64_t total = n * dp;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total; x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = x / dp;
+    const int64_t k = x - r * dp;
+    dhs[x] = dagg[(int64_t)perm[r] * dp + k];
+    dcs[x] = 0.f;
+  }
+}
+
+// step t of the backward: gate pre-activation gradients (written over the saved gates), h_{t-1}
+// (recomputed from step t-1's o and c) for dW_hh, dc carried to t-1.
+__global__ void k_lstm_cell_bwd(float* __restrict__ G, int64_t ldg, const float* __restrict__ Cs, int64_t dp,
+                                int64_t off_t, int64_t s_t, int64_t c_t, int64_t off_p, int64_t s_p, int t, int d,
+                                const float* __restrict__ dhs, float* __restrict__ dcs, float* __restrict__ Hprev) {
+  const int64_t total = c_t * d;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total; x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t q = x / d;
+    const int k = (int)(x - q * d);
+    const int64_t r = s_t + q, p = off_t + q;
+    float* g = G + p * ldg;
+    const float gi = g[k], gf = g[d + k], gu = g[2 * d + k], go = g[3 * d + k];
+    const float c = Cs[p * dp + k];
+    float cp = 0.f, hp = 0.f;
+    if (t) {
+      const int64_t pp = off_p + (r - s_p);
+      cp = Cs[pp * dp + k];
+      hp = G[pp * ldg + 3 * d + k] * tanhf(cp);
+    }
+    Hprev[p * dp + k] = hp;
+    const float dh = dhs[r * dp + k];
+    const float tc = tanhf(c);
+    const float dc = dcs[r * dp + k] + dh * go * (1.f - tc * tc);
+    g[k] = dc * gu * gi * (1.f - gi);
+    g[d + k] = dc * cp * gf * (1.f - gf);
+    g[2 * d + k] = dc * gi * (1.f - gu * gu);
+    g[3 * d + k] = dh * tc * go * (1.f - go);
+    dcs[r * dp + k] = dc * gf;
+  }
+}
+
+// dh_src[j] += sum over the dst i of src j (ascending i) of dx at the packed position of edge
+// (i, j); warp per src row, the edge found by a ballot over row i.
+__global__ void __launch_bounds__(256) k_lstm_scatterT(const int32_t* __restrict__ trp, const int32_t* __restrict__ tcol,
+                                                       const int32_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                                       const int32_t* __restrict__ ppos, int64_t n_src,
+                                                       const float* __restrict__ dx, int64_t dp, int d,
+                                                       float* __restrict__ out, int64_t ldo) {
+  const int lane = threadIdx.x & 31;
+  const int nch = (int)(dp / 4);
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t j = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; j < n_src; j += warps) {
+    const int32_t t0 = trp[j], t1 = trp[j + 1];
+    for (int c0 = 0; c0 < nch; c0 += 32) {
+      const int c = c0 + lane;
+      float acc[4] = {0.f, 0.f, 0.f, 0.f};
+      for (int32_t t = t0; t < t1; ++t) {
+        const int32_t i = tcol[t];
+        int32_t e = -1;
+        for (int32_t e0 = rp[i]; e0 < rp[i + 1] && e < 0; e0 += 32) {
+          const bool hit = e0 + lane < rp[i + 1] && col[e0 + lane] == (int32_t)j;
+          const unsigned m = __ballot_sync(0xffffffffu, hit);
+          if (m) e = e0 + __ffs(m) - 1;
+        }
+        if (c < nch) {
+          float v[4];
+          VecIO<float, 4>::load(dx + (int64_t)ppos[e] * dp + c * 4, v);
+#pragma unroll
+          for (int k = 0; k < 4; ++k) acc[k] += v[k];
+        }
+      }
+      if (c < nch) {
+        float o[4];
+        VecIO<float, 4>::load(out + j * ldo + c * 4, o);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) o[k] = (c * 4 + k < d) ? o[k] + acc[k] : o[k];
+        VecIO<float, 4>::store(out + j * ldo + c * 4, o);
+      }
+    }
+  }
+}
+
+int lstm_dw_splits(int64_t n_rows, int d) {
+  const int64_t tiles = ceil_div(4 * d, 64) * ceil_div(d, 64);
+  const int64_t a = ceil_div(296, tiles), b = ceil_div(n_rows > 0 ? n_rows : 1, 512);
+  const int64_t sp = a < b ? a : b;
+  return (int)(sp < 1 ? 1 : sp);
+}
+
+int64_t lstm_saved_bytes(int64_t n, int64_t e, int d) {
+  const int64_t dp = pitch_of(d), ldg = pitch_of(4 * d);
+  return R(e * ldg * 4) + R(e * dp * 4) + 2 * R(e * 4) + 2 * R(n * dp * 4) + R(4 * 256);
+}
+
+struct LstmSaved {
+  float *G, *Cs;
+  int32_t *gix, *ppos;
+  float *Hs, *Cst;
+  int32_t* cnt;
+};
+static LstmSaved lstm_saved_view(void* base, int64_t n, int64_t e, int d) {
+  const int64_t dp = pitch_of(d), ldg = pitch_of(4 * d);
+  char* q = (char*)base;
+  LstmSaved v;
+  v.G = (float*)q; q += R(e * ldg * 4);
+  v.Cs = (float*)q; q += R(e * dp * 4);
+  v.gix = (int32_t*)q; q += R(e * 4);
+  v.ppos = (int32_t*)q; q += R(e * 4);
+  v.Hs = (float*)q; q += R(n * dp * 4);
+  v.Cst = (float*)q; q += R(n * dp * 4);
+  v.cnt = (int32_t*)q;
+  return v;
+}
+
+int64_t lstm_bwd_scratch_bytes(int64_t n_dst, int64_t e, int layer, int d_in, int d_out) {
+  const int S = dw_splits(n_dst, d_out, d_in), S3 = lstm_dw_splits(e, d_in);
+  const int64_t dp = pitch_of(d_in);
+  int64_t b = R((int64_t)S * d_out * 2 * d_in * 4) + R((int64_t)S * pitch_of(d_out) * 4);
+  b += R(n_dst * dp * 4) + R(e * dp * 4);
+  if (layer >= 2) b += R(e * dp * 4);
+  b += R((int64_t)S3 * 4 * d_in * d_in * 4) + R((int64_t)S3 * pitch_of(4 * d_in) * 4);
+  return b;
+}
+
+// Step table from the degree-class counts (one 520-byte read-back: the GEMM sizes are
+// data dependent).  s[t] = first running row at step t, off[t] = packed offset, T = max D.
+static buffalo_status lstm_steps(const buffalo_block* blk, int32_t* cnt_dev, std::vector<int64_t>& s,
+                                 std::vector<int64_t>& off, int& T, cudaStream_t st) {
+  const int64_t n = blk->n_dst;
+  int32_t h[kHeavyT + 3] = {0};
+  if (n > 0) {
+    BF_CUDA(cudaMemcpyAsync(h, cnt_dev, sizeof(h), cudaMemcpyDeviceToHost, st));
+    BF_CUDA(cudaStreamSynchronize(st));
+  }
+  if (h[kHeavyT + 1] > 0) {
+    set_error("lstm: rows with more than %d neighbours are not supported (max degree %d)", kHeavyT, h[kHeavyT + 2]);
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
+  T = h[kHeavyT + 2];
+  s.assign(T + 1, n);
+  off.assign(T + 1, 0);
+  int64_t run = n - h[0];            // rows with D > 0
+  int64_t o = 0;
+  for (int t = 0; t < T; ++t) {
+    s[t] = n - run;
+    off[t] = o;
+    o += run;
+    run -= h[t + 1];                 // rows with D = t + 1 stop after step t
+  }
+  off[T] = o;
+  if (o != blk->n_edges) {
+    set_error("lstm: packed steps %lld != edges %lld", (long long)o, (long long)blk->n_edges);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  return BUFFALO_OK;
+}
+
+template <class TI>
+static buffalo_status lstm_fwd_t(const LstmArgs& a, cudaStream_t st) {
+  const buffalo_block* blk = a.blk;
+  const int64_t n = blk->n_dst, e = blk->n_edges;
+  const int d = a.d_in;
+  const int64_t dp = pitch_of(d), ldg = pitch_of(4 * d);
+  LstmSaved v = lstm_saved_view(a.saved, n, e, d);
+  BF_CUDA(cudaMemsetAsync(v.cnt, 0, 4 * (kHeavyT + 3), st));
+  if (n > 0) {
+    k_lstm_hist<<<grid_for(n, 256, 4), 256, 0, st>>>(blk->row_ptr, n, v.cnt);
+    BF_LAUNCHED("k_lstm_hist");
+  }
+  std::vector<int64_t> s, off;
+  int T = 0;
+  BF_CHECK(lstm_steps(blk, v.cnt, s, off, T, st));
+  const int32_t* colsrc = a.layer1 ? blk->col_global : blk->col_local;
+  for (int t = 0; t < T; ++t) {
+    const int64_t c_t = n - s[t];
+    k_lstm_gix<<<grid_for(c_t, 256), 256, 0, st>>>(blk->cls_perm, blk->row_ptr, colsrc, s[t], c_t, t, off[t], v.gix,
+                                                   v.ppos);
+    BF_LAUNCHED("k_lstm_gix");
+    dim3 grid((unsigned)ceil_div(c_t, GB_M), (unsigned)ceil_div(ldg, GB_N));
+    const ProfSlot ps = prof_begin_launch("lstm_gates", st);
+    k_gemm2<TI, float, float, true><<<grid, 256, 0, st>>>(c_t, 4 * d, (int)ldg, d, t ? d : 0, (const TI*)a.h_src,
+                                                         a.ld_src, v.gix + off[t], c_t, v.Hs + s[t] * dp, dp,
+                                                         a.W_ih, d, a.W_hh, d, a.b_lstm, 0, v.G + off[t] * ldg, ldg);
+    BF_LAUNCHED("k_gemm2");
+    // "algorithmic bytes" of this family are FLOPs: 2 * rows * 4d * (d [x_t] + d [h_{t-1}, t > 0])
+    prof_end_launch(ps, st, 2.0 * (double)c_t * 4.0 * d * (double)(t ? 2 * d : d), 0.0);
+    k_lstm_cell<<<grid_for(c_t * d, 256), 256, 0, st>>>(v.G + off[t] * ldg, ldg, v.Cs + off[t] * dp, v.Hs, v.Cst,
+                                                        s[t], c_t, t, d, dp);
+    BF_LAUNCHED("k_lstm_cell");
+  }
+  if (n <= 0) return BUFFALO_OK;
+  k_lstm_final<<<grid_for(n * dp, 256), 256, 0, st>>>(blk->cls_perm, blk->row_ptr, v.Hs, n, d, dp, a.agg, a.ld_agg);
+  BF_LAUNCHED("k_lstm_final");
+  const int Np = (int)pitch_of(a.d_out);
+  dim3 grid((unsigned)ceil_div(n, GB_M), (unsigned)ceil_div(Np, GB_N));
+  const float* Wt = a.W_packed;   // [2 d_in][d_out]
+  k_gemm2<TI, float, float><<<grid, 256, 0, st>>>(n, a.d_out, Np, d, d, (const TI*)a.h_src, a.ld_src,
+                                                 a.layer1 ? blk->src_global : nullptr, n, a.agg, a.ld_agg, Wt,
+                                                 a.d_out, Wt + (int64_t)d * a.d_out, a.d_out, a.b, !a.last, a.out,
+                                                 a.ld_out);
+  BF_LAUNCHED("k_gemm2");
+  return BUFFALO_OK;
+}
+
+buffalo_status lstm_fwd_ffma(const LstmArgs& a, cudaStream_t s) {
+  return a.in_bf16 ? lstm_fwd_t<__nv_bfloat16>(a, s) : lstm_fwd_t<float>(a, s);
+}
+
+template <class TI>
+static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
+  const buffalo_block* blk = a.blk;
+  const int64_t n = blk->n_dst, e = blk->n_edges, ns = blk->n_src;
+  const int d = a.d_in, d_out = a.d_out;
+  const int64_t dp = pitch_of(d), ldg = pitch_of(4 * d);
+  const int32_t* gidx = a.layer1 ? blk->src_global : nullptr;
+  LstmSaved v = lstm_saved_view(a.saved, n, e, d);
+  if (!a.last && n > 0) {
+    k_dz_mask<float><<<grid_for(n * d_out, 256), 256, 0, st>>>(a.dh, a.ld_dh, a.h_dst, a.ld_hdst, n, d_out);
+    BF_LAUNCHED("k_dz_mask");
+  }
+  const int S = dw_splits(n, d_out, d), S3 = lstm_dw_splits(e, d);
+  char* q = (char*)a.scratch;
+  float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * d * 4);
+  float* db_part = (float*)q; q += R((int64_t)S * pitch_of(d_out) * 4);
+  float* dagg = (float*)q; q += R(n * dp * 4);
+  float* Hprev = (float*)q; q += R(e * dp * 4);
+  float* dX = nullptr;
+  if (a.dh_src) { dX = (float*)q; q += R(e * dp * 4); }
+  float* dwl_part = (float*)q; q += R((int64_t)S3 * 4 * d * d * 4);
+  float* dbl_part = (float*)q;
+  if (n > 0) {
+    dim3 g((unsigned)ceil_div(2 * d, 64), (unsigned)ceil_div(d_out, 64), (unsigned)S);
+    k_dw_partial<TI, float><<<g, 256, 0, st>>>(n, d_out, d, 2 * d, a.dh, a.ld_dh, (const TI*)a.h_src, a.ld_src, gidx,
+                                               a.agg, a.ld_agg, ceil_div(n, S), dw_part, db_part);
+    BF_LAUNCHED("k_dw_partial");
+    k_reduce_partials<<<grid_for((int64_t)d_out * 2 * d, 256), 256, 0, st>>>(dw_part, S, (int64_t)d_out * 2 * d, a.dW);
+    BF_LAUNCHED("k_reduce_partials");
+    k_reduce_partials<<<1, 256, 0, st>>>(db_part, S, d_out, a.db);
+    BF_LAUNCHED("k_reduce_partials");
+    dim3 gg((unsigned)ceil_div(n, GB_M), (unsigned)ceil_div(dp, GB_N));
+    k_gemm2<float, float, float><<<gg, 256, 0, st>>>(n, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
+                                                    a.W + d, 2 * d, nullptr, 0, nullptr, 0, dagg, dp);
+    BF_LAUNCHED("k_gemm2");
+    k_lstm_bwd_init<<<grid_for(n * dp, 256), 256, 0, st>>>(blk->cls_perm, dagg, n, dp, v.Hs, v.Cst);
+    BF_LAUNCHED("k_lstm_bwd_init");
+  }
+  std::vector<int64_t> s, off;
+  int T = 0;
+  BF_CHECK(lstm_steps(blk, v.cnt, s, off, T, st));
+  for (int t = T - 1; t >= 0; --t) {
+    const int64_t c_t = n - s[t];
+    k_lstm_cell_bwd<<<grid_for(c_t * d, 256), 256, 0, st>>>(v.G, ldg, v.Cs, dp, off[t], s[t], c_t, t ? off[t - 1] : 0,
+                                                            t ? s[t - 1] : 0, t, d, v.Hs, v.Cst, Hprev);
+    BF_LAUNCHED("k_lstm_cell_bwd");
+    if (t > 0) {   // dh_{t-1} = dG_t W_hh into the running rows' state
+      dim3 gg((unsigned)ceil_div(c_t, GB_M), (unsigned)ceil_div(dp, GB_N));
+      k_gemm2<float, float, float><<<gg, 256, 0, st>>>(c_t, d, (int)dp, 4 * d, 0, v.G + off[t] * ldg, ldg, nullptr, c_t,
+                                                      nullptr, 0, a.W_hh, d, nullptr, 0, nullptr, 0, v.Hs + s[t] * dp,
+                                                      dp);
+      BF_LAUNCHED("k_gemm2");
+    }
+  }
+  if (e > 0) {
+    // dW_ih (+ db_lstm) = dG^T X over the packed rows, then dW_hh = dG^T H_prev
+    dim3 g3((unsigned)ceil_div(d, 64), (unsigned)ceil_div(4 * d, 64), (unsigned)S3);
+    k_dw_partial<TI, float><<<g3, 256, 0, st>>>(e, 4 * d, d, d, v.G, ldg, (const TI*)a.h_src, a.ld_src, v.gix, nullptr,
+                                                0, ceil_div(e, S3), dwl_part, dbl_part);
+    BF_LAUNCHED("k_dw_partial");
+    k_reduce_partials<<<grid_for((int64_t)4 * d * d, 256), 256, 0, st>>>(dwl_part, S3, (int64_t)4 * d * d, a.dW_ih);
+    BF_LAUNCHED("k_reduce_partials");
+    k_reduce_partials<<<grid_for(4 * d, 256), 256, 0, st>>>(dbl_part, S3, 4 * d, a.db_lstm);
+    BF_LAUNCHED("k_reduce_partials");
+    k_dw_partial<float, float><<<g3, 256, 0, st>>>(e, 4 * d, d, d, v.G, ldg, Hprev, dp, nullptr, nullptr, 0,
+                                                   ceil_div(e, S3), dwl_part, dbl_part);
+    BF_LAUNCHED("k_dw_partial");
+    k_reduce_partials<<<grid_for((int64_t)4 * d * d, 256), 256, 0, st>>>(dwl_part, S3, (int64_t)4 * d * d, a.dW_hh);
+    BF_LAUNCHED("k_reduce_partials");
+  }
+  if (a.dh_src && ns > 0) {   // dH_{l-1} = pad(dZ W_self) + sum over edges of dG W_ih
+    dim3 gg((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dp, GB_N));
+    k_gemm2<float, float, float><<<gg, 256, 0, st>>>(ns, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
+                                                    a.W, 2 * d, nullptr, 0, nullptr, 0, a.dh_src, a.ld_dh_src);
+    BF_LAUNCHED("k_gemm2");
+    if (e > 0) {
+      dim3 gx((unsigned)ceil_div(e, GB_M), (unsigned)ceil_div(dp, GB_N));
+      k_gemm2<float, float, float><<<gx, 256, 0, st>>>(e, d, (int)dp, 4 * d, 0, v.G, ldg, nullptr, e, nullptr, 0,
+                                                      a.W_ih, d, nullptr, 0, nullptr, 0, dX, dp);
+      BF_LAUNCHED("k_gemm2");
+      k_lstm_scatterT<<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(blk->t_row_ptr, blk->t_col, blk->row_ptr,
+                                                                  blk->col_local, v.ppos, ns, dX, dp, d, a.dh_src,
+                                                                  a.ld_dh_src);
+      BF_LAUNCHED("k_lstm_scatterT");
+    }
+  }
+  return BUFFALO_OK;
+}
+
+buffalo_status lstm_bwd_ffma(const LstmArgs& a, cudaStream_t s) {
+  return a.in_bf16 ? lstm_bwd_t<__nv_bfloat16>(a, s) : lstm_bwd_t<float>(a, s);
 }
 
 }  // namespace buffalo

@@ -56,6 +56,29 @@ int64_t pool_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int d_in, int d_out
 buffalo_status pool_fwd_ffma(const PoolArgs& a, cudaStream_t s);
 buffalo_status pool_bwd_ffma(const PoolArgs& a, cudaStream_t s);
 
+// GraphSAGE-LSTM (R29): FFMA path, fp32 activations.
+struct LstmArgs {
+  const buffalo_block* blk;
+  bool layer1, in_bf16, last;
+  int d_in, d_out;
+  const void* h_src; int64_t ld_src;
+  const float* W_ih; const float* W_hh; const float* b_lstm;
+  const float* W; const float* W_packed; const float* b;
+  float* out; int64_t ld_out;
+  float* agg; int64_t ld_agg;
+  void* saved;
+  float* dh; int64_t ld_dh;
+  const float* h_dst; int64_t ld_hdst;
+  float* dW_ih; float* dW_hh; float* db_lstm; float* dW; float* db;
+  float* dh_src; int64_t ld_dh_src;
+  void* scratch;
+};
+int lstm_dw_splits(int64_t n_rows, int d);
+int64_t lstm_saved_bytes(int64_t n, int64_t e, int d);
+int64_t lstm_bwd_scratch_bytes(int64_t n_dst, int64_t e, int layer, int d_in, int d_out);
+buffalo_status lstm_fwd_ffma(const LstmArgs& a, cudaStream_t s);
+buffalo_status lstm_bwd_ffma(const LstmArgs& a, cudaStream_t s);
+
 int dw_splits(int64_t n_l, int d_out, int d_in);
 int64_t bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int layer, int d_in, int d_out);
 

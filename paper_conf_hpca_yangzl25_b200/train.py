@@ -47,11 +47,14 @@ class DeviceGraph:
 class SageParams:
     """fp32 master weights/biases (Xavier init from synth), flat gradient buffer, packed copies."""
 
-    def __init__(self, model, Ws, bs, device="cuda", Wps=None, bps=None):
+    def __init__(self, model, Ws, bs, device="cuda", Wps=None, bps=None, lstm=None):
         self.model = model
         self.L = model.num_layers
         Wps, bps = list(Wps or []), list(bps or [])
-        sizes = [w.size for w in Ws] + [b.size for b in bs] + [w.size for w in Wps] + [b.size for b in bps]
+        Wih, Whh, bl = [list(x) for x in lstm] if lstm else ([], [], [])
+        extra = Wih + Whh + bl
+        sizes = [w.size for w in Ws] + [b.size for b in bs] + [w.size for w in Wps] + [b.size for b in bps] + \
+            [w.size for w in extra]
         self.flat = torch.zeros(sum(sizes), dtype=torch.float32, device=device)
         self.grad = torch.zeros_like(self.flat)
         self.W, self.b, self.dW, self.db = [], [], [], []
@@ -78,6 +81,14 @@ class SageParams:
             self.dbp.append(self.grad[off:off + b.size])
             self.bp[-1].copy_(torch.as_tensor(b))
             off += b.size
+        # GraphSAGE-LSTM weights (R29): W_ih, W_hh [4d, d], b [4d] per layer
+        self.lstm, self.dlstm = [[], [], []], [[], [], []]
+        for k, group in enumerate((Wih, Whh, bl)):
+            for w in group:
+                self.lstm[k].append(self.flat[off:off + w.size].view(w.shape))
+                self.dlstm[k].append(self.grad[off:off + w.size].view(w.shape))
+                self.lstm[k][-1].copy_(torch.as_tensor(w))
+                off += w.size
         self.packed = [torch.empty(B.packed_weight_bytes(model, l), dtype=torch.uint8, device=device)
                        for l in range(1, self.L + 1)]
         self.repack()
@@ -91,7 +102,7 @@ class Trainer:
     def __init__(self, graph, feats, labels, seeds, dims, fanout, F, Ws, bs, feat_dtype=B.FP32,
                  gemm_mode=B.GEMM_FFMA, mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096,
                  base_seed=3, rank=0, world=1, process_group=None, device="cuda", aggregator=B.AGG_MEAN,
-                 Wps=None, bps=None):
+                 Wps=None, bps=None, lstm=None):
         self.graph = graph if isinstance(graph, DeviceGraph) else DeviceGraph(*graph, device=device)
         self.feats = feats
         self.labels = labels
@@ -103,11 +114,14 @@ class Trainer:
         self.F = F
         self.base_seed = base_seed
         self.pool = aggregator == B.AGG_POOL
+        self.is_lstm = aggregator == B.AGG_LSTM
         if self.pool and Wps is None:
             raise ValueError("the pool aggregator needs its weights (Wps, bps)")
+        if self.is_lstm and lstm is None:
+            raise ValueError("the LSTM aggregator needs its weights (W_ih, W_hh, b per layer)")
         self.model = B.make_model(dims, feat_dtype, gemm_mode, feats.shape[1], aggregator)
         self.sched = B.make_sched(mem_budget, C_ppm, k_min, k_max, world)
-        self.params = SageParams(self.model, Ws, bs, device, Wps, bps)
+        self.params = SageParams(self.model, Ws, bs, device, Wps, bps, lstm)
         self.rank, self.world, self.pg = rank, world, process_group
         self.device = device
         # scheduler outputs
@@ -171,7 +185,10 @@ class Trainer:
         h, ld = self.feats, self.feats.shape[1]
         for l in range(1, self.L + 1):
             b = blks.layer[l - 1]
-            if self.pool:
+            if self.is_lstm:
+                B.lstm_fwd(b, l, m, h, ld, p.lstm[0][l - 1], p.lstm[1][l - 1], p.lstm[2][l - 1], p.W[l - 1],
+                           p.packed[l - 1], p.b[l - 1], b.out, b.ld_out, b.agg, b.ld_agg)
+            elif self.pool:
                 B.pool_fwd(b, l, m, h, ld, p.Wp[l - 1], p.bp[l - 1], p.W[l - 1], p.packed[l - 1], p.b[l - 1],
                            b.out, b.ld_out, b.agg, b.ld_agg, b.pool_P, b.pool_arg, b.ld_pool)
             else:
@@ -190,6 +207,12 @@ class Trainer:
             else:
                 h_src, ld_src, dh_src, ld_dh_src, prev_rp = self.feats, self.feats.shape[1], None, 0, None
             h_dst = b.out if l < self.L else None
+            if self.is_lstm:
+                B.lstm_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out,
+                           p.lstm[0][l - 1], p.lstm[1][l - 1], p.W[l - 1], p.dlstm[0][l - 1], p.dlstm[1][l - 1],
+                           p.dlstm[2][l - 1], p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src, b.bwd_scratch,
+                           b.bwd_scratch_bytes)
+                continue
             if self.pool:
                 B.pool_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out, b.pool_P,
                            b.pool_arg, b.ld_pool, p.Wp[l - 1], p.W[l - 1], p.dWp[l - 1], p.dbp[l - 1],

@@ -283,6 +283,10 @@ CONFIGS = {
     # configs[2]: ogbn-products-shaped, 3-layer, fanout (10,25,30), budget forcing K >= 8.
     "products": Config("products", 2449029, 61859140, "powerlaw", 100, 47, 256, 3, [10, 25, 30], 30,
                        196615, 8, 4096),
+    # The paper's LSTM workload: arxiv-shaped, 2-layer SAGE-LSTM, LSTM hidden 128,
+    # cut-offs 25 (1-hop) and 10 (2-hop) = fanout (10, 25) in DGL order; budget forcing K >= 2.
+    "arxiv_lstm": Config("arxiv_lstm", 169343, 1166243, "powerlaw", 128, 40, 128, 2, [10, 25], 25, 90941, 2,
+                         4096),
     # configs[3]: ogbn-papers100M-shaped, 2-layer, fanout (10,25).
     "papers": Config("papers", 111059956, 1615685872, "powerlaw", 128, 172, 256, 2, [10, 25], 25,
                      1207179, 8, 4096),
