@@ -56,8 +56,9 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="products", choices=list(WORKLOADS))
     ap.add_argument("--gemm", default="bf16", choices=["bf16", "ffma"])
-    ap.add_argument("--aggregator", default="mean", choices=["mean", "pool", "lstm"],
-                    help="pool / lstm: GraphSAGE-pool / -LSTM (SURVEY §8(f) NEXT 2 / 1), fp32 FFMA path only")
+    ap.add_argument("--aggregator", default="mean", choices=["mean", "pool", "lstm", "gat"],
+                    help="pool / lstm: GraphSAGE-pool / -LSTM, gat: GAT (SURVEY §8(f) NEXT 2 / 1 / 3), fp32 FFMA "
+                         "path only")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-baseline-seconds", type=float, default=20.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -247,7 +248,8 @@ def run_ours(args, cfg):
     t_gen = time.perf_counter() - t_gen
     pool = args.aggregator == "pool"
     lstm = args.aggregator == "lstm"
-    if pool or lstm:
+    gat = args.aggregator == "gat"
+    if pool or lstm or gat:
         args.gemm = "ffma"                             # the pool / LSTM aggregators are built for fp32 only
     gemm = B.GEMM_BF16 if args.gemm == "bf16" else B.GEMM_FFMA
     agg_kw = {}
@@ -258,6 +260,10 @@ def run_ours(args, cfg):
     if lstm:
         from synth.graphs import lstm_weights
         agg_kw = dict(aggregator=B.AGG_LSTM, lstm=lstm_weights(cfg.dims))
+    if gat:
+        from synth.graphs import gat_weights
+        Ws, bs, als, ars = gat_weights(cfg.dims)
+        agg_kw = dict(aggregator=B.AGG_GAT, gat=(als, ars))
     feat_dtype = B.BF16 if args.gemm == "bf16" else B.FP32
     feats = X
     if feat_dtype == B.BF16:
@@ -297,7 +303,7 @@ def run_ours(args, cfg):
     clocks.start()
     # live roofline of the dominant kernel (k_gather_rows, the Aggregate): CUDA events around
     # each of its launches on its stream, algorithmic bytes from the edges it aggregated
-    B.profile_begin("lstm_gates" if lstm else "pool_max" if pool else "gather", prof_counters)
+    B.profile_begin("lstm_gates" if lstm else "pool_max" if pool else "gat_attn" if gat else "gather", prof_counters)
     l0 = B.launch_count()
     step_ms, edges, sizes, ks = [], 0, [], []
     torch.cuda.synchronize()
@@ -366,7 +372,8 @@ def run_ours(args, cfg):
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
-        traffic = json.load(open(tpath)).get(f"{args.config}/{args.gemm}" + ("/pool" if pool else ""))
+        traffic = json.load(open(tpath)).get(f"{args.config}/{args.gemm}" + ("" if args.aggregator == "mean" else
+                                                                              "/" + args.aggregator))
     if lstm:   # the LSTM path is bound by its fp32 SIMT gate GEMMs: FLOP roofline ("alu")
         tf = g_bytes / (g_ms / 1e3) / 1e12 if g_ms > 0 else 0.0
         roof = {"bound": "alu", "kernel": "k_gemm2 (LSTM gate GEMM of every step, fp32 SIMT)",
@@ -379,6 +386,7 @@ def run_ours(args, cfg):
     else:
         roof = {"bound": "hbm",
                 "kernel": ("k_pool_max (GraphSAGE-pool neighbour max + argmax)" if pool else
+                           "k_gat_attn (GAT edge softmax + attention-weighted neighbour sum)" if gat else
                            "k_gather_v2 (Aggregate: fwd neighbour mean, bwd transposed sum)"),
                 "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": traffic, "peak_source": peak_src,
@@ -387,7 +395,7 @@ def run_ours(args, cfg):
                 "share_of_step": g_ms / total_ms}
     if rank == 0:
         cpu = None
-        if world == 1 and not args.no_cpu_baseline and not (pool or lstm):   # (the pool oracle is loop-plain: tests only)
+        if world == 1 and not args.no_cpu_baseline and not (pool or lstm or gat):   # (the pool oracle is loop-plain: tests only)
             rp_h, col_h, X_h, y_h, seeds_h = host_copies(rp, col, X, y, tr.seeds)
             cpu = oracle_sample(cfg, rp_h, col_h, X_h, y_h, seeds_h, Ws, bs, args.cpu_baseline_seconds)
         line = dict(
@@ -395,7 +403,10 @@ def run_ours(args, cfg):
             n_gpus=world, steps=args.steps, warmup=args.warmup, ms_per_step=total_ms / args.steps,
             higher_is_better=True, scaling="strong", vs_baseline=None,
             dtype="bf16" if gemm == B.GEMM_BF16 else "f32", data="synthetic",
-            config={"workload": WORKLOADS[args.config], "config": args.config, "K": ks[-1],
+            config={"workload": WORKLOADS[args.config].replace(
+                        "SAGE-mean", {"mean": "SAGE-mean", "pool": "SAGE-pool", "lstm": "SAGE-LSTM",
+                                      "gat": "GAT (one head)"}[args.aggregator]),
+                    "config": args.config, "K": ks[-1],
                     "gemm": args.gemm, "aggregator": args.aggregator,
                     "l2": "flushed (512 MiB write) between timed steps",
                     "epoch_ms": total_ms / args.steps, "edges_per_epoch": edges / args.steps,

@@ -42,7 +42,8 @@ typedef enum {
 
 enum { BUFFALO_FP32 = 0, BUFFALO_BF16 = 1 };            /* storage dtypes                  */
 enum { BUFFALO_GEMM_FFMA = 0, BUFFALO_GEMM_BF16 = 1 };  /* Update GEMM: fp32 SIMT | tcgen05 */
-enum { BUFFALO_AGG_MEAN = 0, BUFFALO_AGG_POOL = 1, BUFFALO_AGG_LSTM = 2 }; /* aggregator (R20, R28, R29) */
+/* model: GraphSAGE with aggregator MEAN / POOL / LSTM, or GAT (R20, R28, R29, R30) */
+enum { BUFFALO_AGG_MEAN = 0, BUFFALO_AGG_POOL = 1, BUFFALO_AGG_LSTM = 2, BUFFALO_AGG_GAT = 3 };
 enum { BUFFALO_MAX_LAYERS = 8, BUFFALO_MAX_FANOUT = 32, BUFFALO_MAX_DIM = 4096 };
 
 /* Input graph (the batch's host graph): CSR, rows sorted ascending, symmetric,
@@ -135,10 +136,11 @@ typedef struct {
   float* pool_P;
   int32_t* pool_arg;
   int64_t ld_pool;
-  /* aggregator LSTM only (else NULL / 0): the layer's saved sequence state (gates, cell states,
-   * per-edge source rows and packed positions, running h/c, degree-class counts), R29. */
-  void* lstm_saved;
-  int64_t lstm_saved_bytes;
+  /* aggregator LSTM / GAT only (else NULL / 0): the layer's saved state — LSTM: gates, cell
+   * states, per-edge source rows and packed positions, running h/c, degree-class counts (R29);
+   * GAT: Z = H W^T, the attention scores el / er and the attention weights per edge (R30). */
+  void* agg_saved;
+  int64_t agg_saved_bytes;
 } buffalo_block;
 
 typedef struct {
@@ -285,15 +287,15 @@ BUFFALO_API buffalo_status buffalo_pool_bwd(const buffalo_block* blk, int32_t la
  * order from zero state; h_agg = its last hidden state (0 for D = 0); then the Update of
  * buffalo_sage_fwd.  The dst rows are processed in degree-class order (the block's cls_perm:
  * the degree buckets of Alg. 2 l.6), so step t is one batched gate GEMM over the rows with
- * D > t.  saved = the block's lstm_saved (kept for the backward).  Synchronises the stream once
+ * D > t.  saved = the block's agg_saved (kept for the backward).  Synchronises the stream once
  * (an 520-byte read of the degree-class counts sizes the per-step launches).  Errors:
  * UNSUPPORTED (a row with more than 128 neighbours; aggregator/gemm_mode), INVALID_ARG. */
 BUFFALO_API buffalo_status buffalo_lstm_fwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
                                 const void* h_src, int64_t ld_src, const float* W_ih,
                                 const float* W_hh, const float* b_lstm, const float* W,
                                 const void* W_packed, const float* b, void* out, int64_t ld_out,
-                                void* saved_agg, int64_t ld_agg, void* lstm_saved,
-                                size_t lstm_saved_bytes, void* stream);
+                                void* saved_agg, int64_t ld_agg, void* agg_saved,
+                                size_t agg_saved_bytes, void* stream);
 /* Backward (back-propagation through the neighbour sequences; gradients accumulated, +=):
  * dZ, dW, db as buffalo_sage_bwd; dh_agg = dZ W_neigh; per step t = T-1..0 the gate gradients,
  * dW_ih += sum dG x^T, dW_hh += sum dG h_{t-1}^T, db_lstm += sum dG (deterministic split
@@ -302,11 +304,35 @@ BUFFALO_API buffalo_status buffalo_lstm_fwd(const buffalo_block* blk, int32_t la
 BUFFALO_API buffalo_status buffalo_lstm_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
                                 float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
                                 const void* saved_agg, int64_t ld_agg, const void* h_dst,
-                                int64_t ld_hdst, void* lstm_saved, size_t lstm_saved_bytes,
+                                int64_t ld_hdst, void* agg_saved, size_t agg_saved_bytes,
                                 const float* W_ih, const float* W_hh, const float* W,
                                 float* dW_ih_accum, float* dW_hh_accum, float* db_lstm_accum,
                                 float* dW_accum, float* db_accum, float* dh_src, int64_t ld_dh_src,
                                 void* scratch, size_t scratch_bytes, void* stream);
+
+/* ------------------------------------------------------------------ GAT */
+/* GAT, the paper's second model (Table IV :499-513), on the
+ * same blocks, reading R30: one attention head per layer.  For block `layer` (model.aggregator =
+ * GAT, gemm_mode FFMA, fp32; W fp32 [d_l][d_{l-1}], a_l, a_r, b fp32 [d_l]): Z = H W^T over the
+ * block's src rows; s_ij = LeakyReLU_0.2(a_l . Z[j] + a_r . Z[i]); alpha = softmax over i's
+ * sampled neighbours; out_i = sum_j alpha_ij Z[j] + b (b for D = 0); ELU for l < L, logits at
+ * l = L.  gat_saved = the block's agg_saved (Z, scores, alpha per edge).  Every reduction order
+ * depends only on the row (deterministic).  Block 1 carries its transpose (the backward needs
+ * dZ over all src rows for dW). */
+BUFFALO_API buffalo_status buffalo_gat_fwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                               const void* h_src, int64_t ld_src, const float* W, const float* a_l,
+                               const float* a_r, const float* b, void* out, int64_t ld_out,
+                               void* gat_saved, size_t gat_saved_bytes, void* stream);
+/* Backward (accumulated, +=): dOut = dH * ELU'(out) (in place), db += sum dOut; per dst the
+ * softmax backward; per src (transposed block, ascending dst) dZ; da_l, da_r, dW = dZ^T H by
+ * deterministic split reductions; dh_src (l >= 2) = dZ W.  scratch: the block's bwd_scratch. */
+BUFFALO_API buffalo_status buffalo_gat_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
+                               float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
+                               const void* h_dst, int64_t ld_hdst, void* gat_saved,
+                               size_t gat_saved_bytes, const float* W, const float* a_l,
+                               const float* a_r, float* dW_accum, float* db_accum, float* da_l_accum,
+                               float* da_r_accum, float* dh_src, int64_t ld_dh_src, void* scratch,
+                               size_t scratch_bytes, void* stream);
 
 /* ------------------------------------------------------------------ a10: optimizer */
 /* SGD (Alg. 2 l.13, R18): param -= lr * grad; grad = 0 (ready for the next epoch). */
@@ -346,7 +372,9 @@ BUFFALO_API buffalo_status buffalo_avg_clustering(const buffalo_graph* g, const 
 BUFFALO_API int64_t buffalo_launch_count(void);
 
 /* Diagnostics (bench roofline): time every launch of one kernel family with CUDA events on the
- * stream it is launched on.  family "lstm_gates": the LSTM gate GEMM of every step; its
+ * stream it is launched on.  family "gat_attn": k_gat_attn (GAT softmax + weighted neighbour
+ * sum; per row 16 B + the output row, per edge 32 B of indices / scores / alpha + the Z row).
+ * family "lstm_gates": the LSTM gate GEMM of every step; its
  * "algorithmic bytes" are FLOPs (2 x rows x 4d x (d + d)).  family "pool_max": k_pool_max, the GraphSAGE-pool neighbour max
  * (per row 12 B + the max and argmax rows, per edge the index and the pooled fp32 row).
  * family "gather": k_gather_rows, the Aggregate of the forward (mean

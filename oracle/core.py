@@ -35,6 +35,11 @@ Functions and the passages they follow:
                        aggregator, Table III :479-497): an LSTM with
                        hidden size d_{l-1} run over each destination's sampled neighbours in CSR
                        order, h_agg = its last hidden state (R29)
+  gat_forward, gat_backward
+                       GAT (the paper's second model, Table IV
+                       :499-513; GAT [68]/[32]) on the same blocks: one attention head per layer,
+                       LeakyReLU(0.2) scores, softmax over the sampled neighbours, ELU between
+                       layers (R30)
   triangles, avg_clustering
                        C of Eq. 1 (Newman's local clustering
                        coefficient, "page 142 of reference [27]"): T_v by definition (C),
@@ -235,6 +240,12 @@ def pool_dw_splits(n_rows, d):
     return max(1, min(_ceil(296, tiles), _ceil(n_rows, 512)))
 
 
+def gemm_splits(n_rows, rows_out, K):
+    """Split count of a deterministic split-K reduction over n_rows (rows_out x K result)."""
+    tiles = _ceil(rows_out, 64) * _ceil(K, 64)
+    return max(1, min(_ceil(296, tiles), _ceil(max(int(n_rows), 1), 512)))
+
+
 def lstm_dw_splits(n_rows, d):
     """Split count of the LSTM weights' dW reduction (4d rows, K = d columns)."""
     tiles = _ceil(4 * d, 64) * _ceil(d, 64)
@@ -251,6 +262,7 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
     s = 4 if act_dtype == FP32 else 2
     pool = aggregator == "pool"                  # R28: fp32 only; block 1 keeps a transpose too
     lstm = aggregator == "lstm"                  # R29: fp32 only
+    gat = aggregator == "gat"                    # R30: fp32 only; block 1 keeps a transpose too
     blocks = 0
     build = 0
     for l in range(1, L + 1):
@@ -258,7 +270,7 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
         blocks += _R(4 * (nl + 1)) + _R(4 * nl) + _R(4 * el) + _R(4 * nm)   # row_ptr cls_perm col src
         if l == 1:
             blocks += _R(4 * el)                                # col_global kept for layer 1
-            if pool:
+            if pool or gat:
                 blocks += _R(4 * (nm + 1)) + _R(4 * el) + _R(4 * nm)
         else:
             blocks += _R(4 * (nm + 1)) + _R(4 * el) + _R(4 * nm)  # transposed block + its classes
@@ -267,15 +279,19 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
         frame += _R(4 * (pne + 1))                              # partition counts (classes, radix)
         if l >= 2:
             frame += _R(4 * el) + _R(4 * (nl + el))             # col_global + transpose cursors
-        elif pool:
+        elif pool or gat:
             frame += _R(4 * (nl + el))                          # transpose cursors of block 1
         build = max(build, frame)
     acts = 0
     for l in range(1, L + 1):
-        acts += _R(n[l] * pitch(dims[l - 1]) * s)               # saved h_agg
+        if not gat:
+            acts += _R(n[l] * pitch(dims[l - 1]) * s)           # saved h_agg
         if l < L:
             acts += _R(n[l] * pitch(dims[l]) * s)               # H_l
     acts += _R(n[L] * pitch(dims[L]) * 4)                       # logits
+    if gat:
+        for l in range(1, L + 1):                               # Z, el, er, alpha per edge
+            acts += _R(n[l - 1] * pitch(dims[l]) * 4) + _R(4 * n[l - 1]) + _R(4 * n[l]) + _R(4 * e[l - 1])
     if lstm:
         for l in range(1, L + 1):
             d, el, nl = dims[l - 1], e[l - 1], n[l]
@@ -305,6 +321,14 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
             frame += _R(n[l] * pitch(d) * 4) + _R(n[l - 1] * pitch(d) * 4)     # dh_agg, dQ
             S2 = pool_dw_splits(n[l - 1], d)
             frame += _R(S2 * d * d * 4) + _R(S2 * pitch(d) * 4)               # dW_pool, db_pool partials
+        if gat:
+            din, dl, ns, nd, el = dims[l - 1], dims[l], n[l - 1], n[l], e[l - 1]
+            frame += _R(ns * pitch(dl) * 4) + _R(4 * el) + _R(4 * ns) + _R(4 * nd)   # dZ, ds, d_el, d_er
+            S4, Sl, Sr = gemm_splits(ns, dl, din), gemm_splits(ns, 1, dl), gemm_splits(nd, 1, dl)
+            frame += _R(S4 * dl * din * 4) + _R(S4 * pitch(dl) * 4)                 # dW partials
+            frame += _R(Sl * dl * 4) + _R(Sl * 4) + _R(Sr * dl * 4) + _R(Sr * 4)     # da_l, da_r partials
+            bwd = max(bwd, frame)
+            continue
         if lstm:
             d, el = dims[l - 1], e[l - 1]
             frame += _R(n[l] * pitch(d) * 4)                     # dh_agg
@@ -684,6 +708,85 @@ def lstm_backward(blocks, cache, Ws, Wihs, Whhs, dlogits):
         if l > 1:
             dHin[:n] += dZ @ W[:, :d]
             dH = dHin
+    return grads
+
+
+def gat_forward(blocks, X, Ws, bs, als, ars, slope=0.2):
+    """GAT forward in float64 (R30; one head per layer, as DGL's GATConv computes it with
+    allow_zero_in_degree).  For block l with input rows H (its src): Z = H W_l^T;
+    el[j] = a_l . Z[j] (every src), er[i] = a_r . Z[i] (dst, the prefix of src);
+    s_ij = LeakyReLU(el[j] + er[i]);  alpha_ij = softmax of s_ij over the sampled neighbours j
+    of i;  out_i = sum_j alpha_ij Z[j] + b_l (b_l alone when D(i) = 0);  H_l = ELU(out) for
+    l < L, logits = out at l = L.  W_l: [d_l, d_{l-1}], a_l, a_r, b_l: [d_l]."""
+    L = len(blocks)
+    H = np.asarray(X, dtype=np.float64)[blocks[0]["src_global"]]
+    cache = []
+    for l in range(1, L + 1):
+        b = blocks[l - 1]
+        W = np.asarray(Ws[l - 1], dtype=np.float64)
+        al = np.asarray(als[l - 1], dtype=np.float64)
+        ar = np.asarray(ars[l - 1], dtype=np.float64)
+        Z = H @ W.T
+        el = Z @ al
+        n = b["n_dst"]
+        er = Z[:n] @ ar
+        rp, col = b["row_ptr"], b["col_local"]
+        alpha = np.zeros(b["n_edges"])
+        out = np.tile(np.asarray(bs[l - 1], dtype=np.float64), (n, 1))
+        for i in range(n):
+            e0, e1 = rp[i], rp[i + 1]
+            if e1 == e0:
+                continue
+            sc = el[col[e0:e1]] + er[i]
+            sc = np.where(sc > 0, sc, slope * sc)
+            w = np.exp(sc - sc.max())
+            alpha[e0:e1] = w / w.sum()
+            out[i] += alpha[e0:e1] @ Z[col[e0:e1]]
+        cache.append(dict(H_in=H, Z=Z, el=el, er=er, alpha=alpha, out=out))
+        H = np.where(out > 0, out, np.expm1(out)) if l < L else out
+    return H, cache
+
+
+def gat_backward(blocks, cache, Ws, als, ars, dlogits, slope=0.2):
+    """Backward of gat_forward: per layer (dW_l, db_l, da_l, da_r).
+    dOut = dH * ELU'(out) (dOut_L = dlogits);  db = sum dOut;  dZ[j] = sum_i alpha_ij dOut_i;
+    dalpha_ij = dOut_i . Z[j];  ds_ij = alpha_ij (dalpha_ij - sum_k alpha_ik dalpha_ik) * LeakyReLU';
+    dZ[j] += (sum_i ds_ij) a_l;  dZ[i] += (sum_j ds_ij) a_r;  da_l = sum_j (sum_i ds_ij) Z[j];
+    da_r = sum_i (sum_j ds_ij) Z[i];  dW = dZ^T H;  dH_{l-1} = dZ W."""
+    L = len(blocks)
+    grads = [None] * L
+    dH = np.asarray(dlogits, dtype=np.float64)
+    for l in range(L, 0, -1):
+        c = cache[l - 1]
+        b = blocks[l - 1]
+        W = np.asarray(Ws[l - 1], dtype=np.float64)
+        al = np.asarray(als[l - 1], dtype=np.float64)
+        ar = np.asarray(ars[l - 1], dtype=np.float64)
+        out, Z, alpha = c["out"], c["Z"], c["alpha"]
+        dO = dH if l == L else dH * np.where(out > 0, 1.0, np.exp(out))
+        n = dO.shape[0]
+        rp, col = b["row_ptr"], b["col_local"]
+        dZ = np.zeros_like(Z)
+        d_el = np.zeros(Z.shape[0])
+        d_er = np.zeros(n)
+        for i in range(n):
+            e0, e1 = rp[i], rp[i + 1]
+            if e1 == e0:
+                continue
+            nb = col[e0:e1]
+            a = alpha[e0:e1]
+            dZ[nb] += np.outer(a, dO[i])
+            da = Z[nb] @ dO[i]
+            de = a * (da - a @ da)
+            sc = c["el"][nb] + c["er"][i]
+            ds = de * np.where(sc > 0, 1.0, slope)
+            d_er[i] = ds.sum()
+            np.add.at(d_el, nb, ds)
+        dZ += np.outer(d_el, al)
+        dZ[:n] += np.outer(d_er, ar)
+        grads[l - 1] = (dZ.T @ c["H_in"], dO.sum(axis=0), d_el @ Z, d_er @ Z[:n])
+        if l > 1:
+            dH = dZ @ W
     return grads
 
 

@@ -20,7 +20,7 @@ c_i32, c_i64, c_u64, c_p, c_sz, c_f = (ctypes.c_int32, ctypes.c_int64, ctypes.c_
 OK, ERR_INVALID_ARG, ERR_BUDGET, ERR_CAPACITY, ERR_CUDA, ERR_UNSUPPORTED = range(6)
 FP32, BF16 = 0, 1
 GEMM_FFMA, GEMM_BF16 = 0, 1
-AGG_MEAN, AGG_POOL, AGG_LSTM = 0, 1, 2
+AGG_MEAN, AGG_POOL, AGG_LSTM, AGG_GAT = 0, 1, 2, 3
 MAX_LAYERS = 8
 
 EXPORTS = [
@@ -32,6 +32,7 @@ EXPORTS = [
     "buffalo_status_str", "buffalo_last_error",
     "buffalo_clustering_workspace_bytes", "buffalo_triangles", "buffalo_avg_clustering",
     "buffalo_pool_fwd", "buffalo_pool_bwd", "buffalo_lstm_fwd", "buffalo_lstm_bwd",
+    "buffalo_gat_fwd", "buffalo_gat_bwd",
 ]
 
 
@@ -78,7 +79,7 @@ class Block(ctypes.Structure):
                 ("agg", c_p), ("out", c_p), ("dh", c_p), ("bwd_scratch", c_p),
                 ("ld_agg", c_i64), ("ld_out", c_i64), ("ld_dh", c_i64), ("bwd_scratch_bytes", c_i64),
                 ("pool_P", c_p), ("pool_arg", c_p), ("ld_pool", c_i64),
-                ("lstm_saved", c_p), ("lstm_saved_bytes", c_i64)]
+                ("agg_saved", c_p), ("agg_saved_bytes", c_i64)]
 
 
 class Blocks(ctypes.Structure):
@@ -124,6 +125,9 @@ def lib(require_gpu=True):
             "buffalo_lstm_fwd": (c_i32, [P, c_i32, P, P, c_i64, P, P, P, P, P, P, P, c_i64, P, c_i64, P, c_sz, P]),
             "buffalo_lstm_bwd": (c_i32, [P, c_i32, P, P, c_i64, P, c_i64, P, c_i64, P, c_i64, P, c_sz, P, P, P,
                                          P, P, P, P, P, P, c_i64, P, c_sz, P]),
+            "buffalo_gat_fwd": (c_i32, [P, c_i32, P, P, c_i64, P, P, P, P, P, c_i64, P, c_sz, P]),
+            "buffalo_gat_bwd": (c_i32, [P, c_i32, P, P, c_i64, P, c_i64, P, c_i64, P, c_sz, P, P, P, P, P, P, P, P,
+                                        c_i64, P, c_sz, P]),
             "buffalo_status_str": (ctypes.c_char_p, [c_i32]),
             "buffalo_last_error": (ctypes.c_char_p, []),
         }
@@ -247,16 +251,29 @@ def lstm_fwd(blk, layer, model, h_src, ld_src, W_ih, W_hh, b_lstm, W, W_packed, 
              stream=None):
     _check(lib().buffalo_lstm_fwd(ref(blk), layer, ref(model), ptr(h_src), ld_src, ptr(W_ih), ptr(W_hh), ptr(b_lstm),
                                   ptr(W), ptr(W_packed), ptr(b), ptr(out), ld_out, ptr(saved_agg), ld_agg,
-                                  ptr(blk.lstm_saved), blk.lstm_saved_bytes, stream_ptr(stream)))
+                                  ptr(blk.agg_saved), blk.agg_saved_bytes, stream_ptr(stream)))
 
 
 def lstm_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg, h_dst, ld_hdst, W_ih, W_hh, W,
              dW_ih, dW_hh, db_lstm, dW, db, dh_src, ld_dh_src, scratch, scratch_bytes, stream=None):
     _check(lib().buffalo_lstm_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh, ptr(h_src), ld_src,
-                                  ptr(saved_agg), ld_agg, ptr(h_dst), ld_hdst, ptr(blk.lstm_saved),
-                                  blk.lstm_saved_bytes, ptr(W_ih), ptr(W_hh), ptr(W), ptr(dW_ih), ptr(dW_hh),
+                                  ptr(saved_agg), ld_agg, ptr(h_dst), ld_hdst, ptr(blk.agg_saved),
+                                  blk.agg_saved_bytes, ptr(W_ih), ptr(W_hh), ptr(W), ptr(dW_ih), ptr(dW_hh),
                                   ptr(db_lstm), ptr(dW), ptr(db), ptr(dh_src), ld_dh_src, ptr(scratch),
                                   scratch_bytes, stream_ptr(stream)))
+
+
+def gat_fwd(blk, layer, model, h_src, ld_src, W, a_l, a_r, b, out, ld_out, stream=None):
+    _check(lib().buffalo_gat_fwd(ref(blk), layer, ref(model), ptr(h_src), ld_src, ptr(W), ptr(a_l), ptr(a_r), ptr(b),
+                                 ptr(out), ld_out, ptr(blk.agg_saved), blk.agg_saved_bytes, stream_ptr(stream)))
+
+
+def gat_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, h_dst, ld_hdst, W, a_l, a_r, dW, db, da_l, da_r,
+            dh_src, ld_dh_src, scratch, scratch_bytes, stream=None):
+    _check(lib().buffalo_gat_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh, ptr(h_src), ld_src, ptr(h_dst),
+                                 ld_hdst, ptr(blk.agg_saved), blk.agg_saved_bytes, ptr(W), ptr(a_l), ptr(a_r),
+                                 ptr(dW), ptr(db), ptr(da_l), ptr(da_r), ptr(dh_src), ld_dh_src, ptr(scratch),
+                                 scratch_bytes, stream_ptr(stream)))
 
 
 def sgd_step(param, grad, lr, stream=None):

@@ -92,6 +92,7 @@ __global__ void k_fill_i32(int32_t* a, int64_t n, int32_t v) {
 static int64_t bwd_scratch_for(const buffalo_model* m, int64_t n_dst, int64_t n_src, int64_t e, int l) {
   if (m->aggregator == BUFFALO_AGG_POOL) return pool_bwd_scratch_bytes(n_dst, n_src, m->dim[l - 1], m->dim[l]);
   if (m->aggregator == BUFFALO_AGG_LSTM) return lstm_bwd_scratch_bytes(n_dst, e, l, m->dim[l - 1], m->dim[l]);
+  if (m->aggregator == BUFFALO_AGG_GAT) return gat_bwd_scratch_bytes(n_src, n_dst, e, m->dim[l - 1], m->dim[l]);
   if (m->gemm_mode == BUFFALO_GEMM_BF16)
     return tc_bwd_scratch_bytes(n_dst, n_src, e, l, m->dim[l - 1], m->dim[l], l == m->num_layers);
   return bwd_scratch_bytes(n_dst, n_src, l, m->dim[l - 1], m->dim[l]);
@@ -108,7 +109,8 @@ static int64_t dh_slot_bytes(const buffalo_model* m, int64_t n, int l) {
 static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_model* m,
                       int64_t* lo, int64_t* hi) {
   const int64_t s = m->gemm_mode == BUFFALO_GEMM_BF16 ? 2 : 4;
-  const bool pool = m->aggregator == BUFFALO_AGG_POOL;    // R28: block 1 keeps a transpose too
+  const bool pool = m->aggregator == BUFFALO_AGG_POOL || m->aggregator == BUFFALO_AGG_GAT;  // R28/R30: block 1
+                                                                                              // keeps a transpose too
   int64_t blocks = 0, build = 0, acts = 0, bwd = 0;
   for (int l = 1; l <= L; ++l) {
     const int64_t nl = n[l], nm = n[l - 1], el = e[l - 1];
@@ -118,13 +120,15 @@ static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_m
     build = std::max(build, build_frame_bytes(nl, el, l, false, pool));
   }
   for (int l = 1; l <= L; ++l) {
-    acts += R(n[l] * pitch_of(m->dim[l - 1]) * s);
+    if (m->aggregator != BUFFALO_AGG_GAT) acts += R(n[l] * pitch_of(m->dim[l - 1]) * s);   // saved h_agg
     if (l < L) acts += R(n[l] * pitch_of(m->dim[l]) * s);
   }
+  if (m->aggregator == BUFFALO_AGG_GAT)
+    for (int l = 1; l <= L; ++l) acts += gat_saved_bytes(n[l - 1], n[l], e[l - 1], m->dim[l]);
   acts += R(n[L] * pitch_of(m->dim[L]) * 4);
   if (m->aggregator == BUFFALO_AGG_LSTM)
     for (int l = 1; l <= L; ++l) acts += R(lstm_saved_bytes(n[l], e[l - 1], m->dim[l - 1]));
-  if (pool)
+  if (m->aggregator == BUFFALO_AGG_POOL)
     for (int l = 1; l <= L; ++l)   // P [n_{l-1}] and argmax [n_l] rows of width pitch(d_{l-1})
       acts += R(n[l - 1] * pitch_of(m->dim[l - 1]) * 4) + R(n[l] * pitch_of(m->dim[l - 1]) * 4);
   for (int l = L; l >= 1; --l) {
@@ -155,12 +159,12 @@ static buffalo_status validate_model(const buffalo_model* m) {
         set_error("model: the bf16 tensor-core path supports dim[l] <= 256 for l >= 1");
         return BUFFALO_ERR_UNSUPPORTED;
       }
-  if (m->aggregator != BUFFALO_AGG_MEAN && m->aggregator != BUFFALO_AGG_POOL && m->aggregator != BUFFALO_AGG_LSTM) {
+  if (m->aggregator < BUFFALO_AGG_MEAN || m->aggregator > BUFFALO_AGG_GAT) {
     set_error("model: unknown aggregator %d", m->aggregator);
     return BUFFALO_ERR_INVALID_ARG;
   }
   if (m->aggregator != BUFFALO_AGG_MEAN && m->gemm_mode != BUFFALO_GEMM_FFMA) {
-    set_error("model: the pool and LSTM aggregators are built for gemm_mode FFMA (fp32) only");
+    set_error("model: the pool, LSTM and GAT models are built for gemm_mode FFMA (fp32) only");
     return BUFFALO_ERR_UNSUPPORTED;
   }
   if (m->feat_pitch < round_up(m->dim[0], 8) || m->feat_pitch % 8) {
@@ -289,7 +293,7 @@ int64_t buffalo_launch_count(void) { return g_launches.load(); }
 
 buffalo_status buffalo_profile_begin(const char* family, void* counters, int64_t max_launches, void* stream) {
   const std::string fam = family ? family : "";
-  if (!family || (fam != "gather" && fam != "pool_max" && fam != "lstm_gates") || !counters ||
+  if (!family || (fam != "gather" && fam != "pool_max" && fam != "lstm_gates" && fam != "gat_attn") || !counters ||
       max_launches <= 0) {
     set_error("profile_begin: unknown kernel family or no counter buffer");
     return BUFFALO_ERR_INVALID_ARG;
@@ -623,7 +627,7 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
     }
     buffalo_status st = build_layer(g, dst, nd, sp->fanout[l - 1], (uint32_t)(L - l + 1), sp->seed, l,
                                     false, A, b, s, sizes_h ? known : nullptr,
-                                    m->aggregator == BUFFALO_AGG_POOL);
+                                    m->aggregator == BUFFALO_AGG_POOL || m->aggregator == BUFFALO_AGG_GAT);
     if (st == BUFFALO_ERR_CAPACITY || A.overflow) {
       if (required_bytes_h) *required_bytes_h = A.need;
       set_error("build_blocks: arena of %lld bytes too small (need >= %lld)", (long long)A.cap,
@@ -643,7 +647,7 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
   for (int l = 1; l <= L; ++l) {
     buffalo_block* b = &out->layer[l - 1];
     b->ld_agg = pitch_of(m->dim[l - 1]);
-    b->agg = A.take(b->n_dst * b->ld_agg * sa);
+    b->agg = m->aggregator == BUFFALO_AGG_GAT ? nullptr : A.take(b->n_dst * b->ld_agg * sa);
     b->ld_out = pitch_of(m->dim[l]);
     b->out = A.take(b->n_dst * b->ld_out * (l < L ? sa : 4));
   }
@@ -654,11 +658,17 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
       b->pool_P = (float*)A.take(b->n_src * b->ld_pool * 4);
       b->pool_arg = (int32_t*)A.take(b->n_dst * b->ld_pool * 4);
     }
+  if (m->aggregator == BUFFALO_AGG_GAT)
+    for (int l = 1; l <= L; ++l) {
+      buffalo_block* b = &out->layer[l - 1];
+      b->agg_saved_bytes = gat_saved_bytes(b->n_src, b->n_dst, b->n_edges, m->dim[l]);
+      b->agg_saved = A.take(b->agg_saved_bytes);
+    }
   if (m->aggregator == BUFFALO_AGG_LSTM)
     for (int l = 1; l <= L; ++l) {
       buffalo_block* b = &out->layer[l - 1];
-      b->lstm_saved_bytes = R(lstm_saved_bytes(b->n_dst, b->n_edges, m->dim[l - 1]));
-      b->lstm_saved = A.take(b->lstm_saved_bytes);
+      b->agg_saved_bytes = R(lstm_saved_bytes(b->n_dst, b->n_edges, m->dim[l - 1]));
+      b->agg_saved = A.take(b->agg_saved_bytes);
     }
   // backward region: ping-pong dH buffers at the two ends, scratch in between
   int64_t B = 0;
@@ -1030,6 +1040,94 @@ buffalo_status buffalo_lstm_bwd(const buffalo_block* blk, int32_t layer, const b
   a.ld_dh_src = ld_dh_src;
   a.scratch = scratch;
   return lstm_bwd_ffma(a, (cudaStream_t)stream);
+}
+
+buffalo_status buffalo_gat_fwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m, const void* h_src,
+                               int64_t ld_src, const float* W, const float* a_l, const float* a_r, const float* b,
+                               void* out, int64_t ld_out, void* gat_saved, size_t gat_saved_bytes, void* stream) {
+  BF_CHECK(require_sm100());
+  BF_CHECK(validate_model(m));
+  if (m->aggregator != BUFFALO_AGG_GAT) {
+    set_error("gat_fwd: model.aggregator is not BUFFALO_AGG_GAT");
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
+  if (!blk || layer < 1 || layer > m->num_layers || !h_src || !W || !a_l || !a_r || !b || !out || !gat_saved ||
+      !blk->cls_perm) {
+    set_error("gat_fwd: null argument or bad layer");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  GatArgs a{};
+  a.blk = blk;
+  a.layer1 = layer == 1;
+  a.in_bf16 = a.layer1 && m->feat_dtype == BUFFALO_BF16;
+  a.last = layer == m->num_layers;
+  a.d_in = m->dim[layer - 1];
+  a.d_out = m->dim[layer];
+  a.h_src = h_src;
+  a.ld_src = a.layer1 ? m->feat_pitch : ld_src;
+  if ((int64_t)gat_saved_bytes < buffalo::gat_saved_bytes(blk->n_src, blk->n_dst, blk->n_edges, a.d_out) ||
+      ld_out < pitch_of(a.d_out) || ld_out % 8 || a.ld_src < pitch_of(a.d_in) || a.ld_src % 8) {
+    set_error("gat_fwd: saved region too small or bad leading dimensions");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  a.W = W;
+  a.a_l = a_l;
+  a.a_r = a_r;
+  a.b = b;
+  a.out = (float*)out;
+  a.ld_out = ld_out;
+  a.saved = gat_saved;
+  return gat_fwd_ffma(a, (cudaStream_t)stream);
+}
+
+buffalo_status buffalo_gat_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m, float* dh_dst,
+                               int64_t ld_dh, const void* h_src, int64_t ld_src, const void* h_dst, int64_t ld_hdst,
+                               void* gat_saved, size_t gat_saved_bytes, const float* W, const float* a_l,
+                               const float* a_r, float* dW_accum, float* db_accum, float* da_l_accum,
+                               float* da_r_accum, float* dh_src, int64_t ld_dh_src, void* scratch,
+                               size_t scratch_bytes, void* stream) {
+  BF_CHECK(require_sm100());
+  BF_CHECK(validate_model(m));
+  if (m->aggregator != BUFFALO_AGG_GAT) {
+    set_error("gat_bwd: model.aggregator is not BUFFALO_AGG_GAT");
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
+  if (!blk || layer < 1 || layer > m->num_layers || !dh_dst || !h_src || !gat_saved || !W || !a_l || !a_r ||
+      !dW_accum || !db_accum || !da_l_accum || !da_r_accum || !scratch || (layer < m->num_layers && !h_dst) ||
+      !blk->t_row_ptr || (dh_src && layer == 1)) {
+    set_error("gat_bwd: null argument, bad layer or no transposed block");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  GatArgs a{};
+  a.blk = blk;
+  a.layer1 = layer == 1;
+  a.in_bf16 = a.layer1 && m->feat_dtype == BUFFALO_BF16;
+  a.last = layer == m->num_layers;
+  a.d_in = m->dim[layer - 1];
+  a.d_out = m->dim[layer];
+  a.h_src = h_src;
+  a.ld_src = a.layer1 ? m->feat_pitch : ld_src;
+  if ((int64_t)gat_saved_bytes < buffalo::gat_saved_bytes(blk->n_src, blk->n_dst, blk->n_edges, a.d_out) ||
+      (int64_t)scratch_bytes < gat_bwd_scratch_bytes(blk->n_src, blk->n_dst, blk->n_edges, a.d_in, a.d_out)) {
+    set_error("gat_bwd: saved region or scratch too small");
+    return BUFFALO_ERR_CAPACITY;
+  }
+  a.dh = dh_dst;
+  a.ld_dh = ld_dh;
+  a.h_dst = (const float*)h_dst;
+  a.ld_hdst = ld_hdst;
+  a.saved = gat_saved;
+  a.W = W;
+  a.a_l = a_l;
+  a.a_r = a_r;
+  a.dW = dW_accum;
+  a.db = db_accum;
+  a.da_l = da_l_accum;
+  a.da_r = da_r_accum;
+  a.dh_src = dh_src;
+  a.ld_dh_src = ld_dh_src;
+  a.scratch = scratch;
+  return gat_bwd_ffma(a, (cudaStream_t)stream);
 }
 
 buffalo_status buffalo_softmax_ce(const float* logits, int64_t ld, int64_t n, int32_t classes,

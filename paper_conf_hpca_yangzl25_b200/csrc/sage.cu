@@ -1179,4 +1179,326 @@ buffalo_status lstm_bwd_ffma(const LstmArgs& a, cudaStream_t s) {
   return a.in_bf16 ? lstm_bwd_t<__nv_bfloat16>(a, s) : lstm_bwd_t<float>(a, s);
 }
 
+// ================================================================== GAT (R30)
+// One attention head per layer.  Z = H W^T over the block's src rows (SIMT GEMM), scores
+// el[j] = a_l . Z[j], er[i] = a_r . Z[i]; per dst row (degree-class order) a warp takes the
+// max and the sum of exp over its edges in a fixed lane/shuffle order, stores alpha per edge,
+// then sums alpha Z[col] over the edges in CSR order (lanes over 4-column chunks).
+__device__ __forceinline__ float leaky(float x) { return x > 0.f ? x : 0.2f * x; }
+
+__device__ __forceinline__ float warp_dot(const float* __restrict__ a, const float* __restrict__ z, int d) {
+  float s = 0.f;
+  for (int k = threadIdx.x & 31; k < d; k += 32) s = fmaf(a[k], z[k], s);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  return s;
+}
+
+__global__ void __launch_bounds__(256) k_gat_scores(const float* __restrict__ Z, int64_t ldz, int64_t n_src,
+                                                    int64_t n_dst, int d, const float* __restrict__ al,
+                                                    const float* __restrict__ ar, float* __restrict__ el,
+                                                    float* __restrict__ er) {
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t j = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; j < n_src; j += warps) {
+    const float l = warp_dot(al, Z + j * ldz, d);
+    const float r = j < n_dst ? warp_dot(ar, Z + j * ldz, d) : 0.f;
+    if ((threadIdx.x & 31) == 0) {
+      el[j] = l;
+      if (j < n_dst) er[j] = r;
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_gat_attn(const int32_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                                  const int32_t* __restrict__ perm, int64_t n,
+                                                  const float* __restrict__ Z, int64_t ldz, int d,
+                                                  const float* __restrict__ el, const float* __restrict__ er,
+                                                  const float* __restrict__ b, int elu, float* __restrict__ alpha,
+                                                  float* __restrict__ out, int64_t ldo) {
+  const int lane = threadIdx.x & 31;
+  const int nch = (int)(pitch_of(d) / 4);
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < n; w += warps) {
+    const int64_t i = perm[w];
+    const int32_t e0 = rp[i], e1 = rp[i + 1];
+    const float eri = er[i];
+    float m = -INFINITY;
+    for (int32_t e = e0 + lane; e < e1; e += 32) m = fmaxf(m, leaky(el[col[e]] + eri));
+#pragma unroll
+    for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    float sum = 0.f;
+    for (int32_t e = e0 + lane; e < e1; e += 32) sum += expf(leaky(el[col[e]] + eri) - m);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+    const float inv = 1.f / sum;
+    for (int32_t e = e0 + lane; e < e1; e += 32) alpha[e] = expf(leaky(el[col[e]] + eri) - m) * inv;
+    __syncwarp();
+    for (int c = lane; c < nch; c += 32) {
+      float acc[4] = {0.f, 0.f, 0.f, 0.f};
+      for (int32_t e = e0; e < e1; ++e) {
+        const float a = alpha[e];
+        float v[4];
+        VecIO<float, 4>::load(Z + (int64_t)col[e] * ldz + c * 4, v);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) acc[k] = fmaf(a, v[k], acc[k]);
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const int kk = c * 4 + k;
+        float x = kk < d ? acc[k] + b[kk] : 0.f;
+        if (elu && x <= 0.f) x = expm1f(x);
+        acc[k] = x;
+      }
+      VecIO<float, 4>::store(out + i * ldo + c * 4, acc);
+    }
+  }
+}
+
+// dOut = dH * ELU'(out), ELU'(out) = 1 (H > 0) or H + 1 (H = expm1(out) <= 0)
+__global__ void k_gat_elu_bwd(float* __restrict__ dh, int64_t ldd, const float* __restrict__ h, int64_t ldh,
+                              int64_t n, int d) {
+  const int64_t total = n * d;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total; x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = x / d;
+    const int k = (int)(x - i * d);
+    const float hv = h[i * ldh + k];
+    if (!(hv > 0.f)) dh[i * ldd + k] *= hv + 1.f;
+  }
+}
+
+// db += column sums of dOut: CTA per 32 columns, 8 warps over rows, fixed-order combine
+__global__ void __launch_bounds__(256) k_colsum(const float* __restrict__ x, int64_t ldx, int64_t n, int d,
+                                                float* __restrict__ out) {
+  __shared__ float sh[8][33];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + lane;
+  float s = 0.f;
+  if (c < d)
+    for (int64_t i = warp; i < n; i += 8) s += x[i * ldx + c];
+  sh[warp][lane] = s;
+  __syncthreads();
+  if (warp == 0 && c < d) {
+    float t = 0.f;
+    for (int w = 0; w < 8; ++w) t += sh[w][lane];
+    out[c] += t;
+  }
+}
+
+// per dst row: dalpha_e = dOut_i . Z[col_e] (kept in ds), then ds_e = alpha_e (dalpha_e - sum
+// alpha dalpha) LeakyReLU'(s_e), d_er[i] = sum_e ds_e
+__global__ void __launch_bounds__(256) k_gat_row_bwd(const int32_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                                     int64_t n, const float* __restrict__ Z, int64_t ldz, int d,
+                                                     const float* __restrict__ dO, int64_t ldo,
+                                                     const float* __restrict__ el, const float* __restrict__ er,
+                                                     const float* __restrict__ alpha, float* __restrict__ ds,
+                                                     float* __restrict__ d_er) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n; i += warps) {
+    const int32_t e0 = rp[i], e1 = rp[i + 1];
+    float c = 0.f;
+    for (int32_t e = e0; e < e1; ++e) {
+      const float da = warp_dot(dO + i * ldo, Z + (int64_t)col[e] * ldz, d);
+      if (lane == 0) ds[e] = da;
+      c = fmaf(alpha[e], da, c);
+    }
+    __syncwarp();
+    const float eri = er[i];
+    float s = 0.f;
+    for (int32_t e = e0 + lane; e < e1; e += 32) {
+      const float x = el[col[e]] + eri;
+      const float g = alpha[e] * (ds[e] - c) * (x > 0.f ? 1.f : 0.2f);
+      ds[e] = g;
+      s += g;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) d_er[i] = s;
+  }
+}
+
+// per src row j (transposed block, ascending dst i): dZ[j] = sum alpha_e dOut_i + d_el[j] a_l
+// (+ d_er[j] a_r for j < n_dst), d_el[j] = sum ds_e; edge e = (i, j) found by a ballot.
+__global__ void __launch_bounds__(256) k_gat_src_bwd(const int32_t* __restrict__ trp, const int32_t* __restrict__ tcol,
+                                                     const int32_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                                     int64_t n_src, int64_t n_dst, const float* __restrict__ alpha,
+                                                     const float* __restrict__ ds, const float* __restrict__ dO,
+                                                     int64_t ldo, int d, const float* __restrict__ al,
+                                                     const float* __restrict__ ar, const float* __restrict__ d_er,
+                                                     float* __restrict__ d_el, float* __restrict__ dZ, int64_t ldz) {
+  const int lane = threadIdx.x & 31;
+  const int nch = (int)(pitch_of(d) / 4);
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t j = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; j < n_src; j += warps) {
+    const int32_t t0 = trp[j], t1 = trp[j + 1];
+    float del = 0.f;
+    for (int c0 = 0; c0 < nch; c0 += 32) {
+      const int c = c0 + lane;
+      float acc[4] = {0.f, 0.f, 0.f, 0.f};
+      float dsum = 0.f;
+      for (int32_t t = t0; t < t1; ++t) {
+        const int32_t i = tcol[t];
+        int32_t e = -1;
+        for (int32_t e0 = rp[i]; e0 < rp[i + 1] && e < 0; e0 += 32) {
+          const bool hit = e0 + lane < rp[i + 1] && col[e0 + lane] == (int32_t)j;
+          const unsigned m = __ballot_sync(0xffffffffu, hit);
+          if (m) e = e0 + __ffs(m) - 1;
+        }
+        const float a = alpha[e];
+        dsum += ds[e];
+        if (c < nch) {
+          float v[4];
+          VecIO<float, 4>::load(dO + (int64_t)i * ldo + c * 4, v);
+#pragma unroll
+          for (int k = 0; k < 4; ++k) acc[k] = fmaf(a, v[k], acc[k]);
+        }
+      }
+      del = dsum;
+      if (c < nch) {
+        const float der = j < n_dst ? d_er[j] : 0.f;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int kk = c * 4 + k;
+          acc[k] = kk < d ? acc[k] + del * al[kk] + der * ar[kk] : 0.f;
+        }
+        VecIO<float, 4>::store(dZ + j * ldz + c * 4, acc);
+      }
+    }
+    if (lane == 0) d_el[j] = del;
+  }
+}
+
+int gemm_splits(int64_t n_rows, int rows_out, int K) {
+  const int64_t tiles = ceil_div(rows_out, 64) * ceil_div(K, 64);
+  const int64_t a = ceil_div(296, tiles), b = ceil_div(n_rows > 0 ? n_rows : 1, 512);
+  const int64_t sp = a < b ? a : b;
+  return (int)(sp < 1 ? 1 : sp);
+}
+
+int64_t gat_saved_bytes(int64_t n_src, int64_t n_dst, int64_t e, int d_out) {
+  return R(n_src * pitch_of(d_out) * 4) + R(4 * n_src) + R(4 * n_dst) + R(4 * e);
+}
+
+int64_t gat_bwd_scratch_bytes(int64_t n_src, int64_t n_dst, int64_t e, int d_in, int d_out) {
+  const int S4 = gemm_splits(n_src, d_out, d_in), Sl = gemm_splits(n_src, 1, d_out), Sr = gemm_splits(n_dst, 1, d_out);
+  return R(n_src * pitch_of(d_out) * 4) + R(4 * e) + R(4 * n_src) + R(4 * n_dst) +
+         R((int64_t)S4 * d_out * d_in * 4) + R((int64_t)S4 * pitch_of(d_out) * 4) +
+         R((int64_t)Sl * d_out * 4) + R((int64_t)Sl * 4) + R((int64_t)Sr * d_out * 4) + R((int64_t)Sr * 4);
+}
+
+struct GatSaved {
+  float *Z, *el, *er, *alpha;
+};
+static GatSaved gat_saved_view(void* base, int64_t n_src, int64_t n_dst, int64_t e, int d_out) {
+  char* q = (char*)base;
+  GatSaved v;
+  v.Z = (float*)q; q += R(n_src * pitch_of(d_out) * 4);
+  v.el = (float*)q; q += R(4 * n_src);
+  v.er = (float*)q; q += R(4 * n_dst);
+  v.alpha = (float*)q;
+  return v;
+}
+
+template <class TI>
+static buffalo_status gat_fwd_t(const GatArgs& a, cudaStream_t st) {
+  const buffalo_block* blk = a.blk;
+  const int64_t ns = blk->n_src, nd = blk->n_dst, e = blk->n_edges;
+  const int dl = a.d_out;
+  const int64_t ldz = pitch_of(dl);
+  GatSaved v = gat_saved_view(a.saved, ns, nd, e, dl);
+  if (ns > 0) {
+    dim3 grid((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(ldz, GB_N));
+    k_gemm2<TI, float, float, true><<<grid, 256, 0, st>>>(ns, dl, (int)ldz, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
+                                                         a.layer1 ? blk->src_global : nullptr, ns, nullptr, 0, a.W,
+                                                         a.d_in, nullptr, 0, nullptr, 0, v.Z, ldz);
+    BF_LAUNCHED("k_gemm2");
+    k_gat_scores<<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(v.Z, ldz, ns, nd, dl, a.a_l, a.a_r, v.el, v.er);
+    BF_LAUNCHED("k_gat_scores");
+  }
+  if (nd <= 0) return BUFFALO_OK;
+  const ProfSlot ps = prof_begin_launch("gat_attn", st);
+  k_gat_attn<<<grid_for(nd * 32, 256, 16), 256, 0, st>>>(blk->row_ptr, blk->col_local, blk->cls_perm, nd, v.Z, ldz, dl,
+                                                         v.el, v.er, a.b, !a.last, v.alpha, a.out, a.ld_out);
+  BF_LAUNCHED("k_gat_attn");
+  // algorithmic bytes: per row perm + row_ptr pair + er + output row; per edge the index (read
+  // by the three passes: 12 B), el (12 B), alpha write + read (8 B) and the Z row
+  prof_end_launch(ps, st, (double)nd * (16.0 + 4.0 * ldz) + (double)e * (32.0 + 4.0 * ldz), 0.0);
+  return BUFFALO_OK;
+}
+
+buffalo_status gat_fwd_ffma(const GatArgs& a, cudaStream_t s) {
+  return a.in_bf16 ? gat_fwd_t<__nv_bfloat16>(a, s) : gat_fwd_t<float>(a, s);
+}
+
+template <class TI>
+static buffalo_status gat_bwd_t(const GatArgs& a, cudaStream_t st) {
+  const buffalo_block* blk = a.blk;
+  const int64_t ns = blk->n_src, nd = blk->n_dst, e = blk->n_edges;
+  const int dl = a.d_out, d_in = a.d_in;
+  const int64_t ldz = pitch_of(dl);
+  GatSaved v = gat_saved_view(a.saved, ns, nd, e, dl);
+  const int S4 = gemm_splits(ns, dl, d_in), Sl = gemm_splits(ns, 1, dl), Sr = gemm_splits(nd, 1, dl);
+  char* q = (char*)a.scratch;
+  float* dZ = (float*)q; q += R(ns * ldz * 4);
+  float* ds = (float*)q; q += R(4 * e);
+  float* d_el = (float*)q; q += R(4 * ns);
+  float* d_er = (float*)q; q += R(4 * nd);
+  float* dw_part = (float*)q; q += R((int64_t)S4 * dl * d_in * 4);
+  float* db_part = (float*)q; q += R((int64_t)S4 * pitch_of(dl) * 4);
+  float* dal_part = (float*)q; q += R((int64_t)Sl * dl * 4);
+  float* dal_b = (float*)q; q += R((int64_t)Sl * 4);
+  float* dar_part = (float*)q; q += R((int64_t)Sr * dl * 4);
+  float* dar_b = (float*)q;
+  if (!a.last && nd > 0) {
+    k_gat_elu_bwd<<<grid_for(nd * dl, 256), 256, 0, st>>>(a.dh, a.ld_dh, a.h_dst, a.ld_hdst, nd, dl);
+    BF_LAUNCHED("k_gat_elu_bwd");
+  }
+  if (nd > 0) {
+    k_colsum<<<(unsigned)ceil_div(dl, 32), 256, 0, st>>>(a.dh, a.ld_dh, nd, dl, a.db);
+    BF_LAUNCHED("k_colsum");
+    k_gat_row_bwd<<<grid_for(nd * 32, 256, 16), 256, 0, st>>>(blk->row_ptr, blk->col_local, nd, v.Z, ldz, dl, a.dh,
+                                                              a.ld_dh, v.el, v.er, v.alpha, ds, d_er);
+    BF_LAUNCHED("k_gat_row_bwd");
+  }
+  if (ns <= 0) return BUFFALO_OK;
+  k_gat_src_bwd<<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(blk->t_row_ptr, blk->t_col, blk->row_ptr, blk->col_local,
+                                                            ns, nd, v.alpha, ds, a.dh, a.ld_dh, dl, a.a_l, a.a_r,
+                                                            d_er, d_el, dZ, ldz);
+  BF_LAUNCHED("k_gat_src_bwd");
+  // da_l = d_el^T Z, da_r = d_er^T Z[:n_dst], dW = dZ^T H (deterministic split reductions)
+  dim3 gl((unsigned)ceil_div(dl, 64), 1, (unsigned)Sl);
+  k_dw_partial<float, float><<<gl, 256, 0, st>>>(ns, 1, dl, dl, d_el, 1, v.Z, ldz, nullptr, nullptr, 0,
+                                                 ceil_div(ns, Sl), dal_part, dal_b);
+  BF_LAUNCHED("k_dw_partial");
+  k_reduce_partials<<<1, 256, 0, st>>>(dal_part, Sl, dl, a.da_l);
+  BF_LAUNCHED("k_reduce_partials");
+  if (nd > 0) {
+    dim3 gr((unsigned)ceil_div(dl, 64), 1, (unsigned)Sr);
+    k_dw_partial<float, float><<<gr, 256, 0, st>>>(nd, 1, dl, dl, d_er, 1, v.Z, ldz, nullptr, nullptr, 0,
+                                                   ceil_div(nd, Sr), dar_part, dar_b);
+    BF_LAUNCHED("k_dw_partial");
+    k_reduce_partials<<<1, 256, 0, st>>>(dar_part, Sr, dl, a.da_r);
+    BF_LAUNCHED("k_reduce_partials");
+  }
+  dim3 gw((unsigned)ceil_div(d_in, 64), (unsigned)ceil_div(dl, 64), (unsigned)S4);
+  k_dw_partial<TI, float><<<gw, 256, 0, st>>>(ns, dl, d_in, d_in, dZ, ldz, (const TI*)a.h_src, a.ld_src,
+                                              a.layer1 ? blk->src_global : nullptr, nullptr, 0, ceil_div(ns, S4),
+                                              dw_part, db_part);
+  BF_LAUNCHED("k_dw_partial");
+  k_reduce_partials<<<grid_for((int64_t)dl * d_in, 256), 256, 0, st>>>(dw_part, S4, (int64_t)dl * d_in, a.dW);
+  BF_LAUNCHED("k_reduce_partials");
+  if (a.dh_src) {   // dH_{l-1} = dZ W
+    const int64_t dpi = pitch_of(d_in);
+    dim3 gg((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dpi, GB_N));
+    k_gemm2<float, float, float><<<gg, 256, 0, st>>>(ns, d_in, (int)dpi, dl, 0, dZ, ldz, nullptr, ns, nullptr, 0, a.W,
+                                                    d_in, nullptr, 0, nullptr, 0, a.dh_src, a.ld_dh_src);
+    BF_LAUNCHED("k_gemm2");
+  }
+  return BUFFALO_OK;
+}
+
+buffalo_status gat_bwd_ffma(const GatArgs& a, cudaStream_t s) {
+  return a.in_bf16 ? gat_bwd_t<__nv_bfloat16>(a, s) : gat_bwd_t<float>(a, s);
+}
+
 }  // namespace buffalo

@@ -79,6 +79,27 @@ int64_t lstm_bwd_scratch_bytes(int64_t n_dst, int64_t e, int layer, int d_in, in
 buffalo_status lstm_fwd_ffma(const LstmArgs& a, cudaStream_t s);
 buffalo_status lstm_bwd_ffma(const LstmArgs& a, cudaStream_t s);
 
+// GAT (R30): one head per layer, FFMA path, fp32 activations.
+struct GatArgs {
+  const buffalo_block* blk;
+  bool layer1, in_bf16, last;
+  int d_in, d_out;
+  const void* h_src; int64_t ld_src;
+  const float* W; const float* a_l; const float* a_r; const float* b;
+  float* out; int64_t ld_out;
+  void* saved;
+  float* dh; int64_t ld_dh;
+  const float* h_dst; int64_t ld_hdst;
+  float* dW; float* db; float* da_l; float* da_r;
+  float* dh_src; int64_t ld_dh_src;
+  void* scratch;
+};
+int gemm_splits(int64_t n_rows, int rows_out, int K);
+int64_t gat_saved_bytes(int64_t n_src, int64_t n_dst, int64_t e, int d_out);
+int64_t gat_bwd_scratch_bytes(int64_t n_src, int64_t n_dst, int64_t e, int d_in, int d_out);
+buffalo_status gat_fwd_ffma(const GatArgs& a, cudaStream_t s);
+buffalo_status gat_bwd_ffma(const GatArgs& a, cudaStream_t s);
+
 int dw_splits(int64_t n_l, int d_out, int d_in);
 int64_t bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int layer, int d_in, int d_out);
 

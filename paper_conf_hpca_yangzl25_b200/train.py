@@ -47,12 +47,13 @@ class DeviceGraph:
 class SageParams:
     """fp32 master weights/biases (Xavier init from synth), flat gradient buffer, packed copies."""
 
-    def __init__(self, model, Ws, bs, device="cuda", Wps=None, bps=None, lstm=None):
+    def __init__(self, model, Ws, bs, device="cuda", Wps=None, bps=None, lstm=None, gat=None):
         self.model = model
         self.L = model.num_layers
         Wps, bps = list(Wps or []), list(bps or [])
         Wih, Whh, bl = [list(x) for x in lstm] if lstm else ([], [], [])
-        extra = Wih + Whh + bl
+        als, ars = [list(x) for x in gat] if gat else ([], [])
+        extra = Wih + Whh + bl + als + ars
         sizes = [w.size for w in Ws] + [b.size for b in bs] + [w.size for w in Wps] + [b.size for b in bps] + \
             [w.size for w in extra]
         self.flat = torch.zeros(sum(sizes), dtype=torch.float32, device=device)
@@ -89,11 +90,23 @@ class SageParams:
                 self.dlstm[k].append(self.grad[off:off + w.size].view(w.shape))
                 self.lstm[k][-1].copy_(torch.as_tensor(w))
                 off += w.size
-        self.packed = [torch.empty(B.packed_weight_bytes(model, l), dtype=torch.uint8, device=device)
+        # GAT attention vectors (R30): a_l, a_r [d_l] per layer
+        self.al, self.ar, self.dal, self.dar = [], [], [], []
+        for dst, gdst, group in ((self.al, self.dal, als), (self.ar, self.dar, ars)):
+            for w in group:
+                dst.append(self.flat[off:off + w.size])
+                gdst.append(self.grad[off:off + w.size])
+                dst[-1].copy_(torch.as_tensor(w))
+                off += w.size
+        self.is_gat = model.aggregator == B.AGG_GAT      # GAT's W_l is [d_l, d_{l-1}]: no packed Update copy
+        self.packed = [None if self.is_gat else
+                       torch.empty(B.packed_weight_bytes(model, l), dtype=torch.uint8, device=device)
                        for l in range(1, self.L + 1)]
         self.repack()
 
     def repack(self):
+        if self.is_gat:
+            return
         for l in range(1, self.L + 1):
             B.pack_weights(self.model, l, self.W[l - 1], self.packed[l - 1])
 
@@ -102,7 +115,7 @@ class Trainer:
     def __init__(self, graph, feats, labels, seeds, dims, fanout, F, Ws, bs, feat_dtype=B.FP32,
                  gemm_mode=B.GEMM_FFMA, mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096,
                  base_seed=3, rank=0, world=1, process_group=None, device="cuda", aggregator=B.AGG_MEAN,
-                 Wps=None, bps=None, lstm=None):
+                 Wps=None, bps=None, lstm=None, gat=None):
         self.graph = graph if isinstance(graph, DeviceGraph) else DeviceGraph(*graph, device=device)
         self.feats = feats
         self.labels = labels
@@ -117,11 +130,14 @@ class Trainer:
         self.is_lstm = aggregator == B.AGG_LSTM
         if self.pool and Wps is None:
             raise ValueError("the pool aggregator needs its weights (Wps, bps)")
+        self.is_gat = aggregator == B.AGG_GAT
+        if self.is_gat and gat is None:
+            raise ValueError("GAT needs its attention vectors (a_l, a_r per layer)")
         if self.is_lstm and lstm is None:
             raise ValueError("the LSTM aggregator needs its weights (W_ih, W_hh, b per layer)")
         self.model = B.make_model(dims, feat_dtype, gemm_mode, feats.shape[1], aggregator)
         self.sched = B.make_sched(mem_budget, C_ppm, k_min, k_max, world)
-        self.params = SageParams(self.model, Ws, bs, device, Wps, bps, lstm)
+        self.params = SageParams(self.model, Ws, bs, device, Wps, bps, lstm, gat)
         self.rank, self.world, self.pg = rank, world, process_group
         self.device = device
         # scheduler outputs
@@ -185,7 +201,9 @@ class Trainer:
         h, ld = self.feats, self.feats.shape[1]
         for l in range(1, self.L + 1):
             b = blks.layer[l - 1]
-            if self.is_lstm:
+            if self.is_gat:
+                B.gat_fwd(b, l, m, h, ld, p.W[l - 1], p.al[l - 1], p.ar[l - 1], p.b[l - 1], b.out, b.ld_out)
+            elif self.is_lstm:
                 B.lstm_fwd(b, l, m, h, ld, p.lstm[0][l - 1], p.lstm[1][l - 1], p.lstm[2][l - 1], p.W[l - 1],
                            p.packed[l - 1], p.b[l - 1], b.out, b.ld_out, b.agg, b.ld_agg)
             elif self.pool:
@@ -207,6 +225,11 @@ class Trainer:
             else:
                 h_src, ld_src, dh_src, ld_dh_src, prev_rp = self.feats, self.feats.shape[1], None, 0, None
             h_dst = b.out if l < self.L else None
+            if self.is_gat:
+                B.gat_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, h_dst, b.ld_out, p.W[l - 1], p.al[l - 1],
+                          p.ar[l - 1], p.dW[l - 1], p.db[l - 1], p.dal[l - 1], p.dar[l - 1], dh_src, ld_dh_src,
+                          b.bwd_scratch, b.bwd_scratch_bytes)
+                continue
             if self.is_lstm:
                 B.lstm_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out,
                            p.lstm[0][l - 1], p.lstm[1][l - 1], p.W[l - 1], p.dlstm[0][l - 1], p.dlstm[1][l - 1],

@@ -250,6 +250,33 @@ def lstm_weights(dims, seed=WEIGHT_SEED):
     return Wih, Whh, bl
 
 
+def gat_weights(dims, seed=WEIGHT_SEED, bias_scale=0.0):
+    """GAT weights per layer l = 1..L (one head): W_l float32 [d_l, d_{l-1}] (Xavier-uniform),
+    attention vectors a_l, a_r [d_l] (Xavier-uniform of a [2 d_l] vector as GATConv) and b_l
+    [d_l]; Philox counters c0 = 224 + l (W), 240 + l (a), 248 + l (b)."""
+    Ws, als, ars, bs = [], [], [], []
+    for l in range(1, len(dims)):
+        din, dout = dims[l - 1], dims[l]
+        a = math.sqrt(6.0 / (din + dout))
+        r = np.arange(dout, dtype=np.uint64)[:, None]
+        c = np.arange(din, dtype=np.uint64)[None, :]
+        w = words(seed, 224 + l, r, c >> np.uint64(2), TAG_WEIGHT)
+        sel = np.choose((c & np.uint64(3)).astype(np.int64), w)
+        u = (sel.astype(np.float64) + 0.5) / 4294967296.0
+        Ws.append(((2.0 * u - 1.0) * a).astype(np.float32))
+        aa = math.sqrt(6.0 / (1 + 2 * dout))
+        wa = words(seed, 240 + l, 0, np.arange(2 * dout, dtype=np.uint64), TAG_WEIGHT)[0]
+        ua = ((wa.astype(np.float64) + 0.5) / 4294967296.0 * 2.0 - 1.0) * aa
+        als.append(ua[:dout].astype(np.float32))
+        ars.append(ua[dout:].astype(np.float32))
+        if bias_scale:
+            wb = words(seed, 248 + l, 0, np.arange(dout, dtype=np.uint64), TAG_WEIGHT)[0]
+            bs.append((((wb.astype(np.float64) + 0.5) / 4294967296.0 * 2.0 - 1.0) * bias_scale).astype(np.float32))
+        else:
+            bs.append(np.zeros(dout, dtype=np.float32))
+    return Ws, bs, als, ars
+
+
 # ----------------------------------------------------------------------------- configs
 @dataclass
 class Config:

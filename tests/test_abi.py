@@ -44,7 +44,7 @@ def test_library_is_sm100a_only(blib):
     assert "sm_100a" in out and "sm_90" not in out
 
 
-@pytest.mark.parametrize("gemm,agg", [(0, 0), (1, 0), (0, 1), (0, 2)])
+@pytest.mark.parametrize("gemm,agg", [(0, 0), (1, 0), (0, 1), (0, 2), (0, 3)])
 def test_estimate_mem_equals_oracle(blib, gemm, agg):
     rng = np.random.default_rng(gemm + 7 * agg)
     for _ in range(200):
@@ -55,7 +55,7 @@ def test_estimate_mem_equals_oracle(blib, gemm, agg):
         e = [int(x) for x in rng.integers(0, 3000000, L)]
         m = blib.make_model(dims, gemm_mode=gemm, aggregator=agg)
         assert blib.estimate_mem(n, e, m) == O.mem_model(n, e, dims, O.BF16 if gemm else O.FP32,
-                                                         ("mean", "pool", "lstm")[agg])
+                                                         ("mean", "pool", "lstm", "gat")[agg])
 
 
 def test_cuda_philox_known_answers(tmp_path):
