@@ -373,7 +373,7 @@ BUFFALO_API int64_t buffalo_launch_count(void);
 
 /* Diagnostics (bench roofline): time every launch of one kernel family with CUDA events on the
  * stream it is launched on.  family "gat_attn": k_gat_attn (GAT softmax + weighted neighbour
- * sum; per row 16 B + the output row, per edge 32 B of indices / scores / alpha + the Z row).
+ * sum; per row 16 B + the output row, per edge 12 B of index / score / alpha + the Z row).
  * family "lstm_gates": the LSTM gate GEMM of every step; its
  * "algorithmic bytes" are FLOPs (2 x rows x 4d x (d + d)).  family "pool_max": k_pool_max, the GraphSAGE-pool neighbour max
  * (per row 12 B + the max and argmax rows, per edge the index and the pooled fp32 row).

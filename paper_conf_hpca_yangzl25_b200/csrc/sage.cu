@@ -257,14 +257,23 @@ __global__ void __launch_bounds__(256) k_gemm2(int64_t M, int N, int Np, int K1,
         }
         As[ak + q][ar] = v;
       }
-      const int k = k0 + bk;
       const float* B = first ? B1 : B2;
       const int64_t ldb = first ? ldb1 : ldb2;
+      if (TB) {   // Bt[n][k]: thread = (n = tid / 4, 4 consecutive k), 4 threads per 64-B row run
+        const int tn = tid >> 2, tk = (tid & 3) * 4;
+        const int nn = n0 + tn;
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const int nn = n0 + bn + q;
-        Bs[bk][bn + q] = (k < K && nn < N) ? __ldg(TB ? B + (int64_t)nn * ldb + k : B + (int64_t)k * ldb + nn)
-                                           : 0.f;
+        for (int q = 0; q < 4; ++q) {
+          const int k = k0 + tk + q;
+          Bs[tk + q][tn] = (k < K && nn < N) ? __ldg(B + (int64_t)nn * ldb + k) : 0.f;
+        }
+      } else {
+        const int k = k0 + bk;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const int nn = n0 + bn + q;
+          Bs[bk][bn + q] = (k < K && nn < N) ? __ldg(B + (int64_t)k * ldb + nn) : 0.f;
+        }
       }
     }
     __syncthreads();
@@ -1266,21 +1275,23 @@ __global__ void k_gat_elu_bwd(float* __restrict__ dh, int64_t ldd, const float* 
   }
 }
 
-// db += column sums of dOut: CTA per 32 columns, 8 warps over rows, fixed-order combine
-__global__ void __launch_bounds__(256) k_colsum(const float* __restrict__ x, int64_t ldx, int64_t n, int d,
-                                                float* __restrict__ out) {
+// column sums of dOut, split-K: CTA (32 columns, row split z of rps rows), 8 warps over the
+// rows, fixed-order combine into part[z][c]; k_reduce_partials then adds the splits in order
+__global__ void __launch_bounds__(256) k_colsum_partial(const float* __restrict__ x, int64_t ldx, int64_t n, int d,
+                                                        int64_t rps, float* __restrict__ part) {
   __shared__ float sh[8][33];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + lane;
+  const int64_t r0 = (int64_t)blockIdx.y * rps, r1 = min(n, r0 + rps);
   float s = 0.f;
   if (c < d)
-    for (int64_t i = warp; i < n; i += 8) s += x[i * ldx + c];
+    for (int64_t i = r0 + warp; i < r1; i += 8) s += x[i * ldx + c];
   sh[warp][lane] = s;
   __syncthreads();
   if (warp == 0 && c < d) {
     float t = 0.f;
     for (int w = 0; w < 8; ++w) t += sh[w][lane];
-    out[c] += t;
+    part[(int64_t)blockIdx.y * d + c] = t;
   }
 }
 
@@ -1420,9 +1431,10 @@ static buffalo_status gat_fwd_t(const GatArgs& a, cudaStream_t st) {
   k_gat_attn<<<grid_for(nd * 32, 256, 16), 256, 0, st>>>(blk->row_ptr, blk->col_local, blk->cls_perm, nd, v.Z, ldz, dl,
                                                          v.el, v.er, a.b, !a.last, v.alpha, a.out, a.ld_out);
   BF_LAUNCHED("k_gat_attn");
-  // algorithmic bytes: per row perm + row_ptr pair + er + output row; per edge the index (read
-  // by the three passes: 12 B), el (12 B), alpha write + read (8 B) and the Z row
-  prof_end_launch(ps, st, (double)nd * (16.0 + 4.0 * ldz) + (double)e * (32.0 + 4.0 * ldz), 0.0);
+  // algorithmic bytes (each datum once; the three passes re-read indices and scores from L1/L2):
+  // per row perm + row_ptr pair + er + the output row; per edge the index, el, the alpha
+  // written and the Z row
+  prof_end_launch(ps, st, (double)nd * (16.0 + 4.0 * ldz) + (double)e * (12.0 + 4.0 * ldz), 0.0);
   return BUFFALO_OK;
 }
 
@@ -1454,8 +1466,12 @@ static buffalo_status gat_bwd_t(const GatArgs& a, cudaStream_t st) {
     BF_LAUNCHED("k_gat_elu_bwd");
   }
   if (nd > 0) {
-    k_colsum<<<(unsigned)ceil_div(dl, 32), 256, 0, st>>>(a.dh, a.ld_dh, nd, dl, a.db);
-    BF_LAUNCHED("k_colsum");
+    // db: the da_r partial buffer (Sr x dl floats) holds the column-sum splits first
+    k_colsum_partial<<<dim3((unsigned)ceil_div(dl, 32), (unsigned)Sr), 256, 0, st>>>(a.dh, a.ld_dh, nd, dl,
+                                                                                     ceil_div(nd, Sr), dar_part);
+    BF_LAUNCHED("k_colsum_partial");
+    k_reduce_partials<<<1, 256, 0, st>>>(dar_part, Sr, dl, a.db);
+    BF_LAUNCHED("k_reduce_partials");
     k_gat_row_bwd<<<grid_for(nd * 32, 256, 16), 256, 0, st>>>(blk->row_ptr, blk->col_local, nd, v.Z, ldz, dl, a.dh,
                                                               a.ld_dh, v.el, v.er, v.alpha, ds, d_er);
     BF_LAUNCHED("k_gat_row_bwd");
