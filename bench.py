@@ -38,6 +38,9 @@ WORKLOADS = {
     "arxiv_lstm": ("ogbn-arxiv-shaped power-law graph (169,343 nodes, 1,166,243 undirected edges, 128-d), "
                    "2-layer SAGE-LSTM 128-128-40 (LSTM hidden 128, PAPER.md:351), fanout (10,25), F=25, "
                    "90,941 seeds, budget forcing >= 2 bucket groups"),
+    "papers": ("ogbn-papers100M-shaped power-law graph (111,059,956 nodes, 1,615,685,872 undirected edges, "
+               "128-d), 2-layer SAGE-mean 128-256-172, fanout (10,25), F=25, 1,207,179 seeds, budget forcing >= 8 "
+               "bucket groups"),
     "products": ("ogbn-products-shaped power-law graph (2,449,029 nodes, 61,859,140 edges, 100-d), 3-layer "
                  "SAGE-mean 100-256-256-47, fanout (10,25,30), budget forcing >= 8 bucket groups"),
 }
@@ -72,13 +75,16 @@ def dist_env():
     return rank, world, local
 
 
-def make_inputs_device(cfg):
+def make_inputs_device(cfg, feat_dtype=None):
     """The same inputs as make_inputs, generated on the GPU by synth.device (bit-identical to
-    the numpy recipe; a products-shaped graph takes seconds instead of minutes on one core)."""
+    the numpy recipe; a products-shaped graph takes seconds instead of minutes on one core).
+    feat_dtype: generate the feature table directly in that dtype (k/128 values are exact in
+    bf16; the papers-shaped table is 28 GB in bf16, 57 GB in fp32)."""
     import torch
     from synth import device as SD
     rp, col = SD.random_graph(cfg.N, cfg.pairs, cfg.kind)
-    X = SD.features(cfg.N, cfg.d0, ((cfg.d0 + 31) // 32) * 32)
+    torch.cuda.empty_cache()
+    X = SD.features(cfg.N, cfg.d0, ((cfg.d0 + 31) // 32) * 32, dtype=feat_dtype or torch.float32)
     y = SD.labels(cfg.N, cfg.classes)
     seeds = SD.seed_nodes(cfg.N, cfg.S)
     Ws, bs = xavier_weights(cfg.dims)
@@ -244,7 +250,8 @@ def run_ours(args, cfg):
 
     B.lib()
     t_gen = time.perf_counter()
-    rp, col, X, y, seeds, Ws, bs = make_inputs_device(cfg)
+    big = cfg.N > 50_000_000              # papers / IGB shapes: bf16 table generated directly, no fp32 copy
+    rp, col, X, y, seeds, Ws, bs = make_inputs_device(cfg, torch.bfloat16 if (big and args.gemm == "bf16") else None)
     t_gen = time.perf_counter() - t_gen
     pool = args.aggregator == "pool"
     lstm = args.aggregator == "lstm"
@@ -266,7 +273,7 @@ def run_ours(args, cfg):
         agg_kw = dict(aggregator=B.AGG_GAT, gat=(als, ars))
     feat_dtype = B.BF16 if args.gemm == "bf16" else B.FP32
     feats = X
-    if feat_dtype == B.BF16:
+    if feat_dtype == B.BF16 and feats.dtype != torch.bfloat16:
         feats = feats.to(torch.bfloat16).contiguous()      # k/128 features are exact in bf16
     kmin = max(cfg.k_min, world)
     budget = cfg.mem_budget
@@ -280,7 +287,7 @@ def run_ours(args, cfg):
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, mem_budget=budget,
                  C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg,
                  **agg_kw)
-    if args.config in ("products", "arxiv_lstm"):
+    if args.config in ("products", "papers", "arxiv_lstm"):
         # calibrate M_ctr once so that one GPU needs >= 8 groups (products; 2 for the LSTM
         # workload), then freeze it for every N
         B_full = Trainer(graph, feats, y, seeds, cfg.dims,
@@ -288,7 +295,7 @@ def run_ours(args, cfg):
                          k_min=1, k_max=1, **agg_kw)
         _, _, est1, _ = B_full.schedule(0)
         del B_full
-        tr.sched.mem_budget = int(est1[0]) // (8 if args.config == "products" else 2)
+        tr.sched.mem_budget = int(est1[0]) // (2 if args.config == "arxiv_lstm" else 8)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
 
@@ -395,7 +402,7 @@ def run_ours(args, cfg):
                 "share_of_step": g_ms / total_ms}
     if rank == 0:
         cpu = None
-        if world == 1 and not args.no_cpu_baseline and not (pool or lstm or gat):   # (the pool oracle is loop-plain: tests only)
+        if world == 1 and not args.no_cpu_baseline and not (pool or lstm or gat or big):   # (the pool oracle is loop-plain: tests only)
             rp_h, col_h, X_h, y_h, seeds_h = host_copies(rp, col, X, y, tr.seeds)
             cpu = oracle_sample(cfg, rp_h, col_h, X_h, y_h, seeds_h, Ws, bs, args.cpu_baseline_seconds)
         line = dict(

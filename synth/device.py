@@ -78,13 +78,16 @@ def _gnm_candidates(N, start, count, seed, dev):
     return scale(w[0]), scale(w[1])
 
 
-def undirected_pairs(N, E, kind, seed=GRAPH_SEED, device="cuda"):
-    """The E distinct undirected pairs (u < v) with the smallest first-draw index (int64 [E,2])."""
+def undirected_keys(N, E, kind, seed=GRAPH_SEED, device="cuda"):
+    """The E distinct undirected pairs (u < v) with the smallest first-draw index, as keys
+    u * N + v (int64 [E], in first-draw order).  Memory-lean for billion-edge shapes: the
+    candidates live in one growing buffer (draw order = position), a stable sort marks each
+    key's first draw, and the E earliest first draws are cut by a prefix count."""
     dev = torch.device(device)
     cdf = torch.as_tensor(_powerlaw_cdf(N, 0.55, 10.0), device=dev) if kind == "powerlaw" else None
-    keys, firsts = [], []
-    drawn = 0
     target = int(E * 1.15) + 1024
+    buf = torch.empty(target, dtype=torch.int64, device=dev)
+    n = drawn = 0
     while True:
         while drawn < target:
             cnt = min(_CHUNK * 4, target - drawn)
@@ -94,25 +97,39 @@ def undirected_pairs(N, E, kind, seed=GRAPH_SEED, device="cuda"):
                 u, v = _gnm_candidates(N, drawn, cnt, seed, dev)
             else:
                 raise ValueError(f"device generator: kind {kind!r} not supported")
-            ok = u != v
-            lo = torch.minimum(u, v)[ok]
-            hi = torch.maximum(u, v)[ok]
-            keys.append(lo * N + hi)
-            firsts.append(torch.arange(drawn, drawn + cnt, dtype=torch.int64, device=dev)[ok])
+            k = (torch.minimum(u, v) * N + torch.maximum(u, v))[u != v]
+            del u, v
+            if n + k.numel() > buf.numel():
+                grown = torch.empty(max(n + k.numel(), int(buf.numel() * 1.5)), dtype=torch.int64, device=dev)
+                grown[:n] = buf[:n]
+                buf = grown
+            buf[n:n + k.numel()] = k
+            n += k.numel()
             drawn += cnt
-        allk = torch.cat(keys)
-        allf = torch.cat(firsts)
-        # first occurrence of each distinct key = smallest draw index (stable sort keeps draw order)
-        sk, order = torch.sort(allk, stable=True)
-        head = torch.ones_like(sk, dtype=torch.bool)
+        allk = buf[:n]
+        sk, order = torch.sort(allk, stable=True)      # equal keys keep draw order: head = first draw
+        head = torch.ones(n, dtype=torch.bool, device=dev)
         head[1:] = sk[1:] != sk[:-1]
-        uk = sk[head]
-        fi = allf[order[head]]
-        if uk.numel() >= E:
-            sel = uk[torch.sort(fi, stable=True)[1][:E]]
-            return torch.stack([sel // N, sel % N], dim=1)
-        keys, firsts = [allk], [allf]
-        target = drawn + max(int((E - uk.numel()) * 2.0), _CHUNK)
+        del sk
+        fpos = order[head]
+        del order, head
+        if fpos.numel() >= E:
+            first = torch.zeros(n, dtype=torch.bool, device=dev)
+            first[fpos] = True
+            del fpos
+            c = torch.cumsum(first, 0, dtype=torch.int32 if n < (1 << 31) else torch.int64)
+            cut = int(torch.searchsorted(c, torch.tensor([E], dtype=c.dtype, device=dev))[0])
+            del c
+            first[cut + 1:] = False                    # keep the E earliest first draws
+            return allk[first]
+        del fpos
+        target = drawn + max(int((E - 0) * 0.2), _CHUNK)
+
+
+def undirected_pairs(N, E, kind, seed=GRAPH_SEED, device="cuda"):
+    """The E distinct undirected pairs (u < v) with the smallest first-draw index (int64 [E,2])."""
+    sel = undirected_keys(N, E, kind, seed, device)
+    return torch.stack([sel // N, sel % N], dim=1)
 
 
 def pairs_to_csr(N, pairs):
@@ -126,8 +143,36 @@ def pairs_to_csr(N, pairs):
     return row_ptr, col
 
 
+def keys_to_csr(N, sel, max_chunk=400_000_000):
+    """Symmetric sorted CSR of the pairs sel = u * N + v (u < v), built in row ranges so that no
+    more than ~max_chunk keys are sorted at once (the same CSR as pairs_to_csr)."""
+    dev = sel.device
+    lo = (sel // N).to(torch.int32)
+    hi = (sel - lo.to(torch.int64) * N).to(torch.int32)
+    deg = torch.bincount(lo, minlength=N) + torch.bincount(hi, minlength=N)
+    row_ptr = torch.zeros(N + 1, dtype=torch.int64, device=dev)
+    torch.cumsum(deg, 0, out=row_ptr[1:])
+    del deg
+    col = torch.empty(2 * sel.numel(), dtype=torch.int32, device=dev)
+    nchunks = max(1, -(-2 * sel.numel() // max_chunk))
+    bounds = [int(x) for x in torch.searchsorted(
+        row_ptr, torch.linspace(0, 2 * sel.numel(), nchunks + 1, device=dev).to(torch.int64)).cpu()]
+    bounds[0], bounds[-1] = 0, N
+    for a, b in zip(bounds[:-1], bounds[1:]):
+        if b <= a:
+            continue
+        m1 = (lo >= a) & (lo < b)
+        m2 = (hi >= a) & (hi < b)
+        key = torch.cat([lo[m1].to(torch.int64) * N + hi[m1], hi[m2].to(torch.int64) * N + lo[m2]])
+        del m1, m2
+        key = torch.sort(key)[0]
+        col[int(row_ptr[a]):int(row_ptr[b])] = (key % N).to(torch.int32)
+        del key
+    return row_ptr, col
+
+
 def random_graph(N, E, kind, seed=GRAPH_SEED, device="cuda"):
-    return pairs_to_csr(N, undirected_pairs(N, E, kind, seed, device))
+    return keys_to_csr(N, undirected_keys(N, E, kind, seed, device))
 
 
 def features(N, d, pitch=None, seed=DATA_SEED, dtype=torch.float32, device="cuda"):

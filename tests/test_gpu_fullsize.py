@@ -1,7 +1,9 @@
 """Full-size parity at BASELINE.json configs[2] (ogbn-products-shaped: 2,449,029 nodes, 123.7 M
-CSR entries, 100-d features, 3-layer SAGE-mean 100-256-256-47, fanout (10,25,30), the memory
-budget bench.py calibrates so that one GPU needs >= 8 bucket groups), in the launch
-configuration bench.py times (bf16 feature table, tcgen05 bf16 Update GEMM).
+CSR entries, 100-d features, 3-layer SAGE-mean 100-256-256-47, fanout (10,25,30)) and configs[3]
+(ogbn-papers100M-shaped: 111,059,956 nodes, 3.23 B CSR entries, 128-d, 2-layer 128-256-172,
+fanout (10,25)), each with the memory budget bench.py calibrates so that one GPU needs >= 8
+bucket groups, in the launch configuration bench.py times (bf16 feature table, tcgen05 bf16
+Update GEMM).
 
 * the plan: every seed in exactly one group, group sizes = the plan's exact block sizes,
   estimates within the budget;
@@ -29,12 +31,12 @@ if torch.cuda.is_available():
     from paper_conf_hpca_yangzl25_b200.train import DeviceGraph, Trainer
 
 
-@pytest.fixture(scope="module")
-def products():
+@pytest.fixture(scope="module", params=["products", "papers"])
+def products(request):
     import bench
-    cfg = CONFIGS["products"]
-    rp, col, X, y, seeds, Ws, bs = bench.make_inputs_device(cfg)
-    feats = X.to(torch.bfloat16).contiguous()
+    cfg = CONFIGS[request.param]
+    rp, col, X, y, seeds, Ws, bs = bench.make_inputs_device(cfg, torch.bfloat16)
+    feats = X.contiguous()
     graph = DeviceGraph(rp, col)
     kw = dict(feat_dtype=B.BF16, gemm_mode=B.GEMM_BF16)
     full = Trainer(graph, feats, y, seeds, cfg.dims, cfg.fanout, cfg.F, Ws, bs, k_min=1, k_max=1, **kw)
@@ -43,10 +45,17 @@ def products():
     tr = Trainer(graph, feats, y, seeds, cfg.dims, cfg.fanout, cfg.F, Ws, bs, k_min=cfg.k_min, k_max=cfg.k_max,
                  mem_budget=int(est1[0]) // 8, **kw)
     K, offs, est, ranks = tr.schedule(0)
-    host = dict(rp=rp.cpu().numpy(), col=col.cpu().numpy(), X=X[:, :cfg.d0].float().cpu().numpy(),
-                y=y.cpu().numpy())
-    return dict(cfg=cfg, tr=tr, K=K, offs=offs, est=est, budget=int(est1[0]) // 8, Ws=Ws, bs=bs, **host,
-                g=O.Graph(host["rp"], host["col"]))
+    host = dict(rp=rp.cpu().numpy(), col=col.cpu().numpy(), y=y.cpu().numpy())
+
+    def xrows(ids):
+        """Feature rows of the given nodes, read from the synth-generated table (inputs only)."""
+        idx = torch.as_tensor(np.asarray(ids, np.int64), device="cuda")
+        return feats[idx, :cfg.d0].float().cpu().numpy()
+
+    yield dict(cfg=cfg, tr=tr, K=K, offs=offs, est=est, budget=int(est1[0]) // 8, Ws=Ws, bs=bs, Xrows=xrows,
+               **host, g=O.Graph(host["rp"], host["col"]))
+    del tr, feats, graph, rp, col, X
+    torch.cuda.empty_cache()
 
 
 def test_products_plan(products):
@@ -97,7 +106,7 @@ def test_products_group_blocks_bit_exact(products, which):
             np.testing.assert_array_equal(a["t_col"], r["t_col"], err_msg=f"layer {l} t_col")
 
 
-def _restricted_forward(blocks, X, Ws, bs, out_rows):
+def _restricted_forward(blocks, Xrows, Ws, bs, out_rows):
     """The oracle's forward (O.mean_adjacency, O.round_bf16: bf16-storage reading R26) restricted
     to the receptive field of `out_rows` of the last block: same arithmetic as
     O.sage_forward, evaluated on the rows it needs only."""
@@ -110,7 +119,7 @@ def _restricted_forward(blocks, X, Ws, bs, out_rows):
         nb = np.concatenate([cl[rp[i]:rp[i + 1]] for i in need[l]] + [need[l]])   # neighbours + self (prefix)
         need[l - 1] = np.unique(nb)
     rnd = O.round_bf16
-    H = np.asarray(X, np.float64)[blocks[0]["src_global"][need[0]]]
+    H = Xrows(blocks[0]["src_global"][need[0]]).astype(np.float64)
     for l in range(1, L + 1):
         b = blocks[l - 1]
         A = O.mean_adjacency(b)[need[l]][:, need[l - 1]]
@@ -138,8 +147,12 @@ def test_products_forward_sampled(products):
     A = O.mean_adjacency(ref[0])
     r0 = ref[0]
     rp = r0["row_ptr"].astype(np.int64)
-    X = products["X"]
-    exact = np.stack([X[r0["src_global"][r0["col_local"][rp[i]:rp[i + 1]]]].astype(np.float64).sum(0) for i in rows])
+    Xrows = products["Xrows"]
+    nb = [r0["src_global"][r0["col_local"][rp[i]:rp[i + 1]]] for i in rows]
+    flat = Xrows(np.concatenate(nb)).astype(np.float64)
+    cut = np.cumsum([0] + [len(v) for v in nb])
+    exact = np.stack([flat[cut[j]:cut[j + 1]].sum(0) if cut[j + 1] > cut[j] else np.zeros(cfg.d0)
+                      for j in range(len(rows))])
     D = r0["D"][rows].astype(np.float32)[:, None]
     want = np.where(D > 0, exact.astype(np.float32) / np.maximum(D, 1), np.float32(0))
     want = torch.as_tensor(want).to(torch.bfloat16).float().numpy()
@@ -149,7 +162,7 @@ def test_products_forward_sampled(products):
     bL = tr.blocks.layer[tr.L - 1]
     srows = np.sort(rng.choice(bL.n_dst, 24, replace=False))
     logits = act_view(tr.arena, bL.out, bL.n_dst, bL.ld_out, torch.float32)[srows, :cfg.classes]
-    want = _restricted_forward(ref, X, products["Ws"], products["bs"], srows)
+    want = _restricted_forward(ref, Xrows, products["Ws"], products["bs"], srows)
     assert_bf16_close(logits, want, "sampled logits")
 
 
