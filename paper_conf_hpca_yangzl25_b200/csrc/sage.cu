@@ -214,97 +214,121 @@ static buffalo_status launch_agg(const buffalo_block* blk, const int32_t* col, c
 // ------------------------------------------------------------------ SIMT GEMM
 // C[M][Np] = A1[M][K1] B1[K1][N] + A2[M][K2] B2[K2][N] (+ bias) (ReLU); columns N..Np-1 = 0.
 // A1 row r is A1[gidx ? gidx[r] : r] and is zero for r >= m1.
-constexpr int GB_M = 64, GB_N = 64, GB_K = 16;
+// CTA tile 128 x 128, K step 8, 256 threads with an 8 x 8 register tile each (rows
+// 8 ty .. 8 ty + 7, columns in two 4-wide runs tx * 4 and 64 + tx * 4, so that both fragments
+// are two float4 shared loads per k); the next K step's operands are prefetched into registers while the
+// current one is multiplied.  The K loop order is fixed, so results are deterministic.
+constexpr int GB_M = 128, GB_N = 128, GB_K = 8;
 
 // TB: B1 and B2 are read transposed (B[k][n] = Bt[n][k], ldb = row pitch of Bt).
 template <class TA1, class TA2, class TO, bool TB = false>
-__global__ void __launch_bounds__(256) k_gemm2(int64_t M, int N, int Np, int K1, int K2,
-                                               const TA1* __restrict__ A1, int64_t lda1,
-                                               const int32_t* __restrict__ gidx, int64_t m1,
-                                               const TA2* __restrict__ A2, int64_t lda2,
-                                               const float* __restrict__ B1, int64_t ldb1,
-                                               const float* __restrict__ B2, int64_t ldb2,
-                                               const float* __restrict__ bias, int relu,
-                                               TO* __restrict__ Cm, int64_t ldc) {
-  __shared__ float As[GB_K][GB_M + 4];
-  __shared__ float Bs[GB_K][GB_N];
+__global__ void __launch_bounds__(256, 2) k_gemm2(int64_t M, int N, int Np, int K1, int K2,
+                                                  const TA1* __restrict__ A1, int64_t lda1,
+                                                  const int32_t* __restrict__ gidx, int64_t m1,
+                                                  const TA2* __restrict__ A2, int64_t lda2,
+                                                  const float* __restrict__ B1, int64_t ldb1,
+                                                  const float* __restrict__ B2, int64_t ldb2,
+                                                  const float* __restrict__ bias, int relu,
+                                                  TO* __restrict__ Cm, int64_t ldc) {
+  __shared__ __align__(16) float As[GB_K][GB_M + 4];
+  __shared__ __align__(16) float Bs[GB_K][GB_N + 4];
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
   const int64_t m0 = (int64_t)blockIdx.x * GB_M;
   const int n0 = blockIdx.y * GB_N;
-  float acc[4][4] = {};
+  float acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
   const int nk1 = (K1 + GB_K - 1) / GB_K, nk2 = (K2 + GB_K - 1) / GB_K;
-  const int ar = tid >> 2, ak = (tid & 3) * 4;     // A: row ar, k ak..ak+3
-  const int bk = tid >> 4, bn = (tid & 15) * 4;    // B: k bk, n bn..bn+3
-  for (int kt = 0; kt < nk1 + nk2; ++kt) {
+  // A loads: row ar = tid / 2, k ak .. ak + 3 (ak = 0 or 4); gathered row index read once
+  const int ar = tid >> 1, ak = (tid & 1) * 4;
+  const int64_t r = m0 + ar;
+  int64_t rr1 = -1;
+  if (r < M && r < m1) rr1 = gidx ? (int64_t)gidx[r] : r;
+  // B loads: plain: k bk = tid / 32, n bn .. bn + 3; transposed: n tn = tid / 2, k tk .. tk + 3
+  const int bk = tid >> 5, bn = (tid & 31) * 4;
+  float ra[4], rb[4];
+  auto load = [&](int kt) {
     const bool first = kt < nk1;
     const int k0 = first ? kt * GB_K : (kt - nk1) * GB_K;
     const int K = first ? K1 : K2;
-    {
-      const int64_t r = m0 + ar;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int k = k0 + ak + q;
+      float v = 0.f;
+      if (k < K) {
+        if (first) {
+          if (rr1 >= 0) v = ld1<TA1>(A1 + rr1 * lda1 + k);
+        } else if (r < M) {
+          v = ld1<TA2>(A2 + r * lda2 + k);
+        }
+      }
+      ra[q] = v;
+    }
+    const float* B = first ? B1 : B2;
+    const int64_t ldb = first ? ldb1 : ldb2;
+    if (TB) {
+      const int nn = n0 + ar;
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const int k = k0 + ak + q;
-        float v = 0.f;
-        if (r < M && k < K) {
-          if (first) {
-            if (r < m1) {
-              const int64_t rr = gidx ? (int64_t)gidx[r] : r;
-              v = ld1<TA1>(A1 + rr * lda1 + k);
-            }
-          } else {
-            v = ld1<TA2>(A2 + r * lda2 + k);
-          }
-        }
-        As[ak + q][ar] = v;
+        rb[q] = (k < K && nn < N) ? __ldg(B + (int64_t)nn * ldb + k) : 0.f;
       }
-      const float* B = first ? B1 : B2;
-      const int64_t ldb = first ? ldb1 : ldb2;
-      if (TB) {   // Bt[n][k]: thread = (n = tid / 4, 4 consecutive k), 4 threads per 64-B row run
-        const int tn = tid >> 2, tk = (tid & 3) * 4;
-        const int nn = n0 + tn;
+    } else {
+      const int k = k0 + bk;
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          const int k = k0 + tk + q;
-          Bs[tk + q][tn] = (k < K && nn < N) ? __ldg(B + (int64_t)nn * ldb + k) : 0.f;
-        }
-      } else {
-        const int k = k0 + bk;
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          const int nn = n0 + bn + q;
-          Bs[bk][bn + q] = (k < K && nn < N) ? __ldg(B + (int64_t)k * ldb + nn) : 0.f;
-        }
+      for (int q = 0; q < 4; ++q) {
+        const int nn = n0 + bn + q;
+        rb[q] = (k < K && nn < N) ? __ldg(B + (int64_t)k * ldb + nn) : 0.f;
       }
     }
+  };
+  const int nkt = nk1 + nk2;
+  if (nkt > 0) load(0);
+  for (int kt = 0; kt < nkt; ++kt) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) As[ak + q][ar] = ra[q];
+    if (TB) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) Bs[ak + q][ar] = rb[q];
+    } else {
+      *reinterpret_cast<float4*>(&Bs[bk][bn]) = make_float4(rb[0], rb[1], rb[2], rb[3]);
+    }
     __syncthreads();
+    if (kt + 1 < nkt) load(kt + 1);              // global loads in flight during the math
 #pragma unroll
     for (int kk = 0; kk < GB_K; ++kk) {
-      float a[4], b[4];
+      float a[8], b[8];
+      const float4 a0 = *reinterpret_cast<const float4*>(&As[kk][ty * 8]);
+      const float4 a1 = *reinterpret_cast<const float4*>(&As[kk][ty * 8 + 4]);
+      a[0] = a0.x; a[1] = a0.y; a[2] = a0.z; a[3] = a0.w;
+      a[4] = a1.x; a[5] = a1.y; a[6] = a1.z; a[7] = a1.w;
+      const float4 b0 = *reinterpret_cast<const float4*>(&Bs[kk][tx * 4]);
+      const float4 b1 = *reinterpret_cast<const float4*>(&Bs[kk][64 + tx * 4]);
+      b[0] = b0.x; b[1] = b0.y; b[2] = b0.z; b[3] = b0.w;
+      b[4] = b1.x; b[5] = b1.y; b[6] = b1.z; b[7] = b1.w;
 #pragma unroll
-      for (int i = 0; i < 4; ++i) a[i] = As[kk][ty * 4 + i];
+      for (int i = 0; i < 8; ++i)
 #pragma unroll
-      for (int j = 0; j < 4; ++j) b[j] = Bs[kk][tx * 4 + j];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
     }
     __syncthreads();
   }
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int64_t r = m0 + ty * 4 + i;
-    if (r >= M) continue;
+  for (int i = 0; i < 8; ++i) {
+    const int64_t row = m0 + ty * 8 + i;
+    if (row >= M) continue;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int nn = n0 + tx * 4 + j;
+    for (int j = 0; j < 8; ++j) {
+      const int nn = n0 + (j < 4 ? tx * 4 + j : 64 + tx * 4 + (j - 4));
       if (nn >= Np) continue;
       float v = 0.f;
       if (nn < N) {
         v = acc[i][j] + (bias ? bias[nn] : 0.f);
         if (relu) v = fmaxf(v, 0.f);
       }
-      st1<TO>(Cm + r * ldc + nn, v);
+      st1<TO>(Cm + row * ldc + nn, v);
     }
   }
 }
@@ -352,73 +376,86 @@ __global__ void __launch_bounds__(256) k_aggT(const int32_t* __restrict__ trp, c
 // dW partial of split s: part[s][n][k] = sum_{r in split s} dZ[r][n] * Afwd[r][k],
 // Afwd[r] = [self(r) || agg(r)].
 // K = 2 d_in (Update weight: [self || agg]) or d_in (pool weight: self rows only).
+// CTA tile 128 (n) x 128 (k) over one row split, 8 rows per step, 8 x 8 register tile per
+// thread, next step prefetched into registers; db partial (column sums of dZ, fixed row order)
+// by the CTAs of k-tile 0.
+constexpr int DW_T = 128, DW_R = 8;
 template <class TS, class TG>
-__global__ void __launch_bounds__(256) k_dw_partial(int64_t nrows, int d_out, int d_in, int K,
-                                                    const float* __restrict__ dz, int64_t ldz,
-                                                    const TS* __restrict__ self, int64_t lds,
-                                                    const int32_t* __restrict__ gidx,
-                                                    const TG* __restrict__ agg, int64_t ldg,
-                                                    int64_t rows_per_split, float* __restrict__ part,
-                                                    float* __restrict__ db_part) {
-  __shared__ float Zs[16][64];
-  __shared__ float As[16][64];
+__global__ void __launch_bounds__(256, 2) k_dw_partial(int64_t nrows, int d_out, int d_in, int K,
+                                                       const float* __restrict__ dz, int64_t ldz,
+                                                       const TS* __restrict__ self, int64_t lds,
+                                                       const int32_t* __restrict__ gidx,
+                                                       const TG* __restrict__ agg, int64_t ldg,
+                                                       int64_t rows_per_split, float* __restrict__ part,
+                                                       float* __restrict__ db_part) {
+  __shared__ __align__(16) float Zs[DW_R][DW_T + 4];
+  __shared__ __align__(16) float As[DW_R][DW_T + 4];
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
-  const int k0 = blockIdx.x * 64, n0 = blockIdx.y * 64;
+  const int k0 = blockIdx.x * DW_T, n0 = blockIdx.y * DW_T;
   const int64_t r_beg = (int64_t)blockIdx.z * rows_per_split;
   const int64_t r_end = min(nrows, r_beg + rows_per_split);
-  float acc[4][4] = {};
-  float dbs[4] = {0.f, 0.f, 0.f, 0.f};      // column sums of dZ (CTAs of k-tile 0, threads ty == 0)
-  const bool do_db = blockIdx.x == 0 && ty == 0;
-  const int lr = tid >> 4, lc = (tid & 15) * 4;
-  for (int64_t r0 = r_beg; r0 < r_end; r0 += 16) {
-    const int64_t r = r0 + lr;
+  float acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+  const bool do_db = blockIdx.x == 0 && tid < DW_T;
+  float dbs = 0.f;
+  // loads: row lr = tid / 32 of the step, 4 consecutive columns lc .. lc + 3
+  const int lr = tid >> 5, lc = (tid & 31) * 4;
+  float rz[4], ra[4];
+  auto load = [&](int64_t r0) {
+    const int64_t rw = r0 + lr;
+    const bool in = rw < r_end;
+    const int64_t rs = (in && gidx) ? (int64_t)gidx[rw] : rw;
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
       const int nn = n0 + lc + q, k = k0 + lc + q;
-      float z = 0.f, a = 0.f;
-      if (r < r_end) {
-        if (nn < d_out) z = dz[r * ldz + nn];
-        if (k < d_in) {
-          const int64_t rr = gidx ? (int64_t)gidx[r] : r;
-          a = ld1<TS>(self + rr * lds + k);
-        } else if (k < K) {
-          a = ld1<TG>(agg + r * ldg + (k - d_in));
-        }
+      rz[q] = (in && nn < d_out) ? dz[rw * ldz + nn] : 0.f;
+      float a = 0.f;
+      if (in) {
+        if (k < d_in) a = ld1<TS>(self + rs * lds + k);
+        else if (k < K) a = ld1<TG>(agg + rw * ldg + (k - d_in));
       }
-      Zs[lr][lc + q] = z;
-      As[lr][lc + q] = a;
+      ra[q] = a;
     }
+  };
+  if (r_beg < r_end) load(r_beg);
+  for (int64_t r0 = r_beg; r0 < r_end; r0 += DW_R) {
+    *reinterpret_cast<float4*>(&Zs[lr][lc]) = make_float4(rz[0], rz[1], rz[2], rz[3]);
+    *reinterpret_cast<float4*>(&As[lr][lc]) = make_float4(ra[0], ra[1], ra[2], ra[3]);
     __syncthreads();
+    if (r0 + DW_R < r_end) load(r0 + DW_R);
     if (do_db)
-      for (int rr = 0; rr < 16; ++rr)
 #pragma unroll
-        for (int j = 0; j < 4; ++j) dbs[j] += Zs[rr][tx * 4 + j];
+      for (int rr = 0; rr < DW_R; ++rr) dbs += Zs[rr][tid];
 #pragma unroll
-    for (int rr = 0; rr < 16; ++rr) {
-      float zz[4], aa[4];
+    for (int rr = 0; rr < DW_R; ++rr) {
+      float z[8], a[8];
+      const float4 z0 = *reinterpret_cast<const float4*>(&Zs[rr][ty * 8]);
+      const float4 z1 = *reinterpret_cast<const float4*>(&Zs[rr][ty * 8 + 4]);
+      z[0] = z0.x; z[1] = z0.y; z[2] = z0.z; z[3] = z0.w;
+      z[4] = z1.x; z[5] = z1.y; z[6] = z1.z; z[7] = z1.w;
+      const float4 a0 = *reinterpret_cast<const float4*>(&As[rr][tx * 4]);
+      const float4 a1 = *reinterpret_cast<const float4*>(&As[rr][64 + tx * 4]);
+      a[0] = a0.x; a[1] = a0.y; a[2] = a0.z; a[3] = a0.w;
+      a[4] = a1.x; a[5] = a1.y; a[6] = a1.z; a[7] = a1.w;
 #pragma unroll
-      for (int i = 0; i < 4; ++i) zz[i] = Zs[rr][ty * 4 + i];
+      for (int i = 0; i < 8; ++i)
 #pragma unroll
-      for (int j = 0; j < 4; ++j) aa[j] = As[rr][tx * 4 + j];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(zz[i], aa[j], acc[i][j]);
+        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(z[i], a[j], acc[i][j]);
     }
     __syncthreads();
   }
-  if (do_db)
-#pragma unroll
-    for (int j = 0; j < 4; ++j)
-      if (n0 + tx * 4 + j < d_out) db_part[(int64_t)blockIdx.z * d_out + n0 + tx * 4 + j] = dbs[j];
+  if (do_db && n0 + tid < d_out) db_part[(int64_t)blockIdx.z * d_out + n0 + tid] = dbs;
   float* P = part + (int64_t)blockIdx.z * d_out * K;
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int nn = n0 + ty * 4 + i;
+  for (int i = 0; i < 8; ++i) {
+    const int nn = n0 + ty * 8 + i;
     if (nn >= d_out) continue;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int k = k0 + tx * 4 + j;
+    for (int j = 0; j < 8; ++j) {
+      const int k = k0 + (j < 4 ? tx * 4 + j : 64 + tx * 4 + (j - 4));
       if (k < K) P[(int64_t)nn * K + k] = acc[i][j];
     }
   }
@@ -595,7 +632,7 @@ static buffalo_status bwd_ffma_t(const BwdArgs& a, cudaStream_t s) {
   float* aggT = (float*)q;
   const int64_t rps = ceil_div(n > 0 ? n : 1, S);
   if (n > 0) {
-    dim3 g((unsigned)ceil_div(2 * d_in, 64), (unsigned)ceil_div(d_out, 64), (unsigned)S);
+    dim3 g((unsigned)ceil_div(2 * d_in, DW_T), (unsigned)ceil_div(d_out, DW_T), (unsigned)S);
     k_dw_partial<TS, TG><<<g, 256, 0, s>>>(n, d_out, d_in, 2 * d_in, a.dh, a.ld_dh, (const TS*)a.h_src, a.ld_src,
                                            a.layer1 ? blk->src_global : nullptr, (const TG*)a.agg,
                                            a.ld_agg, rps, dw_part, db_part);
@@ -768,7 +805,7 @@ static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
   float* dbp_part = (float*)q;
   if (n > 0) {
     // dW, db of the Update weight (as the mean path)
-    dim3 g((unsigned)ceil_div(2 * d_in, 64), (unsigned)ceil_div(d_out, 64), (unsigned)S);
+    dim3 g((unsigned)ceil_div(2 * d_in, DW_T), (unsigned)ceil_div(d_out, DW_T), (unsigned)S);
     k_dw_partial<TI, float><<<g, 256, 0, s>>>(n, d_out, d_in, 2 * d_in, a.dh, a.ld_dh, (const TI*)a.h_src,
                                               a.ld_src, gidx, a.agg, a.ld_agg, ceil_div(n, S), dw_part, db_part);
     BF_LAUNCHED("k_dw_partial");
@@ -791,7 +828,7 @@ static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
     BF_CUDA(cudaMemsetAsync(dq, 0, sizeof(float) * ns * dp, s));
   }
   // dW_pool, db_pool over the src rows
-  dim3 g2((unsigned)ceil_div(d_in, 64), (unsigned)ceil_div(d_in, 64), (unsigned)S2);
+  dim3 g2((unsigned)ceil_div(d_in, DW_T), (unsigned)ceil_div(d_in, DW_T), (unsigned)S2);
   k_dw_partial<TI, float><<<g2, 256, 0, s>>>(ns, d_in, d_in, d_in, dq, dp, (const TI*)a.h_src, a.ld_src, gidx,
                                              nullptr, 0, ceil_div(ns, S2), dwp_part, dbp_part);
   BF_LAUNCHED("k_dw_partial");
@@ -1118,7 +1155,7 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
   float* dwl_part = (float*)q; q += R((int64_t)S3 * 4 * d * d * 4);
   float* dbl_part = (float*)q;
   if (n > 0) {
-    dim3 g((unsigned)ceil_div(2 * d, 64), (unsigned)ceil_div(d_out, 64), (unsigned)S);
+    dim3 g((unsigned)ceil_div(2 * d, DW_T), (unsigned)ceil_div(d_out, DW_T), (unsigned)S);
     k_dw_partial<TI, float><<<g, 256, 0, st>>>(n, d_out, d, 2 * d, a.dh, a.ld_dh, (const TI*)a.h_src, a.ld_src, gidx,
                                                a.agg, a.ld_agg, ceil_div(n, S), dw_part, db_part);
     BF_LAUNCHED("k_dw_partial");
@@ -1151,7 +1188,7 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
   }
   if (e > 0) {
     // dW_ih (+ db_lstm) = dG^T X over the packed rows, then dW_hh = dG^T H_prev
-    dim3 g3((unsigned)ceil_div(d, 64), (unsigned)ceil_div(4 * d, 64), (unsigned)S3);
+    dim3 g3((unsigned)ceil_div(d, DW_T), (unsigned)ceil_div(4 * d, DW_T), (unsigned)S3);
     k_dw_partial<TI, float><<<g3, 256, 0, st>>>(e, 4 * d, d, d, v.G, ldg, (const TI*)a.h_src, a.ld_src, v.gix, nullptr,
                                                 0, ceil_div(e, S3), dwl_part, dbl_part);
     BF_LAUNCHED("k_dw_partial");
@@ -1482,21 +1519,21 @@ static buffalo_status gat_bwd_t(const GatArgs& a, cudaStream_t st) {
                                                             d_er, d_el, dZ, ldz);
   BF_LAUNCHED("k_gat_src_bwd");
   // da_l = d_el^T Z, da_r = d_er^T Z[:n_dst], dW = dZ^T H (deterministic split reductions)
-  dim3 gl((unsigned)ceil_div(dl, 64), 1, (unsigned)Sl);
+  dim3 gl((unsigned)ceil_div(dl, DW_T), 1, (unsigned)Sl);
   k_dw_partial<float, float><<<gl, 256, 0, st>>>(ns, 1, dl, dl, d_el, 1, v.Z, ldz, nullptr, nullptr, 0,
                                                  ceil_div(ns, Sl), dal_part, dal_b);
   BF_LAUNCHED("k_dw_partial");
   k_reduce_partials<<<1, 256, 0, st>>>(dal_part, Sl, dl, a.da_l);
   BF_LAUNCHED("k_reduce_partials");
   if (nd > 0) {
-    dim3 gr((unsigned)ceil_div(dl, 64), 1, (unsigned)Sr);
+    dim3 gr((unsigned)ceil_div(dl, DW_T), 1, (unsigned)Sr);
     k_dw_partial<float, float><<<gr, 256, 0, st>>>(nd, 1, dl, dl, d_er, 1, v.Z, ldz, nullptr, nullptr, 0,
                                                    ceil_div(nd, Sr), dar_part, dar_b);
     BF_LAUNCHED("k_dw_partial");
     k_reduce_partials<<<1, 256, 0, st>>>(dar_part, Sr, dl, a.da_r);
     BF_LAUNCHED("k_reduce_partials");
   }
-  dim3 gw((unsigned)ceil_div(d_in, 64), (unsigned)ceil_div(dl, 64), (unsigned)S4);
+  dim3 gw((unsigned)ceil_div(d_in, DW_T), (unsigned)ceil_div(dl, DW_T), (unsigned)S4);
   k_dw_partial<TI, float><<<gw, 256, 0, st>>>(ns, dl, d_in, d_in, dZ, ldz, (const TI*)a.h_src, a.ld_src,
                                               a.layer1 ? blk->src_global : nullptr, nullptr, 0, ceil_div(ns, S4),
                                               dw_part, db_part);
