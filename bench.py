@@ -65,6 +65,9 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-baseline-seconds", type=float, default=20.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-pipeline", action="store_true",
+                    help="schedule each epoch synchronously (default: the next epoch's plan is computed on a "
+                         "side stream while the current epoch trains)")
     return ap.parse_args()
 
 
@@ -286,7 +289,7 @@ def run_ours(args, cfg):
     tr = Trainer(graph, feats, y, seeds, cfg.dims,
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, mem_budget=budget,
                  C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg,
-                 **agg_kw)
+                 pipeline=not args.no_pipeline, **agg_kw)
     if args.config in ("products", "papers", "arxiv_lstm"):
         # calibrate M_ctr once so that one GPU needs >= 8 groups (products; 2 for the LSTM
         # workload), then freeze it for every N
@@ -418,6 +421,7 @@ def run_ours(args, cfg):
                     "l2": "flushed (512 MiB write) between timed steps",
                     "epoch_ms": total_ms / args.steps, "edges_per_epoch": edges / args.steps,
                     "parallelism": f"dp{world} over bucket groups",
+                    "pipeline": "scheduler of epoch e+1 overlapped with epoch e" if not args.no_pipeline else "off",
                     "C_eq1": C_eq1, "C_ppm": C_ppm, "C_table2": C_TABLE2.get(args.config),
                     "C_seconds": t_c},
             roofline=roof,

@@ -212,7 +212,9 @@ BUFFALO_API buffalo_status buffalo_sage_fwd(const buffalo_block* blk, int32_t la
 
 /* ------------------------------------------------------------------ a8: loss */
 /* Partial loss of a group (Alg. 2 l.10, R19): loss_accum[0] += sum_i CE(softmax(Z_i), y_i) / S
- * and dlogits = (softmax(Z) - onehot(y)) / S, with y_i = labels[row_ids[i]]. */
+ * and dlogits = (softmax(Z) - onehot(y)) / S, with y_i = labels[row_ids[i]].  dlogits (and so
+ * every gradient) is deterministic; the loss scalar is a reported value accumulated with one
+ * float atomic per CTA, so its last bits depend on the CTA completion order. */
 BUFFALO_API buffalo_status buffalo_softmax_ce(const float* logits, int64_t ld, int64_t n, int32_t classes,
                                   const int32_t* labels, const int32_t* row_ids,
                                   int64_t batch_size, float* loss_accum, float* dlogits,

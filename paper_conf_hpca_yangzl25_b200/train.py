@@ -42,6 +42,43 @@ class DeviceGraph:
         self.g.row_ptr = self.row_ptr.data_ptr()
         self.g.col = self.col.data_ptr()
         B.graph_prepare(self.g, self.ws)
+        self._sched_ws = None
+        self._g_sched = None
+
+    @property
+    def g_sched(self):
+        """A second view of the graph with its own node_map / bitmap workspace, for a scheduler
+        that runs on another stream while the blocks of the current epoch are built."""
+        if self._g_sched is None:
+            self._sched_ws = torch.empty_like(self.ws)
+            self._g_sched = B.Graph()
+            self._g_sched.num_nodes, self._g_sched.nnz = self.g.num_nodes, self.g.nnz
+            self._g_sched.row_ptr, self._g_sched.col = self.g.row_ptr, self.g.col
+            B.graph_prepare(self._g_sched, self._sched_ws)
+        return self._g_sched
+
+
+class PlanBuffers:
+    """One set of buffalo_bucketize outputs (device arrays + host arrays + the Plan struct)."""
+
+    def __init__(self, S, k_max, F, L, device):
+        self.group_of_seed = torch.empty(S, dtype=torch.int32, device=device)
+        self.group_seeds = torch.empty(S, dtype=torch.int32, device=device)
+        self.group_offsets = torch.empty(k_max + 1, dtype=torch.int64, device=device)
+        self.offs_h = np.zeros(k_max + 1, np.int64)
+        self.est_h = np.zeros(k_max, np.int64)
+        self.rank_h = np.zeros(k_max, np.int32)
+        self.hist_h = np.zeros(F + 1, np.int64)
+        self.sizes_h = np.zeros((k_max, 2 * L + 1), np.int64)     # exact per-group block sizes
+        self.plan = B.Plan()
+        self.plan.group_of_seed = self.group_of_seed.data_ptr()
+        self.plan.group_seeds = self.group_seeds.data_ptr()
+        self.plan.group_offsets = self.group_offsets.data_ptr()
+        self.plan.group_offsets_h = self.offs_h.ctypes.data
+        self.plan.est_bytes_h = self.est_h.ctypes.data
+        self.plan.rank_of_group_h = self.rank_h.ctypes.data
+        self.plan.hist_h = self.hist_h.ctypes.data
+        self.plan.group_sizes_h = self.sizes_h.ctypes.data
 
 
 class SageParams:
@@ -115,7 +152,7 @@ class Trainer:
     def __init__(self, graph, feats, labels, seeds, dims, fanout, F, Ws, bs, feat_dtype=B.FP32,
                  gemm_mode=B.GEMM_FFMA, mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096,
                  base_seed=3, rank=0, world=1, process_group=None, device="cuda", aggregator=B.AGG_MEAN,
-                 Wps=None, bps=None, lstm=None, gat=None):
+                 Wps=None, bps=None, lstm=None, gat=None, pipeline=False):
         self.graph = graph if isinstance(graph, DeviceGraph) else DeviceGraph(*graph, device=device)
         self.feats = feats
         self.labels = labels
@@ -140,25 +177,17 @@ class Trainer:
         self.params = SageParams(self.model, Ws, bs, device, Wps, bps, lstm, gat)
         self.rank, self.world, self.pg = rank, world, process_group
         self.device = device
-        # scheduler outputs
+        # scheduler outputs: two buffer sets, so that with pipeline=True the plan of epoch e+1 is
+        # computed (on a side stream, with its own graph workspace) while epoch e trains from the
+        # other set.  The plan is a function of (seeds, epoch) only, never of the weights.
         self.k_cap = k_max
-        self.group_of_seed = torch.empty(self.S, dtype=torch.int32, device=device)
-        self.group_seeds = torch.empty(self.S, dtype=torch.int32, device=device)
-        self.group_offsets = torch.empty(k_max + 1, dtype=torch.int64, device=device)
-        self.offs_h = np.zeros(k_max + 1, np.int64)
-        self.est_h = np.zeros(k_max, np.int64)
-        self.rank_h = np.zeros(k_max, np.int32)
-        self.hist_h = np.zeros(F + 1, np.int64)
-        self.sizes_h = np.zeros((k_max, 2 * self.L + 1), np.int64)     # exact per-group block sizes
-        self.plan = B.Plan()
-        self.plan.group_of_seed = self.group_of_seed.data_ptr()
-        self.plan.group_seeds = self.group_seeds.data_ptr()
-        self.plan.group_offsets = self.group_offsets.data_ptr()
-        self.plan.group_offsets_h = self.offs_h.ctypes.data
-        self.plan.est_bytes_h = self.est_h.ctypes.data
-        self.plan.rank_of_group_h = self.rank_h.ctypes.data
-        self.plan.hist_h = self.hist_h.ctypes.data
-        self.plan.group_sizes_h = self.sizes_h.ctypes.data
+        self._pb = [PlanBuffers(self.S, k_max, F, self.L, device)]
+        self._cur = 0
+        self.pipeline = pipeline
+        self._ahead = None
+        if pipeline:
+            self._pb.append(PlanBuffers(self.S, k_max, F, self.L, device))
+            self._side = torch.cuda.Stream(device=device)
         sampler = B.make_sampler(self.fanout, F, base_seed)
         wsb = B.bucketize_workspace_bytes(self.graph.g, self.S, sampler, self.model)
         self.bucket_ws = torch.empty(wsb, dtype=torch.uint8, device=device)
@@ -167,15 +196,31 @@ class Trainer:
         self.blocks = B.Blocks()
         self.last = {}
 
+    # plan of the current epoch (the buffer set in use)
+    group_of_seed = property(lambda self: self._pb[self._cur].group_of_seed)
+    group_seeds = property(lambda self: self._pb[self._cur].group_seeds)
+    group_offsets = property(lambda self: self._pb[self._cur].group_offsets)
+    offs_h = property(lambda self: self._pb[self._cur].offs_h)
+    est_h = property(lambda self: self._pb[self._cur].est_h)
+    rank_h = property(lambda self: self._pb[self._cur].rank_h)
+    hist_h = property(lambda self: self._pb[self._cur].hist_h)
+    sizes_h = property(lambda self: self._pb[self._cur].sizes_h)
+    plan = property(lambda self: self._pb[self._cur].plan)
+
     # --------------------------------------------------------------- pieces of Alg. 2
     def sampler(self, epoch):
         return B.make_sampler(self.fanout, self.F, self.base_seed + epoch)
 
     def schedule(self, epoch):
-        B.bucketize(self.graph.g, self.seeds, self.sampler(epoch), self.model, self.sched, self.plan,
-                    self.bucket_ws)
-        K = self.plan.k_out
-        return K, self.offs_h[:K + 1].copy(), self.est_h[:K].copy(), self.rank_h[:K].copy()
+        """Alg. 3 for `epoch` into the current plan buffers (stream-ordered on the current stream)."""
+        self._ahead = None
+        return self._schedule_into(self._cur, epoch, self.graph.g)
+
+    def _schedule_into(self, buf, epoch, g):
+        pb = self._pb[buf]
+        B.bucketize(g, self.seeds, self.sampler(epoch), self.model, self.sched, pb.plan, self.bucket_ws)
+        K = pb.plan.k_out
+        return K, pb.offs_h[:K + 1].copy(), pb.est_h[:K].copy(), pb.rank_h[:K].copy()
 
     def _ensure_arena(self, nbytes):
         """Grows the micro-batch arena (with 1/8 headroom, so that the need drifting between
@@ -269,9 +314,20 @@ class Trainer:
         self.params.repack()
 
     def run_epoch(self, epoch=0, lr=0.01, timers=False):
-        """One Buffalo iteration; returns stats (K, own groups, aggregated edges, ...)."""
+        """One Buffalo iteration; returns stats (K, own groups, aggregated edges, ...).
+        pipeline=True: the plan was computed during the previous call (if it was for this epoch),
+        and the next epoch's plan is computed on the side stream while this epoch's work runs."""
+        main = torch.cuda.current_stream()
+        a = self._ahead
+        self._ahead = None
+        if self.pipeline and a is not None and a["epoch"] == epoch:
+            self._cur = a["buf"]
+            main.wait_event(a["done"])
+            K, offs, est, ranks = a["K"], a["offs"], a["est"], a["ranks"]
+        else:
+            K, offs, est, ranks = self._schedule_into(self._cur, epoch, self.graph.g)
+        before = main.record_event()        # the next plan depends on nothing enqueued after this
         self.loss.zero_()
-        K, offs, est, ranks = self.schedule(epoch)
         mine = own_groups(ranks, self.rank)
         L = self.L
         need = [B.estimate_mem(self.sizes_h[k, :L + 1], self.sizes_h[k, L + 1:], self.model)[0] for k in mine]
@@ -285,4 +341,13 @@ class Trainer:
         self.last = dict(K=K, k_tried=self.plan.k_tried, exploded=self.plan.exploded, est=est,
                          ranks=ranks, groups=groups, edges=sum(g["edges"] for g in groups),
                          hist=self.hist_h.copy())
+        if self.pipeline:
+            # Alg. 3 of epoch + 1 on the side stream (own graph workspace, the other plan buffers),
+            # overlapping this epoch's build / forward / backward on the main stream
+            nb = 1 - self._cur
+            self._side.wait_event(before)
+            with torch.cuda.stream(self._side):
+                Kn, offn, estn, rankn = self._schedule_into(nb, epoch + 1, self.graph.g_sched)
+                done = self._side.record_event()
+            self._ahead = dict(epoch=epoch + 1, buf=nb, K=Kn, offs=offn, est=estn, ranks=rankn, done=done)
         return self.last
