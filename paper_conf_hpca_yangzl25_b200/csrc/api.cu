@@ -336,7 +336,10 @@ size_t buffalo_graph_workspace_bytes(int64_t num_nodes) { return (size_t)graph_w
 
 buffalo_status buffalo_graph_prepare(buffalo_graph* g, void* workspace, size_t bytes, void* stream) {
   BF_CHECK(require_sm100());
-  if (!g || !workspace || !g->row_ptr || !g->col || g->num_nodes <= 0) return BUFFALO_ERR_INVALID_ARG;
+  if (!g || !workspace || !g->row_ptr || (!g->col && g->nnz > 0) || g->nnz < 0 || g->num_nodes <= 0) {
+    set_error("graph_prepare: null graph/workspace, empty graph or col NULL with nnz > 0");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
   if ((int64_t)bytes < (int64_t)buffalo_graph_workspace_bytes(g->num_nodes)) return BUFFALO_ERR_CAPACITY;
   g->node_map = (int32_t*)workspace;
   cudaStream_t s = (cudaStream_t)stream;
