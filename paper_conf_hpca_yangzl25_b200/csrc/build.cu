@@ -617,7 +617,7 @@ __device__ __forceinline__ void mask_or(unsigned long long* __restrict__ m_out, 
 // One layer: 32/SEG active nodes of layer l per warp; accumulates n_l, e_l per item and ORs
 // each node's mask into layer l-1 for the node itself and its sampled neighbours.
 template <int SEG, int W>
-__global__ void __launch_bounds__(256) k_mask_layer(const int32_t* __restrict__ act, int64_t n_act,
+__global__ void __launch_bounds__(256, (W >= 4 ? 4 : 6)) k_mask_layer(const int32_t* __restrict__ act, int64_t n_act,
                                                     const unsigned long long* __restrict__ m_in,
                                                     unsigned long long* __restrict__ m_out, uint32_t* __restrict__ bits,
                                                     const int64_t* __restrict__ grow, const int32_t* __restrict__ gcol,
