@@ -243,10 +243,16 @@ class Clocks:
 def run_ours(args, cfg):
     import torch
     rank, world, local = dist_env()
-    torch.cuda.set_device(local)
+    # one process per GPU; BUFFALO_DIST_BACKEND=gloo (testing only) lets several ranks share a GPU
+    backend = os.environ.get("BUFFALO_DIST_BACKEND", "nccl")
+    dev = local % torch.cuda.device_count() if backend != "nccl" else local
+    torch.cuda.set_device(dev)
     pg = None
     if world > 1:
-        torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            torch.distributed.init_process_group(backend)
         pg = torch.distributed.group.WORLD
     from paper_conf_hpca_yangzl25_b200 import buffalo as B
     from paper_conf_hpca_yangzl25_b200.train import DeviceGraph, Trainer
@@ -309,7 +315,7 @@ def run_ours(args, cfg):
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
-    clocks = Clocks(local)
+    clocks = Clocks(dev)
     clocks.start()
     # live roofline of the dominant kernel (k_gather_rows, the Aggregate): CUDA events around
     # each of its launches on its stream, algorithmic bytes from the edges it aggregated
