@@ -763,6 +763,12 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   const int npieces = (pitch_in + E - 1) / E;
   int lpr_log = 0;
   while ((1 << lpr_log) < npieces && lpr_log < 5) ++lpr_log;
+  // transposed rows are short (~1-2 entries per src row): two rows per warp (two passes over
+  // the row's pieces) keep twice the per-row metadata chains in flight
+  if (MODE == 1 && lpr_log == 5) {
+    const char* ev = getenv("BUFFALO_T_LPR_LOG");      // diagnostic override (A/B runs)
+    lpr_log = ev ? atoi(ev) : 4;
+  }
   if (n > INT32_MAX || ldh * (int64_t)sizeof(TI) > INT32_MAX) {
     set_error("gather: %lld rows of stride %lld elements exceed the 32-bit row / byte-stride range",
               (long long)n, (long long)ldh);
