@@ -335,7 +335,7 @@ class Trainer:
         sampler = self.sampler(epoch)
         groups = []
         for k in mine:
-            groups.append(self.microbatch(offs[k], int(offs[k + 1] - offs[k]), sampler, self.sizes_h[k]))
+            groups.append(dict(self.microbatch(offs[k], int(offs[k + 1] - offs[k]), sampler, self.sizes_h[k]), k=k))
         self.allreduce()
         self.step(lr)
         self.last = dict(K=K, k_tried=self.plan.k_tried, exploded=self.plan.exploded, est=est,
