@@ -405,11 +405,11 @@ def run_ours(args, cfg):
                        "over-estimates shared nodes; the exact arena model (lo, hi) brackets the measured peak"}
     if lstm:   # the LSTM path is bound by its fp32 SIMT gate GEMMs: FLOP roofline ("alu")
         tf = g_bytes / (g_ms / 1e3) / 1e12 if g_ms > 0 else 0.0
-        roof = {"bound": "alu", "kernel": "k_gemm2 (LSTM gate GEMM of every step, fp32 SIMT)",
+        roof = {"bound": "alu", "kernel": "k_gemm2_tc (LSTM gate GEMM of every step, fp32 as 3xTF32 mma.sync)",
                 "achieved": tf, "peak": FP32_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": tf / FP32_PEAK_TFLOPS,
                 "traffic": None,
                 "peak_source": "derived: 148 SMs x 128 FP32 FMA/clk x 2 flop x 1.965 GHz (no FP32 figure in "
-                               "B200_PROFILING.md)",
+                               "B200_PROFILING.md); achieved counts useful fp32 flops (not the 3 TF32 passes)",
                 "flops_per_launch": g_bytes / max(1, g_launches), "launch_ms": g_ms / max(1, g_launches),
                 "launches": g_launches, "share_of_step": g_ms / total_ms}
     else:

@@ -333,6 +333,167 @@ __global__ void __launch_bounds__(256, 2) k_gemm2(int64_t M, int N, int Np, int 
   }
 }
 
+// ------------------------------------------------------------------ fp32 GEMM on tensor pipes (3xTF32)
+// Same contract as k_gemm2 (used by the pool / LSTM / GAT paths, whose GEMMs have K <= 2 d <= 512):
+// each operand is split x = hi + lo into two TF32 values and the product summed as
+// hi*hi + hi*lo + lo*hi (mma.sync m16n8k8, fp32 accumulate), fp32-level accuracy for these short
+// K.  The long split-K reductions (k_dw_partial) and the mean model's FFMA parity path stay on
+// the CUDA-core kernels: their K runs over thousands of rows with heavy cancellation, where the
+// tensor pipe's accumulation measured outside the fp32 parity tolerance (Cora dW_1).
+// CTA tile 128 x 128, K step 8, 8 warps as 4 (M) x 2 (N), each 32 x 64 = 2 x 8 MMA tiles;
+// operands staged fp32 in shared memory (pitch 136), next K step prefetched into registers.
+constexpr int GB_P = 136;   // shared pitch of the 3xTF32 kernel (conflict-free fragment reads)
+
+__device__ __forceinline__ uint32_t tf32_hi(float x) {
+  uint32_t r;
+  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ void split_tf32(float x, uint32_t& hi, uint32_t& lo) {
+  hi = tf32_hi(x);
+  lo = tf32_hi(x - __uint_as_float(hi));
+}
+__device__ __forceinline__ void mma_tf32(float (&c)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm volatile("mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+               "{%0,%1,%2,%3};"
+               : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+               : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+// One K step of 8 on the warp's 32 x 64 tile: A element (m, k) = As[k][m], B element (k, n) =
+// Bs[k][n]; wm0 / wn0: the warp's first row / column inside the CTA tile.
+__device__ __forceinline__ void warp_mma_k8(const float (*As)[GB_P], const float (*Bs)[GB_P], int wm0, int wn0,
+                                            float (&acc)[2][8][4]) {
+  const int lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
+  uint32_t ah[2][4], al[2][4];
+#pragma unroll
+  for (int mt = 0; mt < 2; ++mt) {
+    const int m = wm0 + mt * 16 + g;
+    split_tf32(As[t][m], ah[mt][0], al[mt][0]);
+    split_tf32(As[t][m + 8], ah[mt][1], al[mt][1]);
+    split_tf32(As[t + 4][m], ah[mt][2], al[mt][2]);
+    split_tf32(As[t + 4][m + 8], ah[mt][3], al[mt][3]);
+  }
+#pragma unroll
+  for (int nt = 0; nt < 8; ++nt) {
+    const int n = wn0 + nt * 8 + g;
+    uint32_t bh0, bl0, bh1, bl1;
+    split_tf32(Bs[t][n], bh0, bl0);
+    split_tf32(Bs[t + 4][n], bh1, bl1);
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt) {
+      mma_tf32(acc[mt][nt], al[mt], bh0, bh1);
+      mma_tf32(acc[mt][nt], ah[mt], bl0, bl1);
+      mma_tf32(acc[mt][nt], ah[mt], bh0, bh1);
+    }
+  }
+}
+
+// TB: B1 and B2 are read transposed (B[k][n] = Bt[n][k], ldb = row pitch of Bt).
+template <class TA1, class TA2, class TO, bool TB = false>
+__global__ void __launch_bounds__(256, 2) k_gemm2_tc(int64_t M, int N, int Np, int K1, int K2,
+                                                  const TA1* __restrict__ A1, int64_t lda1,
+                                                  const int32_t* __restrict__ gidx, int64_t m1,
+                                                  const TA2* __restrict__ A2, int64_t lda2,
+                                                  const float* __restrict__ B1, int64_t ldb1,
+                                                  const float* __restrict__ B2, int64_t ldb2,
+                                                  const float* __restrict__ bias, int relu,
+                                                  TO* __restrict__ Cm, int64_t ldc) {
+  __shared__ __align__(16) float As[GB_K][GB_P];
+  __shared__ __align__(16) float Bs[GB_K][GB_P];
+  const int tid = threadIdx.x, warp = tid >> 5;
+  const int wm0 = (warp >> 1) * 32, wn0 = (warp & 1) * 64;
+  const int64_t m0 = (int64_t)blockIdx.x * GB_M;
+  const int n0 = blockIdx.y * GB_N;
+  float acc[2][8][4];
+#pragma unroll
+  for (int i = 0; i < 2; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+#pragma unroll
+      for (int c = 0; c < 4; ++c) acc[i][j][c] = 0.f;
+  const int nk1 = (K1 + GB_K - 1) / GB_K, nk2 = (K2 + GB_K - 1) / GB_K;
+  // A loads: row ar = tid / 2, k ak .. ak + 3 (ak = 0 or 4); gathered row index read once
+  const int ar = tid >> 1, ak = (tid & 1) * 4;
+  const int64_t r = m0 + ar;
+  int64_t rr1 = -1;
+  if (r < M && r < m1) rr1 = gidx ? (int64_t)gidx[r] : r;
+  // B loads: plain: k bk = tid / 32, n bn .. bn + 3; transposed: n = tid / 2, k ak .. ak + 3
+  const int bk = tid >> 5, bn = (tid & 31) * 4;
+  float ra[4], rb[4];
+  auto load = [&](int kt) {
+    const bool first = kt < nk1;
+    const int k0 = first ? kt * GB_K : (kt - nk1) * GB_K;
+    const int K = first ? K1 : K2;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int k = k0 + ak + q;
+      float v = 0.f;
+      if (k < K) {
+        if (first) {
+          if (rr1 >= 0) v = ld1<TA1>(A1 + rr1 * lda1 + k);
+        } else if (r < M) {
+          v = ld1<TA2>(A2 + r * lda2 + k);
+        }
+      }
+      ra[q] = v;
+    }
+    const float* B = first ? B1 : B2;
+    const int64_t ldb = first ? ldb1 : ldb2;
+    if (TB) {
+      const int nn = n0 + ar;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int k = k0 + ak + q;
+        rb[q] = (k < K && nn < N) ? __ldg(B + (int64_t)nn * ldb + k) : 0.f;
+      }
+    } else {
+      const int k = k0 + bk;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int nn = n0 + bn + q;
+        rb[q] = (k < K && nn < N) ? __ldg(B + (int64_t)k * ldb + nn) : 0.f;
+      }
+    }
+  };
+  const int nkt = nk1 + nk2;
+  if (nkt > 0) load(0);
+  for (int kt = 0; kt < nkt; ++kt) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) As[ak + q][ar] = ra[q];
+    if (TB) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) Bs[ak + q][ar] = rb[q];
+    } else {
+      *reinterpret_cast<float4*>(&Bs[bk][bn]) = make_float4(rb[0], rb[1], rb[2], rb[3]);
+    }
+    __syncthreads();
+    if (kt + 1 < nkt) load(kt + 1);              // global loads in flight during the MMAs
+    warp_mma_k8(As, Bs, wm0, wn0, acc);
+    __syncthreads();
+  }
+  const int lane = tid & 31, g = lane >> 2, t = lane & 3;
+#pragma unroll
+  for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+    for (int hh = 0; hh < 2; ++hh) {
+      const int64_t row = m0 + wm0 + mt * 16 + g + 8 * hh;
+      if (row >= M) continue;
+#pragma unroll
+      for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+        for (int cc = 0; cc < 2; ++cc) {
+          const int nn = n0 + wn0 + nt * 8 + 2 * t + cc;
+          if (nn >= Np) continue;
+          float v = 0.f;
+          if (nn < N) {
+            v = acc[mt][nt][2 * hh + cc] + (bias ? bias[nn] : 0.f);
+            if (relu) v = fmaxf(v, 0.f);
+          }
+          st1<TO>(Cm + row * ldc + nn, v);
+        }
+    }
+}
+
 // ------------------------------------------------------------------ backward pieces
 template <class TH>
 __global__ void k_dz_mask(float* __restrict__ dz, int64_t ldz, const TH* __restrict__ h, int64_t ldh,
@@ -757,7 +918,7 @@ static buffalo_status pool_fwd_t(const PoolArgs& a, cudaStream_t s) {
   const int32_t* gidx = a.layer1 ? blk->src_global : nullptr;
   if (ns > 0) {   // P = ReLU(H W_pool^T + b_pool)
     dim3 grid((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2<TI, float, float, true><<<grid, 256, 0, s>>>(ns, a.d_in, dp, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
+    k_gemm2_tc<TI, float, float, true><<<grid, 256, 0, s>>>(ns, a.d_in, dp, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
                                                         gidx, ns, nullptr, 0, a.W_pool, a.d_in, nullptr, 0,
                                                         a.b_pool, 1, a.P, a.ld_pool);
     BF_LAUNCHED("k_gemm2");
@@ -773,7 +934,7 @@ static buffalo_status pool_fwd_t(const PoolArgs& a, cudaStream_t s) {
   const int Np = (int)pitch_of(a.d_out);
   dim3 grid((unsigned)ceil_div(nd, GB_M), (unsigned)ceil_div(Np, GB_N));
   const float* Wt = a.W_packed;   // [2 d_in][d_out]
-  k_gemm2<TI, float, float><<<grid, 256, 0, s>>>(nd, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
+  k_gemm2_tc<TI, float, float><<<grid, 256, 0, s>>>(nd, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
                                                 gidx, nd, a.agg, a.ld_agg, Wt, a.d_out,
                                                 Wt + (int64_t)a.d_in * a.d_out, a.d_out, a.b, !a.last, a.out,
                                                 a.ld_out);
@@ -815,7 +976,7 @@ static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
     BF_LAUNCHED("k_reduce_partials");
     // dh_agg = dZ W_neigh  (B[k][n] = W[k][d_in + n])
     dim3 gg((unsigned)ceil_div(n, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2<float, float, float><<<gg, 256, 0, s>>>(n, d_in, dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
+    k_gemm2_tc<float, float, float><<<gg, 256, 0, s>>>(n, d_in, dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
                                                    a.W + d_in, 2 * d_in, nullptr, 0, nullptr, 0, dagg, dp);
     BF_LAUNCHED("k_gemm2");
   }
@@ -838,7 +999,7 @@ static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
   BF_LAUNCHED("k_reduce_partials");
   if (a.dh_src) {   // dH_{l-1} = pad(dZ W_self) + dQ W_pool
     dim3 gg((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2<float, float, float><<<gg, 256, 0, s>>>(ns, d_in, dp, d_out, d_in, a.dh, a.ld_dh, nullptr, n, dq, dp,
+    k_gemm2_tc<float, float, float><<<gg, 256, 0, s>>>(ns, d_in, dp, d_out, d_in, a.dh, a.ld_dh, nullptr, n, dq, dp,
                                                    a.W, 2 * d_in, a.W_pool, d_in, nullptr, 0, a.dh_src,
                                                    a.ld_dh_src);
     BF_LAUNCHED("k_gemm2");
@@ -1104,7 +1265,7 @@ static buffalo_status lstm_fwd_t(const LstmArgs& a, cudaStream_t st) {
     BF_LAUNCHED("k_lstm_gix");
     dim3 grid((unsigned)ceil_div(c_t, GB_M), (unsigned)ceil_div(ldg, GB_N));
     const ProfSlot ps = prof_begin_launch("lstm_gates", st);
-    k_gemm2<TI, float, float, true><<<grid, 256, 0, st>>>(c_t, 4 * d, (int)ldg, d, t ? d : 0, (const TI*)a.h_src,
+    k_gemm2_tc<TI, float, float, true><<<grid, 256, 0, st>>>(c_t, 4 * d, (int)ldg, d, t ? d : 0, (const TI*)a.h_src,
                                                          a.ld_src, v.gix + off[t], c_t, v.Hs + s[t] * dp, dp,
                                                          a.W_ih, d, a.W_hh, d, a.b_lstm, 0, v.G + off[t] * ldg, ldg);
     BF_LAUNCHED("k_gemm2");
@@ -1120,7 +1281,7 @@ static buffalo_status lstm_fwd_t(const LstmArgs& a, cudaStream_t st) {
   const int Np = (int)pitch_of(a.d_out);
   dim3 grid((unsigned)ceil_div(n, GB_M), (unsigned)ceil_div(Np, GB_N));
   const float* Wt = a.W_packed;   // [2 d_in][d_out]
-  k_gemm2<TI, float, float><<<grid, 256, 0, st>>>(n, a.d_out, Np, d, d, (const TI*)a.h_src, a.ld_src,
+  k_gemm2_tc<TI, float, float><<<grid, 256, 0, st>>>(n, a.d_out, Np, d, d, (const TI*)a.h_src, a.ld_src,
                                                  a.layer1 ? blk->src_global : nullptr, n, a.agg, a.ld_agg, Wt,
                                                  a.d_out, Wt + (int64_t)d * a.d_out, a.d_out, a.b, !a.last, a.out,
                                                  a.ld_out);
@@ -1164,7 +1325,7 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
     k_reduce_partials<<<1, 256, 0, st>>>(db_part, S, d_out, a.db);
     BF_LAUNCHED("k_reduce_partials");
     dim3 gg((unsigned)ceil_div(n, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2<float, float, float><<<gg, 256, 0, st>>>(n, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
+    k_gemm2_tc<float, float, float><<<gg, 256, 0, st>>>(n, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
                                                     a.W + d, 2 * d, nullptr, 0, nullptr, 0, dagg, dp);
     BF_LAUNCHED("k_gemm2");
     k_lstm_bwd_init<<<grid_for(n * dp, 256), 256, 0, st>>>(blk->cls_perm, dagg, n, dp, v.Hs, v.Cst);
@@ -1180,7 +1341,7 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
     BF_LAUNCHED("k_lstm_cell_bwd");
     if (t > 0) {   // dh_{t-1} = dG_t W_hh into the running rows' state
       dim3 gg((unsigned)ceil_div(c_t, GB_M), (unsigned)ceil_div(dp, GB_N));
-      k_gemm2<float, float, float><<<gg, 256, 0, st>>>(c_t, d, (int)dp, 4 * d, 0, v.G + off[t] * ldg, ldg, nullptr, c_t,
+      k_gemm2_tc<float, float, float><<<gg, 256, 0, st>>>(c_t, d, (int)dp, 4 * d, 0, v.G + off[t] * ldg, ldg, nullptr, c_t,
                                                       nullptr, 0, a.W_hh, d, nullptr, 0, nullptr, 0, v.Hs + s[t] * dp,
                                                       dp);
       BF_LAUNCHED("k_gemm2");
@@ -1204,12 +1365,12 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
   }
   if (a.dh_src && ns > 0) {   // dH_{l-1} = pad(dZ W_self) + sum over edges of dG W_ih
     dim3 gg((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2<float, float, float><<<gg, 256, 0, st>>>(ns, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
+    k_gemm2_tc<float, float, float><<<gg, 256, 0, st>>>(ns, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
                                                     a.W, 2 * d, nullptr, 0, nullptr, 0, a.dh_src, a.ld_dh_src);
     BF_LAUNCHED("k_gemm2");
     if (e > 0) {
       dim3 gx((unsigned)ceil_div(e, GB_M), (unsigned)ceil_div(dp, GB_N));
-      k_gemm2<float, float, float><<<gx, 256, 0, st>>>(e, d, (int)dp, 4 * d, 0, v.G, ldg, nullptr, e, nullptr, 0,
+      k_gemm2_tc<float, float, float><<<gx, 256, 0, st>>>(e, d, (int)dp, 4 * d, 0, v.G, ldg, nullptr, e, nullptr, 0,
                                                       a.W_ih, d, nullptr, 0, nullptr, 0, dX, dp);
       BF_LAUNCHED("k_gemm2");
       k_lstm_scatterT<<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(blk->t_row_ptr, blk->t_col, blk->row_ptr,
@@ -1456,7 +1617,7 @@ static buffalo_status gat_fwd_t(const GatArgs& a, cudaStream_t st) {
   GatSaved v = gat_saved_view(a.saved, ns, nd, e, dl);
   if (ns > 0) {
     dim3 grid((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(ldz, GB_N));
-    k_gemm2<TI, float, float, true><<<grid, 256, 0, st>>>(ns, dl, (int)ldz, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
+    k_gemm2_tc<TI, float, float, true><<<grid, 256, 0, st>>>(ns, dl, (int)ldz, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
                                                          a.layer1 ? blk->src_global : nullptr, ns, nullptr, 0, a.W,
                                                          a.d_in, nullptr, 0, nullptr, 0, v.Z, ldz);
     BF_LAUNCHED("k_gemm2");
@@ -1543,7 +1704,7 @@ static buffalo_status gat_bwd_t(const GatArgs& a, cudaStream_t st) {
   if (a.dh_src) {   // dH_{l-1} = dZ W
     const int64_t dpi = pitch_of(d_in);
     dim3 gg((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dpi, GB_N));
-    k_gemm2<float, float, float><<<gg, 256, 0, st>>>(ns, d_in, (int)dpi, dl, 0, dZ, ldz, nullptr, ns, nullptr, 0, a.W,
+    k_gemm2_tc<float, float, float><<<gg, 256, 0, st>>>(ns, d_in, (int)dpi, dl, 0, dZ, ldz, nullptr, ns, nullptr, 0, a.W,
                                                     d_in, nullptr, 0, nullptr, 0, a.dh_src, a.ld_dh_src);
     BF_LAUNCHED("k_gemm2");
   }
