@@ -113,11 +113,15 @@ __global__ void k_reset_map(const int32_t* __restrict__ src, int64_t n, int32_t*
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
     node_map[src[j]] = INT32_MAX;
 }
+// mapped (nullable): node_map[u] per edge, kept for k_col_local (a coalesced re-read instead of a
+// second random node-map lookup).
 __global__ void k_mark_bits(const int32_t* __restrict__ colg, int64_t e, const int32_t* __restrict__ node_map,
-                            uint32_t* __restrict__ bits) {
+                            uint32_t* __restrict__ bits, int32_t* __restrict__ mapped) {
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x) {
     const int32_t u = colg[k];
-    if (node_map[u] != INT32_MAX) continue;                      // a dst: keeps its prefix id
+    const int32_t m = node_map[u];
+    if (mapped) mapped[k] = m;
+    if (m != INT32_MAX) continue;                                // a dst: keeps its prefix id
     const uint32_t b = 1u << (u & 31);
     if (!(bits[u >> 5] & b)) atomicOr(&bits[u >> 5], b);
   }
@@ -145,13 +149,14 @@ __global__ void k_emit_bits(const uint32_t* __restrict__ bits, const int32_t* __
     }
   }
 }
-// col_local of every edge; tcnt (layers >= 2, zeroed): transposed row lengths counted on the way.
+// col_local of every edge (holding node_map[u] from k_mark_bits on entry); tcnt (layers >= 2,
+// zeroed): transposed row lengths counted on the way.
 __global__ void k_col_local(const int32_t* __restrict__ colg, int64_t e, const int32_t* __restrict__ node_map,
                             const uint32_t* __restrict__ bits, const int32_t* __restrict__ prefix, int32_t n_dst,
                             int32_t* __restrict__ col_local, int32_t* __restrict__ tcnt) {
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x) {
     const int32_t u = colg[k];
-    const int32_t m = node_map[u];
+    const int32_t m = col_local[k];                              // node_map[u], kept by k_mark_bits
     const int32_t c = m != INT32_MAX ? m : n_dst + prefix[u >> 5] + __popc(bits[u >> 5] & ((1u << (u & 31)) - 1u));
     col_local[k] = c;
     if (tcnt) atomicAdd(&tcnt[c], 1);
@@ -388,7 +393,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     BF_LAUNCHED("k_set_map");
   }
   if (e > 0) {
-    k_mark_bits<<<grid_for(e, 256), 256, 0, s>>>(colg, e, g->node_map, gw.bits);
+    k_mark_bits<<<grid_for(e, 256), 256, 0, s>>>(colg, e, g->node_map, gw.bits, col_local);
     BF_LAUNCHED("k_mark_bits");
   }
   int64_t n_src = 0;
