@@ -66,6 +66,14 @@ typedef struct {
   int32_t fanout[BUFFALO_MAX_LAYERS];
   int32_t cutoff_F;
   uint64_t seed;
+  /* Optional sample cache (all NULL: none).  cache[l-1] (for fanout[l-1] > 0, else ignored):
+   * device int32 [num_nodes][fanout[l-1]], caller-owned.  buffalo_bucketize writes into it the
+   * sampled neighbour list (ascending CSR position) of every node its first statistics pass
+   * visits at block l — the whole receptive field of the seed batch — and buffalo_build_blocks
+   * copies the rows from it instead of sampling again.  Contract: the cache was filled by
+   * buffalo_bucketize on the same graph with a sampler of the same seed and fanouts, and the
+   * groups built are groups of that batch; otherwise pass NULLs. */
+  int32_t* cache[BUFFALO_MAX_LAYERS];
 } buffalo_sampler;
 
 /* GraphSAGE-mean model (R20): dim[0] = input feature width, dim[L] = #classes.

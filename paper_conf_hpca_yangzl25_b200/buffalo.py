@@ -51,7 +51,8 @@ class Graph(ctypes.Structure):
 
 
 class Sampler(ctypes.Structure):
-    _fields_ = [("num_layers", c_i32), ("fanout", c_i32 * MAX_LAYERS), ("cutoff_F", c_i32), ("seed", c_u64)]
+    _fields_ = [("num_layers", c_i32), ("fanout", c_i32 * MAX_LAYERS), ("cutoff_F", c_i32), ("seed", c_u64),
+                ("cache", c_p * MAX_LAYERS)]
 
 
 class Model(ctypes.Structure):
@@ -334,8 +335,12 @@ def profile_end():
 
 
 # ------------------------------------------------------------------------- struct helpers
-def make_sampler(fanout, F, seed):
+def make_sampler(fanout, F, seed, cache=None):
+    """cache: None or a list of per-block int32 CUDA tensors [num_nodes * fanout] (None entries
+    allowed), the optional sample cache of include/buffalo.h."""
     s = Sampler()
+    for i, c in enumerate(cache or []):
+        s.cache[i] = ptr(c) if c is not None else None
     s.num_layers = len(fanout)
     for i, f in enumerate(fanout):
         s.fanout[i] = int(f)

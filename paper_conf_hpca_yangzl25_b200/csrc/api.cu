@@ -414,7 +414,10 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
     bucket_item[d] = Item{d, 0, bstart[d], plan->hist_h[d], 0, 0, 0, 0, 0};
     if (plan->hist_h[d] > 0) todo.push_back(&bucket_item[d]);
   }
+  // the first statistics pass (every seed) also fills the sample cache; later passes do not
   BF_CHECK(items_stats(g, sorted_ids, todo, sp, m, stats_ws, stats_bytes, masks_clean, s));
+  buffalo_sampler sp_nc = *sp;
+  for (int l = 0; l < BUFFALO_MAX_LAYERS; ++l) sp_nc.cache[l] = nullptr;
   std::vector<int> non_split;
   int64_t sum_M_all = 0, sum_w = 0, max_w = 0;
   for (int d = 0; d <= F; ++d) {
@@ -469,7 +472,7 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
           }
           for (int K2 : ks)
             for (Item& it : piece_cache[K2]) ptrs.push_back(&it);
-          BF_CHECK(items_stats(g, sorted_ids, ptrs, sp, m, stats_ws, stats_bytes, masks_clean, s));
+          BF_CHECK(items_stats(g, sorted_ids, ptrs, &sp_nc, m, stats_ws, stats_bytes, masks_clean, s));
         }
         for (Item it : piece_cache[K]) {
           it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
@@ -556,7 +559,8 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
           ct[k] = offs[k0 + k + 1] - offs[k0 + k];
         }
         static thread_local int64_t nh[kStatsBatch][BUFFALO_MAX_LAYERS + 1], eh[kStatsBatch][BUFFALO_MAX_LAYERS];
-        BF_CHECK(mask_stats(g, plan->group_seeds, st, ct, nit, sp, L, stats_ws, stats_bytes, masks_clean, nh, eh, s));
+        BF_CHECK(mask_stats(g, plan->group_seeds, st, ct, nit, &sp_nc, L, stats_ws, stats_bytes, masks_clean, nh, eh,
+                            s));
         masks_clean = true;
         for (int k = 0; k < nit; ++k) {
           int64_t* row = plan->group_sizes_h + (int64_t)(k0 + k) * W;
@@ -630,7 +634,8 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
     }
     buffalo_status st = build_layer(g, dst, nd, sp->fanout[l - 1], (uint32_t)(L - l + 1), sp->seed, l,
                                     false, A, b, s, sizes_h ? known : nullptr,
-                                    m->aggregator == BUFFALO_AGG_POOL || m->aggregator == BUFFALO_AGG_GAT);
+                                    m->aggregator == BUFFALO_AGG_POOL || m->aggregator == BUFFALO_AGG_GAT,
+                                    sp->fanout[l - 1] > 0 ? sp->cache[l - 1] : nullptr);
     if (st == BUFFALO_ERR_CAPACITY || A.overflow) {
       if (required_bytes_h) *required_bytes_h = A.need;
       set_error("build_blocks: arena of %lld bytes too small (need >= %lld)", (long long)A.cap,

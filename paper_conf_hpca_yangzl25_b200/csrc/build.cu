@@ -89,6 +89,24 @@ __global__ void __launch_bounds__(256) k_sample_fill(const int32_t* __restrict__
     });
 }
 
+// Rows from the sample cache (filled by the scheduler's statistics pass): SEG lanes per row,
+// lane k copies entry k of the row's cached list (D = min(deg, f) entries, CSR order).
+template <int SEG>
+__global__ void __launch_bounds__(256) k_cache_fill(const int32_t* __restrict__ dst, int64_t n,
+                                                    const int32_t* __restrict__ cache, int32_t f,
+                                                    const int32_t* __restrict__ row_ptr, int32_t* __restrict__ out,
+                                                    int64_t cap) {
+  constexpr int G = 32 / SEG;
+  const int lane = threadIdx.x & 31, g = lane / SEG, sl = lane % SEG;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n; w += warps) {
+    const int64_t slot = w * G + g;
+    if (slot >= n) continue;
+    const int32_t b = row_ptr[slot], D = row_ptr[slot + 1] - b;
+    if (sl < D && b + sl < cap) out[b + sl] = cache[(int64_t)dst[slot] * f + sl];
+  }
+}
+
 static inline int sample_seg(int32_t f) { return (f > 0 && f <= 8) ? 8 : (f > 0 && f <= 16) ? 16 : 32; }
 
 template <class... Args>
@@ -327,7 +345,8 @@ int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only, 
 
 buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
                            uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
-                           buffalo_block* blk, cudaStream_t s, const int64_t* known, bool t1) {
+                           buffalo_block* blk, cudaStream_t s, const int64_t* known, bool t1,
+                           const int32_t* cache) {
   memset(blk, 0, sizeof(*blk));
   blk->n_dst = n_dst;
   int32_t* rp = (int32_t*)A.take(4 * (n_dst + 1));
@@ -381,7 +400,14 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     // degree classes of the dst rows: stable counting sort by min(D, kHeavyT + 1)
     BF_CHECK(stable_partition(DegClass{rp}, EmitPerm{perm}, n_dst, counts, ws, s));
   }
-  if (n_dst > 0) {
+  if (n_dst > 0 && cache && f > 0) {                             // rows sampled by the scheduler
+    const int seg = sample_seg(f), G = 32 / seg;
+    const int grid = grid_for(ceil_div(n_dst, G) * 32, 256, 16);
+    if (seg == 8) k_cache_fill<8><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e);
+    else if (seg == 16) k_cache_fill<16><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e);
+    else k_cache_fill<32><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e);
+    BF_LAUNCHED("k_cache_fill");
+  } else if (n_dst > 0) {
     launch_sample_fill(sample_seg(f), n_dst, s, dst, n_dst, g->row_ptr, g->col, f, hop, seed, (const int32_t*)rp,
                        colg, e);
     BF_LAUNCHED("k_sample_fill");
@@ -627,7 +653,8 @@ __global__ void __launch_bounds__(256, (W >= 4 ? 4 : 6)) k_mask_layer(const int3
                                                     unsigned long long* __restrict__ m_out, uint32_t* __restrict__ bits,
                                                     const int64_t* __restrict__ grow, const int32_t* __restrict__ gcol,
                                                     int32_t f, uint32_t hop, uint64_t seed,
-                                                    unsigned long long* __restrict__ gn, unsigned long long* __restrict__ ge) {
+                                                    unsigned long long* __restrict__ gn, unsigned long long* __restrict__ ge,
+                                                    int32_t* __restrict__ cache) {
   constexpr int G = 32 / SEG;
   __shared__ unsigned long long sn[64 * W], se[64 * W];
   for (int k = threadIdx.x; k < 64 * W; k += blockDim.x) { sn[k] = 0; se[k] = 0; }
@@ -659,7 +686,8 @@ __global__ void __launch_bounds__(256, (W >= 4 ? 4 : 6)) k_mask_layer(const int3
       }
     }
     if (slot < n_act && (lane % SEG) == 0) mask_or<W>(m_out, bits, v, mask);
-    sample_warp_rows<SEG>(w, n_act, DstRows{act}, grow, gcol, f, hop, seed, [&](int64_t s_, int32_t, int32_t u) {
+    sample_warp_rows<SEG>(w, n_act, DstRows{act}, grow, gcol, f, hop, seed, [&](int64_t s_, int32_t k, int32_t u) {
+      if (cache) cache[(int64_t)act[s_] * f + k] = u;           // sample cache for the build (f > 0)
       unsigned long long ms[W];
 #pragma unroll
       for (int q = 0; q < W; ++q) ms[q] = m_in[(int64_t)act[s_] * W + q];
@@ -734,18 +762,19 @@ static buffalo_status mask_stats_w(const buffalo_graph* g, const int32_t* sorted
     int32_t na = 0;
     if (n_act > 0) {
       const int32_t fl = sp->fanout[l - 1];
+      int32_t* cache = fl > 0 ? sp->cache[l - 1] : nullptr;
       const int seg = sample_seg(fl);
       const int grid = grid_for(ceil_div(n_act, 32 / seg) * 32, 256, 16);
       const uint32_t hop = (uint32_t)(L - l + 1);
       if (seg == 8)
         k_mask_layer<8, W><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], gw.bits, g->row_ptr, g->col, fl,
-                                               hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1));
+                                               hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1), cache);
       else if (seg == 16)
         k_mask_layer<16, W><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], gw.bits, g->row_ptr, g->col, fl,
-                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1));
+                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1), cache);
       else
         k_mask_layer<32, W><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], gw.bits, g->row_ptr, g->col, fl,
-                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1));
+                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1), cache);
       BF_LAUNCHED("k_mask_layer");
       // masks of layer l are no longer needed: clear them for reuse by layer l-2
       k_mask_count<W><<<grid_for(n_act, 256), 256, 0, s>>>(act[cur], n_act, m[cur], nullptr);

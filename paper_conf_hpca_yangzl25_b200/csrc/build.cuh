@@ -44,7 +44,7 @@ inline GraphWs graph_ws(const buffalo_graph* g) {
 buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
                            uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
                            buffalo_block* blk, cudaStream_t s, const int64_t* known = nullptr,
-                           bool t1 = false);
+                           bool t1 = false, const int32_t* cache = nullptr);
 
 // Degree bucketing of the seeds (Alg. 3 l.1): bucket[i] = min(D(seed_i), F); order = seed
 // positions grouped by bucket (stable); sorted_ids = seeds[order]; hist_h[0..F].

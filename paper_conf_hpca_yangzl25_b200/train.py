@@ -152,7 +152,7 @@ class Trainer:
     def __init__(self, graph, feats, labels, seeds, dims, fanout, F, Ws, bs, feat_dtype=B.FP32,
                  gemm_mode=B.GEMM_FFMA, mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096,
                  base_seed=3, rank=0, world=1, process_group=None, device="cuda", aggregator=B.AGG_MEAN,
-                 Wps=None, bps=None, lstm=None, gat=None, pipeline=False):
+                 Wps=None, bps=None, lstm=None, gat=None, pipeline=False, sample_cache=True):
         self.graph = graph if isinstance(graph, DeviceGraph) else DeviceGraph(*graph, device=device)
         self.feats = feats
         self.labels = labels
@@ -188,6 +188,12 @@ class Trainer:
         if pipeline:
             self._pb.append(PlanBuffers(self.S, k_max, F, self.L, device))
             self._side = torch.cuda.Stream(device=device)
+        # sample cache per plan-buffer set (include/buffalo.h): the scheduler's first statistics
+        # pass stores every sampled neighbour list of the batch, the build copies them
+        N = self.graph.N
+        self._cache = [[torch.empty(N * f, dtype=torch.int32, device=device) if (sample_cache and f > 0) else None
+                        for f in self.fanout] for _ in self._pb]
+        self._cache_epoch = [None] * len(self._pb)
         sampler = B.make_sampler(self.fanout, F, base_seed)
         wsb = B.bucketize_workspace_bytes(self.graph.g, self.S, sampler, self.model)
         self.bucket_ws = torch.empty(wsb, dtype=torch.uint8, device=device)
@@ -209,7 +215,10 @@ class Trainer:
 
     # --------------------------------------------------------------- pieces of Alg. 2
     def sampler(self, epoch):
-        return B.make_sampler(self.fanout, self.F, self.base_seed + epoch)
+        """The sampler of `epoch`; it carries the current buffer set's sample cache when that
+        cache was filled by the scheduler for this epoch."""
+        cache = self._cache[self._cur] if self._cache_epoch[self._cur] == epoch else None
+        return B.make_sampler(self.fanout, self.F, self.base_seed + epoch, cache)
 
     def schedule(self, epoch):
         """Alg. 3 for `epoch` into the current plan buffers (stream-ordered on the current stream)."""
@@ -218,7 +227,10 @@ class Trainer:
 
     def _schedule_into(self, buf, epoch, g):
         pb = self._pb[buf]
-        B.bucketize(g, self.seeds, self.sampler(epoch), self.model, self.sched, pb.plan, self.bucket_ws)
+        self._cache_epoch[buf] = None
+        sp = B.make_sampler(self.fanout, self.F, self.base_seed + epoch, self._cache[buf])
+        B.bucketize(g, self.seeds, sp, self.model, self.sched, pb.plan, self.bucket_ws)
+        self._cache_epoch[buf] = epoch
         K = pb.plan.k_out
         return K, pb.offs_h[:K + 1].copy(), pb.est_h[:K].copy(), pb.rank_h[:K].copy()
 
