@@ -202,9 +202,11 @@ constexpr int kStatsBatch = 256;       // items per statistics pass (mask_stats)
 
 // Item statistics (R13, R15): exact layer sizes of up to 256 items per pass (mask_stats), then
 // O = #seeds, E = e_L, I = n_{L-1} and M_est = hi of the memory model.
+// cache_mode (the sampler's sample cache, when it has one): 1 = sample and store, 2 = read the
+// rows stored by an earlier pass of the same call.
 static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_ids, std::vector<Item*>& items,
                                   const buffalo_sampler* sp, const buffalo_model* m, char* ws, int64_t ws_bytes,
-                                  bool& masks_clean, cudaStream_t s) {
+                                  bool& masks_clean, cudaStream_t s, int cache_mode) {
   const int L = m->num_layers;
   for (size_t b0 = 0; b0 < items.size(); b0 += kStatsBatch) {
     const int nit = (int)std::min<size_t>(kStatsBatch, items.size() - b0);
@@ -214,7 +216,7 @@ static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_
       counts[k] = items[b0 + k]->count;
     }
     static thread_local int64_t nh[kStatsBatch][BUFFALO_MAX_LAYERS + 1], eh[kStatsBatch][BUFFALO_MAX_LAYERS];
-    BF_CHECK(mask_stats(g, sorted_ids, starts, counts, nit, sp, L, ws, ws_bytes, masks_clean, nh, eh, s));
+    BF_CHECK(mask_stats(g, sorted_ids, starts, counts, nit, sp, L, ws, ws_bytes, masks_clean, nh, eh, s, cache_mode));
     masks_clean = true;
     for (int k = 0; k < nit; ++k) {
       Item& it = *items[b0 + k];
@@ -414,10 +416,8 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
     bucket_item[d] = Item{d, 0, bstart[d], plan->hist_h[d], 0, 0, 0, 0, 0};
     if (plan->hist_h[d] > 0) todo.push_back(&bucket_item[d]);
   }
-  // the first statistics pass (every seed) also fills the sample cache; later passes do not
-  BF_CHECK(items_stats(g, sorted_ids, todo, sp, m, stats_ws, stats_bytes, masks_clean, s));
-  buffalo_sampler sp_nc = *sp;
-  for (int l = 0; l < BUFFALO_MAX_LAYERS; ++l) sp_nc.cache[l] = nullptr;
+  // the first statistics pass (every seed) fills the sample cache; later passes read it
+  BF_CHECK(items_stats(g, sorted_ids, todo, sp, m, stats_ws, stats_bytes, masks_clean, s, 1));
   std::vector<int> non_split;
   int64_t sum_M_all = 0, sum_w = 0, max_w = 0;
   for (int d = 0; d <= F; ++d) {
@@ -472,7 +472,7 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
           }
           for (int K2 : ks)
             for (Item& it : piece_cache[K2]) ptrs.push_back(&it);
-          BF_CHECK(items_stats(g, sorted_ids, ptrs, &sp_nc, m, stats_ws, stats_bytes, masks_clean, s));
+          BF_CHECK(items_stats(g, sorted_ids, ptrs, sp, m, stats_ws, stats_bytes, masks_clean, s, 2));
         }
         for (Item it : piece_cache[K]) {
           it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
@@ -559,8 +559,8 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
           ct[k] = offs[k0 + k + 1] - offs[k0 + k];
         }
         static thread_local int64_t nh[kStatsBatch][BUFFALO_MAX_LAYERS + 1], eh[kStatsBatch][BUFFALO_MAX_LAYERS];
-        BF_CHECK(mask_stats(g, plan->group_seeds, st, ct, nit, &sp_nc, L, stats_ws, stats_bytes, masks_clean, nh, eh,
-                            s));
+        BF_CHECK(mask_stats(g, plan->group_seeds, st, ct, nit, sp, L, stats_ws, stats_bytes, masks_clean, nh, eh, s,
+                            2));
         masks_clean = true;
         for (int k = 0; k < nit; ++k) {
           int64_t* row = plan->group_sizes_h + (int64_t)(k0 + k) * W;

@@ -654,7 +654,7 @@ __global__ void __launch_bounds__(256, (W >= 4 ? 4 : 6)) k_mask_layer(const int3
                                                     const int64_t* __restrict__ grow, const int32_t* __restrict__ gcol,
                                                     int32_t f, uint32_t hop, uint64_t seed,
                                                     unsigned long long* __restrict__ gn, unsigned long long* __restrict__ ge,
-                                                    int32_t* __restrict__ cache) {
+                                                    int32_t* __restrict__ cache, int cache_read) {
   constexpr int G = 32 / SEG;
   __shared__ unsigned long long sn[64 * W], se[64 * W];
   for (int k = threadIdx.x; k < 64 * W; k += blockDim.x) { sn[k] = 0; se[k] = 0; }
@@ -686,13 +686,20 @@ __global__ void __launch_bounds__(256, (W >= 4 ? 4 : 6)) k_mask_layer(const int3
       }
     }
     if (slot < n_act && (lane % SEG) == 0) mask_or<W>(m_out, bits, v, mask);
-    sample_warp_rows<SEG>(w, n_act, DstRows{act}, grow, gcol, f, hop, seed, [&](int64_t s_, int32_t k, int32_t u) {
-      if (cache) cache[(int64_t)act[s_] * f + k] = u;           // sample cache for the build (f > 0)
-      unsigned long long ms[W];
+    if (cache_read) {                                            // rows cached by the first pass
+      if (slot < n_act && (lane % SEG) < D) {
+        const int32_t u = cache[(int64_t)v * f + (lane % SEG)];
+        mask_or<W>(m_out, bits, u, mask);
+      }
+    } else {
+      sample_warp_rows<SEG>(w, n_act, DstRows{act}, grow, gcol, f, hop, seed, [&](int64_t s_, int32_t k, int32_t u) {
+        if (cache) cache[(int64_t)act[s_] * f + k] = u;         // sample cache for the build (f > 0)
+        unsigned long long ms[W];
 #pragma unroll
-      for (int q = 0; q < W; ++q) ms[q] = m_in[(int64_t)act[s_] * W + q];
-      mask_or<W>(m_out, bits, u, ms);
-    });
+        for (int q = 0; q < W; ++q) ms[q] = m_in[(int64_t)act[s_] * W + q];
+        mask_or<W>(m_out, bits, u, ms);
+      });
+    }
   }
   flush_item_counters<W>(cnt, gn, ge, sn, se);
 }
@@ -749,7 +756,7 @@ template <int W>
 static buffalo_status mask_stats_w(const buffalo_graph* g, const int32_t* sorted_ids, int64_t lo_pos, int64_t n_seed,
                                    const int64_t* se, int nitems, const buffalo_sampler* sp, int L,
                                    unsigned long long* const* m, int32_t* const* act, unsigned long long* accn,
-                                   unsigned long long* acce, cudaStream_t s) {
+                                   unsigned long long* acce, cudaStream_t s, int cache_mode) {
   const GraphWs gw = graph_ws(g);
   if (n_seed > 0) {
     k_mask_seed<W><<<grid_for(n_seed, 256), 256, 0, s>>>(sorted_ids, lo_pos, n_seed, se, nitems, m[0], act[0]);
@@ -762,19 +769,20 @@ static buffalo_status mask_stats_w(const buffalo_graph* g, const int32_t* sorted
     int32_t na = 0;
     if (n_act > 0) {
       const int32_t fl = sp->fanout[l - 1];
-      int32_t* cache = fl > 0 ? sp->cache[l - 1] : nullptr;
+      int32_t* cache = (fl > 0 && cache_mode > 0) ? sp->cache[l - 1] : nullptr;
+      const int cread = cache && cache_mode == 2;
       const int seg = sample_seg(fl);
       const int grid = grid_for(ceil_div(n_act, 32 / seg) * 32, 256, 16);
       const uint32_t hop = (uint32_t)(L - l + 1);
       if (seg == 8)
         k_mask_layer<8, W><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], gw.bits, g->row_ptr, g->col, fl,
-                                               hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1), cache);
+                                               hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1), cache, cread);
       else if (seg == 16)
         k_mask_layer<16, W><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], gw.bits, g->row_ptr, g->col, fl,
-                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1), cache);
+                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1), cache, cread);
       else
         k_mask_layer<32, W><<<grid, 256, 0, s>>>(act[cur], n_act, m[cur], m[cur ^ 1], gw.bits, g->row_ptr, g->col, fl,
-                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1), cache);
+                                                hop, sp->seed, accn + 64 * W * l, acce + 64 * W * (l - 1), cache, cread);
       BF_LAUNCHED("k_mask_layer");
       // masks of layer l are no longer needed: clear them for reuse by layer l-2
       k_mask_count<W><<<grid_for(n_act, 256), 256, 0, s>>>(act[cur], n_act, m[cur], nullptr);
@@ -801,7 +809,7 @@ buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, con
                           const int64_t* item_count_h, int nitems, const buffalo_sampler* sp, int L, char* ws,
                           int64_t ws_bytes,
                           bool masks_clean, int64_t (*n_h)[BUFFALO_MAX_LAYERS + 1],
-                          int64_t (*e_h)[BUFFALO_MAX_LAYERS], cudaStream_t s) {
+                          int64_t (*e_h)[BUFFALO_MAX_LAYERS], cudaStream_t s, int cache_mode) {
   const int64_t N = g->num_nodes;
   if (ws_bytes < mask_stats_bytes(N, L)) {
     set_error("bucketize workspace too small for the item statistics");
@@ -842,11 +850,11 @@ buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, con
   unsigned long long* accn = acc;
   unsigned long long* acce = acc + stride * (L + 1);
   if (W == 1)
-    BF_CHECK(mask_stats_w<1>(g, sorted_ids, lo_pos, n_seed, se, nitems, sp, L, m, act, accn, acce, s));
+    BF_CHECK(mask_stats_w<1>(g, sorted_ids, lo_pos, n_seed, se, nitems, sp, L, m, act, accn, acce, s, cache_mode));
   else if (W == 2)
-    BF_CHECK(mask_stats_w<2>(g, sorted_ids, lo_pos, n_seed, se, nitems, sp, L, m, act, accn, acce, s));
+    BF_CHECK(mask_stats_w<2>(g, sorted_ids, lo_pos, n_seed, se, nitems, sp, L, m, act, accn, acce, s, cache_mode));
   else
-    BF_CHECK(mask_stats_w<4>(g, sorted_ids, lo_pos, n_seed, se, nitems, sp, L, m, act, accn, acce, s));
+    BF_CHECK(mask_stats_w<4>(g, sorted_ids, lo_pos, n_seed, se, nitems, sp, L, m, act, accn, acce, s, cache_mode));
   static thread_local unsigned long long host[kMaskMaxItems * (2 * BUFFALO_MAX_LAYERS + 1)];
   BF_CUDA(cudaMemcpyAsync(host, acc, sizeof(unsigned long long) * stride * (2 * L + 1), cudaMemcpyDeviceToHost, s));
   BF_CUDA(cudaStreamSynchronize(s));

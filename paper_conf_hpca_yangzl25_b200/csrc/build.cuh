@@ -62,6 +62,6 @@ buffalo_status mask_stats(const buffalo_graph* g, const int32_t* sorted_ids, con
                           const int64_t* item_count_h, int nitems, const buffalo_sampler* sp, int L, char* ws,
                           int64_t ws_bytes,
                           bool masks_clean, int64_t (*n_h)[BUFFALO_MAX_LAYERS + 1],
-                          int64_t (*e_h)[BUFFALO_MAX_LAYERS], cudaStream_t s);
+                          int64_t (*e_h)[BUFFALO_MAX_LAYERS], cudaStream_t s, int cache_mode = 1);
 
 }  // namespace buffalo
