@@ -1165,11 +1165,22 @@ __global__ void k_reduce_dw(const float* __restrict__ part, int S, int d_out, in
   }
 }
 
-__global__ void k_reduce_db(const float* __restrict__ part, int S, int d, float* __restrict__ db) {
-  for (int c = threadIdx.x; c < d; c += blockDim.x) {
-    float s = 0.f;
-    for (int q = 0; q < S; ++q) s += part[(int64_t)q * d + c];
-    db[c] += s;
+// db += sum of the S partial rows: CTA per 32 columns, warp w sums partials w, w + 8, ... and the
+// eight warp sums are combined in warp order (fixed order: deterministic).
+__global__ void __launch_bounds__(256) k_reduce_db(const float* __restrict__ part, int S, int d,
+                                                   float* __restrict__ db) {
+  __shared__ float sh[8][33];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + lane;
+  float s = 0.f;
+  if (c < d)
+    for (int q = w; q < S; q += 8) s += part[(int64_t)q * d + c];
+  sh[w][lane] = s;
+  __syncthreads();
+  if (w == 0 && c < d) {
+    float t = 0.f;
+    for (int k = 0; k < 8; ++k) t += sh[k][lane];
+    db[c] += t;
   }
 }
 
@@ -1311,7 +1322,7 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   }
   k_reduce_dw<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, d_out, d_in, (int)Dp, a.dW);
   BF_LAUNCHED("k_reduce_dw");
-  k_reduce_db<<<1, 256, 0, s>>>(db_part, nparts, d_out, a.db);
+  k_reduce_db<<<(unsigned)ceil_div(d_out, 32), 256, 0, s>>>(db_part, nparts, d_out, a.db);
   BF_LAUNCHED("k_reduce_db");
   // dH_{l-1} = [dZ (rows < n_dst) || sum_{i in T(j)} dZ[i]/D(i)] [W_self; W_neigh], written in the
   // prepared form of layer l-1 by the GEMM epilogue (ReLU' with H_{l-1}, /D_{l-1}, db partials)
