@@ -400,69 +400,92 @@ def mem_balanced_grouping(items, K, M_ctr):
     return max(loads) <= M_ctr, groups, loads
 
 
-def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT64_MAX,
-             C_ppm=0, k_min=1, k_max=4096, num_gpus=1, aggregator="mean"):
-    """Alg. 3 Buffalo_Scheduler (PAPER.md:269-280, :333) with the readings of DESIGN.md
-    (R7 explosion test, R11 sort/placement keys, R16 K_max, R17 empty groups dropped,
-    R27 k_min = #GPUs and LPT rank assignment).  Returns a dict plan or None (budget)."""
-    seeds = np.asarray(seeds, dtype=np.int32)
-    f_L = fanout[L - 1]
-    D, bucket, order, hist = degree_bucketing(g, seeds, f_L, F)
-    pos_of = {d: np.nonzero(bucket == d)[0] for d in range(F + 1)}
-    stats = {}
-    for d in range(F + 1):
-        if pos_of[d].size:
-            st = item_stats(g, seeds[pos_of[d]], L, fanout, seed, dims, act_dtype, aggregator)
-            st["w"] = grouping_weight(st["M"], st["I"], st["E"], C_ppm)
-            stats[d] = st
+def _alg3_k_loop(stats, F, piece_stats, mem_budget, C_ppm, k_lo, k_max, fast_paths=True):
+    """The K loop of Alg. 3 with MemBalancedGrouping (Alg. 4) over the
+    per-bucket statistics `stats` {d: dict(M, I, E, O, w, ...)} (non-empty buckets only).
+    piece_stats(K) -> [(k, st), ...]: statistics of the K micro-buckets of bucket F (R8).
+    For K = k_lo .. k_max: explosion test (R7: K >= 2 and M_est[F] > sum_d M_est[d] / K) ->
+    split bucket F into K micro-buckets, else keep it whole; group (Alg. 4); the first K whose
+    every group estimate is <= M_ctr wins.
+    fast_paths (R25) skips a K without building micro-buckets when sum_{d != F} w_d > K*M_ctr
+    and stops at once when a never-split bucket alone exceeds M_ctr; both imply that the plain
+    loop (fast_paths=False) fails at that K too, so the result is identical (pinned by
+    tests/test_oracle_scheduler.py on random instances).
+    Returns (K, items, groups, loads, exploded) or None."""
     non_split = [d for d in stats if d != F]
     sum_M_all = sum(stats[d]["M"] for d in stats)
     max_w = max([stats[d]["w"] for d in non_split], default=0)
     sum_w = sum(stats[d]["w"] for d in non_split)
-    k_lo = max(k_min, num_gpus, 1)
     for K in range(k_lo, k_max + 1):
-        if max_w > mem_budget:
-            return None                      # a never-split bucket exceeds M_ctr for every K
-        if sum_w > K * mem_budget:
-            continue                         # some group must exceed M_ctr (weights >= 0)
-        items = [dict(d=d, k=0, pos=pos_of[d], **stats[d]) for d in non_split]
+        if fast_paths:
+            if max_w > mem_budget:
+                return None                  # a never-split bucket exceeds M_ctr for every K
+            if sum_w > K * mem_budget:
+                continue                     # some group must exceed M_ctr (weights >= 0)
+        items = [dict(d=d, k=0, **stats[d]) for d in non_split]
+        exploded = False
         if F in stats:
-            explosion = K >= 2 and stats[F]["M"] * K > sum_M_all
-            if explosion:
-                for k, piece in enumerate(split_explosion(pos_of[F], K)):
-                    if piece.size == 0:
-                        continue
-                    st = item_stats(g, seeds[piece], L, fanout, seed, dims, act_dtype, aggregator)
-                    st["w"] = grouping_weight(st["M"], st["I"], st["E"], C_ppm)
-                    items.append(dict(d=F, k=k, pos=piece, **st))
+            exploded = K >= 2 and stats[F]["M"] * K > sum_M_all          # R7
+            if exploded:
+                for k, st in piece_stats(K):
+                    items.append(dict(d=F, k=k, **st))
             else:
-                items.append(dict(d=F, k=0, pos=pos_of[F], **stats[F]))
+                items.append(dict(d=F, k=0, **stats[F]))
         ok, groups, loads = mem_balanced_grouping(items, K, mem_budget)
-        if not ok:
-            continue
-        kept = [(grp, ld) for grp, ld in zip(groups, loads) if grp]
-        offsets = [0]
-        group_seeds = []
-        group_of_seed = np.full(seeds.size, -1, dtype=np.int32)
-        for gi, (grp, _) in enumerate(kept):
-            for it in sorted(grp, key=lambda it: (it["d"], it["k"])):
-                group_seeds.append(seeds[it["pos"]])
-                group_of_seed[it["pos"]] = gi
-            offsets.append(offsets[-1] + sum(it["O"] for it in grp))
-        est = [ld for _, ld in kept]
-        rank_load = [0] * max(1, num_gpus)
-        rank_of_group = [0] * len(kept)
-        for gi in sorted(range(len(kept)), key=lambda j: (-est[j], j)):
-            r = min(range(len(rank_load)), key=lambda j: (rank_load[j], j))
-            rank_of_group[gi] = r
-            rank_load[r] += est[gi]
-        return dict(K=len(kept), K_tried=K, group_offsets=np.array(offsets, dtype=np.int64),
-                    group_seeds=(np.concatenate(group_seeds).astype(np.int32) if group_seeds
-                                 else np.zeros(0, np.int32)),
-                    group_of_seed=group_of_seed, est_bytes=np.array(est, dtype=np.int64),
-                    rank_of_group=np.array(rank_of_group, dtype=np.int32),
-                    D=D, bucket=bucket, hist=hist)
+        if ok:
+            return K, items, groups, loads, exploded
     return None
+
+
+def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT64_MAX,
+             C_ppm=0, k_min=1, k_max=4096, num_gpus=1, aggregator="mean", fast_paths=True):
+    """Alg. 3 Buffalo_Scheduler (PAPER.md:269-280, :333) with the readings of DESIGN.md
+    (R7 explosion test, R11 sort/placement keys, R16 K_max, R17 empty groups dropped,
+    R24 k_min = #GPUs and LPT rank assignment, R25 fast paths).  Returns a dict plan or None
+    (budget)."""
+    seeds = np.asarray(seeds, dtype=np.int32)
+    f_L = fanout[L - 1]
+    D, bucket, order, hist = degree_bucketing(g, seeds, f_L, F)
+    pos_of = {d: np.nonzero(bucket == d)[0] for d in range(F + 1)}
+
+    def stats_of(pos):
+        st = item_stats(g, seeds[pos], L, fanout, seed, dims, act_dtype, aggregator)
+        st["w"] = grouping_weight(st["M"], st["I"], st["E"], C_ppm)
+        st["pos"] = pos
+        return st
+
+    stats = {d: stats_of(pos_of[d]) for d in range(F + 1) if pos_of[d].size}
+
+    def piece_stats(K):
+        return [(k, stats_of(piece)) for k, piece in enumerate(split_explosion(pos_of[F], K)) if piece.size]
+
+    res = _alg3_k_loop(stats, F, piece_stats, mem_budget, C_ppm, max(k_min, num_gpus, 1), k_max, fast_paths)
+    if res is None:
+        return None
+    K, items, groups, loads, exploded = res
+    kept = [(grp, ld) for grp, ld in zip(groups, loads) if grp]
+    offsets = [0]
+    group_seeds = []
+    group_of_seed = np.full(seeds.size, -1, dtype=np.int32)
+    for gi, (grp, _) in enumerate(kept):
+        for it in sorted(grp, key=lambda it: (it["d"], it["k"])):
+            group_seeds.append(seeds[it["pos"]])
+            group_of_seed[it["pos"]] = gi
+        offsets.append(offsets[-1] + sum(it["O"] for it in grp))
+    est = [ld for _, ld in kept]
+    rank_load = [0] * max(1, num_gpus)
+    rank_of_group = [0] * len(kept)
+    for gi in sorted(range(len(kept)), key=lambda j: (-est[j], j)):
+        r = min(range(len(rank_load)), key=lambda j: (rank_load[j], j))
+        rank_of_group[gi] = r
+        rank_load[r] += est[gi]
+    return dict(K=len(kept), K_tried=K, exploded=exploded, num_items=len(items),
+                group_offsets=np.array(offsets, dtype=np.int64),
+                group_seeds=(np.concatenate(group_seeds).astype(np.int32) if group_seeds
+                             else np.zeros(0, np.int32)),
+                group_of_seed=group_of_seed, est_bytes=np.array(est, dtype=np.int64),
+                rank_of_group=np.array(rank_of_group, dtype=np.int32),
+                D=D, bucket=bucket, hist=hist)
 
 
 # ============================================================================ layer math

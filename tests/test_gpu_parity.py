@@ -135,6 +135,7 @@ def test_bucketize_plan_bit_exact(name, variant):
                       **{k: v for k, v in kw.items() if k != "num_gpus"}, world=kw["num_gpus"])
     K, offs, est, ranks = tr.schedule(0)
     assert K == ref["K"] and tr.plan.k_tried == ref["K_tried"]
+    assert bool(tr.plan.exploded) == ref["exploded"] and tr.plan.num_items == ref["num_items"]
     np.testing.assert_array_equal(offs, ref["group_offsets"])
     np.testing.assert_array_equal(est, ref["est_bytes"])
     np.testing.assert_array_equal(ranks, ref["rank_of_group"])
@@ -148,6 +149,46 @@ def test_bucketize_plan_bit_exact(name, variant):
         blocks = O.build_blocks(g, gs[offs[k]:offs[k + 1]], L, fan, 3)
         want = [blocks[0]["n_src"]] + [b["n_dst"] for b in blocks] + [b["n_edges"] for b in blocks]
         np.testing.assert_array_equal(tr.sizes_h[k], want, err_msg=f"group {k}")
+
+
+def test_bucketize_random_instances_vs_plain_loop():
+    """The library's K loop (with the R25 fast paths and batched micro-bucket statistics)
+    against the oracle's plain Alg. 3 loop (fast_paths=False) on random instances: K, the
+    explosion flag (R7) and the whole plan bit for bit."""
+    rng = np.random.default_rng(77)
+    rp, col = random_graph(2000, 12000, "powerlaw")
+    g = O.Graph(rp, col)
+    n_exp = 0
+    for it in range(24):
+        S = int(rng.integers(50, 1500))
+        seeds = np.sort(rng.choice(g.N, S, replace=False)).astype(np.int32)
+        L = int(rng.integers(1, 4))
+        fan = [int(rng.choice([0, 3, 5, 10])) for _ in range(L)]
+        F = int(rng.integers(2, 11)) if fan[-1] <= 0 else fan[-1]
+        dims = [int(rng.integers(4, 48)) for _ in range(L + 1)]
+        full = O.schedule(g, seeds, L, fan, F, 3, dims, k_min=1, k_max=1)
+        budget = int(full["est_bytes"][0] * rng.uniform(0.1, 1.0))
+        gpus = int(rng.choice([1, 2, 3]))
+        ref = O.schedule(g, seeds, L, fan, F, 3, dims, mem_budget=budget, k_max=40, num_gpus=gpus,
+                         fast_paths=False)
+        X = np.zeros((g.N, dims[0]), np.float32)
+        y = np.zeros(g.N, np.int32)
+        Ws, bs = xavier_weights(dims)
+        tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, base_seed=3, mem_budget=budget, k_max=40,
+                          world=gpus)
+        if ref is None:
+            with pytest.raises(B.BuffaloError) as ei:
+                tr.schedule(0)
+            assert ei.value.status == B.ERR_BUDGET
+            continue
+        K, offs, est, ranks = tr.schedule(0)
+        n_exp += ref["exploded"]
+        assert (K, tr.plan.k_tried, bool(tr.plan.exploded)) == (ref["K"], ref["K_tried"], ref["exploded"]), it
+        np.testing.assert_array_equal(offs, ref["group_offsets"])
+        np.testing.assert_array_equal(est, ref["est_bytes"])
+        np.testing.assert_array_equal(ranks, ref["rank_of_group"])
+        np.testing.assert_array_equal(tr.group_seeds.cpu().numpy(), ref["group_seeds"])
+    assert n_exp >= 3
 
 
 def test_bucketize_budget_error():

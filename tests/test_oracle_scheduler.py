@@ -182,3 +182,80 @@ def test_schedule_budget_error_and_multi_gpu():
     assert O.schedule(g, seeds, 2, [3, 4], 4, 3, [8, 8, 3], mem_budget=1000, k_max=64) is None
     plan = O.schedule(g, seeds, 2, [3, 4], 4, 3, [8, 8, 3], num_gpus=4)
     assert plan["K"] == 4 and sorted(plan["rank_of_group"].tolist()) == [0, 1, 2, 3]
+
+
+# ---------------------------------------------------------------- R7 / R25 pins
+def _hand_stats(Ms, F):
+    return {d: dict(M=M, w=M, O=10, I=1, E=1, pos=np.arange(1)) for d, M in Ms.items()}
+
+
+def _pieces(M_F):
+    def piece_stats(K):
+        return [(k, dict(M=M_F // K + 10, w=M_F // K + 10, O=1, I=1, E=1, pos=np.arange(1))) for k in range(K)]
+    return piece_stats
+
+
+def test_explosion_flips_at_known_K():
+    """Hand instance of R7 ("bucket explosion detected"): M_est = 200, 200 for
+    the buckets of degree 1, 2 and 100 for bucket F = 3; sum M = 500, so M_F * K > 500 first
+    holds at K = 6 (K = 5 is the equality, not an explosion).  At K = 6 the six micro-buckets
+    (M = 100 // 6 + 10 = 26 each) are placed by Alg. 4: 200 -> g0, 200 -> g1, then pieces
+    k0..k3 -> g2..g5, k4 -> g2 (lowest load, lowest index), k5 -> g3."""
+    stats = _hand_stats({1: 200, 2: 200, 3: 100}, 3)
+    for K, boom in ((2, False), (5, False), (6, True), (7, True)):
+        res = O.core._alg3_k_loop(stats, 3, _pieces(100), 1000, 0, K, K)
+        assert res is not None and res[0] == K and res[4] is boom, K
+        assert len(res[1]) == (2 + K if boom else 3)
+    K, items, groups, loads, boom = O.core._alg3_k_loop(stats, 3, _pieces(100), 1000, 0, 6, 6)
+    got = [[(it["d"], it["k"]) for it in g] for g in groups]
+    assert got == [[(1, 0)], [(2, 0)], [(3, 0), (3, 4)], [(3, 1), (3, 5)], [(3, 2)], [(3, 3)]]
+    assert loads == [200, 200, 52, 52, 26, 26]
+    # with a budget of 200 the loop succeeds at K = 3 without a split (the first feasible K)
+    res = O.core._alg3_k_loop(stats, 3, _pieces(100), 200, 0, 1, 64)
+    assert res[0] == 3 and res[4] is False
+    # below 200 no K can succeed: the fast path stops at once, the plain loop tries every K
+    calls = []
+
+    def counting(K):
+        calls.append(K)
+        return _pieces(100)(K)
+    assert O.core._alg3_k_loop(stats, 3, counting, 199, 0, 1, 64) is None and calls == []
+    assert O.core._alg3_k_loop(stats, 3, counting, 199, 0, 1, 64, fast_paths=False) is None
+    assert calls == list(range(6, 65))          # the plain loop splits at every exploding K
+
+
+def test_fast_paths_equal_plain_loop_random():
+    """R25: the scheduler's fast paths (skip a K when the never-split buckets cannot fit,
+    stop when one of them alone exceeds M_ctr) give exactly the plan of the plain Alg. 3
+    loop, on 200 random instances (graph shape, fanouts, F, budget, C, #GPUs)."""
+    rng = np.random.default_rng(1234)
+    graphs = [random_graph(n, p, kind) for n, p, kind in ((150, 600, "powerlaw"), (300, 2400, "powerlaw"),
+                                                          (200, 500, "gnm"))]
+    n_exploded = n_none = n_skipped = 0
+    for it in range(200):
+        rp, col = graphs[it % 3]
+        g = O.Graph(rp, col)
+        S = int(rng.integers(20, g.N))
+        seeds = np.sort(rng.choice(g.N, S, replace=False)).astype(np.int32)
+        L = int(rng.integers(1, 3))
+        fan = [int(rng.choice([0, 2, 3, 5, 8])) for _ in range(L)]
+        F = int(rng.integers(1, 9)) if fan[-1] <= 0 else min(fan[-1], int(rng.integers(1, 9)))
+        dims = [int(rng.integers(4, 40)) for _ in range(L + 1)]
+        full = O.schedule(g, seeds, L, fan, F, 3, dims, k_min=1, k_max=1)
+        budget = int(full["est_bytes"][0] * rng.uniform(0.05, 1.1))
+        kw = dict(mem_budget=budget, C_ppm=int(rng.choice([0, 0, 50000, 226000, 1000000])),
+                  num_gpus=int(rng.choice([1, 1, 2, 3])), k_max=int(rng.integers(1, 13)))
+        a = O.schedule(g, seeds, L, fan, F, 3, dims, **kw)
+        b = O.schedule(g, seeds, L, fan, F, 3, dims, fast_paths=False, **kw)
+        assert (a is None) == (b is None), it
+        if a is None:
+            n_none += 1
+            continue
+        n_exploded += bool(a["exploded"])
+        n_skipped += a["K_tried"] > max(1, kw["num_gpus"])
+        for k in ("K", "K_tried", "exploded", "num_items"):
+            assert a[k] == b[k], (it, k)
+        for k in ("group_offsets", "group_seeds", "group_of_seed", "est_bytes", "rank_of_group"):
+            np.testing.assert_array_equal(a[k], b[k], err_msg=f"instance {it} {k}")
+    # the instances exercise every branch
+    assert n_exploded >= 10 and n_none >= 10 and n_skipped >= 10, (n_exploded, n_none, n_skipped)
