@@ -111,26 +111,36 @@ def make_inputs(cfg):
 
 
 # ----------------------------------------------------------------------------- oracle arm
-def oracle_sample(cfg, rp, col, X, y, seeds, Ws, bs, seconds):
+def oracle_sample(cfg, rp, col, X, y, seeds, Ws, bs, seconds, edges_per_epoch=None):
     """The CPU oracle (oracle/, as it stands) on a bounded sample of the workload: one
-    micro-batch of a contiguous slice of the seed batch, grown until ~`seconds` of work."""
+    micro-batch of a contiguous slice of the seed batch, grown until ~`seconds` of work.  The
+    oracle is single-threaded C (blocks) plus numpy/scipy (layer math); BLAS is pinned to one
+    thread so `cores` = 1 is what it used.  Its epoch time is extrapolated from the measured
+    rate (aggregated edges of our epoch / oracle edges per second)."""
     import oracle as O
+    from threadpoolctl import threadpool_limits
     g = O.Graph(rp, col)
     frac = 64
     n_edges, elapsed, used = 0, 0.0, 0
-    while True:
-        part = seeds[: max(1, len(seeds) // frac)]
-        t = time.perf_counter()
-        loss, grads, blocks = O.microbatch_step(g, part, X[:, :cfg.d0], y, Ws, bs, cfg.L, cfg.fanout, 3,
-                                                len(seeds))
-        dt = time.perf_counter() - t
-        n_edges, elapsed, used = sum(b["n_edges"] for b in blocks), dt, len(part)
-        if dt * 3 > seconds or frac == 1:
-            break
-        frac = max(1, frac // 4)
-    return dict(value=n_edges / elapsed, unit="edges/s", cores=len(os.sched_getaffinity(0)), kind="oracle",
-                sample=f"one micro-batch of {used} of {len(seeds)} seeds ({n_edges} block edges, "
-                       f"{elapsed:.2f} s): C block generation + float64 numpy/scipy SAGE fwd/bwd")
+    with threadpool_limits(limits=1):
+        while True:
+            part = seeds[: max(1, len(seeds) // frac)]
+            t = time.perf_counter()
+            loss, grads, blocks = O.microbatch_step(g, part, X[:, :cfg.d0], y, Ws, bs, cfg.L, cfg.fanout, 3,
+                                                    len(seeds))
+            dt = time.perf_counter() - t
+            n_edges, elapsed, used = sum(b["n_edges"] for b in blocks), dt, len(part)
+            if dt * 3 > seconds or frac == 1:
+                break
+            frac = max(1, frac // 4)
+    rate = n_edges / elapsed
+    out = dict(value=rate, unit="edges/s", cores=1, kind="oracle",
+               sample=f"one micro-batch of {used} of {len(seeds)} seeds ({n_edges} block edges, "
+                      f"{elapsed:.2f} s, measured): C block generation + float64 numpy/scipy SAGE fwd/bwd, "
+                      f"1 thread (BLAS pinned)")
+    if edges_per_epoch:
+        out["epoch_s_extrapolated"] = edges_per_epoch / rate
+    return out
 
 
 def run_reference(args, cfg):
@@ -239,6 +249,91 @@ class Clocks:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
+# ----------------------------------------------------------------------------- diagnostics
+def phase_breakdown(tr, epoch):
+    """One sequential epoch (outside the timed region) with CUDA events around each phase on the
+    main stream: schedule (Alg. 3), and per group build / forward / loss / backward, summed; plus
+    the block-build rates of SURVEY §8(d): sampled (block) edges per second of build time and a
+    sector-based effective bandwidth (per edge: one 32-B sector for the cached sample row or CSR
+    entry, two random 32-B sectors for the relabel's node bitmap and node map, 8 B of col_local /
+    col_global writes, 8 B for the transpose; per dst row 16 B of row_ptr, 4 B of id)."""
+    import torch
+    from paper_conf_hpca_yangzl25_b200 import buffalo as B
+
+    def ev():
+        e = torch.cuda.Event(enable_timing=True)
+        e.record()
+        return e
+    torch.cuda.synchronize()
+    e0 = ev()
+    K, offs, est, ranks = tr.schedule(epoch)
+    e1 = ev()
+    L = tr.L
+    mine = [k for k in range(K) if int(ranks[k]) == tr.rank]
+    tr._ensure_arena(max(B.estimate_mem(tr.sizes_h[k, :L + 1], tr.sizes_h[k, L + 1:], tr.model)[0] for k in mine))
+    sampler = tr.sampler(epoch)
+    marks, edges, dsts = [], 0, 0
+    tr.loss.zero_()
+    for k in mine:
+        n = int(offs[k + 1] - offs[k])
+        a = ev()
+        tr.build(offs[k], n, sampler, tr.sizes_h[k])
+        b = ev()
+        tr.forward()
+        c = ev()
+        tr.loss_and_grad(offs[k], n)
+        d = ev()
+        tr.backward()
+        e = ev()
+        marks.append((a, b, c, d, e))
+        edges += int(sum(tr.sizes_h[k, L + 1:]))
+        dsts += int(sum(tr.sizes_h[k, 1:L + 1]))
+    torch.cuda.synchronize()
+    tr.params.grad.zero_()
+    ph = {"schedule": e0.elapsed_time(e1), "build": 0.0, "forward": 0.0, "loss": 0.0, "backward": 0.0}
+    for a, b, c, d, e in marks:
+        ph["build"] += a.elapsed_time(b)
+        ph["forward"] += b.elapsed_time(c)
+        ph["loss"] += c.elapsed_time(d)
+        ph["backward"] += d.elapsed_time(e)
+    sector_bytes = edges * (3 * 32 + 8 + 8) + dsts * 20
+    build = {"ms": ph["build"], "sampled_edges": edges, "edges_per_s": edges / (ph["build"] / 1e3),
+             "sector_gbs": sector_bytes / (ph["build"] / 1e3) / 1e9, "launches_note": "sync-free (plan sizes)"}
+    return {k: round(v, 3) for k, v in ph.items()}, build
+
+
+def measured_memory(tr, epoch):
+    """Per own group of `epoch`: the measured arena high-water (sentinel fill, Trainer.
+    measure_high_water: independent of the memory model and of the allocator's bookkeeping)
+    against the exact model (lo, hi) and the Eq. 2 group estimate (Table III's
+    estimate-vs-measured comparison, :477-497)."""
+    K, offs, est, ranks = tr.schedule(epoch)
+    rows = []
+    for k in range(K):
+        if int(ranks[k]) != tr.rank:
+            continue
+        hw, lo, hi, ok = tr.measure_high_water(k, epoch)
+        rows.append((k, hw, lo, hi, int(est[k]), ok))
+    tr.params.grad.zero_()
+    hw = np.array([r[1] for r in rows], np.float64)
+    eq2 = np.array([r[4] for r in rows], np.float64)
+    return {"budget_bytes": int(tr.sched.mem_budget), "groups": len(rows),
+            "measured_high_water_max_bytes": int(hw.max()), "measured_high_water_min_bytes": int(hw.min()),
+            "measured_spread_max_over_min": float(hw.max() / hw.min()),
+            "measured_within_exact_model": bool(all(r[1] <= r[2] <= r[3] and r[5] for r in rows)),
+            "exact_lo_minus_measured_max_bytes": int(max(r[2] - r[1] for r in rows)),
+            "eq2_over_measured_mean": float(np.mean(eq2 / hw - 1.0)),
+            "eq2_over_measured_max": float(np.max(eq2 / hw - 1.0)),
+            "eq2_over_measured_min": float(np.min(eq2 / hw - 1.0)),
+            "max_measured_over_budget": float(hw.max() / tr.sched.mem_budget),
+            "fixed_device_bytes_outside_arena": tr.fixed_bytes(),
+            "method": "arena filled with a sentinel word, library given exactly lo bytes; high-water = highest "
+                      "overwritten word after build+fwd+loss+bwd; a 1 MiB sentinel guard past lo stays intact",
+            "note": "Eq. 2 with R = 1 (C of the synthetic graphs is ~5e-4) sums the items' own estimates, so it "
+                    "over-estimates the nodes they share; fixed bytes (graph workspaces, scheduler workspace, "
+                    "sample caches, plans, weights) are outside M_ctr"}
+
+
 # ----------------------------------------------------------------------------- our arm
 def run_ours(args, cfg):
     import torch
@@ -296,13 +391,15 @@ def run_ours(args, cfg):
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, mem_budget=budget,
                  C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg,
                  pipeline=not args.no_pipeline, **agg_kw)
+    full_batch_edges = None
     if args.config in ("products", "papers", "arxiv_lstm"):
         # calibrate M_ctr once so that one GPU needs >= 8 groups (products; 2 for the LSTM
         # workload), then freeze it for every N
         B_full = Trainer(graph, feats, y, seeds, cfg.dims,
                          cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, C_ppm=C_ppm,
-                         k_min=1, k_max=1, **agg_kw)
+                         k_min=1, k_max=1, sample_cache=False, **agg_kw)
         _, _, est1, _ = B_full.schedule(0)
+        full_batch_edges = int(B_full.sizes_h[0, cfg.L + 1:].sum())       # K = 1: no redundancy
         del B_full
         tr.sched.mem_budget = int(est1[0]) // (2 if args.config == "arxiv_lstm" else 8)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
@@ -364,8 +461,14 @@ def run_ours(args, cfg):
         s0 = torch.cuda.Event(enable_timing=True)
         s1 = torch.cuda.Event(enable_timing=True)
         s0.record(stream)
-        tr.seeds.copy_(seeds_h, non_blocking=True)
-        st = tr.run_epoch(epoch=1000 + i, lr=lr)
+        if tr.pipeline:
+            # the seed batch of step i+1 goes up (pinned H2D on the scheduler's stream) before the
+            # plan made for it during step i; the plan used by step i was made for the batch sent
+            # during step i-1 (the first e2e step schedules its batch itself: epoch mismatch)
+            st = tr.run_epoch(epoch=1000 + i, lr=lr, next_seeds=seeds_h)
+        else:
+            tr.set_seeds(seeds_h)
+            st = tr.run_epoch(epoch=1000 + i, lr=lr)
         loss_h.copy_(tr.loss, non_blocking=True)
         s1.record(stream)
         s1.synchronize()
@@ -391,18 +494,10 @@ def run_ours(args, cfg):
     if os.path.exists(tpath):
         traffic = json.load(open(tpath)).get(f"{args.config}/{args.gemm}" + ("" if args.aggregator == "mean" else
                                                                               "/" + args.aggregator))
-    # memory: the Eq. 2 group estimates (the paper's Table III reports its
-    # estimation error) against each group's measured arena high-water mark, the exact arena
-    # model (R15) and the fixed budget M_ctr, for the groups of the last timed epoch on this rank
-    gs = last_st["groups"]
-    peaks = np.array([g["peak"] for g in gs], np.float64)
-    eq2 = np.array([last_st["est"][g["k"]] for g in gs], np.float64)
-    mem_est = {"budget_bytes": int(tr.sched.mem_budget), "max_peak_bytes": int(peaks.max()),
-               "eq2_over_peak_mean": float(np.mean(eq2 / peaks - 1.0)),
-               "eq2_over_peak_max": float(np.max(eq2 / peaks - 1.0)),
-               "model_brackets_peak": bool(all(g["est_lo"] <= g["peak"] <= g["est_hi"] for g in gs)),
-               "note": "Eq. 2 with R = 1 (the synthetic graphs' C is ~5e-4) sums the items' own estimates, so it "
-                       "over-estimates shared nodes; the exact arena model (lo, hi) brackets the measured peak"}
+    # diagnostics outside the timed region: measured memory high-water of every own group of
+    # the first timed epoch, and one sequential epoch's phase breakdown + block-build rates
+    mem_est = measured_memory(tr, args.warmup)
+    phases, build_rates = phase_breakdown(tr, args.warmup)
     if lstm:   # the LSTM path is bound by its fp32 SIMT gate GEMMs: FLOP roofline ("alu")
         tf = g_bytes / (g_ms / 1e3) / 1e12 if g_ms > 0 else 0.0
         roof = {"bound": "alu", "kernel": "k_gemm2_tc (LSTM gate GEMM of every step, fp32 as 3xTF32 mma.sync)",
@@ -426,7 +521,8 @@ def run_ours(args, cfg):
         cpu = None
         if world == 1 and not args.no_cpu_baseline and not (pool or lstm or gat or big):   # (the pool oracle is loop-plain: tests only)
             rp_h, col_h, X_h, y_h, seeds_h = host_copies(rp, col, X, y, tr.seeds)
-            cpu = oracle_sample(cfg, rp_h, col_h, X_h, y_h, seeds_h, Ws, bs, args.cpu_baseline_seconds)
+            cpu = oracle_sample(cfg, rp_h, col_h, X_h, y_h, seeds_h, Ws, bs, args.cpu_baseline_seconds,
+                                edges / args.steps)
         line = dict(
             metric="aggregated edges/s (epoch of Buffalo hot path)", value=value, unit="edges/s",
             n_gpus=world, steps=args.steps, warmup=args.warmup, ms_per_step=total_ms / args.steps,
@@ -439,6 +535,9 @@ def run_ours(args, cfg):
                     "gemm": args.gemm, "aggregator": args.aggregator,
                     "l2": "flushed (512 MiB write) between timed steps",
                     "epoch_ms": total_ms / args.steps, "edges_per_epoch": edges / args.steps,
+                    "full_batch_edges": full_batch_edges,
+                    "redundancy": (edges / args.steps / full_batch_edges) if full_batch_edges else None,
+                    "phases_ms_sequential": phases, "block_build": build_rates,
                     "parallelism": f"dp{world} over bucket groups",
                     "pipeline": "scheduler of epoch e+1 overlapped with epoch e" if not args.no_pipeline else "off",
                     "C_eq1": C_eq1, "C_ppm": C_ppm, "C_table2": C_TABLE2.get(args.config),

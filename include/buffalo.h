@@ -9,8 +9,17 @@
  *    allocated and owned by the caller; the library never calls cudaMalloc/cudaFree.
  *  - `stream` is a cudaStream_t passed as void*.  Work is stream-ordered; the only host
  *    synchronisations are the documented ones (data-dependent sizes).
- *  - Errors are returned as buffalo_status (never exceptions/abort); on error, outputs are
- *    unspecified except *required_bytes_h.  buffalo_last_error() gives a thread-local message.
+ *  - Errors are returned as buffalo_status (never exceptions/abort).  Validation errors
+ *    (INVALID_ARG, UNSUPPORTED, CAPACITY, BUDGET) leave the outputs (plan, blocks struct,
+ *    accumulators) untouched, except *required_bytes_h; caller workspaces and arenas are scratch.
+ *    After BUFFALO_ERR_CUDA the outputs are unspecified.  buffalo_last_error() gives a
+ *    thread-local message.
+ *  - Validated inputs: dims, fanouts, pointers, leading dimensions and alignment on every call;
+ *    seed ids (in [0, N), distinct) in buffalo_bucketize and in buffalo_build_blocks without
+ *    sizes_h; the CSR itself (O(N + nnz)) on request by buffalo_graph_validate.
+ *  - Thread safety: no mutable global state affects results; per-thread state is the error
+ *    message, the launch counter and the diagnostic profiler; a per-(kernel, device) cache of
+ *    the shared-memory attribute is idempotent.
  *  - Deterministic: identical inputs and seed give bit-identical outputs.
  *  - Built for sm_100a only; on any other device BUFFALO_ERR_UNSUPPORTED.
  *  - A graph's node_map workspace must not be used by two streams at once.
@@ -167,6 +176,14 @@ BUFFALO_API size_t buffalo_graph_workspace_bytes(int64_t num_nodes);
  * (stream-ordered). */
 BUFFALO_API buffalo_status buffalo_graph_prepare(buffalo_graph* g, void* workspace, size_t bytes, void* stream);
 
+/* O(N + nnz) check of the CSR contract above on the device: row_ptr monotone from 0 to nnz, ids
+ * in [0, N), rows strictly increasing (sorted, no duplicates), no self loops and, with
+ * check_symmetric != 0, every (v, c) matched by (c, v) (binary search).  g must be prepared
+ * (uses its workspace's scan space).  Synchronises once.  BUFFALO_ERR_INVALID_ARG names the
+ * first violated rule.  The hot-path calls trust a validated graph (Alg. 3 input G, PAPER.md:
+ * 261-265). */
+BUFFALO_API buffalo_status buffalo_graph_validate(const buffalo_graph* g, int32_t check_symmetric, void* stream);
+
 /* ------------------------------------------------------------------ a1-a3: scheduler */
 /* Upper bound of the workspace buffalo_bucketize needs for n_seeds seeds. */
 BUFFALO_API size_t buffalo_bucketize_workspace_bytes(const buffalo_graph* g, int64_t n_seeds,
@@ -175,8 +192,9 @@ BUFFALO_API size_t buffalo_bucketize_workspace_bytes(const buffalo_graph* g, int
  * BucketMemEstimator (R13, R15, obtained by building each item's blocks on the GPU),
  * Eq. 1-2, SplitExplosionBucket (R7, R8) and MemBalancedGrouping (Alg. 4,
  * PAPER.md:313-326, R10-R12).  seeds: device int32[n_seeds] (distinct global ids).
- * Synchronises the stream (data-dependent sizes).  BUFFALO_ERR_BUDGET if no K fits M_ctr;
- * BUFFALO_ERR_CAPACITY if workspace_bytes is too small. */
+ * Synchronises the stream (data-dependent sizes).  BUFFALO_ERR_INVALID_ARG if a seed id is
+ * outside [0, N) or occurs twice; BUFFALO_ERR_BUDGET if no K fits M_ctr; BUFFALO_ERR_CAPACITY if
+ * workspace_bytes is too small.  The plan is written only on success. */
 BUFFALO_API buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, int64_t n_seeds,
                                  const buffalo_sampler* s, const buffalo_model* m,
                                  const buffalo_sched* sc, buffalo_plan* plan, void* workspace,
@@ -193,8 +211,10 @@ BUFFALO_API buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32
  *   any host synchronisation; n_heavy / n_heavy_t / heavy are then left at -1 / NULL (kernels
  *   find the long rows at the tail of cls_perm / t_perm).  Sizes that do not match the group
  *   give undefined block contents (writes stay inside the arena).
- *   NULL: the sizes are read back while building (two to three synchronisations per layer);
- *   BUFFALO_ERR_CAPACITY then reports a lower bound of the need in *required_bytes_h. */
+ *   NULL: the group's ids are validated (in [0, N), distinct: BUFFALO_ERR_INVALID_ARG), then the
+ *   sizes are read back while building (two to three synchronisations per layer);
+ *   BUFFALO_ERR_CAPACITY then reports a lower bound of the need in *required_bytes_h.
+ * *out is written only on success. */
 BUFFALO_API buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group_seeds, int64_t n,
                                     const buffalo_sampler* s, const buffalo_model* m,
                                     buffalo_blocks* out, void* arena, size_t arena_bytes,

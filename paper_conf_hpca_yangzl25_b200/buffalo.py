@@ -32,7 +32,7 @@ EXPORTS = [
     "buffalo_status_str", "buffalo_last_error",
     "buffalo_clustering_workspace_bytes", "buffalo_triangles", "buffalo_avg_clustering",
     "buffalo_pool_fwd", "buffalo_pool_bwd", "buffalo_lstm_fwd", "buffalo_lstm_bwd",
-    "buffalo_gat_fwd", "buffalo_gat_bwd",
+    "buffalo_gat_fwd", "buffalo_gat_bwd", "buffalo_graph_validate",
 ]
 
 
@@ -129,6 +129,7 @@ def lib(require_gpu=True):
             "buffalo_gat_fwd": (c_i32, [P, c_i32, P, P, c_i64, P, P, P, P, P, c_i64, P, c_sz, P]),
             "buffalo_gat_bwd": (c_i32, [P, c_i32, P, P, c_i64, P, c_i64, P, c_i64, P, c_sz, P, P, P, P, P, P, P, P,
                                         c_i64, P, c_sz, P]),
+            "buffalo_graph_validate": (c_i32, [P, c_i32, P]),
             "buffalo_status_str": (ctypes.c_char_p, [c_i32]),
             "buffalo_last_error": (ctypes.c_char_p, []),
         }
@@ -155,6 +156,31 @@ def ptr(t):
     return t.data_ptr()
 
 
+def dev(t, dtypes, name):
+    """Pointer of a device tensor argument after checking what the C ABI assumes of it: a CUDA,
+    C-contiguous tensor of one of `dtypes` (an int64 tensor read as int32 ids, or an fp32 table
+    read as bf16, would otherwise give wrong results silently).  Raw ints pass through."""
+    if t is None or isinstance(t, int):
+        return t
+    if not (t.is_cuda and t.is_contiguous()):
+        raise ValueError(f"{name}: expected a contiguous CUDA tensor")
+    if t.dtype not in dtypes:
+        raise TypeError(f"{name}: dtype {t.dtype}, expected {' or '.join(str(d) for d in dtypes)}")
+    return t.data_ptr()
+
+
+I32 = (torch.int32,)
+F32 = (torch.float32,)
+FEAT = {FP32: (torch.float32,), BF16: (torch.bfloat16,)}
+
+
+def act_dtypes(model, layer):
+    """dtype of layer `layer`'s input rows: the feature table at layer 1, else the activations."""
+    if layer == 1:
+        return FEAT[model.feat_dtype]
+    return (torch.bfloat16,) if model.gemm_mode == GEMM_BF16 else (torch.float32,)
+
+
 def stream_ptr(stream=None):
     s = stream if stream is not None else torch.cuda.current_stream()
     return s.cuda_stream
@@ -174,12 +200,17 @@ def graph_prepare(graph, workspace, stream=None):
                                        stream_ptr(stream)))
 
 
+def graph_validate(graph, check_symmetric=True, stream=None):
+    """O(N + nnz) check of the CSR contract on the device (raises BuffaloError)."""
+    _check(lib().buffalo_graph_validate(ref(graph), int(bool(check_symmetric)), stream_ptr(stream)))
+
+
 def bucketize_workspace_bytes(graph, n_seeds, sampler, model):
     return lib(False).buffalo_bucketize_workspace_bytes(ref(graph), n_seeds, ref(sampler), ref(model))
 
 
 def bucketize(graph, seeds, sampler, model, sched, plan, workspace, stream=None):
-    _check(lib().buffalo_bucketize(ref(graph), ptr(seeds), seeds.numel(), ref(sampler), ref(model),
+    _check(lib().buffalo_bucketize(ref(graph), dev(seeds, I32, "seeds"), seeds.numel(), ref(sampler), ref(model),
                                    ref(sched), ref(plan), ptr(workspace), workspace.numel(),
                                    stream_ptr(stream)))
 
@@ -192,7 +223,7 @@ def build_blocks(graph, group_seeds, n, sampler, model, blocks, arena, sizes=Non
     if sizes is not None:
         assert sizes.dtype == np.int64 and sizes.flags["C_CONTIGUOUS"]
         sz = sizes.ctypes.data
-    st = lib().buffalo_build_blocks(ref(graph), ptr(group_seeds), n, ref(sampler), ref(model),
+    st = lib().buffalo_build_blocks(ref(graph), dev(group_seeds, I32, "group_seeds"), n, ref(sampler), ref(model),
                                     ref(blocks), ptr(arena), arena.numel(), ctypes.byref(req), sz,
                                     stream_ptr(stream))
     if st == ERR_CAPACITY:
@@ -212,12 +243,14 @@ def pack_weights(model, layer, W, packed, stream=None):
 
 
 def sage_fwd(blk, layer, model, h_src, ld_src, W, W_packed, b, out, ld_out, saved_agg, ld_agg, stream=None):
-    _check(lib().buffalo_sage_fwd(ref(blk), layer, ref(model), ptr(h_src), ld_src, ptr(W), ptr(W_packed),
+    _check(lib().buffalo_sage_fwd(ref(blk), layer, ref(model), dev(h_src, act_dtypes(model, layer), "h_src"), ld_src,
+                                  dev(W, F32, "W"), ptr(W_packed),
                                   ptr(b), ptr(out), ld_out, ptr(saved_agg), ld_agg, stream_ptr(stream)))
 
 
 def softmax_ce(logits, ld, n, classes, labels, row_ids, batch_size, loss_accum, dlogits, ld_d, stream=None):
-    _check(lib().buffalo_softmax_ce(ptr(logits), ld, n, classes, ptr(labels), ptr(row_ids), batch_size,
+    _check(lib().buffalo_softmax_ce(ptr(logits), ld, n, classes, dev(labels, I32, "labels"),
+                                    dev(row_ids, I32, "row_ids"), batch_size,
                                     ptr(loss_accum), ptr(dlogits), ld_d, stream_ptr(stream)))
 
 
@@ -227,7 +260,8 @@ def sage_bwd_scratch_bytes(blk, layer, model):
 
 def sage_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg, h_dst, ld_hdst, W,
              W_packed, dW, db, dh_src, ld_dh_src, prev_row_ptr, scratch, scratch_bytes, stream=None):
-    _check(lib().buffalo_sage_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh, ptr(h_src), ld_src,
+    _check(lib().buffalo_sage_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh,
+                                  dev(h_src, act_dtypes(model, layer), "h_src"), ld_src,
                                   ptr(saved_agg), ld_agg, ptr(h_dst), ld_hdst, ptr(W), ptr(W_packed),
                                   ptr(dW), ptr(db), ptr(dh_src), ld_dh_src, ptr(prev_row_ptr), ptr(scratch),
                                   scratch_bytes, stream_ptr(stream)))
@@ -235,14 +269,15 @@ def sage_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg,
 
 def pool_fwd(blk, layer, model, h_src, ld_src, W_pool, b_pool, W, W_packed, b, out, ld_out, saved_agg, ld_agg,
              P, arg, ld_pool, stream=None):
-    _check(lib().buffalo_pool_fwd(ref(blk), layer, ref(model), ptr(h_src), ld_src, ptr(W_pool), ptr(b_pool), ptr(W),
+    _check(lib().buffalo_pool_fwd(ref(blk), layer, ref(model), dev(h_src, act_dtypes(model, layer), "h_src"), ld_src, ptr(W_pool), ptr(b_pool), ptr(W),
                                   ptr(W_packed), ptr(b), ptr(out), ld_out, ptr(saved_agg), ld_agg, ptr(P), ptr(arg),
                                   ld_pool, stream_ptr(stream)))
 
 
 def pool_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg, h_dst, ld_hdst, P, arg, ld_pool,
              W_pool, W, dW_pool, db_pool, dW, db, dh_src, ld_dh_src, scratch, scratch_bytes, stream=None):
-    _check(lib().buffalo_pool_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh, ptr(h_src), ld_src,
+    _check(lib().buffalo_pool_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh,
+                                  dev(h_src, act_dtypes(model, layer), "h_src"), ld_src,
                                   ptr(saved_agg), ld_agg, ptr(h_dst), ld_hdst, ptr(P), ptr(arg), ld_pool,
                                   ptr(W_pool), ptr(W), ptr(dW_pool), ptr(db_pool), ptr(dW), ptr(db), ptr(dh_src),
                                   ld_dh_src, ptr(scratch), scratch_bytes, stream_ptr(stream)))
@@ -250,14 +285,15 @@ def pool_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg,
 
 def lstm_fwd(blk, layer, model, h_src, ld_src, W_ih, W_hh, b_lstm, W, W_packed, b, out, ld_out, saved_agg, ld_agg,
              stream=None):
-    _check(lib().buffalo_lstm_fwd(ref(blk), layer, ref(model), ptr(h_src), ld_src, ptr(W_ih), ptr(W_hh), ptr(b_lstm),
+    _check(lib().buffalo_lstm_fwd(ref(blk), layer, ref(model), dev(h_src, act_dtypes(model, layer), "h_src"), ld_src, ptr(W_ih), ptr(W_hh), ptr(b_lstm),
                                   ptr(W), ptr(W_packed), ptr(b), ptr(out), ld_out, ptr(saved_agg), ld_agg,
                                   ptr(blk.agg_saved), blk.agg_saved_bytes, stream_ptr(stream)))
 
 
 def lstm_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg, h_dst, ld_hdst, W_ih, W_hh, W,
              dW_ih, dW_hh, db_lstm, dW, db, dh_src, ld_dh_src, scratch, scratch_bytes, stream=None):
-    _check(lib().buffalo_lstm_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh, ptr(h_src), ld_src,
+    _check(lib().buffalo_lstm_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh,
+                                  dev(h_src, act_dtypes(model, layer), "h_src"), ld_src,
                                   ptr(saved_agg), ld_agg, ptr(h_dst), ld_hdst, ptr(blk.agg_saved),
                                   blk.agg_saved_bytes, ptr(W_ih), ptr(W_hh), ptr(W), ptr(dW_ih), ptr(dW_hh),
                                   ptr(db_lstm), ptr(dW), ptr(db), ptr(dh_src), ld_dh_src, ptr(scratch),
@@ -265,13 +301,14 @@ def lstm_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg,
 
 
 def gat_fwd(blk, layer, model, h_src, ld_src, W, a_l, a_r, b, out, ld_out, stream=None):
-    _check(lib().buffalo_gat_fwd(ref(blk), layer, ref(model), ptr(h_src), ld_src, ptr(W), ptr(a_l), ptr(a_r), ptr(b),
+    _check(lib().buffalo_gat_fwd(ref(blk), layer, ref(model), dev(h_src, act_dtypes(model, layer), "h_src"), ld_src, ptr(W), ptr(a_l), ptr(a_r), ptr(b),
                                  ptr(out), ld_out, ptr(blk.agg_saved), blk.agg_saved_bytes, stream_ptr(stream)))
 
 
 def gat_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, h_dst, ld_hdst, W, a_l, a_r, dW, db, da_l, da_r,
             dh_src, ld_dh_src, scratch, scratch_bytes, stream=None):
-    _check(lib().buffalo_gat_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh, ptr(h_src), ld_src, ptr(h_dst),
+    _check(lib().buffalo_gat_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh,
+                                  dev(h_src, act_dtypes(model, layer), "h_src"), ld_src, ptr(h_dst),
                                  ld_hdst, ptr(blk.agg_saved), blk.agg_saved_bytes, ptr(W), ptr(a_l), ptr(a_r),
                                  ptr(dW), ptr(db), ptr(da_l), ptr(da_r), ptr(dh_src), ld_dh_src, ptr(scratch),
                                  scratch_bytes, stream_ptr(stream)))

@@ -39,7 +39,7 @@ struct Profiler {
   std::vector<cudaEvent_t> ev;
   std::vector<double> fixed, per_edge;
 };
-Profiler g_prof;
+thread_local Profiler g_prof;   // per host thread (launch sites record on the calling thread)
 }  // namespace
 
 ProfSlot prof_begin_launch(const char* family, cudaStream_t s) {
@@ -342,7 +342,15 @@ buffalo_status buffalo_graph_prepare(buffalo_graph* g, void* workspace, size_t b
     set_error("graph_prepare: null graph/workspace, empty graph or col NULL with nnz > 0");
     return BUFFALO_ERR_INVALID_ARG;
   }
-  if ((int64_t)bytes < (int64_t)buffalo_graph_workspace_bytes(g->num_nodes)) return BUFFALO_ERR_CAPACITY;
+  if (g->num_nodes >= INT32_MAX) {
+    set_error("graph_prepare: node ids are int32: num_nodes must be < 2^31 - 1");
+    return BUFFALO_ERR_UNSUPPORTED;
+  }
+  if ((int64_t)bytes < (int64_t)buffalo_graph_workspace_bytes(g->num_nodes)) {
+    set_error("graph_prepare: workspace of %lld bytes, need %lld", (long long)bytes,
+              (long long)buffalo_graph_workspace_bytes(g->num_nodes));
+    return BUFFALO_ERR_CAPACITY;
+  }
   g->node_map = (int32_t*)workspace;
   cudaStream_t s = (cudaStream_t)stream;
   k_fill_i32<<<grid_for(g->num_nodes, 256), 256, 0, s>>>(g->node_map, g->num_nodes, INT32_MAX);
@@ -350,6 +358,15 @@ buffalo_status buffalo_graph_prepare(buffalo_graph* g, void* workspace, size_t b
   const GraphWs gw = graph_ws(g);
   BF_CUDA(cudaMemsetAsync(gw.bits, 0, sizeof(uint32_t) * gw.words, s));
   return BUFFALO_OK;
+}
+
+buffalo_status buffalo_graph_validate(const buffalo_graph* g, int32_t check_symmetric, void* stream) {
+  BF_CHECK(require_sm100());
+  if (!g || !g->node_map || !g->row_ptr || (!g->col && g->nnz > 0) || g->num_nodes <= 0 || g->nnz < 0) {
+    set_error("graph_validate: null or unprepared graph");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  return validate_graph(g, check_symmetric ? 1 : 0, (cudaStream_t)stream);
 }
 
 buffalo_status buffalo_estimate_mem(int32_t num_layers, const int64_t* n, const int64_t* e,
@@ -403,25 +420,27 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
   char* stats_ws = q;
   const int64_t stats_bytes = (int64_t)workspace_bytes - used;
 
-  // a1: DegreeBucketing (Alg. 3 l.1)
-  BF_CHECK(seed_bucketing(g, seeds, S, fL, F, bucket, order, sorted_ids, counts, ws, starts, plan->hist_h, s));
+  // a1: DegreeBucketing (Alg. 3 l.1); validates the seed ids (in range, distinct).  The plan's
+  // outputs are written only once a K succeeded (outputs untouched on error).
+  std::vector<int64_t> hist(F + 1, 0);
+  BF_CHECK(seed_bucketing(g, seeds, S, fL, F, bucket, order, sorted_ids, counts, ws, starts, hist.data(), s));
   std::vector<int64_t> bstart(F + 2, 0);
-  for (int b = 0; b <= F; ++b) bstart[b + 1] = bstart[b] + plan->hist_h[b];
+  for (int b = 0; b <= F; ++b) bstart[b + 1] = bstart[b] + hist[b];
 
   // a2: per-bucket statistics and estimates (K-independent); item k = degree bucket k
   bool masks_clean = false;
   std::vector<Item> bucket_item(F + 1);
   std::vector<Item*> todo;
   for (int d = 0; d <= F; ++d) {
-    bucket_item[d] = Item{d, 0, bstart[d], plan->hist_h[d], 0, 0, 0, 0, 0};
-    if (plan->hist_h[d] > 0) todo.push_back(&bucket_item[d]);
+    bucket_item[d] = Item{d, 0, bstart[d], hist[d], 0, 0, 0, 0, 0};
+    if (hist[d] > 0) todo.push_back(&bucket_item[d]);
   }
   // the first statistics pass (every seed) fills the sample cache; later passes read it
   BF_CHECK(items_stats(g, sorted_ids, todo, sp, m, stats_ws, stats_bytes, masks_clean, s, 1));
   std::vector<int> non_split;
   int64_t sum_M_all = 0, sum_w = 0, max_w = 0;
   for (int d = 0; d <= F; ++d) {
-    if (plan->hist_h[d] == 0) continue;
+    if (hist[d] == 0) continue;
     Item& it = bucket_item[d];
     it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
     sum_M_all += it.M;
@@ -431,7 +450,7 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
       max_w = std::max(max_w, it.w);
     }
   }
-  const bool hasF = plan->hist_h[F] > 0;
+  const bool hasF = hist[F] > 0;
 
   // a3: the K loop (Alg. 3) with MemBalancedGrouping (Alg. 4).  The micro-bucket statistics
   // of several consecutive K candidates are computed in one statistics pass (their pieces
@@ -569,6 +588,7 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
         }
       }
     }
+    for (int d = 0; d <= F; ++d) plan->hist_h[d] = hist[d];
     plan->k_out = gk;
     plan->k_tried = K;
     plan->exploded = exploded ? 1 : 0;
@@ -617,6 +637,20 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
       return BUFFALO_ERR_CAPACITY;
     }
   }
+  if (!sizes_h) {
+    // the read-back path synchronises anyway: validate the group's ids first (in range,
+    // distinct); with sizes_h the group comes from a plan whose seeds buffalo_bucketize checked
+    int32_t* err_dev = graph_ws(g).scan_ws;
+    BF_CUDA(cudaMemsetAsync(err_dev, 0, sizeof(int32_t), s));
+    BF_CHECK(check_ids(g, group_seeds, n, err_dev, s));
+    int32_t err = 0;
+    BF_CUDA(cudaMemcpyAsync(&err, err_dev, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    BF_CUDA(cudaStreamSynchronize(s));
+    BF_CHECK(ids_error(err, "build_blocks"));
+  }
+  buffalo_blocks* const user_out = out;     // written only on success (outputs untouched on error)
+  buffalo_blocks local;
+  out = &local;
   memset(out, 0, sizeof(*out));
   out->num_layers = L;
   Arena A;
@@ -704,6 +738,7 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
   out->arena_peak = A.peak;
   mem_model(L, nn, ee, m, &out->est_lo, &out->est_hi);
   if (required_bytes_h) *required_bytes_h = A.peak;
+  *user_out = local;
   return BUFFALO_OK;
 }
 

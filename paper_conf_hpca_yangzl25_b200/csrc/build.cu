@@ -503,12 +503,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
       if (hg > 0) {
         const int64_t words = ceil_div(n_dst, 32);
         if (words <= kBitsortMaxWords) {
-          static bool attr = false;
-          if (!attr) {
-            BF_CUDA(cudaFuncSetAttribute(k_tsort_heavy_bits, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         kBitsortMaxWords * 4));
-            attr = true;
-          }
+          BF_CHECK(set_max_smem_once(k_tsort_heavy_bits, kBitsortMaxWords * 4));
           k_tsort_heavy_bits<<<hg, 256, words * 4, s>>>(tperm, n_src, trp, tcol, (int32_t)words);
           BF_LAUNCHED("k_tsort_heavy_bits");
         } else {
@@ -526,11 +521,119 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   return BUFFALO_OK;
 }
 
+// ------------------------------------------------------------------ input validation
+// Id lists (seeds, group seeds; Alg. 3's input G is a set of nodes): every id
+// in [0, N) and none twice.  Duplicates are found through the graph workspace's node bitmap,
+// which k_clear_ids leaves all-zero again (its between-calls invariant).
+__global__ void k_check_ids(const int32_t* __restrict__ ids, int64_t n, int64_t N, uint32_t* __restrict__ bits,
+                            int32_t* __restrict__ err) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t v = ids[i];
+    if (v < 0 || v >= N) {
+      atomicOr(err, 1);
+      continue;
+    }
+    const uint32_t m = 1u << (v & 31);
+    if (atomicOr(bits + (v >> 5), m) & m) atomicOr(err, 2);
+  }
+}
+__global__ void k_clear_ids(const int32_t* __restrict__ ids, int64_t n, int64_t N, uint32_t* __restrict__ bits) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t v = ids[i];
+    if (v >= 0 && v < N) bits[v >> 5] = 0u;
+  }
+}
+buffalo_status check_ids(const buffalo_graph* g, const int32_t* ids, int64_t n, int32_t* err_dev, cudaStream_t s) {
+  if (n <= 0) return BUFFALO_OK;
+  const GraphWs gw = graph_ws(g);
+  k_check_ids<<<grid_for(n, 256), 256, 0, s>>>(ids, n, g->num_nodes, gw.bits, err_dev);
+  BF_LAUNCHED("k_check_ids");
+  k_clear_ids<<<grid_for(n, 256), 256, 0, s>>>(ids, n, g->num_nodes, gw.bits);
+  BF_LAUNCHED("k_clear_ids");
+  return BUFFALO_OK;
+}
+buffalo_status ids_error(int32_t err, const char* what) {
+  if (err & 1) {
+    set_error("%s: a node id is outside [0, num_nodes)", what);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (err & 2) {
+    set_error("%s: a node id occurs twice (the batch is a set of nodes)", what);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  return BUFFALO_OK;
+}
+
+// The graph's CSR (include/buffalo.h: rows sorted ascending, simple, symmetric): a warp per
+// node walks its row.  Error bits: 1 row_ptr not a monotone offset array from 0 to nnz, 2 an
+// id outside [0, N), 4 a row not strictly increasing (unsorted or duplicate entries), 8 a self
+// loop, 16 an edge (v, c) without (c, v) (checked only with `sym`, by binary search of row c).
+__global__ void __launch_bounds__(256) k_validate_csr(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                                      int64_t N, int64_t nnz, int sym, int32_t* __restrict__ err) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  if (blockIdx.x == 0 && threadIdx.x == 0 && (rp[0] != 0 || rp[N] != nnz)) atomicOr(err, 1);
+  for (int64_t v = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; v < N; v += warps) {
+    const int64_t b = rp[v], e = rp[v + 1];
+    if (b < 0 || e < b || e > nnz) {
+      if (lane == 0) atomicOr(err, 1);
+      continue;
+    }
+    int bad = 0;
+    for (int64_t k = b + lane; k < e; k += 32) {
+      const int32_t c = col[k];
+      if (c < 0 || c >= N) {
+        bad |= 2;
+        continue;
+      }
+      if (c == v) bad |= 8;
+      if (k > b && col[k - 1] >= c) bad |= 4;
+      if (sym) {
+        int64_t lo = rp[c], hi = rp[c + 1];
+        if (lo < 0 || hi < lo || hi > nnz) {
+          bad |= 1;
+          continue;
+        }
+        while (lo < hi) {                               // first entry >= v in row c
+          const int64_t mid = (lo + hi) >> 1;
+          if (col[mid] < v) lo = mid + 1; else hi = mid;
+        }
+        if (lo == rp[c + 1] || col[lo] != v) bad |= 16;
+      }
+    }
+    bad = __reduce_or_sync(0xffffffffu, bad);
+    if (lane == 0 && bad) atomicOr(err, bad);
+  }
+}
+
+buffalo_status validate_graph(const buffalo_graph* g, int sym, cudaStream_t s) {
+  const GraphWs gw = graph_ws(g);
+  int32_t* err_dev = gw.scan_ws;                 // scratch between calls
+  BF_CUDA(cudaMemsetAsync(err_dev, 0, sizeof(int32_t), s));
+  k_validate_csr<<<grid_for(g->num_nodes * 32, 256), 256, 0, s>>>(g->row_ptr, g->col, g->num_nodes, g->nnz, sym,
+                                                                  err_dev);
+  BF_LAUNCHED("k_validate_csr");
+  int32_t err = 0;
+  BF_CUDA(cudaMemcpyAsync(&err, err_dev, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  BF_CUDA(cudaStreamSynchronize(s));
+  static const char* what[5] = {"row_ptr is not a monotone offset array from 0 to nnz",
+                                "a column id is outside [0, num_nodes)",
+                                "a row is not strictly increasing (unsorted or duplicate entries)",
+                                "a self loop", "the graph is not symmetric"};
+  for (int k = 0; k < 5; ++k)
+    if (err & (1 << k)) {
+      set_error("graph_validate: %s", what[k]);
+      return BUFFALO_ERR_INVALID_ARG;
+    }
+  return BUFFALO_OK;
+}
+
 // ------------------------------------------------------------------ a1: seed bucketing
 __global__ void k_seed_bucket(const int32_t* __restrict__ seeds, int64_t n, const int64_t* __restrict__ grow,
-                              int32_t fL, int32_t F, uint8_t* __restrict__ bucket) {
+                              int64_t N, int32_t fL, int32_t F, uint8_t* __restrict__ bucket) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     int64_t v = seeds[i];
+    if (v < 0 || v >= N) { bucket[i] = 0; continue; }     // rejected by k_check_ids (no read)
     int64_t deg = grow[v + 1] - grow[v];
     int64_t D = (fL > 0 && deg > fL) ? fL : deg;
     bucket[i] = (uint8_t)(D < F ? D : F);
@@ -564,14 +667,20 @@ buffalo_status seed_bucketing(const buffalo_graph* g, const int32_t* seeds, int6
     for (int b = 0; b <= F; ++b) hist_h[b] = 0;
     return BUFFALO_OK;
   }
-  k_seed_bucket<<<grid_for(n, 256), 256, 0, s>>>(seeds, n, g->row_ptr, fL, F, bucket);
+  // input validation (include/buffalo.h): ids in [0, N), no id twice; the error word is read
+  // back with the bucket starts (one synchronisation)
+  int32_t* err_dev = starts_dev + 257;
+  BF_CUDA(cudaMemsetAsync(err_dev, 0, sizeof(int32_t), s));
+  BF_CHECK(check_ids(g, seeds, n, err_dev, s));
+  k_seed_bucket<<<grid_for(n, 256), 256, 0, s>>>(seeds, n, g->row_ptr, g->num_nodes, fL, F, bucket);
   BF_LAUNCHED("k_seed_bucket");
   BF_CHECK(stable_partition(BucketKey{bucket}, BucketEmit{seeds, order, sorted_ids}, n, counts, ws, s));
   k_bin_starts<<<1, 256, 0, s>>>(counts, part_tiles(n), F + 1, (int32_t)n, starts_dev);
   BF_LAUNCHED("k_bin_starts");
   int32_t st[258];
-  BF_CUDA(cudaMemcpyAsync(st, starts_dev, sizeof(int32_t) * (F + 2), cudaMemcpyDeviceToHost, s));
+  BF_CUDA(cudaMemcpyAsync(st, starts_dev, sizeof(int32_t) * 258, cudaMemcpyDeviceToHost, s));
   BF_CUDA(cudaStreamSynchronize(s));
+  BF_CHECK(ids_error(st[257], "seeds"));
   for (int b = 0; b <= F; ++b) hist_h[b] = st[b + 1] - st[b];
   return BUFFALO_OK;
 }

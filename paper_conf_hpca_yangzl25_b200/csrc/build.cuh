@@ -46,6 +46,13 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
                            buffalo_block* blk, cudaStream_t s, const int64_t* known = nullptr,
                            bool t1 = false, const int32_t* cache = nullptr);
 
+// Input validation: ids in [0, N) and distinct (err_dev |= 1 / 2, stream-ordered, graph
+// bitmap left cleared); ids_error maps the word to a status; validate_graph checks the CSR
+// (synchronises once).
+buffalo_status check_ids(const buffalo_graph* g, const int32_t* ids, int64_t n, int32_t* err_dev, cudaStream_t s);
+buffalo_status ids_error(int32_t err, const char* what);
+buffalo_status validate_graph(const buffalo_graph* g, int sym, cudaStream_t s);
+
 // Degree bucketing of the seeds (Alg. 3 l.1): bucket[i] = min(D(seed_i), F); order = seed
 // positions grouped by bucket (stable); sorted_ids = seeds[order]; hist_h[0..F].
 buffalo_status seed_bucketing(const buffalo_graph* g, const int32_t* seeds, int64_t n, int32_t fL,

@@ -694,11 +694,7 @@ buffalo_status tc_dw_tma(int64_t n, int S, const __nv_bfloat16* z, int64_t ldz, 
   const int stage = (2 * p.MT + p.NT / 64) * kDwStrip2;
   p.nstages = std::max(2, std::min(6, (200 * 1024) / stage));
   const int smem = p.nstages * stage + 16 * p.nstages + 64 + 1024;
-  static bool attr = false;
-  if (!attr) {
-    BF_CUDA(cudaFuncSetAttribute(k_tc_dw_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
-    attr = true;
-  }
+  BF_CHECK(set_max_smem_once(k_tc_dw_tma, 227 * 1024));
   dim3 grid((unsigned)ceil_div(2 * Dp, p.NT), (unsigned)S);
   k_tc_dw_tma<<<grid, kDwThreads2, smem, s>>>(zm, sm, am, p);
   BF_LAUNCHED("k_tc_dw_tma");
@@ -737,7 +733,6 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   const int misc = 16 * 8 + 48 + 4 * p.Np + 1024;                    // barriers, slot, bias, alignment
   p.nsplit = 1;
   p.w_res = (227 * 1024 - w_all - kStaging - misc) / kChunkA >= 4 ? 1 : 0;
-  if (getenv("BUFFALO_GEMM_STREAM_W")) p.w_res = 0;                  // A/B switch (diagnostic)
   p.Nsub = p.Np / p.nsplit;
   p.db_parts = (int)gemm_grid(n_rows);
   int cols = 32;
@@ -773,12 +768,8 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
     om = am;                                                          // unused (fp32 rows stored directly)
     om2 = am;
   }
-  static bool attr = false;
-  if (!attr) {
-    BF_CUDA(cudaFuncSetAttribute(k_tc_gemm_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
-    BF_CUDA(cudaFuncSetAttribute(k_tc_gemm_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
-    attr = true;
-  }
+  BF_CHECK(set_max_smem_once(k_tc_gemm_tma<false>, 227 * 1024));
+  BF_CHECK(set_max_smem_once(k_tc_gemm_tma<true>, 227 * 1024));
   const int64_t sets = std::min<int64_t>(ceil_div(n_rows, kTM), 148 / p.nsplit);
   const int grid = (int)(sets * p.nsplit);
   if (epi) k_tc_gemm_tma<true><<<grid, kGemmThreads, smem, s>>>(sm, am, om, om2, p);

@@ -157,9 +157,6 @@ struct TcFwdParams {
   const __nv_bfloat16* agg_src;  // MODE 2: the aggregate half, bf16 rows [n_dst][ld_agg_src]
   int64_t ld_agg_src;
   int a_chunks, nb;          // K-chunks per A buffer (2 buffers), weight stages
-  int64_t heavy_base;        // MODE 1: positions >= heavy_base are long-tail rows, pre-summed
-  const __nv_bfloat16* heavy_buf;  // MODE 1: [pos - heavy_base][heavy_ld]
-  int64_t heavy_ld;
   int d_in, pitch_in;        // pitch_in: valid columns readable in a row (multiple of 8)
   int nkc_self, nkc;         // K-chunks for the self half, total (= 2 nkc_self)
   const uint8_t* wpk;        // pre-swizzled bf16 W chunks, each Np x 128 B
@@ -249,15 +246,15 @@ template <int E> struct Sched {
   }
 };
 
-// MODE 0: forward (mean of neighbour rows, long-tail rows pre-aggregated, h_agg saved,
-//         + bias, ReLU; tile rows taken in degree-sorted order through `perm`).
-// MODE 1: backward dH (plain sum of pre-scaled dZ/D rows over the transposed block, self half
-//         = dZ for rows < self_rows, fp32 output, natural row order).
-template <class TI, int MODE>
-__global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p) {
+// Update GEMM for an fp32 feature table (layer 1, gemm_mode BF16): the self half is read from
+// the fp32 rows and rounded to bf16 into the swizzled A tile, the aggregate half (the bf16
+// h_agg written by the gather) is copied with cp.async; one elected lane issues tcgen05.mma
+// into a double-buffered TMEM accumulator; the epilogue adds the bias, applies ReLU and stores.
+// (bf16 tables take the TMA kernel of tc_gemm.cu.)
+template <class TI>
+__global__ void __launch_bounds__(kThreads, 1) k_tc_update_copy(const TcFwdParams p) {
   constexpr int E = InTraits<TI>::kElems;      // elements per 16-B piece
   constexpr int P = kKC / E;                   // pieces per 64-column chunk row (8 or 16)
-  constexpr int kUnroll = 8;                   // independent 16-B loads in flight per lane
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const int AC = p.a_chunks, NB = p.nb;                        // chunks per A buffer, B stages
@@ -275,7 +272,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t ntiles = (p.n_dst + kTileM - 1) / kTileM;
-  const Sched<E> sched(p.nkc_self, p.nkc, AC, MODE == 2);
+  const Sched<E> sched(p.nkc_self, p.nkc, AC, true);
   const int nsc = sched.count();
 
   if (threadIdx.x == 0) {
@@ -421,7 +418,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
               st_swz<E>(abuf + (pc / P) * kChunkBytesA, r, pc % P, v);
             }
           }
-        } else if (MODE == 2) {
+        } else {
           // aggregate half precomputed (bf16 rows): plain copy
           const int cb = (c0 - p.nkc_self) * kKC;
           const int pcs = ncs * 8;
@@ -434,116 +431,20 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_sage_fwd(const TcFwdParams p
             cp_async16(abuf + (pc >> 3) * kChunkBytesA + off,
                        ok ? (const void*)(p.agg_src + row_of(pos) * p.ld_agg_src + col0) : (const void*)p.agg_src, ok);
           }
-        } else if (MODE != 2) {
-          // aggregate: one lane group per destination row, lane = 16-B column piece
-          const int cbase = (c0 - p.nkc_self) * kKC;                 // first column of this slice
-          const int need = min(ncs * P, (p.pitch_in - cbase + E - 1) / E);
-          int pact = 1;
-          while (pact < need) pact <<= 1;                            // lanes per row (<= 32)
-          const int G = 32 / pact;                                   // rows per warp step
-          const int grp_id = lane / pact, pc = lane % pact;
-          const int col0 = cbase + pc * E;
-          const bool colok = pc < need && col0 < p.pitch_in;
-          for (int rb = warp * G; rb < kTileM; rb += kGatherWarps * G) {
-            const int r = rb + grp_id;
-            const int64_t pos = pos0 + r;
-            const int64_t row = (r < kTileM && pos < p.n_dst) ? row_of(pos) : -1;
-            int32_t b = 0, e_end = 0;
-            if (row >= 0) { b = __ldg(p.row_ptr + row); e_end = __ldg(p.row_ptr + row + 1); }
-            const int32_t D = e_end - b;
-            const bool heavy = (MODE == 0) ? (D > kHeavyT) : (row >= 0 && pos >= p.heavy_base);
-            float acc[E];
-#pragma unroll
-            for (int k = 0; k < E; ++k) acc[k] = 0.f;
-            const int32_t Dl = heavy ? 0 : D;
-            const int32_t Dmax = __reduce_max_sync(0xffffffffu, Dl);
-            for (int32_t base = 0; base < Dmax; base += pact) {
-              const int32_t jj = (base + pc < Dl) ? __ldg(p.col + b + base + pc) : 0;
-              const int lim = min(pact, Dmax - base);
-              for (int u = 0; u < lim; u += kUnroll) {
-                uint4 raw[kUnroll];
-#pragma unroll
-                for (int uu = 0; uu < kUnroll; ++uu) {
-                  const int tt = u + uu;
-                  const int32_t jn = __shfl_sync(0xffffffffu, jj, (grp_id * pact + (tt & (pact - 1))) & 31);
-                  raw[uu] = make_uint4(0u, 0u, 0u, 0u);
-                  if (tt < pact && base + tt < Dl && colok)
-                    raw[uu] = __ldg(reinterpret_cast<const uint4*>(h + (int64_t)jn * p.ldh + col0));
-                }
-#pragma unroll
-                for (int uu = 0; uu < kUnroll; ++uu) {
-                  float v[E];
-                  raw_to_f32<TI>(raw[uu], v);
-#pragma unroll
-                  for (int k = 0; k < E; ++k) acc[k] += v[k];
-                }
-              }
-            }
-            if (r < kTileM && pc < ncs * P) {
-              if (heavy) {
-                // long-tail row: pre-aggregated by k_agg_heavy into the saved h_agg (bf16)
-                if (colok) {
-                  const __nv_bfloat16* src = (MODE == 0) ? p.agg + row * p.ld_agg + col0
-                                                         : p.heavy_buf + (pos - p.heavy_base) * p.heavy_ld + col0;
-                  if constexpr (E == 8) {
-                    bf16x8_to_f32(*reinterpret_cast<const uint4*>(src), acc);
-                  } else {
-                    uint2 w = *reinterpret_cast<const uint2*>(src);
-                    acc[0] = __uint_as_float(w.x << 16); acc[1] = __uint_as_float(w.x & 0xffff0000u);
-                    acc[2] = __uint_as_float(w.y << 16); acc[3] = __uint_as_float(w.y & 0xffff0000u);
-                  }
-                }
-              } else {
-                if (MODE == 0) {
-                  const float fd = (float)D;
-#pragma unroll
-                  for (int k = 0; k < E; ++k) acc[k] = D > 0 ? acc[k] / fd : 0.f;
-                }
-                if (MODE == 0 && row >= 0 && colok) {
-                  __nv_bfloat16* dstp = p.agg + row * p.ld_agg + col0;
-                  if constexpr (E == 8) {
-                    *reinterpret_cast<uint4*>(dstp) =
-                        make_uint4(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]),
-                                   pack_bf16x2(acc[4], acc[5]), pack_bf16x2(acc[6], acc[7]));
-                  } else {
-                    *reinterpret_cast<uint2*>(dstp) = make_uint2(pack_bf16x2(acc[0], acc[1]),
-                                                                 pack_bf16x2(acc[2], acc[3]));
-                  }
-                }
-              }
-              st_swz<E>(abuf + (pc / P) * kChunkBytesA, r, pc % P, acc);
-            }
-          }
-          // pieces of this slice beyond pact (zero columns past the row pitch)
-          for (int u = threadIdx.x; u < kTileM * ncs * P; u += kGatherThreads) {
-            const int r = u / (ncs * P), pcz = u % (ncs * P);
-            if (pcz >= pact) {
-              float z[E];
-#pragma unroll
-              for (int k = 0; k < E; ++k) z[k] = 0.f;
-              st_swz<E>(abuf + (pcz / P) * kChunkBytesA, r, pcz % P, z);
-            }
-          }
         }
-        if (MODE == 2) {
-          // copy-only tiles: keep two super-chunks of cp.async in flight; super-chunk q-1 is
-          // handed to the MMA once its copies landed
-          cp_async_commit();
-          if (q > 0) {
-            cp_async_wait<1>();
-            fence_proxy_async_smem();
-            mbar_arrive(&a_full[(q - 1) & 1]);
-          }
-        } else {
-          asm volatile("cp.async.wait_all;" ::: "memory");
+        // keep two super-chunks of cp.async in flight; super-chunk q-1 is handed to the MMA
+        // once its copies landed
+        cp_async_commit();
+        if (q > 0) {
+          cp_async_wait<1>();
           fence_proxy_async_smem();
-          mbar_arrive(&a_full[buf]);
+          mbar_arrive(&a_full[(q - 1) & 1]);
         }
       }
       if (prev_tile >= 0) epilogue(prev_tile, i - 1);
       prev_tile = t;
     }
-    if (MODE == 2 && q > 0) {
+    if (q > 0) {
       cp_async_wait<0>();
       fence_proxy_async_smem();
       mbar_arrive(&a_full[(q - 1) & 1]);
@@ -765,10 +666,7 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   while ((1 << lpr_log) < npieces && lpr_log < 5) ++lpr_log;
   // transposed rows are short (~1-2 entries per src row): two rows per warp (two passes over
   // the row's pieces) keep twice the per-row metadata chains in flight
-  if (MODE == 1 && lpr_log == 5) {
-    const char* ev = getenv("BUFFALO_T_LPR_LOG");      // diagnostic override (A/B runs)
-    lpr_log = ev ? atoi(ev) : 4;
-  }
+  if (MODE == 1 && lpr_log == 5) lpr_log = 4;
   if (n > INT32_MAX || ldh * (int64_t)sizeof(TI) > INT32_MAX) {
     set_error("gather: %lld rows of stride %lld elements exceed the 32-bit row / byte-stride range",
               (long long)n, (long long)ldh);
@@ -798,45 +696,18 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
 // largest row count TMA accepts and tile padding rows gather row 0 (their outputs are dropped).
 constexpr int64_t kGatherTableRows = 0x7fffffff;
 
-static bool use_cpasync_gemm() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("BUFFALO_CPASYNC_GEMM");
-    v = (e && e[0] == '1') ? 1 : 0;
-  }
-  return v == 1;
-}
-
-static bool use_fused() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("BUFFALO_FUSED");
-    v = (e && e[0] == '1') ? 1 : 0;
-  }
-  return v == 1;
-}
-
-template <class TI, int MODE>
-static buffalo_status launch_tc(TcFwdParams p, cudaStream_t s) {
-  if (MODE == 2) {
-    // copy mode: small A buffers, deep weight prefetch (the weights stream once per tile)
-    p.a_chunks = 2;
-    const int budget = 220 * 1024 - smem_bytes_for(p.Np, 2, 0);
-    p.nb = std::max(2, std::min(8, budget / (p.Np * 128)));
-  } else {
-    p.a_chunks = kSuper;
-    p.nb = 2;
-  }
+template <class TI>
+static buffalo_status launch_tc_copy(TcFwdParams p, cudaStream_t s) {
+  // small A buffers, deep weight prefetch (the weights stream once per tile)
+  p.a_chunks = 2;
+  const int budget = 220 * 1024 - smem_bytes_for(p.Np, 2, 0);
+  p.nb = std::max(2, std::min(8, budget / (p.Np * 128)));
   const int smem = smem_bytes_for(p.Np, p.a_chunks, p.nb);
-  static bool attr_set = false;
-  if (!attr_set) {
-    BF_CUDA(cudaFuncSetAttribute(k_tc_sage_fwd<TI, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
-    attr_set = true;
-  }
+  BF_CHECK(set_max_smem_once(k_tc_update_copy<TI>, 227 * 1024));
   const int64_t ntiles = ceil_div(p.n_dst, kTileM);
   const int grid = (int)std::min<int64_t>(ntiles, 148);
-  k_tc_sage_fwd<TI, MODE><<<grid, kThreads, smem, s>>>(p);
-  BF_LAUNCHED(MODE == 0 ? "k_tc_sage_fwd" : MODE == 1 ? "k_tc_sage_bwd_dh" : "k_tc_update_gemm");
+  k_tc_update_copy<TI><<<grid, kThreads, smem, s>>>(p);
+  BF_LAUNCHED("k_tc_update_copy");
   return BUFFALO_OK;
 }
 
@@ -877,18 +748,17 @@ static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   p.out = a.out;
   p.agg = (__nv_bfloat16*)a.agg;
   p.ld_agg = a.ld_agg;
-  if (use_fused()) return launch_tc<TI, 0>(p, s);
-  // split: high-occupancy gather of the non-heavy rows, then the Update GEMM over copies
+  // high-occupancy gather of the non-heavy rows, then the Update GEMM over copies
   BF_CHECK((launch_gather<TI, 0>(blk->cls_perm, blk->row_ptr, p.col, blk->n_dst, (const TI*)a.h_src, a.ld_src,
                                  p.pitch_in, (__nv_bfloat16*)a.agg, a.ld_agg, s)));
-  if (a.in_bf16 && !use_cpasync_gemm())
+  if (a.in_bf16)
     return tc_gemm_tma(blk->n_dst, a.layer1 ? kGatherTableRows : blk->n_dst, a.layer1 ? blk->src_global : nullptr,
                        (const __nv_bfloat16*)a.h_src, a.ld_src, (const __nv_bfloat16*)a.agg, a.ld_agg,
                        a.d_in, p.wpk, a.d_out, a.b, a.relu, a.out_f32, a.out, a.ld_out, s);
   p.perm = nullptr;
   p.agg_src = (const __nv_bfloat16*)a.agg;
   p.ld_agg_src = a.ld_agg;
-  return launch_tc<TI, 2>(p, s);
+  return launch_tc_copy<TI>(p, s);
 }
 
 buffalo_status tc_sage_fwd(const FwdArgs& a, cudaStream_t s) {
@@ -1314,9 +1184,8 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     w.part = dw_part;
     const int smem = kDwStages * (2 * w.MT + w.NT / 64) * kDwStrip + 128 + 1024;
     dim3 grid((unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
-    static bool attr = false;
     constexpr int kMaxDwSmem = kDwStages * (4 + 4) * kDwStrip + 128 + 1024;
-    if (!attr) { BF_CUDA(cudaFuncSetAttribute(k_tc_dw<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDwSmem)); attr = true; }
+    BF_CHECK(set_max_smem_once(k_tc_dw<float>, kMaxDwSmem));
     k_tc_dw<float><<<grid, kDwThreads, smem, s>>>(w);
     BF_LAUNCHED("k_tc_dw");
   }

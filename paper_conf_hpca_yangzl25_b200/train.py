@@ -156,7 +156,10 @@ class Trainer:
         self.graph = graph if isinstance(graph, DeviceGraph) else DeviceGraph(*graph, device=device)
         self.feats = feats
         self.labels = labels
-        self.seeds = seeds
+        if not (seeds.is_cuda and seeds.dtype == torch.int32 and labels.dtype == torch.int32):
+            raise TypeError("seeds and labels must be int32 CUDA tensors")
+        self._seeds = [seeds]
+        self._seeds_version = 0
         self.S = seeds.numel()
         self.dims = list(dims)
         self.L = len(dims) - 1
@@ -187,6 +190,7 @@ class Trainer:
         self._ahead = None
         if pipeline:
             self._pb.append(PlanBuffers(self.S, k_max, F, self.L, device))
+            self._seeds.append(torch.empty_like(seeds))       # the seed batch the ahead plan is for
             self._side = torch.cuda.Stream(device=device)
         # sample cache per plan-buffer set (include/buffalo.h): the scheduler's first statistics
         # pass stores every sampled neighbour list of the batch, the build copies them
@@ -202,7 +206,8 @@ class Trainer:
         self.blocks = B.Blocks()
         self.last = {}
 
-    # plan of the current epoch (the buffer set in use)
+    # plan of the current epoch (the buffer set in use) and the seed batch it was made for
+    seeds = property(lambda self: self._seeds[self._cur])
     group_of_seed = property(lambda self: self._pb[self._cur].group_of_seed)
     group_seeds = property(lambda self: self._pb[self._cur].group_seeds)
     group_offsets = property(lambda self: self._pb[self._cur].group_offsets)
@@ -225,11 +230,29 @@ class Trainer:
         self._ahead = None
         return self._schedule_into(self._cur, epoch, self.graph.g)
 
+    def set_seeds(self, seeds):
+        """Replaces the seed batch (a device or pinned host int32 tensor of the same size).  A plan
+        computed ahead for the old batch is dropped, so the next epoch schedules the new one."""
+        if seeds.numel() != self.S or seeds.dtype != torch.int32:
+            raise ValueError("set_seeds: expected int32 seeds of the trainer's batch size")
+        self.seeds.copy_(seeds, non_blocking=True)
+        self._seeds_version += 1
+        self._ahead = None
+
+    def fixed_bytes(self):
+        """Device bytes the trainer holds outside the micro-batch arena (graph workspaces,
+        scheduler workspace, plan buffers, sample caches, seeds, parameters and gradients)."""
+        ts = [self.graph.ws, self.graph._sched_ws, self.bucket_ws, self.loss, self.params.flat, self.params.grad]
+        ts += [t for t in self._seeds] + [p for p in self.params.packed if p is not None]
+        ts += [c for cs in self._cache for c in cs if c is not None]
+        ts += [t for pb in self._pb for t in (pb.group_of_seed, pb.group_seeds, pb.group_offsets)]
+        return int(sum(t.numel() * t.element_size() for t in ts if t is not None))
+
     def _schedule_into(self, buf, epoch, g):
         pb = self._pb[buf]
         self._cache_epoch[buf] = None
         sp = B.make_sampler(self.fanout, self.F, self.base_seed + epoch, self._cache[buf])
-        B.bucketize(g, self.seeds, sp, self.model, self.sched, pb.plan, self.bucket_ws)
+        B.bucketize(g, self._seeds[buf], sp, self.model, self.sched, pb.plan, self.bucket_ws)
         self._cache_epoch[buf] = epoch
         K = pb.plan.k_out
         return K, pb.offs_h[:K + 1].copy(), pb.est_h[:K].copy(), pb.rank_h[:K].copy()
@@ -318,6 +341,48 @@ class Trainer:
                     e=[blk.layer[l].n_edges for l in range(self.L)],
                     peak=blk.arena_peak, est_lo=blk.est_lo, est_hi=blk.est_hi)
 
+    # a 4-byte word no kernel writes: a NaN payload in fp32, a NaN high half in bf16, and an int32
+    # above every node id / offset of a micro-batch
+    HW_SENTINEL = 0x7FBADF00
+
+    def measure_high_water(self, k, epoch, guard=1 << 20):
+        """Measured arena high-water mark of group k (independent of the memory model): the arena
+        is filled with HW_SENTINEL, the library is handed exactly lo = buffalo_estimate_mem's
+        exact need of the group, and after build + forward + loss + backward the highest word
+        that no longer holds the sentinel gives the bytes actually touched (a `guard` of sentinel
+        words past lo must stay intact).  Accumulates into the gradients like microbatch().
+        Returns (high_water_bytes, lo, hi, guard_intact)."""
+        L = self.L
+        sizes = self.sizes_h[k]
+        lo, hi = B.estimate_mem(sizes[:L + 1], sizes[L + 1:], self.model)
+        total = (lo + guard + 255) // 256 * 256
+        self._ensure_arena(total)
+        keep = self.arena
+        words = keep[:total].view(torch.int32)
+        words.fill_(self.HW_SENTINEL)
+        self.arena = keep[:lo]
+        try:
+            offs = self.offs_h
+            self.microbatch(int(offs[k]), int(offs[k + 1] - offs[k]), self.sampler(epoch), sizes)
+        finally:
+            self.arena = keep
+        torch.cuda.synchronize()
+        changed = words != self.HW_SENTINEL
+        CH = 1 << 16
+        full = changed.numel() // CH * CH
+        last = -1
+        if changed.numel() > full and bool(changed[full:].any()):
+            last = full + int(torch.nonzero(changed[full:]).max())
+        elif full:
+            hit = torch.nonzero(changed[:full].view(-1, CH).any(dim=1))
+            if hit.numel():
+                c = int(hit.max())
+                last = c * CH + int(torch.nonzero(changed[c * CH:(c + 1) * CH]).max())
+        hw = 4 * (last + 1)
+        guard_ok = not bool(changed[(lo + 3) // 4:].any())
+        del changed
+        return hw, lo, hi, guard_ok
+
     def allreduce(self):
         allreduce_grads(self.params.grad, self.world, self.pg)
 
@@ -325,14 +390,16 @@ class Trainer:
         B.sgd_step(self.params.flat, self.params.grad, lr)
         self.params.repack()
 
-    def run_epoch(self, epoch=0, lr=0.01, timers=False):
+    def run_epoch(self, epoch=0, lr=0.01, timers=False, next_seeds=None):
         """One Buffalo iteration; returns stats (K, own groups, aggregated edges, ...).
-        pipeline=True: the plan was computed during the previous call (if it was for this epoch),
-        and the next epoch's plan is computed on the side stream while this epoch's work runs."""
+        pipeline=True: the plan was computed during the previous call (if it was for this epoch
+        and the seed batch has not been replaced since), and the next epoch's plan is computed on
+        the side stream while this epoch's work runs — for `next_seeds` (a pinned host or device
+        int32 tensor, copied on the side stream) if given, else for the current batch."""
         main = torch.cuda.current_stream()
         a = self._ahead
         self._ahead = None
-        if self.pipeline and a is not None and a["epoch"] == epoch:
+        if self.pipeline and a is not None and a["epoch"] == epoch and a["version"] == self._seeds_version:
             self._cur = a["buf"]
             main.wait_event(a["done"])
             K, offs, est, ranks = a["K"], a["offs"], a["est"], a["ranks"]
@@ -359,7 +426,15 @@ class Trainer:
             nb = 1 - self._cur
             self._side.wait_event(before)
             with torch.cuda.stream(self._side):
+                if next_seeds is not None:
+                    if next_seeds.numel() != self.S or next_seeds.dtype != torch.int32:
+                        raise ValueError("next_seeds: expected int32 seeds of the trainer's batch size")
+                    self._seeds[nb].copy_(next_seeds, non_blocking=True)
+                    self._seeds_version += 1
+                else:
+                    self._seeds[nb].copy_(self._seeds[self._cur])
                 Kn, offn, estn, rankn = self._schedule_into(nb, epoch + 1, self.graph.g_sched)
                 done = self._side.record_event()
-            self._ahead = dict(epoch=epoch + 1, buf=nb, K=Kn, offs=offn, est=estn, ranks=rankn, done=done)
+            self._ahead = dict(epoch=epoch + 1, buf=nb, K=Kn, offs=offn, est=estn, ranks=rankn, done=done,
+                               version=self._seeds_version)
         return self.last

@@ -72,6 +72,28 @@ def test_products_plan(products):
     assert np.all(est <= products["budget"])
 
 
+@pytest.mark.slow
+def test_products_plan_equals_oracle_schedule(products):
+    """The full-size plan (products-shaped only: the oracle's C builder makes every item's blocks
+    on the host) equals oracle.schedule run at the K the library settled on, and the same
+    procedure fails at K - 1 (Alg. 3 keeps the first feasible K)."""
+    if products["cfg"].N > 10_000_000:
+        pytest.skip("papers100M-shaped: the host oracle would build ~60 full-size item blocks")
+    tr, cfg = products["tr"], products["cfg"]
+    Kt = tr.plan.k_tried
+    seeds = tr.seeds.cpu().numpy()
+    kw = dict(act_dtype=O.BF16, mem_budget=products["budget"], C_ppm=0)
+    ref = O.schedule(products["g"], seeds, tr.L, cfg.fanout, cfg.F, tr.base_seed + 0, cfg.dims, k_min=Kt, k_max=Kt,
+                     **kw)
+    assert ref is not None and ref["K"] == products["K"] and ref["exploded"] == bool(tr.plan.exploded)
+    np.testing.assert_array_equal(products["offs"], ref["group_offsets"])
+    np.testing.assert_array_equal(products["est"], ref["est_bytes"])
+    np.testing.assert_array_equal(tr.group_seeds.cpu().numpy(), ref["group_seeds"])
+    if Kt > 1:
+        assert O.schedule(products["g"], seeds, tr.L, cfg.fanout, cfg.F, tr.base_seed + 0, cfg.dims, k_min=Kt - 1,
+                          k_max=Kt - 1, **kw) is None
+
+
 def _group_blocks(products, k, seed=0):
     """Builds group k with the sampling seed of the planned epoch (seed 0): the plan's exact
     block sizes (tr.sizes_h, passed for the sync-free build) are those of that sampling."""

@@ -258,6 +258,70 @@ def test_microbatch_fwd_bwd_parity(name, gemm):
     assert lo <= info["peak"] <= hi
 
 
+@pytest.mark.parametrize("name", list(CASES))
+def test_bf16_layer_outputs_vs_plain_fp64(name):
+    """bf16 mode against the PLAIN float64 oracle (no bf16 rounding anywhere in the reference),
+    layer by layer and fed the same inputs: for each layer l the reference takes the GPU's own
+    layer input H_{l-1} (the feature table at l = 1) and computes h_agg = D^-1 A H_{l-1} and
+    Z_l = [H_self || h_agg] W_l^T + b_l in float64 with the fp32 master weights; the GPU's H_l
+    (= ReLU(Z_l) stored in bf16) and logits must match elementwise within the north star's
+    rel 2e-2 (+ 2e-2 rms floor).  Feeding each layer the GPU's input keeps
+    near-zero pre-activations of earlier layers from compounding (R26)."""
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case(name)
+    g = O.Graph(rp, col)
+    L = len(fan)
+    tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, gemm=B.GEMM_BF16, feat_dtype=B.BF16)
+    _run_microbatch(tr, seeds, fan, F, 7)
+    blocks = O.build_blocks(g, seeds, L, fan, 7)
+    H = np.asarray(X, np.float64)[blocks[0]["src_global"]][:, :dims[0]]
+    for l in range(1, L + 1):
+        b = tr.blocks.layer[l - 1]
+        A = O.mean_adjacency(blocks[l - 1])
+        agg = A @ H
+        W = np.asarray(Ws[l - 1], np.float64)
+        d_in = dims[l - 1]
+        Z = H[: b.n_dst] @ W[:, :d_in].T + agg @ W[:, d_in:].T + np.asarray(bs[l - 1], np.float64)
+        if l < L:
+            got = act_view(tr.arena, b.out, b.n_dst, b.ld_out, torch.bfloat16)[:, :dims[l]]
+            assert_bf16_close(got, np.maximum(Z, 0.0), f"H_{l} vs plain fp64")
+            H = got.astype(np.float64)                 # the GPU's layer input for the next layer
+        else:
+            got = act_view(tr.arena, b.out, b.n_dst, b.ld_out, torch.float32)[:, :dims[l]]
+            assert_bf16_close(got, Z, "logits vs plain fp64")
+
+
+@pytest.mark.parametrize("name", ["sampled2", "mixed3"])
+def test_ffma_general_fp32_features(name):
+    """FFMA mode on Gaussian fp32 features (not the k/128 grid, so fp32 sums round and their
+    order matters) against the float64 oracle at rel 1e-4 / abs 1e-5: h_agg of every layer,
+    logits, loss and all gradients."""
+    rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case(name)
+    g = O.Graph(rp, col)
+    L = len(fan)
+    Xg = np.random.default_rng(5).standard_normal(X.shape).astype(np.float32)
+    tr = make_trainer(rp, col, Xg, y, seeds, dims, fan, F, Ws, bs)
+    _run_microbatch(tr, seeds, fan, F, 7)
+    blocks = O.build_blocks(g, seeds, L, fan, 7)
+    logits, cache = O.sage_forward(blocks, Xg, Ws, bs)
+    loss, dlog = O.softmax_ce(logits, y[seeds], seeds.size)
+    grads = O.sage_backward(blocks, cache, Ws, dlog)
+    H = np.asarray(Xg, np.float64)[blocks[0]["src_global"]][:, :dims[0]]
+    for l in range(1, L + 1):
+        b = tr.blocks.layer[l - 1]
+        agg = act_view(tr.arena, b.agg, b.n_dst, b.ld_agg, torch.float32)[:, :dims[l - 1]]
+        ref_agg = O.mean_adjacency(blocks[l - 1]) @ H
+        assert_close(agg, ref_agg, 1e-4, 1e-5, f"h_agg layer {l}")
+        if l < L:
+            H = act_view(tr.arena, b.out, b.n_dst, b.ld_out, torch.float32)[:, :dims[l]].astype(np.float64)
+    bl = tr.blocks.layer[L - 1]
+    assert_close(act_view(tr.arena, bl.out, bl.n_dst, bl.ld_out, torch.float32)[:, :dims[-1]], logits, 1e-4, 1e-5,
+                 "logits")
+    assert abs(tr.loss.item() - loss) <= 1e-5 + 1e-4 * abs(loss)
+    for l in range(L):
+        assert_close(tr.params.dW[l].cpu().numpy(), grads[l][0], 1e-4, 1e-5, f"dW{l + 1}")
+        assert_close(tr.params.db[l].cpu().numpy(), grads[l][1], 1e-4, 1e-5, f"db{l + 1}")
+
+
 def test_mean_of_constant_is_constant():
     rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case("full3")
     Xc = np.full_like(X, 0.5)
