@@ -503,7 +503,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
       if (hg > 0) {
         const int64_t words = ceil_div(n_dst, 32);
         if (words <= kBitsortMaxWords) {
-          BF_CHECK(set_max_smem_once(k_tsort_heavy_bits, kBitsortMaxWords * 4));
+          BF_CHECK(set_max_smem_once<k_tsort_heavy_bits>(kBitsortMaxWords * 4));
           k_tsort_heavy_bits<<<hg, 256, words * 4, s>>>(tperm, n_src, trp, tcol, (int32_t)words);
           BF_LAUNCHED("k_tsort_heavy_bits");
         } else {
@@ -678,7 +678,8 @@ buffalo_status seed_bucketing(const buffalo_graph* g, const int32_t* seeds, int6
   k_bin_starts<<<1, 256, 0, s>>>(counts, part_tiles(n), F + 1, (int32_t)n, starts_dev);
   BF_LAUNCHED("k_bin_starts");
   int32_t st[258];
-  BF_CUDA(cudaMemcpyAsync(st, starts_dev, sizeof(int32_t) * 258, cudaMemcpyDeviceToHost, s));
+  BF_CUDA(cudaMemcpyAsync(st, starts_dev, sizeof(int32_t) * (F + 2), cudaMemcpyDeviceToHost, s));
+  BF_CUDA(cudaMemcpyAsync(st + 257, err_dev, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
   BF_CUDA(cudaStreamSynchronize(s));
   BF_CHECK(ids_error(st[257], "seeds"));
   for (int b = 0; b <= F; ++b) hist_h[b] = st[b + 1] - st[b];

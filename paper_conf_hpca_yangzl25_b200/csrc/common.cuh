@@ -69,17 +69,18 @@ inline int grid_for(int64_t work_items, int per_block, int blocks_per_sm = 8) {
 // sm_100a check of the current device.
 buffalo_status require_sm100();
 
-// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once per (kernel, device).  The attribute
-// is per device, so the done-mask has one bit per device ordinal; the mask is an idempotent
-// cache (two threads racing both set the same attribute), not state that changes results.
-template <class Kern>
-inline buffalo_status set_max_smem_once(Kern* kernel, int bytes) {
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once per (kernel, device): the kernel is a
+// template argument, so every kernel has its own done-mask (one bit per device ordinal: the
+// attribute is per device).  The mask is an idempotent cache (two threads racing both set the
+// same attribute), not state that changes results.
+template <auto Kern>
+inline buffalo_status set_max_smem_once(int bytes) {
   static std::atomic<uint64_t> done{0};
   int dev = 0;
   BF_CUDA(cudaGetDevice(&dev));
   const uint64_t bit = dev < 64 ? (1ull << dev) : 0ull;
   if (bit && (done.load(std::memory_order_acquire) & bit)) return BUFFALO_OK;
-  BF_CUDA(cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
+  BF_CUDA(cudaFuncSetAttribute(Kern, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
   done.fetch_or(bit, std::memory_order_release);
   return BUFFALO_OK;
 }

@@ -694,7 +694,7 @@ buffalo_status tc_dw_tma(int64_t n, int S, const __nv_bfloat16* z, int64_t ldz, 
   const int stage = (2 * p.MT + p.NT / 64) * kDwStrip2;
   p.nstages = std::max(2, std::min(6, (200 * 1024) / stage));
   const int smem = p.nstages * stage + 16 * p.nstages + 64 + 1024;
-  BF_CHECK(set_max_smem_once(k_tc_dw_tma, 227 * 1024));
+  BF_CHECK(set_max_smem_once<k_tc_dw_tma>(227 * 1024));
   dim3 grid((unsigned)ceil_div(2 * Dp, p.NT), (unsigned)S);
   k_tc_dw_tma<<<grid, kDwThreads2, smem, s>>>(zm, sm, am, p);
   BF_LAUNCHED("k_tc_dw_tma");
@@ -768,8 +768,8 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
     om = am;                                                          // unused (fp32 rows stored directly)
     om2 = am;
   }
-  BF_CHECK(set_max_smem_once(k_tc_gemm_tma<false>, 227 * 1024));
-  BF_CHECK(set_max_smem_once(k_tc_gemm_tma<true>, 227 * 1024));
+  BF_CHECK(set_max_smem_once<k_tc_gemm_tma<false>>(227 * 1024));
+  BF_CHECK(set_max_smem_once<k_tc_gemm_tma<true>>(227 * 1024));
   const int64_t sets = std::min<int64_t>(ceil_div(n_rows, kTM), 148 / p.nsplit);
   const int grid = (int)(sets * p.nsplit);
   if (epi) k_tc_gemm_tma<true><<<grid, kGemmThreads, smem, s>>>(sm, am, om, om2, p);

@@ -703,7 +703,7 @@ static buffalo_status launch_tc_copy(TcFwdParams p, cudaStream_t s) {
   const int budget = 220 * 1024 - smem_bytes_for(p.Np, 2, 0);
   p.nb = std::max(2, std::min(8, budget / (p.Np * 128)));
   const int smem = smem_bytes_for(p.Np, p.a_chunks, p.nb);
-  BF_CHECK(set_max_smem_once(k_tc_update_copy<TI>, 227 * 1024));
+  BF_CHECK(set_max_smem_once<k_tc_update_copy<TI>>(227 * 1024));
   const int64_t ntiles = ceil_div(p.n_dst, kTileM);
   const int grid = (int)std::min<int64_t>(ntiles, 148);
   k_tc_update_copy<TI><<<grid, kThreads, smem, s>>>(p);
@@ -1185,7 +1185,7 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     const int smem = kDwStages * (2 * w.MT + w.NT / 64) * kDwStrip + 128 + 1024;
     dim3 grid((unsigned)ceil_div(2 * Dp, w.NT), (unsigned)S);
     constexpr int kMaxDwSmem = kDwStages * (4 + 4) * kDwStrip + 128 + 1024;
-    BF_CHECK(set_max_smem_once(k_tc_dw<float>, kMaxDwSmem));
+    BF_CHECK(set_max_smem_once<k_tc_dw<float>>(kMaxDwSmem));
     k_tc_dw<float><<<grid, kDwThreads, smem, s>>>(w);
     BF_LAUNCHED("k_tc_dw");
   }

@@ -2,7 +2,9 @@
 "race detection / failure detection"): memcheck (out-of-bounds and misaligned device accesses,
 also the arena bounds), racecheck (shared-memory hazards: the look-back scan, the partition
 passes, the mbarrier / TMEM pipelines' staging buffers), synccheck (barrier misuse) and initcheck
-(reads of uninitialised device memory).  Each must report 0 errors."""
+(reads of uninitialised device memory; on the paths without TMA stores — initcheck does not see
+global writes made by the tensor-memory-access unit, so every read of a TMA-stored activation
+would be reported).  Each must report 0 errors."""
 import os
 import shutil
 import subprocess
@@ -23,7 +25,9 @@ def test_sanitizer_clean(tool):
     cmd = [SAN, "--tool", tool, "--error-exitcode", "99", "--target-processes", "all"]
     if tool == "memcheck":
         cmd += ["--leak-check", "no"]
-    cmd += [sys.executable, os.path.join(ROOT, "tools", "sanitize_run.py"), "all"]
+    which = "mean_ffma,pool,lstm,gat,clustering" if tool == "initcheck" else "all"
+    cmd += [sys.executable, os.path.join(ROOT, "tools", "sanitize_run.py"), which]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=1500, cwd=ROOT)
     out = r.stdout + r.stderr
-    assert r.returncode == 0 and "ERROR SUMMARY: 0 errors" in out, out[-4000:]
+    clean = "ERROR SUMMARY: 0 errors" in out or "RACECHECK SUMMARY: 0 hazards displayed (0 errors, 0 warnings)" in out
+    assert r.returncode == 0 and clean, out[-4000:]

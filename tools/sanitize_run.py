@@ -18,6 +18,7 @@ from synth.graphs import (features, gat_weights, labels, lstm_weights, pool_weig
 
 
 def main(which):
+    which = set(which.split(","))
     N, dims, fan, F = 1500, [24, 40, 6], [4, 0], 10
     rp, col = random_graph(N, 9000, "powerlaw")
     X, y, seeds = features(N, dims[0]), labels(N, dims[-1]), seed_nodes(N, 300)
@@ -30,7 +31,7 @@ def main(which):
         "lstm": dict(aggregator=B.AGG_LSTM, lstm=lstm_weights(dims)),
     }
     for name, kw in runs.items():
-        if which not in ("all", name):
+        if not ({"all", name} & which):
             continue
         tr = make_trainer(rp, col, X, y, seeds, dims, [4, 6] if name == "lstm" else fan, F, Ws, bs, k_min=2,
                           k_max=2, **kw)
@@ -38,14 +39,14 @@ def main(which):
         tr.run_epoch(epoch=0, lr=0.01)
         torch.cuda.synchronize()
         print(name, "ok", flush=True)
-    if which in ("all", "gat"):
+    if {"all", "gat"} & which:
         Wg, bg, als, ars = gat_weights(dims, bias_scale=0.05)
         tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Wg, bg, k_min=2, k_max=2, aggregator=B.AGG_GAT,
                           gat=(als, ars))
         tr.run_epoch(epoch=0, lr=0.01)
         torch.cuda.synchronize()
         print("gat ok", flush=True)
-    if which in ("all", "clustering"):
+    if {"all", "clustering"} & which:
         T, C, ppm = B.clustering(tr.graph.g)
         torch.cuda.synchronize()
         print("clustering ok", C, flush=True)
