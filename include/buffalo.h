@@ -259,20 +259,20 @@ BUFFALO_API size_t buffalo_sage_bwd_scratch_bytes(const buffalo_block* blk, int3
  * FFMA mode: dh_dst holds dH_l fp32 (l < L; masked IN PLACE using h_dst) or dlogits (l = L);
  * dh_src receives dH_{l-1} fp32.
  * BF16 mode: dh_dst holds dlogits fp32 at l = L; for l < L it holds the layer's prepared
- * backward input as written by the layer above: bf16 dZ_l [n_dst][p(d_l)], then (l >= 2) bf16
- * dZ_l / D_l [n_dst][p(d_l)], then at byte offset R(4 n_dst p(d_l)) fp32 column-sum partials
- * of dZ_l [min(ceil(n_dst/128), 148)][d_l]; dh_src receives the same prepared form of layer
- * l-1 (the Update GEMM's epilogue applies ReLU' with h_src = H_{l-1} and divides by
- * D_{l-1}(j) = prev_row_ptr[j+1] - prev_row_ptr[j]), so the buffer must hold
- * R(4 n_src p(d_{l-1})) + R(4 * 148 * d_{l-1}) bytes.  prev_row_ptr: block l-1's row_ptr (l >= 3
- * in BF16 mode; NULL otherwise).  Pass dh_src = NULL for layer 1 (features are not trained). */
+ * backward input as written by the layer above: bf16 dZ_l [n_dst][p(d_l)], then at byte offset
+ * R(2 n_dst p(d_l)) fp32 column-sum partials of dZ_l [1036][d_l] (summed in row order for db).
+ * For l >= 2 the layer computes Ys = dZ W_self and Yn = (dZ W_neigh) / D over its n_dst rows
+ * (tcgen05), then the transposed Aggregate dH_{l-1}[j] = [j < n_dst] Ys[j] + sum_{i in T(j)} Yn[i]
+ * over the n_src rows with the layer-below epilogue fused: ReLU' with h_src = H_{l-1}, bf16
+ * dZ_{l-1} into dh_src and its column-sum partials, i.e. dh_src receives the same prepared form
+ * of layer l-1 and must hold R(2 n_src p(d_{l-1})) + R(4 * 1036 * d_{l-1}) bytes.
+ * Pass dh_src = NULL for layer 1 (features are not trained). */
 BUFFALO_API buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
                                 float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
                                 const void* saved_agg, int64_t ld_agg, const void* h_dst,
                                 int64_t ld_hdst, const float* W, const void* W_packed,
                                 float* dW_accum, float* db_accum, float* dh_src,
-                                int64_t ld_dh_src, const int32_t* prev_row_ptr, void* scratch,
-                                size_t scratch_bytes, void* stream);
+                                int64_t ld_dh_src, void* scratch, size_t scratch_bytes, void* stream);
 
 /* ------------------------------------------------------------------ GraphSAGE-pool */
 /* the pooling aggregator (the paper's aggregator list "mean, pool or

@@ -198,6 +198,7 @@ FP32, BF16 = 0, 1
 SCAN_TILE = 4096       # elements per tile of the implementation's device-wide scans
 PART_TILE = 4096       # elements per tile of its stable radix/bin partition passes
 DB_SPLITS = 296        # row splits of the bf16 path's deterministic db reduction
+BWD_DB_PARTS = 148 * 6 + 148   # db partial rows of the bf16 backward's fused transposed Aggregate
 
 
 def _R(x):
@@ -306,10 +307,9 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
             acts += _R(n[l] * pitch(dims[l - 1]) * 4)           # argmax (local src index)
 
     def dh_slot(l):                                             # dH_l slot of the backward region
-        b = _R(n[l] * pitch(dims[l]) * 4)                       # fp32 dH / dlogits; bf16 dZ + dZ/D
-        if act_dtype == BF16 and l < L:
-            b += _R(4 * 148 * dims[l])                          # GEMM-epilogue db partials
-        return b
+        if act_dtype == BF16 and l < L:                         # bf16 dZ_l + its db partial rows
+            return _R(n[l] * pitch(dims[l]) * 2) + _R(4 * BWD_DB_PARTS * dims[l])
+        return _R(n[l] * pitch(dims[l]) * 4)                    # fp32 dH / dlogits
 
     bwd = 0
     for l in range(L, 0, -1):
@@ -345,10 +345,8 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
         else:
             if l == L:
                 frame += _R(n[l] * pitch(dims[l]) * 2)          # dZ in bf16 (from dlogits)
-                if l >= 2:
-                    frame += _R(n[l] * pitch(dims[l]) * 2)      # dZ / D in bf16
             if l >= 2:
-                frame += _R(n[l - 1] * pitch(dims[l]) * 2)      # transposed sums in bf16
+                frame += 2 * _R(n[l] * pitch(dims[l - 1]) * 2)  # Ys = dZ W_self, Yn = dZ W_neigh / D (bf16)
             S = tc_dw_splits(n[l], dims[l], dims[l - 1])
             Dp = _ceil(dims[l - 1], 64) * 64
             frame += _R(S * dims[l] * 2 * Dp * 4)               # dW partials

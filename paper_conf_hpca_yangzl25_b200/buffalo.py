@@ -111,7 +111,7 @@ def lib(require_gpu=True):
             "buffalo_softmax_ce": (c_i32, [P, c_i64, c_i64, c_i32, P, P, c_i64, P, P, c_i64, P]),
             "buffalo_sage_bwd_scratch_bytes": (c_sz, [P, c_i32, P]),
             "buffalo_sage_bwd": (c_i32, [P, c_i32, P, P, c_i64, P, c_i64, P, c_i64, P, c_i64, P, P,
-                                         P, P, P, c_i64, P, P, c_sz, P]),
+                                         P, P, P, c_i64, P, c_sz, P]),
             "buffalo_sgd_step": (c_i32, [P, P, c_i64, c_f, P]),
             "buffalo_estimate_mem": (c_i32, [c_i32, P, P, P, P, P]),
             "buffalo_launch_count": (c_i64, []),
@@ -259,11 +259,11 @@ def sage_bwd_scratch_bytes(blk, layer, model):
 
 
 def sage_bwd(blk, layer, model, dh_dst, ld_dh, h_src, ld_src, saved_agg, ld_agg, h_dst, ld_hdst, W,
-             W_packed, dW, db, dh_src, ld_dh_src, prev_row_ptr, scratch, scratch_bytes, stream=None):
+             W_packed, dW, db, dh_src, ld_dh_src, scratch, scratch_bytes, stream=None):
     _check(lib().buffalo_sage_bwd(ref(blk), layer, ref(model), ptr(dh_dst), ld_dh,
                                   dev(h_src, act_dtypes(model, layer), "h_src"), ld_src,
                                   ptr(saved_agg), ld_agg, ptr(h_dst), ld_hdst, ptr(W), ptr(W_packed),
-                                  ptr(dW), ptr(db), ptr(dh_src), ld_dh_src, ptr(prev_row_ptr), ptr(scratch),
+                                  ptr(dW), ptr(db), ptr(dh_src), ld_dh_src, ptr(scratch),
                                   scratch_bytes, stream_ptr(stream)))
 
 

@@ -99,11 +99,11 @@ static int64_t bwd_scratch_for(const buffalo_model* m, int64_t n_dst, int64_t n_
 }
 
 // dH_l slot of the backward region: fp32 dH (FFMA) / dlogits; in BF16 mode layers l < L hold
-// bf16 dZ and dZ/D (same bytes) plus the epilogue's column-sum partials.
+// bf16 dZ_l plus the column-sum partials of the fused transposed Aggregate that wrote it.
 static int64_t dh_slot_bytes(const buffalo_model* m, int64_t n, int l) {
-  int64_t b = R(n * pitch_of(m->dim[l]) * 4);
-  if (m->gemm_mode == BUFFALO_GEMM_BF16 && l < m->num_layers) b += R((int64_t)4 * 148 * m->dim[l]);
-  return b;
+  if (m->gemm_mode == BUFFALO_GEMM_BF16 && l < m->num_layers)     // bf16 dZ_l + its db partial rows
+    return R(n * pitch_of(m->dim[l]) * 2) + R((int64_t)4 * tc_bwd_db_parts() * m->dim[l]);
+  return R(n * pitch_of(m->dim[l]) * 4);                          // fp32 dH / dlogits
 }
 
 static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_model* m,
@@ -816,7 +816,7 @@ buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const b
                                 float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
                                 const void* saved_agg, int64_t ld_agg, const void* h_dst,
                                 int64_t ld_hdst, const float* W, const void* W_packed, float* dW_accum,
-                                float* db_accum, float* dh_src, int64_t ld_dh_src, const int32_t* prev_row_ptr,
+                                float* db_accum, float* dh_src, int64_t ld_dh_src,
                                 void* scratch, size_t scratch_bytes, void* stream) {
   BF_CHECK(require_sm100());
   BF_CHECK(validate_model(m));
@@ -858,11 +858,6 @@ buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const b
   a.db = db_accum;
   a.dh_src = dh_src;
   a.ld_dh_src = ld_dh_src;
-  a.prev_row_ptr = prev_row_ptr;
-  if (m->gemm_mode == BUFFALO_GEMM_BF16 && dh_src && layer >= 3 && !prev_row_ptr) {
-    set_error("sage_bwd: bf16 mode needs block l-1's row_ptr for l >= 3");
-    return BUFFALO_ERR_INVALID_ARG;
-  }
   a.scratch = scratch;
   a.scratch_bytes = (int64_t)scratch_bytes;
   cudaStream_t s = (cudaStream_t)stream;

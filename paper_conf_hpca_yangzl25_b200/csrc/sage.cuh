@@ -29,7 +29,6 @@ struct BwdArgs {
   const float* W; const void* W_packed;
   float* dW; float* db;
   float* dh_src; int64_t ld_dh_src;
-  const int32_t* prev_row_ptr;
   void* scratch; int64_t scratch_bytes;
 };
 

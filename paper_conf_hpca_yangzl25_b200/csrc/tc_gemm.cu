@@ -176,6 +176,7 @@ struct GemmParams {
   int stage_off, stage_bytes; // epilogue staging area (8 warps x 2 x 2 KB; 0 for the backward)
   const float* bias;
   int relu, out_f32;
+  const int32_t* scale_rp;    // non-null: output row i is scaled by 1 / D(i), D(i) = rp[i+1] - rp[i] (0 if D = 0)
   void* out;
   // backward epilogue (epi != 0): out = prepared dZ of the layer below
   int epi;
@@ -345,6 +346,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         const int32_t d = __ldg(p.rp + row + 1) - __ldg(p.rp + row);
         invd = d > 0 ? 1.f / (float)d : 0.f;
       }
+      float rscale = 1.f;
+      if (!kBwd && rok && p.scale_rp) {
+        const int32_t d = __ldg(p.scale_rp + row + 1) - __ldg(p.scale_rp + row);
+        rscale = d > 0 ? 1.f / (float)d : 0.f;
+      }
       uint32_t r[2][32];
       if (nj > 0) {
         ld32_issue(tbase + h * 32, r[0]);
@@ -423,6 +429,10 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             if (p.relu) {
 #pragma unroll
               for (int k = 0; k < 32; ++k) v[k] = fmaxf(v[k], 0.f);
+            }
+            if (p.scale_rp) {
+#pragma unroll
+              for (int k = 0; k < 32; ++k) v[k] *= rscale;
             }
             if (p.out_f32) {
               if (rok) {
@@ -706,21 +716,24 @@ buffalo_status tc_dw_tma(int64_t n, int S, const __nv_bfloat16* z, int64_t ldz, 
 buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* self_idx, const __nv_bfloat16* self,
                            int64_t ld_self, const __nv_bfloat16* agg, int64_t ld_agg, int d_in, const uint8_t* wpk,
                            int d_out, const float* bias, int relu, int out_f32, void* out, int64_t ld_out,
-                           cudaStream_t s, const GemmEpi* epi) {
+                           cudaStream_t s, const GemmEpi* epi, const int32_t* scale_rp) {
   if (n_rows <= 0) return BUFFALO_OK;
   CUtensorMap sm, am;
   const int64_t pin = pitch_of(d_in);
   // self_idx: self rows gathered (row i = self_idx[i] of a [self_rows] table, box 64 x 1);
-  // else rows >= self_rows of the self half read as zero (TMA out-of-bounds fill)
+  // else rows >= self_rows of the self half read as zero (TMA out-of-bounds fill).
+  // agg = null: a single operand (K = d_in): out = self W^T over the first nkc_self weight chunks
   BF_CHECK(encode_map(&sm, self, pin, self_rows, ld_self, self_idx ? 1 : kTM));
-  BF_CHECK(encode_map(&am, agg, pin, n_rows, ld_agg));
+  if (agg) BF_CHECK(encode_map(&am, agg, pin, n_rows, ld_agg));
+  else am = sm;
   GemmParams p{};
   p.n_rows = n_rows;
   p.self_tiles = self_idx ? ceil_div(n_rows, kTM) : ceil_div(self_rows, kTM);
   p.self_idx = self_idx;
   p.self_oob = self_idx ? 0 : (int32_t)self_rows;
   p.nkc_self = (int)ceil_div(d_in, 64);
-  p.nkc = 2 * p.nkc_self;
+  p.nkc = agg ? 2 * p.nkc_self : p.nkc_self;
+  p.scale_rp = scale_rp;
   p.wpk = wpk;
   p.Np = (int)round_up(d_out, 16);
   p.d_out = d_out;

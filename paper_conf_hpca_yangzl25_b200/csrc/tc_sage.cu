@@ -541,14 +541,28 @@ buffalo_status launch_agg_heavy_bf16(const FwdArgs& a, cudaStream_t s);
 // SM), and the next row's perm / row_ptr entries fetched one iteration ahead so short rows do
 // not pay the whole perm -> row_ptr -> col -> row dependency chain each.  MODE 0 writes the
 // mean as x * (1/D) corrected by one FMA residual step (Markstein), MODE 1 the plain sum; the
-// per-row sum order is the CSR order (R21).
+// per-row sum order is the CSR order (R21).  MODE 2 is the backward's transposed Aggregate with
+// the layer-below epilogue fused (GatherEpi): for src row j the sum of the pre-scaled rows
+// Yn[i] = (dZ_l W_neigh)[i] / D(i) over T(j), plus Ys[j] = (dZ_l W_self)[j] for j < n_dst, gives
+// dH_{l-1}[j]; ReLU' with H_{l-1}[j] makes dZ_{l-1}[j], stored in bf16, and its columns are
+// summed (db_{l-1}) per lane group in shared memory and per CTA in a fixed order (one partial
+// row per CTA: deterministic).
+struct GatherEpi {
+  const __nv_bfloat16* ys; int64_t ldy;   // Ys [n_self][ldy]
+  int64_t n_self;
+  const __nv_bfloat16* H; int64_t ldH;    // H_{l-1} (ReLU' mask source)
+  int d;                                  // valid columns (d_{l-1}); pad columns are stored as 0
+  float* db_part;                         // [gridDim.x][d]
+};
+
 template <class TI, int MODE, int LPR, int kU, int MINB>
 __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restrict__ perm,
                                                          const int32_t* __restrict__ rp,
                                                          const int32_t* __restrict__ col, int32_t n,
                                                          const TI* __restrict__ h, int32_t ldb, int npieces,
                                                          __nv_bfloat16* __restrict__ out, int64_t ldo,
-                                                         unsigned long long* __restrict__ edges_dev) {
+                                                         unsigned long long* __restrict__ edges_dev,
+                                                         const GatherEpi ep) {
   constexpr int E = InTraits<TI>::kElems;
   constexpr int G = 32 / LPR;
   constexpr unsigned kFull = 0xffffffffu;
@@ -558,6 +572,14 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
   const int32_t warps = (int32_t)(gridDim.x * (blockDim.x >> 5));
   int32_t w = (int32_t)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
   unsigned my_edges = 0;
+  // MODE 2: column sums of dZ_{l-1}, one slice per (warp, lane group) [8][G][ncols]
+  extern __shared__ float sdb[];
+  const int ncols = npieces * E;
+  float* my_db = sdb + ((threadIdx.x >> 5) * G + g) * ncols;
+  if constexpr (MODE == 2) {
+    for (int c = threadIdx.x; c < 8 * G * ncols; c += blockDim.x) sdb[c] = 0.f;
+    __syncthreads();
+  }
   // row metadata of the first iteration
   int32_t row = -1, b = 0, e = 0;
   {
@@ -636,6 +658,26 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
 #pragma unroll
           for (int k = 0; k < E; ++k) v[k] = acc[k];
         }
+        if constexpr (MODE == 2) {
+          static_assert(E == 8, "the backward epilogue reads bf16 rows");
+          if (row < ep.n_self) {
+            float y[8];
+            bf16x8_to_f32(__ldg(reinterpret_cast<const uint4*>(ep.ys + (int64_t)row * ep.ldy + piece * 8)), y);
+#pragma unroll
+            for (int k = 0; k < 8; ++k) v[k] += y[k];
+          }
+          float hv[8];
+          bf16x8_to_f32(__ldg(reinterpret_cast<const uint4*>(ep.H + (int64_t)row * ep.ldH + piece * 8)), hv);
+#pragma unroll
+          for (int k = 0; k < 8; ++k)
+            if (!(hv[k] > 0.f) || piece * 8 + k >= ep.d) v[k] = 0.f;
+          float4* sd = reinterpret_cast<float4*>(my_db + piece * 8);
+          float4 a0 = sd[0], a1 = sd[1];
+          a0.x += v[0]; a0.y += v[1]; a0.z += v[2]; a0.w += v[3];
+          a1.x += v[4]; a1.y += v[5]; a1.z += v[6]; a1.w += v[7];
+          sd[0] = a0;
+          sd[1] = a1;
+        }
         __nv_bfloat16* dst = out + (int64_t)row * ldo + piece * E;
         if constexpr (E == 8) {
           *reinterpret_cast<uint4*>(dst) = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
@@ -652,6 +694,14 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
   if (edges_dev) {                                      // one atomic per warp per launch
     my_edges = __reduce_add_sync(kFull, my_edges);
     if (lane == 0 && my_edges) atomicAdd(edges_dev, (unsigned long long)my_edges);
+  }
+  if constexpr (MODE == 2) {
+    __syncthreads();
+    for (int c = threadIdx.x; c < ep.d; c += blockDim.x) {
+      float t = 0.f;
+      for (int s2 = 0; s2 < 8 * G; ++s2) t += sdb[s2 * ncols + c];
+      ep.db_part[(int64_t)blockIdx.x * ep.d + c] = t;
+    }
   }
 }
 
@@ -680,7 +730,7 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   const int32_t n32 = (int32_t)n;
   const int32_t ldb = (int32_t)(ldh * (int64_t)sizeof(TI));             // row stride in bytes
 #define BF_V2(L) k_gather_v2<TI, MODE, L, kU, kMinB><<<fgrid, 256, 0, s>>>(perm, rp, col, n32, h, ldb, npieces, out, \
-                                                                          ldo, ps.edges_dev)
+                                                                          ldo, ps.edges_dev, GatherEpi{})
   if (lpr_log <= 2) BF_V2(4);
   else if (lpr_log == 3) BF_V2(8);
   else if (lpr_log == 4) BF_V2(16);
@@ -689,6 +739,42 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   BF_LAUNCHED(MODE == 0 ? "k_gather_mean" : "k_gather_sum");
   // algorithmic bytes: per row perm + row_ptr pair + bf16 output row; per edge index + source row
   prof_end_launch(ps, s, (double)n * (12.0 + 2.0 * pitch_in), 4.0 + (double)pitch_in * sizeof(TI));
+  return BUFFALO_OK;
+}
+
+// MODE 2 (backward, fused epilogue): a fixed grid of kGatherDbCtas CTAs (one db partial row
+// each; the heavy-row kernel owns the kHeavyDbCtas rows after them).
+constexpr int kGatherDbCtas = 148 * 6, kHeavyDbCtas = 148;
+constexpr int kBwdDbParts = kGatherDbCtas + kHeavyDbCtas;
+
+static buffalo_status launch_gather_epi(const int32_t* perm, const int32_t* rp, const int32_t* col, int64_t n,
+                                        const __nv_bfloat16* yn, int64_t ldy, int pitch_in, __nv_bfloat16* out,
+                                        int64_t ldo, const GatherEpi& ep, cudaStream_t s) {
+  const int npieces = (pitch_in + 7) / 8;
+  int lpr_log = 0;
+  while ((1 << lpr_log) < npieces && lpr_log < 4) ++lpr_log;     // <= 16 lanes per row (short rows)
+  lpr_log = std::max(lpr_log, 2);
+  if (n > INT32_MAX || ldy * 2 > INT32_MAX) {
+    set_error("gather: %lld rows of stride %lld elements exceed the 32-bit row / byte-stride range",
+              (long long)n, (long long)ldy);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  const ProfSlot ps = prof_begin_launch("gather", s);
+  constexpr int kU = 2, kMinB = 6;
+  const int G = 32 >> lpr_log;
+  const int smem = 8 * G * npieces * 8 * 4;
+  const int32_t n32 = (int32_t)(n > 0 ? n : 0);
+  const int32_t ldb = (int32_t)(ldy * 2);
+#define BF_V2E(L) k_gather_v2<__nv_bfloat16, 2, L, kU, kMinB><<<kGatherDbCtas, 256, smem, s>>>( \
+      perm, rp, col, n32, yn, ldb, npieces, out, ldo, ps.edges_dev, ep)
+  if (lpr_log <= 2) BF_V2E(4);
+  else if (lpr_log == 3) BF_V2E(8);
+  else BF_V2E(16);
+#undef BF_V2E
+  BF_LAUNCHED("k_gather_bwd_epi");
+  // algorithmic bytes: per row perm + row_ptr pair + the H row + the bf16 dZ row (+ Ys for the
+  // dst prefix rows, not counted); per edge index + the Yn row
+  prof_end_launch(ps, s, (double)n * (12.0 + 4.0 * pitch_in), 4.0 + (double)pitch_in * 2);
   return BUFFALO_OK;
 }
 
@@ -1104,6 +1190,77 @@ __global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restric
   }
 }
 
+// The backward's long-tail transposed rows with the fused epilogue of GatherEpi: the same sum
+// as k_sum_heavy_rows (8 warps over the entries, combined in warp order), then + Ys[j] (j <
+// n_self), ReLU' with H[j], bf16 dZ_{l-1}[j], and the column sums of this CTA's heavy rows (in
+// row order) as db partial row kGatherDbCtas + blockIdx.x.  A fixed grid of kHeavyDbCtas CTAs:
+// CTAs without heavy rows write zero partials.
+__global__ void __launch_bounds__(256) k_heavy_bwd_epi(const int32_t* __restrict__ perm, int64_t n,
+                                                       const int32_t* __restrict__ rp,
+                                                       const int32_t* __restrict__ col,
+                                                       const __nv_bfloat16* __restrict__ z, int64_t ldz, int dp,
+                                                       __nv_bfloat16* __restrict__ out, int64_t ldo,
+                                                       const GatherEpi ep, int part_row0) {
+  __shared__ float part[8][32][8];
+  __shared__ float sdb[256];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int nch = dp / 8;                        // <= 32 pieces (d <= 256)
+  for (int c = threadIdx.x; c < 256; c += blockDim.x) sdb[c] = 0.f;
+  __syncthreads();
+  for (int64_t hh = blockIdx.x; hh < n; hh += gridDim.x) {
+    const int64_t j = perm[n - 1 - hh];          // heavy rows: the tail of the degree-class perm
+    const int32_t b = rp[j], e_end = rp[j + 1];
+    if (e_end - b <= kHeavyT) break;
+    const int c = lane;
+    float acc[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) acc[k] = 0.f;
+    if (c < nch) {
+      int32_t t = b + w;
+      for (; t + 24 < e_end; t += 32) {
+        uint4 r[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) r[u] = __ldg(reinterpret_cast<const uint4*>(z + (int64_t)col[t + 8 * u] * ldz + c * 8));
+#pragma unroll
+        for (int u = 0; u < 4; ++u) acc_piece<__nv_bfloat16>(acc, r[u]);
+      }
+      for (; t < e_end; t += 8)
+        acc_piece<__nv_bfloat16>(acc, __ldg(reinterpret_cast<const uint4*>(z + (int64_t)col[t] * ldz + c * 8)));
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) part[w][lane][k] = acc[k];
+    __syncthreads();
+    if (w == 0 && c < nch) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        float s2 = part[0][lane][k];
+        for (int ww = 1; ww < 8; ++ww) s2 += part[ww][lane][k];
+        acc[k] = s2;
+      }
+      if (j < ep.n_self) {
+        float y[8];
+        bf16x8_to_f32(__ldg(reinterpret_cast<const uint4*>(ep.ys + j * ep.ldy + c * 8)), y);
+#pragma unroll
+        for (int k = 0; k < 8; ++k) acc[k] += y[k];
+      }
+      float hv[8];
+      bf16x8_to_f32(__ldg(reinterpret_cast<const uint4*>(ep.H + j * ep.ldH + c * 8)), hv);
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        if (!(hv[k] > 0.f) || c * 8 + k >= ep.d) acc[k] = 0.f;
+        sdb[c * 8 + k] += acc[k];
+      }
+      *reinterpret_cast<uint4*>(out + j * ldo + c * 8) =
+          make_uint4(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]), pack_bf16x2(acc[4], acc[5]),
+                     pack_bf16x2(acc[6], acc[7]));
+    }
+    __syncthreads();
+  }
+  __syncthreads();
+  for (int c = threadIdx.x; c < ep.d; c += blockDim.x)
+    ep.db_part[(int64_t)(part_row0 + blockIdx.x) * ep.d + c] = sdb[c];
+}
+
 int tc_dw_splits(int64_t n, int d_out, int d_in) {
   (void)d_out;
   const int64_t Dp = round_up(d_in, 64);
@@ -1112,18 +1269,18 @@ int tc_dw_splits(int64_t n, int d_out, int d_in) {
   return (int)std::max<int64_t>(1, sp);
 }
 
+int64_t tc_bwd_db_parts() { return kBwdDbParts; }
+
 int64_t tc_bwd_scratch_bytes(int64_t n_dst, int64_t n_src, int64_t e, int layer, int d_in, int d_out, bool last) {
   (void)e;
+  (void)n_src;
   const int S = tc_dw_splits(n_dst, d_out, d_in);
   const int64_t Dp = round_up(d_in, 64);
   int64_t b = 0;
-  if (last) {
-    b += R(n_dst * pitch_of(d_out) * 2);                              // dZ bf16
-    if (layer >= 2) b += R(n_dst * pitch_of(d_out) * 2);              // dZ / D bf16
-  }
-  if (layer >= 2) b += R(n_src * pitch_of(d_out) * 2);                // transposed sums (bf16)
-  b += R((int64_t)S * d_out * 2 * Dp * 4);                            // dW partials
-  if (last) b += R((int64_t)kDbSplits * d_out * 4);                   // db partials (dz_prep)
+  if (last) b += R(n_dst * pitch_of(d_out) * 2);                    // dZ bf16
+  if (layer >= 2) b += 2 * R(n_dst * pitch_of(d_in) * 2);           // Ys = dZ W_self, Yn = dZ W_neigh / D (bf16)
+  b += R((int64_t)S * d_out * 2 * Dp * 4);                          // dW partials
+  if (last) b += R((int64_t)kDbSplits * d_out * 4);                 // db partials (dz_prep)
   return b;
 }
 
@@ -1136,35 +1293,36 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   const int64_t n = blk->n_dst;
   const int d_in = a.d_in, d_out = a.d_out;
   const int dp = (int)pitch_of(d_out);
+  const int dpp = (int)pitch_of(d_in);
   const int S = tc_dw_splits(n, d_out, d_in);
   const int64_t Dp = round_up(d_in, 64);
-  const bool need_zs = a.dh_src != nullptr;
-  // prepared input of this layer: bf16 dZ (+ dZ/D) and db partials
-  __nv_bfloat16 *zb, *zs = nullptr;
+  // prepared input of this layer: bf16 dZ and db partials
+  __nv_bfloat16* zb;
   float* db_part;
   int nparts;
   char* q = (char*)a.scratch;
   if (a.last) {
     zb = (__nv_bfloat16*)q; q += R(n * dp * 2);
-    if (need_zs) { zs = (__nv_bfloat16*)q; q += R(n * dp * 2); }
   } else {
     zb = (__nv_bfloat16*)a.dh;
-    if (need_zs) zs = zb + n * dp;
   }
-  __nv_bfloat16* aggT = nullptr;
-  if (need_zs) { aggT = (__nv_bfloat16*)q; q += R(blk->n_src * dp * 2); }
+  __nv_bfloat16 *ys = nullptr, *yn = nullptr;
+  if (a.dh_src) {
+    ys = (__nv_bfloat16*)q; q += R(n * dpp * 2);
+    yn = (__nv_bfloat16*)q; q += R(n * dpp * 2);
+  }
   float* dw_part = (float*)q; q += R((int64_t)S * d_out * 2 * Dp * 4);
   if (a.last) {
     db_part = (float*)q;
     nparts = kDbSplits;
   } else {
-    db_part = (float*)((char*)a.dh + R(n * dp * 4));
-    nparts = (int)gemm_grid(n);
+    db_part = (float*)((char*)a.dh + R(n * dp * 2));
+    nparts = kBwdDbParts;
   }
   if (n <= 0) return BUFFALO_OK;
   if (a.last) {
-    k_dz_prep<__nv_bfloat16><<<kDbSplits, 256, 0, s>>>(a.dh, a.ld_dh, nullptr, 0, blk->row_ptr, n, d_out, dp, zb, zs,
-                                                       db_part);
+    k_dz_prep<__nv_bfloat16><<<kDbSplits, 256, 0, s>>>(a.dh, a.ld_dh, nullptr, 0, blk->row_ptr, n, d_out, dp, zb,
+                                                       nullptr, db_part);
     BF_LAUNCHED("k_dz_prep");
   }
   // dW (TMA-fed tensor cores, deterministic split reduction) and db
@@ -1193,28 +1351,31 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   BF_LAUNCHED("k_reduce_dw");
   k_reduce_db<<<(unsigned)ceil_div(d_out, 32), 256, 0, s>>>(db_part, nparts, d_out, a.db);
   BF_LAUNCHED("k_reduce_db");
-  // dH_{l-1} = [dZ (rows < n_dst) || sum_{i in T(j)} dZ[i]/D(i)] [W_self; W_neigh], written in the
-  // prepared form of layer l-1 by the GEMM epilogue (ReLU' with H_{l-1}, /D_{l-1}, db partials)
-  if (a.dh_src && blk->n_src > 0) {
-    const int hg = heavy_tail_grid(blk->n_heavy_t, blk->n_edges);
-    if (hg > 0) {
-      k_sum_heavy_rows<<<hg, 256, 0, s>>>(blk->t_perm, blk->n_src, blk->t_row_ptr, blk->t_col, zs, dp, dp, aggT, 1);
-      BF_LAUNCHED("k_sum_heavy_rows");
-    }
-    BF_CHECK((launch_gather<__nv_bfloat16, 1>(blk->t_perm, blk->t_row_ptr, blk->t_col, blk->n_src, zs, dp, dp,
-                                              aggT, dp, s)));
-    const int64_t ns = blk->n_src;
-    const int dpp = (int)pitch_of(d_in);
-    GemmEpi epi{};
-    epi.H = (const __nv_bfloat16*)a.h_src;
-    epi.ldH = a.ld_src;
-    epi.zb = (__nv_bfloat16*)a.dh_src;
-    epi.zs = a.prev_row_ptr ? epi.zb + ns * dpp : nullptr;     // layer l-1 >= 2 needs dZ/D
-    epi.rp = a.prev_row_ptr;
-    epi.db_part = (float*)((char*)a.dh_src + R(ns * dpp * 4));
+  // dH_{l-1}[j] = [j < n_dst] (dZ W_self)[j] + sum_{i in T(j)} (dZ W_neigh)[i] / D(i): the two
+  // products over the n_dst rows first (tcgen05, the 1/D row scale in the epilogue), then the
+  // transposed Aggregate over the n_src rows with the layer-below epilogue fused (+ Ys, ReLU'
+  // with H_{l-1}, bf16 dZ_{l-1}, db_{l-1} partials) — no n_src x d intermediate.
+  if (a.dh_src) {
     const uint8_t* wpk = (const uint8_t*)a.W_packed + R((int64_t)2 * d_in * d_out * 4) + tc_fwd_packed_bytes(d_in, d_out);
-    // self half = dZ rows (rows >= n_dst are zero: the map covers n_dst rows only)
-    BF_CHECK(tc_gemm_tma(ns, n, nullptr, zb, dp, aggT, dp, d_out, wpk, d_in, nullptr, 0, 0, nullptr, 0, s, &epi));
+    const int64_t wchunk = round_up(d_in, 16) * 128;              // one packed K-chunk (Np rows x 128 B)
+    const int nkc = (int)ceil_div(d_out, kKC);
+    BF_CHECK(tc_gemm_tma(n, n, nullptr, zb, dp, nullptr, 0, d_out, wpk, d_in, nullptr, 0, 0, ys, dpp, s));
+    BF_CHECK(tc_gemm_tma(n, n, nullptr, zb, dp, nullptr, 0, d_out, wpk + nkc * wchunk, d_in, nullptr, 0, 0, yn, dpp,
+                         s, nullptr, blk->row_ptr));
+    const int64_t ns = blk->n_src;
+    GatherEpi ep{};
+    ep.ys = ys;
+    ep.ldy = dpp;
+    ep.n_self = n;
+    ep.H = (const __nv_bfloat16*)a.h_src;
+    ep.ldH = a.ld_src;
+    ep.d = d_in;
+    ep.db_part = (float*)((char*)a.dh_src + R(ns * dpp * 2));
+    __nv_bfloat16* zprev = (__nv_bfloat16*)a.dh_src;
+    k_heavy_bwd_epi<<<kHeavyDbCtas, 256, 0, s>>>(blk->t_perm, ns, blk->t_row_ptr, blk->t_col, yn, dpp, dpp, zprev,
+                                                  dpp, ep, kGatherDbCtas);
+    BF_LAUNCHED("k_heavy_bwd_epi");
+    BF_CHECK(launch_gather_epi(blk->t_perm, blk->t_row_ptr, blk->t_col, ns, yn, dpp, dpp, zprev, dpp, ep, s));
   }
   return BUFFALO_OK;
 }

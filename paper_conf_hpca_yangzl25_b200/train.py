@@ -301,9 +301,8 @@ class Trainer:
             if l > 1:
                 prev = blks.layer[l - 2]
                 h_src, ld_src, dh_src, ld_dh_src = prev.out, prev.ld_out, prev.dh, prev.ld_dh
-                prev_rp = prev.row_ptr if l > 2 else None
             else:
-                h_src, ld_src, dh_src, ld_dh_src, prev_rp = self.feats, self.feats.shape[1], None, 0, None
+                h_src, ld_src, dh_src, ld_dh_src = self.feats, self.feats.shape[1], None, 0
             h_dst = b.out if l < self.L else None
             if self.is_gat:
                 B.gat_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, h_dst, b.ld_out, p.W[l - 1], p.al[l - 1],
@@ -322,7 +321,7 @@ class Trainer:
                            p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src, b.bwd_scratch, b.bwd_scratch_bytes)
                 continue
             B.sage_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out,
-                       p.W[l - 1], p.packed[l - 1], p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src, prev_rp,
+                       p.W[l - 1], p.packed[l - 1], p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src,
                        b.bwd_scratch, b.bwd_scratch_bytes)
 
     def loss_and_grad(self, off, n):

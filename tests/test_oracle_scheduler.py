@@ -137,8 +137,11 @@ def test_mem_model_hand_instance():
 def test_mem_model_monotone_and_bf16_smaller():
     a = O.mem_model([1000, 300, 50], [2000, 400], [64, 32, 8], O.FP32)
     b = O.mem_model([1000, 300, 60], [2000, 500], [64, 32, 8], O.FP32)
-    c = O.mem_model([1000, 300, 50], [2000, 400], [64, 32, 8], O.BF16)
-    assert b[0] >= a[0] and b[1] >= a[1] and c[0] < a[0]
+    assert b[0] >= a[0] and b[1] >= a[1]
+    # bf16 activations halve the per-row terms; the bf16 backward's fixed db partial rows
+    # (BWD_DB_PARTS x d) only matter for tiny micro-batches
+    big = ([100000, 30000, 5000], [200000, 40000], [64, 32, 8])
+    assert O.mem_model(*big, O.BF16)[0] < O.mem_model(*big, O.FP32)[0]
 
 
 def _plan_invariants(plan, seeds, budget):
