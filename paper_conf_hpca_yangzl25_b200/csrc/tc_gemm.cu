@@ -1,14 +1,16 @@
 // tc_gemm.cu — the Update GEMM over contiguous operands, TMA-fed (sm_100a).
 //
-//   out[i] = act([self[i] || agg[i]] W^T + b),   i < n_rows
+//   out[i] = act([self[i] || agg[i]] W^T + b) (* 1/D(i) optionally),   i < n_rows
 //
 // self and agg are row-major bf16 matrices whose rows are the tile rows (layers >= 2 of the
-// forward: H_{l-1} and the saved h_agg; the backward dH: dZ and the transposed sums), so both
-// halves of the A operand are plain 2D tiles: one TMA load (box 64 x 128, SWIZZLE_128B) per
-// K-chunk lands them in the UMMA K-major SW128 layout.  The pre-swizzled weight chunk of the
-// same K range comes with a 1D bulk copy into the same pipeline stage.  Roles: warp 4 lane 0
-// produces (TMA), warp 5 lane 0 issues tcgen05.mma into a double-buffered TMEM accumulator,
-// warps 0-3 run the epilogue (tcgen05.ld -> +bias -> ReLU -> store) of the previous tile.
+// forward: H_{l-1} and the saved h_agg; layer 1: feature rows gathered by tile::gather4), so
+// both halves of the A operand are plain 2D tiles: one TMA load (box 64 x 128, SWIZZLE_128B)
+// per K-chunk lands them in the UMMA K-major SW128 layout.  With agg = null the A operand is
+// self alone (the backward's Ys = dZ W_self and Yn = dZ W_neigh / D products).  The
+// pre-swizzled weight chunks stay resident in shared memory when they fit, else each comes
+// with a 1D bulk copy into the A chunk's pipeline stage.  Roles: two producer warps issue the
+// TMA loads, one elected lane issues tcgen05.mma into a double-buffered TMEM accumulator, and
+// eight epilogue warps run tcgen05.ld -> +bias -> ReLU -> bf16 -> TMA store of the previous tile.
 #include <cuda.h>
 
 #include <algorithm>
@@ -130,21 +132,6 @@ __device__ __forceinline__ void ld32_wait(uint32_t (&r)[32]) {
                :
                : "memory");
 }
-// Column sums of a warp's 32 x 32 register tile in 31 shuffles: each step halves the columns a
-// lane keeps and adds its partner's copy; afterwards v[0] of lane k holds the sum of column k.
-__device__ __forceinline__ float warp_colsum32(float (&v)[32], int lane) {
-#pragma unroll
-  for (int o = 16; o >= 1; o >>= 1) {
-    const bool up = (lane & o) != 0;
-#pragma unroll
-    for (int j = 0; j < o; ++j) {
-      const float send = up ? v[j] : v[j + o];
-      const float keep = up ? v[j + o] : v[j];
-      v[j] = keep + __shfl_xor_sync(0xffffffffu, send, o);
-    }
-  }
-  return v[0];
-}
 __device__ __forceinline__ uint32_t pk(float a, float b) {
   __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
   return *reinterpret_cast<uint32_t*>(&h);
@@ -172,25 +159,17 @@ struct GemmParams {
   // weight chunk in shared memory for the whole launch (one 1D bulk copy per chunk at start), so
   // the pipeline stages carry A tiles only; with nsplit = 2 the two CTAs of a tile set compute
   // the two column halves of the same tiles (A is read twice, the second time from L2).
-  int w_res, nsplit, Nsub, db_parts;
-  int stage_off, stage_bytes; // epilogue staging area (8 warps x 2 x 2 KB; 0 for the backward)
+  int w_res, nsplit, Nsub;
+  int stage_off, stage_bytes; // epilogue staging area (8 warps x 2 x 2 KB)
   const float* bias;
   int relu, out_f32;
   const int32_t* scale_rp;    // non-null: output row i is scaled by 1 / D(i), D(i) = rp[i+1] - rp[i] (0 if D = 0)
   void* out;
-  // backward epilogue (epi != 0): out = prepared dZ of the layer below
-  int epi;
-  const __nv_bfloat16* H; int64_t ldH;   // ReLU' mask source H_{l-1}
-  const int32_t* rp;                     // block l-1 row_ptr (D for the dZ/D copy) or null
-  __nv_bfloat16* zb; __nv_bfloat16* zs;  // [n_rows][pitch_out] bf16 outputs (zs nullable)
-  float* db_part;                        // [gridDim.x][d_out]
 };
 
-template <bool kBwd>
 __global__ void __launch_bounds__(kGemmThreads, 1)
     k_tc_gemm_tma(const __grid_constant__ CUtensorMap self_map, const __grid_constant__ CUtensorMap agg_map,
-                  const __grid_constant__ CUtensorMap out_map, const __grid_constant__ CUtensorMap out2_map,
-                  const GemmParams p) {
+                  const __grid_constant__ CUtensorMap out_map, const GemmParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-B alignment by offset (keeps the shared address space visible to the compiler)
   uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
@@ -300,10 +279,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     __syncwarp();
   } else {
     // ---------------- epilogue: warp e owns TMEM lane quadrant q = e & 3 (tile rows 32q..32q+31)
-    // and the 32-column groups g = 2j + h (h = e >> 2).  Forward: +bias, ReLU, store.  Backward
-    // (kBwd): dZ = acc * 1[H > 0] -> bf16 dZ, bf16 dZ/D, and per-warp column sums (fixed row
-    // order) combined per CTA at the end.  H of the next tile is prefetched into registers while
-    // the current one is processed; the next TMEM load is issued before the current group's math.
+    // and the 32-column groups g = 2j + h (h = e >> 2): +bias, ReLU, optional 1/D row scale,
+    // store.  The next TMEM load is issued before the current group's math.
     const int q = warp & 3, h = warp >> 2;
     float* sbias = reinterpret_cast<float*>(tmem_slot + 4);   // 16-B aligned
     uint8_t* stg = smem + p.stage_off + warp * 4096;          // this warp's two 2-KB staging boxes
@@ -314,25 +291,6 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     const int ncol_cta = min(p.Nsub, p.pitch_out - col_base);   // output columns of this CTA
     const int ng = (ncol_cta + 31) / 32;
     const int nj = (ng - h + 1) / 2;              // groups of this warp (<= 4)
-    float dbacc[4] = {0.f, 0.f, 0.f, 0.f};
-    uint4 hreg[4][4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j)
-#pragma unroll
-      for (int k = 0; k < 4; ++k) hreg[j][k] = make_uint4(0u, 0u, 0u, 0u);
-    if (kBwd) {
-      const int64_t row = set0 * kTM + q * 32 + lane;
-      if (row < p.n_rows) {
-        const __nv_bfloat16* hr = p.H + row * p.ldH + col_base;
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const int c0 = (2 * j + h) * 32;
-#pragma unroll
-          for (int k = 0; k < 4; ++k)
-            if (j < nj && c0 + 8 * k < ncol_cta) hreg[j][k] = __ldg(reinterpret_cast<const uint4*>(hr + c0 + 8 * k));
-        }
-      }
-    }
     int64_t i = 0;
     for (int64_t t = set0; t < ntiles; t += nsets, ++i) {
       const int acc = (int)(i & 1);
@@ -341,13 +299,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       const int64_t row = t * kTM + q * 32 + lane;
       const bool rok = row < p.n_rows;
       const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + acc * p.Nsub;
-      float invd = 1.f;
-      if (kBwd && rok && p.zs) {
-        const int32_t d = __ldg(p.rp + row + 1) - __ldg(p.rp + row);
-        invd = d > 0 ? 1.f / (float)d : 0.f;
-      }
       float rscale = 1.f;
-      if (!kBwd && rok && p.scale_rp) {
+      if (rok && p.scale_rp) {
         const int32_t d = __ldg(p.scale_rp + row + 1) - __ldg(p.scale_rp + row);
         rscale = d > 0 ? 1.f / (float)d : 0.f;
       }
@@ -360,107 +313,51 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       for (int j = 0; j < 4; ++j) {
         if (j < nj) {
           const int c0 = (2 * j + h) * 32;
-          if (kBwd && j > 0) {                          // backward: registers go to the H prefetch
-            ld32_issue(tbase + c0, r[j & 1]);
-            ld32_wait(r[j & 1]);
-          }
-          if (!kBwd && j + 1 < nj) ld32_issue(tbase + c0 + 64, r[(j + 1) & 1]);
+          if (j + 1 < nj) ld32_issue(tbase + c0 + 64, r[(j + 1) & 1]);
           const int ncols = min(32, ncol_cta - c0);      // multiple of 8
           const int gc0 = col_base + c0;                 // global output column
           float v[32];
 #pragma unroll
           for (int k = 0; k < 32; ++k) v[k] = __uint_as_float(r[j & 1][k]);
-          if (kBwd) {
+#pragma unroll
+          for (int k = 0; k < 32; k += 4) {
+            const float4 bb = *reinterpret_cast<const float4*>(sbias + c0 + k);
+            v[k] += bb.x; v[k + 1] += bb.y; v[k + 2] += bb.z; v[k + 3] += bb.w;
+          }
+          if (p.relu) {
+#pragma unroll
+            for (int k = 0; k < 32; ++k) v[k] = fmaxf(v[k], 0.f);
+          }
+          if (p.scale_rp) {
+#pragma unroll
+            for (int k = 0; k < 32; ++k) v[k] *= rscale;
+          }
+          if (p.out_f32) {
             if (rok) {
+              float* o = (float*)p.out + row * p.ld_out + gc0;
 #pragma unroll
-              for (int k = 0; k < 32; k += 8) {
-                if (k < ncols) {
-                  const uint32_t hw[4] = {hreg[j][k / 8].x, hreg[j][k / 8].y, hreg[j][k / 8].z, hreg[j][k / 8].w};
-#pragma unroll
-                  for (int e = 0; e < 4; ++e) {
-                    const float h0 = __uint_as_float(hw[e] << 16), h1 = __uint_as_float(hw[e] & 0xffff0000u);
-                    if (!(h0 > 0.f) || gc0 + k + 2 * e >= p.d_out) v[k + 2 * e] = 0.f;
-                    if (!(h1 > 0.f) || gc0 + k + 2 * e + 1 >= p.d_out) v[k + 2 * e + 1] = 0.f;
-                  }
-                } else {
-#pragma unroll
-                  for (int e = 0; e < 8; ++e) v[k + e] = 0.f;
-                }
-              }
-              // bf16 dZ and dZ/D rows (direct stores: measured faster here than staging two
-              // boxes per group through the TMA-store path)
-              __nv_bfloat16* zo = p.zb + row * p.pitch_out + gc0;
-#pragma unroll
-              for (int k = 0; k < 32; k += 8)
-                if (k < ncols)
-                  *reinterpret_cast<uint4*>(zo + k) = make_uint4(pk(v[k], v[k + 1]), pk(v[k + 2], v[k + 3]),
-                                                                 pk(v[k + 4], v[k + 5]), pk(v[k + 6], v[k + 7]));
-              if (p.zs) {
-                __nv_bfloat16* so = p.zs + row * p.pitch_out + gc0;
-#pragma unroll
-                for (int k = 0; k < 32; k += 8)
-                  if (k < ncols)
-                    *reinterpret_cast<uint4*>(so + k) =
-                        make_uint4(pk(v[k] * invd, v[k + 1] * invd), pk(v[k + 2] * invd, v[k + 3] * invd),
-                                   pk(v[k + 4] * invd, v[k + 5] * invd), pk(v[k + 6] * invd, v[k + 7] * invd));
-              }
-            } else {
-#pragma unroll
-              for (int k = 0; k < 32; ++k) v[k] = 0.f;
+              for (int k = 0; k < 32; k += 4)
+                if (k < ncols) *reinterpret_cast<float4*>(o + k) = make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]);
             }
-            // prefetch this group's H of the next tile (its registers are free now)
-            {
-              const int64_t tn = t + nsets;
-              const int64_t rn = tn * kTM + q * 32 + lane;
-              if (tn < ntiles && rn < p.n_rows) {
-                const __nv_bfloat16* hr = p.H + rn * p.ldH + gc0;
-#pragma unroll
-                for (int k = 0; k < 4; ++k)
-                  if (8 * k < ncols) hreg[j][k] = __ldg(reinterpret_cast<const uint4*>(hr + 8 * k));
-              }
-            }
-            dbacc[j] += warp_colsum32(v, lane);
           } else {
+            // bf16 rows through a staging box and one TMA store per warp and column group
+            // (coalesced, asynchronous; rows past n_rows are clipped by the map)
+            uint8_t* box = stg + sbuf * 2048;
+            sbuf ^= 1;
+            if (lane == 0) bulk_wait_read<1>();       // the store that used this box has read it
+            __syncwarp();
 #pragma unroll
-            for (int k = 0; k < 32; k += 4) {
-              const float4 bb = *reinterpret_cast<const float4*>(sbias + c0 + k);
-              v[k] += bb.x; v[k + 1] += bb.y; v[k + 2] += bb.z; v[k + 3] += bb.w;
-            }
-            if (p.relu) {
-#pragma unroll
-              for (int k = 0; k < 32; ++k) v[k] = fmaxf(v[k], 0.f);
-            }
-            if (p.scale_rp) {
-#pragma unroll
-              for (int k = 0; k < 32; ++k) v[k] *= rscale;
-            }
-            if (p.out_f32) {
-              if (rok) {
-                float* o = (float*)p.out + row * p.ld_out + gc0;
-#pragma unroll
-                for (int k = 0; k < 32; k += 4)
-                  if (k < ncols) *reinterpret_cast<float4*>(o + k) = make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]);
-              }
-            } else {
-              // bf16 rows through a staging box and one TMA store per warp and column group
-              // (coalesced, asynchronous; rows past n_rows are clipped by the map)
-              uint8_t* box = stg + sbuf * 2048;
-              sbuf ^= 1;
-              if (lane == 0) bulk_wait_read<1>();       // the store that used this box has read it
-              __syncwarp();
-#pragma unroll
-              for (int k = 0; k < 4; ++k)
-                st_stage64(box, lane, k, make_uint4(pk(v[8 * k], v[8 * k + 1]), pk(v[8 * k + 2], v[8 * k + 3]),
-                                                     pk(v[8 * k + 4], v[8 * k + 5]), pk(v[8 * k + 6], v[8 * k + 7])));
-              fence_async_smem();
-              __syncwarp();
-              if (lane == 0) {
-                tma_store_2d(&out_map, box, gc0, (int)(t * kTM + q * 32));
-                bulk_commit();
-              }
+            for (int k = 0; k < 4; ++k)
+              st_stage64(box, lane, k, make_uint4(pk(v[8 * k], v[8 * k + 1]), pk(v[8 * k + 2], v[8 * k + 3]),
+                                                   pk(v[8 * k + 4], v[8 * k + 5]), pk(v[8 * k + 6], v[8 * k + 7])));
+            fence_async_smem();
+            __syncwarp();
+            if (lane == 0) {
+              tma_store_2d(&out_map, box, gc0, (int)(t * kTM + q * 32));
+              bulk_commit();
             }
           }
-          if (!kBwd && j + 1 < nj) ld32_wait(r[(j + 1) & 1]);
+          if (j + 1 < nj) ld32_wait(r[(j + 1) & 1]);
         }
       }
       fence_before();
@@ -468,24 +365,6 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     }
     if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
     __syncwarp();
-    if (kBwd) {
-      // combine the four lane quadrants in order -> one partial per CTA
-      float* red = reinterpret_cast<float*>(sA);     // stage 0 A buffer: every MMA has completed
-      asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
-#pragma unroll
-      for (int j = 0; j < 4; ++j)
-        if (j < nj) red[q * 256 + (2 * j + h) * 32 + lane] = dbacc[j];
-      asm volatile("bar.sync 1, %0;" ::"n"(kEpiWarps * 32) : "memory");
-      const int ncd = min(p.Nsub, p.d_out - col_base);
-      for (int c = threadIdx.x; c < ncd; c += kEpiWarps * 32) {
-        float tsum = 0.f;
-        for (int w = 0; w < 4; ++w) tsum += red[w * 256 + c];
-        p.db_part[set0 * p.d_out + col_base + c] = tsum;
-      }
-      // the reader sums db_parts rows: rows no tile set wrote are zero
-      for (int64_t r = nsets + set0; r < p.db_parts; r += nsets)
-        for (int c = threadIdx.x; c < ncd; c += kEpiWarps * 32) p.db_part[r * p.d_out + col_base + c] = 0.f;
-    }
   }
   fence_before();
   __syncthreads();
@@ -716,7 +595,7 @@ buffalo_status tc_dw_tma(int64_t n, int S, const __nv_bfloat16* z, int64_t ldz, 
 buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* self_idx, const __nv_bfloat16* self,
                            int64_t ld_self, const __nv_bfloat16* agg, int64_t ld_agg, int d_in, const uint8_t* wpk,
                            int d_out, const float* bias, int relu, int out_f32, void* out, int64_t ld_out,
-                           cudaStream_t s, const GemmEpi* epi, const int32_t* scale_rp) {
+                           cudaStream_t s, const int32_t* scale_rp) {
   if (n_rows <= 0) return BUFFALO_OK;
   CUtensorMap sm, am;
   const int64_t pin = pitch_of(d_in);
@@ -742,12 +621,11 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   // resident weights when all weight chunks fit next to >= 4 A stages and the store staging
   // (a CTA-pair column split, nsplit = 2, is supported by the kernel but measured slower)
   const int64_t w_all = (int64_t)p.nkc * p.Np * 128;
-  const int64_t kStaging = epi ? 0 : kEpiWarps * 4096;
+  const int64_t kStaging = kEpiWarps * 4096;
   const int misc = 16 * 8 + 48 + 4 * p.Np + 1024;                    // barriers, slot, bias, alignment
   p.nsplit = 1;
   p.w_res = (227 * 1024 - w_all - kStaging - misc) / kChunkA >= 4 ? 1 : 0;
   p.Nsub = p.Np / p.nsplit;
-  p.db_parts = (int)gemm_grid(n_rows);
   int cols = 32;
   while (cols < 2 * p.Nsub) cols *= 2;
   p.tmem_cols = cols;
@@ -755,11 +633,6 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   p.relu = relu;
   p.out_f32 = out_f32;
   p.out = out;
-  if (epi) {
-    p.epi = 1;
-    p.H = epi->H; p.ldH = epi->ldH; p.rp = epi->rp;
-    p.zb = epi->zb; p.zs = epi->zs; p.db_part = epi->db_part;
-  }
   int smem;
   if (p.w_res) {
     const int64_t wres = (int64_t)p.nkc * p.Nsub * 128;               // chunks < c_lo stay unused
@@ -772,21 +645,14 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   }
   p.stage_bytes = (int)kStaging;
   smem = (int)(p.stage_off + kStaging + misc);
-  // output maps for the TMA-store epilogue: {32 col, 32 row} boxes, SWIZZLE_64B staging
-  CUtensorMap om, om2;
-  if (!epi && !out_f32) {
-    BF_CHECK(encode_map(&om, out, p.pitch_out, n_rows, ld_out, 32, 32, CU_TENSOR_MAP_SWIZZLE_64B));
-    om2 = om;
-  } else {
-    om = am;                                                          // unused (fp32 rows stored directly)
-    om2 = am;
-  }
-  BF_CHECK(set_max_smem_once<k_tc_gemm_tma<false>>(227 * 1024));
-  BF_CHECK(set_max_smem_once<k_tc_gemm_tma<true>>(227 * 1024));
+  // output map for the TMA-store epilogue: {32 col, 32 row} boxes, SWIZZLE_64B staging
+  CUtensorMap om;
+  if (!out_f32) BF_CHECK(encode_map(&om, out, p.pitch_out, n_rows, ld_out, 32, 32, CU_TENSOR_MAP_SWIZZLE_64B));
+  else om = am;                                                       // unused (fp32 rows stored directly)
+  BF_CHECK(set_max_smem_once<k_tc_gemm_tma>(227 * 1024));
   const int64_t sets = std::min<int64_t>(ceil_div(n_rows, kTM), 148 / p.nsplit);
   const int grid = (int)(sets * p.nsplit);
-  if (epi) k_tc_gemm_tma<true><<<grid, kGemmThreads, smem, s>>>(sm, am, om, om2, p);
-  else k_tc_gemm_tma<false><<<grid, kGemmThreads, smem, s>>>(sm, am, om, om2, p);
+  k_tc_gemm_tma<<<grid, kGemmThreads, smem, s>>>(sm, am, om, p);
   BF_LAUNCHED("k_tc_gemm_tma");
   return BUFFALO_OK;
 }

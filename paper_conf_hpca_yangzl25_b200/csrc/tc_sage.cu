@@ -1361,7 +1361,7 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     const int nkc = (int)ceil_div(d_out, kKC);
     BF_CHECK(tc_gemm_tma(n, n, nullptr, zb, dp, nullptr, 0, d_out, wpk, d_in, nullptr, 0, 0, ys, dpp, s));
     BF_CHECK(tc_gemm_tma(n, n, nullptr, zb, dp, nullptr, 0, d_out, wpk + nkc * wchunk, d_in, nullptr, 0, 0, yn, dpp,
-                         s, nullptr, blk->row_ptr));
+                         s, blk->row_ptr));
     const int64_t ns = blk->n_src;
     GatherEpi ep{};
     ep.ys = ys;

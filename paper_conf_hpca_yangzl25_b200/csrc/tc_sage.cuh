@@ -18,21 +18,10 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s);
 buffalo_status tc_dw_tma(int64_t n, int S, const __nv_bfloat16* z, int64_t ldz, int d_out,
                          const __nv_bfloat16* self, int64_t lds, const int32_t* gidx, int64_t self_table_rows,
                          const __nv_bfloat16* agg, int64_t lda, int d_in, float* part, cudaStream_t s);
-// Backward epilogue of the Update GEMM: writes the prepared dZ of the layer below.
-struct GemmEpi {
-  const __nv_bfloat16* H; int64_t ldH;   // ReLU' mask source
-  const int32_t* rp;                     // row_ptr for D (null if no dZ/D copy)
-  __nv_bfloat16* zb; __nv_bfloat16* zs;  // outputs [n_rows][pitch(d_out)]
-  float* db_part;                        // [gemm_grid(n_rows)][d_out]
-};
-inline int64_t gemm_grid(int64_t n_rows) {
-  const int64_t t = (n_rows + 127) / 128;
-  return t < 148 ? t : 148;
-}
 buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* self_idx, const __nv_bfloat16* self,
                            int64_t ld_self, const __nv_bfloat16* agg,
                            int64_t ld_agg, int d_in, const uint8_t* wpk, int d_out, const float* bias, int relu,
-                           int out_f32, void* out, int64_t ld_out, cudaStream_t s, const GemmEpi* epi = nullptr,
+                           int out_f32, void* out, int64_t ld_out, cudaStream_t s,
                            const int32_t* scale_rp = nullptr);
 
 }  // namespace buffalo
