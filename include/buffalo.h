@@ -158,6 +158,10 @@ typedef struct {
    * GAT: Z = H W^T, the attention scores el / er and the attention weights per edge (R30). */
   void* agg_saved;
   int64_t agg_saved_bytes;
+  /* the sampling fanout the block was built with (<= 0: all neighbours).  A sampled block has no
+   * row longer than the fanout (<= BUFFALO_MAX_FANOUT < 129), so the forward Aggregate walks its
+   * rows in natural order (sequential row_ptr / col reads) instead of through cls_perm. */
+  int64_t fanout;
 } buffalo_block;
 
 typedef struct {

@@ -80,7 +80,7 @@ class Block(ctypes.Structure):
                 ("agg", c_p), ("out", c_p), ("dh", c_p), ("bwd_scratch", c_p),
                 ("ld_agg", c_i64), ("ld_out", c_i64), ("ld_dh", c_i64), ("bwd_scratch_bytes", c_i64),
                 ("pool_P", c_p), ("pool_arg", c_p), ("ld_pool", c_i64),
-                ("agg_saved", c_p), ("agg_saved_bytes", c_i64)]
+                ("agg_saved", c_p), ("agg_saved_bytes", c_i64), ("fanout", c_i64)]
 
 
 class Blocks(ctypes.Structure):

@@ -349,6 +349,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
                            const int32_t* cache) {
   memset(blk, 0, sizeof(*blk));
   blk->n_dst = n_dst;
+  blk->fanout = f;
   int32_t* rp = (int32_t*)A.take(4 * (n_dst + 1));
   int32_t* perm = sizes_only ? nullptr : (int32_t*)A.take(4 * n_dst);
   // frame 1: totals + scan workspace for the count scan and the heavy compaction

@@ -835,7 +835,9 @@ static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   p.agg = (__nv_bfloat16*)a.agg;
   p.ld_agg = a.ld_agg;
   // high-occupancy gather of the non-heavy rows, then the Update GEMM over copies
-  BF_CHECK((launch_gather<TI, 0>(blk->cls_perm, blk->row_ptr, p.col, blk->n_dst, (const TI*)a.h_src, a.ld_src,
+  // sampled blocks (no row past the fanout): rows in natural order; else the degree-class order
+  const int32_t* order = (blk->fanout > 0 && blk->fanout <= kHeavyT) ? nullptr : blk->cls_perm;
+  BF_CHECK((launch_gather<TI, 0>(order, blk->row_ptr, p.col, blk->n_dst, (const TI*)a.h_src, a.ld_src,
                                  p.pitch_in, (__nv_bfloat16*)a.agg, a.ld_agg, s)));
   if (a.in_bf16)
     return tc_gemm_tma(blk->n_dst, a.layer1 ? kGatherTableRows : blk->n_dst, a.layer1 ? blk->src_global : nullptr,
