@@ -85,6 +85,20 @@ typedef struct {
   int32_t* cache[BUFFALO_MAX_LAYERS];
 } buffalo_sampler;
 
+/* A node-id-range sharded feature table (BASELINE.json configs[4], the IGB-shaped
+ * 1024-d table of 205 GB that no single GPU holds; the paper's data-parallel mode, PAPER.md:
+ * 458-471): rows [k * rows_per_shard, (k + 1) * rows_per_shard) live in shard k, a row-major
+ * table with the model's feat_pitch.  shard[k] are device pointers valid in the calling process:
+ * its own shard and the peers' shards opened with buffalo_ipc_open (NVLink peer mappings across
+ * the GPUs of one NVSwitch box; on one GPU, memory of other processes or plain allocations).
+ * Supported for feat_dtype BF16 with gemm_mode BF16 on sampled first blocks (fanout[0] > 0). */
+enum { BUFFALO_MAX_SHARDS = 8 };
+typedef struct {
+  int32_t num_shards;
+  int64_t rows_per_shard;
+  const void* shard[BUFFALO_MAX_SHARDS];
+} buffalo_feature_shards;
+
 /* GraphSAGE-mean model (R20): dim[0] = input feature width, dim[L] = #classes.
  * feat_dtype: dtype of the global feature table (row pitch feat_pitch elements, 16-B aligned
  * rows).  gemm_mode FFMA keeps activations in fp32; BF16 stores activations (H_l, saved
@@ -96,6 +110,11 @@ typedef struct {
   int32_t gemm_mode;
   int64_t feat_pitch;
   int32_t aggregator;       /* BUFFALO_AGG_MEAN (default) | _POOL | _LSTM (the last two: gemm_mode FFMA) */
+  /* nullable: the feature table is sharded (see buffalo_feature_shards); layer-1 h_src is then
+   * ignored, the Aggregate reads neighbour rows from their shards and also copies the dst rows'
+   * own feature rows into the block's self_rows (the Update and dW operands: one tensor map
+   * cannot span several allocations) */
+  const buffalo_feature_shards* feat_shards;
 } buffalo_model;
 
 /* Scheduler parameters (Alg. 3): mem_budget = M_ctr in bytes (arena bytes
@@ -162,6 +181,10 @@ typedef struct {
    * row longer than the fanout (<= BUFFALO_MAX_FANOUT < 129), so the forward Aggregate walks its
    * rows in natural order (sequential row_ptr / col reads) instead of through cls_perm. */
   int64_t fanout;
+  /* block 1 of a sharded feature table only (else NULL / 0): the dst rows' own feature rows,
+   * bf16 [n_dst][ld_self], written by the layer-1 Aggregate, read by the Update and dW GEMMs */
+  void* self_rows;
+  int64_t ld_self;
 } buffalo_block;
 
 typedef struct {
@@ -401,6 +424,19 @@ BUFFALO_API buffalo_status buffalo_triangles(const buffalo_graph* g, int64_t* T,
 BUFFALO_API buffalo_status buffalo_avg_clustering(const buffalo_graph* g, const int64_t* T, double* C_h,
                                       int64_t* C_ppm_h, void* workspace, size_t workspace_bytes,
                                       void* stream);
+
+/* ------------------------------------------------------------------ feature shards over IPC */
+/* Cross-process sharing of a feature shard (one process per GPU): the owner exports
+ * a device pointer as a handle (cudaIpcGetMemHandle of the driver allocation that contains it,
+ * followed by the pointer's 8-byte offset inside that allocation), the handles are exchanged over
+ * the process group (torch.distributed), every peer opens them (cudaIpcOpenMemHandle with lazy
+ * peer access: NVLink P2P loads on an NVSwitch box) and closes them (with the same handle) when
+ * done.  handle_h: host buffer of BUFFALO_IPC_HANDLE_BYTES.  Errors: INVALID_ARG (nulls, pointer
+ * outside a device allocation), CUDA (driver refusal). */
+enum { BUFFALO_IPC_HANDLE_BYTES = 72 };
+BUFFALO_API buffalo_status buffalo_ipc_export(const void* dev_ptr, void* handle_h);
+BUFFALO_API buffalo_status buffalo_ipc_open(const void* handle_h, void** dev_ptr_out_h);
+BUFFALO_API buffalo_status buffalo_ipc_close(const void* handle_h, void* dev_ptr);
 
 /* Number of kernels this thread has launched through the library (for bench accounting). */
 BUFFALO_API int64_t buffalo_launch_count(void);

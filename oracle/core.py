@@ -253,12 +253,14 @@ def lstm_dw_splits(n_rows, d):
     return max(1, min(_ceil(296, tiles), _ceil(max(int(n_rows), 1), 512)))
 
 
-def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
+def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean", sharded=False):
     """BucketMemEstimator reading R15: the exact arena bytes of one
     micro-batch with layer sizes n[0..L], e[1..L] (e indexed l-1) and widths dims[0..L].
     Returns (lo, hi): hi = capacity that always suffices (used as M_est), lo = bytes the
     backward pass is certain to touch; the measured arena peak lies in [lo, hi].
-    Every buffer is rounded up to 256 B.  Restated from DESIGN.md §5 "Arena"."""
+    Every buffer is rounded up to 256 B.  Restated from DESIGN.md §5 "Arena".  sharded: the
+    feature table is sharded over processes, so block 1 keeps a bf16 copy of its
+    dst rows' feature rows (the Update / dW operand)."""
     L = len(e)
     s = 4 if act_dtype == FP32 else 2
     pool = aggregator == "pool"                  # R28: fp32 only; block 1 keeps a transpose too
@@ -290,6 +292,8 @@ def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean"):
         if l < L:
             acts += _R(n[l] * pitch(dims[l]) * s)               # H_l
     acts += _R(n[L] * pitch(dims[L]) * 4)                       # logits
+    if sharded:
+        acts += _R(n[1] * pitch(dims[0]) * 2)                   # block 1's self-row copy (bf16)
     if gat:
         for l in range(1, L + 1):                               # Z, el, er, alpha per edge
             acts += _R(n[l - 1] * pitch(dims[l]) * 4) + _R(4 * n[l - 1]) + _R(4 * n[l]) + _R(4 * e[l - 1])
@@ -369,11 +373,11 @@ def grouping_weight(M, I, E, C_ppm):
     return min(M, (M * I * 1_000_000) // (E * C_ppm))
 
 
-def item_stats(g, seeds, L, fanout, seed, dims, act_dtype, aggregator="mean"):
+def item_stats(g, seeds, L, fanout, seed, dims, act_dtype, aggregator="mean", sharded=False):
     """O, E = sum D, I = unique src of the item's own output block, sizes, M_est (R13, R15)."""
     seeds = np.asarray(seeds, dtype=np.int32)
     n, e = block_sizes(g, seeds, L, fanout, seed)
-    lo, hi = mem_model(n, e, dims, act_dtype, aggregator)
+    lo, hi = mem_model(n, e, dims, act_dtype, aggregator, sharded)
     return dict(O=int(seeds.size), E=int(e[L - 1]), I=int(n[L - 1]), n=n, e=e, M=hi)
 
 
@@ -436,7 +440,7 @@ def _alg3_k_loop(stats, F, piece_stats, mem_budget, C_ppm, k_lo, k_max, fast_pat
 
 
 def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT64_MAX,
-             C_ppm=0, k_min=1, k_max=4096, num_gpus=1, aggregator="mean", fast_paths=True):
+             C_ppm=0, k_min=1, k_max=4096, num_gpus=1, aggregator="mean", fast_paths=True, sharded=False):
     """Alg. 3 Buffalo_Scheduler with the readings of DESIGN.md
     (R7 explosion test, R11 sort/placement keys, R16 K_max, R17 empty groups dropped,
     R24 k_min = #GPUs and LPT rank assignment, R25 fast paths).  Returns a dict plan or None
@@ -447,7 +451,7 @@ def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT6
     pos_of = {d: np.nonzero(bucket == d)[0] for d in range(F + 1)}
 
     def stats_of(pos):
-        st = item_stats(g, seeds[pos], L, fanout, seed, dims, act_dtype, aggregator)
+        st = item_stats(g, seeds[pos], L, fanout, seed, dims, act_dtype, aggregator, sharded)
         st["w"] = grouping_weight(st["M"], st["I"], st["E"], C_ppm)
         st["pos"] = pos
         return st

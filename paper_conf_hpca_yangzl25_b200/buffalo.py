@@ -33,6 +33,7 @@ EXPORTS = [
     "buffalo_clustering_workspace_bytes", "buffalo_triangles", "buffalo_avg_clustering",
     "buffalo_pool_fwd", "buffalo_pool_bwd", "buffalo_lstm_fwd", "buffalo_lstm_bwd",
     "buffalo_gat_fwd", "buffalo_gat_bwd", "buffalo_graph_validate",
+    "buffalo_ipc_export", "buffalo_ipc_open", "buffalo_ipc_close",
 ]
 
 
@@ -55,9 +56,18 @@ class Sampler(ctypes.Structure):
                 ("cache", c_p * MAX_LAYERS)]
 
 
+MAX_SHARDS = 8
+IPC_HANDLE_BYTES = 72
+
+
+class FeatureShards(ctypes.Structure):
+    _fields_ = [("num_shards", c_i32), ("rows_per_shard", c_i64), ("shard", c_p * MAX_SHARDS)]
+
+
 class Model(ctypes.Structure):
     _fields_ = [("num_layers", c_i32), ("dim", c_i32 * (MAX_LAYERS + 1)), ("feat_dtype", c_i32),
-                ("gemm_mode", c_i32), ("feat_pitch", c_i64), ("aggregator", c_i32)]
+                ("gemm_mode", c_i32), ("feat_pitch", c_i64), ("aggregator", c_i32),
+                ("feat_shards", ctypes.POINTER(FeatureShards))]
 
 
 class Sched(ctypes.Structure):
@@ -80,7 +90,8 @@ class Block(ctypes.Structure):
                 ("agg", c_p), ("out", c_p), ("dh", c_p), ("bwd_scratch", c_p),
                 ("ld_agg", c_i64), ("ld_out", c_i64), ("ld_dh", c_i64), ("bwd_scratch_bytes", c_i64),
                 ("pool_P", c_p), ("pool_arg", c_p), ("ld_pool", c_i64),
-                ("agg_saved", c_p), ("agg_saved_bytes", c_i64), ("fanout", c_i64)]
+                ("agg_saved", c_p), ("agg_saved_bytes", c_i64), ("fanout", c_i64),
+                ("self_rows", c_p), ("ld_self", c_i64)]
 
 
 class Blocks(ctypes.Structure):
@@ -130,6 +141,9 @@ def lib(require_gpu=True):
             "buffalo_gat_bwd": (c_i32, [P, c_i32, P, P, c_i64, P, c_i64, P, c_i64, P, c_sz, P, P, P, P, P, P, P, P,
                                         c_i64, P, c_sz, P]),
             "buffalo_graph_validate": (c_i32, [P, c_i32, P]),
+            "buffalo_ipc_export": (c_i32, [P, P]),
+            "buffalo_ipc_open": (c_i32, [P, P]),
+            "buffalo_ipc_close": (c_i32, [P, P]),
             "buffalo_status_str": (ctypes.c_char_p, [c_i32]),
             "buffalo_last_error": (ctypes.c_char_p, []),
         }
@@ -355,6 +369,24 @@ def clustering(graph, stream=None):
     return T, C, ppm
 
 
+def ipc_export(t):
+    """IPC handle (bytes) of the device memory at tensor t's data pointer."""
+    buf = ctypes.create_string_buffer(IPC_HANDLE_BYTES)
+    _check(lib().buffalo_ipc_export(ptr(t), buf))
+    return buf.raw
+
+
+def ipc_open(handle):
+    """Device pointer (int) of a peer's memory from its handle (lazy NVLink peer access)."""
+    out = c_p(0)
+    _check(lib().buffalo_ipc_open(ctypes.create_string_buffer(bytes(handle), IPC_HANDLE_BYTES), ctypes.byref(out)))
+    return out.value
+
+
+def ipc_close(handle, p):
+    _check(lib().buffalo_ipc_close(ctypes.create_string_buffer(bytes(handle), IPC_HANDLE_BYTES), p))
+
+
 def launch_count():
     return lib(False).buffalo_launch_count()
 
@@ -386,8 +418,24 @@ def make_sampler(fanout, F, seed, cache=None):
     return s
 
 
-def make_model(dims, feat_dtype=FP32, gemm_mode=GEMM_FFMA, feat_pitch=None, aggregator=AGG_MEAN):
+def make_shards(pointers, rows_per_shard):
+    """buffalo_feature_shards for a node-id-range sharded table (device pointers / tensors)."""
+    s = FeatureShards()
+    if not 1 <= len(pointers) <= MAX_SHARDS:
+        raise ValueError(f"1..{MAX_SHARDS} shards")
+    s.num_shards = len(pointers)
+    s.rows_per_shard = int(rows_per_shard)
+    for i, p in enumerate(pointers):
+        s.shard[i] = ptr(p)
+    return s
+
+
+def make_model(dims, feat_dtype=FP32, gemm_mode=GEMM_FFMA, feat_pitch=None, aggregator=AGG_MEAN, shards=None):
+    """shards: None or a FeatureShards struct (kept alive by the returned model)."""
     m = Model()
+    if shards is not None:
+        m.feat_shards = ctypes.pointer(shards)
+        m._shards_ref = shards
     m.num_layers = len(dims) - 1
     for i, d in enumerate(dims):
         m.dim[i] = int(d)

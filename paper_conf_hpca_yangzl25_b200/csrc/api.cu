@@ -1,6 +1,8 @@
 // api.cu — the C ABI (include/buffalo.h): validation, arena layout, the scheduler's K loop
 // (Alg. 3/4) and the memory model (R15).  Host code; all compute is in build.cu / sage.cu /
 // tc_sage.cu kernels.
+#include <cuda.h>
+
 #include <algorithm>
 #include <atomic>
 #include <cstdarg>
@@ -126,6 +128,7 @@ static void mem_model(int L, const int64_t* n, const int64_t* e, const buffalo_m
   if (m->aggregator == BUFFALO_AGG_GAT)
     for (int l = 1; l <= L; ++l) acts += gat_saved_bytes(n[l - 1], n[l], e[l - 1], m->dim[l]);
   acts += R(n[L] * pitch_of(m->dim[L]) * 4);
+  if (m->feat_shards) acts += R(n[1] * pitch_of(m->dim[0]) * 2);     // block 1's self_rows copy
   if (m->aggregator == BUFFALO_AGG_LSTM)
     for (int l = 1; l <= L; ++l) acts += R(lstm_saved_bytes(n[l], e[l - 1], m->dim[l - 1]));
   if (m->aggregator == BUFFALO_AGG_POOL)
@@ -170,6 +173,22 @@ static buffalo_status validate_model(const buffalo_model* m) {
   if (m->feat_pitch < round_up(m->dim[0], 8) || m->feat_pitch % 8) {
     set_error("model: feat_pitch must be a multiple of 8 and >= round_up(dim[0], 8)");
     return BUFFALO_ERR_INVALID_ARG;
+  }
+  if (const buffalo_feature_shards* sh = m->feat_shards) {
+    if (sh->num_shards < 1 || sh->num_shards > BUFFALO_MAX_SHARDS || sh->rows_per_shard < 1 ||
+        sh->rows_per_shard > INT32_MAX) {
+      set_error("model: feat_shards needs 1..%d shards of 1..2^31-1 rows", BUFFALO_MAX_SHARDS);
+      return BUFFALO_ERR_INVALID_ARG;
+    }
+    for (int k = 0; k < sh->num_shards; ++k)
+      if (!sh->shard[k] || ((uintptr_t)sh->shard[k]) % 16) {
+        set_error("model: feat_shards.shard[%d] is null or not 16-B aligned", k);
+        return BUFFALO_ERR_INVALID_ARG;
+      }
+    if (m->feat_dtype != BUFFALO_BF16 || m->gemm_mode != BUFFALO_GEMM_BF16 || m->aggregator != BUFFALO_AGG_MEAN) {
+      set_error("model: a sharded feature table is supported for the bf16 SAGE-mean path only");
+      return BUFFALO_ERR_UNSUPPORTED;
+    }
   }
   return BUFFALO_OK;
 }
@@ -331,6 +350,61 @@ buffalo_status buffalo_profile_end(double* ms_total_h, int64_t* launches_h, doub
   if (algo_bytes_h) *algo_bytes_h = bytes;
   for (cudaEvent_t e : g_prof.ev) cudaEventDestroy(e);
   g_prof = Profiler();
+  return BUFFALO_OK;
+}
+
+// The IPC handle covers a whole driver allocation (a caching allocator sub-allocates tensors
+// inside larger ones), so the exported handle carries the pointer's offset from its allocation
+// base after the 64-byte cudaIpcMemHandle_t.
+typedef CUresult (*MemGetAddressRangeFn)(CUdeviceptr*, size_t*, CUdeviceptr);
+
+buffalo_status buffalo_ipc_export(const void* dev_ptr, void* handle_h) {
+  if (!dev_ptr || !handle_h) {
+    set_error("ipc_export: null argument");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  static_assert(sizeof(cudaIpcMemHandle_t) + 8 == BUFFALO_IPC_HANDLE_BYTES, "IPC handle size");
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  BF_CUDA(cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q));
+  if (!fn || q != cudaDriverEntryPointSuccess) {
+    set_error("ipc_export: cuMemGetAddressRange unavailable");
+    return BUFFALO_ERR_CUDA;
+  }
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  if (((MemGetAddressRangeFn)fn)(&base, &size, (CUdeviceptr)dev_ptr) != CUDA_SUCCESS) {
+    set_error("ipc_export: the pointer is not inside a device allocation");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  cudaIpcMemHandle_t hd;
+  BF_CUDA(cudaIpcGetMemHandle(&hd, (void*)base));
+  const uint64_t off = (uint64_t)((CUdeviceptr)dev_ptr - base);
+  memcpy(handle_h, &hd, sizeof(hd));
+  memcpy((char*)handle_h + sizeof(hd), &off, 8);
+  return BUFFALO_OK;
+}
+
+buffalo_status buffalo_ipc_open(const void* handle_h, void** dev_ptr_out_h) {
+  if (!handle_h || !dev_ptr_out_h) {
+    set_error("ipc_open: null argument");
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  cudaIpcMemHandle_t hd;
+  uint64_t off = 0;
+  memcpy(&hd, handle_h, sizeof(hd));
+  memcpy(&off, (const char*)handle_h + sizeof(hd), 8);
+  void* p = nullptr;
+  BF_CUDA(cudaIpcOpenMemHandle(&p, hd, cudaIpcMemLazyEnablePeerAccess));
+  *dev_ptr_out_h = (char*)p + off;
+  return BUFFALO_OK;
+}
+
+buffalo_status buffalo_ipc_close(const void* handle_h, void* dev_ptr) {
+  if (!handle_h || !dev_ptr) return BUFFALO_ERR_INVALID_ARG;
+  uint64_t off = 0;
+  memcpy(&off, (const char*)handle_h + sizeof(cudaIpcMemHandle_t), 8);
+  BF_CUDA(cudaIpcCloseMemHandle((char*)dev_ptr - off));
   return BUFFALO_OK;
 }
 
@@ -613,6 +687,16 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
     set_error("build_blocks: null argument or empty group");
     return BUFFALO_ERR_INVALID_ARG;
   }
+  if (m->feat_shards) {
+    if ((int64_t)m->feat_shards->num_shards * m->feat_shards->rows_per_shard < g->num_nodes) {
+      set_error("build_blocks: the feature shards cover fewer rows than the graph has nodes");
+      return BUFFALO_ERR_INVALID_ARG;
+    }
+    if (sp->fanout[0] <= 0) {
+      set_error("build_blocks: a sharded feature table needs a sampled first block (fanout[0] > 0)");
+      return BUFFALO_ERR_UNSUPPORTED;
+    }
+  }
   if (((uintptr_t)arena) % 256) {
     set_error("build_blocks: arena must be 256-B aligned");
     return BUFFALO_ERR_INVALID_ARG;
@@ -692,6 +776,11 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
     b->agg = m->aggregator == BUFFALO_AGG_GAT ? nullptr : A.take(b->n_dst * b->ld_agg * sa);
     b->ld_out = pitch_of(m->dim[l]);
     b->out = A.take(b->n_dst * b->ld_out * (l < L ? sa : 4));
+  }
+  if (m->feat_shards) {
+    buffalo_block* b = &out->layer[0];
+    b->ld_self = pitch_of(m->dim[0]);
+    b->self_rows = A.take(b->n_dst * b->ld_self * 2);
   }
   if (m->aggregator == BUFFALO_AGG_POOL)
     for (int l = 1; l <= L; ++l) {
@@ -797,6 +886,13 @@ buffalo_status buffalo_sage_fwd(const buffalo_block* blk, int32_t layer, const b
   a.agg = saved_agg;
   a.ld_agg = ld_agg;
   if (a.layer1 && !blk->col_global) return BUFFALO_ERR_INVALID_ARG;
+  if (a.layer1 && m->feat_shards) {
+    if (!blk->self_rows || blk->fanout <= 0 || blk->fanout > 128) {
+      set_error("sage_fwd: sharded features need block 1 built with the sharded model and a sampled fanout");
+      return BUFFALO_ERR_INVALID_ARG;
+    }
+    a.shards = m->feat_shards;
+  }
   if (ld_out < pitch_of(a.d_out) || ld_agg < pitch_of(a.d_in) || a.ld_src < pitch_of(a.d_in) ||
       ld_out % 8 || ld_agg % 8 || a.ld_src % 8) {
     set_error("sage_fwd: leading dimensions must be multiples of 8 and >= the padded widths");
@@ -860,6 +956,13 @@ buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const b
   a.ld_dh_src = ld_dh_src;
   a.scratch = scratch;
   a.scratch_bytes = (int64_t)scratch_bytes;
+  if (a.layer1 && m->feat_shards) {
+    if (!blk->self_rows) {
+      set_error("sage_bwd: sharded features need block 1 built with the sharded model");
+      return BUFFALO_ERR_INVALID_ARG;
+    }
+    a.shards = m->feat_shards;
+  }
   cudaStream_t s = (cudaStream_t)stream;
   if (m->gemm_mode == BUFFALO_GEMM_BF16) {
     if (!tc_bwd_supported(a)) return BUFFALO_ERR_UNSUPPORTED;

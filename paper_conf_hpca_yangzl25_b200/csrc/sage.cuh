@@ -16,6 +16,7 @@ struct FwdArgs {
   const float* W; const void* W_packed; const float* b;
   void* out; int64_t ld_out;
   void* agg; int64_t ld_agg;
+  const buffalo_feature_shards* shards;   // layer 1 of a sharded feature table (else null)
 };
 
 struct BwdArgs {
@@ -30,6 +31,7 @@ struct BwdArgs {
   float* dW; float* db;
   float* dh_src; int64_t ld_dh_src;
   void* scratch; int64_t scratch_bytes;
+  const buffalo_feature_shards* shards;   // layer 1 of a sharded feature table (else null)
 };
 
 // GraphSAGE-pool (R28): FFMA path, fp32 activations.

@@ -222,9 +222,6 @@ template <> __device__ __forceinline__ void acc_piece<float>(float* acc, const u
   acc[2] += __uint_as_float(u.z); acc[3] += __uint_as_float(u.w);
 }
 
-// MODE 0: forward (mean of neighbour rows, long-tail rows pre-aggregated, h_agg saved,
-//         + bias, ReLU).  MODE 1: backward dH (plain sum of pre-scaled dZ/D rows over the
-//         transposed block, self half = dZ for rows < self_rows, fp32 output).
 // Super-chunk schedule of a tile (identical on the gather and the MMA side): the self half in
 // groups of kSuper K-chunks, then the aggregate half in groups of kAggChunks(E) K-chunks
 // (32 lanes x 16 B = one warp-wide row slice).
@@ -547,13 +544,27 @@ buffalo_status launch_agg_heavy_bf16(const FwdArgs& a, cudaStream_t s);
 // dH_{l-1}[j]; ReLU' with H_{l-1}[j] makes dZ_{l-1}[j], stored in bf16, and its columns are
 // summed (db_{l-1}) per lane group in shared memory and per CTA in a fixed order (one partial
 // row per CTA: deterministic).
+// MODE 3 is MODE 0 over a node-range sharded feature table (buffalo_feature_shards): a
+// neighbour's row address is shard[j / rps] + (j % rps) * row bytes, computed once per index by
+// the lane that fetched it and broadcast as a 64-bit address; the dst row's own feature row
+// (global id gidx[row]) is copied to self_out for the Update and dW GEMMs.
 struct GatherEpi {
   const __nv_bfloat16* ys; int64_t ldy;   // Ys [n_self][ldy]
   int64_t n_self;
   const __nv_bfloat16* H; int64_t ldH;    // H_{l-1} (ReLU' mask source)
   int d;                                  // valid columns (d_{l-1}); pad columns are stored as 0
   float* db_part;                         // [gridDim.x][d]
+  // MODE 3
+  const char* shard[BUFFALO_MAX_SHARDS];
+  uint32_t rps;                           // rows per shard
+  const int32_t* gidx;                    // global id of each dst row (block 1's src_global)
+  __nv_bfloat16* self_out; int64_t ld_self;
 };
+
+__device__ __forceinline__ long long shard_row(const GatherEpi& ep, int32_t j, int32_t ldb) {
+  const uint32_t u = (uint32_t)j;
+  return (long long)(ep.shard[u / ep.rps] + (int64_t)(u % ep.rps) * ldb);
+}
 
 template <class TI, int MODE, int LPR, int kU, int MINB>
 __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restrict__ perm,
@@ -566,6 +577,7 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
   constexpr int E = InTraits<TI>::kElems;
   constexpr int G = 32 / LPR;
   constexpr unsigned kFull = 0xffffffffu;
+  constexpr bool SH = MODE == 3;                      // sharded feature table
   const int lane = threadIdx.x & 31;
   const int g = lane / LPR, pc = lane & (LPR - 1);
   const int gbase = g * LPR;
@@ -611,11 +623,16 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
       const bool colok = piece < npieces;
       // lanes past the row read piece 0 again (same sectors, in bounds) and store nothing
       const char* hb = reinterpret_cast<const char*>(h) + (colok ? piece : 0) * 16;
+      const int64_t poff = (colok ? piece : 0) * 16;
       float acc[E];
 #pragma unroll
       for (int k = 0; k < E; ++k) acc[k] = 0.f;
       for (int32_t base = 0; base < Dmax; base += LPR) {
         const int32_t jj = (base + pc < Dl) ? __ldg(col + b + base + pc) : -1;
+        long long ja = -1;                              // MODE 3: the row's address
+        if constexpr (SH) {
+          if (jj >= 0) ja = shard_row(ep, jj, ldb);
+        }
         const int m = min(LPR, Dmax - base);
         int k = 0;
         if (uni) {                                      // full groups of kU edges: no predicates
@@ -623,8 +640,13 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
             uint4 raw[kU];
 #pragma unroll
             for (int uu = 0; uu < kU; ++uu) {
-              const int32_t jn = __shfl_sync(kFull, jj, gbase + k + uu);
-              raw[uu] = __ldg(reinterpret_cast<const uint4*>(hb + (int64_t)jn * ldb));
+              if constexpr (SH) {
+                const long long an = __shfl_sync(kFull, ja, gbase + k + uu);
+                raw[uu] = __ldg(reinterpret_cast<const uint4*>(an + poff));
+              } else {
+                const int32_t jn = __shfl_sync(kFull, jj, gbase + k + uu);
+                raw[uu] = __ldg(reinterpret_cast<const uint4*>(hb + (int64_t)jn * ldb));
+              }
             }
 #pragma unroll
             for (int uu = 0; uu < kU; ++uu) acc_piece<TI>(acc, raw[uu]);
@@ -635,18 +657,31 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
           bool ok[kU];
 #pragma unroll
           for (int uu = 0; uu < kU; ++uu) {
-            const int32_t jn = __shfl_sync(kFull, jj, gbase + ((k + uu) & (LPR - 1)));
-            ok[uu] = k + uu < m && jn >= 0;
-            if (ok[uu]) raw[uu] = __ldg(reinterpret_cast<const uint4*>(hb + (int64_t)jn * ldb));
+            if constexpr (SH) {
+              const long long an = __shfl_sync(kFull, ja, gbase + ((k + uu) & (LPR - 1)));
+              ok[uu] = k + uu < m && an != -1;
+              if (ok[uu]) raw[uu] = __ldg(reinterpret_cast<const uint4*>(an + poff));
+            } else {
+              const int32_t jn = __shfl_sync(kFull, jj, gbase + ((k + uu) & (LPR - 1)));
+              ok[uu] = k + uu < m && jn >= 0;
+              if (ok[uu]) raw[uu] = __ldg(reinterpret_cast<const uint4*>(hb + (int64_t)jn * ldb));
+            }
           }
 #pragma unroll
           for (int uu = 0; uu < kU; ++uu)
             if (ok[uu]) acc_piece<TI>(acc, raw[uu]);
         }
       }
+      if constexpr (SH) {                               // the dst row's own feature row
+        if (row >= 0 && colok) {
+          const long long sa = shard_row(ep, __ldg(ep.gidx + row), ldb);
+          *reinterpret_cast<uint4*>(ep.self_out + (int64_t)row * ep.ld_self + piece * E) =
+              __ldg(reinterpret_cast<const uint4*>(sa + poff));
+        }
+      }
       if (row >= 0 && D <= kHeavyT && colok) {
         float v[E];
-        if (MODE == 0 && D > 0) {
+        if ((MODE == 0 || MODE == 3) && D > 0) {
           const float fd = (float)D;
           const float y = 1.0f / fd;                    // once per row
 #pragma unroll
@@ -714,9 +749,6 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   const int npieces = (pitch_in + E - 1) / E;
   int lpr_log = 0;
   while ((1 << lpr_log) < npieces && lpr_log < 5) ++lpr_log;
-  // transposed rows are short (~1-2 entries per src row): two rows per warp (two passes over
-  // the row's pieces) keep twice the per-row metadata chains in flight
-  if (MODE == 1 && lpr_log == 5) lpr_log = 4;
   if (n > INT32_MAX || ldh * (int64_t)sizeof(TI) > INT32_MAX) {
     set_error("gather: %lld rows of stride %lld elements exceed the 32-bit row / byte-stride range",
               (long long)n, (long long)ldh);
@@ -778,6 +810,44 @@ static buffalo_status launch_gather_epi(const int32_t* perm, const int32_t* rp, 
   return BUFFALO_OK;
 }
 
+// MODE 3: the layer-1 Aggregate over a sharded feature table (bf16), plus the self-row copy.
+static buffalo_status launch_gather_sharded(const buffalo_block* blk, const buffalo_feature_shards* sh, int64_t ld_src,
+                                           int pitch_in, __nv_bfloat16* out, int64_t ldo, cudaStream_t s) {
+  const int64_t n = blk->n_dst;
+  if (n <= 0) return BUFFALO_OK;
+  const int npieces = (pitch_in + 7) / 8;
+  int lpr_log = 0;
+  while ((1 << lpr_log) < npieces && lpr_log < 5) ++lpr_log;
+  if (n > INT32_MAX || ld_src * 2 > INT32_MAX) {
+    set_error("gather: %lld rows of stride %lld elements exceed the 32-bit row / byte-stride range",
+              (long long)n, (long long)ld_src);
+    return BUFFALO_ERR_INVALID_ARG;
+  }
+  GatherEpi ep{};
+  for (int k = 0; k < sh->num_shards; ++k) ep.shard[k] = (const char*)sh->shard[k];
+  ep.rps = (uint32_t)sh->rows_per_shard;
+  ep.gidx = blk->src_global;
+  ep.self_out = (__nv_bfloat16*)blk->self_rows;
+  ep.ld_self = blk->ld_self;
+  const ProfSlot ps = prof_begin_launch("gather", s);
+  constexpr int kU = 2, kMinB = 6;
+  const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
+  const int32_t n32 = (int32_t)n, ldb = (int32_t)(ld_src * 2);
+  const __nv_bfloat16* h0 = (const __nv_bfloat16*)sh->shard[0];
+#define BF_V2S(L) k_gather_v2<__nv_bfloat16, 3, L, kU, kMinB><<<fgrid, 256, 0, s>>>( \
+      nullptr, blk->row_ptr, blk->col_global, n32, h0, ldb, npieces, out, ldo, ps.edges_dev, ep)
+  if (lpr_log <= 2) BF_V2S(4);
+  else if (lpr_log == 3) BF_V2S(8);
+  else if (lpr_log == 4) BF_V2S(16);
+  else BF_V2S(32);
+#undef BF_V2S
+  BF_LAUNCHED("k_gather_sharded");
+  // algorithmic bytes: per row row_ptr pair + id + the self row read and copied + bf16 output
+  // row; per edge index + source row
+  prof_end_launch(ps, s, (double)n * (12.0 + 6.0 * pitch_in), 4.0 + (double)pitch_in * 2);
+  return BUFFALO_OK;
+}
+
 // Feature-table rows are addressed through src_global only; the gathered tensor map spans the
 // largest row count TMA accepts and tile padding rows gather row 0 (their outputs are dropped).
 constexpr int64_t kGatherTableRows = 0x7fffffff;
@@ -807,6 +877,16 @@ template <class TI>
 static buffalo_status tc_fwd_t(const FwdArgs& a, cudaStream_t s) {
   const buffalo_block* blk = a.blk;
   if (blk->n_dst <= 0) return BUFFALO_OK;
+  if (a.shards) {
+    // sharded feature table (layer 1, sampled block): Aggregate + self-row copy, then the Update
+    // over two contiguous bf16 operands
+    BF_CHECK(launch_gather_sharded(blk, a.shards, a.ld_src, (int)pitch_of(a.d_in), (__nv_bfloat16*)a.agg, a.ld_agg,
+                                   s));
+    const uint8_t* wpk = (const uint8_t*)a.W_packed + R((int64_t)2 * a.d_in * a.d_out * 4);
+    return tc_gemm_tma(blk->n_dst, blk->n_dst, nullptr, (const __nv_bfloat16*)blk->self_rows, blk->ld_self,
+                       (const __nv_bfloat16*)a.agg, a.ld_agg, a.d_in, wpk, a.d_out, a.b, a.relu, a.out_f32, a.out,
+                       a.ld_out, s);
+  }
   BF_CHECK(launch_agg_heavy_bf16(a, s));
   TcFwdParams p{};
   p.row_ptr = blk->row_ptr;
@@ -1142,58 +1222,10 @@ __global__ void __launch_bounds__(256) k_reduce_db(const float* __restrict__ par
   }
 }
 
-// Long-tail transposed rows (more than kHeavyT dst): out[h] = sum_{t in T(list[h])} z[t_col[t]],
-// 8 warps over the entries (warp w takes t = w, w+8, ...), combined in warp order.
-__global__ void __launch_bounds__(256) k_sum_heavy_rows(const int32_t* __restrict__ perm, int64_t n,
-                                                        const int32_t* __restrict__ rp,
-                                                        const int32_t* __restrict__ col,
-                                                        const __nv_bfloat16* __restrict__ z, int64_t ldz,
-                                                        int dp, __nv_bfloat16* __restrict__ out, int by_row) {
-  __shared__ float part[8][32][8];
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  for (int64_t hh = blockIdx.x; hh < n; hh += gridDim.x) {
-  const int64_t j = perm[n - 1 - hh];          // heavy rows: the tail of the degree-class perm
-  const int32_t b = rp[j], e_end = rp[j + 1];
-  if (e_end - b <= kHeavyT) break;
-  const int nch = dp / 8;
-  for (int c0 = 0; c0 < nch; c0 += 32) {
-    const int c = c0 + lane;
-    float acc[8];
-#pragma unroll
-    for (int k = 0; k < 8; ++k) acc[k] = 0.f;
-    if (c < nch) {
-      int32_t t = b + w;
-      for (; t + 24 < e_end; t += 32) {                  // four rows in flight per lane
-        uint4 r[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) r[u] = __ldg(reinterpret_cast<const uint4*>(z + (int64_t)col[t + 8 * u] * ldz + c * 8));
-#pragma unroll
-        for (int u = 0; u < 4; ++u) acc_piece<__nv_bfloat16>(acc, r[u]);
-      }
-      for (; t < e_end; t += 8)
-        acc_piece<__nv_bfloat16>(acc, __ldg(reinterpret_cast<const uint4*>(z + (int64_t)col[t] * ldz + c * 8)));
-    }
-#pragma unroll
-    for (int k = 0; k < 8; ++k) part[w][lane][k] = acc[k];
-    __syncthreads();
-    if (w == 0 && c < nch) {
-#pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        float s = part[0][lane][k];
-        for (int ww = 1; ww < 8; ++ww) s += part[ww][lane][k];
-        acc[k] = s;
-      }
-      *reinterpret_cast<uint4*>(out + (by_row ? j : hh) * dp + c * 8) =
-          make_uint4(pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]), pack_bf16x2(acc[4], acc[5]),
-                     pack_bf16x2(acc[6], acc[7]));
-    }
-    __syncthreads();
-  }
-  }
-}
 
-// The backward's long-tail transposed rows with the fused epilogue of GatherEpi: the same sum
-// as k_sum_heavy_rows (8 warps over the entries, combined in warp order), then + Ys[j] (j <
+// The backward's long-tail transposed rows (more than kHeavyT dst) with the fused epilogue of
+// GatherEpi: 8 warps over the row's entries (warp w takes t = w, w+8, ...), combined in warp
+// order (the split depends only on the row: deterministic), then + Ys[j] (j <
 // n_self), ReLU' with H[j], bf16 dZ_{l-1}[j], and the column sums of this CTA's heavy rows (in
 // row order) as db partial row kGatherDbCtas + blockIdx.x.  A fixed grid of kHeavyDbCtas CTAs:
 // CTAs without heavy rows write zero partials.
@@ -1328,7 +1360,10 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     BF_LAUNCHED("k_dz_prep");
   }
   // dW (TMA-fed tensor cores, deterministic split reduction) and db
-  if (a.in_bf16) {
+  if (a.shards) {            // layer 1 of a sharded table: the self rows were copied by the forward
+    BF_CHECK(tc_dw_tma(n, S, zb, dp, d_out, (const __nv_bfloat16*)blk->self_rows, blk->ld_self, nullptr, n,
+                       (const __nv_bfloat16*)a.agg, a.ld_agg, d_in, dw_part, s));
+  } else if (a.in_bf16) {
     BF_CHECK(tc_dw_tma(n, S, zb, dp, d_out, (const __nv_bfloat16*)a.h_src, a.ld_src,
                        a.layer1 ? blk->src_global : nullptr, kGatherTableRows, (const __nv_bfloat16*)a.agg,
                        a.ld_agg, d_in, dw_part, s));

@@ -81,6 +81,45 @@ class PlanBuffers:
         self.plan.group_sizes_h = self.sizes_h.ctypes.data
 
 
+class ShardedFeatures:
+    """A node-id-range sharded bf16 feature table (include/buffalo.h buffalo_feature_shards; the
+    IGB-shaped configuration): shard k holds the rows [k * rows_per_shard, ...).
+    `shards` are CUDA tensors of this process (its own shard, or all of them on one GPU) or raw
+    device pointers opened from peers (buffalo_ipc_open); `pitch` is the row pitch in elements."""
+
+    def __init__(self, shards, rows_per_shard, num_rows, pitch, keep=()):
+        self.struct = B.make_shards(shards, rows_per_shard)
+        self.rows_per_shard = int(rows_per_shard)
+        self.shape = (int(num_rows), int(pitch))
+        self.dtype = torch.bfloat16
+        self._keep = list(shards) + list(keep)
+        local = [s for s in shards if torch.is_tensor(s)]
+        self.first = local[0] if local else None        # a local tensor for the binding's dtype check
+
+
+def exchange_shards(local, rank, world, rows_per_shard, num_rows, group=None):
+    """One process per GPU: export this rank's shard (a CUDA tensor), all-gather the 64-byte IPC
+    handles over the process group, open the peers' shards (NVLink peer mappings on an NVSwitch
+    box).  Returns (ShardedFeatures, close) — call close() before the peers free their shards."""
+    import torch.distributed as dist
+    handles = [None] * world
+    dist.all_gather_object(handles, B.ipc_export(local), group=group)
+    ptrs, opened = [], []
+    for r in range(world):
+        if r == rank:
+            ptrs.append(local)
+        else:
+            p = B.ipc_open(handles[r])
+            opened.append((handles[r], p))
+            ptrs.append(p)
+
+    def close():
+        for h, p in opened:
+            B.ipc_close(h, p)
+        opened.clear()
+    return ShardedFeatures(ptrs, rows_per_shard, num_rows, local.shape[1], keep=[local]), close
+
+
 class SageParams:
     """fp32 master weights/biases (Xavier init from synth), flat gradient buffer, packed copies."""
 
@@ -175,7 +214,9 @@ class Trainer:
             raise ValueError("GAT needs its attention vectors (a_l, a_r per layer)")
         if self.is_lstm and lstm is None:
             raise ValueError("the LSTM aggregator needs its weights (W_ih, W_hh, b per layer)")
-        self.model = B.make_model(dims, feat_dtype, gemm_mode, feats.shape[1], aggregator)
+        self.sharded = isinstance(feats, ShardedFeatures)
+        self.model = B.make_model(dims, feat_dtype, gemm_mode, feats.shape[1], aggregator,
+                                  shards=feats.struct if self.sharded else None)
         self.sched = B.make_sched(mem_budget, C_ppm, k_min, k_max, world)
         self.params = SageParams(self.model, Ws, bs, device, Wps, bps, lstm, gat)
         self.rank, self.world, self.pg = rank, world, process_group
@@ -276,9 +317,13 @@ class Trainer:
                     raise
                 self._ensure_arena(max(int(e.required * 1.25), 2 * self.arena.numel(), 1 << 20))
 
+    def _feat_arg(self):
+        """Layer-1 h_src: the feature table (ignored by the library for a sharded one)."""
+        return self.feats.first if self.sharded else self.feats
+
     def forward(self):
         m, p, blks = self.model, self.params, self.blocks
-        h, ld = self.feats, self.feats.shape[1]
+        h, ld = self._feat_arg(), self.feats.shape[1]
         for l in range(1, self.L + 1):
             b = blks.layer[l - 1]
             if self.is_gat:
@@ -302,7 +347,7 @@ class Trainer:
                 prev = blks.layer[l - 2]
                 h_src, ld_src, dh_src, ld_dh_src = prev.out, prev.ld_out, prev.dh, prev.ld_dh
             else:
-                h_src, ld_src, dh_src, ld_dh_src = self.feats, self.feats.shape[1], None, 0
+                h_src, ld_src, dh_src, ld_dh_src = self._feat_arg(), self.feats.shape[1], None, 0
             h_dst = b.out if l < self.L else None
             if self.is_gat:
                 B.gat_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, h_dst, b.ld_out, p.W[l - 1], p.al[l - 1],

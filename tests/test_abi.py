@@ -58,6 +58,21 @@ def test_estimate_mem_equals_oracle(blib, gemm, agg):
                                                          ("mean", "pool", "lstm", "gat")[agg])
 
 
+def test_estimate_mem_sharded_equals_oracle(blib):
+    """The sharded-feature-table model (bf16, SAGE-mean) adds block 1's self-row copy."""
+    rng = np.random.default_rng(99)
+    sh = blib.make_shards([1 << 20, 2 << 20, 3 << 20], 1000)        # pointers are not dereferenced here
+    for _ in range(100):
+        L = int(rng.integers(1, 4))
+        dims = [int(x) for x in rng.integers(1, 257, L + 1)]
+        dims[0] = int(rng.integers(1, 2000))
+        n = [int(x) for x in rng.integers(0, 300000, L + 1)]
+        e = [int(x) for x in rng.integers(0, 3000000, L)]
+        m = blib.make_model(dims, feat_dtype=1, gemm_mode=1, shards=sh)
+        assert blib.estimate_mem(n, e, m) == O.mem_model(n, e, dims, O.BF16, sharded=True)
+        assert blib.estimate_mem(n, e, m)[0] > O.mem_model(n, e, dims, O.BF16)[0] or n[1] == 0
+
+
 def test_cuda_philox_known_answers(tmp_path):
     src = tmp_path / "kat.cu"
     src.write_text('#include <cstdio>\n#include "philox.cuh"\nint main(){unsigned v[6];\n'
