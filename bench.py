@@ -43,7 +43,15 @@ WORKLOADS = {
                "bucket groups"),
     "products": ("ogbn-products-shaped power-law graph (2,449,029 nodes, 61,859,140 edges, 100-d), 3-layer "
                  "SAGE-mean 100-256-256-47, fanout (10,25,30), budget forcing >= 8 bucket groups"),
+    "igb_small": ("IGB-large-shaped power-law graph at 1/8 scale (12,500,000 nodes, 150,000,000 undirected edges, "
+                  "1024-d bf16 features = 25.6 GB held as node-range shards: 8 on one GPU, one per rank over "
+                  "CUDA IPC / NVLink at N > 1), 3-layer SAGE-mean 1024-256-256-19, fanout (5,10,15), F=15, "
+                  "125,000 seeds, budget forcing >= 8 bucket groups"),
+    "igb": ("IGB-large-shaped power-law graph (100,000,000 nodes, 1,200,000,000 undirected edges, 1024-d bf16 "
+            "features = 205 GB sharded by node range, one shard per rank over CUDA IPC / NVLink), 3-layer "
+            "SAGE-mean 1024-256-256-19, fanout (5,10,15), F=15, 1,000,000 seeds, budget forcing >= 8 groups"),
 }
+SHARDED = ("igb", "igb_small")
 
 
 # Table II's average clustering coefficients, logged beside the C measured
@@ -78,16 +86,21 @@ def dist_env():
     return rank, world, local
 
 
-def make_inputs_device(cfg, feat_dtype=None):
+def make_inputs_device(cfg, feat_dtype=None, shards=None):
     """The same inputs as make_inputs, generated on the GPU by synth.device (bit-identical to
     the numpy recipe; a products-shaped graph takes seconds instead of minutes on one core).
     feat_dtype: generate the feature table directly in that dtype (k/128 values are exact in
-    bf16; the papers-shaped table is 28 GB in bf16, 57 GB in fp32)."""
+    bf16; the papers-shaped table is 28 GB in bf16, 57 GB in fp32).  shards: a list of node
+    ranges (r0, r1): X is then the list of those row ranges of the table (separate allocations)."""
     import torch
     from synth import device as SD
     rp, col = SD.random_graph(cfg.N, cfg.pairs, cfg.kind)
     torch.cuda.empty_cache()
-    X = SD.features(cfg.N, cfg.d0, ((cfg.d0 + 31) // 32) * 32, dtype=feat_dtype or torch.float32)
+    pitch = ((cfg.d0 + 31) // 32) * 32
+    if shards is not None:
+        X = [SD.features_range(r0, r1, cfg.d0, pitch, dtype=feat_dtype or torch.float32) for r0, r1 in shards]
+    else:
+        X = SD.features(cfg.N, cfg.d0, pitch, dtype=feat_dtype or torch.float32)
     y = SD.labels(cfg.N, cfg.classes)
     seeds = SD.seed_nodes(cfg.N, cfg.S)
     Ws, bs = xavier_weights(cfg.dims)
@@ -146,6 +159,10 @@ def oracle_sample(cfg, rp, col, X, y, seeds, Ws, bs, seconds, edges_per_epoch=No
 def run_reference(args, cfg):
     rank, world, _ = dist_env()
     if rank != 0:
+        return
+    if args.config in SHARDED:
+        print(json.dumps({"impl": "reference", "unavailable": "the IGB-shaped 1024-d table (25.6-205 GB) is not "
+                          "copied to the host for the oracle; its arm runs on the products/papers/arxiv configs"}))
         return
     try:
         import torch
@@ -354,9 +371,26 @@ def run_ours(args, cfg):
 
     B.lib()
     t_gen = time.perf_counter()
-    big = cfg.N > 50_000_000              # papers / IGB shapes: bf16 table generated directly, no fp32 copy
-    rp, col, X, y, seeds, Ws, bs = make_inputs_device(cfg, torch.bfloat16 if (big and args.gemm == "bf16") else None)
+    big = cfg.N > 50_000_000 or args.config in SHARDED  # bf16 table generated directly, no fp32 copy
+    sharded = args.config in SHARDED
+    shard_ranges, rps = None, None
+    if sharded:
+        if args.gemm != "bf16" or args.aggregator != "mean":
+            raise SystemExit("the sharded IGB-shaped configs run the bf16 SAGE-mean path")
+        P = 8 if world == 1 else world            # one GPU: 8 local shards; else one shard per rank
+        rps = (cfg.N + P - 1) // P
+        mine = range(P) if world == 1 else [rank]
+        shard_ranges = [(k * rps, min(cfg.N, (k + 1) * rps)) for k in mine]
+    rp, col, X, y, seeds, Ws, bs = make_inputs_device(cfg, torch.bfloat16 if (big and args.gemm == "bf16") else None,
+                                                      shard_ranges)
     t_gen = time.perf_counter() - t_gen
+    shard_close = None
+    if sharded:
+        from paper_conf_hpca_yangzl25_b200.train import ShardedFeatures, exchange_shards
+        if world == 1:
+            X = ShardedFeatures(X, rps, cfg.N, X[0].shape[1])
+        else:
+            X, shard_close = exchange_shards(X[0], rank, world, rps, cfg.N, group=pg)
     pool = args.aggregator == "pool"
     lstm = args.aggregator == "lstm"
     gat = args.aggregator == "gat"
@@ -377,7 +411,7 @@ def run_ours(args, cfg):
         agg_kw = dict(aggregator=B.AGG_GAT, gat=(als, ars))
     feat_dtype = B.BF16 if args.gemm == "bf16" else B.FP32
     feats = X
-    if feat_dtype == B.BF16 and feats.dtype != torch.bfloat16:
+    if not sharded and feat_dtype == B.BF16 and feats.dtype != torch.bfloat16:
         feats = feats.to(torch.bfloat16).contiguous()      # k/128 features are exact in bf16
     kmin = max(cfg.k_min, world)
     budget = cfg.mem_budget
@@ -392,7 +426,7 @@ def run_ours(args, cfg):
                  C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg,
                  pipeline=not args.no_pipeline, **agg_kw)
     full_batch_edges = None
-    if args.config in ("products", "papers", "arxiv_lstm"):
+    if args.config in ("products", "papers", "arxiv_lstm") + SHARDED:
         # calibrate M_ctr once so that one GPU needs >= 8 groups (products; 2 for the LSTM
         # workload), then freeze it for every N
         B_full = Trainer(graph, feats, y, seeds, cfg.dims,
@@ -539,6 +573,7 @@ def run_ours(args, cfg):
                     "redundancy": (edges / args.steps / full_batch_edges) if full_batch_edges else None,
                     "phases_ms_sequential": phases, "block_build": build_rates,
                     "parallelism": f"dp{world} over bucket groups",
+                    "feature_shards": ((8 if world == 1 else world) if sharded else None),
                     "pipeline": "scheduler of epoch e+1 overlapped with epoch e" if not args.no_pipeline else "off",
                     "C_eq1": C_eq1, "C_ppm": C_ppm, "C_table2": C_TABLE2.get(args.config),
                     "C_seconds": t_c},
@@ -548,7 +583,11 @@ def run_ours(args, cfg):
                  "d2h_bytes_per_step": 4},
             gpu_launches=launches, clocks=clk, memory=mem_est)
         print(json.dumps(line), flush=True)
+    if shard_close is not None:
+        torch.distributed.barrier()          # every rank is done reading the peers' shards
+        shard_close()
     if world > 1:
+        torch.distributed.barrier()
         torch.distributed.destroy_process_group()
 
 

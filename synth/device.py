@@ -177,17 +177,22 @@ def random_graph(N, E, kind, seed=GRAPH_SEED, device="cuda"):
 
 def features(N, d, pitch=None, seed=DATA_SEED, dtype=torch.float32, device="cuda"):
     """x[v][k] = ((w>>24)-128)/128 with w = word (k&3) of Philox(seed; v, 0, k>>2, tag 1)."""
+    return features_range(0, N, d, pitch, seed, dtype, device)
+
+
+def features_range(r0, r1, d, pitch=None, seed=DATA_SEED, dtype=torch.float32, device="cuda"):
+    """Rows [r0, r1) of the feature table of `features` (one shard of a node-range sharded table)."""
     pitch = pitch or d
-    out = torch.zeros((N, pitch), dtype=dtype, device=device)
+    out = torch.zeros((r1 - r0, pitch), dtype=dtype, device=device)
     nb = (d + 3) // 4
     rows = max(1, (_CHUNK * 4) // nb)
     blk = torch.arange(nb, dtype=torch.int64, device=device)[None, :]
-    for s in range(0, N, rows):
-        e = min(N, s + rows)
+    for s in range(r0, r1, rows):
+        e = min(r1, s + rows)
         v = torch.arange(s, e, dtype=torch.int64, device=device)[:, None]
         w = philox_words(seed, v, 0, blk, TAG_FEAT)
         vals = torch.stack([(x >> 24) - 128 for x in w], dim=2).reshape(e - s, nb * 4)[:, :d]
-        out[s:e, :d] = (vals.to(torch.float32) / 128.0).to(dtype)
+        out[s - r0:e - r0, :d] = (vals.to(torch.float32) / 128.0).to(dtype)
     return out
 
 

@@ -320,6 +320,10 @@ CONFIGS = {
     # configs[4]: IGB-large-shaped, 3-layer, fanout (5,10,15).
     "igb": Config("igb", 100000000, 1200000000, "powerlaw", 1024, 19, 256, 3, [5, 10, 15], 15,
                   1000000, 8, 4096),
+    # configs[4] at 1/8 of the nodes, edges and seeds (one GPU's share of the 8-GPU run: a 25.6 GB
+    # 1024-d bf16 table, held as 8 node-range shards), for the single-GPU bench and tests.
+    "igb_small": Config("igb_small", 12500000, 150000000, "powerlaw", 1024, 19, 256, 3, [5, 10, 15], 15,
+                        125000, 8, 4096),
 }
 
 
