@@ -73,6 +73,10 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-baseline-seconds", type=float, default=20.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--world-sim", type=int, default=0,
+                    help="one GPU plays each of N ranks in turn (plan for N GPUs, per-rank epoch times)")
+    ap.add_argument("--rank-balanced-k", action="store_true",
+                    help="reading R31: only K that are multiples of the GPU count (rank-aware grouping)")
     ap.add_argument("--no-pipeline", action="store_true",
                     help="schedule each epoch synchronously (default: the next epoch's plan is computed on a "
                          "side stream while the current epoch trains)")
@@ -351,6 +355,49 @@ def measured_memory(tr, epoch):
                     "sample caches, plans, weights) are outside M_ctr"}
 
 
+# ----------------------------------------------------------------------------- world-sim
+def run_world_sim(args, tr, sim, flush, stream):
+    """--world-sim N on one GPU: the plan is made for N GPUs (k_min = N, LPT rank assignment,
+    optionally rank-aware K), and this one process plays each rank r in turn — its replicated
+    scheduler (the pipelined side stream, full Alg. 3 every epoch) plus its own groups — timing
+    `steps` epochs per rank with CUDA events.  The N-GPU epoch is then bounded by the slowest
+    rank (the NCCL allreduce of the 0.6-2.7 MB gradient, tens of microseconds over NVLink, is not
+    simulated).  Prints one JSON line with "mode": "world_sim" (not the driver's bench line)."""
+    import torch
+    per = []
+    for r in range(sim):
+        tr.rank = r
+        tr.sched.rank = r                       # group sizes are measured for the own groups only
+        tr._ahead = None
+        for i in range(args.warmup):
+            tr.run_epoch(epoch=i, lr=0.01)
+        torch.cuda.synchronize()
+        ms, edges, groups, K = [], 0, 0, 0
+        for i in range(args.steps):
+            flush.zero_()
+            s0 = torch.cuda.Event(enable_timing=True)
+            s1 = torch.cuda.Event(enable_timing=True)
+            s0.record(stream)
+            st = tr.run_epoch(epoch=args.warmup + i, lr=0.01)
+            s1.record(stream)
+            s1.synchronize()
+            ms.append(s0.elapsed_time(s1))
+            edges += st["edges"]
+            groups = len(st["groups"])
+            K = st["K"]
+        per.append({"rank": r, "ms_per_step": sum(ms) / len(ms), "groups": groups,
+                    "edges_per_epoch": edges / args.steps})
+    worst = max(p["ms_per_step"] for p in per)
+    total_edges = sum(p["edges_per_epoch"] for p in per)
+    line = {"mode": "world_sim", "world_sim": sim, "config": args.config, "K": K,
+            "rank_balanced_k": bool(args.rank_balanced_k), "per_rank": per,
+            "projected_epoch_ms": worst, "projected_edges_per_s": total_edges / (worst / 1e3),
+            "rank_spread_max_over_min": worst / min(p["ms_per_step"] for p in per),
+            "note": "one B200 plays each rank in turn (replicated scheduler + own groups); NCCL allreduce "
+                    "not included; the projected N-GPU epoch is the slowest rank"}
+    print(json.dumps(line), flush=True)
+
+
 # ----------------------------------------------------------------------------- our arm
 def run_ours(args, cfg):
     import torch
@@ -413,7 +460,10 @@ def run_ours(args, cfg):
     feats = X
     if not sharded and feat_dtype == B.BF16 and feats.dtype != torch.bfloat16:
         feats = feats.to(torch.bfloat16).contiguous()      # k/128 features are exact in bf16
-    kmin = max(cfg.k_min, world)
+    sim = args.world_sim if world == 1 and args.world_sim > 1 else 0
+    plan_world = sim or world                     # #GPUs the plan is made for (R24 k_min, LPT ranks)
+    kmin = max(cfg.k_min, plan_world)
+    kmult = plan_world if args.rank_balanced_k else 1
     budget = cfg.mem_budget
     graph = DeviceGraph(rp, col)
     # C of Eq. 1 ("offline graph analysis"): exact, on the GPU, once per graph,
@@ -423,8 +473,8 @@ def run_ours(args, cfg):
     t_c = time.perf_counter() - t_c
     tr = Trainer(graph, feats, y, seeds, cfg.dims,
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, mem_budget=budget,
-                 C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=world, process_group=pg,
-                 pipeline=not args.no_pipeline, **agg_kw)
+                 C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=plan_world, process_group=pg,
+                 pipeline=not args.no_pipeline, k_multiple=kmult, **agg_kw)
     full_batch_edges = None
     if args.config in ("products", "papers", "arxiv_lstm") + SHARDED:
         # calibrate M_ctr once so that one GPU needs >= 8 groups (products; 2 for the LSTM
@@ -439,6 +489,8 @@ def run_ours(args, cfg):
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
 
+    if sim:
+        return run_world_sim(args, tr, sim, flush, stream)
     prof_counters = torch.zeros(1 << 16, dtype=torch.int64, device="cuda")
     lr = 0.01
     for i in range(args.warmup):

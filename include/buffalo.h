@@ -119,11 +119,28 @@ typedef struct {
 
 /* Scheduler parameters (Alg. 3): mem_budget = M_ctr in bytes (arena bytes
  * of one micro-batch, R15); C_ppm = average clustering coefficient x 10^6 (Eq. 1, <= 0: R = 1);
- * K searched in [max(k_min, num_gpus), k_max]. */
+ * K searched in [max(k_min, num_gpus), k_max]; k_multiple > 1 (reading R31, rank-aware grouping
+ * for data-parallel runs): only multiples of k_multiple are tried, so with k_multiple = num_gpus
+ * the K groups can spread evenly over the ranks (the LPT rank assignment still decides; 0 or 1:
+ * every K, the paper's loop). */
+typedef int32_t (*buffalo_allgather_fn)(void* ctx, const void* send_h, void* recv_h, int64_t bytes);
 typedef struct {
   int64_t mem_budget;
   int64_t C_ppm;
   int32_t k_min, k_max, num_gpus;
+  int32_t k_multiple;
+  /* Data-parallel scheduling: every rank calls buffalo_bucketize with the same
+   * inputs and derives the same plan.  rank (0..num_gpus-1) = the caller's rank: the exact block
+   * sizes (plan.group_sizes_h) are measured for its own groups only (other rows: -1).
+   * allgather (nullable): host all-gather over the ranks — recv_h[r * bytes ...] receives rank
+   * r's send_h, returns 0 on success; given, every statistics pass (the degree buckets, the K
+   * loop's micro-bucket candidates) is shared out — each rank measures every num_gpus-th item —
+   * and the int64 size rows exchanged, so the replicated scheduler work shrinks; the sampler's
+   * cache is then not used (no rank visits the whole receptive field); every rank must call
+   * bucketize in the same order.  NULL: every rank measures every item. */
+  int32_t rank;
+  buffalo_allgather_fn allgather;
+  void* allgather_ctx;
 } buffalo_sched;
 
 /* Output of buffalo_bucketize.  Device arrays sized by the caller: group_of_seed[n_seeds],

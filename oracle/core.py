@@ -402,7 +402,7 @@ def mem_balanced_grouping(items, K, M_ctr):
     return max(loads) <= M_ctr, groups, loads
 
 
-def _alg3_k_loop(stats, F, piece_stats, mem_budget, C_ppm, k_lo, k_max, fast_paths=True):
+def _alg3_k_loop(stats, F, piece_stats, mem_budget, C_ppm, k_lo, k_max, fast_paths=True, k_multiple=1):
     """The K loop of Alg. 3 with MemBalancedGrouping (Alg. 4) over the
     per-bucket statistics `stats` {d: dict(M, I, E, O, w, ...)} (non-empty buckets only).
     piece_stats(K) -> [(k, st), ...]: statistics of the K micro-buckets of bucket F (R8).
@@ -412,13 +412,16 @@ def _alg3_k_loop(stats, F, piece_stats, mem_budget, C_ppm, k_lo, k_max, fast_pat
     fast_paths (R25) skips a K without building micro-buckets when sum_{d != F} w_d > K*M_ctr
     and stops at once when a never-split bucket alone exceeds M_ctr; both imply that the plain
     loop (fast_paths=False) fails at that K too, so the result is identical (pinned by
-    tests/test_oracle_scheduler.py on random instances).
+    tests/test_oracle_scheduler.py on random instances).  k_multiple > 1 (reading R31,
+    rank-balanced grouping): only multiples of k_multiple are candidates.
     Returns (K, items, groups, loads, exploded) or None."""
     non_split = [d for d in stats if d != F]
     sum_M_all = sum(stats[d]["M"] for d in stats)
     max_w = max([stats[d]["w"] for d in non_split], default=0)
     sum_w = sum(stats[d]["w"] for d in non_split)
     for K in range(k_lo, k_max + 1):
+        if k_multiple > 1 and K % k_multiple:
+            continue
         if fast_paths:
             if max_w > mem_budget:
                 return None                  # a never-split bucket exceeds M_ctr for every K
@@ -440,7 +443,8 @@ def _alg3_k_loop(stats, F, piece_stats, mem_budget, C_ppm, k_lo, k_max, fast_pat
 
 
 def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT64_MAX,
-             C_ppm=0, k_min=1, k_max=4096, num_gpus=1, aggregator="mean", fast_paths=True, sharded=False):
+             C_ppm=0, k_min=1, k_max=4096, num_gpus=1, aggregator="mean", fast_paths=True, sharded=False,
+             k_multiple=1):
     """Alg. 3 Buffalo_Scheduler with the readings of DESIGN.md
     (R7 explosion test, R11 sort/placement keys, R16 K_max, R17 empty groups dropped,
     R24 k_min = #GPUs and LPT rank assignment, R25 fast paths).  Returns a dict plan or None
@@ -461,7 +465,8 @@ def schedule(g, seeds, L, fanout, F, seed, dims, act_dtype=FP32, mem_budget=INT6
     def piece_stats(K):
         return [(k, stats_of(piece)) for k, piece in enumerate(split_explosion(pos_of[F], K)) if piece.size]
 
-    res = _alg3_k_loop(stats, F, piece_stats, mem_budget, C_ppm, max(k_min, num_gpus, 1), k_max, fast_paths)
+    res = _alg3_k_loop(stats, F, piece_stats, mem_budget, C_ppm, max(k_min, num_gpus, 1), k_max, fast_paths,
+                       k_multiple)
     if res is None:
         return None
     K, items, groups, loads, exploded = res

@@ -70,9 +70,13 @@ class Model(ctypes.Structure):
                 ("feat_shards", ctypes.POINTER(FeatureShards))]
 
 
+ALLGATHER_FN = ctypes.CFUNCTYPE(c_i32, c_p, c_p, c_p, c_i64)
+
+
 class Sched(ctypes.Structure):
     _fields_ = [("mem_budget", c_i64), ("C_ppm", c_i64), ("k_min", c_i32), ("k_max", c_i32),
-                ("num_gpus", c_i32)]
+                ("num_gpus", c_i32), ("k_multiple", c_i32), ("rank", c_i32), ("allgather", ALLGATHER_FN),
+                ("allgather_ctx", c_p)]
 
 
 class Plan(ctypes.Structure):
@@ -446,10 +450,36 @@ def make_model(dims, feat_dtype=FP32, gemm_mode=GEMM_FFMA, feat_pitch=None, aggr
     return m
 
 
-def make_sched(mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096, num_gpus=1):
+def make_sched(mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096, num_gpus=1, k_multiple=1, rank=0,
+               allgather=None):
+    """allgather: None or an ALLGATHER_FN (kept alive by the returned struct)."""
     s = Sched()
     s.mem_budget, s.C_ppm, s.k_min, s.k_max, s.num_gpus = int(mem_budget), int(C_ppm), k_min, k_max, num_gpus
+    s.k_multiple = int(k_multiple)
+    s.rank = int(rank)
+    if allgather is not None:
+        s.allgather = allgather
+        s._allgather_ref = allgather
     return s
+
+
+def make_allgather(world, group=None, device=None):
+    """An ALLGATHER_FN over torch.distributed (host buffers; NCCL groups go through `device`)."""
+    import torch.distributed as dist
+
+    def fn(ctx, send, recv, nbytes):
+        try:
+            src = torch.frombuffer((ctypes.c_char * nbytes).from_address(send), dtype=torch.uint8).clone()
+            if device is not None:
+                src = src.to(device)
+            out = torch.empty(world * nbytes, dtype=torch.uint8, device=src.device)
+            dist.all_gather_into_tensor(out, src, group=group)
+            out = out.cpu().contiguous()
+            ctypes.memmove(recv, out.data_ptr(), world * nbytes)
+            return 0
+        except Exception:                    # noqa: BLE001 (reported to the library as a failure)
+            return 1
+    return ALLGATHER_FN(fn)
 
 
 def pitch(d):

@@ -223,10 +223,12 @@ constexpr int kStatsBatch = 256;       // items per statistics pass (mask_stats)
 // O = #seeds, E = e_L, I = n_{L-1} and M_est = hi of the memory model.
 // cache_mode (the sampler's sample cache, when it has one): 1 = sample and store, 2 = read the
 // rows stored by an earlier pass of the same call.
-static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_ids, std::vector<Item*>& items,
-                                  const buffalo_sampler* sp, const buffalo_model* m, char* ws, int64_t ws_bytes,
-                                  bool& masks_clean, cudaStream_t s, int cache_mode) {
-  const int L = m->num_layers;
+// sizes: one row [2L+1] per item: n_0..n_L, e_1..e_L.
+static buffalo_status items_sizes(const buffalo_graph* g, const int32_t* sorted_ids, const std::vector<Item*>& items,
+                                  const buffalo_sampler* sp, int L, char* ws, int64_t ws_bytes, bool& masks_clean,
+                                  cudaStream_t s, int cache_mode, std::vector<int64_t>& sizes) {
+  const int W = 2 * L + 1;
+  sizes.assign(items.size() * W, 0);
   for (size_t b0 = 0; b0 < items.size(); b0 += kStatsBatch) {
     const int nit = (int)std::min<size_t>(kStatsBatch, items.size() - b0);
     int64_t starts[kStatsBatch], counts[kStatsBatch];
@@ -238,14 +240,61 @@ static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_
     BF_CHECK(mask_stats(g, sorted_ids, starts, counts, nit, sp, L, ws, ws_bytes, masks_clean, nh, eh, s, cache_mode));
     masks_clean = true;
     for (int k = 0; k < nit; ++k) {
-      Item& it = *items[b0 + k];
-      int64_t lo, hi;
-      mem_model(L, nh[k], eh[k], m, &lo, &hi);
-      it.O = it.count;
-      it.E = eh[k][L - 1];
-      it.I = nh[k][L - 1];
-      it.M = hi;
+      int64_t* row = sizes.data() + (b0 + k) * W;
+      for (int l = 0; l <= L; ++l) row[l] = nh[k][l];
+      for (int l = 1; l <= L; ++l) row[L + l] = eh[k][l - 1];
     }
+  }
+  return BUFFALO_OK;
+}
+
+static void derive_item(Item& it, const int64_t* row, int L, const buffalo_model* m) {
+  int64_t lo, hi;
+  mem_model(L, row, row + L + 1, m, &lo, &hi);
+  it.O = it.count;
+  it.E = row[L + L];          // e_L
+  it.I = row[L - 1];          // n_{L-1}
+  it.M = hi;
+}
+
+static buffalo_status items_stats(const buffalo_graph* g, const int32_t* sorted_ids, std::vector<Item*>& items,
+                                  const buffalo_sampler* sp, const buffalo_model* m, char* ws, int64_t ws_bytes,
+                                  bool& masks_clean, cudaStream_t s, int cache_mode) {
+  const int L = m->num_layers;
+  std::vector<int64_t> sizes;
+  BF_CHECK(items_sizes(g, sorted_ids, items, sp, L, ws, ws_bytes, masks_clean, s, cache_mode, sizes));
+  for (size_t k = 0; k < items.size(); ++k) derive_item(*items[k], sizes.data() + k * (2 * L + 1), L, m);
+  return BUFFALO_OK;
+}
+
+// The same statistics with the items shared out over the ranks (sched.allgather given, more
+// than one GPU): rank r measures the items k = r, r + G, r + 2G, ... and one all-gather of their
+// int64 size rows gives every rank the whole table (identical on every rank: the plan stays
+// deterministic without a broadcast).  Used for every statistics pass of Alg. 3 (the degree
+// buckets and the K loop's micro-bucket candidates); the group-size pass measures own groups.
+static buffalo_status items_stats_shared(const buffalo_graph* g, const int32_t* sorted_ids, std::vector<Item*>& items,
+                                         const buffalo_sampler* sp, const buffalo_model* m, const buffalo_sched* sc,
+                                         char* ws, int64_t ws_bytes, bool& masks_clean, cudaStream_t s,
+                                         int cache_mode) {
+  const int G = sc->num_gpus;
+  if (!sc->allgather || G <= 1)
+    return items_stats(g, sorted_ids, items, sp, m, ws, ws_bytes, masks_clean, s, cache_mode);
+  const int L = m->num_layers, W = 2 * L + 1;
+  std::vector<Item*> mine;
+  for (size_t k = sc->rank; k < items.size(); k += G) mine.push_back(items[k]);
+  std::vector<int64_t> sizes;
+  BF_CHECK(items_sizes(g, sorted_ids, mine, sp, L, ws, ws_bytes, masks_clean, s, cache_mode, sizes));
+  const int64_t per = (int64_t)((items.size() + G - 1) / G);          // rows per rank (padded)
+  std::vector<int64_t> send(per * W, -1), recv((size_t)G * per * W, -1);
+  std::copy(sizes.begin(), sizes.end(), send.begin());
+  if (sc->allgather(sc->allgather_ctx, send.data(), recv.data(), per * W * (int64_t)sizeof(int64_t)) != 0) {
+    set_error("bucketize: the all-gather of the item statistics failed");
+    return BUFFALO_ERR_CUDA;
+  }
+  for (size_t k = 0; k < items.size(); ++k) {
+    const int r = (int)(k % G);
+    const int64_t j = (int64_t)(k / G);
+    derive_item(*items[k], recv.data() + ((int64_t)r * per + j) * W, L, m);
   }
   return BUFFALO_OK;
 }
@@ -469,7 +518,8 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
     set_error("bucketize: null argument or empty seed set");
     return BUFFALO_ERR_INVALID_ARG;
   }
-  if (sc->mem_budget <= 0 || sc->k_max < 1 || sc->k_max > 4096 || sc->num_gpus < 1) {
+  if (sc->mem_budget <= 0 || sc->k_max < 1 || sc->k_max > 4096 || sc->num_gpus < 1 || sc->k_multiple < 0 ||
+      sc->rank < 0 || sc->rank >= sc->num_gpus) {
     set_error("bucketize: bad scheduler parameters");
     return BUFFALO_ERR_INVALID_ARG;
   }
@@ -494,6 +544,13 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
   char* stats_ws = q;
   const int64_t stats_bytes = (int64_t)workspace_bytes - used;
 
+  // shared statistics (include/buffalo.h buffalo_sched.allgather): no rank visits the whole
+  // receptive field, so the per-rank sample cache cannot be filled; every pass samples
+  const bool shared = sc->allgather && sc->num_gpus > 1;
+  buffalo_sampler sp_local = *sp;
+  if (shared)
+    for (auto& c : sp_local.cache) c = nullptr;
+  sp = &sp_local;
   // a1: DegreeBucketing (Alg. 3 l.1); validates the seed ids (in range, distinct).  The plan's
   // outputs are written only once a K succeeded (outputs untouched on error).
   std::vector<int64_t> hist(F + 1, 0);
@@ -510,7 +567,7 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
     if (hist[d] > 0) todo.push_back(&bucket_item[d]);
   }
   // the first statistics pass (every seed) fills the sample cache; later passes read it
-  BF_CHECK(items_stats(g, sorted_ids, todo, sp, m, stats_ws, stats_bytes, masks_clean, s, 1));
+  BF_CHECK(items_stats_shared(g, sorted_ids, todo, sp, m, sc, stats_ws, stats_bytes, masks_clean, s, 1));
   std::vector<int> non_split;
   int64_t sum_M_all = 0, sum_w = 0, max_w = 0;
   for (int d = 0; d <= F; ++d) {
@@ -530,7 +587,10 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
   // of several consecutive K candidates are computed in one statistics pass (their pieces
   // overlap, each seed carries one bit per candidate); the loop itself stays sequential.
   const int k_lo = std::max(std::max(sc->k_min, sc->num_gpus), 1);
+  // R31: with k_multiple > 1 only multiples of it are candidates (every rank gets K / #GPUs groups)
+  auto candidate = [&](int K) { return sc->k_multiple <= 1 || K % sc->k_multiple == 0; };
   auto needs_split = [&](int K) {
+    if (!candidate(K)) return false;
     if (max_w > sc->mem_budget) return false;
     if ((__int128)sum_w > (__int128)K * sc->mem_budget) return false;
     return hasF && K >= 2 && (__int128)bucket_item[F].M * K > (__int128)sum_M_all;
@@ -538,6 +598,7 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
   std::vector<std::vector<Item>> piece_cache(sc->k_max + 1);
   std::vector<char> have(sc->k_max + 1, 0);
   for (int K = k_lo; K <= sc->k_max; ++K) {
+    if (!candidate(K)) continue;
     if (max_w > sc->mem_budget) break;                         // R25: fails for every K
     if ((__int128)sum_w > (__int128)K * sc->mem_budget) continue;  // R25: some group exceeds M_ctr
     std::vector<Item> items;
@@ -565,7 +626,7 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
           }
           for (int K2 : ks)
             for (Item& it : piece_cache[K2]) ptrs.push_back(&it);
-          BF_CHECK(items_stats(g, sorted_ids, ptrs, sp, m, stats_ws, stats_bytes, masks_clean, s, 2));
+          BF_CHECK(items_stats_shared(g, sorted_ids, ptrs, sp, m, sc, stats_ws, stats_bytes, masks_clean, s, 2));
         }
         for (Item it : piece_cache[K]) {
           it.w = grouping_weight(it.M, it.I, it.E, sc->C_ppm);
@@ -641,26 +702,27 @@ buffalo_status buffalo_bucketize(const buffalo_graph* g, const int32_t* seeds, i
     }
     for (int k = 0; k < gk; ++k) plan->est_bytes_h[k] = est[k];
     if (plan->group_sizes_h) {
-      // exact block sizes of every group (groups as items of the mask statistics), so that
-      // buffalo_build_blocks can lay out the arena up front and run without host round trips
+      // exact block sizes of this rank's groups (groups as items of the mask statistics), so
+      // that buffalo_build_blocks can lay out the arena up front and run without host round
+      // trips; the rows of other ranks' groups are set to -1 (each rank measures its own)
       const int W = 2 * L + 1;
-      for (int k0 = 0; k0 < gk; k0 += kStatsBatch) {
-        const int nit = std::min(kStatsBatch, gk - k0);
-        int64_t st[kStatsBatch], ct[kStatsBatch];
-        for (int k = 0; k < nit; ++k) {
-          st[k] = offs[k0 + k];
-          ct[k] = offs[k0 + k + 1] - offs[k0 + k];
+      std::vector<Item> gitems;
+      std::vector<int> gidx;
+      for (int k = 0; k < gk; ++k) {
+        int64_t* row = plan->group_sizes_h + (int64_t)k * W;
+        if (sc->num_gpus > 1 && plan->rank_of_group_h[k] != sc->rank) {
+          for (int c = 0; c < W; ++c) row[c] = -1;
+          continue;
         }
-        static thread_local int64_t nh[kStatsBatch][BUFFALO_MAX_LAYERS + 1], eh[kStatsBatch][BUFFALO_MAX_LAYERS];
-        BF_CHECK(mask_stats(g, plan->group_seeds, st, ct, nit, sp, L, stats_ws, stats_bytes, masks_clean, nh, eh, s,
-                            2));
-        masks_clean = true;
-        for (int k = 0; k < nit; ++k) {
-          int64_t* row = plan->group_sizes_h + (int64_t)(k0 + k) * W;
-          for (int l = 0; l <= L; ++l) row[l] = nh[k][l];
-          for (int l = 1; l <= L; ++l) row[L + l] = eh[k][l - 1];
-        }
+        gitems.push_back(Item{0, k, offs[k], offs[k + 1] - offs[k], 0, 0, 0, 0, 0});
+        gidx.push_back(k);
       }
+      std::vector<Item*> gp;
+      for (Item& it : gitems) gp.push_back(&it);
+      std::vector<int64_t> sizes;
+      BF_CHECK(items_sizes(g, plan->group_seeds, gp, sp, L, stats_ws, stats_bytes, masks_clean, s, 2, sizes));
+      for (size_t j = 0; j < gidx.size(); ++j)
+        std::copy(sizes.begin() + j * W, sizes.begin() + (j + 1) * W, plan->group_sizes_h + (int64_t)gidx[j] * W);
     }
     for (int d = 0; d <= F; ++d) plan->hist_h[d] = hist[d];
     plan->k_out = gk;

@@ -19,8 +19,10 @@ def own_groups(rank_of_group, rank):
 
 
 def allreduce_grads(grad, world, group=None):
-    """The one data-path collective: sum of the flat gradient buffer over the ranks."""
-    if world > 1:
+    """The one data-path collective: sum of the flat gradient buffer over the ranks.  Without an
+    initialised process group (bench.py --world-sim: one process plays each rank in turn) there
+    is nothing to reduce with."""
+    if world > 1 and torch.distributed.is_available() and torch.distributed.is_initialized():
         torch.distributed.all_reduce(grad, group=group)
 
 
@@ -191,7 +193,8 @@ class Trainer:
     def __init__(self, graph, feats, labels, seeds, dims, fanout, F, Ws, bs, feat_dtype=B.FP32,
                  gemm_mode=B.GEMM_FFMA, mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096,
                  base_seed=3, rank=0, world=1, process_group=None, device="cuda", aggregator=B.AGG_MEAN,
-                 Wps=None, bps=None, lstm=None, gat=None, pipeline=False, sample_cache=True):
+                 Wps=None, bps=None, lstm=None, gat=None, pipeline=False, sample_cache=True, k_multiple=1,
+                 share_stats=True):
         self.graph = graph if isinstance(graph, DeviceGraph) else DeviceGraph(*graph, device=device)
         self.feats = feats
         self.labels = labels
@@ -217,7 +220,13 @@ class Trainer:
         self.sharded = isinstance(feats, ShardedFeatures)
         self.model = B.make_model(dims, feat_dtype, gemm_mode, feats.shape[1], aggregator,
                                   shards=feats.struct if self.sharded else None)
-        self.sched = B.make_sched(mem_budget, C_ppm, k_min, k_max, world)
+        # with a process group, the K loop's micro-bucket statistics are shared out over the ranks
+        # (buffalo_sched.allgather); every rank still derives the identical plan
+        ag = None
+        if share_stats and world > 1 and torch.distributed.is_available() and torch.distributed.is_initialized():
+            nccl = torch.distributed.get_backend(process_group) == "nccl"
+            ag = B.make_allgather(world, process_group, torch.device(device) if nccl else None)
+        self.sched = B.make_sched(mem_budget, C_ppm, k_min, k_max, world, k_multiple, rank, ag)
         self.params = SageParams(self.model, Ws, bs, device, Wps, bps, lstm, gat)
         self.rank, self.world, self.pg = rank, world, process_group
         self.device = device
@@ -236,6 +245,8 @@ class Trainer:
         # sample cache per plan-buffer set (include/buffalo.h): the scheduler's first statistics
         # pass stores every sampled neighbour list of the batch, the build copies them
         N = self.graph.N
+        if self.sched.allgather:
+            sample_cache = False             # shared statistics: the scheduler fills no cache
         self._cache = [[torch.empty(N * f, dtype=torch.int32, device=device) if (sample_cache and f > 0) else None
                         for f in self.fanout] for _ in self._pb]
         self._cache_epoch = [None] * len(self._pb)

@@ -74,3 +74,33 @@ def test_two_rank_allreduce_equals_full_batch():
     sets = [set(own_groups(plan["rank_of_group"], r)) for r in range(world)]
     assert sets[0].isdisjoint(sets[1]) and sets[0] | sets[1] == set(range(plan["K"]))
     assert plan["K"] >= world
+
+
+def _ag_worker(rank, world, port, out):
+    """The scheduler's all-gather callback (buffalo_sched.allgather) over gloo: called through
+    its C function pointer exactly as the library calls it."""
+    import ctypes
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_hpca_yangzl25_b200 import buffalo as B
+    fn = B.make_allgather(world)
+    W = 7
+    send = (ctypes.c_int64 * (3 * W))(*[rank * 1000 + i for i in range(3 * W)])
+    recv = (ctypes.c_int64 * (world * 3 * W))()
+    cfn = ctypes.cast(fn, ctypes.c_void_p).value
+    call = B.ALLGATHER_FN(cfn)
+    rc = call(None, ctypes.addressof(send), ctypes.addressof(recv), 3 * W * 8)
+    out[rank] = (rc, list(recv))
+    dist.destroy_process_group()
+
+
+def test_scheduler_allgather_callback_two_ranks():
+    world = 2
+    mgr = mp.Manager()
+    out = mgr.list([None] * world)
+    mp.spawn(_ag_worker, args=(world, _free_port(), out), nprocs=world, join=True)
+    want = [r * 1000 + i for r in range(world) for i in range(21)]
+    for r in range(world):
+        rc, got = out[r]
+        assert rc == 0 and got == want
+

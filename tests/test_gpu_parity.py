@@ -115,7 +115,7 @@ def test_blocks_sync_free_identical(name):
 
 
 @pytest.mark.parametrize("name", ["sampled2", "full3", "mixed3"])
-@pytest.mark.parametrize("variant", ["k4", "budget", "C", "gpus3"])
+@pytest.mark.parametrize("variant", ["k4", "budget", "C", "gpus3", "gpus3_kmult"])
 def test_bucketize_plan_bit_exact(name, variant):
     rp, col, X, y, seeds, fan, F, dims, Ws, bs = _case(name)
     g = O.Graph(rp, col)
@@ -128,11 +128,16 @@ def test_bucketize_plan_bit_exact(name, variant):
     elif variant == "C":
         full = O.schedule(g, seeds, len(fan), fan, F, 3, dims, k_min=1, k_max=1)
         kw.update(mem_budget=int(full["est_bytes"][0] * 0.3), C_ppm=226000)
-    else:
+    elif variant == "gpus3":
         kw.update(num_gpus=3)
+    else:                                       # R31: rank-aware K (multiples of #GPUs) under a budget
+        full = O.schedule(g, seeds, len(fan), fan, F, 3, dims, k_min=1, k_max=1)
+        kw.update(num_gpus=3, k_multiple=3, mem_budget=int(full["est_bytes"][0] * 0.2))
     ref = O.schedule(g, seeds, len(fan), fan, F, 3, dims, **kw)
     tr = make_trainer(rp, col, X, y, seeds, dims, fan, F, Ws, bs, base_seed=3,
                       **{k: v for k, v in kw.items() if k != "num_gpus"}, world=kw["num_gpus"])
+    if variant == "gpus3_kmult":
+        assert ref["K_tried"] % 3 == 0
     K, offs, est, ranks = tr.schedule(0)
     assert K == ref["K"] and tr.plan.k_tried == ref["K_tried"]
     assert bool(tr.plan.exploded) == ref["exploded"] and tr.plan.num_items == ref["num_items"]
@@ -142,10 +147,14 @@ def test_bucketize_plan_bit_exact(name, variant):
     np.testing.assert_array_equal(tr.group_seeds.cpu().numpy(), ref["group_seeds"])
     np.testing.assert_array_equal(tr.group_of_seed.cpu().numpy(), ref["group_of_seed"])
     np.testing.assert_array_equal(tr.hist_h, ref["hist"])
-    # exact block sizes of every group (plan.group_sizes_h) = the oracle's blocks of that group
+    # exact block sizes of this rank's groups (plan.group_sizes_h) = the oracle's blocks of that
+    # group; the rows of other ranks' groups are -1 (each rank measures its own)
     L = len(fan)
     gs = ref["group_seeds"]
     for k in range(K):
+        if kw["num_gpus"] > 1 and ranks[k] != 0:
+            assert np.all(tr.sizes_h[k] == -1)
+            continue
         blocks = O.build_blocks(g, gs[offs[k]:offs[k + 1]], L, fan, 3)
         want = [blocks[0]["n_src"]] + [b["n_dst"] for b in blocks] + [b["n_edges"] for b in blocks]
         np.testing.assert_array_equal(tr.sizes_h[k], want, err_msg=f"group {k}")

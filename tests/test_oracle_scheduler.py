@@ -262,3 +262,31 @@ def test_fast_paths_equal_plain_loop_random():
             np.testing.assert_array_equal(a[k], b[k], err_msg=f"instance {it} {k}")
     # the instances exercise every branch
     assert n_exploded >= 10 and n_none >= 10 and n_skipped >= 10, (n_exploded, n_none, n_skipped)
+
+
+def test_k_multiple_restricts_the_loop_to_multiples():
+    """R31: with k_multiple = m the loop tries only multiples of m; the result is the first
+    multiple at which the plain Alg. 3 step (run alone at that K) succeeds."""
+    rng = np.random.default_rng(31)
+    rp, col = random_graph(300, 2400, "powerlaw")
+    g = O.Graph(rp, col)
+    seen = 0
+    for it in range(40):
+        seeds = np.sort(rng.choice(g.N, int(rng.integers(40, 250)), replace=False)).astype(np.int32)
+        fan, F, dims = [3, 5], 5, [16, 24, 5]
+        full = O.schedule(g, seeds, 2, fan, F, 3, dims, k_min=1, k_max=1)
+        budget = int(full["est_bytes"][0] * rng.uniform(0.08, 0.6))
+        m = int(rng.choice([2, 3, 4]))
+        a = O.schedule(g, seeds, 2, fan, F, 3, dims, mem_budget=budget, k_max=24, num_gpus=m, k_multiple=m)
+        want = None
+        for K in range(m, 25, m):
+            if O.schedule(g, seeds, 2, fan, F, 3, dims, mem_budget=budget, k_min=K, k_max=K, num_gpus=m,
+                          fast_paths=False) is not None:
+                want = K
+                break
+        assert (a is None) == (want is None), it
+        if a is not None:
+            seen += 1
+            assert a["K_tried"] == want and a["K_tried"] % m == 0
+            assert sorted(a["group_seeds"].tolist()) == sorted(seeds.tolist())
+    assert seen >= 20
