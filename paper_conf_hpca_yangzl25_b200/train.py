@@ -123,59 +123,54 @@ def exchange_shards(local, rank, world, rows_per_shard, num_rows, group=None):
 
 
 class SageParams:
-    """fp32 master weights/biases (Xavier init from synth), flat gradient buffer, packed copies."""
+    """fp32 master weights/biases (Xavier init from synth), flat gradient buffer, packed copies.
+    The flat buffers are layer-major: layer l's W, b and aggregator weights (pool W_pool, b_pool;
+    LSTM W_ih, W_hh, b; GAT a_l, a_r) form one contiguous slice (layer_slice[l - 1]), so a
+    layer's gradient can be all-reduced as soon as its last backward has run."""
 
     def __init__(self, model, Ws, bs, device="cuda", Wps=None, bps=None, lstm=None, gat=None):
         self.model = model
-        self.L = model.num_layers
+        self.L = L = model.num_layers
         Wps, bps = list(Wps or []), list(bps or [])
         Wih, Whh, bl = [list(x) for x in lstm] if lstm else ([], [], [])
         als, ars = [list(x) for x in gat] if gat else ([], [])
-        extra = Wih + Whh + bl + als + ars
-        sizes = [w.size for w in Ws] + [b.size for b in bs] + [w.size for w in Wps] + [b.size for b in bps] + \
-            [w.size for w in extra]
-        self.flat = torch.zeros(sum(sizes), dtype=torch.float32, device=device)
+        per_layer = []
+        for l in range(L):
+            items = [("W", Ws[l]), ("b", bs[l])]                  # (name, array) in slice order
+            if Wps:
+                items += [("Wp", Wps[l]), ("bp", bps[l])]
+            if Wih:
+                items += [("Wih", Wih[l]), ("Whh", Whh[l]), ("bl", bl[l])]
+            if als:
+                items += [("al", als[l]), ("ar", ars[l])]
+            per_layer.append(items)
+        total = sum(int(np.asarray(a).size) for items in per_layer for _, a in items)
+        self.flat = torch.zeros(total, dtype=torch.float32, device=device)
         self.grad = torch.zeros_like(self.flat)
-        self.W, self.b, self.dW, self.db = [], [], [], []
+        views = {k: ([], []) for k in ("W", "b", "Wp", "bp", "Wih", "Whh", "bl", "al", "ar")}
+        self.layer_slice = []
         off = 0
-        for w in Ws:
-            self.W.append(self.flat[off:off + w.size].view(w.shape))
-            self.dW.append(self.grad[off:off + w.size].view(w.shape))
-            self.W[-1].copy_(torch.as_tensor(w))
-            off += w.size
-        for b in bs:
-            self.b.append(self.flat[off:off + b.size])
-            self.db.append(self.grad[off:off + b.size])
-            self.b[-1].copy_(torch.as_tensor(b))
-            off += b.size
+        for items in per_layer:
+            start = off
+            for name, a in items:
+                a = np.asarray(a)
+                p = self.flat[off:off + a.size].view(a.shape)
+                p.copy_(torch.as_tensor(a))
+                views[name][0].append(p)
+                views[name][1].append(self.grad[off:off + a.size].view(a.shape))
+                off += a.size
+            self.layer_slice.append((start, off))
+        self.W, self.dW = views["W"]
+        self.b, self.db = views["b"]
         # GraphSAGE-pool weights (R28), in the same flat buffers (one allreduce, one SGD step)
-        self.Wp, self.bp, self.dWp, self.dbp = [], [], [], []
-        for w in Wps:
-            self.Wp.append(self.flat[off:off + w.size].view(w.shape))
-            self.dWp.append(self.grad[off:off + w.size].view(w.shape))
-            self.Wp[-1].copy_(torch.as_tensor(w))
-            off += w.size
-        for b in bps:
-            self.bp.append(self.flat[off:off + b.size])
-            self.dbp.append(self.grad[off:off + b.size])
-            self.bp[-1].copy_(torch.as_tensor(b))
-            off += b.size
+        self.Wp, self.dWp = views["Wp"]
+        self.bp, self.dbp = views["bp"]
         # GraphSAGE-LSTM weights (R29): W_ih, W_hh [4d, d], b [4d] per layer
-        self.lstm, self.dlstm = [[], [], []], [[], [], []]
-        for k, group in enumerate((Wih, Whh, bl)):
-            for w in group:
-                self.lstm[k].append(self.flat[off:off + w.size].view(w.shape))
-                self.dlstm[k].append(self.grad[off:off + w.size].view(w.shape))
-                self.lstm[k][-1].copy_(torch.as_tensor(w))
-                off += w.size
+        self.lstm = [views["Wih"][0], views["Whh"][0], views["bl"][0]]
+        self.dlstm = [views["Wih"][1], views["Whh"][1], views["bl"][1]]
         # GAT attention vectors (R30): a_l, a_r [d_l] per layer
-        self.al, self.ar, self.dal, self.dar = [], [], [], []
-        for dst, gdst, group in ((self.al, self.dal, als), (self.ar, self.dar, ars)):
-            for w in group:
-                dst.append(self.flat[off:off + w.size])
-                gdst.append(self.grad[off:off + w.size])
-                dst[-1].copy_(torch.as_tensor(w))
-                off += w.size
+        self.al, self.dal = views["al"]
+        self.ar, self.dar = views["ar"]
         self.is_gat = model.aggregator == B.AGG_GAT      # GAT's W_l is [d_l, d_{l-1}]: no packed Update copy
         self.packed = [None if self.is_gat else
                        torch.empty(B.packed_weight_bytes(model, l), dtype=torch.uint8, device=device)
@@ -350,9 +345,17 @@ class Trainer:
                            b.ld_agg)
             h, ld = b.out, b.ld_out
 
-    def backward(self):
-        m, p, blks = self.model, self.params, self.blocks
+    def backward(self, after_layer=None):
+        """Alg. 2 l.11-12 for layers L..1; after_layer(l), if given, runs once layer l's backward
+        is enqueued (the last group's hook starts that layer's gradient all-reduce)."""
         for l in range(self.L, 0, -1):
+            self._backward_layer(l)
+            if after_layer is not None:
+                after_layer(l)
+
+    def _backward_layer(self, l):
+        m, p, blks = self.model, self.params, self.blocks
+        if True:
             b = blks.layer[l - 1]
             if l > 1:
                 prev = blks.layer[l - 2]
@@ -364,18 +367,18 @@ class Trainer:
                 B.gat_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, h_dst, b.ld_out, p.W[l - 1], p.al[l - 1],
                           p.ar[l - 1], p.dW[l - 1], p.db[l - 1], p.dal[l - 1], p.dar[l - 1], dh_src, ld_dh_src,
                           b.bwd_scratch, b.bwd_scratch_bytes)
-                continue
+                return
             if self.is_lstm:
                 B.lstm_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out,
                            p.lstm[0][l - 1], p.lstm[1][l - 1], p.W[l - 1], p.dlstm[0][l - 1], p.dlstm[1][l - 1],
                            p.dlstm[2][l - 1], p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src, b.bwd_scratch,
                            b.bwd_scratch_bytes)
-                continue
+                return
             if self.pool:
                 B.pool_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out, b.pool_P,
                            b.pool_arg, b.ld_pool, p.Wp[l - 1], p.W[l - 1], p.dWp[l - 1], p.dbp[l - 1],
                            p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src, b.bwd_scratch, b.bwd_scratch_bytes)
-                continue
+                return
             B.sage_bwd(b, l, m, b.dh, b.ld_dh, h_src, ld_src, b.agg, b.ld_agg, h_dst, b.ld_out,
                        p.W[l - 1], p.packed[l - 1], p.dW[l - 1], p.db[l - 1], dh_src, ld_dh_src,
                        b.bwd_scratch, b.bwd_scratch_bytes)
@@ -385,11 +388,11 @@ class Trainer:
         ids = self.group_seeds.data_ptr() + 4 * int(off)
         B.softmax_ce(b.out, b.ld_out, n, self.dims[-1], self.labels, ids, self.S, self.loss, b.dh, b.ld_dh)
 
-    def microbatch(self, off, n, sampler, sizes=None):
+    def microbatch(self, off, n, sampler, sizes=None, after_layer=None):
         self.build(off, n, sampler, sizes)
         self.forward()
         self.loss_and_grad(off, n)
-        self.backward()
+        self.backward(after_layer)
         blk = self.blocks
         return dict(edges=sum(blk.layer[l].n_edges for l in range(self.L)),
                     n=[blk.layer[0].n_src] + [blk.layer[l].n_dst for l in range(self.L)],
@@ -438,6 +441,15 @@ class Trainer:
         del changed
         return hw, lo, hi, guard_ok
 
+    def _overlap_stream(self):
+        """The communication stream of the per-layer gradient all-reduce (N > 1 with an
+        initialised process group), else None (one all-reduce after the last group)."""
+        if not (self.world > 1 and torch.distributed.is_available() and torch.distributed.is_initialized()):
+            return None
+        if getattr(self, "_comm", None) is None:
+            self._comm = torch.cuda.Stream(device=self.device)
+        return self._comm
+
     def allreduce(self):
         allreduce_grads(self.params.grad, self.world, self.pg)
 
@@ -468,9 +480,30 @@ class Trainer:
         self._ensure_arena(max(need) if need else 1 << 20)          # exact (R15): no build retries
         sampler = self.sampler(epoch)
         groups = []
-        for k in mine:
-            groups.append(dict(self.microbatch(offs[k], int(offs[k + 1] - offs[k]), sampler, self.sizes_h[k]), k=k))
-        self.allreduce()
+        comm = self._overlap_stream()
+        pending = []
+
+        def reduce_layer(l):
+            # the last own group's layer-l backward is enqueued: layer l's gradient slice is final
+            # on this rank, so its all-reduce (NCCL, comm stream) overlaps layers l-1..1
+            a, b_ = self.params.layer_slice[l - 1]
+            ev = torch.cuda.current_stream().record_event()
+            comm.wait_event(ev)
+            with torch.cuda.stream(comm):
+                allreduce_grads(self.params.grad[a:b_], self.world, self.pg)
+            pending.append(l)
+
+        for i, k in enumerate(mine):
+            hook = reduce_layer if (comm is not None and i == len(mine) - 1) else None
+            groups.append(dict(self.microbatch(offs[k], int(offs[k + 1] - offs[k]), sampler, self.sizes_h[k],
+                                               hook), k=k))
+        if comm is None:
+            self.allreduce()
+        else:
+            if not mine:                                   # no own group: contribute zeros
+                for l in range(self.L, 0, -1):
+                    reduce_layer(l)
+            torch.cuda.current_stream().wait_stream(comm)
         self.step(lr)
         self.last = dict(K=K, k_tried=self.plan.k_tried, exploded=self.plan.exploded, est=est,
                          ranks=ranks, groups=groups, edges=sum(g["edges"] for g in groups),
