@@ -170,7 +170,8 @@ typedef struct {
  * cls_perm int32[n_dst]: the dst sorted by degree class min(D, 129), stable (degree bucketing of
  * the block, Alg. 2 l.6 PAPER.md:238); its tail lists the dst with D > 128 (long-tail cooperative
  * path): heavy = cls_perm + n_dst - n_heavy when the build read the sizes back, else n_heavy = -1
- * and heavy = NULL.  t_perm int32[n_src] (block >= 2 only): the src sorted by transposed degree
+ * and heavy = NULL.  Sampled blocks (fanout > 0) of the mean model have no row past the fanout
+ * and are walked in natural order: cls_perm = heavy = NULL, n_heavy = 0.  t_perm int32[n_src] (block >= 2 only): the src sorted by transposed degree
  * class; its tail holds those with more than 128 dst (n_heavy_t of them, or -1 if not counted).
  * Activations of the standard arena layout: agg (saved h_agg [n_dst][ld_agg]), out (H_l
  * [n_dst][ld_out], act dtype, or logits fp32 at l = L), dh (dH_l / dlogits fp32 [n_dst][ld_dh],

@@ -815,7 +815,10 @@ buffalo_status buffalo_build_blocks(const buffalo_graph* g, const int32_t* group
     buffalo_status st = build_layer(g, dst, nd, sp->fanout[l - 1], (uint32_t)(L - l + 1), sp->seed, l,
                                     false, A, b, s, sizes_h ? known : nullptr,
                                     m->aggregator == BUFFALO_AGG_POOL || m->aggregator == BUFFALO_AGG_GAT,
-                                    sp->fanout[l - 1] > 0 ? sp->cache[l - 1] : nullptr);
+                                    sp->fanout[l - 1] > 0 ? sp->cache[l - 1] : nullptr,
+                                    // the mean model walks sampled blocks in natural order: no
+                                    // degree-class permutation (no row exceeds the fanout)
+                                    !(m->aggregator == BUFFALO_AGG_MEAN && sp->fanout[l - 1] > 0));
     if (st == BUFFALO_ERR_CAPACITY || A.overflow) {
       if (required_bytes_h) *required_bytes_h = A.need;
       set_error("build_blocks: arena of %lld bytes too small (need >= %lld)", (long long)A.cap,

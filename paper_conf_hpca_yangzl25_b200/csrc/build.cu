@@ -14,15 +14,17 @@ namespace cg = cooperative_groups;
 namespace buffalo {
 
 // ------------------------------------------------------------------ a4: count D per dst
-__global__ void k_count(const int32_t* __restrict__ dst, int64_t n, const int64_t* __restrict__ grow,
-                        int32_t f, int32_t* __restrict__ counts) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    int64_t v = dst[i];
-    int64_t deg = grow[v + 1] - grow[v];
-    counts[i] = (int32_t)((f > 0 && deg > f) ? f : deg);
+// D(i) = min(deg(dst[i]), f) (all neighbours for f <= 0), evaluated inside the row_ptr scan.
+struct LoadDeg {
+  const int32_t* dst;
+  const int64_t* grow;
+  int32_t f;
+  __device__ __forceinline__ int32_t operator()(int64_t i) const {
+    const int64_t v = dst[i];
+    const int64_t deg = grow[v + 1] - grow[v];
+    return (int32_t)((f > 0 && deg > f) ? f : deg);
   }
-}
+};
 
 // ------------------------------------------------------------------ a4: sample / slice
 // A warp serves 32/SEG destination rows (SEG lanes each, SEG >= f).  deg <= f or f <= 0: the
@@ -73,19 +75,40 @@ struct DstRows {
   __device__ __forceinline__ int64_t operator()(int64_t i) const { return dst[i]; }
 };
 
+// The first step of the relabel (R3) fused into the fills: every written neighbour u is looked
+// up in the node map (the layer's dst were entered by k_set_map before the fill), the result
+// kept in mapped[pos] (the dst prefix id, or INT32_MAX), and a non-dst u is marked in the node
+// bitmap.  mapped == null: fill only (no relabel).
+struct MarkCtx {
+  const int32_t* node_map;
+  uint32_t* bits;
+  int32_t* mapped;
+  __device__ __forceinline__ void operator()(int64_t pos, int32_t u) const {
+    if (!mapped) return;
+    const int32_t m = node_map[u];
+    mapped[pos] = m;
+    if (m != INT32_MAX) return;                                  // a dst: keeps its prefix id
+    const uint32_t b = 1u << (u & 31);
+    if (!(bits[u >> 5] & b)) atomicOr(&bits[u >> 5], b);
+  }
+};
+
 template <int SEG>
 __global__ void __launch_bounds__(256) k_sample_fill(const int32_t* __restrict__ dst, int64_t n,
                                                      const int64_t* __restrict__ grow,
                                                      const int32_t* __restrict__ gcol, int32_t f,
                                                      uint32_t hop, uint64_t seed,
                                                      const int32_t* __restrict__ row_ptr,
-                                                     int32_t* __restrict__ out, int64_t cap) {
+                                                     int32_t* __restrict__ out, int64_t cap, MarkCtx mk) {
   constexpr int G = 32 / SEG;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
   for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n; w += warps)
     sample_warp_rows<SEG>(w, n, DstRows{dst}, grow, gcol, f, hop, seed, [&](int64_t slot, int32_t k, int32_t u) {
       const int64_t pos = (int64_t)row_ptr[slot] + k;
-      if (pos < cap) out[pos] = u;
+      if (pos < cap) {
+        out[pos] = u;
+        mk(pos, u);
+      }
     });
 }
 
@@ -95,7 +118,7 @@ template <int SEG>
 __global__ void __launch_bounds__(256) k_cache_fill(const int32_t* __restrict__ dst, int64_t n,
                                                     const int32_t* __restrict__ cache, int32_t f,
                                                     const int32_t* __restrict__ row_ptr, int32_t* __restrict__ out,
-                                                    int64_t cap) {
+                                                    int64_t cap, MarkCtx mk) {
   constexpr int G = 32 / SEG;
   const int lane = threadIdx.x & 31, g = lane / SEG, sl = lane % SEG;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
@@ -103,7 +126,11 @@ __global__ void __launch_bounds__(256) k_cache_fill(const int32_t* __restrict__ 
     const int64_t slot = w * G + g;
     if (slot >= n) continue;
     const int32_t b = row_ptr[slot], D = row_ptr[slot + 1] - b;
-    if (sl < D && b + sl < cap) out[b + sl] = cache[(int64_t)dst[slot] * f + sl];
+    if (sl < D && b + sl < cap) {
+      const int32_t u = cache[(int64_t)dst[slot] * f + sl];
+      out[b + sl] = u;
+      mk(b + sl, u);
+    }
   }
 }
 
@@ -133,17 +160,6 @@ __global__ void k_reset_map(const int32_t* __restrict__ src, int64_t n, int32_t*
 }
 // mapped (nullable): node_map[u] per edge, kept for k_col_local (a coalesced re-read instead of a
 // second random node-map lookup).
-__global__ void k_mark_bits(const int32_t* __restrict__ colg, int64_t e, const int32_t* __restrict__ node_map,
-                            uint32_t* __restrict__ bits, int32_t* __restrict__ mapped) {
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t u = colg[k];
-    const int32_t m = node_map[u];
-    if (mapped) mapped[k] = m;
-    if (m != INT32_MAX) continue;                                // a dst: keeps its prefix id
-    const uint32_t b = 1u << (u & 31);
-    if (!(bits[u >> 5] & b)) atomicOr(&bits[u >> 5], b);
-  }
-}
 struct PopcWord {
   const uint32_t* bits;
   __device__ __forceinline__ int32_t operator()(int64_t w) const { return __popc(bits[w]); }
@@ -346,7 +362,7 @@ int64_t build_frame_bytes(int64_t n_dst, int64_t e, int layer, bool sizes_only, 
 buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
                            uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
                            buffalo_block* blk, cudaStream_t s, const int64_t* known, bool t1,
-                           const int32_t* cache) {
+                           const int32_t* cache, bool dst_perm) {
   memset(blk, 0, sizeof(*blk));
   blk->n_dst = n_dst;
   blk->fanout = f;
@@ -357,11 +373,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   if (A.overflow) return BUFFALO_ERR_CAPACITY;
   int32_t* totals = (int32_t*)fr;
   int32_t* ws = (int32_t*)(fr + R(64));
-  if (n_dst > 0) {
-    k_count<<<grid_for(n_dst, 256), 256, 0, s>>>(dst, n_dst, g->row_ptr, f, rp);
-    BF_LAUNCHED("k_count");
-  }
-  BF_CHECK(scan_inplace(rp, n_dst, ws, s));
+  BF_CHECK(device_scan(LoadDeg{dst, g->row_ptr, f}, StoreArr{rp}, n_dst, ws, rp + n_dst, s));
   int64_t e = 0, nh = -1;
   if (known) {
     e = known[0];                                                  // exact sizes from the plan: no sync
@@ -377,9 +389,13 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     nh = nh32;
   }
   blk->n_edges = e;
-  blk->n_heavy = nh;
   blk->row_ptr = rp;
+  if (!dst_perm) {                 // sampled block of the mean model: no row past the fanout
+    perm = nullptr;
+    nh = 0;
+  }
   blk->cls_perm = perm;
+  blk->n_heavy = nh;
   blk->heavy = (perm && nh >= 0) ? perm + (n_dst - nh) : nullptr;
 
   // frame 2
@@ -399,29 +415,27 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     counts = (int32_t*)q;
     q += R(4 * (pc + 1));
     // degree classes of the dst rows: stable counting sort by min(D, kHeavyT + 1)
-    BF_CHECK(stable_partition(DegClass{rp}, EmitPerm{perm}, n_dst, counts, ws, s));
+    if (perm) BF_CHECK(stable_partition(DegClass{rp}, EmitPerm{perm}, n_dst, counts, ws, s));
   }
-  if (n_dst > 0 && cache && f > 0) {                             // rows sampled by the scheduler
-    const int seg = sample_seg(f), G = 32 / seg;
-    const int grid = grid_for(ceil_div(n_dst, G) * 32, 256, 16);
-    if (seg == 8) k_cache_fill<8><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e);
-    else if (seg == 16) k_cache_fill<16><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e);
-    else k_cache_fill<32><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e);
-    BF_LAUNCHED("k_cache_fill");
-  } else if (n_dst > 0) {
-    launch_sample_fill(sample_seg(f), n_dst, s, dst, n_dst, g->row_ptr, g->col, f, hop, seed, (const int32_t*)rp,
-                       colg, e);
-    BF_LAUNCHED("k_sample_fill");
-  }
-  // relabel (R3): dst prefix, then the other neighbours in ascending global id
+  // relabel (R3): dst prefix, then the other neighbours in ascending global id; the dst enter
+  // the node map first so that the fill marks the other neighbours in the bitmap as it writes
   const GraphWs gw = graph_ws(g);
   if (n_dst > 0) {
     k_set_map<<<grid_for(n_dst, 256), 256, 0, s>>>(dst, n_dst, g->node_map);
     BF_LAUNCHED("k_set_map");
   }
-  if (e > 0) {
-    k_mark_bits<<<grid_for(e, 256), 256, 0, s>>>(colg, e, g->node_map, gw.bits, col_local);
-    BF_LAUNCHED("k_mark_bits");
+  const MarkCtx mk{g->node_map, gw.bits, col_local};
+  if (n_dst > 0 && cache && f > 0) {                             // rows sampled by the scheduler
+    const int seg = sample_seg(f), G = 32 / seg;
+    const int grid = grid_for(ceil_div(n_dst, G) * 32, 256, 16);
+    if (seg == 8) k_cache_fill<8><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e, mk);
+    else if (seg == 16) k_cache_fill<16><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e, mk);
+    else k_cache_fill<32><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e, mk);
+    BF_LAUNCHED("k_cache_fill");
+  } else if (n_dst > 0) {
+    launch_sample_fill(sample_seg(f), n_dst, s, dst, n_dst, g->row_ptr, g->col, f, hop, seed, (const int32_t*)rp,
+                       colg, e, mk);
+    BF_LAUNCHED("k_sample_fill");
   }
   int64_t n_src = 0;
   if (known) {

@@ -44,7 +44,7 @@ inline GraphWs graph_ws(const buffalo_graph* g) {
 buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n_dst, int32_t f,
                            uint32_t hop, uint64_t seed, int layer, bool sizes_only, Arena& A,
                            buffalo_block* blk, cudaStream_t s, const int64_t* known = nullptr,
-                           bool t1 = false, const int32_t* cache = nullptr);
+                           bool t1 = false, const int32_t* cache = nullptr, bool dst_perm = true);
 
 // Input validation: ids in [0, N) and distinct (err_dev |= 1 / 2, stream-ordered, graph
 // bitmap left cleared); ids_error maps the word to a status; validate_graph checks the CSR

@@ -66,10 +66,14 @@ def test_blocks_bit_exact(name):
         else:
             np.testing.assert_array_equal(a["t_row_ptr"], r["t_row_ptr"])
             np.testing.assert_array_equal(a["t_col"], r["t_col"])
-        np.testing.assert_array_equal(a["heavy"], np.nonzero(r["D"] > O.HEAVY_T)[0])
-        # degree classes (degree bucketing of the block, Alg. 2 l.6): stable sort by min(D, 129)
-        cls = np.minimum(r["D"], O.HEAVY_T + 1)
-        np.testing.assert_array_equal(a["cls_perm"], np.argsort(cls, kind="stable"))
+        if fan[l - 1] > 0:
+            # a sampled block of the mean model: natural row order, no permutation, no long rows
+            assert a["cls_perm"].size == 0 and a["n_heavy"] == 0 and r["D"].max(initial=0) <= fan[l - 1]
+        else:
+            np.testing.assert_array_equal(a["heavy"], np.nonzero(r["D"] > O.HEAVY_T)[0])
+            # degree classes (degree bucketing of the block, Alg. 2 l.6): stable sort by min(D, 129)
+            cls = np.minimum(r["D"], O.HEAVY_T + 1)
+            np.testing.assert_array_equal(a["cls_perm"], np.argsort(cls, kind="stable"))
         if l >= 2:
             Dt = np.diff(r["t_row_ptr"])
             np.testing.assert_array_equal(a["t_perm"], np.argsort(np.minimum(Dt, O.HEAVY_T + 1), kind="stable"))
@@ -104,7 +108,7 @@ def test_blocks_sync_free_identical(name):
     got = blocks_to_numpy(tr.arena, tr.blocks, L)
     assert tr.blocks.arena_peak == peak
     for l, (a, r) in enumerate(zip(got, ref), start=1):
-        assert a["n_heavy"] == -1 and a["heavy"] is None and a["n_heavy_t"] == -1
+        assert a["n_heavy"] == (0 if fan[l - 1] > 0 else -1) and a["heavy"] is None and a["n_heavy_t"] == -1
         for k in ("n_dst", "n_src", "n_edges"):
             assert a[k] == r[k], (l, k)
         for k in ("row_ptr", "col_local", "src_global", "col_global", "t_row_ptr", "t_col", "cls_perm", "t_perm"):
