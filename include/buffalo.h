@@ -305,12 +305,12 @@ BUFFALO_API size_t buffalo_sage_bwd_scratch_bytes(const buffalo_block* blk, int3
  * dh_src receives dH_{l-1} fp32.
  * BF16 mode: dh_dst holds dlogits fp32 at l = L; for l < L it holds the layer's prepared
  * backward input as written by the layer above: bf16 dZ_l [n_dst][p(d_l)], then at byte offset
- * R(2 n_dst p(d_l)) fp32 column-sum partials of dZ_l [1036][d_l] (summed in row order for db).
+ * R(2 n_dst p(d_l)) fp32 column-sum partials of dZ_l [888][d_l] (summed in row order for db).
  * For l >= 2 the layer computes Ys = dZ W_self and Yn = (dZ W_neigh) / D over its n_dst rows
  * (tcgen05), then the transposed Aggregate dH_{l-1}[j] = [j < n_dst] Ys[j] + sum_{i in T(j)} Yn[i]
  * over the n_src rows with the layer-below epilogue fused: ReLU' with h_src = H_{l-1}, bf16
  * dZ_{l-1} into dh_src and its column-sum partials, i.e. dh_src receives the same prepared form
- * of layer l-1 and must hold R(2 n_src p(d_{l-1})) + R(4 * 1036 * d_{l-1}) bytes.
+ * of layer l-1 and must hold R(2 n_src p(d_{l-1})) + R(4 * 888 * d_{l-1}) bytes.
  * Pass dh_src = NULL for layer 1 (features are not trained). */
 BUFFALO_API buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
                                 float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,

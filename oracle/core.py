@@ -198,7 +198,7 @@ FP32, BF16 = 0, 1
 SCAN_TILE = 4096       # elements per tile of the implementation's device-wide scans
 PART_TILE = 4096       # elements per tile of its stable radix/bin partition passes
 DB_SPLITS = 296        # row splits of the bf16 path's deterministic db reduction
-BWD_DB_PARTS = 148 * 6 + 148   # db partial rows of the bf16 backward's fused transposed Aggregate
+BWD_DB_PARTS = 148 * 5 + 148   # db partial rows of the bf16 backward's fused transposed Aggregate
 
 
 def _R(x):

@@ -624,6 +624,15 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
       // lanes past the row read piece 0 again (same sectors, in bounds) and store nothing
       const char* hb = reinterpret_cast<const char*>(h) + (colok ? piece : 0) * 16;
       const int64_t poff = (colok ? piece : 0) * 16;
+      // MODE 2: the row's H (ReLU' mask) and Ys pieces are independent of the neighbour sum:
+      // issued before it, so their latency overlaps the Yn row loads
+      uint4 h_pre = make_uint4(0u, 0u, 0u, 0u), y_pre = make_uint4(0u, 0u, 0u, 0u);
+      if constexpr (MODE == 2) {
+        if (row >= 0 && D <= kHeavyT && colok) {
+          h_pre = __ldg(reinterpret_cast<const uint4*>(ep.H + (int64_t)row * ep.ldH + piece * 8));
+          if (row < ep.n_self) y_pre = __ldg(reinterpret_cast<const uint4*>(ep.ys + (int64_t)row * ep.ldy + piece * 8));
+        }
+      }
       float acc[E];
 #pragma unroll
       for (int k = 0; k < E; ++k) acc[k] = 0.f;
@@ -697,12 +706,12 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
           static_assert(E == 8, "the backward epilogue reads bf16 rows");
           if (row < ep.n_self) {
             float y[8];
-            bf16x8_to_f32(__ldg(reinterpret_cast<const uint4*>(ep.ys + (int64_t)row * ep.ldy + piece * 8)), y);
+            bf16x8_to_f32(y_pre, y);
 #pragma unroll
             for (int k = 0; k < 8; ++k) v[k] += y[k];
           }
           float hv[8];
-          bf16x8_to_f32(__ldg(reinterpret_cast<const uint4*>(ep.H + (int64_t)row * ep.ldH + piece * 8)), hv);
+          bf16x8_to_f32(h_pre, hv);
 #pragma unroll
           for (int k = 0; k < 8; ++k)
             if (!(hv[k] > 0.f) || piece * 8 + k >= ep.d) v[k] = 0.f;
@@ -776,7 +785,7 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
 
 // MODE 2 (backward, fused epilogue): a fixed grid of kGatherDbCtas CTAs (one db partial row
 // each; the heavy-row kernel owns the kHeavyDbCtas rows after them).
-constexpr int kGatherDbCtas = 148 * 6, kHeavyDbCtas = 148;
+constexpr int kGatherDbCtas = 148 * 5, kHeavyDbCtas = 148;
 constexpr int kBwdDbParts = kGatherDbCtas + kHeavyDbCtas;
 
 static buffalo_status launch_gather_epi(const int32_t* perm, const int32_t* rp, const int32_t* col, int64_t n,
@@ -792,7 +801,7 @@ static buffalo_status launch_gather_epi(const int32_t* perm, const int32_t* rp, 
     return BUFFALO_ERR_INVALID_ARG;
   }
   const ProfSlot ps = prof_begin_launch("gather", s);
-  constexpr int kU = 2, kMinB = 6;
+  constexpr int kU = 2, kMinB = 5;   // the H / Ys prefetch registers: 5 CTAs (40 warps) per SM
   const int G = 32 >> lpr_log;
   const int smem = 8 * G * npieces * 8 * 4;
   const int32_t n32 = (int32_t)(n > 0 ? n : 0);
