@@ -644,19 +644,40 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
         }
         const int m = min(LPR, Dmax - base);
         int k = 0;
-        if (uni) {                                      // full groups of kU edges: no predicates
-          for (; k + kU <= m; k += kU) {
-            uint4 raw[kU];
+        // full groups of kU edges: no predicates.  Software-pipelined where the registers allow
+        // (forward, <= 16 lanes per row: the 200-260-B feature rows of layer 1): group g + 1's
+        // loads are issued before group g is summed, so 2 kU row loads per lane stay in flight
+        constexpr bool kPipe = MODE != 2 && LPR <= 16;
+        auto ld_group = [&](int k0, uint4 (&raw)[kU]) {
 #pragma unroll
             for (int uu = 0; uu < kU; ++uu) {
               if constexpr (SH) {
-                const long long an = __shfl_sync(kFull, ja, gbase + k + uu);
+                const long long an = __shfl_sync(kFull, ja, gbase + k0 + uu);
                 raw[uu] = __ldg(reinterpret_cast<const uint4*>(an + poff));
               } else {
-                const int32_t jn = __shfl_sync(kFull, jj, gbase + k + uu);
+                const int32_t jn = __shfl_sync(kFull, jj, gbase + k0 + uu);
                 raw[uu] = __ldg(reinterpret_cast<const uint4*>(hb + (int64_t)jn * ldb));
               }
             }
+          };
+        if (kPipe && uni && m >= kU) {
+          uint4 cur[kU];
+          ld_group(0, cur);
+          for (; k + kU <= m; k += kU) {
+            uint4 nxt[kU];
+            const bool more = k + 2 * kU <= m;
+            if (more) ld_group(k + kU, nxt);
+#pragma unroll
+            for (int uu = 0; uu < kU; ++uu) acc_piece<TI>(acc, cur[uu]);
+            if (more) {
+#pragma unroll
+              for (int uu = 0; uu < kU; ++uu) cur[uu] = nxt[uu];
+            }
+          }
+        } else if (uni) {
+          for (; k + kU <= m; k += kU) {
+            uint4 raw[kU];
+            ld_group(k, raw);
 #pragma unroll
             for (int uu = 0; uu < kU; ++uu) acc_piece<TI>(acc, raw[uu]);
           }
@@ -764,14 +785,17 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
     return BUFFALO_ERR_INVALID_ARG;
   }
   const ProfSlot ps = prof_begin_launch("gather", s);
-  // 2 row loads in flight per lane at 40 registers (6 CTAs, 48 warps per SM) measured best on
-  // products-shaped blocks: occupancy hides the per-row index chain better than deeper unrolling
-  constexpr int kU = 2, kMinB = 6;
+  // 2 row loads per lane per step: at 40 registers (6 CTAs, 48 warps per SM) for the 512-B rows
+  // of layers >= 2; the software-pipelined narrow-row path (<= 16 lanes per row, 4 loads in
+  // flight) takes 48 registers (5 CTAs, 40 warps per SM)
+  constexpr int kU = 2;
+  const int kMinB = lpr_log <= 4 ? 5 : 6;
   const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
   const int32_t n32 = (int32_t)n;
   const int32_t ldb = (int32_t)(ldh * (int64_t)sizeof(TI));             // row stride in bytes
-#define BF_V2(L) k_gather_v2<TI, MODE, L, kU, kMinB><<<fgrid, 256, 0, s>>>(perm, rp, col, n32, h, ldb, npieces, out, \
-                                                                          ldo, ps.edges_dev, GatherEpi{})
+#define BF_V2(L) k_gather_v2<TI, MODE, L, kU, (L <= 16 ? 5 : 6)><<<fgrid, 256, 0, s>>>(perm, rp, col, n32, h, ldb, \
+                                                                                     npieces, out, ldo, ps.edges_dev, \
+                                                                                     GatherEpi{})
   if (lpr_log <= 2) BF_V2(4);
   else if (lpr_log == 3) BF_V2(8);
   else if (lpr_log == 4) BF_V2(16);
@@ -839,11 +863,12 @@ static buffalo_status launch_gather_sharded(const buffalo_block* blk, const buff
   ep.self_out = (__nv_bfloat16*)blk->self_rows;
   ep.ld_self = blk->ld_self;
   const ProfSlot ps = prof_begin_launch("gather", s);
-  constexpr int kU = 2, kMinB = 6;
+  constexpr int kU = 2;
+  const int kMinB = lpr_log <= 4 ? 5 : 6;
   const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
   const int32_t n32 = (int32_t)n, ldb = (int32_t)(ld_src * 2);
   const __nv_bfloat16* h0 = (const __nv_bfloat16*)sh->shard[0];
-#define BF_V2S(L) k_gather_v2<__nv_bfloat16, 3, L, kU, kMinB><<<fgrid, 256, 0, s>>>( \
+#define BF_V2S(L) k_gather_v2<__nv_bfloat16, 3, L, kU, (L <= 16 ? 5 : 6)><<<fgrid, 256, 0, s>>>( \
       nullptr, blk->row_ptr, blk->col_global, n32, h0, ldb, npieces, out, ldo, ps.edges_dev, ep)
   if (lpr_log <= 2) BF_V2S(4);
   else if (lpr_log == 3) BF_V2S(8);
