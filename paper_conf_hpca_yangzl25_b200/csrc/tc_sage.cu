@@ -644,10 +644,10 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
         }
         const int m = min(LPR, Dmax - base);
         int k = 0;
-        // full groups of kU edges: no predicates.  Software-pipelined where the registers allow
-        // (forward, <= 16 lanes per row: the 200-260-B feature rows of layer 1): group g + 1's
-        // loads are issued before group g is summed, so 2 kU row loads per lane stay in flight
-        constexpr bool kPipe = MODE != 2 && LPR <= 16;
+        // full groups of kU edges: no predicates.  Software-pipelined in the forward (the
+        // backward's fused epilogue needs the registers): group g + 1's loads are issued before
+        // group g is summed, so 2 kU row loads per lane stay in flight
+        constexpr bool kPipe = MODE != 2;
         auto ld_group = [&](int k0, uint4 (&raw)[kU]) {
 #pragma unroll
             for (int uu = 0; uu < kU; ++uu) {
@@ -785,15 +785,15 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
     return BUFFALO_ERR_INVALID_ARG;
   }
   const ProfSlot ps = prof_begin_launch("gather", s);
-  // 2 row loads per lane per step: at 40 registers (6 CTAs, 48 warps per SM) for the 512-B rows
-  // of layers >= 2; the software-pipelined narrow-row path (<= 16 lanes per row, 4 loads in
-  // flight) takes 48 registers (5 CTAs, 40 warps per SM)
+  // 2 row loads per lane per step, software-pipelined (4 in flight): 48 registers, 5 CTAs (40
+  // warps) per SM — measured faster than 6 CTAs without the pipeline (layer 1: 48.2 -> 45.4 ms of
+  // forward per products epoch; the 512-B rows of layers >= 2: a further 1.2 ms)
   constexpr int kU = 2;
-  const int kMinB = lpr_log <= 4 ? 5 : 6;
+  const int kMinB = 5;
   const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
   const int32_t n32 = (int32_t)n;
   const int32_t ldb = (int32_t)(ldh * (int64_t)sizeof(TI));             // row stride in bytes
-#define BF_V2(L) k_gather_v2<TI, MODE, L, kU, (L <= 16 ? 5 : 6)><<<fgrid, 256, 0, s>>>(perm, rp, col, n32, h, ldb, \
+#define BF_V2(L) k_gather_v2<TI, MODE, L, kU, 5><<<fgrid, 256, 0, s>>>(perm, rp, col, n32, h, ldb, \
                                                                                      npieces, out, ldo, ps.edges_dev, \
                                                                                      GatherEpi{})
   if (lpr_log <= 2) BF_V2(4);
@@ -864,11 +864,11 @@ static buffalo_status launch_gather_sharded(const buffalo_block* blk, const buff
   ep.ld_self = blk->ld_self;
   const ProfSlot ps = prof_begin_launch("gather", s);
   constexpr int kU = 2;
-  const int kMinB = lpr_log <= 4 ? 5 : 6;
+  const int kMinB = 5;
   const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
   const int32_t n32 = (int32_t)n, ldb = (int32_t)(ld_src * 2);
   const __nv_bfloat16* h0 = (const __nv_bfloat16*)sh->shard[0];
-#define BF_V2S(L) k_gather_v2<__nv_bfloat16, 3, L, kU, (L <= 16 ? 5 : 6)><<<fgrid, 256, 0, s>>>( \
+#define BF_V2S(L) k_gather_v2<__nv_bfloat16, 3, L, kU, 5><<<fgrid, 256, 0, s>>>( \
       nullptr, blk->row_ptr, blk->col_global, n32, h0, ldb, npieces, out, ldo, ps.edges_dev, ep)
   if (lpr_log <= 2) BF_V2S(4);
   else if (lpr_log == 3) BF_V2S(8);
