@@ -216,7 +216,7 @@ def pitch(d):
 def dw_splits(n_l, d_out, d_in):
     """Split count of the deterministic split-K dW reduction."""
     tiles = _ceil(d_out, 64) * _ceil(2 * d_in, 64)
-    return max(1, min(_ceil(296, tiles), _ceil(n_l, 512)))
+    return max(1, min(_ceil(592, tiles), _ceil(n_l, 512)))
 
 
 def tc_dw_splits(n_l, d_out, d_in):
@@ -238,19 +238,19 @@ def _scan_ws_bytes(length):
 def pool_dw_splits(n_rows, d):
     """Split count of the pool weight's dW reduction (K = d columns, d rows)."""
     tiles = _ceil(d, 64) * _ceil(d, 64)
-    return max(1, min(_ceil(296, tiles), _ceil(n_rows, 512)))
+    return max(1, min(_ceil(592, tiles), _ceil(n_rows, 512)))
 
 
 def gemm_splits(n_rows, rows_out, K):
     """Split count of a deterministic split-K reduction over n_rows (rows_out x K result)."""
     tiles = _ceil(rows_out, 64) * _ceil(K, 64)
-    return max(1, min(_ceil(296, tiles), _ceil(max(int(n_rows), 1), 512)))
+    return max(1, min(_ceil(592, tiles), _ceil(max(int(n_rows), 1), 512)))
 
 
 def lstm_dw_splits(n_rows, d):
     """Split count of the LSTM weights' dW reduction (4d rows, K = d columns)."""
     tiles = _ceil(4 * d, 64) * _ceil(d, 64)
-    return max(1, min(_ceil(296, tiles), _ceil(max(int(n_rows), 1), 512)))
+    return max(1, min(_ceil(592, tiles), _ceil(max(int(n_rows), 1), 512)))
 
 
 def mem_model(n, e, dims, act_dtype=FP32, aggregator="mean", sharded=False):

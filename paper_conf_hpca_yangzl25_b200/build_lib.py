@@ -6,7 +6,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libbuffalo.so")
-SOURCES = ["api.cu", "build.cu", "sage.cu", "tc_sage.cu", "tc_gemm.cu", "cluster.cu"]
+SOURCES = ["api.cu", "build.cu", "sage.cu", "tc_sage.cu", "tc_gemm.cu", "tc_f32.cu", "cluster.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr"]

@@ -12,6 +12,7 @@
 #include <vector>
 
 #include "sage.cuh"
+#include "tc_f32.cuh"
 
 namespace buffalo {
 
@@ -630,6 +631,55 @@ __global__ void k_reduce_partials(const float* __restrict__ part, int S, int64_t
   }
 }
 
+// Column sums of x [n][d] over row splits of rps rows: part[s][c] (fixed order: deterministic).
+__global__ void __launch_bounds__(256) k_colsum_partial(const float* __restrict__ x, int64_t ldx, int64_t n, int d,
+                                                        int64_t rps, float* __restrict__ part) {
+  __shared__ float sh[8][33];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + lane;
+  const int64_t r0 = (int64_t)blockIdx.y * rps, r1 = min(n, r0 + rps);
+  float s = 0.f;
+  if (c < d)
+    for (int64_t i = r0 + warp; i < r1; i += 8) s += x[i * ldx + c];
+  sh[warp][lane] = s;
+  __syncthreads();
+  if (warp == 0 && c < d) {
+    float t = 0.f;
+    for (int w = 0; w < 8; ++w) t += sh[w][lane];
+    part[(int64_t)blockIdx.y * d + c] = t;
+  }
+}
+
+// dW partials part[s][n][k] and db partials db_part[s][n] (the k_dw_partial contract): on the
+// tensor cores (tc_f32.cu: 6xTF32 with per-chunk fp32 accumulation) plus a fixed-order column sum
+// for db when the operand rows are 16-B aligned; otherwise (e.g. GAT's d_el vectors, ld = 1) on
+// the CUDA-core kernel above.
+template <class TS, class TG>
+static buffalo_status dw_partial(dim3 grid, cudaStream_t s, int64_t nrows, int d_out, int d_in, int K, const float* dz,
+                                 int64_t ldz, const TS* self, int64_t lds, const int32_t* gidx, const TG* agg,
+                                 int64_t ldg, int64_t rows_per_split, float* part, float* db_part) {
+  const bool halves = K == 2 * d_in && agg;
+  if (std::is_same<TG, float>::value && (halves || (K == d_in && !agg)) && tcf_aligned(dz, ldz, 4) &&
+      tcf_aligned(self, lds, sizeof(TS)) && tcf_aligned(agg, ldg, 4)) {
+    const int S = (int)grid.z;
+    TcfDw p{};
+    p.n = nrows; p.d_out = d_out; p.d_in = d_in;
+    p.Z = dz; p.ldz = ldz; p.self = self; p.lds = lds; p.gidx = gidx;
+    p.agg = (const float*)agg; p.lda = ldg; p.part = part;
+    BF_CHECK(tcf_dw(p, S, std::is_same<TS, __nv_bfloat16>::value, s));
+    if (db_part) {
+      k_colsum_partial<<<dim3((unsigned)ceil_div(d_out, 32), (unsigned)S), 256, 0, s>>>(dz, ldz, nrows, d_out,
+                                                                                         rows_per_split, db_part);
+      BF_LAUNCHED("k_colsum_partial");
+    }
+    return BUFFALO_OK;
+  }
+  k_dw_partial<TS, TG><<<grid, 256, 0, s>>>(nrows, d_out, d_in, K, dz, ldz, self, lds, gidx, agg, ldg, rows_per_split,
+                                            part, db_part);
+  BF_LAUNCHED("k_dw_partial");
+  return BUFFALO_OK;
+}
+
 // ------------------------------------------------------------------ loss, optimizer, packing
 __global__ void __launch_bounds__(256) k_softmax_ce(const float* __restrict__ z, int64_t ld, int64_t n, int classes,
                                                     const int32_t* __restrict__ labels,
@@ -765,7 +815,7 @@ buffalo_status sage_fwd_ffma(const FwdArgs& a, cudaStream_t s) {
 
 int dw_splits(int64_t n_l, int d_out, int d_in) {
   int64_t tiles = ceil_div(d_out, 64) * ceil_div(2 * d_in, 64);
-  int64_t a = ceil_div(296, tiles), b = ceil_div(n_l, 512);
+  int64_t a = ceil_div(592, tiles), b = ceil_div(n_l, 512);
   int64_t sp = a < b ? a : b;
   return (int)(sp < 1 ? 1 : sp);
 }
@@ -794,10 +844,9 @@ static buffalo_status bwd_ffma_t(const BwdArgs& a, cudaStream_t s) {
   const int64_t rps = ceil_div(n > 0 ? n : 1, S);
   if (n > 0) {
     dim3 g((unsigned)ceil_div(2 * d_in, DW_T), (unsigned)ceil_div(d_out, DW_T), (unsigned)S);
-    k_dw_partial<TS, TG><<<g, 256, 0, s>>>(n, d_out, d_in, 2 * d_in, a.dh, a.ld_dh, (const TS*)a.h_src, a.ld_src,
+    BF_CHECK((dw_partial<TS, TG>(g, s, n, d_out, d_in, 2 * d_in, a.dh, a.ld_dh, (const TS*)a.h_src, a.ld_src,
                                            a.layer1 ? blk->src_global : nullptr, (const TG*)a.agg,
-                                           a.ld_agg, rps, dw_part, db_part);
-    BF_LAUNCHED("k_dw_partial");
+                                           a.ld_agg, rps, dw_part, db_part)));
     k_reduce_partials<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, (int64_t)d_out * 2 * d_in, a.dW);
     BF_LAUNCHED("k_reduce_partials");
     k_reduce_partials<<<1, 256, 0, s>>>(db_part, S, d_out, a.db);
@@ -896,7 +945,7 @@ __global__ void __launch_bounds__(256) k_pool_scatterT(const int32_t* __restrict
 
 int pool_dw_splits(int64_t n_rows, int d) {
   const int64_t tiles = ceil_div(d, 64) * ceil_div(d, 64);
-  const int64_t a = ceil_div(296, tiles), b = ceil_div(n_rows, 512);
+  const int64_t a = ceil_div(592, tiles), b = ceil_div(n_rows, 512);
   const int64_t sp = a < b ? a : b;
   return (int)(sp < 1 ? 1 : sp);
 }
@@ -967,9 +1016,8 @@ static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
   if (n > 0) {
     // dW, db of the Update weight (as the mean path)
     dim3 g((unsigned)ceil_div(2 * d_in, DW_T), (unsigned)ceil_div(d_out, DW_T), (unsigned)S);
-    k_dw_partial<TI, float><<<g, 256, 0, s>>>(n, d_out, d_in, 2 * d_in, a.dh, a.ld_dh, (const TI*)a.h_src,
-                                              a.ld_src, gidx, a.agg, a.ld_agg, ceil_div(n, S), dw_part, db_part);
-    BF_LAUNCHED("k_dw_partial");
+    BF_CHECK((dw_partial<TI, float>(g, s, n, d_out, d_in, 2 * d_in, a.dh, a.ld_dh, (const TI*)a.h_src,
+                                              a.ld_src, gidx, a.agg, a.ld_agg, ceil_div(n, S), dw_part, db_part)));
     k_reduce_partials<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, (int64_t)d_out * 2 * d_in, a.dW);
     BF_LAUNCHED("k_reduce_partials");
     k_reduce_partials<<<1, 256, 0, s>>>(db_part, S, d_out, a.db);
@@ -990,9 +1038,8 @@ static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
   }
   // dW_pool, db_pool over the src rows
   dim3 g2((unsigned)ceil_div(d_in, DW_T), (unsigned)ceil_div(d_in, DW_T), (unsigned)S2);
-  k_dw_partial<TI, float><<<g2, 256, 0, s>>>(ns, d_in, d_in, d_in, dq, dp, (const TI*)a.h_src, a.ld_src, gidx,
-                                             nullptr, 0, ceil_div(ns, S2), dwp_part, dbp_part);
-  BF_LAUNCHED("k_dw_partial");
+  BF_CHECK((dw_partial<TI, float>(g2, s, ns, d_in, d_in, d_in, dq, dp, (const TI*)a.h_src, a.ld_src, gidx,
+                                             nullptr, 0, ceil_div(ns, S2), dwp_part, dbp_part)));
   k_reduce_partials<<<grid_for((int64_t)d_in * d_in, 256), 256, 0, s>>>(dwp_part, S2, (int64_t)d_in * d_in, a.dW_pool);
   BF_LAUNCHED("k_reduce_partials");
   k_reduce_partials<<<1, 256, 0, s>>>(dbp_part, S2, d_in, a.db_pool);
@@ -1169,7 +1216,7 @@ __global__ void __launch_bounds__(256) k_lstm_scatterT(const int32_t* __restrict
 
 int lstm_dw_splits(int64_t n_rows, int d) {
   const int64_t tiles = ceil_div(4 * d, 64) * ceil_div(d, 64);
-  const int64_t a = ceil_div(296, tiles), b = ceil_div(n_rows > 0 ? n_rows : 1, 512);
+  const int64_t a = ceil_div(592, tiles), b = ceil_div(n_rows > 0 ? n_rows : 1, 512);
   const int64_t sp = a < b ? a : b;
   return (int)(sp < 1 ? 1 : sp);
 }
@@ -1317,9 +1364,8 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
   float* dbl_part = (float*)q;
   if (n > 0) {
     dim3 g((unsigned)ceil_div(2 * d, DW_T), (unsigned)ceil_div(d_out, DW_T), (unsigned)S);
-    k_dw_partial<TI, float><<<g, 256, 0, st>>>(n, d_out, d, 2 * d, a.dh, a.ld_dh, (const TI*)a.h_src, a.ld_src, gidx,
-                                               a.agg, a.ld_agg, ceil_div(n, S), dw_part, db_part);
-    BF_LAUNCHED("k_dw_partial");
+    BF_CHECK((dw_partial<TI, float>(g, st, n, d_out, d, 2 * d, a.dh, a.ld_dh, (const TI*)a.h_src, a.ld_src, gidx,
+                                               a.agg, a.ld_agg, ceil_div(n, S), dw_part, db_part)));
     k_reduce_partials<<<grid_for((int64_t)d_out * 2 * d, 256), 256, 0, st>>>(dw_part, S, (int64_t)d_out * 2 * d, a.dW);
     BF_LAUNCHED("k_reduce_partials");
     k_reduce_partials<<<1, 256, 0, st>>>(db_part, S, d_out, a.db);
@@ -1350,16 +1396,14 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
   if (e > 0) {
     // dW_ih (+ db_lstm) = dG^T X over the packed rows, then dW_hh = dG^T H_prev
     dim3 g3((unsigned)ceil_div(d, DW_T), (unsigned)ceil_div(4 * d, DW_T), (unsigned)S3);
-    k_dw_partial<TI, float><<<g3, 256, 0, st>>>(e, 4 * d, d, d, v.G, ldg, (const TI*)a.h_src, a.ld_src, v.gix, nullptr,
-                                                0, ceil_div(e, S3), dwl_part, dbl_part);
-    BF_LAUNCHED("k_dw_partial");
+    BF_CHECK((dw_partial<TI, float>(g3, st, e, 4 * d, d, d, v.G, ldg, (const TI*)a.h_src, a.ld_src, v.gix, nullptr,
+                                                0, ceil_div(e, S3), dwl_part, dbl_part)));
     k_reduce_partials<<<grid_for((int64_t)4 * d * d, 256), 256, 0, st>>>(dwl_part, S3, (int64_t)4 * d * d, a.dW_ih);
     BF_LAUNCHED("k_reduce_partials");
     k_reduce_partials<<<grid_for(4 * d, 256), 256, 0, st>>>(dbl_part, S3, 4 * d, a.db_lstm);
     BF_LAUNCHED("k_reduce_partials");
-    k_dw_partial<float, float><<<g3, 256, 0, st>>>(e, 4 * d, d, d, v.G, ldg, Hprev, dp, nullptr, nullptr, 0,
-                                                   ceil_div(e, S3), dwl_part, dbl_part);
-    BF_LAUNCHED("k_dw_partial");
+    BF_CHECK((dw_partial<float, float>(g3, st, e, 4 * d, d, d, v.G, ldg, Hprev, dp, nullptr, nullptr, 0,
+                                                   ceil_div(e, S3), dwl_part, dbl_part)));
     k_reduce_partials<<<grid_for((int64_t)4 * d * d, 256), 256, 0, st>>>(dwl_part, S3, (int64_t)4 * d * d, a.dW_hh);
     BF_LAUNCHED("k_reduce_partials");
   }
@@ -1475,23 +1519,6 @@ __global__ void k_gat_elu_bwd(float* __restrict__ dh, int64_t ldd, const float* 
 
 // column sums of dOut, split-K: CTA (32 columns, row split z of rps rows), 8 warps over the
 // rows, fixed-order combine into part[z][c]; k_reduce_partials then adds the splits in order
-__global__ void __launch_bounds__(256) k_colsum_partial(const float* __restrict__ x, int64_t ldx, int64_t n, int d,
-                                                        int64_t rps, float* __restrict__ part) {
-  __shared__ float sh[8][33];
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int c = blockIdx.x * 32 + lane;
-  const int64_t r0 = (int64_t)blockIdx.y * rps, r1 = min(n, r0 + rps);
-  float s = 0.f;
-  if (c < d)
-    for (int64_t i = r0 + warp; i < r1; i += 8) s += x[i * ldx + c];
-  sh[warp][lane] = s;
-  __syncthreads();
-  if (warp == 0 && c < d) {
-    float t = 0.f;
-    for (int w = 0; w < 8; ++w) t += sh[w][lane];
-    part[(int64_t)blockIdx.y * d + c] = t;
-  }
-}
 
 // per dst row: dalpha_e = dOut_i . Z[col_e] (kept in ds), then ds_e = alpha_e (dalpha_e - sum
 // alpha dalpha) LeakyReLU'(s_e), d_er[i] = sum_e ds_e
@@ -1579,7 +1606,7 @@ __global__ void __launch_bounds__(256) k_gat_src_bwd(const int32_t* __restrict__
 
 int gemm_splits(int64_t n_rows, int rows_out, int K) {
   const int64_t tiles = ceil_div(rows_out, 64) * ceil_div(K, 64);
-  const int64_t a = ceil_div(296, tiles), b = ceil_div(n_rows > 0 ? n_rows : 1, 512);
+  const int64_t a = ceil_div(592, tiles), b = ceil_div(n_rows > 0 ? n_rows : 1, 512);
   const int64_t sp = a < b ? a : b;
   return (int)(sp < 1 ? 1 : sp);
 }
@@ -1681,24 +1708,21 @@ static buffalo_status gat_bwd_t(const GatArgs& a, cudaStream_t st) {
   BF_LAUNCHED("k_gat_src_bwd");
   // da_l = d_el^T Z, da_r = d_er^T Z[:n_dst], dW = dZ^T H (deterministic split reductions)
   dim3 gl((unsigned)ceil_div(dl, DW_T), 1, (unsigned)Sl);
-  k_dw_partial<float, float><<<gl, 256, 0, st>>>(ns, 1, dl, dl, d_el, 1, v.Z, ldz, nullptr, nullptr, 0,
-                                                 ceil_div(ns, Sl), dal_part, dal_b);
-  BF_LAUNCHED("k_dw_partial");
+  BF_CHECK((dw_partial<float, float>(gl, st, ns, 1, dl, dl, d_el, 1, v.Z, ldz, nullptr, nullptr, 0,
+                                                 ceil_div(ns, Sl), dal_part, dal_b)));
   k_reduce_partials<<<1, 256, 0, st>>>(dal_part, Sl, dl, a.da_l);
   BF_LAUNCHED("k_reduce_partials");
   if (nd > 0) {
     dim3 gr((unsigned)ceil_div(dl, DW_T), 1, (unsigned)Sr);
-    k_dw_partial<float, float><<<gr, 256, 0, st>>>(nd, 1, dl, dl, d_er, 1, v.Z, ldz, nullptr, nullptr, 0,
-                                                   ceil_div(nd, Sr), dar_part, dar_b);
-    BF_LAUNCHED("k_dw_partial");
+    BF_CHECK((dw_partial<float, float>(gr, st, nd, 1, dl, dl, d_er, 1, v.Z, ldz, nullptr, nullptr, 0,
+                                                   ceil_div(nd, Sr), dar_part, dar_b)));
     k_reduce_partials<<<1, 256, 0, st>>>(dar_part, Sr, dl, a.da_r);
     BF_LAUNCHED("k_reduce_partials");
   }
   dim3 gw((unsigned)ceil_div(d_in, DW_T), (unsigned)ceil_div(dl, DW_T), (unsigned)S4);
-  k_dw_partial<TI, float><<<gw, 256, 0, st>>>(ns, dl, d_in, d_in, dZ, ldz, (const TI*)a.h_src, a.ld_src,
+  BF_CHECK((dw_partial<TI, float>(gw, st, ns, dl, d_in, d_in, dZ, ldz, (const TI*)a.h_src, a.ld_src,
                                               a.layer1 ? blk->src_global : nullptr, nullptr, 0, ceil_div(ns, S4),
-                                              dw_part, db_part);
-  BF_LAUNCHED("k_dw_partial");
+                                              dw_part, db_part)));
   k_reduce_partials<<<grid_for((int64_t)dl * d_in, 256), 256, 0, st>>>(dw_part, S4, (int64_t)dl * d_in, a.dW);
   BF_LAUNCHED("k_reduce_partials");
   if (a.dh_src) {   // dH_{l-1} = dZ W
