@@ -495,6 +495,37 @@ __global__ void __launch_bounds__(256, 2) k_gemm2_tc(int64_t M, int N, int Np, i
     }
 }
 
+// The dense GEMMs of every fp32-output path: tcgen05 kind::tf32 (tc_f32.cu) when the operands
+// meet its 16-B row alignment, else the fallback kernel (SIMT k_gemm2 or the mma.sync
+// k_gemm2_tc) on the same contract.  SIMT (the mean model's FFMA parity path) asks tcf_gemm for
+// the exact 3-term split.
+template <class TA1, class TA2, class TO, bool TB = false, bool SIMT = false>
+static buffalo_status gemm2(dim3 grid, cudaStream_t s, int64_t M, int N, int Np, int K1, int K2, const TA1* A1,
+                            int64_t lda1, const int32_t* gidx, int64_t m1, const TA2* A2, int64_t lda2,
+                            const float* B1, int64_t ldb1, const float* B2, int64_t ldb2, const float* bias, int relu,
+                            TO* C, int64_t ldc) {
+  if (std::is_same<TA2, float>::value && std::is_same<TO, float>::value && K1 + K2 <= kTcfMaxK &&
+      tcf_aligned(A1, lda1, sizeof(TA1)) &&
+      tcf_aligned(A2, lda2, 4) && tcf_aligned(B1, ldb1, 4) && tcf_aligned(B2, ldb2, 4) && tcf_aligned(C, ldc, 4)) {
+    TcfGemm p{};
+    p.M = M; p.N = N; p.Np = Np; p.K1 = K1; p.K2 = K2;
+    p.A1 = A1; p.lda1 = lda1; p.gidx = gidx; p.m1 = m1;
+    p.A2 = (const float*)A2; p.lda2 = lda2;
+    p.B1 = B1; p.ldb1 = ldb1; p.B2 = B2; p.ldb2 = ldb2;
+    p.bias = bias; p.relu = relu; p.C = (float*)C; p.ldc = ldc;
+    return tcf_gemm(p, std::is_same<TA1, __nv_bfloat16>::value, TB, SIMT, s);
+  }
+  if (SIMT) {
+    k_gemm2<TA1, TA2, TO, TB><<<grid, 256, 0, s>>>(M, N, Np, K1, K2, A1, lda1, gidx, m1, A2, lda2, B1, ldb1, B2, ldb2,
+                                                   bias, relu, C, ldc);
+  } else {
+    k_gemm2_tc<TA1, TA2, TO, TB><<<grid, 256, 0, s>>>(M, N, Np, K1, K2, A1, lda1, gidx, m1, A2, lda2, B1, ldb1, B2,
+                                                      ldb2, bias, relu, C, ldc);
+  }
+  BF_LAUNCHED("k_gemm2");
+  return BUFFALO_OK;
+}
+
 // ------------------------------------------------------------------ backward pieces
 template <class TH>
 __global__ void k_dz_mask(float* __restrict__ dz, int64_t ldz, const TH* __restrict__ h, int64_t ldh,
@@ -666,7 +697,8 @@ static buffalo_status dw_partial(dim3 grid, cudaStream_t s, int64_t nrows, int d
     p.n = nrows; p.d_out = d_out; p.d_in = d_in;
     p.Z = dz; p.ldz = ldz; p.self = self; p.lds = lds; p.gidx = gidx;
     p.agg = (const float*)agg; p.lda = ldg; p.part = part;
-    BF_CHECK(tcf_dw(p, S, std::is_same<TS, __nv_bfloat16>::value, s));
+    if (std::is_same<TS, float>::value) BF_CHECK(tcf_dw_tma(p, S, s));
+    else BF_CHECK(tcf_dw(p, S, true, s));
     if (db_part) {
       k_colsum_partial<<<dim3((unsigned)ceil_div(d_out, 32), (unsigned)S), 256, 0, s>>>(dz, ldz, nrows, d_out,
                                                                                          rows_per_split, db_part);
@@ -792,17 +824,16 @@ static buffalo_status fwd_ffma_t(const FwdArgs& a, cudaStream_t s) {
   dim3 grid((unsigned)ceil_div(M, GB_M), (unsigned)ceil_div(Np, GB_N));
   const float* Wt = (const float*)a.W_packed;   // [2 d_in][d_out]
   if (a.out_f32) {
-    k_gemm2<TI, TA, float><<<grid, 256, 0, s>>>(M, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
+    BF_CHECK((gemm2<TI, TA, float, false, true>(grid, s, M, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
                                                a.layer1 ? blk->src_global : nullptr, M, (const TA*)a.agg,
                                                a.ld_agg, Wt, a.d_out, Wt + (int64_t)a.d_in * a.d_out,
-                                               a.d_out, a.b, a.relu, (float*)a.out, a.ld_out);
+                                               a.d_out, a.b, a.relu, (float*)a.out, a.ld_out)));
   } else {
-    k_gemm2<TI, TA, TA><<<grid, 256, 0, s>>>(M, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
+    BF_CHECK((gemm2<TI, TA, TA, false, true>(grid, s, M, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
                                             a.layer1 ? blk->src_global : nullptr, M, (const TA*)a.agg,
                                             a.ld_agg, Wt, a.d_out, Wt + (int64_t)a.d_in * a.d_out,
-                                            a.d_out, a.b, a.relu, (TA*)a.out, a.ld_out);
+                                            a.d_out, a.b, a.relu, (TA*)a.out, a.ld_out)));
   }
-  BF_LAUNCHED("k_gemm2");
   return BUFFALO_OK;
 }
 
@@ -861,10 +892,9 @@ static buffalo_status bwd_ffma_t(const BwdArgs& a, cudaStream_t s) {
     BF_LAUNCHED("k_aggT");
     const int Np = (int)pitch_of(d_in);
     dim3 grid((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(Np, GB_N));
-    k_gemm2<float, float, float><<<grid, 256, 0, s>>>(ns, d_in, Np, d_out, d_out, a.dh, a.ld_dh, nullptr, n,
+    BF_CHECK((gemm2<float, float, float, false, true>(grid, s, ns, d_in, Np, d_out, d_out, a.dh, a.ld_dh, nullptr, n,
                                                       aggT, dp, a.W, 2 * d_in, a.W + d_in, 2 * d_in,
-                                                      nullptr, 0, a.dh_src, a.ld_dh_src);
-    BF_LAUNCHED("k_gemm2");
+                                                      nullptr, 0, a.dh_src, a.ld_dh_src)));
   }
   return BUFFALO_OK;
 }
@@ -967,10 +997,9 @@ static buffalo_status pool_fwd_t(const PoolArgs& a, cudaStream_t s) {
   const int32_t* gidx = a.layer1 ? blk->src_global : nullptr;
   if (ns > 0) {   // P = ReLU(H W_pool^T + b_pool)
     dim3 grid((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2_tc<TI, float, float, true><<<grid, 256, 0, s>>>(ns, a.d_in, dp, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
+    BF_CHECK((gemm2<TI, float, float, true, false>(grid, s, ns, a.d_in, dp, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
                                                         gidx, ns, nullptr, 0, a.W_pool, a.d_in, nullptr, 0,
-                                                        a.b_pool, 1, a.P, a.ld_pool);
-    BF_LAUNCHED("k_gemm2");
+                                                        a.b_pool, 1, a.P, a.ld_pool)));
   }
   if (nd <= 0) return BUFFALO_OK;
   const ProfSlot ps = prof_begin_launch("pool_max", s);
@@ -983,11 +1012,10 @@ static buffalo_status pool_fwd_t(const PoolArgs& a, cudaStream_t s) {
   const int Np = (int)pitch_of(a.d_out);
   dim3 grid((unsigned)ceil_div(nd, GB_M), (unsigned)ceil_div(Np, GB_N));
   const float* Wt = a.W_packed;   // [2 d_in][d_out]
-  k_gemm2_tc<TI, float, float><<<grid, 256, 0, s>>>(nd, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
+  BF_CHECK((gemm2<TI, float, float, false, false>(grid, s, nd, a.d_out, Np, a.d_in, a.d_in, (const TI*)a.h_src, a.ld_src,
                                                 gidx, nd, a.agg, a.ld_agg, Wt, a.d_out,
                                                 Wt + (int64_t)a.d_in * a.d_out, a.d_out, a.b, !a.last, a.out,
-                                                a.ld_out);
-  BF_LAUNCHED("k_gemm2");
+                                                a.ld_out)));
   return BUFFALO_OK;
 }
 
@@ -1024,9 +1052,8 @@ static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
     BF_LAUNCHED("k_reduce_partials");
     // dh_agg = dZ W_neigh  (B[k][n] = W[k][d_in + n])
     dim3 gg((unsigned)ceil_div(n, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2_tc<float, float, float><<<gg, 256, 0, s>>>(n, d_in, dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
-                                                   a.W + d_in, 2 * d_in, nullptr, 0, nullptr, 0, dagg, dp);
-    BF_LAUNCHED("k_gemm2");
+    BF_CHECK((gemm2<float, float, float, false, false>(gg, s, n, d_in, dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
+                                                   a.W + d_in, 2 * d_in, nullptr, 0, nullptr, 0, dagg, dp)));
   }
   if (ns <= 0) return BUFFALO_OK;
   if (n > 0) {
@@ -1046,10 +1073,9 @@ static buffalo_status pool_bwd_t(const PoolArgs& a, cudaStream_t s) {
   BF_LAUNCHED("k_reduce_partials");
   if (a.dh_src) {   // dH_{l-1} = pad(dZ W_self) + dQ W_pool
     dim3 gg((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2_tc<float, float, float><<<gg, 256, 0, s>>>(ns, d_in, dp, d_out, d_in, a.dh, a.ld_dh, nullptr, n, dq, dp,
+    BF_CHECK((gemm2<float, float, float, false, false>(gg, s, ns, d_in, dp, d_out, d_in, a.dh, a.ld_dh, nullptr, n, dq, dp,
                                                    a.W, 2 * d_in, a.W_pool, d_in, nullptr, 0, a.dh_src,
-                                                   a.ld_dh_src);
-    BF_LAUNCHED("k_gemm2");
+                                                   a.ld_dh_src)));
   }
   return BUFFALO_OK;
 }
@@ -1312,10 +1338,9 @@ static buffalo_status lstm_fwd_t(const LstmArgs& a, cudaStream_t st) {
     BF_LAUNCHED("k_lstm_gix");
     dim3 grid((unsigned)ceil_div(c_t, GB_M), (unsigned)ceil_div(ldg, GB_N));
     const ProfSlot ps = prof_begin_launch("lstm_gates", st);
-    k_gemm2_tc<TI, float, float, true><<<grid, 256, 0, st>>>(c_t, 4 * d, (int)ldg, d, t ? d : 0, (const TI*)a.h_src,
+    BF_CHECK((gemm2<TI, float, float, true, false>(grid, st, c_t, 4 * d, (int)ldg, d, t ? d : 0, (const TI*)a.h_src,
                                                          a.ld_src, v.gix + off[t], c_t, v.Hs + s[t] * dp, dp,
-                                                         a.W_ih, d, a.W_hh, d, a.b_lstm, 0, v.G + off[t] * ldg, ldg);
-    BF_LAUNCHED("k_gemm2");
+                                                         a.W_ih, d, a.W_hh, d, a.b_lstm, 0, v.G + off[t] * ldg, ldg)));
     // "algorithmic bytes" of this family are FLOPs: 2 * rows * 4d * (d [x_t] + d [h_{t-1}, t > 0])
     prof_end_launch(ps, st, 2.0 * (double)c_t * 4.0 * d * (double)(t ? 2 * d : d), 0.0);
     k_lstm_cell<<<grid_for(c_t * d, 256), 256, 0, st>>>(v.G + off[t] * ldg, ldg, v.Cs + off[t] * dp, v.Hs, v.Cst,
@@ -1328,11 +1353,10 @@ static buffalo_status lstm_fwd_t(const LstmArgs& a, cudaStream_t st) {
   const int Np = (int)pitch_of(a.d_out);
   dim3 grid((unsigned)ceil_div(n, GB_M), (unsigned)ceil_div(Np, GB_N));
   const float* Wt = a.W_packed;   // [2 d_in][d_out]
-  k_gemm2_tc<TI, float, float><<<grid, 256, 0, st>>>(n, a.d_out, Np, d, d, (const TI*)a.h_src, a.ld_src,
+  BF_CHECK((gemm2<TI, float, float, false, false>(grid, st, n, a.d_out, Np, d, d, (const TI*)a.h_src, a.ld_src,
                                                  a.layer1 ? blk->src_global : nullptr, n, a.agg, a.ld_agg, Wt,
                                                  a.d_out, Wt + (int64_t)d * a.d_out, a.d_out, a.b, !a.last, a.out,
-                                                 a.ld_out);
-  BF_LAUNCHED("k_gemm2");
+                                                 a.ld_out)));
   return BUFFALO_OK;
 }
 
@@ -1371,9 +1395,8 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
     k_reduce_partials<<<1, 256, 0, st>>>(db_part, S, d_out, a.db);
     BF_LAUNCHED("k_reduce_partials");
     dim3 gg((unsigned)ceil_div(n, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2_tc<float, float, float><<<gg, 256, 0, st>>>(n, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
-                                                    a.W + d, 2 * d, nullptr, 0, nullptr, 0, dagg, dp);
-    BF_LAUNCHED("k_gemm2");
+    BF_CHECK((gemm2<float, float, float, false, false>(gg, st, n, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
+                                                    a.W + d, 2 * d, nullptr, 0, nullptr, 0, dagg, dp)));
     k_lstm_bwd_init<<<grid_for(n * dp, 256), 256, 0, st>>>(blk->cls_perm, dagg, n, dp, v.Hs, v.Cst);
     BF_LAUNCHED("k_lstm_bwd_init");
   }
@@ -1387,10 +1410,9 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
     BF_LAUNCHED("k_lstm_cell_bwd");
     if (t > 0) {   // dh_{t-1} = dG_t W_hh into the running rows' state
       dim3 gg((unsigned)ceil_div(c_t, GB_M), (unsigned)ceil_div(dp, GB_N));
-      k_gemm2_tc<float, float, float><<<gg, 256, 0, st>>>(c_t, d, (int)dp, 4 * d, 0, v.G + off[t] * ldg, ldg, nullptr, c_t,
+      BF_CHECK((gemm2<float, float, float, false, false>(gg, st, c_t, d, (int)dp, 4 * d, 0, v.G + off[t] * ldg, ldg, nullptr, c_t,
                                                       nullptr, 0, a.W_hh, d, nullptr, 0, nullptr, 0, v.Hs + s[t] * dp,
-                                                      dp);
-      BF_LAUNCHED("k_gemm2");
+                                                      dp)));
     }
   }
   if (e > 0) {
@@ -1409,14 +1431,12 @@ static buffalo_status lstm_bwd_t(const LstmArgs& a, cudaStream_t st) {
   }
   if (a.dh_src && ns > 0) {   // dH_{l-1} = pad(dZ W_self) + sum over edges of dG W_ih
     dim3 gg((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dp, GB_N));
-    k_gemm2_tc<float, float, float><<<gg, 256, 0, st>>>(ns, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
-                                                    a.W, 2 * d, nullptr, 0, nullptr, 0, a.dh_src, a.ld_dh_src);
-    BF_LAUNCHED("k_gemm2");
+    BF_CHECK((gemm2<float, float, float, false, false>(gg, st, ns, d, (int)dp, d_out, 0, a.dh, a.ld_dh, nullptr, n, nullptr, 0,
+                                                    a.W, 2 * d, nullptr, 0, nullptr, 0, a.dh_src, a.ld_dh_src)));
     if (e > 0) {
       dim3 gx((unsigned)ceil_div(e, GB_M), (unsigned)ceil_div(dp, GB_N));
-      k_gemm2_tc<float, float, float><<<gx, 256, 0, st>>>(e, d, (int)dp, 4 * d, 0, v.G, ldg, nullptr, e, nullptr, 0,
-                                                      a.W_ih, d, nullptr, 0, nullptr, 0, dX, dp);
-      BF_LAUNCHED("k_gemm2");
+      BF_CHECK((gemm2<float, float, float, false, false>(gx, st, e, d, (int)dp, 4 * d, 0, v.G, ldg, nullptr, e, nullptr, 0,
+                                                      a.W_ih, d, nullptr, 0, nullptr, 0, dX, dp)));
       k_lstm_scatterT<<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(blk->t_row_ptr, blk->t_col, blk->row_ptr,
                                                                   blk->col_local, v.ppos, ns, dX, dp, d, a.dh_src,
                                                                   a.ld_dh_src);
@@ -1644,10 +1664,9 @@ static buffalo_status gat_fwd_t(const GatArgs& a, cudaStream_t st) {
   GatSaved v = gat_saved_view(a.saved, ns, nd, e, dl);
   if (ns > 0) {
     dim3 grid((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(ldz, GB_N));
-    k_gemm2_tc<TI, float, float, true><<<grid, 256, 0, st>>>(ns, dl, (int)ldz, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
+    BF_CHECK((gemm2<TI, float, float, true, false>(grid, st, ns, dl, (int)ldz, a.d_in, 0, (const TI*)a.h_src, a.ld_src,
                                                          a.layer1 ? blk->src_global : nullptr, ns, nullptr, 0, a.W,
-                                                         a.d_in, nullptr, 0, nullptr, 0, v.Z, ldz);
-    BF_LAUNCHED("k_gemm2");
+                                                         a.d_in, nullptr, 0, nullptr, 0, v.Z, ldz)));
     k_gat_scores<<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(v.Z, ldz, ns, nd, dl, a.a_l, a.a_r, v.el, v.er);
     BF_LAUNCHED("k_gat_scores");
   }
@@ -1728,9 +1747,8 @@ static buffalo_status gat_bwd_t(const GatArgs& a, cudaStream_t st) {
   if (a.dh_src) {   // dH_{l-1} = dZ W
     const int64_t dpi = pitch_of(d_in);
     dim3 gg((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(dpi, GB_N));
-    k_gemm2_tc<float, float, float><<<gg, 256, 0, st>>>(ns, d_in, (int)dpi, dl, 0, dZ, ldz, nullptr, ns, nullptr, 0, a.W,
-                                                    d_in, nullptr, 0, nullptr, 0, a.dh_src, a.ld_dh_src);
-    BF_LAUNCHED("k_gemm2");
+    BF_CHECK((gemm2<float, float, float, false, false>(gg, st, ns, d_in, (int)dpi, dl, 0, dZ, ldz, nullptr, ns, nullptr, 0, a.W,
+                                                    d_in, nullptr, 0, nullptr, 0, a.dh_src, a.ld_dh_src)));
   }
   return BUFFALO_OK;
 }
