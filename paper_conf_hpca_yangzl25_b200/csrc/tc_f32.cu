@@ -720,6 +720,224 @@ __global__ void __launch_bounds__(kGemmThreads, 1) k_tcf_gemm(const TcfGemm p) {
   }
 }
 
+// ===================================================================== GEMM, TMA-fed (fp32 A)
+// The k_tcf_gemm contract for fp32 A1, every operand loaded by TMA as it lies in memory: A rows
+// K-major ({32 k, 128 row} SWIZZLE_128B box, or 32 gather4 of 4 rows for gathered A1 rows), B
+// K-major when stored [n][k] (TB) or MN-major when stored [k][n] (four {32 n, 32 k}
+// SWIZZLE_128B_ATOM_32B boxes).  The raw fp32 chunk lands in term tile 0; 8 worker warps split it
+// in place into the NS TF32 terms (zeroing A1 rows >= m1 of a gathered A1), warp 8 issues the TMA,
+// warp 9 the MMAs, warps 10-13 drain the two TMEM accumulators (bias / ReLU, C rows per thread).
+constexpr int kGtWork = 8;
+constexpr int kGtTma = kGtWork, kGtMma = kGtWork + 1, kGtEpi0 = kGtWork + 2;
+constexpr int kGtThreads = (kGtWork + 2 + 4) * 32;
+
+struct TcfGemmTmaP {
+  int64_t M, m1;
+  int N, Np, K1, K2;
+  const int32_t* gidx;
+  const float* bias;
+  int relu;
+  float* C;
+  int64_t ldc;
+};
+
+template <bool TB, int NS, bool GATHER>
+__global__ void __launch_bounds__(kGtThreads, 1)
+    k_tcf_gemm_tma(const __grid_constant__ CUtensorMap a1_map, const __grid_constant__ CUtensorMap a2_map,
+                   const __grid_constant__ CUtensorMap b1_map, const __grid_constant__ CUtensorMap b2_map,
+                   const TcfGemmTmaP p) {
+  constexpr int NT = 128, NST = NS == 2 ? 3 : 2;
+  constexpr int kTile = kTM * 128;                      // 16 KB: 128 rows (or n) x 32 fp32
+  constexpr int kOp = NS * kTile, kStage = 2 * kOp;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
+  uint64_t* full = (uint64_t*)(smem + NST * kStage);
+  uint64_t* split = full + NST;
+  uint64_t* empty = split + NST;
+  uint64_t* tfull = empty + NST;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tslot = (uint32_t*)(tempty + 2);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, tid = threadIdx.x;
+  const int tiles_n = (p.Np + NT - 1) / NT;
+  const int64_t ntiles = (int64_t)((p.M + kTM - 1) / kTM) * tiles_n;
+  const int nk1 = (p.K1 + kKC - 1) / kKC, nk2 = (p.K2 + kKC - 1) / kKC, nk = nk1 + nk2;
+  if (tid == 0) {
+    for (int i = 0; i < NST; ++i) {
+      mb_init(&full[i], 1);
+      mb_init(&split[i], kGtWork * 32);
+      mb_init(&empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mb_init(&tfull[i], 1);
+      mb_init(&tempty[i], 4 * 32);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == kGtMma) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tslot)), "r"(2 * NT));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *tslot;
+
+  if (warp == kGtTma) {
+    if (nk > 0) {
+      int64_t g = 0;
+      for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        const int64_t m0 = (tile / tiles_n) * kTM;
+        const int n0 = (int)(tile % tiles_n) * NT;
+        for (int c = 0; c < nk; ++c, ++g) {
+          const int st = (int)(g % NST);
+          const bool first = c < nk1;
+          const int k0 = (first ? c : c - nk1) * kKC;
+          if (lane == 0) {
+            if (g >= NST) mb_wait(&empty[st], (uint32_t)(((g / NST) - 1) & 1));
+            mb_expect(&full[st], 2 * kTile);
+          }
+          __syncwarp();
+          uint8_t* sa = smem + st * kStage;
+          uint8_t* sb = sa + kOp;
+          if (first && GATHER) {
+            int32_t rr[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+              const int64_t r = m0 + lane * 4 + k;
+              rr[k] = r < p.m1 ? __ldg(p.gidx + r) : 0;   // rows >= m1 are zeroed by the split
+            }
+            tma_gather4(sa + lane * 512, &a1_map, k0, rr[0], rr[1], rr[2], rr[3], &full[st]);
+          } else if (lane == 0) {
+            tma_2d(sa, first ? &a1_map : &a2_map, k0, (int)m0, &full[st]);
+          }
+          if (lane == 0) {
+            const CUtensorMap* bm = first ? &b1_map : &b2_map;
+            if (TB) {
+              tma_2d(sb, bm, k0, n0, &full[st]);
+            } else {
+#pragma unroll
+              for (int j = 0; j < 4; ++j) tma_2d(sb + j * kDwStrip, bm, n0 + 32 * j, k0, &full[st]);
+            }
+          }
+          __syncwarp();
+        }
+      }
+    }
+  } else if (warp == kGtMma) {
+    if (lane == 0 && nk > 0) {
+      constexpr uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | (TB ? 0u : (1u << 16)) |
+                                 ((uint32_t)(NT >> 3) << 17) | ((uint32_t)(kTM >> 4) << 24);
+      int64_t g = 0;
+      int it = 0;
+      for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++it) {
+        const int ab = it & 1;
+        if (it >= 2) mb_wait(&tempty[ab], (uint32_t)(((it >> 1) - 1) & 1));
+        fence_after();
+        const uint32_t d = tmem + ab * NT;
+        for (int c = 0; c < nk; ++c, ++g) {
+          const int st = (int)(g % NST);
+          mb_wait(&split[st], (uint32_t)((g / NST) & 1));
+          fence_after();
+          const uint32_t a0 = su32(smem + st * kStage), b0 = a0 + kOp;
+#pragma unroll
+          for (int kk = 0; kk < kKC / 8; ++kk)
+#pragma unroll
+            for (int i = 0; i < NS; ++i)
+#pragma unroll
+              for (int j = 0; j < NS - i; ++j) {
+                const uint64_t bd = TB ? desc_sw128(b0 + j * kTile + kk * 32) : desc_mn(b0 + j * kTile + kk * 1024, kDwStrip);
+                mma_tf32(d, desc_sw128(a0 + i * kTile + kk * 32), bd, idesc, (c > 0 || kk > 0 || i > 0 || j > 0) ? 1u : 0u);
+              }
+          commit(&empty[st]);
+        }
+        commit(&tfull[ab]);
+      }
+    }
+    __syncwarp();
+  } else if (warp < kGtWork) {
+    if (nk > 0) {
+      int64_t g = 0;
+      for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        const int64_t m0 = (tile / tiles_n) * kTM;
+        for (int c = 0; c < nk; ++c, ++g) {
+          const int st = (int)(g % NST);
+          mb_wait(&full[st], (uint32_t)((g / NST) & 1));
+          uint8_t* sa = smem + st * kStage;
+          const bool mask = GATHER && c < nk1 && m0 + kTM > p.m1;
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const int idx = tid + kGtWork * 32 * i;      // 0 .. 2047: 16-B pieces of both raw tiles
+            const int op = idx >> 10, off = (idx & 1023) * 16;
+            if (op == 0 && mask && m0 + (off >> 7) >= p.m1) {
+#pragma unroll
+              for (int k = 0; k < NS; ++k) *reinterpret_cast<float4*>(sa + k * kTile + off) = make_float4(0.f, 0.f, 0.f, 0.f);
+            } else {
+              split_inplace4<NS>(sa + op * kOp, kTile, off);
+            }
+          }
+          fence_async_smem();
+          mb_arrive(&split[st]);
+        }
+      }
+    }
+  } else {
+    const int q = warp & 3;                            // TMEM lane quadrant of this warp
+    const bool vec = (p.ldc & 3) == 0 && (((uintptr_t)p.C) & 15) == 0;
+    int it = 0;
+    for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++it) {
+      const int ab = it & 1;
+      const int64_t row = (tile / tiles_n) * kTM + q * 32 + lane;
+      const int n0 = (int)(tile % tiles_n) * NT;
+      if (nk > 0) {
+        mb_wait(&tfull[ab], (uint32_t)((it >> 1) & 1));
+        fence_after();
+      }
+#pragma unroll 1
+      for (int h = 0; h < 4; ++h) {
+        float v[32];
+        if (nk > 0) {
+          tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + ab * NT + h * 32, v);
+        } else {
+#pragma unroll
+          for (int k = 0; k < 32; ++k) v[k] = 0.f;
+        }
+        const int nb = n0 + h * 32;
+        if (row < p.M && nb < p.Np) {
+          float* out = p.C + row * p.ldc + nb;
+#pragma unroll
+          for (int k = 0; k < 32; ++k) {
+            const int nn = nb + k;
+            float x = 0.f;
+            if (nn < p.N) {
+              x = v[k] + (p.bias ? __ldg(p.bias + nn) : 0.f);
+              if (p.relu) x = fmaxf(x, 0.f);
+            }
+            v[k] = x;
+          }
+          if (vec && nb + 32 <= p.Np) {
+#pragma unroll
+            for (int k = 0; k < 32; k += 4) *reinterpret_cast<float4*>(out + k) = make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]);
+          } else {
+#pragma unroll
+            for (int k = 0; k < 32; ++k)
+              if (nb + k < p.Np) out[k] = v[k];
+          }
+        }
+      }
+      if (nk > 0) {
+        fence_before();
+        mb_arrive(&tempty[ab]);
+      }
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == kGtMma) {
+    fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(2 * NT));
+  }
+}
+
 // ===================================================================== host launcher
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
@@ -820,8 +1038,45 @@ static buffalo_status launch_tcf_gemm(const TcfGemm& p, bool exact, cudaStream_t
   return exact ? launch_tcf_gemm_ns<TA1, TB, 3>(p, s) : launch_tcf_gemm_ns<TA1, TB, 2>(p, s);
 }
 
+template <bool TB, int NS, bool GATHER>
+static buffalo_status launch_tcf_gemm_tma(const TcfGemm& q, cudaStream_t s) {
+  constexpr int kSmem = (NS == 2 ? 3 : 2) * 2 * NS * kTM * 128 + 256 + 1024;
+  constexpr CUtensorMapSwizzle kK = CU_TENSOR_MAP_SWIZZLE_128B, kMN = CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B;
+  CUtensorMap a1, a2, b1, b2;
+  const float* A1 = (const float*)q.A1;
+  const float* A2 = q.A2 ? q.A2 : A1;
+  const float* B2 = q.B2 ? q.B2 : q.B1;
+  // A1 rows beyond m1 carry no A1 term: the map ends there (gathered: the split zeroes them)
+  BF_CHECK(encode_f32(&a1, A1, q.K1, GATHER ? (int64_t)INT32_MAX : q.m1, q.lda1, GATHER ? 1 : kTM, kK));
+  BF_CHECK(encode_f32(&a2, A2, q.K2 > 0 ? q.K2 : q.K1, q.M, q.A2 ? q.lda2 : q.lda1, kTM, kK));
+  if (TB) {
+    BF_CHECK(encode_f32(&b1, q.B1, q.K1, q.N, q.ldb1, 128, kK));
+    BF_CHECK(encode_f32(&b2, B2, q.K2 > 0 ? q.K2 : q.K1, q.N, q.B2 ? q.ldb2 : q.ldb1, 128, kK));
+  } else {
+    BF_CHECK(encode_f32(&b1, q.B1, q.N, q.K1, q.ldb1, kKC, kMN));
+    BF_CHECK(encode_f32(&b2, B2, q.N, q.K2 > 0 ? q.K2 : q.K1, q.B2 ? q.ldb2 : q.ldb1, kKC, kMN));
+  }
+  TcfGemmTmaP p{};
+  p.M = q.M; p.m1 = q.m1; p.N = q.N; p.Np = q.Np; p.K1 = q.K1; p.K2 = q.K2;
+  p.gidx = q.gidx; p.bias = q.bias; p.relu = q.relu; p.C = q.C; p.ldc = q.ldc;
+  const int64_t tiles = ((q.M + kTM - 1) / kTM) * ((q.Np + 127) / 128);
+  const int grid = (int)std::min<int64_t>(tiles, 148);
+  BF_CHECK((set_max_smem_once<k_tcf_gemm_tma<TB, NS, GATHER>>(kSmem)));
+  k_tcf_gemm_tma<TB, NS, GATHER><<<grid, kGtThreads, kSmem, s>>>(a1, a2, b1, b2, p);
+  BF_LAUNCHED("k_tcf_gemm_tma");
+  return BUFFALO_OK;
+}
+template <bool TB, int NS>
+static buffalo_status launch_tcf_gemm_tma_g(const TcfGemm& q, cudaStream_t s) {
+  return q.gidx && q.K1 > 0 ? launch_tcf_gemm_tma<TB, NS, true>(q, s) : launch_tcf_gemm_tma<TB, NS, false>(q, s);
+}
+
 buffalo_status tcf_gemm(const TcfGemm& p, bool a1_bf16, bool tb, bool exact, cudaStream_t s) {
   if (p.M <= 0 || p.Np <= 0) return BUFFALO_OK;
+  if (!a1_bf16) {
+    if (tb) return exact ? launch_tcf_gemm_tma_g<true, 3>(p, s) : launch_tcf_gemm_tma_g<true, 2>(p, s);
+    return exact ? launch_tcf_gemm_tma_g<false, 3>(p, s) : launch_tcf_gemm_tma_g<false, 2>(p, s);
+  }
   if (a1_bf16)
     return tb ? launch_tcf_gemm<__nv_bfloat16, true>(p, exact, s) : launch_tcf_gemm<__nv_bfloat16, false>(p, exact, s);
   return tb ? launch_tcf_gemm<float, true>(p, exact, s) : launch_tcf_gemm<float, false>(p, exact, s);
