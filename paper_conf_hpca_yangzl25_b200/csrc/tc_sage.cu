@@ -116,6 +116,31 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
   __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
   return *reinterpret_cast<uint32_t*>(&h);
 }
+// L2 eviction-priority hints (createpolicy + .L2::cache_hint): the Aggregate's gathered rows are
+// re-read across rows (hub rows, the dst-side Yn table of the backward), its output rows and
+// per-row side inputs are touched once.
+__device__ __forceinline__ uint64_t l2_policy_keep() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_stream() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint4 ldg_pol(const void* ptr, uint64_t pol) {
+  uint4 r;
+  asm("ld.global.nc.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
+      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+      : "l"(ptr), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ void stg_pol(void* ptr, const uint4& v, uint64_t pol) {
+  asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(ptr), "r"(v.x), "r"(v.y),
+               "r"(v.z), "r"(v.w), "l"(pol)
+               : "memory");
+}
 __device__ __forceinline__ void bf16x8_to_f32(const uint4& u, float* v) {
   const uint32_t w[4] = {u.x, u.y, u.z, u.w};
 #pragma unroll
@@ -566,7 +591,7 @@ __device__ __forceinline__ long long shard_row(const GatherEpi& ep, int32_t j, i
   return (long long)(ep.shard[u / ep.rps] + (int64_t)(u % ep.rps) * ldb);
 }
 
-template <class TI, int MODE, int LPR, int kU, int MINB>
+template <class TI, int MODE, int LPR, int kU, int MINB, int HINT>
 __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restrict__ perm,
                                                          const int32_t* __restrict__ rp,
                                                          const int32_t* __restrict__ col, int32_t n,
@@ -578,6 +603,15 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
   constexpr int G = 32 / LPR;
   constexpr unsigned kFull = 0xffffffffu;
   constexpr bool SH = MODE == 3;                      // sharded feature table
+  // HINT bits: 1 = gathered rows evict_last, 2 = per-row side inputs (MODE 2: H, Ys) evict_first,
+  // 4 = output rows evict_first
+  uint64_t pol_keep = 0, pol_stream = 0;
+  if constexpr (HINT & 1) pol_keep = l2_policy_keep();
+  if constexpr (HINT & 6) pol_stream = l2_policy_stream();
+  auto ld_row = [&](const void* ptr) -> uint4 {
+    if constexpr (HINT & 1) return ldg_pol(ptr, pol_keep);
+    else return __ldg(reinterpret_cast<const uint4*>(ptr));
+  };
   const int lane = threadIdx.x & 31;
   const int g = lane / LPR, pc = lane & (LPR - 1);
   const int gbase = g * LPR;
@@ -629,8 +663,15 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
       uint4 h_pre = make_uint4(0u, 0u, 0u, 0u), y_pre = make_uint4(0u, 0u, 0u, 0u);
       if constexpr (MODE == 2) {
         if (row >= 0 && D <= kHeavyT && colok) {
-          h_pre = __ldg(reinterpret_cast<const uint4*>(ep.H + (int64_t)row * ep.ldH + piece * 8));
-          if (row < ep.n_self) y_pre = __ldg(reinterpret_cast<const uint4*>(ep.ys + (int64_t)row * ep.ldy + piece * 8));
+          const __nv_bfloat16* hp = ep.H + (int64_t)row * ep.ldH + piece * 8;
+          const __nv_bfloat16* yp = ep.ys + (int64_t)row * ep.ldy + piece * 8;
+          if constexpr (HINT & 2) {
+            h_pre = ldg_pol(hp, pol_stream);
+            if (row < ep.n_self) y_pre = ldg_pol(yp, pol_stream);
+          } else {
+            h_pre = __ldg(reinterpret_cast<const uint4*>(hp));
+            if (row < ep.n_self) y_pre = __ldg(reinterpret_cast<const uint4*>(yp));
+          }
         }
       }
       float acc[E];
@@ -653,10 +694,10 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
             for (int uu = 0; uu < kU; ++uu) {
               if constexpr (SH) {
                 const long long an = __shfl_sync(kFull, ja, gbase + k0 + uu);
-                raw[uu] = __ldg(reinterpret_cast<const uint4*>(an + poff));
+                raw[uu] = ld_row(reinterpret_cast<const void*>(an + poff));
               } else {
                 const int32_t jn = __shfl_sync(kFull, jj, gbase + k0 + uu);
-                raw[uu] = __ldg(reinterpret_cast<const uint4*>(hb + (int64_t)jn * ldb));
+                raw[uu] = ld_row(hb + (int64_t)jn * ldb);
               }
             }
           };
@@ -690,11 +731,11 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
             if constexpr (SH) {
               const long long an = __shfl_sync(kFull, ja, gbase + ((k + uu) & (LPR - 1)));
               ok[uu] = k + uu < m && an != -1;
-              if (ok[uu]) raw[uu] = __ldg(reinterpret_cast<const uint4*>(an + poff));
+              if (ok[uu]) raw[uu] = ld_row(reinterpret_cast<const void*>(an + poff));
             } else {
               const int32_t jn = __shfl_sync(kFull, jj, gbase + ((k + uu) & (LPR - 1)));
               ok[uu] = k + uu < m && jn >= 0;
-              if (ok[uu]) raw[uu] = __ldg(reinterpret_cast<const uint4*>(hb + (int64_t)jn * ldb));
+              if (ok[uu]) raw[uu] = ld_row(hb + (int64_t)jn * ldb);
             }
           }
 #pragma unroll
@@ -745,8 +786,10 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
         }
         __nv_bfloat16* dst = out + (int64_t)row * ldo + piece * E;
         if constexpr (E == 8) {
-          *reinterpret_cast<uint4*>(dst) = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
-                                                      pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
+          const uint4 o = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+                                     pack_bf16x2(v[6], v[7]));
+          if constexpr (HINT & 4) stg_pol(dst, o, pol_stream);
+          else *reinterpret_cast<uint4*>(dst) = o;
         } else {
           *reinterpret_cast<uint2*>(dst) = make_uint2(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]));
         }
@@ -769,6 +812,9 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
     }
   }
 }
+
+// L2 eviction hints of the forward (MODE 0 / 3) and backward (MODE 2) Aggregate launches
+constexpr int kHintFwd = 0, kHintBwd = 7;
 
 template <class TI, int MODE>
 static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, const int32_t* col, int64_t n,
@@ -793,7 +839,7 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
   const int32_t n32 = (int32_t)n;
   const int32_t ldb = (int32_t)(ldh * (int64_t)sizeof(TI));             // row stride in bytes
-#define BF_V2(L) k_gather_v2<TI, MODE, L, kU, 5><<<fgrid, 256, 0, s>>>(perm, rp, col, n32, h, ldb, \
+#define BF_V2(L) k_gather_v2<TI, MODE, L, kU, 5, kHintFwd><<<fgrid, 256, 0, s>>>(perm, rp, col, n32, h, ldb, \
                                                                                      npieces, out, ldo, ps.edges_dev, \
                                                                                      GatherEpi{})
   if (lpr_log <= 2) BF_V2(4);
@@ -830,7 +876,7 @@ static buffalo_status launch_gather_epi(const int32_t* perm, const int32_t* rp, 
   const int smem = 8 * G * npieces * 8 * 4;
   const int32_t n32 = (int32_t)(n > 0 ? n : 0);
   const int32_t ldb = (int32_t)(ldy * 2);
-#define BF_V2E(L) k_gather_v2<__nv_bfloat16, 2, L, kU, kMinB><<<kGatherDbCtas, 256, smem, s>>>( \
+#define BF_V2E(L) k_gather_v2<__nv_bfloat16, 2, L, kU, kMinB, kHintBwd><<<kGatherDbCtas, 256, smem, s>>>( \
       perm, rp, col, n32, yn, ldb, npieces, out, ldo, ps.edges_dev, ep)
   if (lpr_log <= 2) BF_V2E(4);
   else if (lpr_log == 3) BF_V2E(8);
@@ -868,7 +914,7 @@ static buffalo_status launch_gather_sharded(const buffalo_block* blk, const buff
   const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
   const int32_t n32 = (int32_t)n, ldb = (int32_t)(ld_src * 2);
   const __nv_bfloat16* h0 = (const __nv_bfloat16*)sh->shard[0];
-#define BF_V2S(L) k_gather_v2<__nv_bfloat16, 3, L, kU, 5><<<fgrid, 256, 0, s>>>( \
+#define BF_V2S(L) k_gather_v2<__nv_bfloat16, 3, L, kU, 5, kHintFwd><<<fgrid, 256, 0, s>>>( \
       nullptr, blk->row_ptr, blk->col_global, n32, h0, ldb, npieces, out, ldo, ps.edges_dev, ep)
   if (lpr_log <= 2) BF_V2S(4);
   else if (lpr_log == 3) BF_V2S(8);
