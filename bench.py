@@ -75,6 +75,10 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--world-sim", type=int, default=0,
                     help="one GPU plays each of N ranks in turn (plan for N GPUs, per-rank epoch times)")
+    ap.add_argument("--sim-shared", action="store_true",
+                    help="with --world-sim N: the ranks share the scheduler's statistics passes "
+                         "(buffalo_sched.allgather) — the all-gathers of the N ranks are recorded untimed, "
+                         "then each rank's timed epochs measure only its own share and replay the rest")
     ap.add_argument("--rank-balanced-k", action="store_true",
                     help="reading R31: only K that are multiples of the GPU count (rank-aware grouping)")
     ap.add_argument("--no-pipeline", action="store_true",
@@ -356,6 +360,69 @@ def measured_memory(tr, epoch):
 
 
 # ----------------------------------------------------------------------------- world-sim
+class AllgatherReplay:
+    """buffalo_sched.allgather for the world-sim with shared statistics (--sim-shared): serves
+    recorded all-gather results (the concatenated rows of all N ranks) in call order, after
+    checking that the calling rank's own rows equal the recorded ones (every rank's passes are
+    deterministic).  In record mode (`record` set) the call past the known results stores the
+    rank's rows and fails, which aborts that bucketize run."""
+
+    def __init__(self, world):
+        import ctypes
+        from paper_conf_hpca_yangzl25_b200 import buffalo as B
+        self.world, self.rank, self.results, self.i, self.record = world, 0, [], 0, None
+        self._ct = ctypes
+        self.fn = B.ALLGATHER_FN(self._call)
+
+    def _call(self, ctx, send, recv, nbytes):
+        ct = self._ct
+        own = ct.string_at(send, nbytes)
+        if self.i >= len(self.results):
+            if self.record is not None:
+                self.record[self.rank] = own
+            return 1
+        res = self.results[self.i]
+        if len(res) != self.world * nbytes or res[self.rank * nbytes:(self.rank + 1) * nbytes] != own:
+            return 1
+        ct.memmove(recv, res, len(res))
+        self.i += 1
+        return 0
+
+
+def record_shared_stats(tr, rep, epochs):
+    """The all-gather results of the scheduler runs of `epochs` for the N simulated ranks
+    (untimed): call i's result is assembled from every rank's rows at call i, each rank replaying
+    calls 0..i-1; repeated until the runs complete.  Returns the results in the order a pipelined
+    Trainer asks for them (one schedule per epoch, ascending)."""
+    import torch
+    from paper_conf_hpca_yangzl25_b200 import buffalo as B
+    from paper_conf_hpca_yangzl25_b200.train import PlanBuffers
+    pb = PlanBuffers(tr.S, tr.k_cap, tr.F, tr.L, tr.device)
+    s = tr.sched
+    out = []
+    for e in epochs:
+        R = []
+        while True:
+            rows = [None] * rep.world
+            for r in range(rep.world):
+                rep.rank, rep.results, rep.i, rep.record = r, R, 0, rows
+                sched = B.make_sched(s.mem_budget, s.C_ppm, s.k_min, s.k_max, rep.world, s.k_multiple, r, rep.fn)
+                sp = B.make_sampler(tr.fanout, tr.F, tr.base_seed + e)
+                try:
+                    B.bucketize(tr.graph.g_sched, tr._seeds[0], sp, tr.model, sched, pb.plan, tr.bucket_ws)
+                except B.BuffaloError:
+                    pass
+                torch.cuda.synchronize()
+            done = [x is None for x in rows]
+            assert all(done) or not any(done), "simulated ranks disagree on the number of all-gathers"
+            if all(done):
+                break
+            R.append(b"".join(rows))
+        out.extend(R)
+    rep.record = None
+    return out
+
+
 def run_world_sim(args, tr, sim, flush, stream):
     """--world-sim N on one GPU: the plan is made for N GPUs (k_min = N, LPT rank assignment,
     optionally rank-aware K), and this one process plays each rank r in turn — its replicated
@@ -365,10 +432,18 @@ def run_world_sim(args, tr, sim, flush, stream):
     simulated).  Prints one JSON line with "mode": "world_sim" (not the driver's bench line)."""
     import torch
     per = []
+    rep = getattr(tr, "_sim_replay", None)
+    recorded = None
+    if rep is not None:
+        t_rec = time.perf_counter()
+        recorded = record_shared_stats(tr, rep, range(args.warmup + args.steps + 1))
+        t_rec = time.perf_counter() - t_rec
     for r in range(sim):
         tr.rank = r
         tr.sched.rank = r                       # group sizes are measured for the own groups only
         tr._ahead = None
+        if rep is not None:
+            rep.rank, rep.results, rep.i = r, recorded, 0
         for i in range(args.warmup):
             tr.run_epoch(epoch=i, lr=0.01)
         torch.cuda.synchronize()
@@ -393,8 +468,15 @@ def run_world_sim(args, tr, sim, flush, stream):
             "rank_balanced_k": bool(args.rank_balanced_k), "per_rank": per,
             "projected_epoch_ms": worst, "projected_edges_per_s": total_edges / (worst / 1e3),
             "rank_spread_max_over_min": worst / min(p["ms_per_step"] for p in per),
-            "note": "one B200 plays each rank in turn (replicated scheduler + own groups); NCCL allreduce "
-                    "not included; the projected N-GPU epoch is the slowest rank"}
+            "shared_stats": rep is not None,
+            "note": ("one B200 plays each rank in turn (" +
+                     ("its share of the scheduler's statistics passes, the other ranks' rows replayed from an "
+                      "untimed recording (all-gather latency not included), no sample cache"
+                      if rep is not None else "replicated scheduler") +
+                     " + own groups); NCCL allreduce not included; the projected N-GPU epoch is the slowest rank")}
+    if rep is not None:
+        line["allgathers_per_epoch"] = len(recorded) / (args.warmup + args.steps + 1)
+        line["record_s"] = t_rec
     print(json.dumps(line), flush=True)
 
 
@@ -471,10 +553,12 @@ def run_ours(args, cfg):
     t_c = time.perf_counter()
     _, C_eq1, C_ppm = B.clustering(graph.g)
     t_c = time.perf_counter() - t_c
+    rep = AllgatherReplay(sim) if (sim and args.sim_shared) else None
     tr = Trainer(graph, feats, y, seeds, cfg.dims,
                  cfg.fanout, cfg.F, Ws, bs, feat_dtype=feat_dtype, gemm_mode=gemm, mem_budget=budget,
                  C_ppm=C_ppm, k_min=kmin, k_max=max(kmin, cfg.k_max), rank=rank, world=plan_world, process_group=pg,
-                 pipeline=not args.no_pipeline, k_multiple=kmult, **agg_kw)
+                 pipeline=not args.no_pipeline, k_multiple=kmult, allgather=rep.fn if rep else None, **agg_kw)
+    tr._sim_replay = rep
     full_batch_edges = None
     if args.config in ("products", "papers", "arxiv_lstm") + SHARDED:
         # calibrate M_ctr once so that one GPU needs >= 8 groups (products; 2 for the LSTM
@@ -597,7 +681,9 @@ def run_ours(args, cfg):
         roof = {"bound": "hbm",
                 "kernel": ("k_pool_max (GraphSAGE-pool neighbour max + argmax)" if pool else
                            "k_gat_attn (GAT edge softmax + attention-weighted neighbour sum)" if gat else
-                           "k_gather_v2 (Aggregate: fwd neighbour mean, bwd transposed sum)"),
+                           "k_gather_v2 (Aggregate: fwd neighbour mean, bwd transposed sum)" if gemm == B.GEMM_BF16
+                           else "k_agg_rows / k_aggT (fp32 Aggregate of the FFMA parity path: fwd neighbour mean, "
+                                "bwd transposed sum)"),
                 "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": traffic, "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": g_bytes / max(1, g_launches),

@@ -195,12 +195,16 @@ static buffalo_status launch_agg(const buffalo_block* blk, const int32_t* col, c
   const int64_t n = blk->n_dst;
   if (n <= 0) return BUFFALO_OK;
   const bool wide = d > 128;
+  const ProfSlot ps = prof_begin_launch("gather", s);
   if (wide) {
     k_agg_rows<TI, TO, 8><<<grid_for(n * 32, 256, 16), 256, 0, s>>>(blk->row_ptr, col, n, h, ldh, d, agg, lda);
   } else {
     k_agg_rows<TI, TO, 4><<<grid_for(n * 32, 256, 16), 256, 0, s>>>(blk->row_ptr, col, n, h, ldh, d, agg, lda);
   }
   BF_LAUNCHED("k_agg_rows");
+  // algorithmic bytes: per row the row_ptr pair + the output row; per edge index + source row
+  prof_end_launch(ps, s, (double)n * (8.0 + (double)pitch_of(d) * sizeof(TO)) +
+                             (double)blk->n_edges * (4.0 + (double)pitch_of(d) * sizeof(TI)), 0.0);
   const int hg = heavy_tail_grid(blk->n_heavy, blk->n_edges);
   if (hg > 0) {
     if (wide)
@@ -662,16 +666,23 @@ __global__ void k_reduce_partials(const float* __restrict__ part, int S, int64_t
   }
 }
 
-// Column sums of x [n][d] over row splits of rps rows: part[s][c] (fixed order: deterministic).
+// Column sums of x [n][d] over row splits of rps rows: part[s][c] (fixed order: deterministic);
+// wt (nullable): weighted sums, row i scaled by wt[i] (GAT's da_l = d_el^T Z, da_r = d_er^T Z).
 __global__ void __launch_bounds__(256) k_colsum_partial(const float* __restrict__ x, int64_t ldx, int64_t n, int d,
-                                                        int64_t rps, float* __restrict__ part) {
+                                                        int64_t rps, float* __restrict__ part,
+                                                        const float* __restrict__ wt = nullptr) {
   __shared__ float sh[8][33];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int c = blockIdx.x * 32 + lane;
   const int64_t r0 = (int64_t)blockIdx.y * rps, r1 = min(n, r0 + rps);
   float s = 0.f;
-  if (c < d)
-    for (int64_t i = r0 + warp; i < r1; i += 8) s += x[i * ldx + c];
+  if (c < d) {
+    if (wt) {
+      for (int64_t i = r0 + warp; i < r1; i += 8) s = fmaf(__ldg(wt + i), __ldg(x + i * ldx + c), s);
+    } else {
+      for (int64_t i = r0 + warp; i < r1; i += 8) s += x[i * ldx + c];
+    }
+  }
   sh[warp][lane] = s;
   __syncthreads();
   if (warp == 0 && c < d) {
@@ -887,9 +898,13 @@ static buffalo_status bwd_ffma_t(const BwdArgs& a, cudaStream_t s) {
     const int64_t ns = blk->n_src;
     if (ns <= 0) return BUFFALO_OK;
     const int dp = (int)pitch_of(d_out);
+    const ProfSlot ps = prof_begin_launch("gather", s);
     k_aggT<<<grid_for(ns * 32, 256, 16), 256, 0, s>>>(blk->t_row_ptr, blk->t_col, blk->row_ptr, ns, a.dh,
                                                      a.ld_dh, d_out, aggT, dp, dp);
     BF_LAUNCHED("k_aggT");
+    // algorithmic bytes: per src row the t_row_ptr pair + the fp32 output row; per entry the dst
+    // index, its row_ptr pair (1/D) and the dZ row
+    prof_end_launch(ps, s, (double)ns * (8.0 + 4.0 * dp) + (double)blk->n_edges * (12.0 + 4.0 * dp), 0.0);
     const int Np = (int)pitch_of(d_in);
     dim3 grid((unsigned)ceil_div(ns, GB_M), (unsigned)ceil_div(Np, GB_N));
     BF_CHECK((gemm2<float, float, float, false, true>(grid, s, ns, d_in, Np, d_out, d_out, a.dh, a.ld_dh, nullptr, n,
@@ -1624,6 +1639,69 @@ __global__ void __launch_bounds__(256) k_gat_src_bwd(const int32_t* __restrict__
   }
 }
 
+// k_gat_src_bwd for pitch(d) <= 128 G floats: each lane holds G 4-float chunks of the row, so the
+// edge search of an entry runs once (not once per 32-chunk pass) and the entry's dOut row loads
+// are issued before it; the per-element sum order (t ascending, fmaf) is that of k_gat_src_bwd.
+template <int G>
+__global__ void __launch_bounds__(256) k_gat_src_bwd_g(const int32_t* __restrict__ trp, const int32_t* __restrict__ tcol,
+                                                       const int32_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                                       int64_t n_src, int64_t n_dst, const float* __restrict__ alpha,
+                                                       const float* __restrict__ ds, const float* __restrict__ dO,
+                                                       int64_t ldo, int d, const float* __restrict__ al,
+                                                       const float* __restrict__ ar, const float* __restrict__ d_er,
+                                                       float* __restrict__ d_el, float* __restrict__ dZ, int64_t ldz) {
+  const int lane = threadIdx.x & 31;
+  const int nch = (int)(pitch_of(d) / 4);
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t j = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; j < n_src; j += warps) {
+    const int32_t t0 = trp[j], t1 = trp[j + 1];
+    float acc[G][4];
+#pragma unroll
+    for (int g = 0; g < G; ++g)
+#pragma unroll
+      for (int k = 0; k < 4; ++k) acc[g][k] = 0.f;
+    float dsum = 0.f;
+    for (int32_t t = t0; t < t1; ++t) {
+      const int32_t i = tcol[t];
+      float v[G][4];
+#pragma unroll
+      for (int g = 0; g < G; ++g) {
+        const int c = g * 32 + lane;
+        if (c < nch) VecIO<float, 4>::load(dO + (int64_t)i * ldo + c * 4, v[g]);
+      }
+      const int32_t eb = rp[i], ee = rp[i + 1];
+      int32_t e = -1;
+      for (int32_t e0 = eb; e0 < ee && e < 0; e0 += 32) {
+        const bool hit = e0 + lane < ee && col[e0 + lane] == (int32_t)j;
+        const unsigned m = __ballot_sync(0xffffffffu, hit);
+        if (m) e = e0 + __ffs(m) - 1;
+      }
+      const float a = alpha[e];
+      dsum += ds[e];
+#pragma unroll
+      for (int g = 0; g < G; ++g)
+        if (g * 32 + lane < nch) {
+#pragma unroll
+          for (int k = 0; k < 4; ++k) acc[g][k] = fmaf(a, v[g][k], acc[g][k]);
+        }
+    }
+    const float der = j < n_dst ? d_er[j] : 0.f;
+#pragma unroll
+    for (int g = 0; g < G; ++g) {
+      const int c = g * 32 + lane;
+      if (c < nch) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int kk = c * 4 + k;
+          acc[g][k] = kk < d ? acc[g][k] + dsum * al[kk] + der * ar[kk] : 0.f;
+        }
+        VecIO<float, 4>::store(dZ + j * ldz + c * 4, acc[g]);
+      }
+    }
+    if (lane == 0) d_el[j] = dsum;
+  }
+}
+
 int gemm_splits(int64_t n_rows, int rows_out, int K) {
   const int64_t tiles = ceil_div(rows_out, 64) * ceil_div(K, 64);
   const int64_t a = ceil_div(592, tiles), b = ceil_div(n_rows > 0 ? n_rows : 1, 512);
@@ -1721,20 +1799,33 @@ static buffalo_status gat_bwd_t(const GatArgs& a, cudaStream_t st) {
     BF_LAUNCHED("k_gat_row_bwd");
   }
   if (ns <= 0) return BUFFALO_OK;
-  k_gat_src_bwd<<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(blk->t_row_ptr, blk->t_col, blk->row_ptr, blk->col_local,
-                                                            ns, nd, v.alpha, ds, a.dh, a.ld_dh, dl, a.a_l, a.a_r,
-                                                            d_er, d_el, dZ, ldz);
+  if (ldz <= 128) {
+    k_gat_src_bwd_g<1><<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(
+        blk->t_row_ptr, blk->t_col, blk->row_ptr, blk->col_local, ns, nd, v.alpha, ds, a.dh, a.ld_dh, dl, a.a_l, a.a_r,
+        d_er, d_el, dZ, ldz);
+  } else if (ldz <= 256) {
+    k_gat_src_bwd_g<2><<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(
+        blk->t_row_ptr, blk->t_col, blk->row_ptr, blk->col_local, ns, nd, v.alpha, ds, a.dh, a.ld_dh, dl, a.a_l, a.a_r,
+        d_er, d_el, dZ, ldz);
+  } else {
+    k_gat_src_bwd<<<grid_for(ns * 32, 256, 16), 256, 0, st>>>(blk->t_row_ptr, blk->t_col, blk->row_ptr,
+                                                              blk->col_local, ns, nd, v.alpha, ds, a.dh, a.ld_dh, dl,
+                                                              a.a_l, a.a_r, d_er, d_el, dZ, ldz);
+  }
   BF_LAUNCHED("k_gat_src_bwd");
   // da_l = d_el^T Z, da_r = d_er^T Z[:n_dst], dW = dZ^T H (deterministic split reductions)
-  dim3 gl((unsigned)ceil_div(dl, DW_T), 1, (unsigned)Sl);
-  BF_CHECK((dw_partial<float, float>(gl, st, ns, 1, dl, dl, d_el, 1, v.Z, ldz, nullptr, nullptr, 0,
-                                                 ceil_div(ns, Sl), dal_part, dal_b)));
+  // (weighted column sums of Z over fixed row splits: one coalesced pass per vector)
+  (void)dal_b;
+  (void)dar_b;
+  k_colsum_partial<<<dim3((unsigned)ceil_div(dl, 32), (unsigned)Sl), 256, 0, st>>>(v.Z, ldz, ns, dl, ceil_div(ns, Sl),
+                                                                                   dal_part, d_el);
+  BF_LAUNCHED("k_colsum_partial");
   k_reduce_partials<<<1, 256, 0, st>>>(dal_part, Sl, dl, a.da_l);
   BF_LAUNCHED("k_reduce_partials");
   if (nd > 0) {
-    dim3 gr((unsigned)ceil_div(dl, DW_T), 1, (unsigned)Sr);
-    BF_CHECK((dw_partial<float, float>(gr, st, nd, 1, dl, dl, d_er, 1, v.Z, ldz, nullptr, nullptr, 0,
-                                                   ceil_div(nd, Sr), dar_part, dar_b)));
+    k_colsum_partial<<<dim3((unsigned)ceil_div(dl, 32), (unsigned)Sr), 256, 0, st>>>(v.Z, ldz, nd, dl,
+                                                                                     ceil_div(nd, Sr), dar_part, d_er);
+    BF_LAUNCHED("k_colsum_partial");
     k_reduce_partials<<<1, 256, 0, st>>>(dar_part, Sr, dl, a.da_r);
     BF_LAUNCHED("k_reduce_partials");
   }

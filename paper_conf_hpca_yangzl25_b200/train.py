@@ -189,7 +189,7 @@ class Trainer:
                  gemm_mode=B.GEMM_FFMA, mem_budget=(1 << 63) - 1, C_ppm=0, k_min=1, k_max=4096,
                  base_seed=3, rank=0, world=1, process_group=None, device="cuda", aggregator=B.AGG_MEAN,
                  Wps=None, bps=None, lstm=None, gat=None, pipeline=False, sample_cache=True, k_multiple=1,
-                 share_stats=True):
+                 share_stats=True, allgather=None):
         self.graph = graph if isinstance(graph, DeviceGraph) else DeviceGraph(*graph, device=device)
         self.feats = feats
         self.labels = labels
@@ -217,8 +217,11 @@ class Trainer:
                                   shards=feats.struct if self.sharded else None)
         # with a process group, the K loop's micro-bucket statistics are shared out over the ranks
         # (buffalo_sched.allgather); every rank still derives the identical plan
-        ag = None
-        if share_stats and world > 1 and torch.distributed.is_available() and torch.distributed.is_initialized():
+        # (allgather: an explicit buffalo_sched.allgather callback instead, e.g. bench.py's world-sim
+        # replay of the all-gathers of N simulated ranks)
+        ag = allgather if (share_stats and world > 1) else None
+        if ag is None and share_stats and world > 1 and torch.distributed.is_available() and \
+                torch.distributed.is_initialized():
             nccl = torch.distributed.get_backend(process_group) == "nccl"
             ag = B.make_allgather(world, process_group, torch.device(device) if nccl else None)
         self.sched = B.make_sched(mem_budget, C_ppm, k_min, k_max, world, k_multiple, rank, ag)
