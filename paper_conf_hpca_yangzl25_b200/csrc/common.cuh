@@ -66,6 +66,26 @@ inline int grid_for(int64_t work_items, int per_block, int blocks_per_sm = 8) {
   return (int)(g < cap ? g : cap);
 }
 
+// A library-owned non-blocking side stream per device, for fork / join overlap of independent
+// launches inside one call (events order it against the caller's stream).  Created once per
+// device; a thread that loses the creation race destroys its duplicate.  nullptr on failure
+// (callers then stay on their stream).
+inline cudaStream_t side_stream() {
+  static std::atomic<cudaStream_t> streams[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  cudaStream_t st = streams[dev].load(std::memory_order_acquire);
+  if (st) return st;
+  cudaStream_t mine = nullptr;
+  if (cudaStreamCreateWithFlags(&mine, cudaStreamNonBlocking) != cudaSuccess) return nullptr;
+  cudaStream_t expected = nullptr;
+  if (!streams[dev].compare_exchange_strong(expected, mine, std::memory_order_acq_rel)) {
+    cudaStreamDestroy(mine);
+    return expected;
+  }
+  return mine;
+}
+
 // sm_100a check of the current device.
 buffalo_status require_sm100();
 

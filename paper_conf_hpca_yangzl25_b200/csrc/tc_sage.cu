@@ -813,6 +813,9 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
   }
 }
 
+// The backward's long-tail kernel runs on a side stream next to the fused Aggregate
+constexpr bool kHeavyOverlap = true;
+
 // L2 eviction hints of the forward (MODE 0 / 3) and backward (MODE 2) Aggregate launches
 constexpr int kHintFwd = 0, kHintBwd = 7;
 
@@ -1516,10 +1519,32 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     ep.d = d_in;
     ep.db_part = (float*)((char*)a.dh_src + R(ns * dpp * 2));
     __nv_bfloat16* zprev = (__nv_bfloat16*)a.dh_src;
-    k_heavy_bwd_epi<<<kHeavyDbCtas, 256, 0, s>>>(blk->t_perm, ns, blk->t_row_ptr, blk->t_col, yn, dpp, dpp, zprev,
-                                                  dpp, ep, kGatherDbCtas);
+    // the long-tail rows (a CTA each: hub src rows with thousands of entries) on a side stream, so
+    // their tail overlaps the regular rows' gather (disjoint dZ rows and db partial rows)
+    cudaStream_t hs = kHeavyOverlap ? side_stream() : nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr;
+    if (hs && (cudaEventCreateWithFlags(&fork, cudaEventDisableTiming) != cudaSuccess ||
+               cudaEventCreateWithFlags(&join, cudaEventDisableTiming) != cudaSuccess)) {
+      if (fork) cudaEventDestroy(fork);
+      fork = nullptr;
+      hs = nullptr;
+    }
+    if (hs) {
+      BF_CUDA(cudaEventRecord(fork, s));
+      BF_CUDA(cudaStreamWaitEvent(hs, fork, 0));
+    }
+    k_heavy_bwd_epi<<<kHeavyDbCtas, 256, 0, hs ? hs : s>>>(blk->t_perm, ns, blk->t_row_ptr, blk->t_col, yn, dpp, dpp,
+                                                            zprev, dpp, ep, kGatherDbCtas);
     BF_LAUNCHED("k_heavy_bwd_epi");
-    BF_CHECK(launch_gather_epi(blk->t_perm, blk->t_row_ptr, blk->t_col, ns, yn, dpp, dpp, zprev, dpp, ep, s));
+    if (hs) BF_CUDA(cudaEventRecord(join, hs));
+    const buffalo_status st_g = launch_gather_epi(blk->t_perm, blk->t_row_ptr, blk->t_col, ns, yn, dpp, dpp, zprev,
+                                                  dpp, ep, s);
+    if (hs) {
+      BF_CUDA(cudaStreamWaitEvent(s, join, 0));
+      cudaEventDestroy(fork);
+      cudaEventDestroy(join);
+    }
+    BF_CHECK(st_g);
   }
   return BUFFALO_OK;
 }
