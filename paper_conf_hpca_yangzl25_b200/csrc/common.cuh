@@ -70,21 +70,51 @@ inline int grid_for(int64_t work_items, int per_block, int blocks_per_sm = 8) {
 // launches inside one call (events order it against the caller's stream).  Created once per
 // device; a thread that loses the creation race destroys its duplicate.  nullptr on failure
 // (callers then stay on their stream).
-inline cudaStream_t side_stream() {
-  static std::atomic<cudaStream_t> streams[64];
+inline cudaStream_t side_stream(int k = 0) {
+  static std::atomic<cudaStream_t> streams[64][2];
   int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
-  cudaStream_t st = streams[dev].load(std::memory_order_acquire);
+  if (k < 0 || k > 1 || cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  cudaStream_t st = streams[dev][k].load(std::memory_order_acquire);
   if (st) return st;
   cudaStream_t mine = nullptr;
   if (cudaStreamCreateWithFlags(&mine, cudaStreamNonBlocking) != cudaSuccess) return nullptr;
   cudaStream_t expected = nullptr;
-  if (!streams[dev].compare_exchange_strong(expected, mine, std::memory_order_acq_rel)) {
+  if (!streams[dev][k].compare_exchange_strong(expected, mine, std::memory_order_acq_rel)) {
     cudaStreamDestroy(mine);
     return expected;
   }
   return mine;
 }
+
+// Fork of side stream k off the caller's stream (work enqueued on stream() after the fork point
+// runs concurrently with later work on the caller's stream); join() — or the destructor, on
+// early error returns — makes the caller's stream wait for it.  Without a side stream (on==false
+// or creation failure) stream() is the caller's stream and join() is a no-op.
+struct SideFork {
+  cudaStream_t main, side = nullptr;
+  cudaEvent_t ev = nullptr;
+  SideFork(cudaStream_t s, int k, bool on) : main(s) {
+    if (!on || !(side = side_stream(k))) return;
+    if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess || cudaEventRecord(ev, main) != cudaSuccess ||
+        cudaStreamWaitEvent(side, ev, 0) != cudaSuccess) {
+      if (ev) cudaEventDestroy(ev);
+      ev = nullptr;
+      side = nullptr;
+    }
+  }
+  cudaStream_t stream() const { return side ? side : main; }
+  bool join() {
+    if (!side) return true;
+    bool ok = cudaEventRecord(ev, side) == cudaSuccess && cudaStreamWaitEvent(main, ev, 0) == cudaSuccess;
+    cudaEventDestroy(ev);
+    ev = nullptr;
+    side = nullptr;
+    return ok;
+  }
+  ~SideFork() { join(); }
+  SideFork(const SideFork&) = delete;
+  SideFork& operator=(const SideFork&) = delete;
+};
 
 // sm_100a check of the current device.
 buffalo_status require_sm100();

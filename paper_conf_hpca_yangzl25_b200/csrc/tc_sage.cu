@@ -815,6 +815,8 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
 
 // The backward's long-tail kernel runs on a side stream next to the fused Aggregate
 constexpr bool kHeavyOverlap = true;
+// The layer's dW / db reductions run on a side stream next to its dH products and Aggregate
+constexpr bool kDwOverlap = true;
 
 // L2 eviction hints of the forward (MODE 0 / 3) and backward (MODE 2) Aggregate launches
 constexpr int kHintFwd = 0, kHintBwd = 7;
@@ -1468,7 +1470,12 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
                                                        nullptr, db_part);
     BF_LAUNCHED("k_dz_prep");
   }
-  // dW (TMA-fed tensor cores, deterministic split reduction) and db
+  // dW (TMA-fed tensor cores, deterministic split reduction) and db: on side stream 1 when the
+  // layer also has the dH products and the transposed Aggregate to run (independent work: both
+  // only read dZ), joined before returning
+  SideFork dwf(s, 1, kDwOverlap && a.dh_src != nullptr);
+  {
+  cudaStream_t s = dwf.stream();
   if (a.shards) {            // layer 1 of a sharded table: the self rows were copied by the forward
     BF_CHECK(tc_dw_tma(n, S, zb, dp, d_out, (const __nv_bfloat16*)blk->self_rows, blk->ld_self, nullptr, n,
                        (const __nv_bfloat16*)a.agg, a.ld_agg, d_in, dw_part, s));
@@ -1498,6 +1505,7 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
   BF_LAUNCHED("k_reduce_dw");
   k_reduce_db<<<(unsigned)ceil_div(d_out, 32), 1024, 0, s>>>(db_part, nparts, d_out, a.db);
   BF_LAUNCHED("k_reduce_db");
+  }
   // dH_{l-1}[j] = [j < n_dst] (dZ W_self)[j] + sum_{i in T(j)} (dZ W_neigh)[i] / D(i): the two
   // products over the n_dst rows first (tcgen05, the 1/D row scale in the epilogue), then the
   // transposed Aggregate over the n_src rows with the layer-below epilogue fused (+ Ys, ReLU'
@@ -1519,32 +1527,17 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     ep.d = d_in;
     ep.db_part = (float*)((char*)a.dh_src + R(ns * dpp * 2));
     __nv_bfloat16* zprev = (__nv_bfloat16*)a.dh_src;
-    // the long-tail rows (a CTA each: hub src rows with thousands of entries) on a side stream, so
+    // the long-tail rows (a CTA each: hub src rows with thousands of entries) on side stream 0, so
     // their tail overlaps the regular rows' gather (disjoint dZ rows and db partial rows)
-    cudaStream_t hs = kHeavyOverlap ? side_stream() : nullptr;
-    cudaEvent_t fork = nullptr, join = nullptr;
-    if (hs && (cudaEventCreateWithFlags(&fork, cudaEventDisableTiming) != cudaSuccess ||
-               cudaEventCreateWithFlags(&join, cudaEventDisableTiming) != cudaSuccess)) {
-      if (fork) cudaEventDestroy(fork);
-      fork = nullptr;
-      hs = nullptr;
-    }
-    if (hs) {
-      BF_CUDA(cudaEventRecord(fork, s));
-      BF_CUDA(cudaStreamWaitEvent(hs, fork, 0));
-    }
-    k_heavy_bwd_epi<<<kHeavyDbCtas, 256, 0, hs ? hs : s>>>(blk->t_perm, ns, blk->t_row_ptr, blk->t_col, yn, dpp, dpp,
+    SideFork hv(s, 0, kHeavyOverlap);
+    k_heavy_bwd_epi<<<kHeavyDbCtas, 256, 0, hv.stream()>>>(blk->t_perm, ns, blk->t_row_ptr, blk->t_col, yn, dpp, dpp,
                                                             zprev, dpp, ep, kGatherDbCtas);
     BF_LAUNCHED("k_heavy_bwd_epi");
-    if (hs) BF_CUDA(cudaEventRecord(join, hs));
-    const buffalo_status st_g = launch_gather_epi(blk->t_perm, blk->t_row_ptr, blk->t_col, ns, yn, dpp, dpp, zprev,
-                                                  dpp, ep, s);
-    if (hs) {
-      BF_CUDA(cudaStreamWaitEvent(s, join, 0));
-      cudaEventDestroy(fork);
-      cudaEventDestroy(join);
+    BF_CHECK(launch_gather_epi(blk->t_perm, blk->t_row_ptr, blk->t_col, ns, yn, dpp, dpp, zprev, dpp, ep, s));
+    if (!hv.join() || !dwf.join()) {
+      set_error("sage_bwd: side-stream join failed");
+      return BUFFALO_ERR_CUDA;
     }
-    BF_CHECK(st_g);
   }
   return BUFFALO_OK;
 }
