@@ -56,7 +56,6 @@ SHARDED = ("igb", "igb_small")
 
 # Table II's average clustering coefficients, logged beside the C measured
 # on the synthetic graph (reading R27; the Chung-Lu graphs have far fewer triangles)
-FP32_PEAK_TFLOPS = 148 * 128 * 2 * 1.965e9 / 1e12     # FP32 FMA pipes at the max SM clock
 C_TABLE2 = {"cora": 0.24, "arxiv": 0.226, "arxiv_lstm": 0.226, "products": 0.411, "papers": 0.085}
 
 
@@ -195,13 +194,21 @@ def run_reference(args, cfg):
             times.append(dt)
             edges += sum(b["n_edges"] for b in blocks)
     v = edges / sum(times)
+    try:                     # the threads the oracle's BLAS calls used (the block builder is single-threaded C)
+        from threadpoolctl import threadpool_info
+        blas_threads = max([1] + [int(i.get("num_threads", 1)) for i in threadpool_info()])
+    except Exception:        # noqa: BLE001
+        blas_threads = 1
     line = dict(metric="aggregated edges/s (epoch of Buffalo hot path)", value=v, unit="edges/s",
                 n_gpus=0, steps=args.steps, warmup=args.warmup, ms_per_step=1e3 * statistics.mean(times),
                 higher_is_better=True, scaling="strong", vs_baseline=None, dtype="f64", data="synthetic",
                 impl="reference",
                 config={"workload": WORKLOADS[args.config], "sample": f"{len(part)} seeds per step"},
-                cpu_baseline=dict(value=v, unit="edges/s", kind="oracle", cores=len(os.sched_getaffinity(0)),
-                                  sample=f"per step one micro-batch of {len(part)} of {len(seeds)} seeds"),
+                cpu_baseline=dict(value=v, unit="edges/s", kind="oracle", cores=blas_threads,
+                                  sample=f"per step one micro-batch of {len(part)} of {len(seeds)} seeds: C block "
+                                         f"generation on 1 thread, float64 numpy/scipy layer math with BLAS on "
+                                         f"{blas_threads} thread(s) ({len(os.sched_getaffinity(0))} host cores "
+                                         f"available)"),
                 e2e=dict(value=v, unit="edges/s", h2d_bytes_per_step=0, d2h_bytes_per_step=0))
     print(json.dumps(line), flush=True)
 
@@ -668,13 +675,19 @@ def run_ours(args, cfg):
     # the first timed epoch, and one sequential epoch's phase breakdown + block-build rates
     mem_est = measured_memory(tr, args.warmup)
     phases, build_rates = phase_breakdown(tr, args.warmup)
-    if lstm:   # the LSTM path is bound by its fp32 SIMT gate GEMMs: FLOP roofline ("alu")
+    if lstm:   # the LSTM path is bound by its gate GEMMs (fp32 as 3xTF32 on tcgen05): FLOP roofline
         tf = g_bytes / (g_ms / 1e3) / 1e12 if g_ms > 0 else 0.0
-        roof = {"bound": "alu", "kernel": "k_gemm2_tc (LSTM gate GEMM of every step, fp32 as 3xTF32 mma.sync)",
-                "achieved": tf, "peak": FP32_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": tf / FP32_PEAK_TFLOPS,
-                "traffic": None,
-                "peak_source": "derived: 148 SMs x 128 FP32 FMA/clk x 2 flop x 1.965 GHz (no FP32 figure in "
-                               "B200_PROFILING.md); achieved counts useful fp32 flops (not the 3 TF32 passes)",
+        if os.path.exists(peaks_path):
+            bf = json.load(open(peaks_path))["bf16_tflops"]
+            src = "measured bf16 (MEASURED_PEAKS.json bf16_tflops)"
+        else:
+            bf, src = 2250.0, "nominal bf16 (B200_PROFILING.md)"
+        tpk = bf * (1.1 / 2.25) / 3.0      # tf32 = bf16 x the guide's 1.1 / 2.25 ratio; 3 TF32 products per fp32 one
+        roof = {"bound": "tensor",
+                "kernel": "k_tcf_gemm_tma (LSTM gate GEMMs of every step, fp32 as 3xTF32 on tcgen05 kind::tf32)",
+                "achieved": tf, "peak": tpk, "unit": "TFLOP/s", "frac": tf / tpk, "traffic": None,
+                "peak_source": src + " x 1.1/2.25 (tf32, B200_PROFILING.md nominal ratio) / 3 (hi*hi + hi*lo + "
+                               "lo*hi TF32 products per fp32 product); achieved counts useful fp32 flops",
                 "flops_per_launch": g_bytes / max(1, g_launches), "launch_ms": g_ms / max(1, g_launches),
                 "launches": g_launches, "share_of_step": g_ms / total_ms}
     else:
