@@ -840,6 +840,39 @@ __global__ void __launch_bounds__(256) k_mask_count(const int32_t* __restrict__ 
   __syncthreads();
   const int lane = threadIdx.x & 31;
   ItemCounters<W> cnt;
+  // Each thread adds its nodes' masks into bit-sliced counters (plane p holds bit p of the count
+  // of every item: a ripple-carry add of P word operations per node); every 2^P - 1 nodes, and
+  // at the end, the planes are reduced over the warp with one ballot per (plane, item bit).  The
+  // loop trip count is warp-uniform (threads past n_act add zero masks), so the flushes are too.
+  constexpr int P = W >= 4 ? 5 : 8;
+  constexpr int kFlush = (1 << P) - 1;
+  unsigned long long plane[P][W];
+#pragma unroll
+  for (int p = 0; p < P; ++p)
+#pragma unroll
+    for (int q = 0; q < W; ++q) plane[p][q] = 0ull;
+  int since = 0;
+  auto flush = [&]() {
+#pragma unroll
+    for (int q = 0; q < W; ++q)
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int p = 0; p < P; ++p) {
+          const unsigned word = (unsigned)(plane[p][q] >> (32 * h));
+          if (__any_sync(0xffffffffu, word != 0u)) {
+#pragma unroll
+            for (int k = 0; k < 32; ++k) {
+              const unsigned b = __ballot_sync(0xffffffffu, (word >> k) & 1u);
+              if (lane == k) cnt.n[2 * q + h] += (uint32_t)__popc(b) << p;
+            }
+          }
+        }
+#pragma unroll
+    for (int p = 0; p < P; ++p)
+#pragma unroll
+      for (int q = 0; q < W; ++q) plane[p][q] = 0ull;
+  };
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i0 = blockIdx.x * (int64_t)blockDim.x; i0 < n_act; i0 += stride) {
     const int64_t i = i0 + threadIdx.x;
@@ -856,17 +889,25 @@ __global__ void __launch_bounds__(256) k_mask_count(const int32_t* __restrict__ 
     }
     if (gn) {
 #pragma unroll
-      for (int j = 0; j < 2 * W; ++j) {
-        const unsigned word = (unsigned)(mask[j >> 1] >> (32 * (j & 1)));
+      for (int q = 0; q < W; ++q) {
+        unsigned long long c = mask[q];
 #pragma unroll
-        for (int k = 0; k < 32; ++k) {
-          const unsigned b = __ballot_sync(0xffffffffu, (word >> k) & 1u);
-          if (lane == k) cnt.n[j] += __popc(b);
+        for (int p = 0; p < P; ++p) {
+          const unsigned long long t = plane[p][q] & c;
+          plane[p][q] ^= c;
+          c = t;
         }
+      }
+      if (++since == kFlush) {
+        flush();
+        since = 0;
       }
     }
   }
-  if (gn) flush_item_counters<W>(cnt, gn, nullptr, sn, nullptr);
+  if (gn) {
+    flush();
+    flush_item_counters<W>(cnt, gn, nullptr, sn, nullptr);
+  }
 }
 
 constexpr int kMaskMaxItems = 256;
