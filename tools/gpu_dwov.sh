@@ -1,4 +1,4 @@
-# A/B: heavy-row backward kernel on a side stream (main) vs on the caller's stream (ndo)
+# A/B: dW chain on side stream 1 (main) vs on the caller stream (ndo)
 python -c "import __graft_entry__ as g; g.build()"
 timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_determinism.py tests/test_gpu_edges.py -x -q -p no:cacheprovider 2>&1 | tail -2
 for v in main ndo main ndo; do
