@@ -311,7 +311,11 @@ BUFFALO_API size_t buffalo_sage_bwd_scratch_bytes(const buffalo_block* blk, int3
  * over the n_src rows with the layer-below epilogue fused: ReLU' with h_src = H_{l-1}, bf16
  * dZ_{l-1} into dh_src and its column-sum partials, i.e. dh_src receives the same prepared form
  * of layer l-1 and must hold R(2 n_src p(d_{l-1})) + R(4 * 888 * d_{l-1}) bytes.
- * Pass dh_src = NULL for layer 1 (features are not trained). */
+ * Pass dh_src = NULL for layer 1 (features are not trained).
+ * Streams: in BF16 mode the layer's dW / db reductions and the long-tail rows of the transposed
+ * Aggregate run on two library-owned non-blocking side streams (one pair per device, created
+ * on first use), forked from and joined back into `stream` with events before the call returns:
+ * the call stays ordered on `stream` for the caller (and for CUDA graph capture). */
 BUFFALO_API buffalo_status buffalo_sage_bwd(const buffalo_block* blk, int32_t layer, const buffalo_model* m,
                                 float* dh_dst, int64_t ld_dh, const void* h_src, int64_t ld_src,
                                 const void* saved_agg, int64_t ld_agg, const void* h_dst,
