@@ -119,17 +119,36 @@ __global__ void __launch_bounds__(256) k_cache_fill(const int32_t* __restrict__ 
                                                     const int32_t* __restrict__ cache, int32_t f,
                                                     const int32_t* __restrict__ row_ptr, int32_t* __restrict__ out,
                                                     int64_t cap, MarkCtx mk) {
-  constexpr int G = 32 / SEG;
+  // kR rows per lane group and iteration: their row_ptr / dst -> cache row -> node map chains
+  // are in flight together (one chain per iteration left the kernel latency-bound)
+  constexpr int G = 32 / SEG, kR = 4;
   const int lane = threadIdx.x & 31, g = lane / SEG, sl = lane % SEG;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n; w += warps) {
-    const int64_t slot = w * G + g;
-    if (slot >= n) continue;
-    const int32_t b = row_ptr[slot], D = row_ptr[slot + 1] - b;
-    if (sl < D && b + sl < cap) {
-      const int32_t u = cache[(int64_t)dst[slot] * f + sl];
-      out[b + sl] = u;
-      mk(b + sl, u);
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n; w += kR * warps) {
+    int32_t b[kR], u[kR], mm[kR];
+#pragma unroll
+    for (int r = 0; r < kR; ++r) {
+      const int64_t slot = (w + r * warps) * G + g;
+      u[r] = -1;
+      b[r] = 0;
+      if (slot < n) {
+        b[r] = __ldg(row_ptr + slot);
+        const int32_t D = __ldg(row_ptr + slot + 1) - b[r];
+        if (sl < D && b[r] + sl < cap) u[r] = __ldg(cache + (int64_t)__ldg(dst + slot) * f + sl);
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < kR; ++r) mm[r] = (u[r] >= 0 && mk.mapped) ? __ldg(mk.node_map + u[r]) : 0;
+#pragma unroll
+    for (int r = 0; r < kR; ++r) {
+      if (u[r] < 0) continue;
+      const int64_t pos = (int64_t)b[r] + sl;
+      out[pos] = u[r];
+      if (!mk.mapped) continue;
+      mk.mapped[pos] = mm[r];
+      if (mm[r] != INT32_MAX) continue;                            // a dst: keeps its prefix id
+      const uint32_t bit = 1u << (u[r] & 31);
+      if (!(mk.bits[u[r] >> 5] & bit)) atomicOr(&mk.bits[u[r] >> 5], bit);
     }
   }
 }
@@ -188,12 +207,38 @@ __global__ void k_emit_bits(const uint32_t* __restrict__ bits, const int32_t* __
 __global__ void k_col_local(const int32_t* __restrict__ colg, int64_t e, const int32_t* __restrict__ node_map,
                             const uint32_t* __restrict__ bits, const int32_t* __restrict__ prefix, int32_t n_dst,
                             int32_t* __restrict__ col_local, int32_t* __restrict__ tcnt) {
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < e; k += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t u = colg[k];
-    const int32_t m = col_local[k];                              // node_map[u], kept by k_mark_bits
-    const int32_t c = m != INT32_MAX ? m : n_dst + prefix[u >> 5] + __popc(bits[u >> 5] & ((1u << (u & 31)) - 1u));
-    col_local[k] = c;
-    if (tcnt) atomicAdd(&tcnt[c], 1);
+  // kR edges per thread and iteration (coalesced per r): their bitmap / prefix lookups in flight together
+  constexpr int kR = 4;
+  (void)node_map;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x * kR;
+  for (int64_t k0 = blockIdx.x * (int64_t)blockDim.x * kR + threadIdx.x; k0 < e; k0 += stride) {
+    int32_t u[kR], m[kR], c[kR];
+#pragma unroll
+    for (int r = 0; r < kR; ++r) {
+      const int64_t k = k0 + (int64_t)r * blockDim.x;
+      u[r] = -1;
+      m[r] = 0;
+      if (k < e) {
+        u[r] = __ldg(colg + k);
+        m[r] = col_local[k];                                    // node_map[u], kept by the fill
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < kR; ++r) {
+      c[r] = m[r];
+      if (u[r] >= 0 && m[r] == INT32_MAX) {
+        const int32_t w = u[r] >> 5;
+        c[r] = n_dst + __ldg(prefix + w) + __popc(__ldg(bits + w) & ((1u << (u[r] & 31)) - 1u));
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < kR; ++r) {
+      const int64_t k = k0 + (int64_t)r * blockDim.x;
+      if (k < e) {
+        col_local[k] = c[r];
+        if (tcnt) atomicAdd(&tcnt[c[r]], 1);
+      }
+    }
   }
 }
 
