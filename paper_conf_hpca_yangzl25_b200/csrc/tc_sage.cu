@@ -1277,37 +1277,15 @@ __global__ void __launch_bounds__(kDwThreads) k_tc_dw(const TcDwParams p) {
 // dW[m][n] += sum_s part[s][m][n'(n)] in split order (deterministic).
 __global__ void k_reduce_dw(const float* __restrict__ part, int S, int d_out, int d_in, int Dp,
                             float* __restrict__ dW) {
+  // thread per dW element, the S partials summed in split order (coalesced over the columns;
+  // a float4-per-thread variant had 4x fewer loads in flight and measured slower)
   const int64_t total = (int64_t)d_out * 2 * d_in;
   const int64_t K2 = 2 * (int64_t)Dp;
-  const int64_t stride = (int64_t)d_out * K2;
-  if ((d_in & 3) == 0 && (reinterpret_cast<uintptr_t>(dW) & 15) == 0) {
-    // four consecutive columns per thread (16-B loads; a quad never straddles the two halves);
-    // each column still sums its S partials in split order
-    for (int64_t t4 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t4 * 4 < total;
-         t4 += (int64_t)gridDim.x * blockDim.x) {
-      const int64_t t = t4 * 4;
-      const int m = (int)(t / (2 * d_in)), n = (int)(t % (2 * d_in));
-      const int np = n < d_in ? n : Dp + (n - d_in);
-      const float* p0 = part + (int64_t)m * K2 + np;
-      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-#pragma unroll 8
-      for (int q = 0; q < S; ++q) {
-        const float4 v = __ldg(reinterpret_cast<const float4*>(p0 + q * stride));
-        acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
-      }
-      float4* o = reinterpret_cast<float4*>(dW + t);
-      float4 w = *o;
-      w.x += acc.x; w.y += acc.y; w.z += acc.z; w.w += acc.w;
-      *o = w;
-    }
-    return;
-  }
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
     const int m = (int)(t / (2 * d_in)), n = (int)(t % (2 * d_in));
     const int np = n < d_in ? n : Dp + (n - d_in);
     float acc = 0.f;
-#pragma unroll 8
-    for (int q = 0; q < S; ++q) acc += part[(int64_t)q * stride + (int64_t)m * K2 + np];
+    for (int q = 0; q < S; ++q) acc += part[(int64_t)q * d_out * K2 + (int64_t)m * K2 + np];
     dW[t] += acc;
   }
 }
@@ -1500,8 +1478,7 @@ buffalo_status tc_sage_bwd(const BwdArgs& a, cudaStream_t s) {
     k_tc_dw<float><<<grid, kDwThreads, smem, s>>>(w);
     BF_LAUNCHED("k_tc_dw");
   }
-  k_reduce_dw<<<grid_for(ceil_div((int64_t)d_out * 2 * d_in, 4), 256), 256, 0, s>>>(dw_part, S, d_out, d_in,
-                                                                                  (int)Dp, a.dW);
+  k_reduce_dw<<<grid_for((int64_t)d_out * 2 * d_in, 256), 256, 0, s>>>(dw_part, S, d_out, d_in, (int)Dp, a.dW);
   BF_LAUNCHED("k_reduce_dw");
   k_reduce_db<<<(unsigned)ceil_div(d_out, 32), 1024, 0, s>>>(db_part, nparts, d_out, a.db);
   BF_LAUNCHED("k_reduce_db");
