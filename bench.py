@@ -396,11 +396,28 @@ class AllgatherReplay:
         return 0
 
 
+def record_allgathers(rep, run_rank):
+    """The all-gather results of one deterministic computation run by each of rep.world ranks:
+    call i's result is assembled from every rank's rows at call i, each rank replaying calls
+    0..i-1 (run_rank(r) runs rank r's computation with rep.fn as its all-gather and returns
+    whether it completed); repeated until the runs complete.  Returns the results in call order."""
+    R = []
+    while True:
+        rows = [None] * rep.world
+        for r in range(rep.world):
+            rep.rank, rep.results, rep.i, rep.record = r, R, 0, rows
+            run_rank(r)
+        done = [x is None for x in rows]
+        assert all(done) or not any(done), "simulated ranks disagree on the number of all-gathers"
+        if all(done):
+            rep.record = None
+            return R
+        R.append(b"".join(rows))
+
+
 def record_shared_stats(tr, rep, epochs):
-    """The all-gather results of the scheduler runs of `epochs` for the N simulated ranks
-    (untimed): call i's result is assembled from every rank's rows at call i, each rank replaying
-    calls 0..i-1; repeated until the runs complete.  Returns the results in the order a pipelined
-    Trainer asks for them (one schedule per epoch, ascending)."""
+    """record_allgathers of the scheduler runs of `epochs` for the N simulated ranks (untimed),
+    in the order a pipelined Trainer asks for them (one schedule per epoch, ascending)."""
     import torch
     from paper_conf_hpca_yangzl25_b200 import buffalo as B
     from paper_conf_hpca_yangzl25_b200.train import PlanBuffers
@@ -408,25 +425,15 @@ def record_shared_stats(tr, rep, epochs):
     s = tr.sched
     out = []
     for e in epochs:
-        R = []
-        while True:
-            rows = [None] * rep.world
-            for r in range(rep.world):
-                rep.rank, rep.results, rep.i, rep.record = r, R, 0, rows
-                sched = B.make_sched(s.mem_budget, s.C_ppm, s.k_min, s.k_max, rep.world, s.k_multiple, r, rep.fn)
-                sp = B.make_sampler(tr.fanout, tr.F, tr.base_seed + e)
-                try:
-                    B.bucketize(tr.graph.g_sched, tr._seeds[0], sp, tr.model, sched, pb.plan, tr.bucket_ws)
-                except B.BuffaloError:
-                    pass
-                torch.cuda.synchronize()
-            done = [x is None for x in rows]
-            assert all(done) or not any(done), "simulated ranks disagree on the number of all-gathers"
-            if all(done):
-                break
-            R.append(b"".join(rows))
-        out.extend(R)
-    rep.record = None
+        def run_rank(r):
+            sched = B.make_sched(s.mem_budget, s.C_ppm, s.k_min, s.k_max, rep.world, s.k_multiple, r, rep.fn)
+            sp = B.make_sampler(tr.fanout, tr.F, tr.base_seed + e)
+            try:
+                B.bucketize(tr.graph.g_sched, tr._seeds[0], sp, tr.model, sched, pb.plan, tr.bucket_ws)
+            except B.BuffaloError:
+                pass
+            torch.cuda.synchronize()
+        out.extend(record_allgathers(rep, run_rank))
     return out
 
 
