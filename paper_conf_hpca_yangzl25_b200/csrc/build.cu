@@ -209,7 +209,7 @@ __global__ void k_col_local(const int32_t* __restrict__ colg, int64_t e, const i
                             int32_t* __restrict__ col_local, int32_t* __restrict__ tcnt) {
   // kR edges per thread and iteration (coalesced per r): their bitmap / prefix lookups in flight together
   constexpr int kR = 4;
-  (void)node_map;
+  (void)node_map;                        // looked up by the fill already (col_local holds node_map[u])
   const int64_t stride = (int64_t)gridDim.x * blockDim.x * kR;
   for (int64_t k0 = blockIdx.x * (int64_t)blockDim.x * kR + threadIdx.x; k0 < e; k0 += stride) {
     int32_t u[kR], m[kR], c[kR];

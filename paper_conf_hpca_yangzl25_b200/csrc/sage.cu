@@ -1814,7 +1814,9 @@ static buffalo_status gat_bwd_t(const GatArgs& a, cudaStream_t st) {
   }
   BF_LAUNCHED("k_gat_src_bwd");
   // da_l = d_el^T Z, da_r = d_er^T Z[:n_dst], dW = dZ^T H (deterministic split reductions)
-  // (weighted column sums of Z over fixed row splits: one coalesced pass per vector)
+  // (weighted column sums of Z over fixed row splits: one coalesced pass per vector; the dal_b /
+  // dar_b slots of the scratch layout, R30, held the 1-row products' bias partials and stay
+  // unused)
   (void)dal_b;
   (void)dar_b;
   k_colsum_partial<<<dim3((unsigned)ceil_div(dl, 32), (unsigned)Sl), 256, 0, st>>>(v.Z, ldz, ns, dl, ceil_div(ns, Sl),
