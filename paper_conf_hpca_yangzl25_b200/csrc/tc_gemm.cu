@@ -147,6 +147,11 @@ constexpr int kProducers = 2;
 constexpr int kMmaWarp = kEpiWarps + kProducers;
 constexpr int kGemmThreads = (kEpiWarps + kProducers + 1) * 32;
 
+// 2-KB TMA-store staging boxes per epilogue warp: one (the warp waits for its previous store to
+// have read the box) leaves 16 KB more for the A-operand pipeline — one more stage for the
+// layer-1 Update with resident weights; measured 0.4 ms per products epoch faster than two
+constexpr int kStageBufs = 1;
+
 struct GemmParams {
   int64_t n_rows;
   int64_t self_tiles;         // tiles t >= self_tiles have no self rows: their self K-chunks are skipped
@@ -160,7 +165,7 @@ struct GemmParams {
   // the pipeline stages carry A tiles only; with nsplit = 2 the two CTAs of a tile set compute
   // the two column halves of the same tiles (A is read twice, the second time from L2).
   int w_res, nsplit, Nsub;
-  int stage_off, stage_bytes; // epilogue staging area (8 warps x 2 x 2 KB)
+  int stage_off, stage_bytes; // epilogue staging area (8 warps x kStageBufs x 2 KB)
   const float* bias;
   int relu, out_f32;
   const int32_t* scale_rp;    // non-null: output row i is scaled by 1 / D(i), D(i) = rp[i+1] - rp[i] (0 if D = 0)
@@ -283,7 +288,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     // store.  The next TMEM load is issued before the current group's math.
     const int q = warp & 3, h = warp >> 2;
     float* sbias = reinterpret_cast<float*>(tmem_slot + 4);   // 16-B aligned
-    uint8_t* stg = smem + p.stage_off + warp * 4096;          // this warp's two 2-KB staging boxes
+    uint8_t* stg = smem + p.stage_off + warp * (2048 * kStageBufs);   // this warp's 2-KB staging box(es)
     int sbuf = 0;
     for (int c = threadIdx.x; c < p.Nsub; c += kEpiWarps * 32)
       sbias[c] = (p.bias && col_base + c < p.d_out) ? __ldg(p.bias + col_base + c) : 0.f;
@@ -343,8 +348,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             // bf16 rows through a staging box and one TMA store per warp and column group
             // (coalesced, asynchronous; rows past n_rows are clipped by the map)
             uint8_t* box = stg + sbuf * 2048;
-            sbuf ^= 1;
-            if (lane == 0) bulk_wait_read<1>();       // the store that used this box has read it
+            sbuf = (sbuf + 1) % kStageBufs;
+            if (lane == 0) bulk_wait_read<kStageBufs - 1>();   // the store that used this box has read it
             __syncwarp();
 #pragma unroll
             for (int k = 0; k < 4; ++k)
@@ -621,7 +626,7 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   // resident weights when all weight chunks fit next to >= 4 A stages and the store staging
   // (a CTA-pair column split, nsplit = 2, is supported by the kernel but measured slower)
   const int64_t w_all = (int64_t)p.nkc * p.Np * 128;
-  const int64_t kStaging = kEpiWarps * 4096;
+  const int64_t kStaging = kEpiWarps * 2048 * kStageBufs;
   const int misc = 16 * 8 + 48 + 4 * p.Np + 1024;                    // barriers, slot, bias, alignment
   p.nsplit = 1;
   p.w_res = (227 * 1024 - w_all - kStaging - misc) / kChunkA >= 4 ? 1 : 0;

@@ -1,0 +1,11 @@
+# A/B: Update/dH GEMM epilogue with 2 staging boxes per warp (main) vs 1 (st1)
+python -c "import __graft_entry__ as g; g.build()"
+timeout 900 BUFFALO_LIB=tools/exp/libbuffalo_st1.so python -m pytest tests/test_gpu_parity.py tests/test_gpu_edges.py tests/test_gpu_sharded.py tests/test_gpu_determinism.py tests/test_gpu_pipeline.py -x -q -p no:cacheprovider 2>&1 | tail -2
+for v in main st1 main st1; do
+  if [ $v = main ]; then L=""; else L="tools/exp/libbuffalo_$v.so"; fi
+  BUFFALO_LIB=$L timeout 600 python bench.py --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/st_$v.json 2> gpurun_out/st_$v.err
+  python -c "
+import json; d=json.load(open('gpurun_out/st_$v.json')); c=d['config']
+print('$v', round(d['ms_per_step'],2), 'frac', round(d['roofline']['frac'],3), c['phases_ms_sequential'])" || tail -3 gpurun_out/st_$v.err
+done
+timeout 1200 python -m pytest tests/test_gpu_fullsize.py -x -q -p no:cacheprovider -k products 2>&1 | tail -2
