@@ -100,6 +100,7 @@ __global__ void __launch_bounds__(256) k_sample_fill(const int32_t* __restrict__
                                                      uint32_t hop, uint64_t seed,
                                                      const int32_t* __restrict__ row_ptr,
                                                      int32_t* __restrict__ out, int64_t cap, MarkCtx mk) {
+  pdl_wait();
   constexpr int G = 32 / SEG;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
   for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w * G < n; w += warps)
@@ -119,6 +120,7 @@ __global__ void __launch_bounds__(256) k_cache_fill(const int32_t* __restrict__ 
                                                     const int32_t* __restrict__ cache, int32_t f,
                                                     const int32_t* __restrict__ row_ptr, int32_t* __restrict__ out,
                                                     int64_t cap, MarkCtx mk) {
+  pdl_wait();
   // kR rows per lane group and iteration: their row_ptr / dst -> cache row -> node map chains
   // are in flight together (one chain per iteration left the kernel latency-bound)
   constexpr int G = 32 / SEG, kR = 4;
@@ -159,9 +161,9 @@ template <class... Args>
 static void launch_sample_fill(int seg, int64_t n, cudaStream_t s, Args... args) {
   const int G = 32 / seg;
   const int grid = grid_for(ceil_div(n, G) * 32, 256, 16);
-  if (seg == 8) k_sample_fill<8><<<grid, 256, 0, s>>>(args...);
-  else if (seg == 16) k_sample_fill<16><<<grid, 256, 0, s>>>(args...);
-  else k_sample_fill<32><<<grid, 256, 0, s>>>(args...);
+  if (seg == 8) launch_pdl(k_sample_fill<8>, dim3(grid), dim3(256), 0, s, args...);
+  else if (seg == 16) launch_pdl(k_sample_fill<16>, dim3(grid), dim3(256), 0, s, args...);
+  else launch_pdl(k_sample_fill<32>, dim3(grid), dim3(256), 0, s, args...);
 }
 
 // ------------------------------------------------------------------ a5: relabel
@@ -170,10 +172,12 @@ static void launch_sample_fill(int seg, int64_t n, cudaStream_t s, Args... args)
 // exclusive popcount scan over its words gives each word's first local id, so that
 // local(u) = n_dst + prefix[u / 32] + popc(bits[u / 32] & below(u % 32)).
 __global__ void k_set_map(const int32_t* __restrict__ src, int64_t n, int32_t* __restrict__ node_map) {
+  pdl_wait();
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
     node_map[src[j]] = (int32_t)j;
 }
 __global__ void k_reset_map(const int32_t* __restrict__ src, int64_t n, int32_t* __restrict__ node_map) {
+  pdl_wait();
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
     node_map[src[j]] = INT32_MAX;
 }
@@ -191,6 +195,7 @@ struct StorePrefix {
 // The marked nodes appended to src (at src + n_dst) in ascending id: thread per bitmap word.
 __global__ void k_emit_bits(const uint32_t* __restrict__ bits, const int32_t* __restrict__ prefix, int64_t words,
                             int32_t* __restrict__ src, int64_t cap) {
+  pdl_wait();
   for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < words; w += (int64_t)gridDim.x * blockDim.x) {
     uint32_t m = bits[w];
     int32_t r = m ? prefix[w] : 0;
@@ -207,6 +212,7 @@ __global__ void k_emit_bits(const uint32_t* __restrict__ bits, const int32_t* __
 __global__ void k_col_local(const int32_t* __restrict__ colg, int64_t e, const int32_t* __restrict__ node_map,
                             const uint32_t* __restrict__ bits, const int32_t* __restrict__ prefix, int32_t n_dst,
                             int32_t* __restrict__ col_local, int32_t* __restrict__ tcnt) {
+  pdl_wait();
   // kR edges per thread and iteration (coalesced per r): their bitmap / prefix lookups in flight together
   constexpr int kR = 4;
   (void)node_map;                        // looked up by the fill already (col_local holds node_map[u])
@@ -268,6 +274,7 @@ struct EmitPerm {
 // Transposed fill: edge (i -> col_local[e]) lands at an atomic cursor of its src row.
 __global__ void __launch_bounds__(256) k_tfill(const int32_t* __restrict__ rp, const int32_t* __restrict__ col_local,
                                                int64_t n, int32_t* __restrict__ cursor, int32_t* __restrict__ tcol) {
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
   for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n; i += warps)
@@ -309,6 +316,7 @@ __device__ __forceinline__ void tsort_segment(const int32_t* __restrict__ trp, i
 __global__ void __launch_bounds__(256) k_tsort_banded(const int32_t* __restrict__ perm, const int32_t* __restrict__ trp,
                                                       int32_t* __restrict__ tcol, const int32_t* __restrict__ cls_off,
                                                       int64_t ntiles) {
+  pdl_wait();
   const int64_t sA = cls_off[2 * ntiles], sB = cls_off[9 * ntiles], sC = cls_off[17 * ntiles];
   const int64_t sH = cls_off[(kHeavyT + 1) * ntiles];
   const int64_t wA = (sB - sA + 3) / 4, wB = (sC - sB + 1) / 2, wC = sH - sC;
@@ -332,6 +340,7 @@ __global__ void __launch_bounds__(256) k_tsort_banded(const int32_t* __restrict_
 __global__ void __launch_bounds__(256) k_tsort_heavy(const int32_t* __restrict__ perm, int64_t n,
                                                      const int32_t* __restrict__ trp,
                                                      int32_t* __restrict__ tcol, int32_t* __restrict__ stage) {
+  pdl_wait();
   for (int64_t hh = blockIdx.x; hh < n; hh += gridDim.x) {
   const int32_t j = perm[n - 1 - hh];          // heavy rows: the tail of the degree-class perm
   const int32_t b = trp[j], len = trp[j + 1] - b;
@@ -354,6 +363,7 @@ constexpr int kBitsortMaxWords = 40 * 1024;      // 160 KB of shared memory (n_d
 __global__ void __launch_bounds__(256) k_tsort_heavy_bits(const int32_t* __restrict__ perm, int64_t n,
                                                           const int32_t* __restrict__ trp,
                                                           int32_t* __restrict__ tcol, int32_t words) {
+  pdl_wait();
   extern __shared__ uint32_t bm[];
   __shared__ int32_t sw[33];
   const int per = (words + blockDim.x - 1) / blockDim.x;
@@ -466,16 +476,16 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   // the node map first so that the fill marks the other neighbours in the bitmap as it writes
   const GraphWs gw = graph_ws(g);
   if (n_dst > 0) {
-    k_set_map<<<grid_for(n_dst, 256), 256, 0, s>>>(dst, n_dst, g->node_map);
+    launch_pdl(k_set_map, dim3(grid_for(n_dst, 256)), dim3(256), 0, s, dst, n_dst, g->node_map);
     BF_LAUNCHED("k_set_map");
   }
   const MarkCtx mk{g->node_map, gw.bits, col_local};
   if (n_dst > 0 && cache && f > 0) {                             // rows sampled by the scheduler
     const int seg = sample_seg(f), G = 32 / seg;
     const int grid = grid_for(ceil_div(n_dst, G) * 32, 256, 16);
-    if (seg == 8) k_cache_fill<8><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e, mk);
-    else if (seg == 16) k_cache_fill<16><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e, mk);
-    else k_cache_fill<32><<<grid, 256, 0, s>>>(dst, n_dst, cache, f, (const int32_t*)rp, colg, e, mk);
+    if (seg == 8) launch_pdl(k_cache_fill<8>, dim3(grid), dim3(256), 0, s, dst, n_dst, cache, f, (const int32_t*)rp, colg, e, mk);
+    else if (seg == 16) launch_pdl(k_cache_fill<16>, dim3(grid), dim3(256), 0, s, dst, n_dst, cache, f, (const int32_t*)rp, colg, e, mk);
+    else launch_pdl(k_cache_fill<32>, dim3(grid), dim3(256), 0, s, dst, n_dst, cache, f, (const int32_t*)rp, colg, e, mk);
     BF_LAUNCHED("k_cache_fill");
   } else if (n_dst > 0) {
     launch_sample_fill(sample_seg(f), n_dst, s, dst, n_dst, g->row_ptr, g->col, f, hop, seed, (const int32_t*)rp,
@@ -495,7 +505,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   // from here on the graph workspace is dirty: an early return must restore it
   auto restore_ws = [&]() -> buffalo_status {
     if (n_dst > 0) {
-      k_reset_map<<<grid_for(n_dst, 256), 256, 0, s>>>(dst, n_dst, g->node_map);
+      launch_pdl(k_reset_map, dim3(grid_for(n_dst, 256)), dim3(256), 0, s, dst, n_dst, g->node_map);
       BF_LAUNCHED("k_reset_map");
     }
     BF_CUDA(cudaMemsetAsync(gw.bits, 0, sizeof(uint32_t) * gw.words, s));
@@ -508,7 +518,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   }
   if (n_dst > 0) BF_CUDA(cudaMemcpyAsync(src, dst, sizeof(int32_t) * n_dst, cudaMemcpyDeviceToDevice, s));
   BF_CHECK(device_scan(PopcWord{gw.bits}, StorePrefix{gw.prefix}, gw.words, gw.scan_ws, totals + 2, s));
-  k_emit_bits<<<grid_for(gw.words, 256), 256, 0, s>>>(gw.bits, gw.prefix, gw.words, src + n_dst, n_src - n_dst);
+  launch_pdl(k_emit_bits, dim3(grid_for(gw.words, 256)), dim3(256), 0, s, gw.bits, gw.prefix, gw.words, src + n_dst, n_src - n_dst);
   BF_LAUNCHED("k_emit_bits");
   blk->n_src = n_src;
   blk->src_global = src;
@@ -527,7 +537,7 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
   }
   if (!sizes_only) {
     if (e > 0) {
-      k_col_local<<<grid_for(e, 256), 256, 0, s>>>(colg, e, g->node_map, gw.bits, gw.prefix, (int32_t)n_dst,
+      launch_pdl(k_col_local, dim3(grid_for(e, 256)), dim3(256), 0, s, colg, e, g->node_map, gw.bits, gw.prefix, (int32_t)n_dst,
                                                    col_local, trp);
       BF_LAUNCHED("k_col_local");
     }
@@ -553,10 +563,10 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
     }
     if (e > 0) {
       BF_CUDA(cudaMemcpyAsync(cursor, trp, sizeof(int32_t) * n_src, cudaMemcpyDeviceToDevice, s));
-      k_tfill<<<grid_for(n_dst * 32, 256, 16), 256, 0, s>>>(rp, col_local, n_dst, cursor, tcol);
+      launch_pdl(k_tfill, dim3(grid_for(n_dst * 32, 256, 16)), dim3(256), 0, s, rp, col_local, n_dst, cursor, tcol);
       BF_LAUNCHED("k_tfill");
       if (n_src > 0) {
-        k_tsort_banded<<<grid_for(n_src * 8, 256, 16), 256, 0, s>>>(tperm, trp, tcol, counts, part_tiles(n_src));
+        launch_pdl(k_tsort_banded, dim3(grid_for(n_src * 8, 256, 16)), dim3(256), 0, s, tperm, trp, tcol, counts, part_tiles(n_src));
         BF_LAUNCHED("k_tsort_banded");
       }
       const int hg = heavy_tail_grid(nht, e);
@@ -564,10 +574,10 @@ buffalo_status build_layer(const buffalo_graph* g, const int32_t* dst, int64_t n
         const int64_t words = ceil_div(n_dst, 32);
         if (words <= kBitsortMaxWords) {
           BF_CHECK(set_max_smem_once<k_tsort_heavy_bits>(kBitsortMaxWords * 4));
-          k_tsort_heavy_bits<<<hg, 256, words * 4, s>>>(tperm, n_src, trp, tcol, (int32_t)words);
+          launch_pdl(k_tsort_heavy_bits, dim3(hg), dim3(256), words * 4, s, tperm, n_src, trp, tcol, (int32_t)words);
           BF_LAUNCHED("k_tsort_heavy_bits");
         } else {
-          k_tsort_heavy<<<hg, 256, 0, s>>>(tperm, n_src, trp, tcol, cursor);
+          launch_pdl(k_tsort_heavy, dim3(hg), dim3(256), 0, s, tperm, n_src, trp, tcol, cursor);
           BF_LAUNCHED("k_tsort_heavy");
         }
       }

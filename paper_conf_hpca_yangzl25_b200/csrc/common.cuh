@@ -116,6 +116,28 @@ struct SideFork {
   SideFork& operator=(const SideFork&) = delete;
 };
 
+// Programmatic dependent launch for the block build's chains of small kernels: a kernel launched
+// with launch_pdl may be scheduled while its predecessor on the stream drains, and waits at its
+// top (pdl_wait: griddepcontrol.wait, a no-op for a normal launch) until that grid has completed
+// and its memory is visible — semantics of a plain launch, minus the launch gap.  Every kernel
+// passed to launch_pdl must call pdl_wait() before touching global memory.
+constexpr bool kPdl = true;
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+template <typename... KArgs, typename... Args>
+inline void launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = kPdl ? 1 : 0;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  cudaLaunchKernelEx(&cfg, k, args...);
+}
+
 // sm_100a check of the current device.
 buffalo_status require_sm100();
 

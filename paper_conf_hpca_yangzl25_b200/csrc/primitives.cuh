@@ -52,6 +52,7 @@ template <class Load, class Store>
 __global__ void __launch_bounds__(kScanThreads) k_scan_lookback(Load ld, Store st, int64_t n,
                                                                 unsigned long long* status,
                                                                 unsigned int* counter, int32_t* total_out) {
+  pdl_wait();
   __shared__ int32_t sv[kScanTile + kScanTile / 32];
   __shared__ int32_t sx[kScanTile + kScanTile / 32];
   __shared__ int32_t sw[33];
@@ -126,7 +127,8 @@ buffalo_status device_scan(Load ld, Store st, int64_t n, int32_t* ws, int32_t* t
   BF_CUDA(cudaMemsetAsync(ws, 0, sizeof(unsigned long long) * (ntiles + 1), s));
   unsigned long long* status = reinterpret_cast<unsigned long long*>(ws);
   unsigned int* counter = reinterpret_cast<unsigned int*>(status + ntiles);
-  k_scan_lookback<<<(unsigned)ntiles, kScanThreads, 0, s>>>(ld, st, n, status, counter, total_out);
+  launch_pdl(k_scan_lookback<Load, Store>, dim3((unsigned)ntiles), dim3(kScanThreads), 0, s, ld, st, n, status, counter,
+             total_out);
   BF_LAUNCHED("k_scan_lookback");
   return BUFFALO_OK;
 }
@@ -134,6 +136,7 @@ buffalo_status device_scan(Load ld, Store st, int64_t n, int32_t* ws, int32_t* t
 // Integer count (sum of a 0/1 or small functor) over [0, n) into *total (zeroed first).
 template <class Load>
 __global__ void __launch_bounds__(256) k_count_sum(Load ld, int64_t n, int32_t* total) {
+  pdl_wait();
   int32_t s = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     s += ld(i);
@@ -145,7 +148,7 @@ template <class Load>
 buffalo_status device_count(Load ld, int64_t n, int32_t* total, cudaStream_t s) {
   BF_CUDA(cudaMemsetAsync(total, 0, sizeof(int32_t), s));
   if (n <= 0) return BUFFALO_OK;
-  k_count_sum<<<grid_for(n, 256), 256, 0, s>>>(ld, n, total);
+  launch_pdl(k_count_sum<Load>, dim3(grid_for(n, 256)), dim3(256), 0, s, ld, n, total);
   BF_LAUNCHED("k_count_sum");
   return BUFFALO_OK;
 }
@@ -176,6 +179,7 @@ inline int64_t part_count_elems(int64_t n) { return 256 * part_tiles(n); }
 template <class Key>
 __global__ void __launch_bounds__(kPartThreads) k_part_hist(Key key, int64_t n, int32_t* counts,
                                                             int64_t ntiles) {
+  pdl_wait();
   __shared__ int32_t h[256];
   if (threadIdx.x < 256) h[threadIdx.x] = 0;
   __syncthreads();
@@ -192,6 +196,7 @@ __global__ void __launch_bounds__(kPartThreads) k_part_hist(Key key, int64_t n, 
 template <class Key, class Emit>
 __global__ void __launch_bounds__(kPartThreads) k_part_scatter(Key key, Emit emit, int64_t n,
                                                                const int32_t* offsets, int64_t ntiles) {
+  pdl_wait();
   constexpr int NW = kPartThreads / 32;
   __shared__ int32_t base[256];
   __shared__ int32_t wcnt[NW][256];
@@ -230,10 +235,10 @@ buffalo_status stable_partition(Key key, Emit emit, int64_t n, int32_t* counts, 
                                 cudaStream_t s) {
   if (n <= 0) return BUFFALO_OK;
   int64_t nt = part_tiles(n);
-  k_part_hist<<<(unsigned)nt, kPartThreads, 0, s>>>(key, n, counts, nt);
+  launch_pdl(k_part_hist<Key>, dim3((unsigned)nt), dim3(kPartThreads), 0, s, key, n, counts, nt);
   BF_LAUNCHED("k_part_hist");
   BF_CHECK(scan_inplace(counts, 256 * nt, scan_ws, s));
-  k_part_scatter<<<(unsigned)nt, kPartThreads, 0, s>>>(key, emit, n, counts, nt);
+  launch_pdl(k_part_scatter<Key, Emit>, dim3((unsigned)nt), dim3(kPartThreads), 0, s, key, emit, n, counts, nt);
   BF_LAUNCHED("k_part_scatter");
   return BUFFALO_OK;
 }
