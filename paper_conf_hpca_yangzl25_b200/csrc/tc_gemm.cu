@@ -175,6 +175,7 @@ struct GemmParams {
 __global__ void __launch_bounds__(kGemmThreads, 1)
     k_tc_gemm_tma(const __grid_constant__ CUtensorMap self_map, const __grid_constant__ CUtensorMap agg_map,
                   const __grid_constant__ CUtensorMap out_map, const GemmParams p) {
+  pdl_wait();
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-B alignment by offset (keeps the shared address space visible to the compiler)
   uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
@@ -407,6 +408,7 @@ constexpr int kDwThreads2 = (kDwMmaWarp + 1) * 32;
 __global__ void __launch_bounds__(kDwThreads2, 1)
     k_tc_dw_tma(const __grid_constant__ CUtensorMap z_map, const __grid_constant__ CUtensorMap self_map,
                 const __grid_constant__ CUtensorMap agg_map, const DwParams p) {
+  pdl_wait();
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
   const int NS = p.nstages;
@@ -590,7 +592,7 @@ buffalo_status tc_dw_tma(int64_t n, int S, const __nv_bfloat16* z, int64_t ldz, 
   const int smem = p.nstages * stage + 16 * p.nstages + 64 + 1024;
   BF_CHECK(set_max_smem_once<k_tc_dw_tma>(227 * 1024));
   dim3 grid((unsigned)ceil_div(2 * Dp, p.NT), (unsigned)S);
-  k_tc_dw_tma<<<grid, kDwThreads2, smem, s>>>(zm, sm, am, p);
+  launch_pdl(k_tc_dw_tma, grid, dim3(kDwThreads2), (size_t)smem, s, zm, sm, am, p);
   BF_LAUNCHED("k_tc_dw_tma");
   return BUFFALO_OK;
 }
@@ -657,7 +659,7 @@ buffalo_status tc_gemm_tma(int64_t n_rows, int64_t self_rows, const int32_t* sel
   BF_CHECK(set_max_smem_once<k_tc_gemm_tma>(227 * 1024));
   const int64_t sets = std::min<int64_t>(ceil_div(n_rows, kTM), 148 / p.nsplit);
   const int grid = (int)(sets * p.nsplit);
-  k_tc_gemm_tma<<<grid, kGemmThreads, smem, s>>>(sm, am, om, p);
+  launch_pdl(k_tc_gemm_tma, dim3(grid), dim3(kGemmThreads), (size_t)smem, s, sm, am, om, p);
   BF_LAUNCHED("k_tc_gemm_tma");
   return BUFFALO_OK;
 }

@@ -599,6 +599,7 @@ __global__ void __launch_bounds__(256, MINB) k_gather_v2(const int32_t* __restri
                                                          __nv_bfloat16* __restrict__ out, int64_t ldo,
                                                          unsigned long long* __restrict__ edges_dev,
                                                          const GatherEpi ep) {
+  pdl_wait();
   constexpr int E = InTraits<TI>::kElems;
   constexpr int G = 32 / LPR;
   constexpr unsigned kFull = 0xffffffffu;
@@ -844,7 +845,7 @@ static buffalo_status launch_gather(const int32_t* perm, const int32_t* rp, cons
   const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
   const int32_t n32 = (int32_t)n;
   const int32_t ldb = (int32_t)(ldh * (int64_t)sizeof(TI));             // row stride in bytes
-#define BF_V2(L) k_gather_v2<TI, MODE, L, kU, 5, kHintFwd><<<fgrid, 256, 0, s>>>(perm, rp, col, n32, h, ldb, \
+#define BF_V2(L) launch_pdl(k_gather_v2<TI, MODE, L, kU, 5, kHintFwd>, dim3(fgrid), dim3(256), 0, s, perm, rp, col, n32, h, ldb, \
                                                                                      npieces, out, ldo, ps.edges_dev, \
                                                                                      GatherEpi{})
   if (lpr_log <= 2) BF_V2(4);
@@ -881,8 +882,8 @@ static buffalo_status launch_gather_epi(const int32_t* perm, const int32_t* rp, 
   const int smem = 8 * G * npieces * 8 * 4;
   const int32_t n32 = (int32_t)(n > 0 ? n : 0);
   const int32_t ldb = (int32_t)(ldy * 2);
-#define BF_V2E(L) k_gather_v2<__nv_bfloat16, 2, L, kU, kMinB, kHintBwd><<<kGatherDbCtas, 256, smem, s>>>( \
-      perm, rp, col, n32, yn, ldb, npieces, out, ldo, ps.edges_dev, ep)
+#define BF_V2E(L) launch_pdl(k_gather_v2<__nv_bfloat16, 2, L, kU, kMinB, kHintBwd>, dim3(kGatherDbCtas), dim3(256), \
+      (size_t)smem, s, perm, rp, col, n32, yn, ldb, npieces, out, ldo, ps.edges_dev, ep)
   if (lpr_log <= 2) BF_V2E(4);
   else if (lpr_log == 3) BF_V2E(8);
   else BF_V2E(16);
@@ -919,8 +920,8 @@ static buffalo_status launch_gather_sharded(const buffalo_block* blk, const buff
   const int fgrid = (int)std::min<int64_t>(ceil_div(ceil_div(n, 32 >> std::max(lpr_log, 2)), 8), 148LL * kMinB * 4);
   const int32_t n32 = (int32_t)n, ldb = (int32_t)(ld_src * 2);
   const __nv_bfloat16* h0 = (const __nv_bfloat16*)sh->shard[0];
-#define BF_V2S(L) k_gather_v2<__nv_bfloat16, 3, L, kU, 5, kHintFwd><<<fgrid, 256, 0, s>>>( \
-      nullptr, blk->row_ptr, blk->col_global, n32, h0, ldb, npieces, out, ldo, ps.edges_dev, ep)
+#define BF_V2S(L) launch_pdl(k_gather_v2<__nv_bfloat16, 3, L, kU, 5, kHintFwd>, dim3(fgrid), dim3(256), 0, s, \
+      (const int32_t*)nullptr, blk->row_ptr, blk->col_global, n32, h0, ldb, npieces, out, ldo, ps.edges_dev, ep)
   if (lpr_log <= 2) BF_V2S(4);
   else if (lpr_log == 3) BF_V2S(8);
   else if (lpr_log == 4) BF_V2S(16);
